@@ -1,0 +1,436 @@
+#!/usr/bin/env python
+"""Benchmark of the CRSD SpMV hot path on B200 (driver contract: one JSON line).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2|c3|c4]
+                    [--dtype f64|f32] [--impl crsd|reference]
+
+A step is one y = A*x (alpha 1, beta 0, the paper's SpMV) over the
+whole workload, inputs resident in HBM. Workload at N=1: BASELINE.json
+configs[1] (C2, 3D 7-point Laplacian 256^3, fp64) unless --config says
+otherwise. N>1 (torchrun): weak scaling, rank r owns a 256^3 slab of a
+256 x 256 x (256 N) 7-point grid; x halos move with NCCL send/recv over
+NVLink inside crsd_spmv_dist, overlapped with the interior segments.
+
+Metric (BASELINE.json): CRSD SpMV GFLOP/s (= 2 nnz / t, whole job) with
+achieved HBM GB/s on algorithmic ("unique") bytes and its fraction of the
+measured B200 copy bandwidth (MEASURED_PEAKS.json).
+--impl reference times the oracle (oracle/coo_spmv.c, long double, 1 thread)
+on the host cores on the same workload (the tier's reference arm).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+L2_BYTES = 126 * 1024 * 1024
+
+
+def _env_int(k, d):
+    try:
+        return int(os.environ.get(k, d))
+    except ValueError:
+        return d
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            j = json.load(f)
+        return float(j.get("hbm_gbs", 6650.0)), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+# ---------------------------------------------------------------- workloads
+def workload(cfg: str, dtype: str, world: int = 1, rank: int = 0):
+    """Returns (COO of this rank's rows, description dict, row range or None, global nrows)."""
+    import gen
+
+    dt = np.float64 if dtype == "f64" else np.float32
+    if cfg == "c2":
+        n = 256
+        nz = n * world
+        N = n * n * nz
+        rb, re = rank * n * n * n, (rank + 1) * n * n * n
+        a = gen.stencil((n, n, nz), "7pt", values="random", seed=2, row_begin=rb, row_end=re)
+        desc = f"C2: 3D 7-point FDM Laplacian 256^3 per GPU (grid 256x256x{nz}, {N:,} rows), {dtype}"
+    elif cfg == "c3":
+        if world != 1:
+            raise SystemExit("config c3 is a single-GPU workload")
+        a = gen.config3()
+        N, rb, re = a.nrows, 0, a.nrows
+        desc = f"C3: 3D 27-point FVM stencil 192^3 with idle sub-blocks and 0.1% scatter points ({N:,} rows), {dtype}"
+    elif cfg == "c4":
+        n = 100_000_000
+        bounds = np.linspace(0, n, world + 1).astype(np.int64) // 512 * 512
+        bounds[-1] = n
+        rb, re = int(bounds[rank]), int(bounds[rank + 1])
+        a = gen.config4(n=n, row_begin=rb, row_end=re)
+        N = n
+        desc = f"C4: banded, 19 offsets in 9 groups / 4 patterns, 100M rows, {dtype}"
+    else:
+        raise SystemExit(f"unknown config {cfg}")
+    a = gen.COO(N, N, a.row, a.col, a.val.astype(dt))
+    return a, desc, (rb, re), N
+
+
+# ---------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled during the timed region."""
+
+    FIELDS = "clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap"
+
+    def __init__(self, index: int):
+        self.index = index
+        self.samples = []
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE,
+                stderr=subprocess.DEVNULL,
+                text=True,
+            )
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) == 7:
+                self.samples.append(parts)
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=2)
+        except Exception:
+            self.proc.kill()
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for s in self.samples:
+            for nm, v in zip(names, s[3:]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {
+            "sm_mhz": statistics.median(sm) if sm else None,
+            "sm_max_mhz": max(mx) if mx else None,
+            "reasons": sorted(reasons),
+            "samples": len(self.samples),
+        }
+
+
+def load_traffic(cfg, dtype):
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            j = json.load(f)
+        return j.get(f"{cfg}_{dtype}")
+    return None
+
+
+# ---------------------------------------------------------------- reference arm
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    from oracle import coo as oracle_coo
+
+    a, desc, _, N = workload(args.config, args.dtype, 1, 0)
+    dt = a.val.dtype
+    x = np.random.default_rng(7).uniform(-1, 1, a.ncols).astype(dt)
+    # bounded sample: calibrate the oracle's rate, then size each step so the
+    # whole --steps/--warmup run stays within ~2 minutes of CPU time
+    n0, r0_, c0_, v0_ = row_sample(a, 2_000_000)
+    t0 = time.perf_counter()
+    oracle_coo.coo_spmv(n0, a.ncols, r0_, c0_, v0_, x)
+    rate = r0_.shape[0] / max(time.perf_counter() - t0, 1e-6)
+    budget = float(os.environ.get("CRSD_REF_BUDGET_S", "120"))
+    cap = int(min(a.nnz, max(1_000_000, rate * budget / (args.steps + args.warmup))))
+    sample_rows, row, col, val = row_sample(a, cap)
+    nnz_s = row.shape[0]
+    for _ in range(args.warmup):
+        oracle_coo.coo_spmv(sample_rows, a.ncols, row, col, val, x)
+    ts = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle_coo.coo_spmv(sample_rows, a.ncols, row, col, val, x)
+        ts.append(time.perf_counter() - t0)
+    t = sum(ts) / len(ts)
+    gflops = 2.0 * nnz_s / t / 1e9
+    sample = f"rows [0,{sample_rows:,}) of the workload, {nnz_s:,} nonzeros per step ({nnz_s / a.nnz:.1%} of the matrix)"
+    line = {
+        "impl": "reference",
+        "metric": "CRSD SpMV GFLOP/s (2*nnz/t)",
+        "value": round(gflops, 4),
+        "unit": "GFLOP/s",
+        "n_gpus": args.gpus,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": round(t * 1e3, 3),
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": "f64" if dt == np.float64 else "f32",
+        "data": "synthetic",
+        "config": {"workload": desc, "alpha": 1.0, "beta": 0.0},
+        "cpu_baseline": {"value": round(gflops, 4), "unit": "GFLOP/s", "cores": 1, "kind": "oracle", "sample": sample},
+        "e2e": {"value": round(gflops, 4), "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def row_sample(a, cap=None):
+    """Rows [0, cut) of the workload, sized to ~cap nonzeros (bounded CPU
+    work); entries selected by mask, so input order is irrelevant."""
+    if cap is None:
+        cap = int(os.environ.get("CRSD_REF_SAMPLE_NNZ", "60000000"))
+    if a.nnz <= cap:
+        return a.nrows, a.row, a.col, a.val
+    cut = max(1, int(a.nrows * cap // a.nnz))
+    m = a.row < cut
+    return cut, a.row[m], a.col[m], a.val[m]
+
+
+# ---------------------------------------------------------------- CRSD arm
+def cpu_baseline(a, seconds_target=10.0):
+    """The oracle as it stands (1 thread, long double) on a bounded row sample."""
+    from oracle import coo as oracle_coo
+
+    dt = a.val.dtype
+    x = np.random.default_rng(7).uniform(-1, 1, a.ncols).astype(dt)
+    nr, row, col, val = row_sample(a)
+    k = row.shape[0]
+    ts = []
+    t_start = time.perf_counter()
+    while True:
+        t0 = time.perf_counter()
+        oracle_coo.coo_spmv(nr, a.ncols, row, col, val, x)
+        ts.append(time.perf_counter() - t0)
+        if time.perf_counter() - t_start > seconds_target or len(ts) >= 20:
+            break
+    t = statistics.median(ts)
+    return {
+        "value": round(2.0 * k / t / 1e9, 4),
+        "unit": "GFLOP/s",
+        "cores": 1,
+        "kind": "oracle",
+        "sample": f"rows [0,{nr:,}) ({k:,} nonzeros, {k / a.nnz:.1%} of the workload), median of {len(ts)} runs, long-double accumulation, 1 thread",
+    }
+
+
+def run_crsd(args):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, Comm
+
+    world = args.gpus
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        dist.init_process_group("nccl", init_method="env://")
+        world = dist.get_world_size()
+        rank = dist.get_rank()
+    torch.cuda.set_device(local_rank)
+    dev = local_rank
+
+    a, desc, (rb, re), N = workload(args.config, args.dtype, world, rank)
+    dt = a.val.dtype
+    tdt = torch.float64 if dt == np.float64 else torch.float32
+    es = np.dtype(dt).itemsize
+    kw = dict(device=dev)
+    if args.mrows:
+        kw["mrows"] = args.mrows
+    if world > 1:
+        kw["row_range"] = (rb, re)
+    t0 = time.perf_counter()
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, **kw)
+    build_s = time.perf_counter() - t0
+    info = A.info()
+    nnz_local = info["nnz"]
+    ub = info["unique_bytes_beta0"]
+    stream = torch.cuda.current_stream()
+
+    x_full = torch.from_numpy(np.random.default_rng(7 + rank).uniform(-1, 1, re - rb).astype(dt)).to(f"cuda:{dev}")
+    comm = None
+    if world > 1:
+        lo, nloc, hi = A.x_layout()
+        xp = torch.zeros(lo + nloc + hi, dtype=tdt, device=f"cuda:{dev}")
+        xp[lo : lo + nloc] = x_full
+        y = torch.empty(nloc, dtype=tdt, device=f"cuda:{dev}")
+        comm = Comm(rank, world, dev)
+        A.dist_bind(comm)
+
+        def step():
+            A.spmv_dist(xp, y, 1.0, 0.0, comm)
+    else:
+        x = x_full
+        y = torch.empty(a.nrows, dtype=tdt, device=f"cuda:{dev}")
+
+        def step():
+            A.spmv(x, y, 1.0, 0.0)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+
+    # timed region: K steps, per-step CUDA events on the launching stream
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    clocks = ClockSampler(dev)
+    clocks.start()
+    time.sleep(0.3)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t_all0 = torch.cuda.Event(enable_timing=True)
+    t_all1 = torch.cuda.Event(enable_timing=True)
+    t_all0.record(stream)
+    launches = 0
+    for i in range(args.steps):
+        ev[i][0].record(stream)
+        step()
+        ev[i][1].record(stream)
+        launches += A.last_launch_count()
+    t_all1.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    total_ms = t_all0.elapsed_time(t_all1)
+    step_ms = [s.elapsed_time(e) for s, e in ev]
+    if world > 1:
+        tt = torch.tensor([total_ms], dtype=torch.float64, device=f"cuda:{dev}")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        total_ms = float(tt.item())
+        nn = torch.tensor([nnz_local, ub], dtype=torch.float64, device=f"cuda:{dev}")
+        dist.all_reduce(nn)
+        nnz_all, ub_all = float(nn[0].item()), float(nn[1].item())
+    else:
+        nnz_all, ub_all = float(nnz_local), float(ub)
+    ms = total_ms / args.steps
+    gflops = 2.0 * nnz_all / (ms * 1e-3) / 1e9
+    kern_ms = statistics.mean(step_ms)
+    peak, peak_src = measured_peaks()
+    achieved = ub / (kern_ms * 1e-3) / 1e9
+
+    # e2e through the public C-ABI with host buffers (pinned), N = 1 path
+    e2e = None
+    if world == 1:
+        xh = torch.from_numpy(np.random.default_rng(7).uniform(-1, 1, a.ncols).astype(dt)).pin_memory()
+        yh = torch.empty(a.nrows, dtype=tdt).pin_memory()
+        for _ in range(2):
+            A.spmv_host_ptr(xh.data_ptr(), yh.data_ptr(), 1.0, 0.0)
+        ke = max(3, min(args.steps, 50))
+        t0 = time.perf_counter()
+        for _ in range(ke):
+            A.spmv_host_ptr(xh.data_ptr(), yh.data_ptr(), 1.0, 0.0)
+        te = (time.perf_counter() - t0) / ke
+        e2e = {
+            "value": round(2.0 * nnz_all / te / 1e9, 3),
+            "unit": "GFLOP/s",
+            "h2d_bytes_per_step": int(a.ncols * es),
+            "d2h_bytes_per_step": int(a.nrows * es),
+            "ms_per_step": round(te * 1e3, 4),
+        }
+    if rank != 0:
+        if comm is not None:
+            comm.close()
+        dist.destroy_process_group()
+        return
+
+    cpu = None if (world > 1 or args.no_cpu) else cpu_baseline(a)
+    traffic = load_traffic(args.config, args.dtype)
+    line = {
+        "metric": "CRSD SpMV GFLOP/s (2*nnz/t) with achieved HBM GB/s (% of B200 peak)",
+        "value": round(gflops, 3),
+        "unit": "GFLOP/s",
+        "n_gpus": world,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": round(ms, 5),
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": args.dtype,
+        "data": "synthetic",
+        "config": {
+            "workload": desc,
+            "nnz": int(nnz_all),
+            "mrows": info["mrows"],
+            "alpha": 1.0,
+            "beta": 0.0,
+            "patterns": info["npat"],
+            "instances": info["ninst"],
+            "fills": info["nfills"],
+            "scatter": info["nscatter"],
+            "l2": f"inputs larger than L2 ({ub / 1e9:.2f} GB streamed per step vs {L2_BYTES / 2**20:.0f} MiB L2); no flush",
+            "build_s": round(build_s, 2),
+        },
+        "hbm_gbs": round(ub_all / (ms * 1e-3) / 1e9, 1),
+        "hbm_frac_of_peak": round(ub_all / (ms * 1e-3) / 1e9 / (peak * world), 4),
+        "roofline": {
+            "bound": "hbm",
+            "kernel": "crsd_spmv_kernel",
+            "achieved": round(achieved, 1),
+            "peak": peak,
+            "peak_source": peak_src,
+            "unit": "GB/s",
+            "frac": round(achieved / peak, 4),
+            "traffic": traffic,
+            "algorithmic_bytes_per_launch": int(ub),
+            "avg_launch_ms": round(kern_ms, 5),
+        },
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gpu_launches": int(launches),
+        "clocks": clk,
+    }
+    print(json.dumps(line), flush=True)
+    if comm is not None:
+        comm.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=500)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--config", default="c2", choices=["c2", "c3", "c4"])
+    ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
+    ap.add_argument("--mrows", type=int, default=0)
+    ap.add_argument("--impl", default="crsd", choices=["crsd", "reference"])
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_crsd(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,270 @@
+/*
+ * crsd.h -- C-ABI of the B200-native CRSD SpMV library (libcrsd.so).
+ *
+ * Operation (PAPER.md P:L33-39 problem statement; "the result
+ * should be stored at ... destination vector y"; generalised to BLAS form by
+ * BASELINE.json north_star (1)):
+ *
+ *     y = alpha * A * x + beta * y
+ *
+ * for a diagonal sparse matrix A stored in CRSD, "Compressed Row Segment with
+ * Diagonal-pattern" (§II; Fig. 4):
+ *   - rows are split into row segments of `mrows` rows;
+ *   - in each segment the diagonals (offset = col - row) that
+ *     carry >= 2 nonzeros, or that belong to a run bridged across idle
+ *     sections of <= idle_max zeros, are stored (R1/R2);
+ *   - consecutive segments with the same diagonal set form a diagonal
+ *     pattern, grouped into AD / NAD groups;
+ *   - values are stored contiguously per segment and per diagonal, filled
+ *     zeros included (address formula P:L613-623);
+ *   - the remaining nonzeros are scatter points, stored separately
+ *     (per-segment list, R5).
+ * At SpMV time only values are read; no per-nonzero index is loaded
+ * (P:L631-635).
+ *
+ * Conventions for every call
+ *   - Every call returns crsd_status_t; CRSD_OK == 0. No call throws, aborts
+ *     or exits. crsd_last_error() returns a thread-local message describing
+ *     the last non-OK status of the calling thread.
+ *   - Pointers documented as HOST must be host-accessible; DEVICE pointers
+ *     must be device memory of the handle's CUDA device. Ownership is stated
+ *     per argument; the library never frees caller memory.
+ *   - `stream` arguments are cudaStream_t values passed as void* (NULL = the
+ *     legacy default stream). Device calls are asynchronous and
+ *     stream-ordered unless stated; launch errors are returned synchronously,
+ *     asynchronous kernel faults surface at the caller's next synchronisation.
+ *   - A handle must not be used by two threads at once.
+ *   - The library holds no global state besides the thread-local error text.
+ */
+#ifndef CRSD_H
+#define CRSD_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    CRSD_OK = 0,
+    CRSD_ERR_INVALID_ARG = 1, /* NULL where not allowed, bad size, misaligned device pointer, ... */
+    CRSD_ERR_INDEX_RANGE = 2, /* a COO row/col outside [0,nrows)x[0,ncols) (or outside the handle's row range) */
+    CRSD_ERR_DUPLICATE = 3,   /* a (row,col) given twice and CRSD_SUM_DUPLICATES not set */
+    CRSD_ERR_UNSUPPORTED = 4, /* valid request the GPU path does not handle (e.g. mrows not a multiple of 32*RPT) */
+    CRSD_ERR_ALLOC = 5,       /* host or device allocation failed */
+    CRSD_ERR_CUDA = 6,        /* a CUDA runtime call or kernel launch failed */
+    CRSD_ERR_NCCL = 7         /* an NCCL call failed */
+} crsd_status_t;
+
+typedef enum { CRSD_R32F = 0, CRSD_R64F = 1 } crsd_dtype_t;
+
+/* opts.flags */
+#define CRSD_SUM_DUPLICATES 0x1u /* duplicates are summed (in input order) instead of rejected */
+#define CRSD_HOST_ONLY 0x2u      /* build the CRSD structure on the host only (export/inspection); no device memory is touched and crsd_spmv* return CRSD_ERR_UNSUPPORTED */
+#define CRSD_DROP_ZEROS 0x4u     /* explicit zero entries are dropped instead of kept in the scatter list (R10) */
+
+/*
+ * Build options. Call crsd_opts_init() for defaults (NULL opts == defaults).
+ *   mrows     row-segment height (token `mrows`); 0 => 256. The
+ *             GPU path needs mrows % (32*RPT) == 0, RPT = 2 rows per thread
+ *             for fp64 and 4 for fp32 (one 128-bit vector per thread and
+ *             diagonal); the host builder accepts any mrows >= 1.
+ *   idle_max  longest run of zeros along a diagonal that is bridged by
+ *             filling zeros (R2); < 0 => mrows - 1.
+ *   flags     CRSD_* flags above.
+ *   row_begin, row_end
+ *             rows owned by this handle for the row-partitioned multi-GPU
+ *             path; both 0 => all rows [0, nrows). COO rows must lie in the
+ *             range. row_begin must be a multiple of mrows.
+ *   device    CUDA device ordinal the handle's memory lives on (-1 => current).
+ *   nthreads  host builder threads (OpenMP); 0 => OpenMP default.
+ */
+typedef struct {
+    int32_t mrows;
+    int32_t idle_max;
+    uint32_t flags;
+    int32_t device;
+    int64_t row_begin;
+    int64_t row_end;
+    int32_t nthreads;
+    int32_t reserved;
+} crsd_opts_t;
+
+typedef struct crsd_matrix_s *crsd_matrix_t;
+typedef struct crsd_comm_s *crsd_comm_t;
+
+/* Sizes and counts of a built matrix (all counts are of the local rows for a
+ * row-partitioned handle). */
+typedef struct {
+    int64_t nrows, ncols;           /* global dimensions */
+    int64_t row_begin, row_end;     /* owned rows */
+    int32_t mrows, idle_max;
+    int32_t dtype;                  /* crsd_dtype_t */
+    int32_t rows_per_thread;        /* RPT of the GPU kernel (2 fp64, 4 fp32) */
+    int64_t nnz;                    /* canonical entries (after duplicate handling) */
+    int64_t nseg;                   /* row segments */
+    int64_t ninst;                  /* pattern instances = the paper's diagonal patterns (Table II rows) */
+    int64_t npat;                   /* distinct diagonal-offset sets */
+    int64_t noffsets;               /* sum over distinct patterns of NDias */
+    int64_t max_ndias;              /* max NDias over patterns */
+    int64_t nslots;                 /* stored diagonal slots = sum NRS_p * NNzRS_p */
+    int64_t ndiag_nnz;              /* nonzeros stored on diagonals */
+    int64_t nfills;                 /* filled zeros = nslots - ndiag_nnz */
+    int64_t nscatter;               /* scatter entries */
+    int64_t nedge_seg;              /* segments run by the guarded (edge) kernel body */
+    int64_t halo_lo, halo_hi;       /* x halo widths (elements) of a row-partitioned handle */
+    int64_t device_bytes;           /* device memory held by the handle */
+    int64_t unique_bytes_beta0;     /* algorithmic bytes of one SpMV with beta == 0 */
+    int64_t unique_bytes_beta1;     /* ... with beta != 0 (y also read) */
+} crsd_info_t;
+
+/*
+ * Host copies of the CRSD structure (B200 layout).
+ * Sizes come from crsd_info_t; any NULL pointer is skipped. Caller-owned.
+ *   inst_first_seg[ninst], inst_nseg[ninst], inst_pattern[ninst]
+ *   pat_ptr[npat+1], pat_offsets[noffsets]  (ascending offsets per pattern)
+ *   vals[nslots]  (dtype) -- instance i, local segment g, diagonal d, row l at
+ *                 base_i + g*NDias*mrows + d*mrows + l, base_i = sum_{j<i}
+ *                 nseg_j*NDias_j*mrows
+ *   scat_ptr[nseg+1], scat_row[nscatter] (row within segment),
+ *   scat_col[nscatter] (global column), scat_val[nscatter] (dtype);
+ *   entries of a segment sorted by (row, col).
+ */
+typedef struct {
+    int64_t *inst_first_seg;
+    int64_t *inst_nseg;
+    int32_t *inst_pattern;
+    int64_t *pat_ptr;
+    int64_t *pat_offsets;
+    void *vals;
+    int64_t *scat_ptr;
+    int32_t *scat_row;
+    int64_t *scat_col;
+    void *scat_val;
+} crsd_export_t;
+
+const char *crsd_last_error(void);
+const char *crsd_version(void);
+crsd_status_t crsd_opts_init(crsd_opts_t *opts);
+
+/*
+ * Build a CRSD matrix from COO (§II; steps in DESIGN.md "Builder").
+ *   nrows, ncols   global dimensions, > 0 and < 2^31.
+ *   nnz            entries, >= 0.
+ *   row, col       HOST int64[nnz], caller-owned, read-only, copied. Any order.
+ *   val            HOST dtype[nnz] (float or double), caller-owned, copied.
+ *   dtype          CRSD_R32F or CRSD_R64F.
+ *   opts           NULL => defaults.
+ *   out            receives the handle (NULL on failure).
+ * Errors: INVALID_ARG, INDEX_RANGE, DUPLICATE, UNSUPPORTED, ALLOC, CUDA.
+ * Synchronous: the device copy is complete when the call returns.
+ */
+crsd_status_t crsd_create_from_coo(int64_t nrows, int64_t ncols, int64_t nnz, const int64_t *row,
+                                   const int64_t *col, const void *val, crsd_dtype_t dtype,
+                                   const crsd_opts_t *opts, crsd_matrix_t *out);
+
+/* Same from CSR: row_ptr HOST int64[nrows_local+1] over the owned rows
+ * (row_ptr[0] may be nonzero: entries are col[row_ptr[0]..row_ptr[n]]). */
+crsd_status_t crsd_create_from_csr(int64_t nrows, int64_t ncols, const int64_t *row_ptr, const int64_t *col,
+                                   const void *val, crsd_dtype_t dtype, const crsd_opts_t *opts,
+                                   crsd_matrix_t *out);
+
+/* Destroy a handle and free its device/host memory. NULL is a no-op. Not
+ * stream-ordered: the caller must ensure no SpMV on the handle is in flight. */
+crsd_status_t crsd_destroy(crsd_matrix_t A);
+
+/*
+ * y = alpha*A*x + beta*y on the GPU (P:L567-719 method; kernels DESIGN.md §Kernels).
+ *   alpha, beta    HOST pointers to one scalar of the matrix dtype.
+ *   x              DEVICE dtype[ncols], 16-byte aligned, read-only.
+ *   y              DEVICE dtype[nrows], 16-byte aligned; not read when
+ *                  *beta == 0 (BLAS convention). Must not alias x.
+ *   stream         cudaStream_t (void*).
+ * Asynchronous; launch errors (CUDA) returned. UNSUPPORTED for host-only or
+ * row-partitioned handles (use crsd_spmv_dist). x must be finite: a filled
+ * zero computes 0*x (as DIA does).
+ */
+crsd_status_t crsd_spmv(crsd_matrix_t A, const void *alpha, const void *x, const void *beta, void *y,
+                        void *stream);
+
+/*
+ * End-to-end form with HOST vectors: copies x (and y when beta != 0) to
+ * device scratch owned by the handle, runs crsd_spmv, copies y back and
+ * synchronises `stream`. x_host dtype[ncols], y_host dtype[nrows] (pinned
+ * memory recommended). Synchronous. Used for the e2e measurement (the
+ * paper's transfer caveat).
+ */
+crsd_status_t crsd_spmv_host(crsd_matrix_t A, const void *alpha, const void *x_host, const void *beta,
+                             void *y_host, void *stream);
+
+/* ------------------------------------------------------------------------
+ * Row-partitioned multi-GPU path (BASELINE.json north_star (3)). Not in the
+ * paper (single GPU). Each rank builds a handle over rows [row_begin,
+ * row_end) of a square matrix (opts.row_begin/row_end, COO with GLOBAL
+ * indices). x is partitioned like the rows. The rank's x lives in a padded
+ * DEVICE buffer x_padded[halo_lo + n_local + halo_hi] whose owned part starts
+ * at x_padded + halo_lo; the library writes the halos.
+ * ---------------------------------------------------------------------- */
+
+/* Halo widths (elements) and local length of a row-partitioned handle.
+ * halo_lo is a multiple of 4 so x_padded + halo_lo stays 16-byte aligned. */
+crsd_status_t crsd_dist_x_layout(crsd_matrix_t A, int64_t *halo_lo, int64_t *n_local, int64_t *halo_hi);
+
+/* Communicator. id: 128 bytes from crsd_comm_unique_id() on rank 0,
+ * broadcast by the caller (e.g. through torch.distributed). Collective over
+ * all ranks. The library creates the NCCL communicator and a comm stream. */
+crsd_status_t crsd_comm_unique_id(void *id128);
+crsd_status_t crsd_comm_init_rank(const void *id128, int rank, int world, int device, crsd_comm_t *out);
+crsd_status_t crsd_comm_destroy(crsd_comm_t comm);
+
+/* Exchange row ranges and halo widths with every rank (collective, once per
+ * handle and communicator) and derive the send/recv plan. */
+crsd_status_t crsd_dist_bind(crsd_matrix_t A_local, crsd_comm_t comm, void *stream);
+
+/*
+ * Distributed SpMV: halo exchange (NCCL send/recv on the comm stream) in
+ * parallel with the interior segments, then the boundary segments.
+ *   x_padded  DEVICE dtype[halo_lo+n_local+halo_hi], 16-byte aligned; the
+ *             owned part must be written before the call (stream-ordered);
+ *             the halo parts are overwritten.
+ *   y_local   DEVICE dtype[n_local].
+ * comm == NULL means "halos already filled by the caller": only the compute
+ * runs (single-process testing of the partitioned layout).
+ */
+crsd_status_t crsd_spmv_dist(crsd_matrix_t A_local, const void *alpha, void *x_padded, const void *beta,
+                             void *y_local, crsd_comm_t comm, void *stream);
+
+/*
+ * Pure host helper (no CUDA, no NCCL): given every rank's [row_begin,
+ * row_end, halo_lo_valid, halo_hi_valid] (int64[world][4], the halo widths
+ * actually needed, without alignment padding) compute what `rank` receives
+ * and sends. Output arrays have capacity `world` entries each:
+ *   recv_peer[k], recv_begin[k] (global col), recv_count[k]; *nrecv
+ *   send_peer[k], send_begin[k] (global col), send_count[k]; *nsend
+ * Multi-hop is handled: a halo wider than a neighbour's block is split over
+ * every owner. Errors: INVALID_ARG (ranges not contiguous / not covering).
+ */
+crsd_status_t crsd_dist_plan(int world, int rank, const int64_t *ranges4, int64_t *recv_peer,
+                             int64_t *recv_begin, int64_t *recv_count, int64_t *nrecv, int64_t *send_peer,
+                             int64_t *send_begin, int64_t *send_count, int64_t *nsend);
+
+/*
+ * Pure host helper: contiguous row blocks aligned to mrows, balanced on
+ * per-row weights (e.g. stored bytes per row). weights HOST double[nrows]
+ * (NULL => uniform). bounds HOST int64[world+1] receives the row boundaries.
+ */
+crsd_status_t crsd_partition_rows(int64_t nrows, int32_t mrows, int world, const double *weights,
+                                  int64_t *bounds);
+
+/* Introspection */
+crsd_status_t crsd_get_info(crsd_matrix_t A, crsd_info_t *info);
+crsd_status_t crsd_export(crsd_matrix_t A, crsd_export_t *out);
+
+/* Number of kernel launches the last crsd_spmv / crsd_spmv_dist call made. */
+crsd_status_t crsd_last_launch_count(crsd_matrix_t A, int32_t *count);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CRSD_H */

@@ -1,0 +1,16 @@
+"""B200-native CRSD SpMV (Sun et al., ICPP 2011): y = alpha*A*x + beta*y for
+diagonal sparse matrices stored in Compressed Row Segment with
+Diagonal-pattern format. The compute path is libcrsd.so (C-ABI in
+include/crsd.h, sm_100a kernels in csrc/); this package is its binding.
+"""
+from .crsd import (  # noqa: F401
+    CRSDMatrix,
+    Comm,
+    CRSDError,
+    dist_plan,
+    partition_rows,
+    version,
+    CRSD_SUM_DUPLICATES,
+    CRSD_HOST_ONLY,
+    CRSD_DROP_ZEROS,
+)

@@ -1,0 +1,409 @@
+// C-ABI of libcrsd (include/crsd.h): handle lifetime, device upload,
+// single-GPU SpMV, host end-to-end SpMV, introspection.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "crsd_internal.h"
+#include "crsd_handle.h"
+
+namespace crsd {
+
+static thread_local std::string g_err;
+
+void set_error(const std::string &msg) { g_err = msg; }
+
+crsd_status_t fail(crsd_status_t st, const std::string &msg) {
+    g_err = msg;
+    return st;
+}
+
+crsd_status_t cuda_fail(cudaError_t e, const char *what) {
+    return fail(CRSD_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+#define CUDA_TRY(expr)                                       \
+    do {                                                     \
+        cudaError_t _e = (expr);                             \
+        if (_e != cudaSuccess) return cuda_fail(_e, #expr); \
+    } while (0)
+
+static crsd_status_t dev_alloc_copy(void **dptr, const void *src, size_t bytes, int64_t &counter) {
+    *dptr = nullptr;
+    if (bytes == 0) return CRSD_OK;
+    cudaError_t e = cudaMalloc(dptr, bytes);
+    if (e != cudaSuccess) {
+        *dptr = nullptr;
+        return fail(e == cudaErrorMemoryAllocation ? CRSD_ERR_ALLOC : CRSD_ERR_CUDA,
+                    "cudaMalloc(" + std::to_string(bytes) + "): " + cudaGetErrorString(e));
+    }
+    counter += (int64_t)bytes;
+    if (src) CUDA_TRY(cudaMemcpy(*dptr, src, bytes, cudaMemcpyHostToDevice));
+    return CRSD_OK;
+}
+
+void free_device(crsd_matrix_s *A) {
+    void *ptrs[] = {A->d_vals, A->d_segs, A->d_offs, A->d_scat_row, A->d_scat_col, A->d_scat_val,
+                    A->d_list_interior, A->d_list_boundary, A->d_list_all_edge, A->d_x_scratch, A->d_y_scratch};
+    if (A->device >= 0) cudaSetDevice(A->device);
+    for (void *p : ptrs)
+        if (p) cudaFree(p);
+    A->d_vals = A->d_segs = A->d_offs = A->d_scat_row = A->d_scat_col = A->d_scat_val = nullptr;
+    A->d_list_interior = A->d_list_boundary = A->d_list_all_edge = A->d_x_scratch = A->d_y_scratch = nullptr;
+}
+
+// Layout of x for this handle: valid range and halo widths (DESIGN.md
+// "Multi-GPU"), segment descriptors and work lists.
+static void plan_layout(crsd_matrix_s *A) {
+    HostCRSD &H = A->H;
+    if (!H.partitioned) {
+        A->halo_lo = A->halo_hi = A->halo_lo_valid = A->halo_hi_valid = 0;
+        A->x_lo = 0;
+        A->x_hi = H.ncols;
+    } else {
+        int64_t need_lo, need_hi;
+        needed_halo(H, A->rpt, need_lo, need_hi);
+        A->halo_lo_valid = std::min<int64_t>(H.row_begin, std::max<int64_t>(0, need_lo));
+        A->halo_hi_valid = std::min<int64_t>(H.ncols - H.row_end, std::max<int64_t>(0, need_hi));
+        A->halo_lo = (A->halo_lo_valid + 3) / 4 * 4;
+        A->halo_hi = (A->halo_hi_valid + 3) / 4 * 4;
+        A->x_lo = -A->halo_lo_valid;
+        A->x_hi = H.n_local + A->halo_hi_valid;
+    }
+    make_segdescs(H, A->rpt, A->x_lo, A->x_hi, A->segdesc);
+    A->list_interior.clear();
+    A->list_boundary.clear();
+    A->nedge = 0;
+    for (int64_t s = 0; s < H.nseg; ++s) {
+        const SegDesc &D = A->segdesc[s];
+        if (D.flags & SEG_EDGE) A->nedge++;
+        if (D.flags & SEG_BOUNDARY) A->list_boundary.push_back((int32_t)s);
+        else A->list_interior.push_back((int32_t)s);
+    }
+}
+
+static crsd_status_t upload(crsd_matrix_s *A) {
+    HostCRSD &H = A->H;
+    if (A->device < 0) CUDA_TRY(cudaGetDevice(&A->device));
+    CUDA_TRY(cudaSetDevice(A->device));
+    CUDA_TRY(cudaDeviceGetAttribute(&A->sm_count, cudaDevAttrMultiProcessorCount, A->device));
+    int64_t &cnt = A->device_bytes;
+    crsd_status_t st;
+    if ((st = dev_alloc_copy(&A->d_vals, H.vals.data(), H.vals.size(), cnt))) return st;
+    if ((st = dev_alloc_copy(&A->d_segs, A->segdesc.data(), A->segdesc.size() * sizeof(SegDesc), cnt))) return st;
+    std::vector<int32_t> offs32(H.pat_offsets.begin(), H.pat_offsets.end());
+    if (offs32.empty()) offs32.push_back(0);
+    if ((st = dev_alloc_copy(&A->d_offs, offs32.data(), offs32.size() * 4, cnt))) return st;
+    const int64_t ns = H.nscatter();
+    std::vector<int64_t> colrel(ns);
+    for (int64_t e = 0; e < ns; ++e) colrel[e] = H.scat_col[e] - H.row_begin;
+    if ((st = dev_alloc_copy(&A->d_scat_row, H.scat_row.data(), ns * 4, cnt))) return st;
+    if ((st = dev_alloc_copy(&A->d_scat_col, colrel.data(), ns * 8, cnt))) return st;
+    if ((st = dev_alloc_copy(&A->d_scat_val, H.scat_val.data(), H.scat_val.size(), cnt))) return st;
+    if ((st = dev_alloc_copy(&A->d_list_interior, A->list_interior.data(), A->list_interior.size() * 4, cnt))) return st;
+    if ((st = dev_alloc_copy(&A->d_list_boundary, A->list_boundary.data(), A->list_boundary.size() * 4, cnt))) return st;
+    // the host copy of the bulk arrays is dropped after upload (export reads the device copy)
+    std::vector<uint8_t>().swap(H.vals);
+    std::vector<uint8_t>().swap(H.scat_val);
+    A->host_vals_dropped = true;
+    return CRSD_OK;
+}
+
+static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_matrix_t *out) {
+    A->rpt = (A->H.dtype == CRSD_R64F) ? 2 : 4;
+    plan_layout(A);
+    if (!A->host_only) {
+        if (A->H.mrows % (32 * A->rpt) != 0) {
+            delete A;
+            return fail(CRSD_ERR_UNSUPPORTED, "GPU path needs mrows % (32*RPT) == 0 (RPT = 2 fp64, 4 fp32); got mrows=" +
+                                                  std::to_string(o.mrows) + " (use CRSD_HOST_ONLY for inspection)");
+        }
+        crsd_status_t st = upload(A);
+        if (st) {
+            free_device(A);
+            delete A;
+            return st;
+        }
+    }
+    *out = A;
+    return CRSD_OK;
+}
+
+static crsd_status_t resolve_opts(int64_t nrows, crsd_dtype_t dtype, const crsd_opts_t *opts, crsd_opts_t &o,
+                                  BuildOptions &b) {
+    if (opts) o = *opts;
+    else crsd_opts_init(&o);
+    const int rpt = (dtype == CRSD_R64F) ? 2 : 4;
+    if (o.mrows == 0) o.mrows = 128 * rpt;
+    if (o.idle_max < 0) o.idle_max = o.mrows - 1;
+    if (o.row_begin == 0 && o.row_end == 0) o.row_end = nrows;
+    b.mrows = o.mrows;
+    b.idle_max = o.idle_max;
+    b.flags = o.flags;
+    b.row_begin = o.row_begin;
+    b.row_end = o.row_end;
+    b.nthreads = o.nthreads;
+    return CRSD_OK;
+}
+
+template <typename T>
+static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *y, const int32_t *list,
+                              int64_t count, void *stream, int &launches) {
+    if (count <= 0) return CRSD_OK;
+    SpmvArgs<T> a;
+    a.vals = (const T *)A->d_vals;
+    a.segs = (const SegDesc *)A->d_segs;
+    a.pat_offs = (const int32_t *)A->d_offs;
+    a.scat_row = (const int32_t *)A->d_scat_row;
+    a.scat_col = (const int64_t *)A->d_scat_col;
+    a.scat_val = (const T *)A->d_scat_val;
+    a.x = x;
+    a.x_lo = A->x_lo;
+    a.x_hi = A->x_hi;
+    a.y = y;
+    a.nrows = A->H.n_local;
+    a.seg_list = list;
+    a.seg_begin = 0;
+    a.seg_count = count;
+    a.mrows = A->H.mrows;
+    a.alpha = alpha;
+    a.beta = beta;
+    int n = launch_spmv<T>(a, A->sm_count, stream);
+    if (n < 0) return fail(CRSD_ERR_CUDA, std::string("kernel launch: ") + cudaGetErrorString(cudaGetLastError()));
+    launches += n;
+    return CRSD_OK;
+}
+
+crsd_status_t run_lists(crsd_matrix_s *A, const void *alpha, const void *x_base, const void *beta, void *y,
+                        const int32_t *list, int64_t count, void *stream, int &launches) {
+    if (A->H.dtype == CRSD_R64F)
+        return run_spmv<double>(A, *(const double *)alpha, (const double *)x_base, *(const double *)beta, (double *)y,
+                                list, count, stream, launches);
+    return run_spmv<float>(A, *(const float *)alpha, (const float *)x_base, *(const float *)beta, (float *)y, list,
+                           count, stream, launches);
+}
+
+}  // namespace crsd
+
+using namespace crsd;
+
+extern "C" {
+
+const char *crsd_last_error(void) { return g_err.c_str(); }
+
+const char *crsd_version(void) { return "crsd-b200 0.1 (sm_100a)"; }
+
+crsd_status_t crsd_opts_init(crsd_opts_t *o) {
+    if (!o) return fail(CRSD_ERR_INVALID_ARG, "opts is NULL");
+    std::memset(o, 0, sizeof(*o));
+    o->mrows = 0;
+    o->idle_max = -1;
+    o->device = -1;
+    return CRSD_OK;
+}
+
+static crsd_status_t create_common(int64_t nrows, int64_t ncols, crsd_dtype_t dtype, const crsd_opts_t *opts,
+                                   crsd_matrix_t *out, bool csr, int64_t nnz, const int64_t *row_or_ptr,
+                                   const int64_t *col, const void *val) {
+    if (!out) return fail(CRSD_ERR_INVALID_ARG, "out is NULL");
+    *out = nullptr;
+    if (dtype != CRSD_R32F && dtype != CRSD_R64F) return fail(CRSD_ERR_INVALID_ARG, "bad dtype");
+    crsd_opts_t o;
+    BuildOptions b;
+    resolve_opts(nrows, dtype, opts, o, b);
+    crsd_matrix_s *A = new (std::nothrow) crsd_matrix_s();
+    if (!A) return fail(CRSD_ERR_ALLOC, "handle allocation failed");
+    A->host_only = (o.flags & CRSD_HOST_ONLY) != 0;
+    A->device = o.device;
+    A->H.partitioned = !(o.row_begin == 0 && o.row_end == nrows);
+    crsd_status_t st = csr ? build_from_csr(nrows, ncols, row_or_ptr, col, val, dtype, b, A->H)
+                           : build_from_coo(nrows, ncols, nnz, row_or_ptr, col, val, dtype, b, A->H);
+    if (st) {
+        delete A;
+        return st;
+    }
+    A->H.partitioned = !(o.row_begin == 0 && o.row_end == nrows);
+    if (A->H.partitioned && nrows != ncols) {
+        delete A;
+        return fail(CRSD_ERR_UNSUPPORTED, "row-partitioned handles need a square matrix");
+    }
+    return finish_create(A, o, out);
+}
+
+crsd_status_t crsd_create_from_coo(int64_t nrows, int64_t ncols, int64_t nnz, const int64_t *row, const int64_t *col,
+                                   const void *val, crsd_dtype_t dtype, const crsd_opts_t *opts, crsd_matrix_t *out) {
+    return create_common(nrows, ncols, dtype, opts, out, false, nnz, row, col, val);
+}
+
+crsd_status_t crsd_create_from_csr(int64_t nrows, int64_t ncols, const int64_t *row_ptr, const int64_t *col,
+                                   const void *val, crsd_dtype_t dtype, const crsd_opts_t *opts, crsd_matrix_t *out) {
+    return create_common(nrows, ncols, dtype, opts, out, true, 0, row_ptr, col, val);
+}
+
+crsd_status_t crsd_destroy(crsd_matrix_t A) {
+    if (!A) return CRSD_OK;
+    free_device(A);
+    delete A;
+    return CRSD_OK;
+}
+
+static crsd_status_t check_vec(const void *p, const char *name) {
+    if (!p) return fail(CRSD_ERR_INVALID_ARG, std::string(name) + " is NULL");
+    if (((uintptr_t)p) & 15) return fail(CRSD_ERR_INVALID_ARG, std::string(name) + " must be 16-byte aligned");
+    return CRSD_OK;
+}
+
+crsd_status_t crsd_spmv(crsd_matrix_t A, const void *alpha, const void *x, const void *beta, void *y, void *stream) {
+    if (!A) return fail(CRSD_ERR_INVALID_ARG, "A is NULL");
+    if (A->host_only) return fail(CRSD_ERR_UNSUPPORTED, "host-only handle");
+    if (A->H.partitioned) return fail(CRSD_ERR_UNSUPPORTED, "row-partitioned handle: use crsd_spmv_dist");
+    if (!alpha || !beta) return fail(CRSD_ERR_INVALID_ARG, "alpha/beta NULL");
+    crsd_status_t st;
+    if ((st = check_vec(x, "x")) || (st = check_vec(y, "y"))) return st;
+    if (x == y) return fail(CRSD_ERR_INVALID_ARG, "x and y must not alias");
+    int launches = 0;
+    cudaSetDevice(A->device);
+    const int64_t nseg = A->H.nseg;
+    st = run_lists(A, alpha, x, beta, y, nullptr, nseg, stream, launches);
+    A->last_launches = launches;
+    return st;
+}
+
+crsd_status_t crsd_spmv_host(crsd_matrix_t A, const void *alpha, const void *x_host, const void *beta, void *y_host,
+                             void *stream) {
+    if (!A) return fail(CRSD_ERR_INVALID_ARG, "A is NULL");
+    if (A->host_only) return fail(CRSD_ERR_UNSUPPORTED, "host-only handle");
+    if (A->H.partitioned) return fail(CRSD_ERR_UNSUPPORTED, "row-partitioned handle");
+    if (!x_host || !y_host || !alpha || !beta) return fail(CRSD_ERR_INVALID_ARG, "NULL argument");
+    cudaSetDevice(A->device);
+    const size_t es = A->H.elem;
+    const size_t xb = A->H.ncols * es, yb = A->H.nrows * es;
+    int64_t dummy = 0;
+    crsd_status_t st;
+    if (!A->d_x_scratch) {
+        if ((st = dev_alloc_copy(&A->d_x_scratch, nullptr, xb, dummy))) return st;
+        if ((st = dev_alloc_copy(&A->d_y_scratch, nullptr, yb, dummy))) return st;
+        A->device_bytes += dummy;
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    const bool beta_nz = (A->H.dtype == CRSD_R64F) ? (*(const double *)beta != 0.0) : (*(const float *)beta != 0.0f);
+    CUDA_TRY(cudaMemcpyAsync(A->d_x_scratch, x_host, xb, cudaMemcpyHostToDevice, s));
+    if (beta_nz) CUDA_TRY(cudaMemcpyAsync(A->d_y_scratch, y_host, yb, cudaMemcpyHostToDevice, s));
+    if ((st = crsd_spmv(A, alpha, A->d_x_scratch, beta, A->d_y_scratch, stream))) return st;
+    CUDA_TRY(cudaMemcpyAsync(y_host, A->d_y_scratch, yb, cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    return CRSD_OK;
+}
+
+crsd_status_t crsd_get_info(crsd_matrix_t A, crsd_info_t *I) {
+    if (!A || !I) return fail(CRSD_ERR_INVALID_ARG, "NULL argument");
+    const HostCRSD &H = A->H;
+    std::memset(I, 0, sizeof(*I));
+    I->nrows = H.nrows;
+    I->ncols = H.ncols;
+    I->row_begin = H.row_begin;
+    I->row_end = H.row_end;
+    I->mrows = H.mrows;
+    I->idle_max = H.idle_max;
+    I->dtype = H.dtype;
+    I->rows_per_thread = A->rpt;
+    I->nnz = H.nnz;
+    I->nseg = H.nseg;
+    I->ninst = (int64_t)H.inst.size();
+    I->npat = H.npat();
+    I->noffsets = (int64_t)H.pat_offsets.size();
+    int64_t mx = 0;
+    for (int64_t p = 0; p < H.npat(); ++p) mx = std::max<int64_t>(mx, H.ndias((int32_t)p));
+    I->max_ndias = mx;
+    I->nslots = H.nslots;
+    I->ndiag_nnz = H.ndiag_nnz;
+    I->nfills = H.nslots - H.ndiag_nnz;
+    I->nscatter = H.nscatter();
+    I->nedge_seg = A->nedge;
+    I->halo_lo = A->halo_lo;
+    I->halo_hi = A->halo_hi;
+    I->device_bytes = A->device_bytes;
+    // algorithmic bytes: stored slots + scatter
+    // (value + row + col) + x once + y written (+ y read when beta != 0)
+    const int64_t es = H.elem;
+    const int64_t xs = H.partitioned ? H.n_local : H.ncols;
+    const int64_t base = H.nslots * es + I->nscatter * (es + 4 + 8) + xs * es + H.n_local * es;
+    I->unique_bytes_beta0 = base;
+    I->unique_bytes_beta1 = base + H.n_local * es;
+    return CRSD_OK;
+}
+
+crsd_status_t crsd_export(crsd_matrix_t A, crsd_export_t *E) {
+    if (!A || !E) return fail(CRSD_ERR_INVALID_ARG, "NULL argument");
+    const HostCRSD &H = A->H;
+    for (size_t i = 0; i < H.inst.size(); ++i) {
+        if (E->inst_first_seg) E->inst_first_seg[i] = H.inst[i].first_seg;
+        if (E->inst_nseg) E->inst_nseg[i] = H.inst[i].nseg;
+        if (E->inst_pattern) E->inst_pattern[i] = H.inst[i].pattern;
+    }
+    if (E->pat_ptr) std::copy(H.pat_ptr.begin(), H.pat_ptr.end(), E->pat_ptr);
+    if (E->pat_offsets) std::copy(H.pat_offsets.begin(), H.pat_offsets.end(), E->pat_offsets);
+    if (E->scat_ptr) std::copy(H.scat_ptr.begin(), H.scat_ptr.end(), E->scat_ptr);
+    if (E->scat_row) std::copy(H.scat_row.begin(), H.scat_row.end(), E->scat_row);
+    if (E->scat_col) std::copy(H.scat_col.begin(), H.scat_col.end(), E->scat_col);
+    const size_t vb = (size_t)H.nslots * H.elem, sb = (size_t)H.nscatter() * H.elem;
+    if (A->host_vals_dropped) {
+        cudaSetDevice(A->device);
+        if (E->vals && vb) CUDA_TRY(cudaMemcpy(E->vals, A->d_vals, vb, cudaMemcpyDeviceToHost));
+        if (E->scat_val && sb) CUDA_TRY(cudaMemcpy(E->scat_val, A->d_scat_val, sb, cudaMemcpyDeviceToHost));
+    } else {
+        if (E->vals && vb) std::memcpy(E->vals, H.vals.data(), vb);
+        if (E->scat_val && sb) std::memcpy(E->scat_val, H.scat_val.data(), sb);
+    }
+    return CRSD_OK;
+}
+
+crsd_status_t crsd_last_launch_count(crsd_matrix_t A, int32_t *count) {
+    if (!A || !count) return fail(CRSD_ERR_INVALID_ARG, "NULL argument");
+    *count = A->last_launches;
+    return CRSD_OK;
+}
+
+crsd_status_t crsd_dist_x_layout(crsd_matrix_t A, int64_t *halo_lo, int64_t *n_local, int64_t *halo_hi) {
+    if (!A) return fail(CRSD_ERR_INVALID_ARG, "A is NULL");
+    if (halo_lo) *halo_lo = A->halo_lo;
+    if (n_local) *n_local = A->H.n_local;
+    if (halo_hi) *halo_hi = A->halo_hi;
+    return CRSD_OK;
+}
+
+crsd_status_t crsd_partition_rows(int64_t nrows, int32_t mrows, int world, const double *weights, int64_t *bounds) {
+    if (nrows <= 0 || mrows <= 0 || world <= 0 || !bounds) return fail(CRSD_ERR_INVALID_ARG, "bad argument");
+    const int64_t nseg = (nrows + mrows - 1) / mrows;
+    // per-segment weight prefix; cut where the prefix crosses k/world of the total
+    std::vector<double> pre(nseg + 1, 0.0);
+    for (int64_t s = 0; s < nseg; ++s) {
+        double w = 0.0;
+        const int64_t r1 = std::min<int64_t>(nrows, (s + 1) * mrows);
+        if (weights) {
+            for (int64_t r = s * mrows; r < r1; ++r) w += weights[r];
+        } else {
+            w = double(r1 - s * mrows);
+        }
+        pre[s + 1] = pre[s] + w;
+    }
+    bounds[0] = 0;
+    int64_t s = 0;
+    for (int k = 1; k < world; ++k) {
+        const double target = pre[nseg] * k / world;
+        while (s < nseg && pre[s + 1] <= target) ++s;
+        // choose the nearer boundary
+        int64_t cut = s;
+        if (s < nseg && (pre[s + 1] - target) < (target - pre[s])) cut = s + 1;
+        int64_t prev = (bounds[k - 1] + mrows - 1) / mrows;
+        cut = std::max(cut, prev);
+        bounds[k] = std::min<int64_t>(nrows, cut * mrows);
+    }
+    bounds[world] = nrows;
+    return CRSD_OK;
+}
+
+}  // extern "C"

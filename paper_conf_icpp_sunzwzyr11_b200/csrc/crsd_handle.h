@@ -1,0 +1,53 @@
+// Opaque handle types behind crsd_matrix_t / crsd_comm_t.
+#pragma once
+
+#include <cstdint>
+#include <vector>
+
+#include "crsd_internal.h"
+
+struct crsd_matrix_s {
+    crsd::HostCRSD H;
+    bool host_only = false;
+    bool host_vals_dropped = false;
+    int device = -1;
+    int sm_count = 148;
+    int rpt = 2;
+    int32_t last_launches = 0;
+    int64_t device_bytes = 0;
+
+    // x layout (relative to the local x base)
+    int64_t halo_lo = 0, halo_hi = 0;              // allocated pads (halo_lo multiple of 4)
+    int64_t halo_lo_valid = 0, halo_hi_valid = 0;  // elements actually exchanged
+    int64_t x_lo = 0, x_hi = 0;                    // valid x range
+
+    std::vector<crsd::SegDesc> segdesc;
+    std::vector<int32_t> list_interior, list_boundary;
+    int64_t nedge = 0;
+
+    // device arrays
+    void *d_vals = nullptr;
+    void *d_segs = nullptr;
+    void *d_offs = nullptr;
+    void *d_scat_row = nullptr;
+    void *d_scat_col = nullptr;
+    void *d_scat_val = nullptr;
+    void *d_list_interior = nullptr;
+    void *d_list_boundary = nullptr;
+    void *d_list_all_edge = nullptr;
+    void *d_x_scratch = nullptr;
+    void *d_y_scratch = nullptr;
+
+    // multi-GPU plan (crsd_dist_bind)
+    bool bound = false;
+    std::vector<int64_t> recv_peer, recv_off, recv_count;  // offsets into x_padded
+    std::vector<int64_t> send_peer, send_off, send_count;
+};
+
+namespace crsd {
+void free_device(crsd_matrix_s *A);
+// Run the SpMV kernel over a device list of segments (list == nullptr: all
+// segments [0, count)). x_base is the local x base (x_padded + halo_lo).
+crsd_status_t run_lists(crsd_matrix_s *A, const void *alpha, const void *x_base, const void *beta, void *y,
+                        const int32_t *list, int64_t count, void *stream, int &launches);
+}  // namespace crsd

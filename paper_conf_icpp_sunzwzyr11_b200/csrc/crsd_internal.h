@@ -1,0 +1,127 @@
+// Internal structures of libcrsd (host builder <-> C-ABI <-> CUDA kernels).
+// Not part of the public ABI (include/crsd.h).
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/crsd.h"
+
+namespace crsd {
+
+// ----------------------------------------------------------------------------
+// errors
+// ----------------------------------------------------------------------------
+void set_error(const std::string &msg);
+crsd_status_t fail(crsd_status_t st, const std::string &msg);
+
+// ----------------------------------------------------------------------------
+// Host CRSD (B200 layout)
+// ----------------------------------------------------------------------------
+struct Instance {          // the paper's diagonal pattern p (Table II)
+    int64_t first_seg;     // SR_p / mrows
+    int64_t nseg;          // NRS_p
+    int32_t pattern;       // index into HostCRSD::pat_*
+    int64_t val_base;      // sum_{i<p} NRS_i * NNzRS_i
+};
+
+// Segment flags
+enum : int32_t { SEG_EDGE = 1, SEG_BOUNDARY = 2 };
+
+// Per-segment descriptor read by one CTA (uniform).
+struct alignas(16) SegDesc {
+    int64_t val_base;    // slot of (segment, d=0, l=0)
+    int64_t scat_begin;  // first scatter entry of the segment
+    int32_t off_begin;   // first offset of the segment's pattern in pat_offs
+    int32_t nscat;       // scatter entries
+    int32_t flags;       // SEG_*
+    int32_t ndias;       // NDias of the pattern
+};
+static_assert(sizeof(SegDesc) == 32, "SegDesc must be 32 bytes");
+
+struct HostCRSD {
+    int64_t nrows = 0, ncols = 0;    // global
+    int64_t row_begin = 0, row_end = 0;
+    int64_t n_local = 0;             // row_end - row_begin
+    bool partitioned = false;
+    int32_t mrows = 256, idle_max = 255;
+    crsd_dtype_t dtype = CRSD_R64F;
+    int elem = 8;                    // sizeof(value)
+    int64_t nseg = 0;
+    int64_t nnz = 0;
+
+    // distinct patterns (ascending offsets)
+    std::vector<int64_t> pat_ptr;     // npat + 1
+    std::vector<int64_t> pat_offsets;
+    std::vector<Instance> inst;
+
+    std::vector<uint8_t> vals;        // nslots * elem
+    int64_t nslots = 0, ndiag_nnz = 0;
+
+    std::vector<int64_t> scat_ptr;    // nseg + 1
+    std::vector<int32_t> scat_row;    // row within segment
+    std::vector<int64_t> scat_col;    // global column
+    std::vector<uint8_t> scat_val;    // nscatter * elem
+
+    // column extent actually referenced (global), over stored entries
+    int64_t min_col_ref = 0, max_col_ref = -1;
+
+    int64_t npat() const { return (int64_t)pat_ptr.size() - 1; }
+    int64_t nscatter() const { return scat_ptr.empty() ? 0 : scat_ptr.back(); }
+    int64_t ndias(int32_t p) const { return pat_ptr[p + 1] - pat_ptr[p]; }
+};
+
+struct BuildOptions {
+    int32_t mrows, idle_max;
+    uint32_t flags;
+    int64_t row_begin, row_end;
+    int32_t nthreads;
+};
+
+// COO -> HostCRSD. val points to float or double per dtype.
+crsd_status_t build_from_coo(int64_t nrows, int64_t ncols, int64_t nnz, const int64_t *row, const int64_t *col,
+                             const void *val, crsd_dtype_t dtype, const BuildOptions &o, HostCRSD &H);
+crsd_status_t build_from_csr(int64_t nrows, int64_t ncols, const int64_t *row_ptr, const int64_t *col,
+                             const void *val, crsd_dtype_t dtype, const BuildOptions &o, HostCRSD &H);
+
+// x window of a segment for the GPU kernel with RPT rows per thread: the
+// element range [lo, hi) relative to the local x base that the vector loads
+// of a non-edge segment touch.
+void segment_x_window(const HostCRSD &H, int64_t s, int rpt, int64_t &lo, int64_t &hi);
+
+// Segment descriptors + flags. x_lo/x_hi: valid x range relative to the
+// local x base; own_hi: n_local (the x the rank owns is [0, own_hi)).
+void make_segdescs(const HostCRSD &H, int rpt, int64_t x_lo, int64_t x_hi, std::vector<SegDesc> &out);
+
+// Halo extents (elements outside [0, n_local) relative to the local x base)
+// the handle needs: from its non-edge windows and its scatter columns.
+void needed_halo(const HostCRSD &H, int rpt, int64_t &need_lo, int64_t &need_hi);
+
+// ----------------------------------------------------------------------------
+// device side
+// ----------------------------------------------------------------------------
+template <typename T>
+struct SpmvArgs {
+    const T *vals;
+    const SegDesc *segs;
+    const int32_t *pat_offs;
+    const int32_t *scat_row;
+    const int64_t *scat_col;  // relative to x base
+    const T *scat_val;
+    const T *x;               // local x base (x_padded + halo_lo for dist)
+    int64_t x_lo, x_hi;       // valid x range relative to x
+    T *y;
+    int64_t nrows;            // local rows
+    const int32_t *seg_list;  // if non-null: CTA work = seg_list[i]
+    int64_t seg_begin, seg_count;
+    int32_t mrows;
+    T alpha, beta;
+};
+
+// Launch the SpMV kernel for the given work (range or list) on `stream`.
+// Returns number of launches (0 if no work) or -1 on launch error.
+template <typename T>
+int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream);
+
+}  // namespace crsd

@@ -1,0 +1,260 @@
+// CRSD SpMV kernels for sm_100a (B200): y = alpha*A*x + beta*y.
+//
+// Work decomposition (§III-B): one CTA per row segment,
+// RPT consecutive rows per thread (RPT = 2 fp64 / 4 fp32) so every value and
+// x access is one 128-bit vector. A CTA reads its segment descriptor once,
+// which selects the diagonal pattern -- the paper's group_id -> pattern lookup
+// precomputed on the host -- so all threads of a CTA take the
+// same path. The pattern's offsets come from a small table
+// (uniform, L1-resident); no per-nonzero index is loaded.
+//
+// Per diagonal d (ascending offset o_d):
+//   value  vals[val_base + d*mrows + l]     -- 128-bit, coalesced, streamed
+//          with an L2 evict_first policy (read exactly once)
+//   x      x[row0 + l + o_d]: the thread loads the ALIGNED vector holding
+//          x[row0 + RPT*(t + floor(o_d/RPT))]; when o_d is not a multiple of
+//          RPT the next vector comes from the neighbour lane by a warp
+//          shuffle (lane 31 loads it). This replaces the paper's local-memory
+//          staging of x for adjacent groups (Fig. 5) by register
+//          exchange: no shared memory, no barrier (the barrier cost the paper
+//          measures on wang3/wang4, does not exist here).
+//   acc_j = fma(value_j, x_j, acc_j)         -- ascending offset order
+// Edge segments (x window outside the valid range, or the partial last
+// segment, R9/R11) run a guarded scalar-x body.
+// Scatter points of the segment (R5) are added by their owner
+// thread after the diagonal part, in (row, col) order; then the epilogue
+// writes y once (y read only when beta != 0).
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "crsd_internal.h"
+
+namespace crsd {
+
+template <typename T>
+struct VecT;
+template <>
+struct VecT<double> {
+    using type = double2;
+    static constexpr int R = 2;
+    static constexpr int LOG = 1;
+};
+template <>
+struct VecT<float> {
+    using type = float4;
+    static constexpr int R = 4;
+    static constexpr int LOG = 2;
+};
+
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+
+// streamed values: no L1 allocation, L2 evict_first
+__device__ __forceinline__ double2 ld_stream(const double2 *ptr, uint64_t pol) {
+    double2 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;"
+                 : "=d"(r.x), "=d"(r.y)
+                 : "l"(ptr), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ float4 ld_stream(const float4 *ptr, uint64_t pol) {
+    float4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
+                 : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+                 : "l"(ptr), "l"(pol));
+    return r;
+}
+// x: reused across diagonals (L1) and segments (L2)
+__device__ __forceinline__ double2 ld_x(const double2 *ptr) { return __ldg(ptr); }
+__device__ __forceinline__ float4 ld_x(const float4 *ptr) { return __ldg(ptr); }
+
+__device__ __forceinline__ void st_stream(double2 *ptr, double2 v) {
+    asm volatile("st.global.L1::no_allocate.v2.f64 [%0], {%1, %2};" ::"l"(ptr), "d"(v.x), "d"(v.y) : "memory");
+}
+__device__ __forceinline__ void st_stream(float4 *ptr, float4 v) {
+    asm volatile("st.global.L1::no_allocate.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(ptr), "f"(v.x), "f"(v.y), "f"(v.z),
+                 "f"(v.w)
+                 : "memory");
+}
+
+__device__ __forceinline__ double2 shfl_down1(double2 v) {
+    return make_double2(__shfl_down_sync(0xffffffffu, v.x, 1), __shfl_down_sync(0xffffffffu, v.y, 1));
+}
+__device__ __forceinline__ float4 shfl_down1(float4 v) {
+    return make_float4(__shfl_down_sync(0xffffffffu, v.x, 1), __shfl_down_sync(0xffffffffu, v.y, 1),
+                       __shfl_down_sync(0xffffffffu, v.z, 1), __shfl_down_sync(0xffffffffu, v.w, 1));
+}
+
+__device__ __forceinline__ double get(const double2 &v, int j) { return j == 0 ? v.x : v.y; }
+__device__ __forceinline__ float get(const float4 &v, int j) {
+    return j == 0 ? v.x : (j == 1 ? v.y : (j == 2 ? v.z : v.w));
+}
+
+// x_j = concat(a, b)[al + j], al in [1, R): uniform al, register-only selects
+__device__ __forceinline__ void window(const double2 &a, const double2 &b, int /*al == 1*/, double (&xs)[2]) {
+    xs[0] = a.y;
+    xs[1] = b.x;
+}
+__device__ __forceinline__ void window(const float4 &a, const float4 &b, int al, float (&xs)[4]) {
+    if (al == 1) {
+        xs[0] = a.y; xs[1] = a.z; xs[2] = a.w; xs[3] = b.x;
+    } else if (al == 2) {
+        xs[0] = a.z; xs[1] = a.w; xs[2] = b.x; xs[3] = b.y;
+    } else {
+        xs[0] = a.w; xs[1] = b.x; xs[2] = b.y; xs[3] = b.z;
+    }
+}
+
+__device__ __forceinline__ double2 make_vec(const double (&v)[2]) { return make_double2(v[0], v[1]); }
+__device__ __forceinline__ float4 make_vec(const float (&v)[4]) { return make_float4(v[0], v[1], v[2], v[3]); }
+
+template <typename T, int CH>
+__global__ void __launch_bounds__(256) crsd_spmv_kernel(const SpmvArgs<T> a) {
+    using V = typename VecT<T>::type;
+    constexpr int R = VecT<T>::R;
+    constexpr int LOG = VecT<T>::LOG;
+    const int t = threadIdx.x;
+    const int lane = t & 31;
+    const int64_t vstride = a.mrows >> LOG;  // vectors per diagonal of a segment
+    const uint64_t pol = policy_evict_first();
+
+    for (int64_t w = blockIdx.x; w < a.seg_count; w += gridDim.x) {
+        const int64_t s = a.seg_list ? (int64_t)__ldg(a.seg_list + w) : a.seg_begin + w;
+        const SegDesc D = a.segs[s];
+        const int64_t row0 = s * a.mrows;
+        const int nd = D.ndias;
+        const int32_t *offs = a.pat_offs + D.off_begin;
+        const V *vb = reinterpret_cast<const V *>(a.vals + D.val_base) + t;
+        T acc[R];
+#pragma unroll
+        for (int j = 0; j < R; ++j) acc[j] = T(0);
+
+        if (!(D.flags & SEG_EDGE)) {
+            const V *xv = reinterpret_cast<const V *>(a.x + row0) + t;
+            for (int d0 = 0; d0 < nd; d0 += CH) {
+                V val[CH], xa[CH], xe[CH];
+                int o[CH];
+#pragma unroll
+                for (int c = 0; c < CH; ++c) {
+                    if (d0 + c < nd) {
+                        o[c] = __ldg(offs + d0 + c);
+                        val[c] = ld_stream(vb + (int64_t)(d0 + c) * vstride, pol);
+                    }
+                }
+#pragma unroll
+                for (int c = 0; c < CH; ++c) {
+                    if (d0 + c < nd) {
+                        const int k = o[c] >> LOG;  // floor(o / R)
+                        xa[c] = ld_x(xv + k);
+                        if ((o[c] & (R - 1)) && lane == 31) xe[c] = ld_x(xv + k + 1);
+                    }
+                }
+#pragma unroll
+                for (int c = 0; c < CH; ++c) {
+                    if (d0 + c < nd) {
+                        const int al = o[c] & (R - 1);  // warp-uniform
+                        T xs[R];
+                        if (al == 0) {
+#pragma unroll
+                            for (int j = 0; j < R; ++j) xs[j] = get(xa[c], j);
+                        } else {
+                            V nb = shfl_down1(xa[c]);
+                            if (lane == 31) nb = xe[c];
+                            window(xa[c], nb, al, xs);
+                        }
+#pragma unroll
+                        for (int j = 0; j < R; ++j) acc[j] = fma(get(val[c], j), xs[j], acc[j]);
+                    }
+                }
+            }
+        } else {
+            // guarded body: x indices outside [x_lo, x_hi) belong to filled
+            // zeros only (R9/R11) and are never dereferenced
+            const int64_t r = row0 + (int64_t)t * R;
+            for (int d = 0; d < nd; ++d) {
+                const int o = __ldg(offs + d);
+                const V v = ld_stream(vb + (int64_t)d * vstride, pol);
+#pragma unroll
+                for (int j = 0; j < R; ++j) {
+                    const int64_t idx = r + j + o;
+                    const T xj = (idx >= a.x_lo && idx < a.x_hi) ? __ldg(a.x + idx) : T(0);
+                    acc[j] = fma(get(v, j), xj, acc[j]);
+                }
+            }
+        }
+
+        // scatter points of this segment, (row, col) order, owner thread adds
+        if (D.nscat > 0) {
+            const int lo = t * R, hi = lo + R;
+            const int32_t *sr = a.scat_row + D.scat_begin;
+            int64_t e = 0;
+            const int64_t ne = D.nscat;
+            if (ne > 32) {  // binary search for the first entry of this thread's rows
+                int64_t l = 0, h = ne;
+                while (l < h) {
+                    const int64_t mid = (l + h) >> 1;
+                    if (__ldg(sr + mid) < lo) l = mid + 1; else h = mid;
+                }
+                e = l;
+            }
+            for (; e < ne; ++e) {
+                const int rr = __ldg(sr + e);
+                if (rr >= hi) {
+                    if (ne > 32) break;
+                    continue;
+                }
+                if (rr < lo) continue;
+                const T v = __ldg(a.scat_val + D.scat_begin + e);
+                const T xv = __ldg(a.x + __ldg(a.scat_col + D.scat_begin + e));
+#pragma unroll
+                for (int j = 0; j < R; ++j)
+                    if (rr - lo == j) acc[j] = fma(v, xv, acc[j]);
+            }
+        }
+
+        // epilogue: y = alpha*acc + beta*y, y not read when beta == 0
+        const T al = a.alpha, be = a.beta;
+        if (!(D.flags & SEG_EDGE)) {
+            V *yv = reinterpret_cast<V *>(a.y + row0) + t;
+            T out[R];
+            if (be != T(0)) {
+                const V yo = *yv;
+#pragma unroll
+                for (int j = 0; j < R; ++j) out[j] = fma(al, acc[j], be * get(yo, j));
+            } else {
+#pragma unroll
+                for (int j = 0; j < R; ++j) out[j] = al * acc[j];
+            }
+            st_stream(yv, make_vec(out));
+        } else {
+            const int64_t r = row0 + (int64_t)t * R;
+#pragma unroll
+            for (int j = 0; j < R; ++j) {
+                if (r + j < a.nrows) {
+                    a.y[r + j] = (be != T(0)) ? fma(al, acc[j], be * a.y[r + j]) : al * acc[j];
+                }
+            }
+        }
+    }
+}
+
+template <typename T>
+int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
+    if (a.seg_count <= 0) return 0;
+    constexpr int R = VecT<T>::R;
+    const int threads = a.mrows / R;
+    int64_t grid = a.seg_count;
+    if (grid > 0x7fffffff) grid = 0x7fffffff;
+    (void)sm_count;
+    crsd_spmv_kernel<T, 4><<<(unsigned)grid, threads, 0, (cudaStream_t)stream>>>(a);
+    return cudaGetLastError() == cudaSuccess ? 1 : -1;
+}
+
+template int launch_spmv<double>(const SpmvArgs<double> &, int, void *);
+template int launch_spmv<float>(const SpmvArgs<float> &, int, void *);
+
+}  // namespace crsd

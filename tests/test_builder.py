@@ -1,0 +1,187 @@
+"""Host CRSD builder (libcrsd, C++) against the oracle (CPU only).
+
+Integer/index work is compared bit-exactly: the product's export must equal
+the paper-order construction of oracle.crsd_ref (instances, offsets, value
+array bytes, scatter lists), and must round-trip to the canonical COO through
+the independent oracle decoder.
+"""
+import ctypes
+
+import numpy as np
+import pytest
+from hypothesis import given, settings, strategies as st
+
+import gen
+from oracle import crsd_ref, decode
+from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, CRSDError, CRSD_SUM_DUPLICATES, CRSD_DROP_ZEROS
+from paper_conf_icpp_sunzwzyr11_b200 import crsd as C
+
+
+def _bits(a):
+    a = np.ascontiguousarray(a)
+    return a.view(np.uint64 if a.dtype == np.float64 else np.uint32)
+
+
+def assert_layout_equal(P, L):
+    assert P["inst_first_seg"].tolist() == L["inst_first_seg"].tolist()
+    assert P["inst_nseg"].tolist() == L["inst_nseg"].tolist()
+    assert P["inst_offsets"] == L["inst_offsets"]
+    assert P["vals"].dtype == L["vals"].dtype
+    assert np.array_equal(_bits(P["vals"]), _bits(L["vals"]))
+    assert P["scat_ptr"].tolist() == L["scat_ptr"].tolist()
+    assert P["scat_row"].tolist() == L["scat_row"].tolist()
+    assert P["scat_col"].tolist() == L["scat_col"].tolist()
+    assert np.array_equal(_bits(P["scat_val"]), _bits(L["scat_val"]))
+
+
+def test_library_exports_every_header_symbol():
+    import re, os
+
+    hdr = open(os.path.join(os.path.dirname(__file__), "..", "include", "crsd.h")).read()
+    declared = set(re.findall(r"\b(crsd_[a-z_0-9]+)\s*\(", hdr))
+    assert declared == set(C.EXPORTED)
+    lib = ctypes.CDLL(C.LIB_PATH)
+    for name in declared:
+        assert hasattr(lib, name), name
+
+
+def test_fig2_export_equals_paper(fig2, fig2_expected):
+    n, m, r, c, v, _ = fig2
+    A = CRSDMatrix.from_coo(n, m, r, c, v, mrows=2, idle_max=1, host_only=True)
+    P = A.export()
+    R = crsd_ref.build(n, m, r, c, v, mrows=2, idle_max=1)
+    assert_layout_equal(P, crsd_ref.to_layout(R))
+    inf = A.info()
+    assert (inf["ninst"], inf["nfills"], inf["nscatter"]) == (2, 1, 1)
+
+
+@settings(max_examples=60, deadline=None)
+@given(
+    n=st.integers(1, 70),
+    m=st.integers(1, 70),
+    seed=st.integers(0, 100_000),
+    mrows=st.sampled_from([1, 2, 3, 4, 7, 32]),
+    im=st.integers(-1, 9),
+    nz=st.integers(0, 3),
+    dt=st.sampled_from([np.float64, np.float32]),
+    shuffle=st.booleans(),
+)
+def test_builder_matches_oracle_random(n, m, seed, mrows, im, nz, dt, shuffle):
+    a = gen.random_diagonal(n, m, seed, ndiag=6, p_break=0.12, max_break=6, n_scatter=5, n_zeros=nz).astype(dt)
+    if shuffle:
+        a = a.shuffled(seed)
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, mrows=mrows, idle_max=im, host_only=True)
+    P = A.export()
+    R = crsd_ref.build(a.nrows, a.ncols, a.row, a.col, a.val, mrows=mrows, idle_max=im, dtype=dt)
+    assert_layout_equal(P, crsd_ref.to_layout(R))
+    decode.check_invariants(P, R.idle_max, a.nrows, a.ncols, a.row, a.col, a.val)
+
+
+@pytest.mark.parametrize("mrows", [64, 256])
+def test_builder_c1_matches_oracle(mrows):
+    a = gen.config1()
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, mrows=mrows, host_only=True)
+    R = crsd_ref.build(a.nrows, a.ncols, a.row, a.col, a.val, mrows=mrows)
+    assert_layout_equal(A.export(), crsd_ref.to_layout(R))
+    assert A.info()["nscatter"] == 16
+
+
+def test_builder_reduced_c3_matches_oracle():
+    a = gen.config3(n=16, scatter_frac=0.002)
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, mrows=64, host_only=True)
+    R = crsd_ref.build(a.nrows, a.ncols, a.row, a.col, a.val, mrows=64)
+    assert_layout_equal(A.export(), crsd_ref.to_layout(R))
+
+
+def test_builder_reduced_c4_structure():
+    """C4 scaled to 400k rows: 4 pattern row ranges; the generator's edge rows
+    drop out-of-range offsets so more instances appear near the ends."""
+    a = gen.config4(n=400_000)
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, mrows=512, host_only=True)
+    P = A.export()
+    decode.check_invariants(P, 511, a.nrows, a.ncols, a.row, a.col, a.val, check_rule=False)
+    sets = [tuple(o) for o in P["inst_offsets"]]
+    for _, _, offs in gen.matrices.c4_ranges(400_000):
+        assert tuple(offs) in sets
+    assert A.info()["nscatter"] == 0
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_roundtrip_c2_reduced(dt):
+    a = gen.config2(n=48).astype(dt)
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, host_only=True)
+    P = A.export()
+    assert decode.roundtrip_equal(P, a.nrows, a.ncols, a.row, a.col, a.val)
+    inf = A.info()
+    assert inf["nnz"] == a.nnz and inf["nscatter"] == 0
+
+
+def test_roundtrip_c3_reduced_shuffled():
+    a = gen.config3(n=32).shuffled(9)
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, mrows=256, host_only=True)
+    P = A.export()
+    decode.check_invariants(P, 255, a.nrows, a.ncols, a.row, a.col, a.val, check_rule=False)
+
+
+def test_duplicates_rejected_or_summed():
+    r = np.array([0, 1, 1, 1])
+    c = np.array([0, 1, 1, 2])
+    v = np.array([1.0, 2.0, 3.0, 4.0])
+    with pytest.raises(CRSDError, match="DUPLICATE"):
+        CRSDMatrix.from_coo(3, 3, r, c, v, mrows=2, host_only=True)
+    A = CRSDMatrix.from_coo(3, 3, r, c, v, mrows=2, host_only=True, flags=CRSD_SUM_DUPLICATES)
+    assert A.info()["nnz"] == 3
+    rr, cc, vv = decode.decode(A.export())
+    assert vv.tolist() == [1.0, 5.0, 4.0]
+
+
+def test_index_range_rejected():
+    with pytest.raises(CRSDError, match="INDEX_RANGE"):
+        CRSDMatrix.from_coo(3, 3, np.array([0]), np.array([3]), np.array([1.0]), host_only=True)
+    with pytest.raises(CRSDError, match="INVALID_ARG"):
+        CRSDMatrix.from_coo(0, 3, np.array([], np.int64), np.array([], np.int64), np.array([]), host_only=True)
+
+
+def test_explicit_zeros_kept_or_dropped():
+    r = np.array([0, 1, 2, 3])
+    c = np.array([0, 1, 2, 3])
+    v = np.array([1.0, -0.0, 2.0, 3.0])
+    A = CRSDMatrix.from_coo(4, 4, r, c, v, mrows=4, host_only=True)
+    P = A.export()
+    assert decode.roundtrip_equal(P, 4, 4, r, c, v)
+    assert P["scat_val"].tolist() == [0.0] and np.signbit(P["scat_val"][0])
+    A = CRSDMatrix.from_coo(4, 4, r, c, v, mrows=4, host_only=True, flags=CRSD_DROP_ZEROS)
+    assert A.info()["nscatter"] == 0 and A.info()["nnz"] == 3
+
+
+def test_empty_matrix_and_empty_segments():
+    A = CRSDMatrix.from_coo(10, 10, np.array([], np.int64), np.array([], np.int64), np.array([]), mrows=4, host_only=True)
+    inf = A.info()
+    assert inf["nseg"] == 3 and inf["ninst"] == 1 and inf["nslots"] == 0
+    P = A.export()
+    assert P["inst_offsets"] == [[]]
+
+
+def test_csr_input_equals_coo():
+    a = gen.config1().sorted()
+    ptr = np.zeros(a.nrows + 1, np.int64)
+    np.add.at(ptr, a.row + 1, 1)
+    ptr = np.cumsum(ptr)
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, mrows=128, host_only=True)
+    B = CRSDMatrix.from_csr(a.nrows, a.ncols, ptr, a.col, a.val, mrows=128, host_only=True)
+    assert_layout_equal(A.export(), B.export())
+
+
+def test_gpu_handle_needs_aligned_mrows():
+    a = gen.config1()
+    with pytest.raises(CRSDError, match="UNSUPPORTED"):
+        CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, mrows=96)
+
+
+def test_unique_bytes_accounting():
+    a = gen.config2(n=16)
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, host_only=True)
+    inf = A.info()
+    n = a.nrows
+    assert inf["unique_bytes_beta0"] == inf["nslots"] * 8 + n * 8 + n * 8
+    assert inf["unique_bytes_beta1"] == inf["unique_bytes_beta0"] + n * 8

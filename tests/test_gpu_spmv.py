@@ -1,0 +1,196 @@
+"""GPU parity of crsd_spmv (C-ABI, sm_100a kernels) against the oracle.
+
+Pass criterion (BASELINE.json north_star):
+    max_r |y - y_ref| / scale_r <= 1e-12 (fp64), 1e-5 (fp32),
+    scale_r = |alpha| sum_c |a_rc x_c| + |beta| |y0_r|; rows with scale 0 exact.
+Derivation of the bound: the kernel accumulates each
+row with k fused multiply-adds, plus the alpha/beta epilogue; the recursive
+summation error is <= (k + 2) u scale_r with u = 2^-53 / 2^-24. For k <= 40
+(27-point stencil + scatter) that is 4.7e-15 (fp64) and 2.5e-6 (fp32), under
+the stated tolerances.
+Closed-form checks (exact integers) are compared with ==.
+"""
+import numpy as np
+import pytest
+
+import gen
+from oracle import closed_forms, coo
+from tests.conftest import have_gpu
+
+pytestmark = pytest.mark.gpu
+
+TOL = {np.float64: 1e-12, np.float32: 1e-5}
+
+_CACHE = {}
+
+
+def cached(name, fn, *args, **kw):
+    """Full-size generators take seconds; share one instance per module."""
+    key = (name, args, tuple(sorted(kw.items())))
+    if key not in _CACHE:
+        _CACHE[key] = fn(*args, **kw)
+    return _CACHE[key]
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+
+    if not torch.cuda.is_available():
+        pytest.fail("no CUDA device: -m gpu tests need a B200")
+    return torch
+
+
+def _mat(a, **kw):
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix
+
+    return CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, **kw)
+
+
+def _run(torch, A, x, alpha=1.0, beta=0.0, y0=None, nrows=None):
+    dt = torch.float64 if A.dtype == np.float64 else torch.float32
+    xd = torch.from_numpy(np.ascontiguousarray(x)).to("cuda", dt)
+    if y0 is None:
+        yd = torch.full((nrows,), float("nan"), device="cuda", dtype=dt)
+    else:
+        yd = torch.from_numpy(np.ascontiguousarray(y0)).to("cuda", dt)
+    A.spmv(xd, yd, alpha, beta)
+    torch.cuda.synchronize()
+    return yd.cpu().numpy()
+
+
+def _parity(torch, a, dt, alpha=1.0, beta=0.0, seed=0, **kw):
+    a = a.astype(dt)
+    A = _mat(a, **kw)
+    rng = np.random.default_rng(seed)
+    x = rng.uniform(-1, 1, a.ncols).astype(dt)
+    y0 = rng.uniform(-1, 1, a.nrows).astype(dt) if beta != 0 else None
+    y = _run(torch, A, x, alpha, beta, y0, a.nrows)
+    yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, x, alpha, beta, y0)
+    err = coo.parity_error(y, yref, scale)
+    assert err <= TOL[dt], f"parity error {err:.3e}"
+    return A, err
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+@pytest.mark.parametrize("alpha,beta", [(1.0, 0.0), (-0.75, 0.0), (1.0, 1.0), (-0.75, 0.5)])
+def test_c1_parity(torch_cuda, dt, alpha, beta):
+    _parity(torch_cuda, gen.config1(), dt, alpha, beta)
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_c2_reduced_parity(torch_cuda, dt):
+    _parity(torch_cuda, gen.config2(n=40), dt, -0.75, 0.5)
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_c3_reduced_parity(torch_cuda, dt):
+    A, _ = _parity(torch_cuda, gen.config3(n=36), dt, 1.0, 0.0)
+    assert A.info()["nscatter"] > 0
+
+
+def test_c4_reduced_parity(torch_cuda):
+    _parity(torch_cuda, gen.config4(n=300_000), np.float32, 1.0, 0.0)
+
+
+@pytest.mark.parametrize("seed", range(12))
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_random_diagonal_parity(torch_cuda, seed, dt):
+    """Random offsets (AD runs), breaks, scatter, rectangular shapes, ragged tails."""
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(1, 5000))
+    m = int(rng.integers(1, 5000))
+    a = gen.random_diagonal(n, m, seed, ndiag=int(rng.integers(1, 30)), max_off=int(rng.integers(1, 3000)), p_break=0.02, max_break=400, n_scatter=int(rng.integers(0, 300)))
+    mrows = [256, 512, 1024][seed % 3] if dt == np.float64 else [128, 512, 1024][seed % 3]
+    _parity(torch_cuda, a, dt, [1.0, -0.75][seed % 2], [0.0, 0.5][(seed // 2) % 2], seed=seed, mrows=mrows)
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_dense_scatter_segments(torch_cuda, dt):
+    """Segments with hundreds of scatter points (binary-search path of the scatter pass)."""
+    n = 2048
+    a = gen.random_diagonal(n, n, 5, ndiag=3, n_scatter=3000)
+    A, _ = _parity(torch_cuda, a, dt, 1.0, 0.0)
+    assert A.info()["nscatter"] > 2000
+
+
+def test_beta_zero_never_reads_y(torch_cuda):
+    a = gen.config1()
+    A = _mat(a)
+    x = np.random.default_rng(1).uniform(-1, 1, a.ncols)
+    y = _run(torch_cuda, A, x, 1.0, 0.0, None, a.nrows)  # y prefilled with NaN
+    assert np.all(np.isfinite(y))
+
+
+def test_tiny_and_empty(torch_cuda):
+    e = np.empty(0, np.int64)
+    A = gen.COO(5, 7, e, e.copy(), np.empty(0))
+    _parity(torch_cuda, A, np.float64, 1.0, 0.5)
+    one = gen.COO(1, 1, np.array([0]), np.array([0]), np.array([2.5]))
+    _parity(torch_cuda, one, np.float64, 1.0, 0.0)
+    _parity(torch_cuda, one, np.float32, 2.0, 1.0)
+
+
+def test_misaligned_vectors_rejected(torch_cuda):
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDError
+
+    torch = torch_cuda
+    a = gen.config1()
+    A = _mat(a)
+    x = torch.zeros(a.ncols + 1, device="cuda", dtype=torch.float64)
+    y = torch.zeros(a.nrows, device="cuda", dtype=torch.float64)
+    with pytest.raises(CRSDError, match="INVALID_ARG"):
+        A.spmv(x[1:], y)
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_spmv_host_e2e(torch_cuda, dt):
+    a = gen.config3(n=24).astype(dt)
+    A = _mat(a)
+    rng = np.random.default_rng(3)
+    x = rng.uniform(-1, 1, a.ncols).astype(dt)
+    y0 = rng.uniform(-1, 1, a.nrows).astype(dt)
+    y = y0.copy()
+    A.spmv_host(x, y, -0.75, 0.5)
+    yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, x, -0.75, 0.5, y0)
+    assert coo.parity_error(y, yref, scale) <= TOL[dt]
+
+
+# ---------------------------------------------------------------- full sizes
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+@pytest.mark.parametrize("xkind", ["linear", "quadratic"])
+def test_c2_full_closed_form(torch_cuda, dt, xkind):
+    """BASELINE config 2 at full size (256^3), every row vs the closed form (exact)."""
+    dims = (256, 256, 256)
+    a = cached("c2x", gen.config2, values="exact").astype(dt)
+    A = _mat(a)
+    x = gen.vectors(a.ncols, xkind, dims=dims).astype(dt)
+    y = _run(torch_cuda, A, x, 1.0, 0.0, None, a.nrows)
+    assert np.array_equal(y.astype(np.float64), closed_forms.stencil_apply(dims, "7pt", xkind))
+
+
+def test_c2_full_random_parity(torch_cuda):
+    """Config 2 at full size with perturbed values, fp64, every row vs the oracle."""
+    _parity(torch_cuda, cached("c2", gen.config2), np.float64, -0.75, 0.5)
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_c3_full_parity(torch_cuda, dt):
+    """Config 3 at full size (192^3 27-pt, idle blocks, 0.1% scatter), every row."""
+    A, _ = _parity(torch_cuda, cached("c3", gen.config3), dt, 1.0, 0.0)
+    inf = A.info()
+    assert inf["nscatter"] > 100_000
+
+
+def test_c3_full_closed_form_ones(torch_cuda):
+    """C3 stencil part with center = present couplings: A*1 == sum of the row's scatter values."""
+    a = cached("c3x", gen.config3, values="exact")
+    A = _mat(a)
+    y = _run(torch_cuda, A, np.ones(a.ncols), 1.0, 0.0, None, a.nrows)
+    nsc = int(round((3 * 192 - 2) ** 3 * 0.001))
+    expect = np.zeros(a.nrows)
+    np.add.at(expect, a.row[-nsc:], a.val[-nsc:])
+    # scatter rows sum a few U(-1,1) values: compare with the oracle tolerance
+    yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, np.ones(a.ncols))
+    assert coo.parity_error(y, yref, scale) <= 1e-12
+    assert np.max(np.abs(yref - expect)) <= 1e-12
