@@ -147,6 +147,10 @@ def stencil(
         vals *= 1.0 + 0.1 * (2.0 * u - 1.0)
     elif values != "exact":
         raise ValueError(values)
+    if center == "present":
+        # a row without couplings has center 0: that is no nonzero at all
+        # (an idle section of the main diagonal), so it is not emitted
+        valid[:, cq] &= vals[:, cq] != 0.0
     cols = idx[:, None] + lin[None, :]
     rows = np.broadcast_to(idx[:, None], valid.shape)
     return COO(n, n, rows[valid], cols[valid], vals[valid])

@@ -66,10 +66,12 @@ typedef enum { CRSD_R32F = 0, CRSD_R64F = 1 } crsd_dtype_t;
 
 /*
  * Build options. Call crsd_opts_init() for defaults (NULL opts == defaults).
- *   mrows     row-segment height (token `mrows`); 0 => 256. The
- *             GPU path needs mrows % (32*RPT) == 0, RPT = 2 rows per thread
- *             for fp64 and 4 for fp32 (one 128-bit vector per thread and
- *             diagonal); the host builder accepts any mrows >= 1.
+ *   mrows     row-segment height (token `mrows`); 0 => 128*RPT
+ *             (256 fp64, 512 fp32: 128 threads per CTA). The
+ *             GPU path needs mrows % (32*RPT) == 0 and mrows <= 256*RPT,
+ *             RPT = 2 rows per thread for fp64 and 4 for fp32 (one 128-bit
+ *             vector per thread and diagonal; <= 256 threads per CTA); the
+ *             host builder accepts any mrows >= 1.
  *   idle_max  longest run of zeros along a diagonal that is bridged by
  *             filling zeros (R2); < 0 => mrows - 1.
  *   flags     CRSD_* flags above.
@@ -79,6 +81,11 @@ typedef enum { CRSD_R32F = 0, CRSD_R64F = 1 } crsd_dtype_t;
  *             range. row_begin must be a multiple of mrows.
  *   device    CUDA device ordinal the handle's memory lives on (-1 => current).
  *   nthreads  host builder threads (OpenMP); 0 => OpenMP default.
+ *   variant   GPU kernel: CRSD_VARIANT_AUTO (0), CRSD_VARIANT_LDG (1: 128-bit
+ *             register loads, x by warp shuffle) or CRSD_VARIANT_TMA (2: bulk
+ *             copies of the segment's values and x windows into shared
+ *             memory). AUTO picks TMA when the largest pattern's staging fits
+ *             in shared memory. DESIGN.md "Kernels".
  */
 typedef struct {
     int32_t mrows;
@@ -88,8 +95,12 @@ typedef struct {
     int64_t row_begin;
     int64_t row_end;
     int32_t nthreads;
-    int32_t reserved;
+    int32_t variant;
 } crsd_opts_t;
+
+#define CRSD_VARIANT_AUTO 0
+#define CRSD_VARIANT_LDG 1
+#define CRSD_VARIANT_TMA 2
 
 typedef struct crsd_matrix_s *crsd_matrix_t;
 typedef struct crsd_comm_s *crsd_comm_t;
@@ -113,8 +124,11 @@ typedef struct {
     int64_t nfills;                 /* filled zeros = nslots - ndiag_nnz */
     int64_t nscatter;               /* scatter entries */
     int64_t nedge_seg;              /* segments run by the guarded (edge) kernel body */
-    int64_t halo_lo, halo_hi;       /* x halo widths (elements) of a row-partitioned handle */
+    int64_t halo_lo, halo_hi;       /* x halo pads (elements) of a row-partitioned handle; halo_lo is a multiple of 4 */
+    int64_t halo_lo_valid, halo_hi_valid; /* halo elements actually exchanged (<= the pads; clipped at the matrix edges) */
     int64_t device_bytes;           /* device memory held by the handle */
+    int32_t variant;                /* kernel variant in use (CRSD_VARIANT_LDG / _TMA) */
+    int32_t smem_bytes;             /* dynamic shared memory per CTA of the TMA variant */
     int64_t unique_bytes_beta0;     /* algorithmic bytes of one SpMV with beta == 0 */
     int64_t unique_bytes_beta1;     /* ... with beta != 0 (y also read) */
 } crsd_info_t;

@@ -27,6 +27,7 @@ STATUS = {
 }
 CRSD_R32F, CRSD_R64F = 0, 1
 CRSD_SUM_DUPLICATES, CRSD_HOST_ONLY, CRSD_DROP_ZEROS = 0x1, 0x2, 0x4
+VARIANT_AUTO, VARIANT_LDG, VARIANT_TMA = 0, 1, 2
 
 # every symbol include/crsd.h declares
 EXPORTED = [
@@ -67,7 +68,7 @@ class Opts(ctypes.Structure):
         ("row_begin", ctypes.c_int64),
         ("row_end", ctypes.c_int64),
         ("nthreads", ctypes.c_int32),
-        ("reserved", ctypes.c_int32),
+        ("variant", ctypes.c_int32),
     ]
 
 
@@ -81,7 +82,9 @@ _INFO_FIELDS = [
     ("nslots", ctypes.c_int64), ("ndiag_nnz", ctypes.c_int64), ("nfills", ctypes.c_int64),
     ("nscatter", ctypes.c_int64), ("nedge_seg", ctypes.c_int64),
     ("halo_lo", ctypes.c_int64), ("halo_hi", ctypes.c_int64),
+    ("halo_lo_valid", ctypes.c_int64), ("halo_hi_valid", ctypes.c_int64),
     ("device_bytes", ctypes.c_int64),
+    ("variant", ctypes.c_int32), ("smem_bytes", ctypes.c_int32),
     ("unique_bytes_beta0", ctypes.c_int64), ("unique_bytes_beta1", ctypes.c_int64),
 ]
 
@@ -195,6 +198,7 @@ class CRSDMatrix:
         row_range: Optional[tuple] = None,
         device: int = -1,
         nthreads: int = 0,
+        variant: int = 0,
     ) -> "CRSDMatrix":
         row = np.ascontiguousarray(row, dtype=np.int64)
         col = np.ascontiguousarray(col, dtype=np.int64)
@@ -210,6 +214,7 @@ class CRSDMatrix:
         o.flags = flags | (CRSD_HOST_ONLY if host_only else 0)
         o.device = device
         o.nthreads = nthreads
+        o.variant = variant
         if row_range is not None:
             o.row_begin, o.row_end = int(row_range[0]), int(row_range[1])
         h = ctypes.c_void_p()

@@ -565,7 +565,8 @@ void make_segdescs(const HostCRSD &H, int rpt, int64_t x_lo, int64_t x_hi, std::
             D.scat_begin = H.scat_ptr[s];
             D.nscat = (int32_t)(H.scat_ptr[s + 1] - H.scat_ptr[s]);
             D.off_begin = (int32_t)H.pat_ptr[I.pattern];
-            D.ndias = (int32_t)nd;
+            D.ndias = (uint16_t)nd;
+            D.plan_begin = 0;
             int64_t lo, hi;
             segment_x_window(H, s, rpt, lo, hi);
             int32_t f = 0;
@@ -580,9 +581,52 @@ void make_segdescs(const HostCRSD &H, int rpt, int64_t x_lo, int64_t x_hi, std::
                 if (c < 0 || c >= H.n_local) bnd = true;
             }
             if (bnd) f |= SEG_BOUNDARY;
-            D.flags = f;
+            D.flags = (uint16_t)f;
         }
     }
+}
+
+int64_t make_plans(const HostCRSD &H, int64_t gap, std::vector<int32_t> &plan, std::vector<SegDesc> &segs) {
+    const int64_t m = H.mrows, es = H.elem, al = 16 / H.elem;  // alignment in elements
+    std::vector<int32_t> begin(H.npat());
+    std::vector<int64_t> smem(H.npat());
+    plan.clear();
+    int64_t mx = 0;
+    for (int64_t p = 0; p < H.npat(); ++p) {
+        const int64_t *o = H.pat_offsets.data() + H.pat_ptr[p];
+        const int64_t nd = H.pat_ptr[p + 1] - H.pat_ptr[p];
+        // clusters of offsets closer than `gap`: one x window each
+        std::vector<std::pair<int64_t, int64_t>> win;  // (start, count) in elements, aligned
+        std::vector<int32_t> xoff(nd);
+        int64_t xbase = 0;
+        for (int64_t d = 0; d < nd;) {
+            int64_t e = d;
+            while (e + 1 < nd && o[e + 1] - o[e] <= gap) ++e;
+            const int64_t st = floordiv(o[d], al) * al;
+            const int64_t en = (floordiv(m - 1 + o[e], al) + 1) * al;
+            for (int64_t q = d; q <= e; ++q) xoff[q] = (int32_t)(xbase + o[q] - st);
+            win.emplace_back(st, en - st);
+            xbase += en - st;
+            d = e + 1;
+        }
+        begin[p] = (int32_t)plan.size();
+        const int64_t bytes = nd * m * es + xbase * es;
+        smem[p] = bytes;
+        mx = std::max(mx, bytes);
+        plan.push_back((int32_t)win.size());
+        plan.push_back((int32_t)std::min<int64_t>(bytes, INT32_MAX));
+        for (auto &w : win) {
+            plan.push_back((int32_t)w.first);
+            plan.push_back((int32_t)w.second);
+        }
+        plan.insert(plan.end(), xoff.begin(), xoff.end());
+    }
+    if (plan.empty()) plan.push_back(0);
+    for (size_t i = 0; i < H.inst.size(); ++i) {
+        const Instance &I = H.inst[i];
+        for (int64_t s = I.first_seg; s < I.first_seg + I.nseg; ++s) segs[s].plan_begin = begin[I.pattern];
+    }
+    return mx;
 }
 
 }  // namespace crsd

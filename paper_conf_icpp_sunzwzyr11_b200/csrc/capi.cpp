@@ -46,12 +46,12 @@ static crsd_status_t dev_alloc_copy(void **dptr, const void *src, size_t bytes, 
 }
 
 void free_device(crsd_matrix_s *A) {
-    void *ptrs[] = {A->d_vals, A->d_segs, A->d_offs, A->d_scat_row, A->d_scat_col, A->d_scat_val,
+    void *ptrs[] = {A->d_vals, A->d_segs, A->d_offs, A->d_plan, A->d_scat_row, A->d_scat_col, A->d_scat_val,
                     A->d_list_interior, A->d_list_boundary, A->d_list_all_edge, A->d_x_scratch, A->d_y_scratch};
     if (A->device >= 0) cudaSetDevice(A->device);
     for (void *p : ptrs)
         if (p) cudaFree(p);
-    A->d_vals = A->d_segs = A->d_offs = A->d_scat_row = A->d_scat_col = A->d_scat_val = nullptr;
+    A->d_vals = A->d_segs = A->d_offs = A->d_plan = A->d_scat_row = A->d_scat_col = A->d_scat_val = nullptr;
     A->d_list_interior = A->d_list_boundary = A->d_list_all_edge = A->d_x_scratch = A->d_y_scratch = nullptr;
 }
 
@@ -74,6 +74,8 @@ static void plan_layout(crsd_matrix_s *A) {
         A->x_hi = H.n_local + A->halo_hi_valid;
     }
     make_segdescs(H, A->rpt, A->x_lo, A->x_hi, A->segdesc);
+    // x windows: offsets closer than 64 elements share one staged window
+    A->smem_bytes = make_plans(H, 64, A->plan, A->segdesc);
     A->list_interior.clear();
     A->list_boundary.clear();
     A->nedge = 0;
@@ -97,6 +99,7 @@ static crsd_status_t upload(crsd_matrix_s *A) {
     std::vector<int32_t> offs32(H.pat_offsets.begin(), H.pat_offsets.end());
     if (offs32.empty()) offs32.push_back(0);
     if ((st = dev_alloc_copy(&A->d_offs, offs32.data(), offs32.size() * 4, cnt))) return st;
+    if ((st = dev_alloc_copy(&A->d_plan, A->plan.data(), A->plan.size() * 4, cnt))) return st;
     const int64_t ns = H.nscatter();
     std::vector<int64_t> colrel(ns);
     for (int64_t e = 0; e < ns; ++e) colrel[e] = H.scat_col[e] - H.row_begin;
@@ -114,8 +117,28 @@ static crsd_status_t upload(crsd_matrix_s *A) {
 
 static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_matrix_t *out) {
     A->rpt = (A->H.dtype == CRSD_R64F) ? 2 : 4;
+    int64_t maxnd = 0;
+    for (int64_t p = 0; p < A->H.npat(); ++p) maxnd = std::max<int64_t>(maxnd, A->H.ndias((int32_t)p));
+    if (maxnd > MAX_NDIAS) {
+        delete A;
+        return fail(CRSD_ERR_UNSUPPORTED, "a pattern has more than " + std::to_string(MAX_NDIAS) + " diagonals");
+    }
     plan_layout(A);
+    const int64_t smem_cap = 200 * 1024;
+    if (o.variant == CRSD_VARIANT_TMA && A->smem_bytes > smem_cap) {
+        const std::string msg = "TMA variant: staging needs " + std::to_string(A->smem_bytes) +
+                                " bytes of shared memory per CTA (> 200 KB); use CRSD_VARIANT_LDG";
+        delete A;
+        return fail(CRSD_ERR_UNSUPPORTED, msg);
+    }
+    if (o.variant == CRSD_VARIANT_LDG) A->variant = VARIANT_LDG;
+    else if (o.variant == CRSD_VARIANT_TMA) A->variant = VARIANT_TMA;
+    else A->variant = (A->smem_bytes <= smem_cap) ? VARIANT_TMA : VARIANT_LDG;
     if (!A->host_only) {
+        if (A->H.mrows / A->rpt > 256) {
+            delete A;
+            return fail(CRSD_ERR_UNSUPPORTED, "GPU path needs mrows / RPT <= 256 threads per CTA (mrows <= 512 fp64, 1024 fp32)");
+        }
         if (A->H.mrows % (32 * A->rpt) != 0) {
             delete A;
             return fail(CRSD_ERR_UNSUPPORTED, "GPU path needs mrows % (32*RPT) == 0 (RPT = 2 fp64, 4 fp32); got mrows=" +
@@ -157,6 +180,9 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
     a.vals = (const T *)A->d_vals;
     a.segs = (const SegDesc *)A->d_segs;
     a.pat_offs = (const int32_t *)A->d_offs;
+    a.plan = (const int32_t *)A->d_plan;
+    a.smem_bytes = (int32_t)A->smem_bytes;
+    a.variant = A->variant;
     a.scat_row = (const int32_t *)A->d_scat_row;
     a.scat_col = (const int64_t *)A->d_scat_col;
     a.scat_val = (const T *)A->d_scat_val;
@@ -172,7 +198,7 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
     a.alpha = alpha;
     a.beta = beta;
     int n = launch_spmv<T>(a, A->sm_count, stream);
-    if (n < 0) return fail(CRSD_ERR_CUDA, std::string("kernel launch: ") + cudaGetErrorString(cudaGetLastError()));
+    if (n < 0) return fail(CRSD_ERR_CUDA, std::string("kernel launch: ") + cudaGetErrorString((cudaError_t)(-n)));
     launches += n;
     return CRSD_OK;
 }
@@ -325,7 +351,11 @@ crsd_status_t crsd_get_info(crsd_matrix_t A, crsd_info_t *I) {
     I->nedge_seg = A->nedge;
     I->halo_lo = A->halo_lo;
     I->halo_hi = A->halo_hi;
+    I->halo_lo_valid = A->halo_lo_valid;
+    I->halo_hi_valid = A->halo_hi_valid;
     I->device_bytes = A->device_bytes;
+    I->variant = A->variant;
+    I->smem_bytes = (int32_t)A->smem_bytes;
     // algorithmic bytes: stored slots + scatter
     // (value + row + col) + x once + y written (+ y read when beta != 0)
     const int64_t es = H.elem;

@@ -13,6 +13,9 @@ struct crsd_matrix_s {
     int device = -1;
     int sm_count = 148;
     int rpt = 2;
+    int variant = crsd::VARIANT_LDG;
+    int64_t smem_bytes = 0;
+    std::vector<int32_t> plan;
     int32_t last_launches = 0;
     int64_t device_bytes = 0;
 
@@ -29,6 +32,7 @@ struct crsd_matrix_s {
     void *d_vals = nullptr;
     void *d_segs = nullptr;
     void *d_offs = nullptr;
+    void *d_plan = nullptr;
     void *d_scat_row = nullptr;
     void *d_scat_col = nullptr;
     void *d_scat_val = nullptr;

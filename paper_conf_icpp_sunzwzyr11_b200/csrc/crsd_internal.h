@@ -35,9 +35,22 @@ struct alignas(16) SegDesc {
     int64_t scat_begin;  // first scatter entry of the segment
     int32_t off_begin;   // first offset of the segment's pattern in pat_offs
     int32_t nscat;       // scatter entries
-    int32_t flags;       // SEG_*
-    int32_t ndias;       // NDias of the pattern
+    uint16_t flags;      // SEG_*
+    uint16_t ndias;      // NDias of the pattern (<= MAX_NDIAS)
+    int32_t plan_begin;  // TMA staging plan of the pattern in `plan`
 };
+constexpr int MAX_NDIAS = 4096;
+
+// Kernel variants
+enum : int32_t { VARIANT_AUTO = 0, VARIANT_LDG = 1, VARIANT_TMA = 2 };
+
+// TMA staging plan of one distinct pattern (int32 words at plan_begin):
+//   [0] nwin  [1] smem bytes (values + windows)
+//   then nwin x (start, count): x window [row0 + start, row0 + start + count)
+//        (start, count multiples of 16/sizeof(T) elements)
+//   then ndias x xoff: element offset in the smem x region of row 0's x for
+//        diagonal d (= window base + o_d - start)
+
 static_assert(sizeof(SegDesc) == 32, "SegDesc must be 32 bytes");
 
 struct HostCRSD {
@@ -94,6 +107,10 @@ void segment_x_window(const HostCRSD &H, int64_t s, int rpt, int64_t &lo, int64_
 // local x base; own_hi: n_local (the x the rank owns is [0, own_hi)).
 void make_segdescs(const HostCRSD &H, int rpt, int64_t x_lo, int64_t x_hi, std::vector<SegDesc> &out);
 
+// TMA staging plans of all distinct patterns (x windows = clusters of offsets
+// closer than `gap` elements); fills SegDesc::plan_begin; returns max smem.
+int64_t make_plans(const HostCRSD &H, int64_t gap, std::vector<int32_t> &plan, std::vector<SegDesc> &segs);
+
 // Halo extents (elements outside [0, n_local) relative to the local x base)
 // the handle needs: from its non-edge windows and its scatter columns.
 void needed_halo(const HostCRSD &H, int rpt, int64_t &need_lo, int64_t &need_hi);
@@ -106,6 +123,7 @@ struct SpmvArgs {
     const T *vals;
     const SegDesc *segs;
     const int32_t *pat_offs;
+    const int32_t *plan;
     const int32_t *scat_row;
     const int64_t *scat_col;  // relative to x base
     const T *scat_val;
@@ -116,6 +134,8 @@ struct SpmvArgs {
     const int32_t *seg_list;  // if non-null: CTA work = seg_list[i]
     int64_t seg_begin, seg_count;
     int32_t mrows;
+    int32_t smem_bytes;       // TMA variant: dynamic shared memory per CTA
+    int32_t variant;          // VARIANT_LDG or VARIANT_TMA
     T alpha, beta;
 };
 

@@ -113,7 +113,7 @@ __device__ __forceinline__ double2 make_vec(const double (&v)[2]) { return make_
 __device__ __forceinline__ float4 make_vec(const float (&v)[4]) { return make_float4(v[0], v[1], v[2], v[3]); }
 
 template <typename T, int CH>
-__global__ void __launch_bounds__(256) crsd_spmv_kernel(const SpmvArgs<T> a) {
+__global__ void __launch_bounds__(256, sizeof(T) == 8 ? 3 : 4) crsd_spmv_ldg(const SpmvArgs<T> a) {
     using V = typename VecT<T>::type;
     constexpr int R = VecT<T>::R;
     constexpr int LOG = VecT<T>::LOG;
@@ -242,6 +242,142 @@ __global__ void __launch_bounds__(256) crsd_spmv_kernel(const SpmvArgs<T> a) {
     }
 }
 
+// ---------------------------------------------------------------------------
+// TMA-staged variant. One elected thread issues bulk copies
+// (cp.async.bulk, Blackwell/Hopper TMA engine) of the segment's contiguous
+// value block and of the pattern's x windows (clusters of nearby offsets =
+// the paper's adjacent groups) into shared memory, completing on
+// one mbarrier; all threads then compute from shared memory. Memory-level
+// parallelism no longer depends on registers: a CTA has its whole segment in
+// flight (values + x), several CTAs per SM. Thread t owns rows t + q*T
+// (T = threads, q < RPT) so shared-memory reads are bank-conflict free.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_fence_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t phase) {
+    uint32_t done = 0;
+    const uint32_t a = smem_u32(bar);
+    while (!done) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(done)
+            : "r"(a), "r"(phase)
+            : "memory");
+    }
+}
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar, uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
+            smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
+        : "memory");
+}
+__device__ __forceinline__ uint64_t policy_evict_normal() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+
+template <typename T>
+__global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a) {
+    constexpr int R = VecT<T>::R;
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ uint64_t bar;
+    const int t = threadIdx.x;
+    const int T_ = blockDim.x;
+    const int64_t s = a.seg_list ? (int64_t)__ldg(a.seg_list + blockIdx.x) : a.seg_begin + blockIdx.x;
+    const SegDesc D = a.segs[s];
+    const int64_t row0 = s * a.mrows;
+    const int nd = D.ndias;
+    const int32_t *plan = a.plan + D.plan_begin;
+    const int nwin = __ldg(plan);
+    const bool edge = (D.flags & SEG_EDGE) != 0;
+    T *vs = reinterpret_cast<T *>(smem);
+    T *xs = vs + (int64_t)nd * a.mrows;
+    const uint32_t vbytes = (uint32_t)nd * (uint32_t)a.mrows * sizeof(T);
+    if (t == 0) {
+        mbar_init(&bar, 1);
+        mbar_fence_init();
+    }
+    __syncthreads();
+    if (t == 0) {
+        uint32_t total = vbytes;
+        if (!edge)
+            for (int w = 0; w < nwin; ++w) total += (uint32_t)__ldg(plan + 3 + 2 * w) * sizeof(T);
+        mbar_expect_tx(&bar, total);
+        if (vbytes) bulk_g2s(vs, a.vals + D.val_base, vbytes, &bar, policy_evict_first());
+        if (!edge) {
+            const uint64_t pn = policy_evict_normal();
+            T *dst = xs;
+            for (int w = 0; w < nwin; ++w) {
+                const int st = __ldg(plan + 2 + 2 * w), cnt = __ldg(plan + 3 + 2 * w);
+                bulk_g2s(dst, a.x + row0 + st, (uint32_t)cnt * sizeof(T), &bar, pn);
+                dst += cnt;
+            }
+        }
+    }
+    T acc[R];
+#pragma unroll
+    for (int q = 0; q < R; ++q) acc[q] = T(0);
+    const int32_t *xoff = plan + 2 + 2 * nwin;
+    const int32_t *offs = a.pat_offs + D.off_begin;
+    mbar_wait(&bar, 0);
+    if (!edge) {
+#pragma unroll 4
+        for (int d = 0; d < nd; ++d) {
+            const int xo = __ldg(xoff + d);
+            const T *vd = vs + d * a.mrows + t;
+            const T *xd = xs + xo + t;
+#pragma unroll
+            for (int q = 0; q < R; ++q) acc[q] = fma(vd[q * T_], xd[q * T_], acc[q]);
+        }
+    } else {
+        for (int d = 0; d < nd; ++d) {
+            const int o = __ldg(offs + d);
+            const T *vd = vs + d * a.mrows + t;
+#pragma unroll
+            for (int q = 0; q < R; ++q) {
+                const int64_t idx = row0 + t + q * T_ + o;
+                const T xj = (idx >= a.x_lo && idx < a.x_hi) ? __ldg(a.x + idx) : T(0);
+                acc[q] = fma(vd[q * T_], xj, acc[q]);
+            }
+        }
+    }
+    // scatter points: owner of local row l is thread l % T, slot l / T
+    if (D.nscat > 0) {
+        const int32_t *sr = a.scat_row + D.scat_begin;
+        for (int64_t e = 0; e < D.nscat; ++e) {
+            const int rr = __ldg(sr + e);
+            if (rr % T_ != t) continue;
+            const T v = __ldg(a.scat_val + D.scat_begin + e);
+            const T xv = __ldg(a.x + __ldg(a.scat_col + D.scat_begin + e));
+            const int q = rr / T_;
+#pragma unroll
+            for (int j = 0; j < R; ++j)
+                if (q == j) acc[j] = fma(v, xv, acc[j]);
+        }
+    }
+    const T al = a.alpha, be = a.beta;
+#pragma unroll
+    for (int q = 0; q < R; ++q) {
+        const int64_t r = row0 + t + q * T_;
+        if (!edge || r < a.nrows) {
+            T *yp = a.y + r;
+            const T out = (be != T(0)) ? fma(al, acc[q], be * *yp) : al * acc[q];
+            __stcs(yp, out);
+        }
+    }
+}
+
 template <typename T>
 int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
     if (a.seg_count <= 0) return 0;
@@ -250,8 +386,22 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
     int64_t grid = a.seg_count;
     if (grid > 0x7fffffff) grid = 0x7fffffff;
     (void)sm_count;
-    crsd_spmv_kernel<T, 4><<<(unsigned)grid, threads, 0, (cudaStream_t)stream>>>(a);
-    return cudaGetLastError() == cudaSuccess ? 1 : -1;
+    cudaError_t e;
+    if (a.variant == VARIANT_TMA) {
+        static bool attr_done[2] = {false, false};
+        auto kern = crsd_spmv_tma<T>;
+        bool &done = attr_done[sizeof(T) == 8];
+        if (!done || a.smem_bytes > 48 * 1024) {
+            e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+            if (e != cudaSuccess) return -(int)e;
+            done = true;
+        }
+        kern<<<(unsigned)grid, threads, a.smem_bytes, (cudaStream_t)stream>>>(a);
+    } else {
+        crsd_spmv_ldg<T, 4><<<(unsigned)grid, threads, 0, (cudaStream_t)stream>>>(a);
+    }
+    e = cudaGetLastError();
+    return e == cudaSuccess ? 1 : -(int)e;
 }
 
 template int launch_spmv<double>(const SpmvArgs<double> &, int, void *);

@@ -1,0 +1,86 @@
+#!/usr/bin/env python
+"""Summarise an ncu --set full report (.ncu-rep) into the metrics DESIGN.md cites.
+
+usage: python scripts/ncu_summary.py gpurun_out/prof_x.ncu-rep [--bytes ALGO_BYTES] > profiles/...
+"""
+import csv
+import io
+import json
+import subprocess
+import sys
+
+KEYS = [
+    "gpu__time_duration.sum",
+    "dram__bytes_read.sum",
+    "dram__bytes_write.sum",
+    "dram__throughput.avg.pct_of_peak_sustained_elapsed",
+    "gpu__compute_memory_throughput.avg.pct_of_peak_sustained_elapsed",
+    "lts__t_sector_hit_rate.pct",
+    "lts__throughput.avg.pct_of_peak_sustained_elapsed",
+    "l1tex__throughput.avg.pct_of_peak_sustained_active",
+    "l1tex__t_sector_hit_rate.pct",
+    "sm__throughput.avg.pct_of_peak_sustained_elapsed",
+    "sm__warps_active.avg.pct_of_peak_sustained_active",
+    "sm__maximum_warps_per_active_cycle_pct",
+    "launch__registers_per_thread",
+    "launch__shared_mem_per_block_dynamic",
+    "launch__occupancy_limit_registers",
+    "launch__occupancy_limit_shared_mem",
+    "launch__grid_size",
+    "launch__block_size",
+    "smsp__sass_inst_executed_op_global_ld.sum",
+    "smsp__sass_inst_executed_op_shared_ld.sum",
+    "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum",
+    "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum",
+    "smsp__average_warp_latency_issue_stalled_long_scoreboard",
+    "smsp__warp_issue_stalled_long_scoreboard_per_warp_active.pct",
+    "smsp__warp_issue_stalled_barrier_per_warp_active.pct",
+    "smsp__warp_issue_stalled_membar_per_warp_active.pct",
+    "smsp__warp_issue_stalled_lg_throttle_per_warp_active.pct",
+    "smsp__warp_issue_stalled_short_scoreboard_per_warp_active.pct",
+    "smsp__warp_issue_stalled_wait_per_warp_active.pct",
+    "smsp__warp_issue_stalled_no_instruction_per_warp_active.pct",
+    "smsp__cycles_active.avg",
+    "sm__cycles_elapsed.avg.per_second",
+    "dram__cycles_elapsed.avg.per_second",
+]
+
+
+def main():
+    rep = sys.argv[1]
+    algo = None
+    if "--bytes" in sys.argv:
+        algo = float(sys.argv[sys.argv.index("--bytes") + 1])
+    out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(io.StringIO(out)))
+    hdr, units = rows[0], rows[1]
+    res = []
+    for r in rows[2:]:
+        d = {"kernel": r[hdr.index("Kernel Name")]}
+        for k in KEYS:
+            if k in hdr:
+                i = hdr.index(k)
+                d[k] = {"value": r[i], "unit": units[i]}
+        # normalise bytes
+        def tob(x):
+            v = float(x["value"].replace(",", ""))
+            u = x["unit"]
+            return v * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(u, 1)
+
+        if "dram__bytes_read.sum" in d:
+            rb, wb = tob(d["dram__bytes_read.sum"]), tob(d["dram__bytes_write.sum"])
+            t = float(d["gpu__time_duration.sum"]["value"].replace(",", ""))
+            tu = d["gpu__time_duration.sum"]["unit"]
+            ts = t * {"ns": 1e-9, "us": 1e-6, "usecond": 1e-6, "ms": 1e-3, "msecond": 1e-3}.get(tu, 1e-9)
+            d["derived"] = {"dram_bytes": rb + wb, "dram_GBps": (rb + wb) / ts / 1e9, "duration_s": ts}
+            if algo:
+                d["derived"]["algorithmic_bytes"] = algo
+                d["derived"]["traffic_over_algorithmic"] = (rb + wb) / algo
+                d["derived"]["algorithmic_GBps"] = algo / ts / 1e9
+        res.append(d)
+    json.dump(res, sys.stdout, indent=1)
+    print()
+
+
+if __name__ == "__main__":
+    main()

@@ -20,6 +20,7 @@ from tests.conftest import have_gpu
 pytestmark = pytest.mark.gpu
 
 TOL = {np.float64: 1e-12, np.float32: 1e-5}
+VARIANTS = [1, 2]  # CRSD_VARIANT_LDG, CRSD_VARIANT_TMA
 
 _CACHE = {}
 
@@ -72,46 +73,54 @@ def _parity(torch, a, dt, alpha=1.0, beta=0.0, seed=0, **kw):
     return A, err
 
 
+@pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
 @pytest.mark.parametrize("alpha,beta", [(1.0, 0.0), (-0.75, 0.0), (1.0, 1.0), (-0.75, 0.5)])
-def test_c1_parity(torch_cuda, dt, alpha, beta):
-    _parity(torch_cuda, gen.config1(), dt, alpha, beta)
+def test_c1_parity(torch_cuda, dt, alpha, beta, variant):
+    A, _ = _parity(torch_cuda, gen.config1(), dt, alpha, beta, variant=variant)
+    assert A.info()["variant"] == variant
 
 
+@pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
-def test_c2_reduced_parity(torch_cuda, dt):
-    _parity(torch_cuda, gen.config2(n=40), dt, -0.75, 0.5)
+def test_c2_reduced_parity(torch_cuda, dt, variant):
+    _parity(torch_cuda, gen.config2(n=40), dt, -0.75, 0.5, variant=variant)
 
 
+@pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
-def test_c3_reduced_parity(torch_cuda, dt):
-    A, _ = _parity(torch_cuda, gen.config3(n=36), dt, 1.0, 0.0)
+def test_c3_reduced_parity(torch_cuda, dt, variant):
+    A, _ = _parity(torch_cuda, gen.config3(n=36), dt, 1.0, 0.0, variant=variant)
     assert A.info()["nscatter"] > 0
 
 
-def test_c4_reduced_parity(torch_cuda):
-    _parity(torch_cuda, gen.config4(n=300_000), np.float32, 1.0, 0.0)
+@pytest.mark.parametrize("variant", VARIANTS)
+def test_c4_reduced_parity(torch_cuda, variant):
+    _parity(torch_cuda, gen.config4(n=300_000), np.float32, 1.0, 0.0, variant=variant)
 
 
+@pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("seed", range(12))
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
-def test_random_diagonal_parity(torch_cuda, seed, dt):
+def test_random_diagonal_parity(torch_cuda, seed, dt, variant):
     """Random offsets (AD runs), breaks, scatter, rectangular shapes, ragged tails."""
     rng = np.random.default_rng(seed)
     n = int(rng.integers(1, 5000))
     m = int(rng.integers(1, 5000))
     a = gen.random_diagonal(n, m, seed, ndiag=int(rng.integers(1, 30)), max_off=int(rng.integers(1, 3000)), p_break=0.02, max_break=400, n_scatter=int(rng.integers(0, 300)))
-    mrows = [256, 512, 1024][seed % 3] if dt == np.float64 else [128, 512, 1024][seed % 3]
-    _parity(torch_cuda, a, dt, [1.0, -0.75][seed % 2], [0.0, 0.5][(seed // 2) % 2], seed=seed, mrows=mrows)
+    mrows = [64, 256, 512][seed % 3] if dt == np.float64 else [128, 512, 1024][seed % 3]
+    _parity(torch_cuda, a, dt, [1.0, -0.75][seed % 2], [0.0, 0.5][(seed // 2) % 2], seed=seed, mrows=mrows, variant=variant)
 
 
+@pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
-def test_dense_scatter_segments(torch_cuda, dt):
+def test_dense_scatter_segments(torch_cuda, dt, variant):
     """Segments with hundreds of scatter points (binary-search path of the scatter pass)."""
     n = 2048
     a = gen.random_diagonal(n, n, 5, ndiag=3, n_scatter=3000)
-    A, _ = _parity(torch_cuda, a, dt, 1.0, 0.0)
-    assert A.info()["nscatter"] > 2000
+    A, _ = _parity(torch_cuda, a, dt, 1.0, 0.0, variant=variant)
+    P = A.export()
+    assert A.info()["nscatter"] > 1000 and np.max(np.diff(P["scat_ptr"])) > 32
 
 
 def test_beta_zero_never_reads_y(torch_cuda):
@@ -157,13 +166,14 @@ def test_spmv_host_e2e(torch_cuda, dt):
 
 
 # ---------------------------------------------------------------- full sizes
+@pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
 @pytest.mark.parametrize("xkind", ["linear", "quadratic"])
-def test_c2_full_closed_form(torch_cuda, dt, xkind):
+def test_c2_full_closed_form(torch_cuda, dt, xkind, variant):
     """BASELINE config 2 at full size (256^3), every row vs the closed form (exact)."""
     dims = (256, 256, 256)
     a = cached("c2x", gen.config2, values="exact").astype(dt)
-    A = _mat(a)
+    A = _mat(a, variant=variant)
     x = gen.vectors(a.ncols, xkind, dims=dims).astype(dt)
     y = _run(torch_cuda, A, x, 1.0, 0.0, None, a.nrows)
     assert np.array_equal(y.astype(np.float64), closed_forms.stencil_apply(dims, "7pt", xkind))
@@ -174,10 +184,11 @@ def test_c2_full_random_parity(torch_cuda):
     _parity(torch_cuda, cached("c2", gen.config2), np.float64, -0.75, 0.5)
 
 
+@pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
-def test_c3_full_parity(torch_cuda, dt):
+def test_c3_full_parity(torch_cuda, dt, variant):
     """Config 3 at full size (192^3 27-pt, idle blocks, 0.1% scatter), every row."""
-    A, _ = _parity(torch_cuda, cached("c3", gen.config3), dt, 1.0, 0.0)
+    A, _ = _parity(torch_cuda, cached("c3", gen.config3), dt, 1.0, 0.0, variant=variant)
     inf = A.info()
     assert inf["nscatter"] > 100_000
 
@@ -194,3 +205,44 @@ def test_c3_full_closed_form_ones(torch_cuda):
     yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, np.ones(a.ncols))
     assert coo.parity_error(y, yref, scale) <= 1e-12
     assert np.max(np.abs(yref - expect)) <= 1e-12
+
+
+# ---------------------------------------------------------------- row-partitioned compute
+@pytest.mark.parametrize("variant", VARIANTS)
+@pytest.mark.parametrize("case", ["c2", "c3", "c4"])
+@pytest.mark.parametrize("world", [2, 3])
+def test_dist_compute_single_gpu(torch_cuda, case, world, variant):
+    """crsd_spmv_dist with comm=NULL: P logical ranks on one GPU, halos filled
+    from the global x on the host; interior + boundary lists must reproduce
+    the global product rows of each rank."""
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, partition_rows
+
+    torch = torch_cuda
+    if case == "c2":
+        a, dt, mrows = gen.config2(n=40), np.float64, 256
+    elif case == "c3":
+        a, dt, mrows = gen.config3(n=36), np.float64, 256
+    else:
+        a, dt, mrows = gen.config4(n=300_000), np.float32, 512
+    a = a.astype(dt)
+    n = a.nrows
+    x = np.random.default_rng(2).uniform(-1, 1, n).astype(dt)
+    yref, scale = coo.coo_spmv(n, n, a.row, a.col, a.val, x)
+    bounds = partition_rows(n, mrows, world, np.bincount(a.row, minlength=n).astype(np.float64))
+    tdt = torch.float64 if dt == np.float64 else torch.float32
+    for r in range(world):
+        rb, re = int(bounds[r]), int(bounds[r + 1])
+        m = (a.row >= rb) & (a.row < re)
+        A = CRSDMatrix.from_coo(n, n, a.row[m], a.col[m], a.val[m], mrows=mrows, row_range=(rb, re), variant=variant)
+        inf = A.info()
+        lo, nloc, hi = A.x_layout()
+        xp = np.zeros(lo + nloc + hi, dt)
+        hlv, hhv = inf["halo_lo_valid"], inf["halo_hi_valid"]
+        xp[lo - hlv : lo + nloc + hhv] = x[rb - hlv : re + hhv]
+        xd = torch.from_numpy(xp).to("cuda", tdt)
+        yd = torch.full((nloc,), float("nan"), device="cuda", dtype=tdt)
+        A.spmv_dist(xd, yd, 1.0, 0.0, None)
+        torch.cuda.synchronize()
+        err = coo.parity_error(yd.cpu().numpy(), yref[rb:re], scale[rb:re])
+        assert err <= TOL[dt], (r, err)
+        assert A.last_launch_count() in (1, 2)
