@@ -140,6 +140,26 @@ class ClockSampler:
         }
 
 
+def copy_bandwidth(dev, reps=5):
+    """Same recipe as MEASURED_PEAKS.json: torch copy of 1 Gi bf16 elements,
+    read+write bytes, best of `reps` (context for this box's HBM)."""
+    import torch
+
+    a = torch.empty(1 << 30, dtype=torch.bfloat16, device=f"cuda:{dev}")
+    b = torch.empty_like(a)
+    best = 0.0
+    for _ in range(reps + 1):
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s.record()
+        b.copy_(a)
+        e.record()
+        e.synchronize()
+        best = max(best, 2 * a.numel() * 2 / (s.elapsed_time(e) * 1e-3) / 1e9)
+    del a, b
+    torch.cuda.empty_cache()
+    return round(best, 1)
+
+
 def load_traffic(cfg, dtype):
     p = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(p):
@@ -361,6 +381,7 @@ def run_crsd(args):
         return
 
     cpu = None if (world > 1 or args.no_cpu) else cpu_baseline(a)
+    box_copy = copy_bandwidth(dev)
     traffic = load_traffic(args.config, args.dtype)
     line = {
         "metric": "CRSD SpMV GFLOP/s (2*nnz/t) with achieved HBM GB/s (% of B200 peak)",
@@ -402,6 +423,8 @@ def run_crsd(args):
             "traffic": traffic,
             "algorithmic_bytes_per_launch": int(ub),
             "avg_launch_ms": round(kern_ms, 5),
+            "copy_gbs_this_box": box_copy,
+            "frac_of_this_box_copy": round(achieved / box_copy, 4) if box_copy else None,
         },
         "cpu_baseline": cpu,
         "e2e": e2e,

@@ -46,6 +46,18 @@ static crsd_status_t dev_alloc_copy(void **dptr, const void *src, size_t bytes, 
 }
 
 void free_device(crsd_matrix_s *A) {
+    if (A->e2e_ready) {
+        if (A->device >= 0) cudaSetDevice(A->device);
+        cudaStreamSynchronize((cudaStream_t)A->e2e_h2d);
+        cudaStreamSynchronize((cudaStream_t)A->e2e_d2h);
+        for (void *e : A->e2e_ev_x) cudaEventDestroy((cudaEvent_t)e);
+        for (void *e : A->e2e_ev_y) cudaEventDestroy((cudaEvent_t)e);
+        cudaEventDestroy((cudaEvent_t)A->e2e_ev_start);
+        cudaEventDestroy((cudaEvent_t)A->e2e_ev_done);
+        cudaStreamDestroy((cudaStream_t)A->e2e_h2d);
+        cudaStreamDestroy((cudaStream_t)A->e2e_d2h);
+        A->e2e_ready = false;
+    }
     void *ptrs[] = {A->d_vals, A->d_segs, A->d_offs, A->d_plan, A->d_scat_row, A->d_scat_col, A->d_scat_val,
                     A->d_list_interior, A->d_list_boundary, A->d_list_all_edge, A->d_x_scratch, A->d_y_scratch};
     if (A->device >= 0) cudaSetDevice(A->device);
@@ -174,7 +186,7 @@ static crsd_status_t resolve_opts(int64_t nrows, crsd_dtype_t dtype, const crsd_
 
 template <typename T>
 static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *y, const int32_t *list,
-                              int64_t count, void *stream, int &launches) {
+                              int64_t seg_begin, int64_t count, void *stream, int &launches) {
     if (count <= 0) return CRSD_OK;
     SpmvArgs<T> a;
     a.vals = (const T *)A->d_vals;
@@ -192,7 +204,7 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
     a.y = y;
     a.nrows = A->H.n_local;
     a.seg_list = list;
-    a.seg_begin = 0;
+    a.seg_begin = seg_begin;
     a.seg_count = count;
     a.mrows = A->H.mrows;
     a.alpha = alpha;
@@ -204,12 +216,12 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
 }
 
 crsd_status_t run_lists(crsd_matrix_s *A, const void *alpha, const void *x_base, const void *beta, void *y,
-                        const int32_t *list, int64_t count, void *stream, int &launches) {
+                        const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches) {
     if (A->H.dtype == CRSD_R64F)
         return run_spmv<double>(A, *(const double *)alpha, (const double *)x_base, *(const double *)beta, (double *)y,
-                                list, count, stream, launches);
+                                list, seg_begin, count, stream, launches);
     return run_spmv<float>(A, *(const float *)alpha, (const float *)x_base, *(const float *)beta, (float *)y, list,
-                           count, stream, launches);
+                           seg_begin, count, stream, launches);
 }
 
 }  // namespace crsd
@@ -293,9 +305,65 @@ crsd_status_t crsd_spmv(crsd_matrix_t A, const void *alpha, const void *x, const
     int launches = 0;
     cudaSetDevice(A->device);
     const int64_t nseg = A->H.nseg;
-    st = run_lists(A, alpha, x, beta, y, nullptr, nseg, stream, launches);
+    st = run_lists(A, alpha, x, beta, y, nullptr, 0, nseg, stream, launches);
     A->last_launches = launches;
     return st;
+}
+
+// End-to-end SpMV with host vectors, pipelined: x is copied in row-aligned
+// chunks on an H2D stream, each row chunk of segments runs as soon as the x
+// chunks its windows reach have landed, and its y chunk is copied back on a
+// D2H stream while later chunks compute (PCIe is full duplex). This answers
+// the paper's transfer caveat by overlapping transfers with
+// the SpMV instead of serialising copy -> kernel -> copy.
+static crsd_status_t e2e_setup(crsd_matrix_s *A) {
+    HostCRSD &H = A->H;
+    const int64_t nseg = H.nseg;
+    int nch = (int)std::min<int64_t>(16, std::max<int64_t>(1, nseg / 64));
+    A->e2e_nchunk = nch;
+    A->e2e_seg.resize(nch + 1);
+    A->e2e_xcut.resize(nch + 1);
+    for (int c = 0; c <= nch; ++c) A->e2e_seg[c] = nseg * c / nch;
+    for (int c = 0; c <= nch; ++c) {
+        int64_t xc = (c == nch) ? H.ncols : std::min<int64_t>(H.ncols, A->e2e_seg[c] * H.mrows);
+        A->e2e_xcut[c] = (c == nch) ? xc : (xc / 4) * 4;
+    }
+    // highest x element each row chunk reads (vector windows, clipped to
+    // [0, ncols) as the guarded edge path does, and scatter columns)
+    A->e2e_need.assign(nch, 0);
+    for (int c = 0; c < nch; ++c) {
+        int64_t hi = 0;
+        for (int64_t sg = A->e2e_seg[c]; sg < A->e2e_seg[c + 1]; ++sg) {
+            int64_t lo_w, hi_w;
+            segment_x_window(H, sg, A->rpt, lo_w, hi_w);
+            if (lo_w < hi_w) hi = std::max(hi, std::min(hi_w, H.ncols));
+            for (int64_t e = H.scat_ptr[sg]; e < H.scat_ptr[sg + 1]; ++e) hi = std::max(hi, H.scat_col[e] + 1);
+        }
+        int j = 0;
+        while (j < nch - 1 && A->e2e_xcut[j + 1] < hi) ++j;
+        A->e2e_need[c] = std::max(j, c * 0);
+    }
+    cudaStream_t h, d;
+    CUDA_TRY(cudaStreamCreateWithFlags(&h, cudaStreamNonBlocking));
+    CUDA_TRY(cudaStreamCreateWithFlags(&d, cudaStreamNonBlocking));
+    A->e2e_h2d = h;
+    A->e2e_d2h = d;
+    A->e2e_ev_x.resize(nch);
+    A->e2e_ev_y.resize(nch);
+    for (int c = 0; c < nch; ++c) {
+        cudaEvent_t e1, e2;
+        CUDA_TRY(cudaEventCreateWithFlags(&e1, cudaEventDisableTiming));
+        CUDA_TRY(cudaEventCreateWithFlags(&e2, cudaEventDisableTiming));
+        A->e2e_ev_x[c] = e1;
+        A->e2e_ev_y[c] = e2;
+    }
+    cudaEvent_t e0, e3;
+    CUDA_TRY(cudaEventCreateWithFlags(&e0, cudaEventDisableTiming));
+    CUDA_TRY(cudaEventCreateWithFlags(&e3, cudaEventDisableTiming));
+    A->e2e_ev_start = e0;
+    A->e2e_ev_done = e3;
+    A->e2e_ready = true;
+    return CRSD_OK;
 }
 
 crsd_status_t crsd_spmv_host(crsd_matrix_t A, const void *alpha, const void *x_host, const void *beta, void *y_host,
@@ -304,7 +372,7 @@ crsd_status_t crsd_spmv_host(crsd_matrix_t A, const void *alpha, const void *x_h
     if (A->host_only) return fail(CRSD_ERR_UNSUPPORTED, "host-only handle");
     if (A->H.partitioned) return fail(CRSD_ERR_UNSUPPORTED, "row-partitioned handle");
     if (!x_host || !y_host || !alpha || !beta) return fail(CRSD_ERR_INVALID_ARG, "NULL argument");
-    cudaSetDevice(A->device);
+    CUDA_TRY(cudaSetDevice(A->device));
     const size_t es = A->H.elem;
     const size_t xb = A->H.ncols * es, yb = A->H.nrows * es;
     int64_t dummy = 0;
@@ -314,12 +382,49 @@ crsd_status_t crsd_spmv_host(crsd_matrix_t A, const void *alpha, const void *x_h
         if ((st = dev_alloc_copy(&A->d_y_scratch, nullptr, yb, dummy))) return st;
         A->device_bytes += dummy;
     }
-    cudaStream_t s = (cudaStream_t)stream;
+    if (!A->e2e_ready && (st = e2e_setup(A))) return st;
+    cudaStream_t s = (cudaStream_t)stream, h = (cudaStream_t)A->e2e_h2d, d = (cudaStream_t)A->e2e_d2h;
     const bool beta_nz = (A->H.dtype == CRSD_R64F) ? (*(const double *)beta != 0.0) : (*(const float *)beta != 0.0f);
-    CUDA_TRY(cudaMemcpyAsync(A->d_x_scratch, x_host, xb, cudaMemcpyHostToDevice, s));
-    if (beta_nz) CUDA_TRY(cudaMemcpyAsync(A->d_y_scratch, y_host, yb, cudaMemcpyHostToDevice, s));
-    if ((st = crsd_spmv(A, alpha, A->d_x_scratch, beta, A->d_y_scratch, stream))) return st;
-    CUDA_TRY(cudaMemcpyAsync(y_host, A->d_y_scratch, yb, cudaMemcpyDeviceToHost, s));
+    const int nch = A->e2e_nchunk;
+    const int64_t m = A->H.mrows;
+    char *dx = (char *)A->d_x_scratch, *dy = (char *)A->d_y_scratch;
+    const char *hx = (const char *)x_host;
+    char *hy = (char *)y_host;
+    auto yrange = [&](int c, int64_t &r0, int64_t &r1) {
+        r0 = A->e2e_seg[c] * m;
+        r1 = std::min<int64_t>(A->H.nrows, A->e2e_seg[c + 1] * m);
+    };
+    CUDA_TRY(cudaEventRecord((cudaEvent_t)A->e2e_ev_start, s));
+    CUDA_TRY(cudaStreamWaitEvent(h, (cudaEvent_t)A->e2e_ev_start, 0));
+    CUDA_TRY(cudaStreamWaitEvent(d, (cudaEvent_t)A->e2e_ev_start, 0));
+    for (int c = 0; c < nch; ++c) {
+        const int64_t x0 = A->e2e_xcut[c], x1 = A->e2e_xcut[c + 1];
+        if (x1 > x0) CUDA_TRY(cudaMemcpyAsync(dx + x0 * es, hx + x0 * es, (x1 - x0) * es, cudaMemcpyHostToDevice, h));
+        if (beta_nz) {
+            int64_t r0, r1;
+            yrange(c, r0, r1);
+            if (r1 > r0) CUDA_TRY(cudaMemcpyAsync(dy + r0 * es, hy + r0 * es, (r1 - r0) * es, cudaMemcpyHostToDevice, h));
+        }
+        CUDA_TRY(cudaEventRecord((cudaEvent_t)A->e2e_ev_x[c], h));
+    }
+    int launches = 0;
+    for (int c = 0; c < nch; ++c) {
+        const int need = std::max(A->e2e_need[c], beta_nz ? c : 0);
+        CUDA_TRY(cudaStreamWaitEvent(s, (cudaEvent_t)A->e2e_ev_x[need], 0));
+        st = run_lists(A, alpha, dx, beta, dy, nullptr, A->e2e_seg[c], A->e2e_seg[c + 1] - A->e2e_seg[c], s, launches);
+        if (st) return st;
+        CUDA_TRY(cudaEventRecord((cudaEvent_t)A->e2e_ev_y[c], s));
+        CUDA_TRY(cudaStreamWaitEvent(d, (cudaEvent_t)A->e2e_ev_y[c], 0));
+        int64_t r0, r1;
+        yrange(c, r0, r1);
+        if (r1 > r0) CUDA_TRY(cudaMemcpyAsync(hy + r0 * es, dy + r0 * es, (r1 - r0) * es, cudaMemcpyDeviceToHost, d));
+    }
+    // all x chunks must have landed before the scratch can be reused (the
+    // last row chunk may not need the last x chunk)
+    CUDA_TRY(cudaStreamWaitEvent(d, (cudaEvent_t)A->e2e_ev_x[nch - 1], 0));
+    CUDA_TRY(cudaEventRecord((cudaEvent_t)A->e2e_ev_done, d));
+    CUDA_TRY(cudaStreamWaitEvent(s, (cudaEvent_t)A->e2e_ev_done, 0));
+    A->last_launches = launches;
     CUDA_TRY(cudaStreamSynchronize(s));
     return CRSD_OK;
 }

@@ -42,6 +42,16 @@ struct crsd_matrix_s {
     void *d_x_scratch = nullptr;
     void *d_y_scratch = nullptr;
 
+    // end-to-end pipeline (crsd_spmv_host): row chunks, x chunks, streams
+    bool e2e_ready = false;
+    int e2e_nchunk = 0;
+    std::vector<int64_t> e2e_seg;      // nchunk + 1 segment boundaries
+    std::vector<int64_t> e2e_xcut;     // nchunk + 1 x element boundaries
+    std::vector<int> e2e_need;         // last x chunk each row chunk needs
+    void *e2e_h2d = nullptr, *e2e_d2h = nullptr;  // cudaStream_t
+    std::vector<void *> e2e_ev_x, e2e_ev_y;         // cudaEvent_t
+    void *e2e_ev_start = nullptr, *e2e_ev_done = nullptr;
+
     // multi-GPU plan (crsd_dist_bind)
     bool bound = false;
     std::vector<int64_t> recv_peer, recv_off, recv_count;  // offsets into x_padded
@@ -53,5 +63,5 @@ void free_device(crsd_matrix_s *A);
 // Run the SpMV kernel over a device list of segments (list == nullptr: all
 // segments [0, count)). x_base is the local x base (x_padded + halo_lo).
 crsd_status_t run_lists(crsd_matrix_s *A, const void *alpha, const void *x_base, const void *beta, void *y,
-                        const int32_t *list, int64_t count, void *stream, int &launches);
+                        const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches);
 }  // namespace crsd

@@ -212,11 +212,11 @@ crsd_status_t crsd_spmv_dist(crsd_matrix_t A, const void *alpha, void *x_padded,
         NCCL_TRY(ncclGroupEnd());
         CU_TRY(cudaEventRecord(c->ev_halo, c->cs));
     }
-    st = crsd::run_lists(A, alpha, xbase, beta, y_local, (const int32_t *)A->d_list_interior,
+    st = crsd::run_lists(A, alpha, xbase, beta, y_local, (const int32_t *)A->d_list_interior, 0,
                          (int64_t)A->list_interior.size(), stream, launches);
     if (st) return st;
     if (c) CU_TRY(cudaStreamWaitEvent(s, c->ev_halo, 0));
-    st = crsd::run_lists(A, alpha, xbase, beta, y_local, (const int32_t *)A->d_list_boundary,
+    st = crsd::run_lists(A, alpha, xbase, beta, y_local, (const int32_t *)A->d_list_boundary, 0,
                          (int64_t)A->list_boundary.size(), stream, launches);
     A->last_launches = launches;
     return st;

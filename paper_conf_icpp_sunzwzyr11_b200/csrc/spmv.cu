@@ -388,13 +388,14 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
     (void)sm_count;
     cudaError_t e;
     if (a.variant == VARIANT_TMA) {
-        static bool attr_done[2] = {false, false};
+        // opt in to the dynamic shared memory this matrix needs (grows only)
+        static int attr_bytes[2] = {0, 0};
         auto kern = crsd_spmv_tma<T>;
-        bool &done = attr_done[sizeof(T) == 8];
-        if (!done || a.smem_bytes > 48 * 1024) {
-            e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+        int &cur = attr_bytes[sizeof(T) == 8];
+        if (a.smem_bytes > cur) {
+            e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, a.smem_bytes);
             if (e != cudaSuccess) return -(int)e;
-            done = true;
+            cur = a.smem_bytes;
         }
         kern<<<(unsigned)grid, threads, a.smem_bytes, (cudaStream_t)stream>>>(a);
     } else {

@@ -152,10 +152,13 @@ def test_misaligned_vectors_rejected(torch_cuda):
         A.spmv(x[1:], y)
 
 
+@pytest.mark.parametrize("variant", VARIANTS)
+@pytest.mark.parametrize("n", [24, 96])
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
-def test_spmv_host_e2e(torch_cuda, dt):
-    a = gen.config3(n=24).astype(dt)
-    A = _mat(a)
+def test_spmv_host_e2e(torch_cuda, dt, n, variant):
+    """crsd_spmv_host: chunked H2D / compute / D2H pipeline (16 chunks at n=96)."""
+    a = gen.config3(n=n).astype(dt)
+    A = _mat(a, variant=variant)
     rng = np.random.default_rng(3)
     x = rng.uniform(-1, 1, a.ncols).astype(dt)
     y0 = rng.uniform(-1, 1, a.nrows).astype(dt)
@@ -163,6 +166,12 @@ def test_spmv_host_e2e(torch_cuda, dt):
     A.spmv_host(x, y, -0.75, 0.5)
     yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, x, -0.75, 0.5, y0)
     assert coo.parity_error(y, yref, scale) <= TOL[dt]
+    y2 = np.full(a.nrows, np.nan, dt)
+    A.spmv_host(x, y2, 1.0, 0.0)
+    yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, x)
+    assert coo.parity_error(y2, yref, scale) <= TOL[dt]
+    if n == 96:
+        assert A.last_launch_count() == 16
 
 
 # ---------------------------------------------------------------- full sizes
