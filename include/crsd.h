@@ -82,10 +82,13 @@ typedef enum { CRSD_R32F = 0, CRSD_R64F = 1 } crsd_dtype_t;
  *   device    CUDA device ordinal the handle's memory lives on (-1 => current).
  *   nthreads  host builder threads (OpenMP); 0 => OpenMP default.
  *   variant   GPU kernel: CRSD_VARIANT_AUTO (0), CRSD_VARIANT_LDG (1: 128-bit
- *             register loads, x by warp shuffle) or CRSD_VARIANT_TMA (2: bulk
- *             copies of the segment's values and x windows into shared
- *             memory). AUTO picks TMA when the largest pattern's staging fits
- *             in shared memory. DESIGN.md "Kernels".
+ *             register loads, x by warp shuffle), CRSD_VARIANT_TMA (2: one CTA
+ *             per segment, bulk copies of its values and x windows into
+ *             shared memory) or CRSD_VARIANT_PIPE (3: persistent CTAs, a
+ *             producer warp streams value chunks through a shared-memory
+ *             ring with TMA bulk copies). AUTO picks PIPE when the largest
+ *             pattern's x windows fit in shared memory, else LDG. DESIGN.md
+ *             "Kernels".
  */
 typedef struct {
     int32_t mrows;
@@ -101,6 +104,7 @@ typedef struct {
 #define CRSD_VARIANT_AUTO 0
 #define CRSD_VARIANT_LDG 1
 #define CRSD_VARIANT_TMA 2
+#define CRSD_VARIANT_PIPE 3
 
 typedef struct crsd_matrix_s *crsd_matrix_t;
 typedef struct crsd_comm_s *crsd_comm_t;
@@ -127,7 +131,7 @@ typedef struct {
     int64_t halo_lo, halo_hi;       /* x halo pads (elements) of a row-partitioned handle; halo_lo is a multiple of 4 */
     int64_t halo_lo_valid, halo_hi_valid; /* halo elements actually exchanged (<= the pads; clipped at the matrix edges) */
     int64_t device_bytes;           /* device memory held by the handle */
-    int32_t variant;                /* kernel variant in use (CRSD_VARIANT_LDG / _TMA) */
+    int32_t variant;                /* kernel variant in use (CRSD_VARIANT_LDG / _TMA / _PIPE) */
     int32_t smem_bytes;             /* dynamic shared memory per CTA of the TMA variant */
     int64_t unique_bytes_beta0;     /* algorithmic bytes of one SpMV with beta == 0 */
     int64_t unique_bytes_beta1;     /* ... with beta != 0 (y also read) */

@@ -27,7 +27,7 @@ STATUS = {
 }
 CRSD_R32F, CRSD_R64F = 0, 1
 CRSD_SUM_DUPLICATES, CRSD_HOST_ONLY, CRSD_DROP_ZEROS = 0x1, 0x2, 0x4
-VARIANT_AUTO, VARIANT_LDG, VARIANT_TMA = 0, 1, 2
+VARIANT_AUTO, VARIANT_LDG, VARIANT_TMA, VARIANT_PIPE = 0, 1, 2, 3
 
 # every symbol include/crsd.h declares
 EXPORTED = [

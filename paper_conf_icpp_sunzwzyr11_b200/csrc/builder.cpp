@@ -586,7 +586,9 @@ void make_segdescs(const HostCRSD &H, int rpt, int64_t x_lo, int64_t x_hi, std::
     }
 }
 
-int64_t make_plans(const HostCRSD &H, int64_t gap, std::vector<int32_t> &plan, std::vector<SegDesc> &segs) {
+int64_t make_plans(const HostCRSD &H, int64_t gap, std::vector<int32_t> &plan, std::vector<SegDesc> &segs,
+                   int64_t *xmax_elems) {
+    int64_t xmx = 0;
     const int64_t m = H.mrows, es = H.elem, al = 16 / H.elem;  // alignment in elements
     std::vector<int32_t> begin(H.npat());
     std::vector<int64_t> smem(H.npat());
@@ -610,6 +612,7 @@ int64_t make_plans(const HostCRSD &H, int64_t gap, std::vector<int32_t> &plan, s
             d = e + 1;
         }
         begin[p] = (int32_t)plan.size();
+        xmx = std::max(xmx, xbase);
         const int64_t bytes = nd * m * es + xbase * es;
         smem[p] = bytes;
         mx = std::max(mx, bytes);
@@ -622,6 +625,7 @@ int64_t make_plans(const HostCRSD &H, int64_t gap, std::vector<int32_t> &plan, s
         plan.insert(plan.end(), xoff.begin(), xoff.end());
     }
     if (plan.empty()) plan.push_back(0);
+    if (xmax_elems) *xmax_elems = xmx;
     for (size_t i = 0; i < H.inst.size(); ++i) {
         const Instance &I = H.inst[i];
         for (int64_t s = I.first_seg; s < I.first_seg + I.nseg; ++s) segs[s].plan_begin = begin[I.pattern];

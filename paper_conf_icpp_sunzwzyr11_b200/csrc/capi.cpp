@@ -87,7 +87,7 @@ static void plan_layout(crsd_matrix_s *A) {
     }
     make_segdescs(H, A->rpt, A->x_lo, A->x_hi, A->segdesc);
     // x windows: offsets closer than 64 elements share one staged window
-    A->smem_bytes = make_plans(H, 64, A->plan, A->segdesc);
+    A->smem_bytes = make_plans(H, 64, A->plan, A->segdesc, &A->xmax_elems);
     A->list_interior.clear();
     A->list_boundary.clear();
     A->nedge = 0;
@@ -143,9 +143,18 @@ static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_
         delete A;
         return fail(CRSD_ERR_UNSUPPORTED, msg);
     }
+    // PIPE needs two x slots of the largest pattern's windows plus >= 2 ring stages
+    const int64_t pipe_need = 2 * A->xmax_elems * A->H.elem + 2 * 8 * (int64_t)A->H.mrows * A->H.elem + 1024;
+    if (o.variant == CRSD_VARIANT_PIPE && pipe_need > smem_cap) {
+        const std::string msg = "PIPE variant: x staging needs " + std::to_string(pipe_need) +
+                                " bytes of shared memory per CTA (> 200 KB); use CRSD_VARIANT_LDG";
+        delete A;
+        return fail(CRSD_ERR_UNSUPPORTED, msg);
+    }
     if (o.variant == CRSD_VARIANT_LDG) A->variant = VARIANT_LDG;
     else if (o.variant == CRSD_VARIANT_TMA) A->variant = VARIANT_TMA;
-    else A->variant = (A->smem_bytes <= smem_cap) ? VARIANT_TMA : VARIANT_LDG;
+    else if (o.variant == CRSD_VARIANT_PIPE) A->variant = VARIANT_PIPE;
+    else A->variant = (pipe_need <= smem_cap) ? VARIANT_PIPE : VARIANT_LDG;
     if (!A->host_only) {
         if (A->H.mrows / A->rpt > 256) {
             delete A;
@@ -194,6 +203,7 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
     a.pat_offs = (const int32_t *)A->d_offs;
     a.plan = (const int32_t *)A->d_plan;
     a.smem_bytes = (int32_t)A->smem_bytes;
+    a.pipe_xmax_elems = (int32_t)A->xmax_elems;
     a.variant = A->variant;
     a.scat_row = (const int32_t *)A->d_scat_row;
     a.scat_col = (const int64_t *)A->d_scat_col;
@@ -210,7 +220,14 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
     a.alpha = alpha;
     a.beta = beta;
     int n = launch_spmv<T>(a, A->sm_count, stream);
-    if (n < 0) return fail(CRSD_ERR_CUDA, std::string("kernel launch: ") + cudaGetErrorString((cudaError_t)(-n)));
+    if (n <= -10000)
+        return fail(CRSD_ERR_CUDA, std::string("cudaFuncSetAttribute(MaxDynamicSharedMemorySize=") +
+                                       std::to_string(a.smem_bytes) + "): " + cudaGetErrorString((cudaError_t)(-n - 10000)));
+    if (n < 0)
+        return fail(CRSD_ERR_CUDA, std::string("kernel launch (variant ") + std::to_string(a.variant) + ", grid " +
+                                       std::to_string(a.seg_count) + ", block " + std::to_string(A->H.mrows / A->rpt) +
+                                       ", smem " + std::to_string(a.variant == VARIANT_TMA ? a.smem_bytes : 0) +
+                                       "): " + cudaGetErrorString((cudaError_t)(-n)));
     launches += n;
     return CRSD_OK;
 }

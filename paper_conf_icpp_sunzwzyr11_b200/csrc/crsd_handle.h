@@ -15,6 +15,7 @@ struct crsd_matrix_s {
     int rpt = 2;
     int variant = crsd::VARIANT_LDG;
     int64_t smem_bytes = 0;
+    int64_t xmax_elems = 0;
     std::vector<int32_t> plan;
     int32_t last_launches = 0;
     int64_t device_bytes = 0;

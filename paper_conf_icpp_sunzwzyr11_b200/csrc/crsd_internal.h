@@ -42,7 +42,7 @@ struct alignas(16) SegDesc {
 constexpr int MAX_NDIAS = 4096;
 
 // Kernel variants
-enum : int32_t { VARIANT_AUTO = 0, VARIANT_LDG = 1, VARIANT_TMA = 2 };
+enum : int32_t { VARIANT_AUTO = 0, VARIANT_LDG = 1, VARIANT_TMA = 2, VARIANT_PIPE = 3 };
 
 // TMA staging plan of one distinct pattern (int32 words at plan_begin):
 //   [0] nwin  [1] smem bytes (values + windows)
@@ -109,7 +109,8 @@ void make_segdescs(const HostCRSD &H, int rpt, int64_t x_lo, int64_t x_hi, std::
 
 // TMA staging plans of all distinct patterns (x windows = clusters of offsets
 // closer than `gap` elements); fills SegDesc::plan_begin; returns max smem.
-int64_t make_plans(const HostCRSD &H, int64_t gap, std::vector<int32_t> &plan, std::vector<SegDesc> &segs);
+int64_t make_plans(const HostCRSD &H, int64_t gap, std::vector<int32_t> &plan, std::vector<SegDesc> &segs,
+                   int64_t *xmax_elems = nullptr);
 
 // Halo extents (elements outside [0, n_local) relative to the local x base)
 // the handle needs: from its non-edge windows and its scatter columns.
@@ -135,6 +136,7 @@ struct SpmvArgs {
     int64_t seg_begin, seg_count;
     int32_t mrows;
     int32_t smem_bytes;       // TMA variant: dynamic shared memory per CTA
+    int32_t pipe_xmax_elems;  // PIPE variant: largest x staging of a pattern (elements)
     int32_t variant;          // VARIANT_LDG or VARIANT_TMA
     T alpha, beta;
 };

@@ -378,6 +378,205 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a) {
     }
 }
 
+// ---------------------------------------------------------------------------
+// Persistent, warp-specialised TMA pipeline (variant PIPE). Warp 0 (one
+// elected lane) is the producer: for each segment of this CTA it stages the
+// segment descriptor and the pattern's x windows into one of two x slots,
+// then streams the segment's value block in chunks of up to KCH diagonals
+// through a ring of NS shared-memory stages (cp.async.bulk + mbarrier
+// complete_tx). The consumer warps (mrows/RPT threads) compute from shared
+// memory and release stages through "empty" mbarriers. Bytes in flight are
+// set by the ring depth, not by the segment size, and the descriptor and
+// window fetches of the next segment overlap the current one.
+// ---------------------------------------------------------------------------
+struct PipeSeg {  // segment info handed from producer to consumers (per x slot)
+    int64_t row0;
+    int64_t scat_begin;
+    int32_t nscat;
+    int32_t flags;
+    int32_t nd;
+    int32_t plan_begin;
+    int32_t off_begin;
+    int32_t pad;
+};
+
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+template <typename T, int KCH>
+__global__ void __launch_bounds__(288, 1) crsd_spmv_pipe(const SpmvArgs<T> a, int ns, int xmax_elems) {
+    constexpr int kch = KCH;
+    constexpr int R = VecT<T>::R;
+    extern __shared__ __align__(128) unsigned char smem[];
+    // layout: [bars: 4 + 2*ns][PipeSeg x2][xbuf x2][vring x ns]
+    uint64_t *full_x = reinterpret_cast<uint64_t *>(smem);
+    uint64_t *empty_x = full_x + 2;
+    uint64_t *full_v = full_x + 4;
+    uint64_t *empty_v = full_v + ns;
+    PipeSeg *sseg = reinterpret_cast<PipeSeg *>(smem + ((8 * (4 + 2 * ns) + 127) / 128) * 128);
+    T *xbuf = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sseg) + 128);
+    T *vring = xbuf + 2 * (int64_t)xmax_elems;
+    const int C = a.mrows / R;  // consumer threads
+    const int nwarps_c = C / 32;
+    const int64_t chunk_elems = (int64_t)kch * a.mrows;
+
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < 2; ++i) {
+            mbar_init(full_x + i, 1);
+            mbar_init(empty_x + i, nwarps_c);
+        }
+        for (int i = 0; i < ns; ++i) {
+            mbar_init(full_v + i, 1);
+            mbar_init(empty_v + i, nwarps_c);
+        }
+        mbar_fence_init();
+    }
+    __syncthreads();
+
+    if (threadIdx.x < 32) {
+        // ------------------------------ producer ------------------------------
+        if (threadIdx.x != 0) return;
+        const uint64_t pf = policy_evict_first(), pn = policy_evict_normal();
+        int xs = 0, vs = 0;
+        uint32_t xph = 0, vph = 0;
+        for (int64_t w = blockIdx.x; w < a.seg_count; w += gridDim.x) {
+            const int64_t sg = a.seg_list ? (int64_t)__ldg(a.seg_list + w) : a.seg_begin + w;
+            const SegDesc D = a.segs[sg];
+            const int64_t row0 = sg * a.mrows;
+            const bool edge = (D.flags & SEG_EDGE) != 0;
+            const int32_t *plan = a.plan + D.plan_begin;
+            const int nwin = __ldg(plan);
+            mbar_wait(empty_x + xs, xph ^ 1);
+            PipeSeg &P = sseg[xs];
+            P.row0 = row0;
+            P.scat_begin = D.scat_begin;
+            P.nscat = D.nscat;
+            P.flags = D.flags;
+            P.nd = D.ndias;
+            P.plan_begin = D.plan_begin;
+            P.off_begin = D.off_begin;
+            uint32_t xbytes = 0;
+            if (!edge)
+                for (int q = 0; q < nwin; ++q) xbytes += (uint32_t)__ldg(plan + 3 + 2 * q) * sizeof(T);
+            mbar_expect_tx(full_x + xs, xbytes);  // arrive (release: P visible) + tx
+            if (!edge) {
+                T *dst = xbuf + (int64_t)xs * xmax_elems;
+                for (int q = 0; q < nwin; ++q) {
+                    const int st = __ldg(plan + 2 + 2 * q), cnt = __ldg(plan + 3 + 2 * q);
+                    bulk_g2s(dst, a.x + row0 + st, (uint32_t)cnt * sizeof(T), full_x + xs, pn);
+                    dst += cnt;
+                }
+            }
+            xs ^= 1;
+            if (xs == 0) xph ^= 1;
+            const int nd = D.ndias;
+            for (int d0 = 0; d0 < nd; d0 += kch) {
+                const int nk = min(kch, nd - d0);
+                mbar_wait(empty_v + vs, vph ^ 1);
+                const uint32_t bytes = (uint32_t)nk * (uint32_t)a.mrows * sizeof(T);
+                mbar_expect_tx(full_v + vs, bytes);
+                bulk_g2s(vring + (int64_t)vs * chunk_elems, a.vals + D.val_base + (int64_t)d0 * a.mrows, bytes,
+                         full_v + vs, pf);
+                if (++vs == ns) {
+                    vs = 0;
+                    vph ^= 1;
+                }
+            }
+        }
+        return;
+    }
+    // ------------------------------ consumers ------------------------------
+    const int ct = threadIdx.x - 32;
+    const int lane = ct & 31;
+    int xs = 0, vs = 0;
+    uint32_t xph = 0, vph = 0;
+    const T al = a.alpha, be = a.beta;
+    for (int64_t w = blockIdx.x; w < a.seg_count; w += gridDim.x) {
+        mbar_wait(full_x + xs, xph);
+        const PipeSeg P = sseg[xs];
+        const bool edge = (P.flags & SEG_EDGE) != 0;
+        const int32_t *plan = a.plan + P.plan_begin;
+        const int nwin = __ldg(plan);
+        const int32_t *xoff = plan + 2 + 2 * nwin;
+        const int32_t *offs = a.pat_offs + P.off_begin;
+        const T *xb = xbuf + (int64_t)xs * xmax_elems;
+        T acc[R];
+#pragma unroll
+        for (int q = 0; q < R; ++q) acc[q] = T(0);
+        for (int d0 = 0; d0 < P.nd; d0 += kch) {
+            const int nk = min(kch, P.nd - d0);
+            mbar_wait(full_v + vs, vph);
+            const T *vb = vring + (int64_t)vs * chunk_elems + ct;
+            if (!edge) {
+                int xo[KCH];
+#pragma unroll
+                for (int k = 0; k < KCH; ++k)
+                    if (k < nk) xo[k] = __ldg(xoff + d0 + k);
+#pragma unroll
+                for (int k = 0; k < KCH; ++k) {
+                    if (k < nk) {
+                        const T *xd = xb + xo[k] + ct;
+                        const T *vd = vb + k * a.mrows;
+#pragma unroll
+                        for (int q = 0; q < R; ++q) acc[q] = fma(vd[q * C], xd[q * C], acc[q]);
+                    }
+                }
+            } else {
+                for (int k = 0; k < nk; ++k) {
+                    const int o = __ldg(offs + d0 + k);
+                    const T *vd = vb + k * a.mrows;
+#pragma unroll
+                    for (int q = 0; q < R; ++q) {
+                        const int64_t idx = P.row0 + ct + q * C + o;
+                        const T xj = (idx >= a.x_lo && idx < a.x_hi) ? __ldg(a.x + idx) : T(0);
+                        acc[q] = fma(vd[q * C], xj, acc[q]);
+                    }
+                }
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(empty_v + vs);
+            if (++vs == ns) {
+                vs = 0;
+                vph ^= 1;
+            }
+        }
+        // scatter points (owner of local row l is consumer l % C, slot l / C)
+        if (P.nscat > 0) {
+            const int32_t *sr = a.scat_row + P.scat_begin;
+            for (int64_t e = 0; e < P.nscat; ++e) {
+                const int rr = __ldg(sr + e);
+                if (rr % C != ct) continue;
+                const T v = __ldg(a.scat_val + P.scat_begin + e);
+                const T xv = __ldg(a.x + __ldg(a.scat_col + P.scat_begin + e));
+                const int q = rr / C;
+#pragma unroll
+                for (int j = 0; j < R; ++j)
+                    if (q == j) acc[j] = fma(v, xv, acc[j]);
+            }
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(empty_x + xs);
+#pragma unroll
+        for (int q = 0; q < R; ++q) {
+            const int64_t r = P.row0 + ct + q * C;
+            if (!edge || r < a.nrows) {
+                T *yp = a.y + r;
+                const T out = (be != T(0)) ? fma(al, acc[q], be * *yp) : al * acc[q];
+                __stcs(yp, out);
+            }
+        }
+        xs ^= 1;
+        if (xs == 0) xph ^= 1;
+    }
+}
+
+// shared memory of the PIPE variant for a given ring depth
+inline int64_t pipe_smem(int ns, int kch, int mrows, int elem, int64_t xmax_elems) {
+    const int64_t bars = ((8 * (4 + 2 * ns) + 127) / 128) * 128;
+    return bars + 128 + 2 * xmax_elems * elem + (int64_t)ns * kch * mrows * elem;
+}
+
 template <typename T>
 int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
     if (a.seg_count <= 0) return 0;
@@ -385,7 +584,6 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
     const int threads = a.mrows / R;
     int64_t grid = a.seg_count;
     if (grid > 0x7fffffff) grid = 0x7fffffff;
-    (void)sm_count;
     cudaError_t e;
     if (a.variant == VARIANT_TMA) {
         // opt in to the dynamic shared memory this matrix needs (grows only)
@@ -394,10 +592,28 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
         int &cur = attr_bytes[sizeof(T) == 8];
         if (a.smem_bytes > cur) {
             e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, a.smem_bytes);
-            if (e != cudaSuccess) return -(int)e;
+            if (e != cudaSuccess) return -(10000 + (int)e);
             cur = a.smem_bytes;
         }
         kern<<<(unsigned)grid, threads, a.smem_bytes, (cudaStream_t)stream>>>(a);
+    } else if (a.variant == VARIANT_PIPE) {
+        // ring of KCH-diagonal value chunks; depth chosen so two CTAs fit per SM
+        constexpr int kch = 8;
+        const int64_t xmax = a.pipe_xmax_elems;
+        int ns = 8;
+        while (ns > 2 && pipe_smem(ns, kch, a.mrows, sizeof(T), xmax) > 110 * 1024) --ns;
+        const int64_t sm = pipe_smem(ns, kch, a.mrows, sizeof(T), xmax);
+        static int attr_pipe[2] = {0, 0};
+        int &cur = attr_pipe[sizeof(T) == 8];
+        if (sm > cur) {
+            e = cudaFuncSetAttribute(crsd_spmv_pipe<T, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+            if (e != cudaSuccess) return -(10000 + (int)e);
+            cur = (int)sm;
+        }
+        const int per_sm = sm <= 110 * 1024 ? 2 : 1;
+        int64_t g = (int64_t)sm_count * per_sm;
+        if (g > a.seg_count) g = a.seg_count;
+        crsd_spmv_pipe<T, kch><<<(unsigned)g, threads + 32, sm, (cudaStream_t)stream>>>(a, ns, (int)xmax);
     } else {
         crsd_spmv_ldg<T, 4><<<(unsigned)grid, threads, 0, (cudaStream_t)stream>>>(a);
     }
