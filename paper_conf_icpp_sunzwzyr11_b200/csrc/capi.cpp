@@ -151,10 +151,14 @@ static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_
         delete A;
         return fail(CRSD_ERR_UNSUPPORTED, msg);
     }
+    if (o.variant == CRSD_VARIANT_PIPE && A->H.mrows > 512) {
+        delete A;
+        return fail(CRSD_ERR_UNSUPPORTED, "PIPE variant runs one row per thread: mrows must be <= 512");
+    }
     if (o.variant == CRSD_VARIANT_LDG) A->variant = VARIANT_LDG;
     else if (o.variant == CRSD_VARIANT_TMA) A->variant = VARIANT_TMA;
     else if (o.variant == CRSD_VARIANT_PIPE) A->variant = VARIANT_PIPE;
-    else A->variant = (pipe_need <= smem_cap) ? VARIANT_PIPE : VARIANT_LDG;
+    else A->variant = (pipe_need <= smem_cap && A->H.mrows <= 512) ? VARIANT_PIPE : VARIANT_LDG;
     if (!A->host_only) {
         if (A->H.mrows / A->rpt > 256) {
             delete A;
@@ -180,8 +184,7 @@ static crsd_status_t resolve_opts(int64_t nrows, crsd_dtype_t dtype, const crsd_
                                   BuildOptions &b) {
     if (opts) o = *opts;
     else crsd_opts_init(&o);
-    const int rpt = (dtype == CRSD_R64F) ? 2 : 4;
-    if (o.mrows == 0) o.mrows = 128 * rpt;
+    if (o.mrows == 0) o.mrows = 256;
     if (o.idle_max < 0) o.idle_max = o.mrows - 1;
     if (o.row_begin == 0 && o.row_end == 0) o.row_end = nrows;
     b.mrows = o.mrows;

@@ -405,9 +405,8 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
 }
 
 template <typename T, int KCH>
-__global__ void __launch_bounds__(288, 1) crsd_spmv_pipe(const SpmvArgs<T> a, int ns, int xmax_elems) {
+__global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, int ns, int xmax_elems) {
     constexpr int kch = KCH;
-    constexpr int R = VecT<T>::R;
     extern __shared__ __align__(128) unsigned char smem[];
     // layout: [bars: 4 + 2*ns][PipeSeg x2][xbuf x2][vring x ns]
     uint64_t *full_x = reinterpret_cast<uint64_t *>(smem);
@@ -417,7 +416,7 @@ __global__ void __launch_bounds__(288, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
     PipeSeg *sseg = reinterpret_cast<PipeSeg *>(smem + ((8 * (4 + 2 * ns) + 127) / 128) * 128);
     T *xbuf = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sseg) + 128);
     T *vring = xbuf + 2 * (int64_t)xmax_elems;
-    const int C = a.mrows / R;  // consumer threads
+    const int C = a.mrows;  // consumer threads (one row each)
     const int nwarps_c = C / 32;
     const int64_t chunk_elems = (int64_t)kch * a.mrows;
 
@@ -440,9 +439,19 @@ __global__ void __launch_bounds__(288, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
         const uint64_t pf = policy_evict_first(), pn = policy_evict_normal();
         int xs = 0, vs = 0;
         uint32_t xph = 0, vph = 0;
+        // descriptors are prefetched one segment ahead so their global-memory
+        // latency overlaps the previous segment's copies
+        auto seg_of = [&](int64_t w) { return a.seg_list ? (int64_t)__ldg(a.seg_list + w) : a.seg_begin + w; };
+        int64_t sg_next = (blockIdx.x < a.seg_count) ? seg_of(blockIdx.x) : 0;
+        SegDesc D_next;
+        if (blockIdx.x < a.seg_count) D_next = a.segs[sg_next];
         for (int64_t w = blockIdx.x; w < a.seg_count; w += gridDim.x) {
-            const int64_t sg = a.seg_list ? (int64_t)__ldg(a.seg_list + w) : a.seg_begin + w;
-            const SegDesc D = a.segs[sg];
+            const int64_t sg = sg_next;
+            const SegDesc D = D_next;
+            if (w + gridDim.x < a.seg_count) {
+                sg_next = seg_of(w + gridDim.x);
+                D_next = a.segs[sg_next];
+            }
             const int64_t row0 = sg * a.mrows;
             const bool edge = (D.flags & SEG_EDGE) != 0;
             const int32_t *plan = a.plan + D.plan_begin;
@@ -487,6 +496,7 @@ __global__ void __launch_bounds__(288, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
         return;
     }
     // ------------------------------ consumers ------------------------------
+    // one row per consumer thread: row0 + ct (conflict-free shared reads)
     const int ct = threadIdx.x - 32;
     const int lane = ct & 31;
     int xs = 0, vs = 0;
@@ -500,10 +510,9 @@ __global__ void __launch_bounds__(288, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
         const int nwin = __ldg(plan);
         const int32_t *xoff = plan + 2 + 2 * nwin;
         const int32_t *offs = a.pat_offs + P.off_begin;
-        const T *xb = xbuf + (int64_t)xs * xmax_elems;
-        T acc[R];
-#pragma unroll
-        for (int q = 0; q < R; ++q) acc[q] = T(0);
+        const T *xb = xbuf + (int64_t)xs * xmax_elems + ct;
+        const int64_t row = P.row0 + ct;
+        T acc = T(0);
         for (int d0 = 0; d0 < P.nd; d0 += kch) {
             const int nk = min(kch, P.nd - d0);
             mbar_wait(full_v + vs, vph);
@@ -514,24 +523,13 @@ __global__ void __launch_bounds__(288, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
                 for (int k = 0; k < KCH; ++k)
                     if (k < nk) xo[k] = __ldg(xoff + d0 + k);
 #pragma unroll
-                for (int k = 0; k < KCH; ++k) {
-                    if (k < nk) {
-                        const T *xd = xb + xo[k] + ct;
-                        const T *vd = vb + k * a.mrows;
-#pragma unroll
-                        for (int q = 0; q < R; ++q) acc[q] = fma(vd[q * C], xd[q * C], acc[q]);
-                    }
-                }
+                for (int k = 0; k < KCH; ++k)
+                    if (k < nk) acc = fma(vb[k * C], xb[xo[k]], acc);
             } else {
                 for (int k = 0; k < nk; ++k) {
-                    const int o = __ldg(offs + d0 + k);
-                    const T *vd = vb + k * a.mrows;
-#pragma unroll
-                    for (int q = 0; q < R; ++q) {
-                        const int64_t idx = P.row0 + ct + q * C + o;
-                        const T xj = (idx >= a.x_lo && idx < a.x_hi) ? __ldg(a.x + idx) : T(0);
-                        acc[q] = fma(vd[q * C], xj, acc[q]);
-                    }
+                    const int64_t idx = row + __ldg(offs + d0 + k);
+                    const T xj = (idx >= a.x_lo && idx < a.x_hi) ? __ldg(a.x + idx) : T(0);
+                    acc = fma(vb[k * C], xj, acc);
                 }
             }
             __syncwarp();
@@ -541,30 +539,19 @@ __global__ void __launch_bounds__(288, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
                 vph ^= 1;
             }
         }
-        // scatter points (owner of local row l is consumer l % C, slot l / C)
+        // scatter points of this row, (row, col) order
         if (P.nscat > 0) {
             const int32_t *sr = a.scat_row + P.scat_begin;
             for (int64_t e = 0; e < P.nscat; ++e) {
-                const int rr = __ldg(sr + e);
-                if (rr % C != ct) continue;
-                const T v = __ldg(a.scat_val + P.scat_begin + e);
-                const T xv = __ldg(a.x + __ldg(a.scat_col + P.scat_begin + e));
-                const int q = rr / C;
-#pragma unroll
-                for (int j = 0; j < R; ++j)
-                    if (q == j) acc[j] = fma(v, xv, acc[j]);
+                if (__ldg(sr + e) != ct) continue;
+                acc = fma(__ldg(a.scat_val + P.scat_begin + e), __ldg(a.x + __ldg(a.scat_col + P.scat_begin + e)), acc);
             }
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(empty_x + xs);
-#pragma unroll
-        for (int q = 0; q < R; ++q) {
-            const int64_t r = P.row0 + ct + q * C;
-            if (!edge || r < a.nrows) {
-                T *yp = a.y + r;
-                const T out = (be != T(0)) ? fma(al, acc[q], be * *yp) : al * acc[q];
-                __stcs(yp, out);
-            }
+        if (!edge || row < a.nrows) {
+            T *yp = a.y + row;
+            __stcs(yp, (be != T(0)) ? fma(al, acc, be * *yp) : al * acc);
         }
         xs ^= 1;
         if (xs == 0) xph ^= 1;
@@ -600,8 +587,11 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
         // ring of KCH-diagonal value chunks; depth chosen so two CTAs fit per SM
         constexpr int kch = 8;
         const int64_t xmax = a.pipe_xmax_elems;
-        int ns = 8;
-        while (ns > 2 && pipe_smem(ns, kch, a.mrows, sizeof(T), xmax) > 110 * 1024) --ns;
+        // two CTAs per SM when the consumer count allows it, else one with a deeper ring
+        const int per_sm = a.mrows <= 256 ? 2 : 1;
+        const int64_t budget = per_sm == 2 ? 110 * 1024 : 220 * 1024;
+        int ns = 16;
+        while (ns > 2 && pipe_smem(ns, kch, a.mrows, sizeof(T), xmax) > budget) --ns;
         const int64_t sm = pipe_smem(ns, kch, a.mrows, sizeof(T), xmax);
         static int attr_pipe[2] = {0, 0};
         int &cur = attr_pipe[sizeof(T) == 8];
@@ -610,10 +600,9 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
             if (e != cudaSuccess) return -(10000 + (int)e);
             cur = (int)sm;
         }
-        const int per_sm = sm <= 110 * 1024 ? 2 : 1;
         int64_t g = (int64_t)sm_count * per_sm;
         if (g > a.seg_count) g = a.seg_count;
-        crsd_spmv_pipe<T, kch><<<(unsigned)g, threads + 32, sm, (cudaStream_t)stream>>>(a, ns, (int)xmax);
+        crsd_spmv_pipe<T, kch><<<(unsigned)g, a.mrows + 32, sm, (cudaStream_t)stream>>>(a, ns, (int)xmax);
     } else {
         crsd_spmv_ldg<T, 4><<<(unsigned)grid, threads, 0, (cudaStream_t)stream>>>(a);
     }
