@@ -207,6 +207,11 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
     a.plan = (const int32_t *)A->d_plan;
     a.smem_bytes = (int32_t)A->smem_bytes;
     a.pipe_xmax_elems = (int32_t)A->xmax_elems;
+    {
+        int64_t mx = 0;
+        for (int64_t p = 0; p < A->H.npat(); ++p) mx = std::max<int64_t>(mx, A->H.ndias((int32_t)p));
+        a.max_ndias = (int32_t)mx;
+    }
     a.variant = A->variant;
     a.scat_row = (const int32_t *)A->d_scat_row;
     a.scat_col = (const int64_t *)A->d_scat_col;

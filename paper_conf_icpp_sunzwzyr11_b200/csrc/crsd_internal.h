@@ -137,6 +137,7 @@ struct SpmvArgs {
     int32_t mrows;
     int32_t smem_bytes;       // TMA variant: dynamic shared memory per CTA
     int32_t pipe_xmax_elems;  // PIPE variant: largest x staging of a pattern (elements)
+    int32_t max_ndias;        // largest NDias over patterns
     int32_t variant;          // VARIANT_LDG or VARIANT_TMA
     T alpha, beta;
 };

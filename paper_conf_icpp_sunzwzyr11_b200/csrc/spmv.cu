@@ -26,7 +26,9 @@
 // writes y once (y read only when beta != 0).
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 
 #include "crsd_internal.h"
 
@@ -405,23 +407,23 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
 }
 
 template <typename T, int KCH>
-__global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, int ns, int xmax_elems) {
+__global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, int ns, int nx, int xmax_elems) {
     constexpr int kch = KCH;
     extern __shared__ __align__(128) unsigned char smem[];
-    // layout: [bars: 4 + 2*ns][PipeSeg x2][xbuf x2][vring x ns]
+    // layout: [bars: 2*nx + 2*ns][PipeSeg x nx][xbuf x nx][vring x ns]
     uint64_t *full_x = reinterpret_cast<uint64_t *>(smem);
-    uint64_t *empty_x = full_x + 2;
-    uint64_t *full_v = full_x + 4;
+    uint64_t *empty_x = full_x + nx;
+    uint64_t *full_v = full_x + 2 * nx;
     uint64_t *empty_v = full_v + ns;
-    PipeSeg *sseg = reinterpret_cast<PipeSeg *>(smem + ((8 * (4 + 2 * ns) + 127) / 128) * 128);
-    T *xbuf = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sseg) + 128);
-    T *vring = xbuf + 2 * (int64_t)xmax_elems;
+    PipeSeg *sseg = reinterpret_cast<PipeSeg *>(smem + ((8 * (2 * nx + 2 * ns) + 127) / 128) * 128);
+    T *xbuf = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sseg) + ((nx * sizeof(PipeSeg) + 127) / 128) * 128);
+    T *vring = xbuf + nx * (int64_t)xmax_elems;
     const int C = a.mrows;  // consumer threads (one row each)
     const int nwarps_c = C / 32;
     const int64_t chunk_elems = (int64_t)kch * a.mrows;
 
     if (threadIdx.x == 0) {
-        for (int i = 0; i < 2; ++i) {
+        for (int i = 0; i < nx; ++i) {
             mbar_init(full_x + i, 1);
             mbar_init(empty_x + i, nwarps_c);
         }
@@ -477,8 +479,10 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
                     dst += cnt;
                 }
             }
-            xs ^= 1;
-            if (xs == 0) xph ^= 1;
+            if (++xs == nx) {
+                xs = 0;
+                xph ^= 1;
+            }
             const int nd = D.ndias;
             for (int d0 = 0; d0 < nd; d0 += kch) {
                 const int nk = min(kch, nd - d0);
@@ -553,15 +557,50 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
             T *yp = a.y + row;
             __stcs(yp, (be != T(0)) ? fma(al, acc, be * *yp) : al * acc);
         }
-        xs ^= 1;
-        if (xs == 0) xph ^= 1;
+        if (++xs == nx) {
+            xs = 0;
+            xph ^= 1;
+        }
     }
 }
 
-// shared memory of the PIPE variant for a given ring depth
-inline int64_t pipe_smem(int ns, int kch, int mrows, int elem, int64_t xmax_elems) {
-    const int64_t bars = ((8 * (4 + 2 * ns) + 127) / 128) * 128;
-    return bars + 128 + 2 * xmax_elems * elem + (int64_t)ns * kch * mrows * elem;
+// shared memory of the PIPE variant for nx x slots and ns value stages
+inline int64_t pipe_smem(int ns, int nx, int kch, int mrows, int elem, int64_t xmax_elems) {
+    const int64_t bars = ((8 * (2 * nx + 2 * ns) + 127) / 128) * 128;
+    const int64_t segs = ((nx * (int64_t)sizeof(PipeSeg) + 127) / 128) * 128;
+    return bars + segs + nx * xmax_elems * elem + (int64_t)ns * kch * mrows * elem;
+}
+
+static int env_int(const char *k, int d) {
+    const char *v = getenv(k);
+    return v ? atoi(v) : d;
+}
+
+// Pipeline shape: CTAs per SM, x slots (segments the producer may run ahead,
+// plus one) and value stages. Maximises the segments in flight per SM,
+// CTAs/SM x min(nx - 1, ns / chunks), under the shared-memory budget.
+// CRSD_PIPE_PERSM / _NX / _NS override (tuning experiments).
+static void pipe_shape(int mrows, int elem, int64_t xmax, int max_nd, int &per_sm, int &nx, int &ns) {
+    constexpr int kch = 8;
+    const int chunks = max_nd > 0 ? (max_nd + kch - 1) / kch : 1;
+    double best = -1.0;
+    per_sm = 1; nx = 2; ns = 2;
+    for (int ps = (mrows <= 256 ? 2 : 1); ps >= 1; --ps) {
+        const int64_t budget = (ps == 2 ? 110 : 220) * 1024;
+        for (int x = 2; x <= 8; ++x) {
+            int n = 0;
+            while (n < 32 && pipe_smem(n + 1, x, kch, mrows, elem, xmax) <= budget) ++n;
+            if (n < 2) continue;
+            const double sc = ps * std::min<double>(x - 1, (double)n / chunks) + 1e-3 * ps;
+            if (sc > best) {
+                best = sc;
+                per_sm = ps; nx = x; ns = n;
+            }
+        }
+    }
+    per_sm = env_int("CRSD_PIPE_PERSM", per_sm);
+    nx = env_int("CRSD_PIPE_NX", nx);
+    ns = env_int("CRSD_PIPE_NS", ns);
 }
 
 template <typename T>
@@ -587,12 +626,9 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
         // ring of KCH-diagonal value chunks; depth chosen so two CTAs fit per SM
         constexpr int kch = 8;
         const int64_t xmax = a.pipe_xmax_elems;
-        // two CTAs per SM when the consumer count allows it, else one with a deeper ring
-        const int per_sm = a.mrows <= 256 ? 2 : 1;
-        const int64_t budget = per_sm == 2 ? 110 * 1024 : 220 * 1024;
-        int ns = 16;
-        while (ns > 2 && pipe_smem(ns, kch, a.mrows, sizeof(T), xmax) > budget) --ns;
-        const int64_t sm = pipe_smem(ns, kch, a.mrows, sizeof(T), xmax);
+        int per_sm, nx, ns;
+        pipe_shape(a.mrows, sizeof(T), xmax, a.max_ndias, per_sm, nx, ns);
+        const int64_t sm = pipe_smem(ns, nx, kch, a.mrows, sizeof(T), xmax);
         static int attr_pipe[2] = {0, 0};
         int &cur = attr_pipe[sizeof(T) == 8];
         if (sm > cur) {
@@ -602,7 +638,7 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
         }
         int64_t g = (int64_t)sm_count * per_sm;
         if (g > a.seg_count) g = a.seg_count;
-        crsd_spmv_pipe<T, kch><<<(unsigned)g, a.mrows + 32, sm, (cudaStream_t)stream>>>(a, ns, (int)xmax);
+        crsd_spmv_pipe<T, kch><<<(unsigned)g, a.mrows + 32, sm, (cudaStream_t)stream>>>(a, ns, nx, (int)xmax);
     } else {
         crsd_spmv_ldg<T, 4><<<(unsigned)grid, threads, 0, (cudaStream_t)stream>>>(a);
     }
