@@ -367,12 +367,32 @@ def run_crsd(args):
         for _ in range(ke):
             A.spmv_host_ptr(xh.data_ptr(), yh.data_ptr(), 1.0, 0.0)
         te = (time.perf_counter() - t0) / ke
+        # transfer bound of the e2e step: pinned H2D / D2H bandwidth alone
+        xd_tmp = torch.empty(a.ncols, dtype=tdt, device=f"cuda:{dev}")
+        yd_tmp = torch.empty(a.nrows, dtype=tdt, device=f"cuda:{dev}")
+
+        def bw(fn, nbytes):
+            fn()
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            for _ in range(5):
+                fn()
+            torch.cuda.synchronize()
+            return nbytes * 5 / (time.perf_counter() - t0) / 1e9
+
+        h2d = bw(lambda: xd_tmp.copy_(xh, non_blocking=True), a.ncols * es)
+        d2h = bw(lambda: yh.copy_(yd_tmp, non_blocking=True), a.nrows * es)
+        del xd_tmp, yd_tmp
         e2e = {
             "value": round(2.0 * nnz_all / te / 1e9, 3),
             "unit": "GFLOP/s",
             "h2d_bytes_per_step": int(a.ncols * es),
             "d2h_bytes_per_step": int(a.nrows * es),
             "ms_per_step": round(te * 1e3, 4),
+            "pinned_h2d_gbs": round(h2d, 1),
+            "pinned_d2h_gbs": round(d2h, 1),
+            "transfer_bound_ms": round(max(a.ncols * es / h2d, a.nrows * es / d2h) / 1e6, 4),
+            "path": "crsd_spmv_host: chunked H2D(x) / kernel / D2H(y) pipeline on three streams",
         }
     if rank != 0:
         if comm is not None:

@@ -437,64 +437,99 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
 
     if (threadIdx.x < 32) {
         // ------------------------------ producer ------------------------------
-        if (threadIdx.x != 0) return;
+        // The whole warp fetches descriptors 32 segments at a time (one
+        // global-memory latency per 32 segments), window plans one window per
+        // lane, and issues the x-window bulk copies in parallel; lane 0 owns the
+        // ring bookkeeping and the value-chunk copies.
+        const int lane = threadIdx.x;
         const uint64_t pf = policy_evict_first(), pn = policy_evict_normal();
         int xs = 0, vs = 0;
         uint32_t xph = 0, vph = 0;
-        // descriptors are prefetched one segment ahead so their global-memory
-        // latency overlaps the previous segment's copies
-        auto seg_of = [&](int64_t w) { return a.seg_list ? (int64_t)__ldg(a.seg_list + w) : a.seg_begin + w; };
-        int64_t sg_next = (blockIdx.x < a.seg_count) ? seg_of(blockIdx.x) : 0;
-        SegDesc D_next;
-        if (blockIdx.x < a.seg_count) D_next = a.segs[sg_next];
-        for (int64_t w = blockIdx.x; w < a.seg_count; w += gridDim.x) {
-            const int64_t sg = sg_next;
-            const SegDesc D = D_next;
-            if (w + gridDim.x < a.seg_count) {
-                sg_next = seg_of(w + gridDim.x);
-                D_next = a.segs[sg_next];
+        const int64_t G = gridDim.x;
+        for (int64_t wb = blockIdx.x; wb < a.seg_count; wb += 32 * G) {
+            const int64_t wl = wb + lane * G;
+            int64_t sgl = 0;
+            SegDesc Dl = {};
+            if (wl < a.seg_count) {
+                sgl = a.seg_list ? (int64_t)__ldg(a.seg_list + wl) : a.seg_begin + wl;
+                Dl = a.segs[sgl];
             }
-            const int64_t row0 = sg * a.mrows;
-            const bool edge = (D.flags & SEG_EDGE) != 0;
-            const int32_t *plan = a.plan + D.plan_begin;
-            const int nwin = __ldg(plan);
-            mbar_wait(empty_x + xs, xph ^ 1);
-            PipeSeg &P = sseg[xs];
-            P.row0 = row0;
-            P.scat_begin = D.scat_begin;
-            P.nscat = D.nscat;
-            P.flags = D.flags;
-            P.nd = D.ndias;
-            P.plan_begin = D.plan_begin;
-            P.off_begin = D.off_begin;
-            uint32_t xbytes = 0;
-            if (!edge)
-                for (int q = 0; q < nwin; ++q) xbytes += (uint32_t)__ldg(plan + 3 + 2 * q) * sizeof(T);
-            mbar_expect_tx(full_x + xs, xbytes);  // arrive (release: P visible) + tx
-            if (!edge) {
-                T *dst = xbuf + (int64_t)xs * xmax_elems;
-                for (int q = 0; q < nwin; ++q) {
-                    const int st = __ldg(plan + 2 + 2 * q), cnt = __ldg(plan + 3 + 2 * q);
-                    bulk_g2s(dst, a.x + row0 + st, (uint32_t)cnt * sizeof(T), full_x + xs, pn);
-                    dst += cnt;
+            const int64_t rem = (a.seg_count - wb + G - 1) / G;
+            const int nb = rem < 32 ? (int)rem : 32;
+            for (int i = 0; i < nb; ++i) {
+                const int64_t sg = __shfl_sync(0xffffffffu, sgl, i);
+                const int64_t val_base = __shfl_sync(0xffffffffu, Dl.val_base, i);
+                const int64_t scat_begin = __shfl_sync(0xffffffffu, Dl.scat_begin, i);
+                const int32_t off_begin = __shfl_sync(0xffffffffu, Dl.off_begin, i);
+                const int32_t nscat = __shfl_sync(0xffffffffu, Dl.nscat, i);
+                const int32_t flags = __shfl_sync(0xffffffffu, (int32_t)Dl.flags, i);
+                const int32_t nd = __shfl_sync(0xffffffffu, (int32_t)Dl.ndias, i);
+                const int32_t plan_begin = __shfl_sync(0xffffffffu, Dl.plan_begin, i);
+                const int64_t row0 = sg * a.mrows;
+                const bool edge = (flags & SEG_EDGE) != 0;
+                const int32_t *plan = a.plan + plan_begin;
+                const int nwin = __ldg(plan);
+                // x bytes of all windows (skipped for guarded edge segments)
+                uint32_t xbytes = 0;
+                if (!edge)
+                    for (int q0 = 0; q0 < nwin; q0 += 32) {
+                        uint32_t c = (q0 + lane < nwin) ? (uint32_t)__ldg(plan + 3 + 2 * (q0 + lane)) : 0u;
+#pragma unroll
+                        for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+                        xbytes += c * sizeof(T);
+                    }
+                if (lane == 0) {
+                    mbar_wait(empty_x + xs, xph ^ 1);
+                    PipeSeg &P = sseg[xs];
+                    P.row0 = row0;
+                    P.scat_begin = scat_begin;
+                    P.nscat = nscat;
+                    P.flags = flags;
+                    P.nd = nd;
+                    P.plan_begin = plan_begin;
+                    P.off_begin = off_begin;
+                    mbar_expect_tx(full_x + xs, xbytes);  // arrive (release: P visible) + tx
                 }
-            }
-            if (++xs == nx) {
-                xs = 0;
-                xph ^= 1;
-            }
-            const int nd = D.ndias;
-            for (int d0 = 0; d0 < nd; d0 += kch) {
-                const int nk = min(kch, nd - d0);
-                mbar_wait(empty_v + vs, vph ^ 1);
-                const uint32_t bytes = (uint32_t)nk * (uint32_t)a.mrows * sizeof(T);
-                mbar_expect_tx(full_v + vs, bytes);
-                bulk_g2s(vring + (int64_t)vs * chunk_elems, a.vals + D.val_base + (int64_t)d0 * a.mrows, bytes,
-                         full_v + vs, pf);
-                if (++vs == ns) {
-                    vs = 0;
-                    vph ^= 1;
+                __syncwarp();
+                if (!edge) {
+                    // lane q copies window q to its prefix offset in the slot
+                    int64_t base = 0;
+                    for (int q0 = 0; q0 < nwin; q0 += 32) {
+                        const int q = q0 + lane;
+                        const int st = q < nwin ? __ldg(plan + 2 + 2 * q) : 0;
+                        const int cnt = q < nwin ? __ldg(plan + 3 + 2 * q) : 0;
+                        int inc = cnt;  // inclusive scan of counts
+#pragma unroll
+                        for (int o = 1; o < 32; o <<= 1) {
+                            const int v = __shfl_up_sync(0xffffffffu, inc, o);
+                            if (lane >= o) inc += v;
+                        }
+                        if (q < nwin)
+                            bulk_g2s(xbuf + (int64_t)xs * xmax_elems + base + inc - cnt, a.x + row0 + st,
+                                     (uint32_t)cnt * sizeof(T), full_x + xs, pn);
+                        base += __shfl_sync(0xffffffffu, inc, 31);
+                    }
                 }
+                if (++xs == nx) {
+                    xs = 0;
+                    xph ^= 1;
+                }
+                if (lane == 0) {
+                    for (int d0 = 0; d0 < nd; d0 += kch) {
+                        const int nk = min(kch, nd - d0);
+                        mbar_wait(empty_v + vs, vph ^ 1);
+                        const uint32_t bytes = (uint32_t)nk * (uint32_t)a.mrows * sizeof(T);
+                        mbar_expect_tx(full_v + vs, bytes);
+                        bulk_g2s(vring + (int64_t)vs * chunk_elems, a.vals + val_base + (int64_t)d0 * a.mrows, bytes,
+                                 full_v + vs, pf);
+                        if (++vs == ns) {
+                            vs = 0;
+                            vph ^= 1;
+                        }
+                    }
+                }
+                vs = __shfl_sync(0xffffffffu, vs, 0);
+                vph = __shfl_sync(0xffffffffu, vph, 0);
             }
         }
         return;

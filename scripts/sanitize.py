@@ -1,0 +1,46 @@
+#!/usr/bin/env python
+"""Small runs of every kernel variant for compute-sanitizer (memcheck /
+racecheck / synccheck / initcheck). Checks parity too, so a silent race shows
+up either as a sanitizer report or as a parity failure.
+
+usage: compute-sanitizer --tool racecheck python scripts/sanitize.py
+"""
+import os
+import sys
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import gen  # noqa: E402
+from oracle import coo  # noqa: E402
+from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix  # noqa: E402
+
+
+def main():
+    torch.cuda.set_device(0)
+    cases = [("c1", gen.config1()), ("c3s", gen.config3(n=20)), ("band", gen.config4(n=120_000))]
+    bad = 0
+    for name, a in cases:
+        for dt in (np.float64, np.float32):
+            b = a.astype(dt)
+            x = np.random.default_rng(1).uniform(-1, 1, b.ncols).astype(dt)
+            y0 = np.random.default_rng(2).uniform(-1, 1, b.nrows).astype(dt)
+            yref, sc = coo.coo_spmv(b.nrows, b.ncols, b.row, b.col, b.val, x, -0.75, 0.5, y0)
+            for v in (1, 2, 3):
+                A = CRSDMatrix.from_coo(b.nrows, b.ncols, b.row, b.col, b.val, variant=v)
+                tdt = torch.float64 if dt == np.float64 else torch.float32
+                xd = torch.from_numpy(x).to("cuda", tdt)
+                yd = torch.from_numpy(y0).to("cuda", tdt)
+                A.spmv(xd, yd, -0.75, 0.5)
+                torch.cuda.synchronize()
+                err = coo.parity_error(yd.cpu().numpy(), yref, sc)
+                ok = err <= (1e-12 if dt == np.float64 else 1e-5)
+                bad += not ok
+                print(f"{name} {np.dtype(dt).name} variant {v}: parity {err:.2e} {'ok' if ok else 'FAIL'}", flush=True)
+    sys.exit(1 if bad else 0)
+
+
+if __name__ == "__main__":
+    main()
