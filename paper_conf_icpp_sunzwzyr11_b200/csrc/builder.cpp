@@ -599,14 +599,17 @@ int64_t make_plans(const HostCRSD &H, int64_t gap, std::vector<int32_t> &plan, s
         const int64_t nd = H.pat_ptr[p + 1] - H.pat_ptr[p];
         // clusters of offsets closer than `gap`: one x window each
         std::vector<std::pair<int64_t, int64_t>> win;  // (start, count) in elements, aligned
-        std::vector<int32_t> xoff(nd);
+        std::vector<int32_t> xoff(nd), xwin(nd);
         int64_t xbase = 0;
         for (int64_t d = 0; d < nd;) {
             int64_t e = d;
             while (e + 1 < nd && o[e + 1] - o[e] <= gap) ++e;
             const int64_t st = floordiv(o[d], al) * al;
             const int64_t en = (floordiv(m - 1 + o[e], al) + 1) * al;
-            for (int64_t q = d; q <= e; ++q) xoff[q] = (int32_t)(xbase + o[q] - st);
+            for (int64_t q = d; q <= e; ++q) {
+                xoff[q] = (int32_t)(xbase + o[q] - st);
+                xwin[q] = (int32_t)win.size();
+            }
             win.emplace_back(st, en - st);
             xbase += en - st;
             d = e + 1;
@@ -623,6 +626,7 @@ int64_t make_plans(const HostCRSD &H, int64_t gap, std::vector<int32_t> &plan, s
             plan.push_back((int32_t)w.second);
         }
         plan.insert(plan.end(), xoff.begin(), xoff.end());
+        plan.insert(plan.end(), xwin.begin(), xwin.end());
     }
     if (plan.empty()) plan.push_back(0);
     if (xmax_elems) *xmax_elems = xmx;

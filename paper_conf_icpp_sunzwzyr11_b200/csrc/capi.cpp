@@ -88,6 +88,30 @@ static void plan_layout(crsd_matrix_s *A) {
     make_segdescs(H, A->rpt, A->x_lo, A->x_hi, A->segdesc);
     // x windows: offsets closer than 64 elements share one staged window
     A->smem_bytes = make_plans(H, 64, A->plan, A->segdesc, &A->xmax_elems);
+    // TMA variant shape: smallest split of a segment into row slices whose
+    // staging (values + x windows) stays <= 40 KB, i.e. >= 5 CTAs per SM
+    A->tma_split = 1;
+    A->tma_smem = A->smem_bytes;
+    for (int split = 1; split <= 8; split *= 2) {
+        const int64_t rc = H.mrows / split;
+        if (H.mrows % split || rc % 32 || (rc * H.elem) % 16) break;
+        int64_t mx = 0;
+        for (const Instance &I : H.inst) {
+            const int64_t p = I.pattern;
+            // plan of pattern p: [nwin, bytes, (st, cnt) x nwin, ...]
+            const int32_t *pl = A->plan.data() + A->segdesc[I.first_seg].plan_begin;
+            int64_t el = H.ndias((int32_t)p) * rc;
+            for (int w = 0; w < pl[0]; ++w) el += pl[3 + 2 * w] - (H.mrows - rc);
+            mx = std::max(mx, el * H.elem);
+        }
+        A->tma_split = split;
+        A->tma_smem = mx;
+        if (mx <= 40 * 1024) break;
+    }
+    {
+        const int64_t rc = H.mrows / A->tma_split;
+        A->tma_q = rc >= 512 ? 4 : (rc >= 256 ? 2 : 1);
+    }
     A->list_interior.clear();
     A->list_boundary.clear();
     A->nedge = 0;
@@ -137,8 +161,8 @@ static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_
     }
     plan_layout(A);
     const int64_t smem_cap = 200 * 1024;
-    if (o.variant == CRSD_VARIANT_TMA && A->smem_bytes > smem_cap) {
-        const std::string msg = "TMA variant: staging needs " + std::to_string(A->smem_bytes) +
+    if (o.variant == CRSD_VARIANT_TMA && A->tma_smem > smem_cap) {
+        const std::string msg = "TMA variant: staging needs " + std::to_string(A->tma_smem) +
                                 " bytes of shared memory per CTA (> 200 KB); use CRSD_VARIANT_LDG";
         delete A;
         return fail(CRSD_ERR_UNSUPPORTED, msg);
@@ -206,6 +230,9 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
     a.pat_offs = (const int32_t *)A->d_offs;
     a.plan = (const int32_t *)A->d_plan;
     a.smem_bytes = (int32_t)A->smem_bytes;
+    a.tma_split = A->tma_split;
+    a.tma_q = A->tma_q;
+    a.tma_smem = A->tma_smem;
     a.pipe_xmax_elems = (int32_t)A->xmax_elems;
     {
         int64_t mx = 0;
@@ -234,7 +261,7 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
     if (n < 0)
         return fail(CRSD_ERR_CUDA, std::string("kernel launch (variant ") + std::to_string(a.variant) + ", grid " +
                                        std::to_string(a.seg_count) + ", block " + std::to_string(A->H.mrows / A->rpt) +
-                                       ", smem " + std::to_string(a.variant == VARIANT_TMA ? a.smem_bytes : 0) +
+                                       ", smem " + std::to_string(a.variant == VARIANT_TMA ? a.tma_smem : 0) +
                                        "): " + cudaGetErrorString((cudaError_t)(-n)));
     launches += n;
     return CRSD_OK;
@@ -485,7 +512,7 @@ crsd_status_t crsd_get_info(crsd_matrix_t A, crsd_info_t *I) {
     I->halo_hi_valid = A->halo_hi_valid;
     I->device_bytes = A->device_bytes;
     I->variant = A->variant;
-    I->smem_bytes = (int32_t)A->smem_bytes;
+    I->smem_bytes = (int32_t)(A->variant == VARIANT_TMA ? A->tma_smem : A->smem_bytes);
     // algorithmic bytes: stored slots + scatter
     // (value + row + col) + x once + y written (+ y read when beta != 0)
     const int64_t es = H.elem;

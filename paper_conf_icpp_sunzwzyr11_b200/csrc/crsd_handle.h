@@ -16,6 +16,8 @@ struct crsd_matrix_s {
     int variant = crsd::VARIANT_LDG;
     int64_t smem_bytes = 0;
     int64_t xmax_elems = 0;
+    int tma_split = 1, tma_q = 2;
+    int64_t tma_smem = 0;
     std::vector<int32_t> plan;
     int32_t last_launches = 0;
     int64_t device_bytes = 0;

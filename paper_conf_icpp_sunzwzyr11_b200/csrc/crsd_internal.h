@@ -50,6 +50,7 @@ enum : int32_t { VARIANT_AUTO = 0, VARIANT_LDG = 1, VARIANT_TMA = 2, VARIANT_PIP
 //        (start, count multiples of 16/sizeof(T) elements)
 //   then ndias x xoff: element offset in the smem x region of row 0's x for
 //        diagonal d (= window base + o_d - start)
+//   then ndias x window index of diagonal d
 
 static_assert(sizeof(SegDesc) == 32, "SegDesc must be 32 bytes");
 
@@ -138,6 +139,9 @@ struct SpmvArgs {
     int32_t smem_bytes;       // TMA variant: dynamic shared memory per CTA
     int32_t pipe_xmax_elems;  // PIPE variant: largest x staging of a pattern (elements)
     int32_t max_ndias;        // largest NDias over patterns
+    int32_t tma_split;        // TMA variant: CTAs per segment (each covers mrows/split rows)
+    int32_t tma_q;            // TMA variant: rows per thread
+    int64_t tma_smem;         // TMA variant: dynamic shared memory per CTA
     int32_t variant;          // VARIANT_LDG or VARIANT_TMA
     T alpha, beta;
 };

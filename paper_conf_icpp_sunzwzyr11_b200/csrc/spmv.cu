@@ -289,88 +289,115 @@ __device__ __forceinline__ uint64_t policy_evict_normal() {
     return p;
 }
 
-template <typename T>
-__global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a) {
-    constexpr int R = VecT<T>::R;
+// A CTA covers `rc` rows of one segment (rc = mrows / split): with split > 1
+// the segment's value block is fetched as one bulk copy per diagonal (its rc
+// consecutive values), so big segments (many diagonals) still leave several
+// CTAs resident per SM. Thread t owns rows t + q*(rc/Q), q < Q.
+template <typename T, int Q>
+__global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int split) {
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ uint64_t bar;
     const int t = threadIdx.x;
     const int T_ = blockDim.x;
-    const int64_t s = a.seg_list ? (int64_t)__ldg(a.seg_list + blockIdx.x) : a.seg_begin + blockIdx.x;
+    const int rc = a.mrows / split;  // rows of this CTA
+    const int64_t cta = a.seg_list ? (int64_t)blockIdx.x : (int64_t)blockIdx.x;
+    const int64_t w = cta / split;
+    const int h = (int)(cta - w * split);
+    const int64_t s = a.seg_list ? (int64_t)__ldg(a.seg_list + w) : a.seg_begin + w;
     const SegDesc D = a.segs[s];
-    const int64_t row0 = s * a.mrows;
+    const int64_t row0 = s * a.mrows + (int64_t)h * rc;
     const int nd = D.ndias;
     const int32_t *plan = a.plan + D.plan_begin;
     const int nwin = __ldg(plan);
     const bool edge = (D.flags & SEG_EDGE) != 0;
+    const int shrink = a.mrows - rc;  // each window is this much shorter than for a full segment
     T *vs = reinterpret_cast<T *>(smem);
-    T *xs = vs + (int64_t)nd * a.mrows;
-    const uint32_t vbytes = (uint32_t)nd * (uint32_t)a.mrows * sizeof(T);
+    T *xs = vs + (int64_t)nd * rc;
+    const uint32_t vbytes = (uint32_t)nd * (uint32_t)rc * sizeof(T);
     if (t == 0) {
         mbar_init(&bar, 1);
         mbar_fence_init();
     }
     __syncthreads();
-    if (t == 0) {
+    if (t < 32) {
+        // warp 0 issues the copies: window / diagonal q by lane q % 32
         uint32_t total = vbytes;
         if (!edge)
-            for (int w = 0; w < nwin; ++w) total += (uint32_t)__ldg(plan + 3 + 2 * w) * sizeof(T);
-        mbar_expect_tx(&bar, total);
-        if (vbytes) bulk_g2s(vs, a.vals + D.val_base, vbytes, &bar, policy_evict_first());
+            for (int q = 0; q < nwin; ++q) total += (uint32_t)(__ldg(plan + 3 + 2 * q) - shrink) * sizeof(T);
+        if (t == 0) mbar_expect_tx(&bar, total);
+        __syncwarp();
+        const uint64_t pf = policy_evict_first();
+        if (split == 1) {
+            if (t == 0 && vbytes) bulk_g2s(vs, a.vals + D.val_base, vbytes, &bar, pf);
+        } else {
+            for (int d = t; d < nd; d += 32)
+                bulk_g2s(vs + (int64_t)d * rc, a.vals + D.val_base + (int64_t)d * a.mrows + (int64_t)h * rc,
+                         (uint32_t)rc * sizeof(T), &bar, pf);
+        }
         if (!edge) {
             const uint64_t pn = policy_evict_normal();
-            T *dst = xs;
-            for (int w = 0; w < nwin; ++w) {
-                const int st = __ldg(plan + 2 + 2 * w), cnt = __ldg(plan + 3 + 2 * w);
-                bulk_g2s(dst, a.x + row0 + st, (uint32_t)cnt * sizeof(T), &bar, pn);
-                dst += cnt;
+            int64_t base = 0;
+            for (int q0 = 0; q0 < nwin; q0 += 32) {
+                const int q = q0 + t;
+                const int st = q < nwin ? __ldg(plan + 2 + 2 * q) : 0;
+                const int cnt = q < nwin ? __ldg(plan + 3 + 2 * q) - shrink : 0;
+                int inc = cnt;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const int v = __shfl_up_sync(0xffffffffu, inc, o);
+                    if (t >= o) inc += v;
+                }
+                if (q < nwin) bulk_g2s(xs + base + inc - cnt, a.x + row0 + st, (uint32_t)cnt * sizeof(T), &bar, pn);
+                base += __shfl_sync(0xffffffffu, inc, 31);
             }
         }
     }
-    T acc[R];
+    T acc[Q];
 #pragma unroll
-    for (int q = 0; q < R; ++q) acc[q] = T(0);
+    for (int q = 0; q < Q; ++q) acc[q] = T(0);
     const int32_t *xoff = plan + 2 + 2 * nwin;
+    const int32_t *xwin = xoff + nd;
     const int32_t *offs = a.pat_offs + D.off_begin;
     mbar_wait(&bar, 0);
     if (!edge) {
 #pragma unroll 4
         for (int d = 0; d < nd; ++d) {
-            const int xo = __ldg(xoff + d);
-            const T *vd = vs + d * a.mrows + t;
+            const int xo = __ldg(xoff + d) - __ldg(xwin + d) * shrink;
+            const T *vd = vs + d * rc + t;
             const T *xd = xs + xo + t;
 #pragma unroll
-            for (int q = 0; q < R; ++q) acc[q] = fma(vd[q * T_], xd[q * T_], acc[q]);
+            for (int q = 0; q < Q; ++q) acc[q] = fma(vd[q * T_], xd[q * T_], acc[q]);
         }
     } else {
         for (int d = 0; d < nd; ++d) {
             const int o = __ldg(offs + d);
-            const T *vd = vs + d * a.mrows + t;
+            const T *vd = vs + d * rc + t;
 #pragma unroll
-            for (int q = 0; q < R; ++q) {
+            for (int q = 0; q < Q; ++q) {
                 const int64_t idx = row0 + t + q * T_ + o;
                 const T xj = (idx >= a.x_lo && idx < a.x_hi) ? __ldg(a.x + idx) : T(0);
                 acc[q] = fma(vd[q * T_], xj, acc[q]);
             }
         }
     }
-    // scatter points: owner of local row l is thread l % T, slot l / T
+    // scatter points of this CTA's rows: owner of local row l (in the
+    // segment) is thread (l - h*rc) % T_, slot (l - h*rc) / T_
     if (D.nscat > 0) {
         const int32_t *sr = a.scat_row + D.scat_begin;
         for (int64_t e = 0; e < D.nscat; ++e) {
-            const int rr = __ldg(sr + e);
-            if (rr % T_ != t) continue;
+            const int rr = __ldg(sr + e) - h * rc;
+            if (rr < 0 || rr >= rc || rr % T_ != t) continue;
             const T v = __ldg(a.scat_val + D.scat_begin + e);
             const T xv = __ldg(a.x + __ldg(a.scat_col + D.scat_begin + e));
-            const int q = rr / T_;
+            const int qq = rr / T_;
 #pragma unroll
-            for (int j = 0; j < R; ++j)
-                if (q == j) acc[j] = fma(v, xv, acc[j]);
+            for (int j = 0; j < Q; ++j)
+                if (qq == j) acc[j] = fma(v, xv, acc[j]);
         }
     }
     const T al = a.alpha, be = a.beta;
 #pragma unroll
-    for (int q = 0; q < R; ++q) {
+    for (int q = 0; q < Q; ++q) {
         const int64_t r = row0 + t + q * T_;
         if (!edge || r < a.nrows) {
             T *yp = a.y + r;
@@ -634,8 +661,11 @@ static void pipe_shape(int mrows, int elem, int64_t xmax, int max_nd, int &per_s
         }
     }
     per_sm = env_int("CRSD_PIPE_PERSM", per_sm);
-    nx = env_int("CRSD_PIPE_NX", nx);
-    ns = env_int("CRSD_PIPE_NS", ns);
+    nx = std::max(2, env_int("CRSD_PIPE_NX", nx));
+    ns = std::max(2, env_int("CRSD_PIPE_NS", ns));
+    // overrides are clamped to the per-CTA opt-in limit
+    while (ns > 2 && pipe_smem(ns, nx, kch, mrows, elem, xmax) > 220 * 1024) --ns;
+    while (nx > 2 && pipe_smem(ns, nx, kch, mrows, elem, xmax) > 220 * 1024) --nx;
 }
 
 template <typename T>
@@ -647,16 +677,22 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
     if (grid > 0x7fffffff) grid = 0x7fffffff;
     cudaError_t e;
     if (a.variant == VARIANT_TMA) {
-        // opt in to the dynamic shared memory this matrix needs (grows only)
-        static int attr_bytes[2] = {0, 0};
-        auto kern = crsd_spmv_tma<T>;
-        int &cur = attr_bytes[sizeof(T) == 8];
-        if (a.smem_bytes > cur) {
-            e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, a.smem_bytes);
+        const int split = a.tma_split, q = a.tma_q;
+        const int rc = a.mrows / split;
+        const int thr = rc / q;
+        const int smem = (int)a.tma_smem;
+        static int attr_bytes[2][3] = {{0, 0, 0}, {0, 0, 0}};
+        const int qi = q == 1 ? 0 : (q == 2 ? 1 : 2);
+        int &cur = attr_bytes[sizeof(T) == 8][qi];
+        auto kern = q == 1 ? crsd_spmv_tma<T, 1> : (q == 2 ? crsd_spmv_tma<T, 2> : crsd_spmv_tma<T, 4>);
+        if (smem > cur) {
+            e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
             if (e != cudaSuccess) return -(10000 + (int)e);
-            cur = a.smem_bytes;
+            cur = smem;
         }
-        kern<<<(unsigned)grid, threads, a.smem_bytes, (cudaStream_t)stream>>>(a);
+        int64_t g = a.seg_count * split;
+        if (g > 0x7fffffff) g = 0x7fffffff;
+        kern<<<(unsigned)g, thr, smem, (cudaStream_t)stream>>>(a, split);
     } else if (a.variant == VARIANT_PIPE) {
         // ring of KCH-diagonal value chunks; depth chosen so two CTAs fit per SM
         constexpr int kch = 8;
