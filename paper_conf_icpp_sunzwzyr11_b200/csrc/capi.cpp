@@ -3,6 +3,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -92,7 +93,9 @@ static void plan_layout(crsd_matrix_s *A) {
     // staging (values + x windows) stays <= 40 KB, i.e. >= 5 CTAs per SM
     A->tma_split = 1;
     A->tma_smem = A->smem_bytes;
+    const int force_split = getenv("CRSD_TMA_SPLIT") ? atoi(getenv("CRSD_TMA_SPLIT")) : 0;
     for (int split = 1; split <= 8; split *= 2) {
+        if (force_split && split < force_split) continue;
         const int64_t rc = H.mrows / split;
         if (H.mrows % split || rc % 32 || (rc * H.elem) % 16) break;
         int64_t mx = 0;
@@ -106,11 +109,16 @@ static void plan_layout(crsd_matrix_s *A) {
         }
         A->tma_split = split;
         A->tma_smem = mx;
-        if (mx <= 40 * 1024) break;
+        if (mx <= 40 * 1024 || force_split) break;
     }
     {
+        // rows per thread: the vector width of the dtype (2 fp64, 4 fp32) as
+        // long as a CTA keeps >= 2 warps; CRSD_TMA_Q / CRSD_TMA_SPLIT override
         const int64_t rc = H.mrows / A->tma_split;
-        A->tma_q = rc >= 512 ? 4 : (rc >= 256 ? 2 : 1);
+        int q = A->rpt;
+        while (q > 1 && rc / q < 64) q /= 2;
+        if (const char *e = getenv("CRSD_TMA_Q")) q = atoi(e);
+        A->tma_q = q;
     }
     A->list_interior.clear();
     A->list_boundary.clear();

@@ -317,19 +317,17 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int sp
     if (t == 0) {
         mbar_init(&bar, 1);
         mbar_fence_init();
+        // plan[1] = values + x bytes of a full segment
+        const uint32_t xfull = (uint32_t)__ldg(plan + 1) - (uint32_t)nd * (uint32_t)a.mrows * sizeof(T);
+        const uint32_t xbytes = edge ? 0u : xfull - (uint32_t)(nwin * shrink) * sizeof(T);
+        mbar_expect_tx(&bar, vbytes + xbytes);
+        if (split == 1 && vbytes) bulk_g2s(vs, a.vals + D.val_base, vbytes, &bar, policy_evict_first());
     }
     __syncthreads();
     if (t < 32) {
-        // warp 0 issues the copies: window / diagonal q by lane q % 32
-        uint32_t total = vbytes;
-        if (!edge)
-            for (int q = 0; q < nwin; ++q) total += (uint32_t)(__ldg(plan + 3 + 2 * q) - shrink) * sizeof(T);
-        if (t == 0) mbar_expect_tx(&bar, total);
-        __syncwarp();
-        const uint64_t pf = policy_evict_first();
-        if (split == 1) {
-            if (t == 0 && vbytes) bulk_g2s(vs, a.vals + D.val_base, vbytes, &bar, pf);
-        } else {
+        // warp 0 issues the remaining copies, window / diagonal q by lane q % 32
+        if (split > 1) {
+            const uint64_t pf = policy_evict_first();
             for (int d = t; d < nd; d += 32)
                 bulk_g2s(vs + (int64_t)d * rc, a.vals + D.val_base + (int64_t)d * a.mrows + (int64_t)h * rc,
                          (uint32_t)rc * sizeof(T), &bar, pf);
@@ -362,7 +360,7 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int sp
     if (!edge) {
 #pragma unroll 4
         for (int d = 0; d < nd; ++d) {
-            const int xo = __ldg(xoff + d) - __ldg(xwin + d) * shrink;
+            const int xo = shrink ? __ldg(xoff + d) - __ldg(xwin + d) * shrink : __ldg(xoff + d);
             const T *vd = vs + d * rc + t;
             const T *xd = xs + xo + t;
 #pragma unroll

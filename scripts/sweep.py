@@ -19,7 +19,8 @@ import bench  # noqa: E402
 from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix  # noqa: E402
 
 PEAK = bench.measured_peaks()[0]
-SHAPES = [None, (2, 4, 4), (2, 2, 4), (2, 3, 3), (1, 4, 8), (1, 3, 10)]
+SHAPES = [None, (2, 4, 4), (2, 2, 4)]
+TMA = [None, ("Q", 1), ("Q", 2), ("Q", 4), ("SPLIT", 2), ("SPLIT", 4)]
 
 
 def time_it(A, x, y, steps=200, warm=10):
@@ -46,11 +47,13 @@ def main():
         tdt = torch.float64 if dt == "f64" else torch.float32
         x = torch.rand(a.ncols, dtype=tdt, device="cuda")
         y = torch.empty(a.nrows, dtype=tdt, device="cuda")
-        runs = [("ldg", 1, None), ("tma", 2, None)] + [("pipe", 3, sh) for sh in SHAPES]
+        runs = [("ldg", 1, None)] + [("tma", 2, t) for t in TMA] + [("pipe", 3, sh) for sh in SHAPES]
         for name, v, sh in runs:
-            for k in ("CRSD_PIPE_PERSM", "CRSD_PIPE_NX", "CRSD_PIPE_NS"):
+            for k in ("CRSD_PIPE_PERSM", "CRSD_PIPE_NX", "CRSD_PIPE_NS", "CRSD_TMA_Q", "CRSD_TMA_SPLIT"):
                 os.environ.pop(k, None)
-            if sh:
+            if sh and name == "tma":
+                os.environ["CRSD_TMA_" + sh[0]] = str(sh[1])
+            elif sh:
                 os.environ["CRSD_PIPE_PERSM"], os.environ["CRSD_PIPE_NX"], os.environ["CRSD_PIPE_NS"] = map(str, sh)
             try:
                 A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, mrows=mrows, variant=v)
