@@ -65,10 +65,11 @@ def workload(cfg: str, dtype: str, world: int = 1, rank: int = 0):
         rb, re = rank * n * n * n, (rank + 1) * n * n * n
         a = gen.stencil((n, n, nz), "7pt", values="random", seed=2, row_begin=rb, row_end=re)
         desc = f"C2: 3D 7-point FDM Laplacian 256^3 per GPU (grid 256x256x{nz}, {N:,} rows), {dtype}"
-    elif cfg == "c3":
+    elif cfg in ("c3", "c3ns"):
         if world != 1:
             raise SystemExit("config c3 is a single-GPU workload")
-        a = gen.config3()
+        # c3ns: the same matrix without its scatter points (diagnostic only)
+        a = gen.config3(scatter_frac=0.001 if cfg == "c3" else 0.0)
         N, rb, re = a.nrows, 0, a.nrows
         desc = f"C3: 3D 27-point FVM stencil 192^3 with idle sub-blocks and 0.1% scatter points ({N:,} rows), {dtype}"
     elif cfg == "c4":
@@ -463,7 +464,7 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=500)
     ap.add_argument("--warmup", type=int, default=20)
-    ap.add_argument("--config", default="c2", choices=["c2", "c3", "c4"])
+    ap.add_argument("--config", default="c2", choices=["c2", "c3", "c3ns", "c4"])
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
     ap.add_argument("--mrows", type=int, default=0)
     ap.add_argument("--variant", default="auto", choices=["auto", "ldg", "tma", "pipe"])

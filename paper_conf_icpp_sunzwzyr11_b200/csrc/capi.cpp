@@ -175,22 +175,18 @@ static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_
         delete A;
         return fail(CRSD_ERR_UNSUPPORTED, msg);
     }
-    // PIPE needs two x slots of the largest pattern's windows plus >= 2 ring stages
-    const int64_t pipe_need = 2 * A->xmax_elems * A->H.elem + 2 * 8 * (int64_t)A->H.mrows * A->H.elem + 1024;
+    // PIPE double-buffers the TMA variant's per-CTA staging
+    const int64_t pipe_need = 2 * A->tma_smem + 1024;
     if (o.variant == CRSD_VARIANT_PIPE && pipe_need > smem_cap) {
-        const std::string msg = "PIPE variant: x staging needs " + std::to_string(pipe_need) +
+        const std::string msg = "PIPE variant: double-buffered staging needs " + std::to_string(pipe_need) +
                                 " bytes of shared memory per CTA (> 200 KB); use CRSD_VARIANT_LDG";
         delete A;
         return fail(CRSD_ERR_UNSUPPORTED, msg);
     }
-    if (o.variant == CRSD_VARIANT_PIPE && A->H.mrows > 512) {
-        delete A;
-        return fail(CRSD_ERR_UNSUPPORTED, "PIPE variant runs one row per thread: mrows must be <= 512");
-    }
     if (o.variant == CRSD_VARIANT_LDG) A->variant = VARIANT_LDG;
     else if (o.variant == CRSD_VARIANT_TMA) A->variant = VARIANT_TMA;
     else if (o.variant == CRSD_VARIANT_PIPE) A->variant = VARIANT_PIPE;
-    else A->variant = (pipe_need <= smem_cap && A->H.mrows <= 512) ? VARIANT_PIPE : VARIANT_LDG;
+    else A->variant = (A->tma_smem <= smem_cap) ? VARIANT_TMA : VARIANT_LDG;
     if (!A->host_only) {
         if (A->H.mrows / A->rpt > 256) {
             delete A;

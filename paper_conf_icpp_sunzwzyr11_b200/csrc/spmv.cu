@@ -289,6 +289,8 @@ __device__ __forceinline__ uint64_t policy_evict_normal() {
     return p;
 }
 
+constexpr int SCAT_STAGE = 128;
+
 // A CTA covers `rc` rows of one segment (rc = mrows / split): with split > 1
 // the segment's value block is fetched as one bulk copy per diagonal (its rc
 // consecutive values), so big segments (many diagonals) still leave several
@@ -350,6 +352,22 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int sp
             }
         }
     }
+    // Scatter points of this CTA's rows are gathered now, while the bulk
+    // copies are in flight: thread e loads entry e (value, x[col], owner), so
+    // the random x reads overlap the TMA wait instead of ending the CTA.
+    __shared__ T sc_v[SCAT_STAGE], sc_x[SCAT_STAGE];
+    __shared__ int32_t sc_own[SCAT_STAGE];
+    const int nst = D.nscat < SCAT_STAGE ? D.nscat : SCAT_STAGE;
+    if (t < nst) {
+        const int rr = __ldg(a.scat_row + D.scat_begin + t) - h * rc;
+        int own = -1;
+        if (rr >= 0 && rr < rc) own = (rr % T_) * Q + rr / T_;  // (thread, slot)
+        sc_own[t] = own;
+        if (own >= 0) {
+            sc_v[t] = __ldg(a.scat_val + D.scat_begin + t);
+            sc_x[t] = __ldg(a.x + __ldg(a.scat_col + D.scat_begin + t));
+        }
+    }
     T acc[Q];
 #pragma unroll
     for (int q = 0; q < Q; ++q) acc[q] = T(0);
@@ -378,11 +396,19 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int sp
             }
         }
     }
-    // scatter points of this CTA's rows: owner of local row l (in the
-    // segment) is thread (l - h*rc) % T_, slot (l - h*rc) / T_
+    // scatter points in (row, col) order: staged ones from shared memory,
+    // any beyond SCAT_STAGE from global memory
     if (D.nscat > 0) {
+        __syncthreads();
+        for (int e = 0; e < nst; ++e) {
+            const int own = sc_own[e];
+            if (own < 0 || own / Q != t) continue;
+#pragma unroll
+            for (int j = 0; j < Q; ++j)
+                if (own - t * Q == j) acc[j] = fma(sc_v[e], sc_x[e], acc[j]);
+        }
         const int32_t *sr = a.scat_row + D.scat_begin;
-        for (int64_t e = 0; e < D.nscat; ++e) {
+        for (int64_t e = nst; e < D.nscat; ++e) {
             const int rr = __ldg(sr + e) - h * rc;
             if (rr < 0 || rr >= rc || rr % T_ != t) continue;
             const T v = __ldg(a.scat_val + D.scat_begin + e);
@@ -406,264 +432,211 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int sp
 }
 
 // ---------------------------------------------------------------------------
-// Persistent, warp-specialised TMA pipeline (variant PIPE). Warp 0 (one
-// elected lane) is the producer: for each segment of this CTA it stages the
-// segment descriptor and the pattern's x windows into one of two x slots,
-// then streams the segment's value block in chunks of up to KCH diagonals
-// through a ring of NS shared-memory stages (cp.async.bulk + mbarrier
-// complete_tx). The consumer warps (mrows/RPT threads) compute from shared
-// memory and release stages through "empty" mbarriers. Bytes in flight are
-// set by the ring depth, not by the segment size, and the descriptor and
-// window fetches of the next segment overlap the current one.
+// Persistent, double-buffered TMA variant (PIPE). Each CTA walks work items
+// i = blockIdx.x, +gridDim.x, ... (item = one row slice of one segment, as in
+// crsd_spmv_tma) with two shared-memory slots: while it computes item i from
+// one slot, the bulk copies of item i + G are already landing in the other,
+// and thread 0 has the descriptor of the item after that in registers. The
+// scatter points of the next item are gathered (value, x[col]) into a
+// double-buffered staging area while the current item computes. This keeps
+// segment-descriptor latency and scatter gathers off the critical path that
+// bounds the one-shot variant (CTA launch -> descriptor -> copies -> wait).
 // ---------------------------------------------------------------------------
-struct PipeSeg {  // segment info handed from producer to consumers (per x slot)
+struct SlotInfo {
     int64_t row0;
     int64_t scat_begin;
-    int32_t nscat;
-    int32_t flags;
-    int32_t nd;
-    int32_t plan_begin;
-    int32_t off_begin;
-    int32_t pad;
+    int32_t nscat, flags, nd, plan_begin, off_begin, h;
 };
 
-__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
-    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+__device__ __forceinline__ void fence_proxy_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
-template <typename T, int KCH>
-__global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, int ns, int nx, int xmax_elems) {
-    constexpr int kch = KCH;
+template <typename T, int Q>
+__global__ void __launch_bounds__(256) crsd_spmv_tmap(const SpmvArgs<T> a, int split, int slot_elems) {
     extern __shared__ __align__(128) unsigned char smem[];
-    // layout: [bars: 2*nx + 2*ns][PipeSeg x nx][xbuf x nx][vring x ns]
-    uint64_t *full_x = reinterpret_cast<uint64_t *>(smem);
-    uint64_t *empty_x = full_x + nx;
-    uint64_t *full_v = full_x + 2 * nx;
-    uint64_t *empty_v = full_v + ns;
-    PipeSeg *sseg = reinterpret_cast<PipeSeg *>(smem + ((8 * (2 * nx + 2 * ns) + 127) / 128) * 128);
-    T *xbuf = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sseg) + ((nx * sizeof(PipeSeg) + 127) / 128) * 128);
-    T *vring = xbuf + nx * (int64_t)xmax_elems;
-    const int C = a.mrows;  // consumer threads (one row each)
-    const int nwarps_c = C / 32;
-    const int64_t chunk_elems = (int64_t)kch * a.mrows;
+    __shared__ uint64_t bar[2];
+    __shared__ SlotInfo info[2];
+    __shared__ T sc_v[2][SCAT_STAGE], sc_x[2][SCAT_STAGE];
+    __shared__ int32_t sc_own[2][SCAT_STAGE];
+    const int t = threadIdx.x;
+    const int T_ = blockDim.x;
+    const int rc = a.mrows / split;
+    const int shrink = a.mrows - rc;
+    const int64_t nitems = a.seg_count * split;
+    const int64_t G = gridDim.x;
+    T *slot0 = reinterpret_cast<T *>(smem);
 
-    if (threadIdx.x == 0) {
-        for (int i = 0; i < nx; ++i) {
-            mbar_init(full_x + i, 1);
-            mbar_init(empty_x + i, nwarps_c);
+    auto seg_of = [&](int64_t item, int &h) {
+        const int64_t w = item / split;
+        h = (int)(item - w * split);
+        return a.seg_list ? (int64_t)__ldg(a.seg_list + w) : a.seg_begin + w;
+    };
+    // thread 0: publish item info in slot sl and issue its bulk copies
+    auto issue = [&](int sl, int64_t sg, int h, const SegDesc &D) {
+        SlotInfo &I = info[sl];
+        I.row0 = sg * a.mrows + (int64_t)h * rc;
+        I.scat_begin = D.scat_begin;
+        I.nscat = D.nscat;
+        I.flags = D.flags;
+        I.nd = D.ndias;
+        I.plan_begin = D.plan_begin;
+        I.off_begin = D.off_begin;
+        I.h = h;
+        const int32_t *plan = a.plan + D.plan_begin;
+        const int nwin = __ldg(plan);
+        const bool edge = (D.flags & SEG_EDGE) != 0;
+        const int nd = D.ndias;
+        const uint32_t vbytes = (uint32_t)nd * (uint32_t)rc * sizeof(T);
+        const uint32_t xfull = (uint32_t)__ldg(plan + 1) - (uint32_t)nd * (uint32_t)a.mrows * sizeof(T);
+        const uint32_t xbytes = edge ? 0u : xfull - (uint32_t)(nwin * shrink) * sizeof(T);
+        T *vs = slot0 + (int64_t)sl * slot_elems;
+        T *xs = vs + (int64_t)nd * rc;
+        mbar_expect_tx(bar + sl, vbytes + xbytes);  // arrive (release: info visible)
+        const uint64_t pf = policy_evict_first();
+        if (split == 1) {
+            if (vbytes) bulk_g2s(vs, a.vals + D.val_base, vbytes, bar + sl, pf);
+        } else {
+            for (int d = 0; d < nd; ++d)
+                bulk_g2s(vs + (int64_t)d * rc, a.vals + D.val_base + (int64_t)d * a.mrows + (int64_t)h * rc,
+                         (uint32_t)rc * sizeof(T), bar + sl, pf);
         }
-        for (int i = 0; i < ns; ++i) {
-            mbar_init(full_v + i, 1);
-            mbar_init(empty_v + i, nwarps_c);
+        if (!edge) {
+            const uint64_t pn = policy_evict_normal();
+            T *dst = xs;
+            for (int q = 0; q < nwin; ++q) {
+                const int st = __ldg(plan + 2 + 2 * q), cnt = __ldg(plan + 3 + 2 * q) - shrink;
+                bulk_g2s(dst, a.x + I.row0 + st, (uint32_t)cnt * sizeof(T), bar + sl, pn);
+                dst += cnt;
+            }
         }
+    };
+    // all threads: gather the scatter points of the item in slot sl
+    auto gather = [&](int sl) {
+        const SlotInfo &I = info[sl];
+        const int nst = I.nscat < SCAT_STAGE ? I.nscat : SCAT_STAGE;
+        for (int e = t; e < nst; e += T_) {
+            const int rr = __ldg(a.scat_row + I.scat_begin + e) - I.h * rc;
+            int own = -1;
+            if (rr >= 0 && rr < rc) own = (rr % T_) * Q + rr / T_;
+            sc_own[sl][e] = own;
+            if (own >= 0) {
+                sc_v[sl][e] = __ldg(a.scat_val + I.scat_begin + e);
+                sc_x[sl][e] = __ldg(a.x + __ldg(a.scat_col + I.scat_begin + e));
+            }
+        }
+    };
+
+    SegDesc Dn;
+    int64_t sn = 0;
+    int hn = 0;
+    if (t == 0) {
+        mbar_init(bar, 1);
+        mbar_init(bar + 1, 1);
         mbar_fence_init();
+        int h;
+        for (int k = 0; k < 2; ++k) {
+            const int64_t it = blockIdx.x + k * G;
+            if (it < nitems) {
+                const int64_t sg = seg_of(it, h);
+                const SegDesc D = a.segs[sg];
+                issue(k, sg, h, D);
+            }
+        }
+        if (blockIdx.x + 2 * G < nitems) {
+            sn = seg_of(blockIdx.x + 2 * G, hn);
+            Dn = a.segs[sn];
+        }
     }
     __syncthreads();
+    if (blockIdx.x < nitems) gather(0);
+    __syncthreads();
 
-    if (threadIdx.x < 32) {
-        // ------------------------------ producer ------------------------------
-        // The whole warp fetches descriptors 32 segments at a time (one
-        // global-memory latency per 32 segments), window plans one window per
-        // lane, and issues the x-window bulk copies in parallel; lane 0 owns the
-        // ring bookkeeping and the value-chunk copies.
-        const int lane = threadIdx.x;
-        const uint64_t pf = policy_evict_first(), pn = policy_evict_normal();
-        int xs = 0, vs = 0;
-        uint32_t xph = 0, vph = 0;
-        const int64_t G = gridDim.x;
-        for (int64_t wb = blockIdx.x; wb < a.seg_count; wb += 32 * G) {
-            const int64_t wl = wb + lane * G;
-            int64_t sgl = 0;
-            SegDesc Dl = {};
-            if (wl < a.seg_count) {
-                sgl = a.seg_list ? (int64_t)__ldg(a.seg_list + wl) : a.seg_begin + wl;
-                Dl = a.segs[sgl];
-            }
-            const int64_t rem = (a.seg_count - wb + G - 1) / G;
-            const int nb = rem < 32 ? (int)rem : 32;
-            for (int i = 0; i < nb; ++i) {
-                const int64_t sg = __shfl_sync(0xffffffffu, sgl, i);
-                const int64_t val_base = __shfl_sync(0xffffffffu, Dl.val_base, i);
-                const int64_t scat_begin = __shfl_sync(0xffffffffu, Dl.scat_begin, i);
-                const int32_t off_begin = __shfl_sync(0xffffffffu, Dl.off_begin, i);
-                const int32_t nscat = __shfl_sync(0xffffffffu, Dl.nscat, i);
-                const int32_t flags = __shfl_sync(0xffffffffu, (int32_t)Dl.flags, i);
-                const int32_t nd = __shfl_sync(0xffffffffu, (int32_t)Dl.ndias, i);
-                const int32_t plan_begin = __shfl_sync(0xffffffffu, Dl.plan_begin, i);
-                const int64_t row0 = sg * a.mrows;
-                const bool edge = (flags & SEG_EDGE) != 0;
-                const int32_t *plan = a.plan + plan_begin;
-                const int nwin = __ldg(plan);
-                // x bytes of all windows (skipped for guarded edge segments)
-                uint32_t xbytes = 0;
-                if (!edge)
-                    for (int q0 = 0; q0 < nwin; q0 += 32) {
-                        uint32_t c = (q0 + lane < nwin) ? (uint32_t)__ldg(plan + 3 + 2 * (q0 + lane)) : 0u;
-#pragma unroll
-                        for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
-                        xbytes += c * sizeof(T);
-                    }
-                if (lane == 0) {
-                    mbar_wait(empty_x + xs, xph ^ 1);
-                    PipeSeg &P = sseg[xs];
-                    P.row0 = row0;
-                    P.scat_begin = scat_begin;
-                    P.nscat = nscat;
-                    P.flags = flags;
-                    P.nd = nd;
-                    P.plan_begin = plan_begin;
-                    P.off_begin = off_begin;
-                    mbar_expect_tx(full_x + xs, xbytes);  // arrive (release: P visible) + tx
-                }
-                __syncwarp();
-                if (!edge) {
-                    // lane q copies window q to its prefix offset in the slot
-                    int64_t base = 0;
-                    for (int q0 = 0; q0 < nwin; q0 += 32) {
-                        const int q = q0 + lane;
-                        const int st = q < nwin ? __ldg(plan + 2 + 2 * q) : 0;
-                        const int cnt = q < nwin ? __ldg(plan + 3 + 2 * q) : 0;
-                        int inc = cnt;  // inclusive scan of counts
-#pragma unroll
-                        for (int o = 1; o < 32; o <<= 1) {
-                            const int v = __shfl_up_sync(0xffffffffu, inc, o);
-                            if (lane >= o) inc += v;
-                        }
-                        if (q < nwin)
-                            bulk_g2s(xbuf + (int64_t)xs * xmax_elems + base + inc - cnt, a.x + row0 + st,
-                                     (uint32_t)cnt * sizeof(T), full_x + xs, pn);
-                        base += __shfl_sync(0xffffffffu, inc, 31);
-                    }
-                }
-                if (++xs == nx) {
-                    xs = 0;
-                    xph ^= 1;
-                }
-                if (lane == 0) {
-                    for (int d0 = 0; d0 < nd; d0 += kch) {
-                        const int nk = min(kch, nd - d0);
-                        mbar_wait(empty_v + vs, vph ^ 1);
-                        const uint32_t bytes = (uint32_t)nk * (uint32_t)a.mrows * sizeof(T);
-                        mbar_expect_tx(full_v + vs, bytes);
-                        bulk_g2s(vring + (int64_t)vs * chunk_elems, a.vals + val_base + (int64_t)d0 * a.mrows, bytes,
-                                 full_v + vs, pf);
-                        if (++vs == ns) {
-                            vs = 0;
-                            vph ^= 1;
-                        }
-                    }
-                }
-                vs = __shfl_sync(0xffffffffu, vs, 0);
-                vph = __shfl_sync(0xffffffffu, vph, 0);
-            }
-        }
-        return;
-    }
-    // ------------------------------ consumers ------------------------------
-    // one row per consumer thread: row0 + ct (conflict-free shared reads)
-    const int ct = threadIdx.x - 32;
-    const int lane = ct & 31;
-    int xs = 0, vs = 0;
-    uint32_t xph = 0, vph = 0;
     const T al = a.alpha, be = a.beta;
-    for (int64_t w = blockIdx.x; w < a.seg_count; w += gridDim.x) {
-        mbar_wait(full_x + xs, xph);
-        const PipeSeg P = sseg[xs];
-        const bool edge = (P.flags & SEG_EDGE) != 0;
-        const int32_t *plan = a.plan + P.plan_begin;
+    uint32_t ph0 = 0, ph1 = 0;
+    int k = 0;
+    for (int64_t it = blockIdx.x; it < nitems; it += G, ++k) {
+        const int sl = k & 1;
+        if (it + G < nitems) gather(sl ^ 1);  // next item's scatter points
+        mbar_wait(bar + sl, sl ? ph1 : ph0);
+        if (sl) ph1 ^= 1; else ph0 ^= 1;
+        const SlotInfo I = info[sl];
+        const bool edge = (I.flags & SEG_EDGE) != 0;
+        const int32_t *plan = a.plan + I.plan_begin;
         const int nwin = __ldg(plan);
         const int32_t *xoff = plan + 2 + 2 * nwin;
-        const int32_t *offs = a.pat_offs + P.off_begin;
-        const T *xb = xbuf + (int64_t)xs * xmax_elems + ct;
-        const int64_t row = P.row0 + ct;
-        T acc = T(0);
-        for (int d0 = 0; d0 < P.nd; d0 += kch) {
-            const int nk = min(kch, P.nd - d0);
-            mbar_wait(full_v + vs, vph);
-            const T *vb = vring + (int64_t)vs * chunk_elems + ct;
-            if (!edge) {
-                int xo[KCH];
+        const int32_t *xwin = xoff + I.nd;
+        const int32_t *offs = a.pat_offs + I.off_begin;
+        const T *vs = slot0 + (int64_t)sl * slot_elems;
+        const T *xs = vs + (int64_t)I.nd * rc;
+        T acc[Q];
 #pragma unroll
-                for (int k = 0; k < KCH; ++k)
-                    if (k < nk) xo[k] = __ldg(xoff + d0 + k);
+        for (int q = 0; q < Q; ++q) acc[q] = T(0);
+        if (!edge) {
+#pragma unroll 4
+            for (int d = 0; d < I.nd; ++d) {
+                const int xo = shrink ? __ldg(xoff + d) - __ldg(xwin + d) * shrink : __ldg(xoff + d);
+                const T *vd = vs + d * rc + t;
+                const T *xd = xs + xo + t;
 #pragma unroll
-                for (int k = 0; k < KCH; ++k)
-                    if (k < nk) acc = fma(vb[k * C], xb[xo[k]], acc);
-            } else {
-                for (int k = 0; k < nk; ++k) {
-                    const int64_t idx = row + __ldg(offs + d0 + k);
+                for (int q = 0; q < Q; ++q) acc[q] = fma(vd[q * T_], xd[q * T_], acc[q]);
+            }
+        } else {
+            for (int d = 0; d < I.nd; ++d) {
+                const int o = __ldg(offs + d);
+                const T *vd = vs + d * rc + t;
+#pragma unroll
+                for (int q = 0; q < Q; ++q) {
+                    const int64_t idx = I.row0 + t + q * T_ + o;
                     const T xj = (idx >= a.x_lo && idx < a.x_hi) ? __ldg(a.x + idx) : T(0);
-                    acc = fma(vb[k * C], xj, acc);
+                    acc[q] = fma(vd[q * T_], xj, acc[q]);
                 }
             }
-            __syncwarp();
-            if (lane == 0) mbar_arrive(empty_v + vs);
-            if (++vs == ns) {
-                vs = 0;
-                vph ^= 1;
+        }
+        if (I.nscat > 0) {
+            const int nst = I.nscat < SCAT_STAGE ? I.nscat : SCAT_STAGE;
+            for (int e = 0; e < nst; ++e) {
+                const int own = sc_own[sl][e];
+                if (own < 0 || own / Q != t) continue;
+#pragma unroll
+                for (int j = 0; j < Q; ++j)
+                    if (own - t * Q == j) acc[j] = fma(sc_v[sl][e], sc_x[sl][e], acc[j]);
+            }
+            for (int64_t e = nst; e < I.nscat; ++e) {
+                const int rr = __ldg(a.scat_row + I.scat_begin + e) - I.h * rc;
+                if (rr < 0 || rr >= rc || rr % T_ != t) continue;
+                const T v = __ldg(a.scat_val + I.scat_begin + e);
+                const T xv = __ldg(a.x + __ldg(a.scat_col + I.scat_begin + e));
+                const int qq = rr / T_;
+#pragma unroll
+                for (int j = 0; j < Q; ++j)
+                    if (qq == j) acc[j] = fma(v, xv, acc[j]);
             }
         }
-        // scatter points of this row, (row, col) order
-        if (P.nscat > 0) {
-            const int32_t *sr = a.scat_row + P.scat_begin;
-            for (int64_t e = 0; e < P.nscat; ++e) {
-                if (__ldg(sr + e) != ct) continue;
-                acc = fma(__ldg(a.scat_val + P.scat_begin + e), __ldg(a.x + __ldg(a.scat_col + P.scat_begin + e)), acc);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) {
+            const int64_t r = I.row0 + t + q * T_;
+            if (!edge || r < a.nrows) {
+                T *yp = a.y + r;
+                __stcs(yp, (be != T(0)) ? fma(al, acc[q], be * *yp) : al * acc[q]);
             }
         }
-        __syncwarp();
-        if (lane == 0) mbar_arrive(empty_x + xs);
-        if (!edge || row < a.nrows) {
-            T *yp = a.y + row;
-            __stcs(yp, (be != T(0)) ? fma(al, acc, be * *yp) : al * acc);
+        __syncthreads();  // slot sl, info[sl], staging[sl] free; staging[sl^1] written
+        if (t == 0 && it + 2 * G < nitems) {
+            fence_proxy_async_smem();
+            issue(sl, sn, hn, Dn);
+            if (it + 3 * G < nitems) {
+                sn = seg_of(it + 3 * G, hn);
+                Dn = a.segs[sn];
+            }
         }
-        if (++xs == nx) {
-            xs = 0;
-            xph ^= 1;
-        }
+        __syncthreads();  // info[sl] of item it + 2G visible for the next gather
     }
-}
-
-// shared memory of the PIPE variant for nx x slots and ns value stages
-inline int64_t pipe_smem(int ns, int nx, int kch, int mrows, int elem, int64_t xmax_elems) {
-    const int64_t bars = ((8 * (2 * nx + 2 * ns) + 127) / 128) * 128;
-    const int64_t segs = ((nx * (int64_t)sizeof(PipeSeg) + 127) / 128) * 128;
-    return bars + segs + nx * xmax_elems * elem + (int64_t)ns * kch * mrows * elem;
 }
 
 static int env_int(const char *k, int d) {
     const char *v = getenv(k);
     return v ? atoi(v) : d;
-}
-
-// Pipeline shape: CTAs per SM, x slots (segments the producer may run ahead,
-// plus one) and value stages. Maximises the segments in flight per SM,
-// CTAs/SM x min(nx - 1, ns / chunks), under the shared-memory budget.
-// CRSD_PIPE_PERSM / _NX / _NS override (tuning experiments).
-static void pipe_shape(int mrows, int elem, int64_t xmax, int max_nd, int &per_sm, int &nx, int &ns) {
-    constexpr int kch = 8;
-    const int chunks = max_nd > 0 ? (max_nd + kch - 1) / kch : 1;
-    double best = -1.0;
-    per_sm = 1; nx = 2; ns = 2;
-    for (int ps = (mrows <= 256 ? 2 : 1); ps >= 1; --ps) {
-        const int64_t budget = (ps == 2 ? 110 : 220) * 1024;
-        for (int x = 2; x <= 8; ++x) {
-            int n = 0;
-            while (n < 32 && pipe_smem(n + 1, x, kch, mrows, elem, xmax) <= budget) ++n;
-            if (n < 2) continue;
-            const double sc = ps * std::min<double>(x - 1, (double)n / chunks) + 1e-3 * ps;
-            if (sc > best) {
-                best = sc;
-                per_sm = ps; nx = x; ns = n;
-            }
-        }
-    }
-    per_sm = env_int("CRSD_PIPE_PERSM", per_sm);
-    nx = std::max(2, env_int("CRSD_PIPE_NX", nx));
-    ns = std::max(2, env_int("CRSD_PIPE_NS", ns));
-    // overrides are clamped to the per-CTA opt-in limit
-    while (ns > 2 && pipe_smem(ns, nx, kch, mrows, elem, xmax) > 220 * 1024) --ns;
-    while (nx > 2 && pipe_smem(ns, nx, kch, mrows, elem, xmax) > 220 * 1024) --nx;
 }
 
 template <typename T>
@@ -692,22 +665,28 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
         if (g > 0x7fffffff) g = 0x7fffffff;
         kern<<<(unsigned)g, thr, smem, (cudaStream_t)stream>>>(a, split);
     } else if (a.variant == VARIANT_PIPE) {
-        // ring of KCH-diagonal value chunks; depth chosen so two CTAs fit per SM
-        constexpr int kch = 8;
-        const int64_t xmax = a.pipe_xmax_elems;
-        int per_sm, nx, ns;
-        pipe_shape(a.mrows, sizeof(T), xmax, a.max_ndias, per_sm, nx, ns);
-        const int64_t sm = pipe_smem(ns, nx, kch, a.mrows, sizeof(T), xmax);
-        static int attr_pipe[2] = {0, 0};
-        int &cur = attr_pipe[sizeof(T) == 8];
-        if (sm > cur) {
-            e = cudaFuncSetAttribute(crsd_spmv_pipe<T, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+        const int split = a.tma_split, q = a.tma_q;
+        const int rc = a.mrows / split;
+        const int thr = rc / q;
+        const int slot_elems = (int)((a.tma_smem / sizeof(T) + 31) / 32 * 32);
+        const int smem = 2 * slot_elems * (int)sizeof(T);
+        static int attr_p[2][3] = {{0, 0, 0}, {0, 0, 0}};
+        const int qi = q == 1 ? 0 : (q == 2 ? 1 : 2);
+        int &cur = attr_p[sizeof(T) == 8][qi];
+        auto kern = q == 1 ? crsd_spmv_tmap<T, 1> : (q == 2 ? crsd_spmv_tmap<T, 2> : crsd_spmv_tmap<T, 4>);
+        if (smem > cur) {
+            e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
             if (e != cudaSuccess) return -(10000 + (int)e);
-            cur = (int)sm;
+            cur = smem;
         }
+        int per_sm = 0;
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, thr, smem);
+        if (e != cudaSuccess || per_sm < 1) per_sm = 1;
+        per_sm = env_int("CRSD_PIPE_PERSM", per_sm);
         int64_t g = (int64_t)sm_count * per_sm;
-        if (g > a.seg_count) g = a.seg_count;
-        crsd_spmv_pipe<T, kch><<<(unsigned)g, a.mrows + 32, sm, (cudaStream_t)stream>>>(a, ns, nx, (int)xmax);
+        const int64_t nitems = a.seg_count * split;
+        if (g > nitems) g = nitems;
+        kern<<<(unsigned)g, thr, smem, (cudaStream_t)stream>>>(a, split, slot_elems);
     } else {
         crsd_spmv_ldg<T, 4><<<(unsigned)grid, threads, 0, (cudaStream_t)stream>>>(a);
     }

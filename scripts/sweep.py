@@ -19,8 +19,10 @@ import bench  # noqa: E402
 from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix  # noqa: E402
 
 PEAK = bench.measured_peaks()[0]
-SHAPES = [None, (2, 4, 4), (2, 2, 4)]
-TMA = [None, ("Q", 1), ("Q", 2), ("Q", 4), ("SPLIT", 2), ("SPLIT", 4)]
+SHAPES = [s for s in os.environ.get("SWEEP_PIPE", "none").split(";") if s]
+SHAPES = [None if s == "none" else tuple(int(v) for v in s.split(",")) for s in SHAPES]
+TMA = [s for s in os.environ.get("SWEEP_TMA", "none").split(";") if s]
+TMA = [None if s == "none" else (s.split("=")[0], int(s.split("=")[1])) for s in TMA]
 
 
 def time_it(A, x, y, steps=200, warm=10):
@@ -47,11 +49,11 @@ def main():
         tdt = torch.float64 if dt == "f64" else torch.float32
         x = torch.rand(a.ncols, dtype=tdt, device="cuda")
         y = torch.empty(a.nrows, dtype=tdt, device="cuda")
-        runs = [("ldg", 1, None)] + [("tma", 2, t) for t in TMA] + [("pipe", 3, sh) for sh in SHAPES]
+        runs = [("ldg", 1, None)] + [("tma", 2, t) for t in TMA] + [("pipe", 3, t) for t in TMA]
         for name, v, sh in runs:
             for k in ("CRSD_PIPE_PERSM", "CRSD_PIPE_NX", "CRSD_PIPE_NS", "CRSD_TMA_Q", "CRSD_TMA_SPLIT"):
                 os.environ.pop(k, None)
-            if sh and name == "tma":
+            if sh and name in ("tma", "pipe"):
                 os.environ["CRSD_TMA_" + sh[0]] = str(sh[1])
             elif sh:
                 os.environ["CRSD_PIPE_PERSM"], os.environ["CRSD_PIPE_NX"], os.environ["CRSD_PIPE_NS"] = map(str, sh)
