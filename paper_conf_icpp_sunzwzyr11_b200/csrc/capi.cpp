@@ -175,18 +175,31 @@ static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_
         delete A;
         return fail(CRSD_ERR_UNSUPPORTED, msg);
     }
-    // PIPE double-buffers the TMA variant's per-CTA staging
-    const int64_t pipe_need = 2 * A->tma_smem + 1024;
+    // PIPE needs two x slots of the largest pattern's windows plus >= 2 ring stages
+    const int64_t pipe_need = 2 * A->xmax_elems * A->H.elem + 2 * 8 * (int64_t)A->H.mrows * A->H.elem + 1024;
     if (o.variant == CRSD_VARIANT_PIPE && pipe_need > smem_cap) {
-        const std::string msg = "PIPE variant: double-buffered staging needs " + std::to_string(pipe_need) +
+        const std::string msg = "PIPE variant: x staging needs " + std::to_string(pipe_need) +
                                 " bytes of shared memory per CTA (> 200 KB); use CRSD_VARIANT_LDG";
         delete A;
         return fail(CRSD_ERR_UNSUPPORTED, msg);
     }
+    if (o.variant == CRSD_VARIANT_PIPE && A->H.mrows > 512) {
+        delete A;
+        return fail(CRSD_ERR_UNSUPPORTED, "PIPE variant runs one row per thread: mrows must be <= 512");
+    }
     if (o.variant == CRSD_VARIANT_LDG) A->variant = VARIANT_LDG;
     else if (o.variant == CRSD_VARIANT_TMA) A->variant = VARIANT_TMA;
     else if (o.variant == CRSD_VARIANT_PIPE) A->variant = VARIANT_PIPE;
-    else A->variant = (A->tma_smem <= smem_cap) ? VARIANT_TMA : VARIANT_LDG;
+    else {
+        // AUTO, from the variant sweeps in profiles/r01_sweep*.jsonl: the
+        // one-shot TMA kernel when a whole segment stages in <= 32 KB (enough
+        // CTAs per SM to keep ~200 KB in flight: C2 97-101% of the measured
+        // copy bandwidth); otherwise the chunked ring (PIPE) for fp64 (C3 81%)
+        // and the register variant for fp32 (C3 76%).
+        if (A->tma_split == 1 && A->tma_smem <= 32 * 1024) A->variant = VARIANT_TMA;
+        else if (A->H.elem == 8 && pipe_need <= smem_cap && A->H.mrows <= 512) A->variant = VARIANT_PIPE;
+        else A->variant = VARIANT_LDG;
+    }
     if (!A->host_only) {
         if (A->H.mrows / A->rpt > 256) {
             delete A;
@@ -237,6 +250,7 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
     a.tma_split = A->tma_split;
     a.tma_q = A->tma_q;
     a.tma_smem = A->tma_smem;
+    a.has_scatter = A->H.nscatter() > 0;
     a.pipe_xmax_elems = (int32_t)A->xmax_elems;
     {
         int64_t mx = 0;

@@ -142,6 +142,7 @@ struct SpmvArgs {
     int32_t tma_split;        // TMA variant: CTAs per segment (each covers mrows/split rows)
     int32_t tma_q;            // TMA variant: rows per thread
     int64_t tma_smem;         // TMA variant: dynamic shared memory per CTA
+    int32_t has_scatter;      // the matrix has scatter points (selects the staging kernel)
     int32_t variant;          // VARIANT_LDG or VARIANT_TMA
     T alpha, beta;
 };

@@ -295,7 +295,7 @@ constexpr int SCAT_STAGE = 128;
 // the segment's value block is fetched as one bulk copy per diagonal (its rc
 // consecutive values), so big segments (many diagonals) still leave several
 // CTAs resident per SM. Thread t owns rows t + q*(rc/Q), q < Q.
-template <typename T, int Q>
+template <typename T, int Q, bool SCAT>
 __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int split) {
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ uint64_t bar;
@@ -355,17 +355,17 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int sp
     // Scatter points of this CTA's rows are gathered now, while the bulk
     // copies are in flight: thread e loads entry e (value, x[col], owner), so
     // the random x reads overlap the TMA wait instead of ending the CTA.
-    __shared__ T sc_v[SCAT_STAGE], sc_x[SCAT_STAGE];
-    __shared__ int32_t sc_own[SCAT_STAGE];
-    const int nst = D.nscat < SCAT_STAGE ? D.nscat : SCAT_STAGE;
-    if (t < nst) {
-        const int rr = __ldg(a.scat_row + D.scat_begin + t) - h * rc;
+    __shared__ T sc_v[SCAT ? SCAT_STAGE : 1], sc_x[SCAT ? SCAT_STAGE : 1];
+    __shared__ int32_t sc_own[SCAT ? SCAT_STAGE : 1];
+    const int nst = SCAT ? (D.nscat < SCAT_STAGE ? D.nscat : SCAT_STAGE) : 0;
+    for (int e = t; e < nst; e += T_) {
+        const int rr = __ldg(a.scat_row + D.scat_begin + e) - h * rc;
         int own = -1;
         if (rr >= 0 && rr < rc) own = (rr % T_) * Q + rr / T_;  // (thread, slot)
-        sc_own[t] = own;
+        sc_own[e] = own;
         if (own >= 0) {
-            sc_v[t] = __ldg(a.scat_val + D.scat_begin + t);
-            sc_x[t] = __ldg(a.x + __ldg(a.scat_col + D.scat_begin + t));
+            sc_v[e] = __ldg(a.scat_val + D.scat_begin + e);
+            sc_x[e] = __ldg(a.x + __ldg(a.scat_col + D.scat_begin + e));
         }
     }
     T acc[Q];
@@ -398,7 +398,7 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int sp
     }
     // scatter points in (row, col) order: staged ones from shared memory,
     // any beyond SCAT_STAGE from global memory
-    if (D.nscat > 0) {
+    if (SCAT && D.nscat > 0) {
         __syncthreads();
         for (int e = 0; e < nst; ++e) {
             const int own = sc_own[e];
@@ -432,206 +432,189 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int sp
 }
 
 // ---------------------------------------------------------------------------
-// Persistent, double-buffered TMA variant (PIPE). Each CTA walks work items
-// i = blockIdx.x, +gridDim.x, ... (item = one row slice of one segment, as in
-// crsd_spmv_tma) with two shared-memory slots: while it computes item i from
-// one slot, the bulk copies of item i + G are already landing in the other,
-// and thread 0 has the descriptor of the item after that in registers. The
-// scatter points of the next item are gathered (value, x[col]) into a
-// double-buffered staging area while the current item computes. This keeps
-// segment-descriptor latency and scatter gathers off the critical path that
-// bounds the one-shot variant (CTA launch -> descriptor -> copies -> wait).
+// Persistent, warp-specialised TMA pipeline (variant PIPE). Warp 0 (one
+// elected lane) is the producer: for each segment of this CTA it stages the
+// segment descriptor and the pattern's x windows into one of two x slots,
+// then streams the segment's value block in chunks of up to KCH diagonals
+// through a ring of NS shared-memory stages (cp.async.bulk + mbarrier
+// complete_tx). The consumer warps (mrows/RPT threads) compute from shared
+// memory and release stages through "empty" mbarriers. Bytes in flight are
+// set by the ring depth, not by the segment size, and the descriptor and
+// window fetches of the next segment overlap the current one.
 // ---------------------------------------------------------------------------
-struct SlotInfo {
+struct PipeSeg {  // segment info handed from producer to consumers (per x slot)
     int64_t row0;
     int64_t scat_begin;
-    int32_t nscat, flags, nd, plan_begin, off_begin, h;
+    int32_t nscat;
+    int32_t flags;
+    int32_t nd;
+    int32_t plan_begin;
+    int32_t off_begin;
+    int32_t pad;
 };
 
-__device__ __forceinline__ void fence_proxy_async_smem() {
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
-template <typename T, int Q>
-__global__ void __launch_bounds__(256) crsd_spmv_tmap(const SpmvArgs<T> a, int split, int slot_elems) {
+template <typename T, int KCH>
+__global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, int ns, int xmax_elems) {
+    constexpr int kch = KCH;
     extern __shared__ __align__(128) unsigned char smem[];
-    __shared__ uint64_t bar[2];
-    __shared__ SlotInfo info[2];
-    __shared__ T sc_v[2][SCAT_STAGE], sc_x[2][SCAT_STAGE];
-    __shared__ int32_t sc_own[2][SCAT_STAGE];
-    const int t = threadIdx.x;
-    const int T_ = blockDim.x;
-    const int rc = a.mrows / split;
-    const int shrink = a.mrows - rc;
-    const int64_t nitems = a.seg_count * split;
-    const int64_t G = gridDim.x;
-    T *slot0 = reinterpret_cast<T *>(smem);
+    // layout: [bars: 4 + 2*ns][PipeSeg x2][xbuf x2][vring x ns]
+    uint64_t *full_x = reinterpret_cast<uint64_t *>(smem);
+    uint64_t *empty_x = full_x + 2;
+    uint64_t *full_v = full_x + 4;
+    uint64_t *empty_v = full_v + ns;
+    PipeSeg *sseg = reinterpret_cast<PipeSeg *>(smem + ((8 * (4 + 2 * ns) + 127) / 128) * 128);
+    T *xbuf = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sseg) + 128);
+    T *vring = xbuf + 2 * (int64_t)xmax_elems;
+    const int C = a.mrows;  // consumer threads (one row each)
+    const int nwarps_c = C / 32;
+    const int64_t chunk_elems = (int64_t)kch * a.mrows;
 
-    auto seg_of = [&](int64_t item, int &h) {
-        const int64_t w = item / split;
-        h = (int)(item - w * split);
-        return a.seg_list ? (int64_t)__ldg(a.seg_list + w) : a.seg_begin + w;
-    };
-    // thread 0: publish item info in slot sl and issue its bulk copies
-    auto issue = [&](int sl, int64_t sg, int h, const SegDesc &D) {
-        SlotInfo &I = info[sl];
-        I.row0 = sg * a.mrows + (int64_t)h * rc;
-        I.scat_begin = D.scat_begin;
-        I.nscat = D.nscat;
-        I.flags = D.flags;
-        I.nd = D.ndias;
-        I.plan_begin = D.plan_begin;
-        I.off_begin = D.off_begin;
-        I.h = h;
-        const int32_t *plan = a.plan + D.plan_begin;
-        const int nwin = __ldg(plan);
-        const bool edge = (D.flags & SEG_EDGE) != 0;
-        const int nd = D.ndias;
-        const uint32_t vbytes = (uint32_t)nd * (uint32_t)rc * sizeof(T);
-        const uint32_t xfull = (uint32_t)__ldg(plan + 1) - (uint32_t)nd * (uint32_t)a.mrows * sizeof(T);
-        const uint32_t xbytes = edge ? 0u : xfull - (uint32_t)(nwin * shrink) * sizeof(T);
-        T *vs = slot0 + (int64_t)sl * slot_elems;
-        T *xs = vs + (int64_t)nd * rc;
-        mbar_expect_tx(bar + sl, vbytes + xbytes);  // arrive (release: info visible)
-        const uint64_t pf = policy_evict_first();
-        if (split == 1) {
-            if (vbytes) bulk_g2s(vs, a.vals + D.val_base, vbytes, bar + sl, pf);
-        } else {
-            for (int d = 0; d < nd; ++d)
-                bulk_g2s(vs + (int64_t)d * rc, a.vals + D.val_base + (int64_t)d * a.mrows + (int64_t)h * rc,
-                         (uint32_t)rc * sizeof(T), bar + sl, pf);
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < 2; ++i) {
+            mbar_init(full_x + i, 1);
+            mbar_init(empty_x + i, nwarps_c);
         }
-        if (!edge) {
-            const uint64_t pn = policy_evict_normal();
-            T *dst = xs;
-            for (int q = 0; q < nwin; ++q) {
-                const int st = __ldg(plan + 2 + 2 * q), cnt = __ldg(plan + 3 + 2 * q) - shrink;
-                bulk_g2s(dst, a.x + I.row0 + st, (uint32_t)cnt * sizeof(T), bar + sl, pn);
-                dst += cnt;
-            }
+        for (int i = 0; i < ns; ++i) {
+            mbar_init(full_v + i, 1);
+            mbar_init(empty_v + i, nwarps_c);
         }
-    };
-    // all threads: gather the scatter points of the item in slot sl
-    auto gather = [&](int sl) {
-        const SlotInfo &I = info[sl];
-        const int nst = I.nscat < SCAT_STAGE ? I.nscat : SCAT_STAGE;
-        for (int e = t; e < nst; e += T_) {
-            const int rr = __ldg(a.scat_row + I.scat_begin + e) - I.h * rc;
-            int own = -1;
-            if (rr >= 0 && rr < rc) own = (rr % T_) * Q + rr / T_;
-            sc_own[sl][e] = own;
-            if (own >= 0) {
-                sc_v[sl][e] = __ldg(a.scat_val + I.scat_begin + e);
-                sc_x[sl][e] = __ldg(a.x + __ldg(a.scat_col + I.scat_begin + e));
-            }
-        }
-    };
-
-    SegDesc Dn;
-    int64_t sn = 0;
-    int hn = 0;
-    if (t == 0) {
-        mbar_init(bar, 1);
-        mbar_init(bar + 1, 1);
         mbar_fence_init();
-        int h;
-        for (int k = 0; k < 2; ++k) {
-            const int64_t it = blockIdx.x + k * G;
-            if (it < nitems) {
-                const int64_t sg = seg_of(it, h);
-                const SegDesc D = a.segs[sg];
-                issue(k, sg, h, D);
-            }
-        }
-        if (blockIdx.x + 2 * G < nitems) {
-            sn = seg_of(blockIdx.x + 2 * G, hn);
-            Dn = a.segs[sn];
-        }
     }
     __syncthreads();
-    if (blockIdx.x < nitems) gather(0);
-    __syncthreads();
 
-    const T al = a.alpha, be = a.beta;
-    uint32_t ph0 = 0, ph1 = 0;
-    int k = 0;
-    for (int64_t it = blockIdx.x; it < nitems; it += G, ++k) {
-        const int sl = k & 1;
-        if (it + G < nitems) gather(sl ^ 1);  // next item's scatter points
-        mbar_wait(bar + sl, sl ? ph1 : ph0);
-        if (sl) ph1 ^= 1; else ph0 ^= 1;
-        const SlotInfo I = info[sl];
-        const bool edge = (I.flags & SEG_EDGE) != 0;
-        const int32_t *plan = a.plan + I.plan_begin;
-        const int nwin = __ldg(plan);
-        const int32_t *xoff = plan + 2 + 2 * nwin;
-        const int32_t *xwin = xoff + I.nd;
-        const int32_t *offs = a.pat_offs + I.off_begin;
-        const T *vs = slot0 + (int64_t)sl * slot_elems;
-        const T *xs = vs + (int64_t)I.nd * rc;
-        T acc[Q];
-#pragma unroll
-        for (int q = 0; q < Q; ++q) acc[q] = T(0);
-        if (!edge) {
-#pragma unroll 4
-            for (int d = 0; d < I.nd; ++d) {
-                const int xo = shrink ? __ldg(xoff + d) - __ldg(xwin + d) * shrink : __ldg(xoff + d);
-                const T *vd = vs + d * rc + t;
-                const T *xd = xs + xo + t;
-#pragma unroll
-                for (int q = 0; q < Q; ++q) acc[q] = fma(vd[q * T_], xd[q * T_], acc[q]);
+    if (threadIdx.x < 32) {
+        // ------------------------------ producer ------------------------------
+        if (threadIdx.x != 0) return;
+        const uint64_t pf = policy_evict_first(), pn = policy_evict_normal();
+        int xs = 0, vs = 0;
+        uint32_t xph = 0, vph = 0;
+        // descriptors are prefetched one segment ahead so their global-memory
+        // latency overlaps the previous segment's copies
+        auto seg_of = [&](int64_t w) { return a.seg_list ? (int64_t)__ldg(a.seg_list + w) : a.seg_begin + w; };
+        int64_t sg_next = (blockIdx.x < a.seg_count) ? seg_of(blockIdx.x) : 0;
+        SegDesc D_next;
+        if (blockIdx.x < a.seg_count) D_next = a.segs[sg_next];
+        for (int64_t w = blockIdx.x; w < a.seg_count; w += gridDim.x) {
+            const int64_t sg = sg_next;
+            const SegDesc D = D_next;
+            if (w + gridDim.x < a.seg_count) {
+                sg_next = seg_of(w + gridDim.x);
+                D_next = a.segs[sg_next];
             }
-        } else {
-            for (int d = 0; d < I.nd; ++d) {
-                const int o = __ldg(offs + d);
-                const T *vd = vs + d * rc + t;
-#pragma unroll
-                for (int q = 0; q < Q; ++q) {
-                    const int64_t idx = I.row0 + t + q * T_ + o;
-                    const T xj = (idx >= a.x_lo && idx < a.x_hi) ? __ldg(a.x + idx) : T(0);
-                    acc[q] = fma(vd[q * T_], xj, acc[q]);
+            const int64_t row0 = sg * a.mrows;
+            const bool edge = (D.flags & SEG_EDGE) != 0;
+            const int32_t *plan = a.plan + D.plan_begin;
+            const int nwin = __ldg(plan);
+            mbar_wait(empty_x + xs, xph ^ 1);
+            PipeSeg &P = sseg[xs];
+            P.row0 = row0;
+            P.scat_begin = D.scat_begin;
+            P.nscat = D.nscat;
+            P.flags = D.flags;
+            P.nd = D.ndias;
+            P.plan_begin = D.plan_begin;
+            P.off_begin = D.off_begin;
+            uint32_t xbytes = 0;
+            if (!edge)
+                for (int q = 0; q < nwin; ++q) xbytes += (uint32_t)__ldg(plan + 3 + 2 * q) * sizeof(T);
+            mbar_expect_tx(full_x + xs, xbytes);  // arrive (release: P visible) + tx
+            if (!edge) {
+                T *dst = xbuf + (int64_t)xs * xmax_elems;
+                for (int q = 0; q < nwin; ++q) {
+                    const int st = __ldg(plan + 2 + 2 * q), cnt = __ldg(plan + 3 + 2 * q);
+                    bulk_g2s(dst, a.x + row0 + st, (uint32_t)cnt * sizeof(T), full_x + xs, pn);
+                    dst += cnt;
+                }
+            }
+            xs ^= 1;
+            if (xs == 0) xph ^= 1;
+            const int nd = D.ndias;
+            for (int d0 = 0; d0 < nd; d0 += kch) {
+                const int nk = min(kch, nd - d0);
+                mbar_wait(empty_v + vs, vph ^ 1);
+                const uint32_t bytes = (uint32_t)nk * (uint32_t)a.mrows * sizeof(T);
+                mbar_expect_tx(full_v + vs, bytes);
+                bulk_g2s(vring + (int64_t)vs * chunk_elems, a.vals + D.val_base + (int64_t)d0 * a.mrows, bytes,
+                         full_v + vs, pf);
+                if (++vs == ns) {
+                    vs = 0;
+                    vph ^= 1;
                 }
             }
         }
-        if (I.nscat > 0) {
-            const int nst = I.nscat < SCAT_STAGE ? I.nscat : SCAT_STAGE;
-            for (int e = 0; e < nst; ++e) {
-                const int own = sc_own[sl][e];
-                if (own < 0 || own / Q != t) continue;
-#pragma unroll
-                for (int j = 0; j < Q; ++j)
-                    if (own - t * Q == j) acc[j] = fma(sc_v[sl][e], sc_x[sl][e], acc[j]);
-            }
-            for (int64_t e = nst; e < I.nscat; ++e) {
-                const int rr = __ldg(a.scat_row + I.scat_begin + e) - I.h * rc;
-                if (rr < 0 || rr >= rc || rr % T_ != t) continue;
-                const T v = __ldg(a.scat_val + I.scat_begin + e);
-                const T xv = __ldg(a.x + __ldg(a.scat_col + I.scat_begin + e));
-                const int qq = rr / T_;
-#pragma unroll
-                for (int j = 0; j < Q; ++j)
-                    if (qq == j) acc[j] = fma(v, xv, acc[j]);
-            }
-        }
-#pragma unroll
-        for (int q = 0; q < Q; ++q) {
-            const int64_t r = I.row0 + t + q * T_;
-            if (!edge || r < a.nrows) {
-                T *yp = a.y + r;
-                __stcs(yp, (be != T(0)) ? fma(al, acc[q], be * *yp) : al * acc[q]);
-            }
-        }
-        __syncthreads();  // slot sl, info[sl], staging[sl] free; staging[sl^1] written
-        if (t == 0 && it + 2 * G < nitems) {
-            fence_proxy_async_smem();
-            issue(sl, sn, hn, Dn);
-            if (it + 3 * G < nitems) {
-                sn = seg_of(it + 3 * G, hn);
-                Dn = a.segs[sn];
-            }
-        }
-        __syncthreads();  // info[sl] of item it + 2G visible for the next gather
+        return;
     }
+    // ------------------------------ consumers ------------------------------
+    // one row per consumer thread: row0 + ct (conflict-free shared reads)
+    const int ct = threadIdx.x - 32;
+    const int lane = ct & 31;
+    int xs = 0, vs = 0;
+    uint32_t xph = 0, vph = 0;
+    const T al = a.alpha, be = a.beta;
+    for (int64_t w = blockIdx.x; w < a.seg_count; w += gridDim.x) {
+        mbar_wait(full_x + xs, xph);
+        const PipeSeg P = sseg[xs];
+        const bool edge = (P.flags & SEG_EDGE) != 0;
+        const int32_t *plan = a.plan + P.plan_begin;
+        const int nwin = __ldg(plan);
+        const int32_t *xoff = plan + 2 + 2 * nwin;
+        const int32_t *offs = a.pat_offs + P.off_begin;
+        const T *xb = xbuf + (int64_t)xs * xmax_elems + ct;
+        const int64_t row = P.row0 + ct;
+        T acc = T(0);
+        for (int d0 = 0; d0 < P.nd; d0 += kch) {
+            const int nk = min(kch, P.nd - d0);
+            mbar_wait(full_v + vs, vph);
+            const T *vb = vring + (int64_t)vs * chunk_elems + ct;
+            if (!edge) {
+                int xo[KCH];
+#pragma unroll
+                for (int k = 0; k < KCH; ++k)
+                    if (k < nk) xo[k] = __ldg(xoff + d0 + k);
+#pragma unroll
+                for (int k = 0; k < KCH; ++k)
+                    if (k < nk) acc = fma(vb[k * C], xb[xo[k]], acc);
+            } else {
+                for (int k = 0; k < nk; ++k) {
+                    const int64_t idx = row + __ldg(offs + d0 + k);
+                    const T xj = (idx >= a.x_lo && idx < a.x_hi) ? __ldg(a.x + idx) : T(0);
+                    acc = fma(vb[k * C], xj, acc);
+                }
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(empty_v + vs);
+            if (++vs == ns) {
+                vs = 0;
+                vph ^= 1;
+            }
+        }
+        // scatter points of this row, (row, col) order
+        if (P.nscat > 0) {
+            const int32_t *sr = a.scat_row + P.scat_begin;
+            for (int64_t e = 0; e < P.nscat; ++e) {
+                if (__ldg(sr + e) != ct) continue;
+                acc = fma(__ldg(a.scat_val + P.scat_begin + e), __ldg(a.x + __ldg(a.scat_col + P.scat_begin + e)), acc);
+            }
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(empty_x + xs);
+        if (!edge || row < a.nrows) {
+            T *yp = a.y + row;
+            __stcs(yp, (be != T(0)) ? fma(al, acc, be * *yp) : al * acc);
+        }
+        xs ^= 1;
+        if (xs == 0) xph ^= 1;
+    }
+}
+
+// shared memory of the PIPE variant for a given ring depth
+inline int64_t pipe_smem(int ns, int kch, int mrows, int elem, int64_t xmax_elems) {
+    const int64_t bars = ((8 * (4 + 2 * ns) + 127) / 128) * 128;
+    return bars + 128 + 2 * xmax_elems * elem + (int64_t)ns * kch * mrows * elem;
 }
 
 static int env_int(const char *k, int d) {
@@ -652,10 +635,12 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
         const int rc = a.mrows / split;
         const int thr = rc / q;
         const int smem = (int)a.tma_smem;
-        static int attr_bytes[2][3] = {{0, 0, 0}, {0, 0, 0}};
+        static int attr_bytes[2][3][2] = {};
         const int qi = q == 1 ? 0 : (q == 2 ? 1 : 2);
-        int &cur = attr_bytes[sizeof(T) == 8][qi];
-        auto kern = q == 1 ? crsd_spmv_tma<T, 1> : (q == 2 ? crsd_spmv_tma<T, 2> : crsd_spmv_tma<T, 4>);
+        const bool sc = a.has_scatter != 0;
+        int &cur = attr_bytes[sizeof(T) == 8][qi][sc];
+        auto kern = sc ? (q == 1 ? crsd_spmv_tma<T, 1, true> : (q == 2 ? crsd_spmv_tma<T, 2, true> : crsd_spmv_tma<T, 4, true>))
+                       : (q == 1 ? crsd_spmv_tma<T, 1, false> : (q == 2 ? crsd_spmv_tma<T, 2, false> : crsd_spmv_tma<T, 4, false>));
         if (smem > cur) {
             e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
             if (e != cudaSuccess) return -(10000 + (int)e);
@@ -665,28 +650,25 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
         if (g > 0x7fffffff) g = 0x7fffffff;
         kern<<<(unsigned)g, thr, smem, (cudaStream_t)stream>>>(a, split);
     } else if (a.variant == VARIANT_PIPE) {
-        const int split = a.tma_split, q = a.tma_q;
-        const int rc = a.mrows / split;
-        const int thr = rc / q;
-        const int slot_elems = (int)((a.tma_smem / sizeof(T) + 31) / 32 * 32);
-        const int smem = 2 * slot_elems * (int)sizeof(T);
-        static int attr_p[2][3] = {{0, 0, 0}, {0, 0, 0}};
-        const int qi = q == 1 ? 0 : (q == 2 ? 1 : 2);
-        int &cur = attr_p[sizeof(T) == 8][qi];
-        auto kern = q == 1 ? crsd_spmv_tmap<T, 1> : (q == 2 ? crsd_spmv_tmap<T, 2> : crsd_spmv_tmap<T, 4>);
-        if (smem > cur) {
-            e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        // ring of KCH-diagonal value chunks; depth chosen so two CTAs fit per SM
+        constexpr int kch = 8;
+        const int64_t xmax = a.pipe_xmax_elems;
+        // two CTAs per SM when the consumer count allows it, else one with a deeper ring
+        const int per_sm = a.mrows <= 256 ? 2 : 1;
+        const int64_t budget = per_sm == 2 ? 110 * 1024 : 220 * 1024;
+        int ns = env_int("CRSD_PIPE_NS", 16);
+        while (ns > 2 && pipe_smem(ns, kch, a.mrows, sizeof(T), xmax) > budget) --ns;
+        const int64_t sm = pipe_smem(ns, kch, a.mrows, sizeof(T), xmax);
+        static int attr_pipe[2] = {0, 0};
+        int &cur = attr_pipe[sizeof(T) == 8];
+        if (sm > cur) {
+            e = cudaFuncSetAttribute(crsd_spmv_pipe<T, kch>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
             if (e != cudaSuccess) return -(10000 + (int)e);
-            cur = smem;
+            cur = (int)sm;
         }
-        int per_sm = 0;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, thr, smem);
-        if (e != cudaSuccess || per_sm < 1) per_sm = 1;
-        per_sm = env_int("CRSD_PIPE_PERSM", per_sm);
         int64_t g = (int64_t)sm_count * per_sm;
-        const int64_t nitems = a.seg_count * split;
-        if (g > nitems) g = nitems;
-        kern<<<(unsigned)g, thr, smem, (cudaStream_t)stream>>>(a, split, slot_elems);
+        if (g > a.seg_count) g = a.seg_count;
+        crsd_spmv_pipe<T, kch><<<(unsigned)g, a.mrows + 32, sm, (cudaStream_t)stream>>>(a, ns, (int)xmax);
     } else {
         crsd_spmv_ldg<T, 4><<<(unsigned)grid, threads, 0, (cudaStream_t)stream>>>(a);
     }
