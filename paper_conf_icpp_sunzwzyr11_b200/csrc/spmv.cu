@@ -302,9 +302,9 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int sp
     const int t = threadIdx.x;
     const int T_ = blockDim.x;
     const int rc = a.mrows / split;  // rows of this CTA
-    const int64_t cta = a.seg_list ? (int64_t)blockIdx.x : (int64_t)blockIdx.x;
-    const int64_t w = cta / split;
-    const int h = (int)(cta - w * split);
+    const int64_t cta = blockIdx.x;
+    const int64_t w = split == 1 ? cta : cta / split;
+    const int h = split == 1 ? 0 : (int)(cta - w * split);
     const int64_t s = a.seg_list ? (int64_t)__ldg(a.seg_list + w) : a.seg_begin + w;
     const SegDesc D = a.segs[s];
     const int64_t row0 = s * a.mrows + (int64_t)h * rc;
@@ -323,12 +323,24 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int sp
         const uint32_t xfull = (uint32_t)__ldg(plan + 1) - (uint32_t)nd * (uint32_t)a.mrows * sizeof(T);
         const uint32_t xbytes = edge ? 0u : xfull - (uint32_t)(nwin * shrink) * sizeof(T);
         mbar_expect_tx(&bar, vbytes + xbytes);
-        if (split == 1 && vbytes) bulk_g2s(vs, a.vals + D.val_base, vbytes, &bar, policy_evict_first());
+        if (split == 1) {
+            // whole segment: one copy of the value block, windows in order
+            if (vbytes) bulk_g2s(vs, a.vals + D.val_base, vbytes, &bar, policy_evict_first());
+            if (!edge) {
+                const uint64_t pn = policy_evict_normal();
+                T *dst = xs;
+                for (int q = 0; q < nwin; ++q) {
+                    const int st = __ldg(plan + 2 + 2 * q), cnt = __ldg(plan + 3 + 2 * q);
+                    bulk_g2s(dst, a.x + row0 + st, (uint32_t)cnt * sizeof(T), &bar, pn);
+                    dst += cnt;
+                }
+            }
+        }
     }
     __syncthreads();
-    if (t < 32) {
-        // warp 0 issues the remaining copies, window / diagonal q by lane q % 32
-        if (split > 1) {
+    if (split > 1 && t < 32) {
+        // row slice: warp 0 issues one copy per diagonal and per window
+        {
             const uint64_t pf = policy_evict_first();
             for (int d = t; d < nd; d += 32)
                 bulk_g2s(vs + (int64_t)d * rc, a.vals + D.val_base + (int64_t)d * a.mrows + (int64_t)h * rc,
@@ -458,23 +470,23 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
 }
 
 template <typename T, int KCH>
-__global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, int ns, int xmax_elems) {
+__global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, int ns, int nx, int xmax_elems) {
     constexpr int kch = KCH;
     extern __shared__ __align__(128) unsigned char smem[];
-    // layout: [bars: 4 + 2*ns][PipeSeg x2][xbuf x2][vring x ns]
+    // layout: [bars: 2*nx + 2*ns][PipeSeg x nx][xbuf x nx][vring x ns]
     uint64_t *full_x = reinterpret_cast<uint64_t *>(smem);
-    uint64_t *empty_x = full_x + 2;
-    uint64_t *full_v = full_x + 4;
+    uint64_t *empty_x = full_x + nx;
+    uint64_t *full_v = full_x + 2 * nx;
     uint64_t *empty_v = full_v + ns;
-    PipeSeg *sseg = reinterpret_cast<PipeSeg *>(smem + ((8 * (4 + 2 * ns) + 127) / 128) * 128);
-    T *xbuf = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sseg) + 128);
-    T *vring = xbuf + 2 * (int64_t)xmax_elems;
+    PipeSeg *sseg = reinterpret_cast<PipeSeg *>(smem + ((8 * (2 * nx + 2 * ns) + 127) / 128) * 128);
+    T *xbuf = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sseg) + ((nx * (int)sizeof(PipeSeg) + 127) / 128) * 128);
+    T *vring = xbuf + nx * (int64_t)xmax_elems;
     const int C = a.mrows;  // consumer threads (one row each)
     const int nwarps_c = C / 32;
     const int64_t chunk_elems = (int64_t)kch * a.mrows;
 
     if (threadIdx.x == 0) {
-        for (int i = 0; i < 2; ++i) {
+        for (int i = 0; i < nx; ++i) {
             mbar_init(full_x + i, 1);
             mbar_init(empty_x + i, nwarps_c);
         }
@@ -530,8 +542,10 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
                     dst += cnt;
                 }
             }
-            xs ^= 1;
-            if (xs == 0) xph ^= 1;
+            if (++xs == nx) {
+                xs = 0;
+                xph ^= 1;
+            }
             const int nd = D.ndias;
             for (int d0 = 0; d0 < nd; d0 += kch) {
                 const int nk = min(kch, nd - d0);
@@ -606,15 +620,18 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
             T *yp = a.y + row;
             __stcs(yp, (be != T(0)) ? fma(al, acc, be * *yp) : al * acc);
         }
-        xs ^= 1;
-        if (xs == 0) xph ^= 1;
+        if (++xs == nx) {
+            xs = 0;
+            xph ^= 1;
+        }
     }
 }
 
-// shared memory of the PIPE variant for a given ring depth
-inline int64_t pipe_smem(int ns, int kch, int mrows, int elem, int64_t xmax_elems) {
-    const int64_t bars = ((8 * (4 + 2 * ns) + 127) / 128) * 128;
-    return bars + 128 + 2 * xmax_elems * elem + (int64_t)ns * kch * mrows * elem;
+// shared memory of the PIPE variant for nx x slots and ns value stages
+inline int64_t pipe_smem(int ns, int nx, int kch, int mrows, int elem, int64_t xmax_elems) {
+    const int64_t bars = ((8 * (2 * nx + 2 * ns) + 127) / 128) * 128;
+    const int64_t segs = ((nx * (int64_t)sizeof(PipeSeg) + 127) / 128) * 128;
+    return bars + segs + nx * xmax_elems * elem + (int64_t)ns * kch * mrows * elem;
 }
 
 static int env_int(const char *k, int d) {
@@ -650,15 +667,17 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
         if (g > 0x7fffffff) g = 0x7fffffff;
         kern<<<(unsigned)g, thr, smem, (cudaStream_t)stream>>>(a, split);
     } else if (a.variant == VARIANT_PIPE) {
-        // ring of KCH-diagonal value chunks; depth chosen so two CTAs fit per SM
+        // ring of KCH-diagonal value chunks; two CTAs per SM when the consumer
+        // count allows it (else one), nx x slots, as many stages as fit
         constexpr int kch = 8;
         const int64_t xmax = a.pipe_xmax_elems;
-        // two CTAs per SM when the consumer count allows it, else one with a deeper ring
-        const int per_sm = a.mrows <= 256 ? 2 : 1;
-        const int64_t budget = per_sm == 2 ? 110 * 1024 : 220 * 1024;
-        int ns = env_int("CRSD_PIPE_NS", 16);
-        while (ns > 2 && pipe_smem(ns, kch, a.mrows, sizeof(T), xmax) > budget) --ns;
-        const int64_t sm = pipe_smem(ns, kch, a.mrows, sizeof(T), xmax);
+        const int per_sm = env_int("CRSD_PIPE_PERSM", a.mrows <= 256 ? 2 : 1);
+        const int64_t budget = (per_sm >= 2 ? 110 : 220) * 1024;
+        int nx = env_int("CRSD_PIPE_NX", 2);
+        while (nx > 2 && pipe_smem(2, nx, kch, a.mrows, sizeof(T), xmax) > budget) --nx;
+        int ns = env_int("CRSD_PIPE_NS", 32);
+        while (ns > 2 && pipe_smem(ns, nx, kch, a.mrows, sizeof(T), xmax) > budget) --ns;
+        const int64_t sm = pipe_smem(ns, nx, kch, a.mrows, sizeof(T), xmax);
         static int attr_pipe[2] = {0, 0};
         int &cur = attr_pipe[sizeof(T) == 8];
         if (sm > cur) {
@@ -668,7 +687,7 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
         }
         int64_t g = (int64_t)sm_count * per_sm;
         if (g > a.seg_count) g = a.seg_count;
-        crsd_spmv_pipe<T, kch><<<(unsigned)g, a.mrows + 32, sm, (cudaStream_t)stream>>>(a, ns, (int)xmax);
+        crsd_spmv_pipe<T, kch><<<(unsigned)g, a.mrows + 32, sm, (cudaStream_t)stream>>>(a, ns, nx, (int)xmax);
     } else {
         crsd_spmv_ldg<T, 4><<<(unsigned)grid, threads, 0, (cudaStream_t)stream>>>(a);
     }

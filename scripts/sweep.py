@@ -49,11 +49,11 @@ def main():
         tdt = torch.float64 if dt == "f64" else torch.float32
         x = torch.rand(a.ncols, dtype=tdt, device="cuda")
         y = torch.empty(a.nrows, dtype=tdt, device="cuda")
-        runs = [("ldg", 1, None)] + [("tma", 2, t) for t in TMA] + [("pipe", 3, t) for t in TMA]
+        runs = [("ldg", 1, None)] + [("tma", 2, t) for t in TMA] + [("pipe", 3, sh) for sh in SHAPES]
         for name, v, sh in runs:
             for k in ("CRSD_PIPE_PERSM", "CRSD_PIPE_NX", "CRSD_PIPE_NS", "CRSD_TMA_Q", "CRSD_TMA_SPLIT"):
                 os.environ.pop(k, None)
-            if sh and name in ("tma", "pipe"):
+            if sh and name == "tma":
                 os.environ["CRSD_TMA_" + sh[0]] = str(sh[1])
             elif sh:
                 os.environ["CRSD_PIPE_PERSM"], os.environ["CRSD_PIPE_NX"], os.environ["CRSD_PIPE_NS"] = map(str, sh)
