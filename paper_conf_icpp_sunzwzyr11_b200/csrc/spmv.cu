@@ -115,7 +115,7 @@ __device__ __forceinline__ double2 make_vec(const double (&v)[2]) { return make_
 __device__ __forceinline__ float4 make_vec(const float (&v)[4]) { return make_float4(v[0], v[1], v[2], v[3]); }
 
 template <typename T, int CH>
-__global__ void __launch_bounds__(256, sizeof(T) == 8 ? 3 : 4) crsd_spmv_ldg(const SpmvArgs<T> a) {
+__global__ void __launch_bounds__(256, sizeof(T) == 8 ? 2 : 3) crsd_spmv_ldg(const SpmvArgs<T> a) {
     using V = typename VecT<T>::type;
     constexpr int R = VecT<T>::R;
     constexpr int LOG = VecT<T>::LOG;
@@ -137,16 +137,27 @@ __global__ void __launch_bounds__(256, sizeof(T) == 8 ? 3 : 4) crsd_spmv_ldg(con
 
         if (!(D.flags & SEG_EDGE)) {
             const V *xv = reinterpret_cast<const V *>(a.x + row0) + t;
+            // software pipeline over chunks of CH diagonals: the values and
+            // offsets of chunk c+1 are in flight while chunk c computes
+            V val[CH], nval[CH];
+            int o[CH], no[CH];
+#pragma unroll
+            for (int c = 0; c < CH; ++c) {
+                if (c < nd) {
+                    o[c] = __ldg(offs + c);
+                    val[c] = ld_stream(vb + (int64_t)c * vstride, pol);
+                }
+            }
             for (int d0 = 0; d0 < nd; d0 += CH) {
-                V val[CH], xa[CH], xe[CH];
-                int o[CH];
+                const int d1 = d0 + CH;
 #pragma unroll
                 for (int c = 0; c < CH; ++c) {
-                    if (d0 + c < nd) {
-                        o[c] = __ldg(offs + d0 + c);
-                        val[c] = ld_stream(vb + (int64_t)(d0 + c) * vstride, pol);
+                    if (d1 + c < nd) {
+                        no[c] = __ldg(offs + d1 + c);
+                        nval[c] = ld_stream(vb + (int64_t)(d1 + c) * vstride, pol);
                     }
                 }
+                V xa[CH], xe[CH];
 #pragma unroll
                 for (int c = 0; c < CH; ++c) {
                     if (d0 + c < nd) {
@@ -171,6 +182,11 @@ __global__ void __launch_bounds__(256, sizeof(T) == 8 ? 3 : 4) crsd_spmv_ldg(con
 #pragma unroll
                         for (int j = 0; j < R; ++j) acc[j] = fma(get(val[c], j), xs[j], acc[j]);
                     }
+                }
+#pragma unroll
+                for (int c = 0; c < CH; ++c) {
+                    val[c] = nval[c];
+                    o[c] = no[c];
                 }
             }
         } else {
@@ -323,24 +339,13 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int sp
         const uint32_t xfull = (uint32_t)__ldg(plan + 1) - (uint32_t)nd * (uint32_t)a.mrows * sizeof(T);
         const uint32_t xbytes = edge ? 0u : xfull - (uint32_t)(nwin * shrink) * sizeof(T);
         mbar_expect_tx(&bar, vbytes + xbytes);
-        if (split == 1) {
-            // whole segment: one copy of the value block, windows in order
-            if (vbytes) bulk_g2s(vs, a.vals + D.val_base, vbytes, &bar, policy_evict_first());
-            if (!edge) {
-                const uint64_t pn = policy_evict_normal();
-                T *dst = xs;
-                for (int q = 0; q < nwin; ++q) {
-                    const int st = __ldg(plan + 2 + 2 * q), cnt = __ldg(plan + 3 + 2 * q);
-                    bulk_g2s(dst, a.x + row0 + st, (uint32_t)cnt * sizeof(T), &bar, pn);
-                    dst += cnt;
-                }
-            }
-        }
+        if (split == 1 && vbytes) bulk_g2s(vs, a.vals + D.val_base, vbytes, &bar, policy_evict_first());
     }
     __syncthreads();
-    if (split > 1 && t < 32) {
-        // row slice: warp 0 issues one copy per diagonal and per window
-        {
+    if (t < 32) {
+        // warp 0 issues the remaining copies: one per diagonal of a row slice,
+        // one per x window (window q by lane q % 32)
+        if (split > 1) {
             const uint64_t pf = policy_evict_first();
             for (int d = t; d < nd; d += 32)
                 bulk_g2s(vs + (int64_t)d * rc, a.vals + D.val_base + (int64_t)d * a.mrows + (int64_t)h * rc,
