@@ -87,8 +87,10 @@ static void plan_layout(crsd_matrix_s *A) {
         A->x_hi = H.n_local + A->halo_hi_valid;
     }
     make_segdescs(H, A->rpt, A->x_lo, A->x_hi, A->segdesc);
-    // x windows: offsets closer than 64 elements share one staged window
-    A->smem_bytes = make_plans(H, 64, A->plan, A->segdesc, &A->xmax_elems);
+    // x windows: offsets closer than mrows share one staged window (merging
+    // two windows whose gap is below mrows never adds bytes, and every window
+    // is one bulk copy: fewer, larger copies)
+    A->smem_bytes = make_plans(H, H.mrows, A->plan, A->segdesc, &A->xmax_elems);
     // TMA variant shape: smallest split of a segment into row slices whose
     // staging (values + x windows) stays <= 40 KB, i.e. >= 5 CTAs per SM
     A->tma_split = 1;

@@ -115,7 +115,7 @@ __device__ __forceinline__ double2 make_vec(const double (&v)[2]) { return make_
 __device__ __forceinline__ float4 make_vec(const float (&v)[4]) { return make_float4(v[0], v[1], v[2], v[3]); }
 
 template <typename T, int CH>
-__global__ void __launch_bounds__(256, sizeof(T) == 8 ? 2 : 3) crsd_spmv_ldg(const SpmvArgs<T> a) {
+__global__ void __launch_bounds__(256, sizeof(T) == 8 ? 3 : 4) crsd_spmv_ldg(const SpmvArgs<T> a) {
     using V = typename VecT<T>::type;
     constexpr int R = VecT<T>::R;
     constexpr int LOG = VecT<T>::LOG;
@@ -137,27 +137,16 @@ __global__ void __launch_bounds__(256, sizeof(T) == 8 ? 2 : 3) crsd_spmv_ldg(con
 
         if (!(D.flags & SEG_EDGE)) {
             const V *xv = reinterpret_cast<const V *>(a.x + row0) + t;
-            // software pipeline over chunks of CH diagonals: the values and
-            // offsets of chunk c+1 are in flight while chunk c computes
-            V val[CH], nval[CH];
-            int o[CH], no[CH];
-#pragma unroll
-            for (int c = 0; c < CH; ++c) {
-                if (c < nd) {
-                    o[c] = __ldg(offs + c);
-                    val[c] = ld_stream(vb + (int64_t)c * vstride, pol);
-                }
-            }
             for (int d0 = 0; d0 < nd; d0 += CH) {
-                const int d1 = d0 + CH;
+                V val[CH], xa[CH], xe[CH];
+                int o[CH];
 #pragma unroll
                 for (int c = 0; c < CH; ++c) {
-                    if (d1 + c < nd) {
-                        no[c] = __ldg(offs + d1 + c);
-                        nval[c] = ld_stream(vb + (int64_t)(d1 + c) * vstride, pol);
+                    if (d0 + c < nd) {
+                        o[c] = __ldg(offs + d0 + c);
+                        val[c] = ld_stream(vb + (int64_t)(d0 + c) * vstride, pol);
                     }
                 }
-                V xa[CH], xe[CH];
 #pragma unroll
                 for (int c = 0; c < CH; ++c) {
                     if (d0 + c < nd) {
@@ -182,11 +171,6 @@ __global__ void __launch_bounds__(256, sizeof(T) == 8 ? 2 : 3) crsd_spmv_ldg(con
 #pragma unroll
                         for (int j = 0; j < R; ++j) acc[j] = fma(get(val[c], j), xs[j], acc[j]);
                     }
-                }
-#pragma unroll
-                for (int c = 0; c < CH; ++c) {
-                    val[c] = nval[c];
-                    o[c] = no[c];
                 }
             }
         } else {

@@ -264,3 +264,41 @@ def test_dist_compute_single_gpu(torch_cuda, case, world, variant):
         err = coo.parity_error(yd.cpu().numpy(), yref[rb:re], scale[rb:re])
         assert err <= TOL[dt], (r, err)
         assert A.last_launch_count() in (1, 2)
+
+
+def test_nccl_comm_world1(torch_cuda):
+    """The NCCL plumbing of crsd_spmv_dist on one GPU: a 1-rank torch.distributed
+    (nccl) group, crsd_comm_init_rank, crsd_dist_bind (allgather of the row
+    ranges) and crsd_spmv_dist with a communicator (empty halo plan)."""
+    import os
+    import socket
+
+    import torch.distributed as dist
+
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, Comm
+
+    torch = torch_cuda
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK="0", WORLD_SIZE="1")
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda:0"))
+    try:
+        a = gen.config2(n=40)
+        n = a.nrows
+        A = CRSDMatrix.from_coo(n, n, a.row, a.col, a.val, row_range=(0, n), device=0)
+        comm = Comm(0, 1, 0)
+        A.dist_bind(comm)
+        lo, nloc, hi = A.x_layout()
+        assert (lo, nloc, hi) == (0, n, 0)
+        x = np.random.default_rng(4).uniform(-1, 1, n)
+        xd = torch.from_numpy(x).to("cuda:0")
+        yd = torch.full((n,), float("nan"), device="cuda:0", dtype=torch.float64)
+        A.spmv_dist(xd, yd, 1.0, 0.0, comm)
+        torch.cuda.synchronize()
+        yref, scale = coo.coo_spmv(n, n, a.row, a.col, a.val, x)
+        assert coo.parity_error(yd.cpu().numpy(), yref, scale) <= 1e-12
+        comm.close()
+    finally:
+        dist.destroy_process_group()
