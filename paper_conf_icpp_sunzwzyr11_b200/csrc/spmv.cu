@@ -457,6 +457,9 @@ struct PipeSeg {  // segment info handed from producer to consumers (per x slot)
     int32_t pad;
 };
 
+__device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
 __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
@@ -465,20 +468,19 @@ template <typename T, int KCH>
 __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, int ns, int nx, int xmax_elems) {
     constexpr int kch = KCH;
     extern __shared__ __align__(128) unsigned char smem[];
-    // layout: [bars: 2*nx + 2*ns][PipeSeg x nx][scatter staging x nx][xbuf x nx][vring x ns]
+    // layout: [bars: 2*nx + 2*ns][PipeSeg x nx][xbuf x nx][vring x ns]
     uint64_t *full_x = reinterpret_cast<uint64_t *>(smem);
     uint64_t *empty_x = full_x + nx;
     uint64_t *full_v = full_x + 2 * nx;
     uint64_t *empty_v = full_v + ns;
     PipeSeg *sseg = reinterpret_cast<PipeSeg *>(smem + ((8 * (2 * nx + 2 * ns) + 127) / 128) * 128);
-    T *sc_v = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sseg) + ((nx * (int)sizeof(PipeSeg) + 127) / 128) * 128);
-    T *sc_x = sc_v + nx * SCAT_STAGE;
-    int32_t *sc_row = reinterpret_cast<int32_t *>(sc_x + nx * SCAT_STAGE);
-    T *xbuf = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sc_row) + ((nx * SCAT_STAGE * 4 + 127) / 128) * 128);
+    T *xbuf = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sseg) + ((nx * (int)sizeof(PipeSeg) + 127) / 128) * 128);
     T *vring = xbuf + nx * (int64_t)xmax_elems;
     const int C = a.mrows;  // consumer threads (one row each)
     const int nwarps_c = C / 32;
     const int64_t chunk_elems = (int64_t)kch * a.mrows;
+    __shared__ T sc_v[SCAT_STAGE], sc_x[SCAT_STAGE];
+    __shared__ int32_t sc_row[SCAT_STAGE];
 
     if (threadIdx.x == 0) {
         for (int i = 0; i < nx; ++i) {
@@ -495,12 +497,7 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
 
     if (threadIdx.x < 32) {
         // ------------------------------ producer ------------------------------
-        // lane 0 owns the rings and issues every bulk copy; the other lanes
-        // gather the segment's scatter points (value, x[col], row) into the
-        // slot's staging area, so the random x reads are done long before the
-        // consumers reach them. The slot's "full" barrier is armed with the
-        // x bytes first and arrived on only after the gathers are written.
-        const int lane = threadIdx.x;
+        if (threadIdx.x != 0) return;
         const uint64_t pf = policy_evict_first(), pn = policy_evict_normal();
         int xs = 0, vs = 0;
         uint32_t xph = 0, vph = 0;
@@ -521,57 +518,43 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
             const bool edge = (D.flags & SEG_EDGE) != 0;
             const int32_t *plan = a.plan + D.plan_begin;
             const int nwin = __ldg(plan);
-            if (lane == 0) {
-                mbar_wait(empty_x + xs, xph ^ 1);
-                PipeSeg &P = sseg[xs];
-                P.row0 = row0;
-                P.scat_begin = D.scat_begin;
-                P.nscat = D.nscat;
-                P.flags = D.flags;
-                P.nd = D.ndias;
-                P.plan_begin = D.plan_begin;
-                P.off_begin = D.off_begin;
-                uint32_t xbytes = 0;
-                if (!edge)
-                    for (int q = 0; q < nwin; ++q) xbytes += (uint32_t)__ldg(plan + 3 + 2 * q) * sizeof(T);
-                mbar_expect_tx_only(full_x + xs, xbytes);
-                if (!edge) {
-                    T *dst = xbuf + (int64_t)xs * xmax_elems;
-                    for (int q = 0; q < nwin; ++q) {
-                        const int st = __ldg(plan + 2 + 2 * q), cnt = __ldg(plan + 3 + 2 * q);
-                        bulk_g2s(dst, a.x + row0 + st, (uint32_t)cnt * sizeof(T), full_x + xs, pn);
-                        dst += cnt;
-                    }
+            mbar_wait(empty_x + xs, xph ^ 1);
+            PipeSeg &P = sseg[xs];
+            P.row0 = row0;
+            P.scat_begin = D.scat_begin;
+            P.nscat = D.nscat;
+            P.flags = D.flags;
+            P.nd = D.ndias;
+            P.plan_begin = D.plan_begin;
+            P.off_begin = D.off_begin;
+            uint32_t xbytes = 0;
+            if (!edge)
+                for (int q = 0; q < nwin; ++q) xbytes += (uint32_t)__ldg(plan + 3 + 2 * q) * sizeof(T);
+            mbar_expect_tx(full_x + xs, xbytes);  // arrive (release: P visible) + tx
+            if (!edge) {
+                T *dst = xbuf + (int64_t)xs * xmax_elems;
+                for (int q = 0; q < nwin; ++q) {
+                    const int st = __ldg(plan + 2 + 2 * q), cnt = __ldg(plan + 3 + 2 * q);
+                    bulk_g2s(dst, a.x + row0 + st, (uint32_t)cnt * sizeof(T), full_x + xs, pn);
+                    dst += cnt;
                 }
             }
-            __syncwarp();
-            const int nst = D.nscat < SCAT_STAGE ? D.nscat : SCAT_STAGE;
-            for (int e = lane; e < nst; e += 32) {
-                sc_row[xs * SCAT_STAGE + e] = __ldg(a.scat_row + D.scat_begin + e);
-                sc_v[xs * SCAT_STAGE + e] = __ldg(a.scat_val + D.scat_begin + e);
-                sc_x[xs * SCAT_STAGE + e] = __ldg(a.x + __ldg(a.scat_col + D.scat_begin + e));
-            }
-            __syncwarp();
-            if (lane == 0) {
-                mbar_arrive(full_x + xs);  // release: P and the staged scatter points
-                const int nd = D.ndias;
-                for (int d0 = 0; d0 < nd; d0 += kch) {
-                    const int nk = min(kch, nd - d0);
-                    mbar_wait(empty_v + vs, vph ^ 1);
-                    const uint32_t bytes = (uint32_t)nk * (uint32_t)a.mrows * sizeof(T);
-                    mbar_expect_tx(full_v + vs, bytes);
-                    bulk_g2s(vring + (int64_t)vs * chunk_elems, a.vals + D.val_base + (int64_t)d0 * a.mrows, bytes,
-                             full_v + vs, pf);
-                    if (++vs == ns) {
-                        vs = 0;
-                        vph ^= 1;
-                    }
-                }
-            }
-            __syncwarp();
             if (++xs == nx) {
                 xs = 0;
                 xph ^= 1;
+            }
+            const int nd = D.ndias;
+            for (int d0 = 0; d0 < nd; d0 += kch) {
+                const int nk = min(kch, nd - d0);
+                mbar_wait(empty_v + vs, vph ^ 1);
+                const uint32_t bytes = (uint32_t)nk * (uint32_t)a.mrows * sizeof(T);
+                mbar_expect_tx(full_v + vs, bytes);
+                bulk_g2s(vring + (int64_t)vs * chunk_elems, a.vals + D.val_base + (int64_t)d0 * a.mrows, bytes,
+                         full_v + vs, pf);
+                if (++vs == ns) {
+                    vs = 0;
+                    vph ^= 1;
+                }
             }
         }
         return;
@@ -593,6 +576,16 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
         const int32_t *offs = a.pat_offs + P.off_begin;
         const T *xb = xbuf + (int64_t)xs * xmax_elems + ct;
         const int64_t row = P.row0 + ct;
+        // scatter points: consumer e gathers entry e now; the loads are in
+        // flight during the diagonal loop and staged for the owners after it
+        const int nst = P.nscat < SCAT_STAGE ? P.nscat : SCAT_STAGE;
+        int g_row = -1;
+        T g_v = T(0), g_x = T(0);
+        if (ct < nst) {
+            g_row = __ldg(a.scat_row + P.scat_begin + ct);
+            g_v = __ldg(a.scat_val + P.scat_begin + ct);
+            g_x = __ldg(a.x + __ldg(a.scat_col + P.scat_begin + ct));
+        }
         T acc = T(0);
         for (int d0 = 0; d0 < P.nd; d0 += kch) {
             const int nk = min(kch, P.nd - d0);
@@ -620,20 +613,26 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
                 vph ^= 1;
             }
         }
-        // scatter points of this row, (row, col) order: staged by the producer
-        // warp (first SCAT_STAGE), the rest from global memory
+        __syncwarp();
+        if (lane == 0) mbar_arrive(empty_x + xs);  // the x slot is no longer needed
+        // scatter points of this row in (row, col) order: staged ones, then
+        // any beyond SCAT_STAGE from global memory
         if (P.nscat > 0) {
-            const int nst = P.nscat < SCAT_STAGE ? P.nscat : SCAT_STAGE;
+            if (ct < nst) {
+                sc_row[ct] = g_row;
+                sc_v[ct] = g_v;
+                sc_x[ct] = g_x;
+            }
+            named_bar_sync(1, C);
             for (int e = 0; e < nst; ++e)
-                if (sc_row[xs * SCAT_STAGE + e] == ct) acc = fma(sc_v[xs * SCAT_STAGE + e], sc_x[xs * SCAT_STAGE + e], acc);
+                if (sc_row[e] == ct) acc = fma(sc_v[e], sc_x[e], acc);
             const int32_t *sr = a.scat_row + P.scat_begin;
             for (int64_t e = nst; e < P.nscat; ++e) {
                 if (__ldg(sr + e) != ct) continue;
                 acc = fma(__ldg(a.scat_val + P.scat_begin + e), __ldg(a.x + __ldg(a.scat_col + P.scat_begin + e)), acc);
             }
+            named_bar_sync(1, C);  // staging is rewritten by the next segment
         }
-        __syncwarp();
-        if (lane == 0) mbar_arrive(empty_x + xs);
         if (!edge || row < a.nrows) {
             T *yp = a.y + row;
             __stcs(yp, (be != T(0)) ? fma(al, acc, be * *yp) : al * acc);
@@ -649,8 +648,7 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
 inline int64_t pipe_smem(int ns, int nx, int kch, int mrows, int elem, int64_t xmax_elems) {
     const int64_t bars = ((8 * (2 * nx + 2 * ns) + 127) / 128) * 128;
     const int64_t segs = ((nx * (int64_t)sizeof(PipeSeg) + 127) / 128) * 128;
-    const int64_t stage = 2 * nx * SCAT_STAGE * elem + ((nx * SCAT_STAGE * 4 + 127) / 128) * 128;
-    return bars + segs + stage + nx * xmax_elems * elem + (int64_t)ns * kch * mrows * elem;
+    return bars + segs + nx * xmax_elems * elem + (int64_t)ns * kch * mrows * elem;
 }
 
 static int env_int(const char *k, int d) {
