@@ -292,7 +292,6 @@ __device__ __forceinline__ uint64_t policy_evict_normal() {
     return p;
 }
 
-constexpr int SCAT_STAGE = 128;
 
 // A CTA covers `rc` rows of one segment (rc = mrows / split): with split > 1
 // the segment's value block is fetched as one bulk copy per diagonal (its rc
@@ -356,20 +355,24 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int sp
             }
         }
     }
-    // Scatter points of this CTA's rows are gathered now, while the bulk
-    // copies are in flight: thread e loads entry e (value, x[col], owner), so
-    // the random x reads overlap the TMA wait instead of ending the CTA.
-    __shared__ T sc_v[SCAT ? SCAT_STAGE : 1], sc_x[SCAT ? SCAT_STAGE : 1];
-    __shared__ int32_t sc_own[SCAT ? SCAT_STAGE : 1];
-    const int nst = SCAT ? (D.nscat < SCAT_STAGE ? D.nscat : SCAT_STAGE) : 0;
-    for (int e = t; e < nst; e += T_) {
-        const int rr = __ldg(a.scat_row + D.scat_begin + e) - h * rc;
-        int own = -1;
-        if (rr >= 0 && rr < rc) own = (rr % T_) * Q + rr / T_;  // (thread, slot)
-        sc_own[e] = own;
-        if (own >= 0) {
-            sc_v[e] = __ldg(a.scat_val + D.scat_begin + e);
-            sc_x[e] = __ldg(a.x + __ldg(a.scat_col + D.scat_begin + e));
+    // Scatter points are gathered now, while the bulk copies are in flight:
+    // each warp takes the segment's first 32 entries (lane l -> entry l) and
+    // keeps, by ballot, those owned by its threads (owner of local row l is
+    // thread l % T_, slot l / T_); entries beyond 32 are read at the end.
+    const int lane = t & 31;
+    int g_own = -1;
+    T g_v = T(0), g_x = T(0);
+    unsigned g_mask = 0u;
+    if (SCAT && D.nscat > 0) {
+        if (lane < D.nscat) {
+            const int rr = __ldg(a.scat_row + D.scat_begin + lane) - h * rc;
+            if (rr >= 0 && rr < rc) g_own = (rr % T_) * Q + rr / T_;
+        }
+        const bool mine = g_own >= 0 && (g_own / Q) / 32 == t / 32;
+        g_mask = __ballot_sync(0xffffffffu, mine);
+        if (mine) {
+            g_v = __ldg(a.scat_val + D.scat_begin + lane);
+            g_x = __ldg(a.x + __ldg(a.scat_col + D.scat_begin + lane));
         }
     }
     T acc[Q];
@@ -400,19 +403,19 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int sp
             }
         }
     }
-    // scatter points in (row, col) order: staged ones from shared memory,
-    // any beyond SCAT_STAGE from global memory
+    // scatter points in (row, col) order: gathered ones, then any beyond 32
     if (SCAT && D.nscat > 0) {
-        __syncthreads();
-        for (int e = 0; e < nst; ++e) {
-            const int own = sc_own[e];
-            if (own < 0 || own / Q != t) continue;
+        for (unsigned m = g_mask; m; m &= m - 1) {
+            const int j = __ffs(m) - 1;
+            const int own = __shfl_sync(0xffffffffu, g_own, j);
+            const T v = __shfl_sync(0xffffffffu, g_v, j);
+            const T xv = __shfl_sync(0xffffffffu, g_x, j);
 #pragma unroll
-            for (int j = 0; j < Q; ++j)
-                if (own - t * Q == j) acc[j] = fma(sc_v[e], sc_x[e], acc[j]);
+            for (int q = 0; q < Q; ++q)
+                if (own == t * Q + q) acc[q] = fma(v, xv, acc[q]);
         }
         const int32_t *sr = a.scat_row + D.scat_begin;
-        for (int64_t e = nst; e < D.nscat; ++e) {
+        for (int64_t e = 32; e < D.nscat; ++e) {
             const int rr = __ldg(sr + e) - h * rc;
             if (rr < 0 || rr >= rc || rr % T_ != t) continue;
             const T v = __ldg(a.scat_val + D.scat_begin + e);
@@ -479,8 +482,6 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
     const int C = a.mrows;  // consumer threads (one row each)
     const int nwarps_c = C / 32;
     const int64_t chunk_elems = (int64_t)kch * a.mrows;
-    __shared__ T sc_v[SCAT_STAGE], sc_x[SCAT_STAGE];
-    __shared__ int32_t sc_row[SCAT_STAGE];
 
     if (threadIdx.x == 0) {
         for (int i = 0; i < nx; ++i) {
@@ -576,15 +577,23 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
         const int32_t *offs = a.pat_offs + P.off_begin;
         const T *xb = xbuf + (int64_t)xs * xmax_elems + ct;
         const int64_t row = P.row0 + ct;
-        // scatter points: consumer e gathers entry e now; the loads are in
-        // flight during the diagonal loop and staged for the owners after it
-        const int nst = P.nscat < SCAT_STAGE ? P.nscat : SCAT_STAGE;
+        // scatter points: each warp gathers the entries of its own 32 rows
+        // now (lane l takes entry l of the first 32 of the segment; a ballot
+        // keeps those in this warp's rows), so the random x loads are in
+        // flight during the diagonal loop; entries beyond 32 are read at the
+        // end (rare)
+        const int wrow0 = ct & ~31;
         int g_row = -1;
         T g_v = T(0), g_x = T(0);
-        if (ct < nst) {
-            g_row = __ldg(a.scat_row + P.scat_begin + ct);
-            g_v = __ldg(a.scat_val + P.scat_begin + ct);
-            g_x = __ldg(a.x + __ldg(a.scat_col + P.scat_begin + ct));
+        unsigned g_mask = 0u;
+        if (P.nscat > 0) {
+            if (lane < P.nscat) g_row = __ldg(a.scat_row + P.scat_begin + lane);
+            const bool mine = g_row >= wrow0 && g_row < wrow0 + 32;
+            g_mask = __ballot_sync(0xffffffffu, mine);
+            if (mine) {
+                g_v = __ldg(a.scat_val + P.scat_begin + lane);
+                g_x = __ldg(a.x + __ldg(a.scat_col + P.scat_begin + lane));
+            }
         }
         T acc = T(0);
         for (int d0 = 0; d0 < P.nd; d0 += kch) {
@@ -615,23 +624,21 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(empty_x + xs);  // the x slot is no longer needed
-        // scatter points of this row in (row, col) order: staged ones, then
-        // any beyond SCAT_STAGE from global memory
+        // scatter points of this row in (row, col) order: the gathered ones
+        // (broadcast from the lane that holds them), then any beyond 32
         if (P.nscat > 0) {
-            if (ct < nst) {
-                sc_row[ct] = g_row;
-                sc_v[ct] = g_v;
-                sc_x[ct] = g_x;
+            for (unsigned m = g_mask; m; m &= m - 1) {
+                const int j = __ffs(m) - 1;
+                const int r = __shfl_sync(0xffffffffu, g_row, j);
+                const T v = __shfl_sync(0xffffffffu, g_v, j);
+                const T xv = __shfl_sync(0xffffffffu, g_x, j);
+                if (r == ct) acc = fma(v, xv, acc);
             }
-            named_bar_sync(1, C);
-            for (int e = 0; e < nst; ++e)
-                if (sc_row[e] == ct) acc = fma(sc_v[e], sc_x[e], acc);
             const int32_t *sr = a.scat_row + P.scat_begin;
-            for (int64_t e = nst; e < P.nscat; ++e) {
+            for (int64_t e = 32; e < P.nscat; ++e) {
                 if (__ldg(sr + e) != ct) continue;
                 acc = fma(__ldg(a.scat_val + P.scat_begin + e), __ldg(a.x + __ldg(a.scat_col + P.scat_begin + e)), acc);
             }
-            named_bar_sync(1, C);  // staging is rewritten by the next segment
         }
         if (!edge || row < a.nrows) {
             T *yp = a.y + row;
