@@ -185,9 +185,9 @@ static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_
         delete A;
         return fail(CRSD_ERR_UNSUPPORTED, msg);
     }
-    if (o.variant == CRSD_VARIANT_PIPE && A->H.mrows > 512) {
+    if (o.variant == CRSD_VARIANT_PIPE && A->H.mrows > 1024) {
         delete A;
-        return fail(CRSD_ERR_UNSUPPORTED, "PIPE variant runs one row per thread: mrows must be <= 512");
+        return fail(CRSD_ERR_UNSUPPORTED, "PIPE variant: mrows must be <= 1024");
     }
     if (o.variant == CRSD_VARIANT_LDG) A->variant = VARIANT_LDG;
     else if (o.variant == CRSD_VARIANT_TMA) A->variant = VARIANT_TMA;
@@ -199,7 +199,7 @@ static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_
         // copy bandwidth); otherwise the chunked ring (PIPE) for fp64 (C3 81%)
         // and the register variant for fp32 (C3 76%).
         if (A->tma_split == 1 && A->tma_smem <= 32 * 1024) A->variant = VARIANT_TMA;
-        else if (A->H.elem == 8 && pipe_need <= smem_cap && A->H.mrows <= 512) A->variant = VARIANT_PIPE;
+        else if (A->H.elem == 8 && pipe_need <= smem_cap && A->H.mrows <= 1024) A->variant = VARIANT_PIPE;
         else A->variant = VARIANT_LDG;
     }
     if (!A->host_only) {

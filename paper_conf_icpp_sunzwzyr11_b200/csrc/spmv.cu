@@ -467,7 +467,7 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
-template <typename T, int KCH>
+template <typename T, int KCH, int Q>
 __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, int ns, int nx, int xmax_elems) {
     constexpr int kch = KCH;
     extern __shared__ __align__(128) unsigned char smem[];
@@ -479,7 +479,7 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
     PipeSeg *sseg = reinterpret_cast<PipeSeg *>(smem + ((8 * (2 * nx + 2 * ns) + 127) / 128) * 128);
     T *xbuf = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sseg) + ((nx * (int)sizeof(PipeSeg) + 127) / 128) * 128);
     T *vring = xbuf + nx * (int64_t)xmax_elems;
-    const int C = a.mrows;  // consumer threads (one row each)
+    const int C = a.mrows / Q;  // consumer threads (Q rows each)
     const int nwarps_c = C / 32;
     const int64_t chunk_elems = (int64_t)kch * a.mrows;
 
@@ -561,7 +561,7 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
         return;
     }
     // ------------------------------ consumers ------------------------------
-    // one row per consumer thread: row0 + ct (conflict-free shared reads)
+    // Q rows per consumer thread: local rows ct + q*C (conflict-free shared reads)
     const int ct = threadIdx.x - 32;
     const int lane = ct & 31;
     int xs = 0, vs = 0;
@@ -576,26 +576,29 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
         const int32_t *xoff = plan + 2 + 2 * nwin;
         const int32_t *offs = a.pat_offs + P.off_begin;
         const T *xb = xbuf + (int64_t)xs * xmax_elems + ct;
-        const int64_t row = P.row0 + ct;
-        // scatter points: each warp gathers the entries of its own 32 rows
+        // scatter points: each warp gathers the entries owned by its threads
         // now (lane l takes entry l of the first 32 of the segment; a ballot
-        // keeps those in this warp's rows), so the random x loads are in
-        // flight during the diagonal loop; entries beyond 32 are read at the
-        // end (rare)
-        const int wrow0 = ct & ~31;
-        int g_row = -1;
+        // keeps the ones whose row belongs to this warp), so the random x
+        // loads are in flight during the diagonal loop; entries beyond 32 are
+        // read at the end (rare)
+        int g_own = -1;
         T g_v = T(0), g_x = T(0);
         unsigned g_mask = 0u;
         if (P.nscat > 0) {
-            if (lane < P.nscat) g_row = __ldg(a.scat_row + P.scat_begin + lane);
-            const bool mine = g_row >= wrow0 && g_row < wrow0 + 32;
+            if (lane < P.nscat) {
+                const int rr = __ldg(a.scat_row + P.scat_begin + lane);
+                g_own = (rr % C) * Q + rr / C;  // (thread, slot)
+            }
+            const bool mine = g_own >= 0 && (g_own / Q) / 32 == ct / 32;
             g_mask = __ballot_sync(0xffffffffu, mine);
             if (mine) {
                 g_v = __ldg(a.scat_val + P.scat_begin + lane);
                 g_x = __ldg(a.x + __ldg(a.scat_col + P.scat_begin + lane));
             }
         }
-        T acc = T(0);
+        T acc[Q];
+#pragma unroll
+        for (int q = 0; q < Q; ++q) acc[q] = T(0);
         for (int d0 = 0; d0 < P.nd; d0 += kch) {
             const int nk = min(kch, P.nd - d0);
             mbar_wait(full_v + vs, vph);
@@ -607,12 +610,19 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
                     if (k < nk) xo[k] = __ldg(xoff + d0 + k);
 #pragma unroll
                 for (int k = 0; k < KCH; ++k)
-                    if (k < nk) acc = fma(vb[k * C], xb[xo[k]], acc);
+                    if (k < nk) {
+#pragma unroll
+                        for (int q = 0; q < Q; ++q) acc[q] = fma(vb[k * a.mrows + q * C], xb[xo[k] + q * C], acc[q]);
+                    }
             } else {
                 for (int k = 0; k < nk; ++k) {
-                    const int64_t idx = row + __ldg(offs + d0 + k);
-                    const T xj = (idx >= a.x_lo && idx < a.x_hi) ? __ldg(a.x + idx) : T(0);
-                    acc = fma(vb[k * C], xj, acc);
+                    const int o = __ldg(offs + d0 + k);
+#pragma unroll
+                    for (int q = 0; q < Q; ++q) {
+                        const int64_t idx = P.row0 + ct + q * C + o;
+                        const T xj = (idx >= a.x_lo && idx < a.x_hi) ? __ldg(a.x + idx) : T(0);
+                        acc[q] = fma(vb[k * a.mrows + q * C], xj, acc[q]);
+                    }
                 }
             }
             __syncwarp();
@@ -624,25 +634,37 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(empty_x + xs);  // the x slot is no longer needed
-        // scatter points of this row in (row, col) order: the gathered ones
-        // (broadcast from the lane that holds them), then any beyond 32
+        // scatter points in (row, col) order: the gathered ones (broadcast
+        // from the lane that holds them), then any beyond 32
         if (P.nscat > 0) {
             for (unsigned m = g_mask; m; m &= m - 1) {
                 const int j = __ffs(m) - 1;
-                const int r = __shfl_sync(0xffffffffu, g_row, j);
+                const int own = __shfl_sync(0xffffffffu, g_own, j);
                 const T v = __shfl_sync(0xffffffffu, g_v, j);
                 const T xv = __shfl_sync(0xffffffffu, g_x, j);
-                if (r == ct) acc = fma(v, xv, acc);
+#pragma unroll
+                for (int q = 0; q < Q; ++q)
+                    if (own == ct * Q + q) acc[q] = fma(v, xv, acc[q]);
             }
             const int32_t *sr = a.scat_row + P.scat_begin;
             for (int64_t e = 32; e < P.nscat; ++e) {
-                if (__ldg(sr + e) != ct) continue;
-                acc = fma(__ldg(a.scat_val + P.scat_begin + e), __ldg(a.x + __ldg(a.scat_col + P.scat_begin + e)), acc);
+                const int rr = __ldg(sr + e);
+                if (rr % C != ct) continue;
+                const T v = __ldg(a.scat_val + P.scat_begin + e);
+                const T xv = __ldg(a.x + __ldg(a.scat_col + P.scat_begin + e));
+                const int qq = rr / C;
+#pragma unroll
+                for (int q = 0; q < Q; ++q)
+                    if (qq == q) acc[q] = fma(v, xv, acc[q]);
             }
         }
-        if (!edge || row < a.nrows) {
-            T *yp = a.y + row;
-            __stcs(yp, (be != T(0)) ? fma(al, acc, be * *yp) : al * acc);
+#pragma unroll
+        for (int q = 0; q < Q; ++q) {
+            const int64_t row = P.row0 + ct + q * C;
+            if (!edge || row < a.nrows) {
+                T *yp = a.y + row;
+                __stcs(yp, (be != T(0)) ? fma(al, acc[q], be * *yp) : al * acc[q]);
+            }
         }
         if (++xs == nx) {
             xs = 0;
@@ -691,27 +713,32 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
         if (g > 0x7fffffff) g = 0x7fffffff;
         kern<<<(unsigned)g, thr, smem, (cudaStream_t)stream>>>(a, split);
     } else if (a.variant == VARIANT_PIPE) {
-        // ring of KCH-diagonal value chunks; two CTAs per SM when the consumer
-        // count allows it (else one), nx x slots, as many stages as fit
+        // ring of KCH-diagonal value chunks; Q rows per consumer thread so a
+        // CTA has <= 256 consumers; two CTAs per SM, nx x slots, as many
+        // stages as fit
         constexpr int kch = 8;
         const int64_t xmax = a.pipe_xmax_elems;
-        const int per_sm = env_int("CRSD_PIPE_PERSM", a.mrows <= 256 ? 2 : 1);
+        const int q = env_int("CRSD_PIPE_Q", a.mrows > 256 ? a.mrows / 256 : 1);
+        const int C = a.mrows / q;
+        const int per_sm = env_int("CRSD_PIPE_PERSM", C <= 256 ? 2 : 1);
         const int64_t budget = (per_sm >= 2 ? 110 : 220) * 1024;
         int nx = env_int("CRSD_PIPE_NX", 2);
         while (nx > 2 && pipe_smem(2, nx, kch, a.mrows, sizeof(T), xmax) > budget) --nx;
         int ns = env_int("CRSD_PIPE_NS", 32);
         while (ns > 2 && pipe_smem(ns, nx, kch, a.mrows, sizeof(T), xmax) > budget) --ns;
         const int64_t sm = pipe_smem(ns, nx, kch, a.mrows, sizeof(T), xmax);
-        static int attr_pipe[2] = {0, 0};
-        int &cur = attr_pipe[sizeof(T) == 8];
+        static int attr_pipe[2][3] = {};
+        const int qi = q == 1 ? 0 : (q == 2 ? 1 : 2);
+        int &cur = attr_pipe[sizeof(T) == 8][qi];
+        auto kern = q == 1 ? crsd_spmv_pipe<T, kch, 1> : (q == 2 ? crsd_spmv_pipe<T, kch, 2> : crsd_spmv_pipe<T, kch, 4>);
         if (sm > cur) {
-            e = cudaFuncSetAttribute(crsd_spmv_pipe<T, kch>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+            e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
             if (e != cudaSuccess) return -(10000 + (int)e);
             cur = (int)sm;
         }
         int64_t g = (int64_t)sm_count * per_sm;
         if (g > a.seg_count) g = a.seg_count;
-        crsd_spmv_pipe<T, kch><<<(unsigned)g, a.mrows + 32, sm, (cudaStream_t)stream>>>(a, ns, nx, (int)xmax);
+        kern<<<(unsigned)g, C + 32, sm, (cudaStream_t)stream>>>(a, ns, nx, (int)xmax);
     } else {
         crsd_spmv_ldg<T, 4><<<(unsigned)grid, threads, 0, (cudaStream_t)stream>>>(a);
     }
