@@ -66,7 +66,8 @@ typedef enum { CRSD_R32F = 0, CRSD_R64F = 1 } crsd_dtype_t;
 
 /*
  * Build options. Call crsd_opts_init() for defaults (NULL opts == defaults).
- *   mrows     row-segment height (token `mrows`); 0 => 256. The
+ *   mrows     row-segment height (token `mrows`); 0 => 2 KB of
+ *             values per diagonal run: 256 (fp64) / 512 (fp32). The
  *             GPU path needs mrows % (32*RPT) == 0 and mrows <= 256*RPT,
  *             RPT = 2 rows per thread for fp64 and 4 for fp32 (one 128-bit
  *             vector per thread and diagonal; <= 256 threads per CTA); the

@@ -120,6 +120,7 @@ static void plan_layout(crsd_matrix_s *A) {
         int q = A->rpt;
         while (q > 1 && rc / q < 64) q /= 2;
         if (const char *e = getenv("CRSD_TMA_Q")) q = atoi(e);
+        while (rc / q > 256) q *= 2;  // <= 256 threads per CTA
         A->tma_q = q;
     }
     A->list_interior.clear();
@@ -195,11 +196,12 @@ static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_
     else {
         // AUTO, from the variant sweeps in profiles/r01_sweep*.jsonl: the
         // one-shot TMA kernel when a whole segment stages in <= 32 KB (enough
-        // CTAs per SM to keep ~200 KB in flight: C2 97-101% of the measured
-        // copy bandwidth); otherwise the chunked ring (PIPE) for fp64 (C3 81%)
-        // and the register variant for fp32 (C3 76%).
+        // CTAs per SM to keep ~200 KB in flight: C2 ~98 % fp64 / ~92 % fp32 of
+        // the measured copy bandwidth); otherwise the persistent chunked ring
+        // (PIPE: C3 83-87 % fp64, 81 % fp32); the register variant when
+        // neither staging fits in shared memory.
         if (A->tma_split == 1 && A->tma_smem <= 32 * 1024) A->variant = VARIANT_TMA;
-        else if (A->H.elem == 8 && pipe_need <= smem_cap && A->H.mrows <= 1024) A->variant = VARIANT_PIPE;
+        else if (pipe_need <= smem_cap && A->H.mrows <= 1024) A->variant = VARIANT_PIPE;
         else A->variant = VARIANT_LDG;
     }
     if (!A->host_only) {
@@ -227,7 +229,8 @@ static crsd_status_t resolve_opts(int64_t nrows, crsd_dtype_t dtype, const crsd_
                                   BuildOptions &b) {
     if (opts) o = *opts;
     else crsd_opts_init(&o);
-    if (o.mrows == 0) o.mrows = 256;
+    // default: 2 KB per diagonal run of a segment (256 fp64, 512 fp32)
+    if (o.mrows == 0) o.mrows = (dtype == CRSD_R64F) ? 256 : 512;
     if (o.idle_max < 0) o.idle_max = o.mrows - 1;
     if (o.row_begin == 0 && o.row_end == 0) o.row_end = nrows;
     b.mrows = o.mrows;
