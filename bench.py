@@ -395,6 +395,36 @@ def run_crsd(args):
             "transfer_bound_ms": round(max(a.ncols * es / h2d, a.nrows * es / d2h) / 1e6, 4),
             "path": "crsd_spmv_host: chunked H2D(x) / kernel / D2H(y) pipeline on three streams",
         }
+    if world > 1:
+        # e2e through crsd_spmv_dist: pinned host x slice -> owned part of
+        # x_padded, halo exchange + SpMV, y slice -> pinned host; max over ranks
+        xh = torch.from_numpy(np.random.default_rng(7 + rank).uniform(-1, 1, re - rb).astype(dt)).pin_memory()
+        yh = torch.empty(re - rb, dtype=tdt).pin_memory()
+
+        def e2e_step():
+            xp[lo : lo + nloc].copy_(xh, non_blocking=True)
+            A.spmv_dist(xp, y, 1.0, 0.0, comm)
+            yh.copy_(y, non_blocking=True)
+            torch.cuda.current_stream().synchronize()
+
+        for _ in range(2):
+            e2e_step()
+        ke = max(3, min(args.steps, 50))
+        dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(ke):
+            e2e_step()
+        te = torch.tensor([(time.perf_counter() - t0) / ke], dtype=torch.float64, device=f"cuda:{dev}")
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        te = float(te.item())
+        e2e = {
+            "value": round(2.0 * nnz_all / te / 1e9, 3),
+            "unit": "GFLOP/s",
+            "h2d_bytes_per_step": int((re - rb) * es) * world,
+            "d2h_bytes_per_step": int((re - rb) * es) * world,
+            "ms_per_step": round(te * 1e3, 4),
+            "path": "per rank: H2D of the owned x slice, crsd_spmv_dist (NCCL halo + SpMV), D2H of the y slice; max over ranks",
+        }
     if rank != 0:
         if comm is not None:
             comm.close()
