@@ -383,6 +383,21 @@ def run_crsd(args):
 
         h2d = bw(lambda: xd_tmp.copy_(xh, non_blocking=True), a.ncols * es)
         d2h = bw(lambda: yh.copy_(yd_tmp, non_blocking=True), a.nrows * es)
+        s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+
+        def both():  # H2D and D2H at the same time on two streams
+            with torch.cuda.stream(s1):
+                xd_tmp.copy_(xh, non_blocking=True)
+            with torch.cuda.stream(s2):
+                yh.copy_(yd_tmp, non_blocking=True)
+
+        bidir_ms = bw(both, 1e6) and None
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(5):
+            both()
+        torch.cuda.synchronize()
+        bidir_ms = (time.perf_counter() - t0) / 5 * 1e3
         del xd_tmp, yd_tmp
         e2e = {
             "value": round(2.0 * nnz_all / te / 1e9, 3),
@@ -393,6 +408,7 @@ def run_crsd(args):
             "pinned_h2d_gbs": round(h2d, 1),
             "pinned_d2h_gbs": round(d2h, 1),
             "transfer_bound_ms": round(max(a.ncols * es / h2d, a.nrows * es / d2h) / 1e6, 4),
+            "concurrent_h2d_d2h_ms": round(bidir_ms, 4),
             "path": "crsd_spmv_host: chunked H2D(x) / kernel / D2H(y) pipeline on three streams",
         }
     if world > 1:
