@@ -449,8 +449,6 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int sp
 // set by the ring depth, not by the segment size, and the descriptor and
 // window fetches of the next segment overlap the current one.
 // ---------------------------------------------------------------------------
-constexpr int PIPE_SG = 64;  // scatter points staged per segment by the gatherer warp
-
 struct PipeSeg {  // segment info handed from producer to consumers (per x slot)
     int64_t row0;
     int64_t scat_begin;
@@ -473,18 +471,13 @@ template <typename T, int KCH, int Q>
 __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, int ns, int nx, int xmax_elems) {
     constexpr int kch = KCH;
     extern __shared__ __align__(128) unsigned char smem[];
-    // layout: [bars: 4*nx + 2*ns][PipeSeg x nx][scatter staging x nx][xbuf x nx][vring x ns]
+    // layout: [bars: 2*nx + 2*ns][PipeSeg x nx][xbuf x nx][vring x ns]
     uint64_t *full_x = reinterpret_cast<uint64_t *>(smem);
     uint64_t *empty_x = full_x + nx;
-    uint64_t *full_s = full_x + 2 * nx;
-    uint64_t *empty_s = full_x + 3 * nx;
-    uint64_t *full_v = full_x + 4 * nx;
+    uint64_t *full_v = full_x + 2 * nx;
     uint64_t *empty_v = full_v + ns;
-    PipeSeg *sseg = reinterpret_cast<PipeSeg *>(smem + ((8 * (4 * nx + 2 * ns) + 127) / 128) * 128);
-    T *sg_v = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sseg) + ((nx * (int)sizeof(PipeSeg) + 127) / 128) * 128);
-    T *sg_x = sg_v + nx * PIPE_SG;
-    int32_t *sg_row = reinterpret_cast<int32_t *>(sg_x + nx * PIPE_SG);
-    T *xbuf = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sg_row) + ((nx * PIPE_SG * 4 + 127) / 128) * 128);
+    PipeSeg *sseg = reinterpret_cast<PipeSeg *>(smem + ((8 * (2 * nx + 2 * ns) + 127) / 128) * 128);
+    T *xbuf = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sseg) + ((nx * (int)sizeof(PipeSeg) + 127) / 128) * 128);
     T *vring = xbuf + nx * (int64_t)xmax_elems;
     const int C = a.mrows / Q;  // consumer threads (Q rows each)
     const int nwarps_c = C / 32;
@@ -494,8 +487,6 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
         for (int i = 0; i < nx; ++i) {
             mbar_init(full_x + i, 1);
             mbar_init(empty_x + i, nwarps_c);
-            mbar_init(full_s + i, 1);
-            mbar_init(empty_s + i, nwarps_c);
         }
         for (int i = 0; i < ns; ++i) {
             mbar_init(full_v + i, 1);
@@ -569,44 +560,9 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
         }
         return;
     }
-    if (threadIdx.x < 64) {
-        // ------------------------------ gatherer ------------------------------
-        // Warp 1 walks the same segments and gathers each one's scatter points
-        // (row, value, x[col]) into the slot's staging area, up to nx segments
-        // ahead of the consumers: the random x reads never sit on their path.
-        const int lane = threadIdx.x - 32;
-        int gs = 0;
-        uint32_t gph = 0;
-        auto seg_of = [&](int64_t w) { return a.seg_list ? (int64_t)__ldg(a.seg_list + w) : a.seg_begin + w; };
-        int64_t sg_next = (blockIdx.x < a.seg_count) ? seg_of(blockIdx.x) : 0;
-        SegDesc D_next;
-        if (blockIdx.x < a.seg_count) D_next = a.segs[sg_next];
-        for (int64_t w = blockIdx.x; w < a.seg_count; w += gridDim.x) {
-            const SegDesc D = D_next;
-            if (w + gridDim.x < a.seg_count) {
-                sg_next = seg_of(w + gridDim.x);
-                D_next = a.segs[sg_next];
-            }
-            if (lane == 0) mbar_wait(empty_s + gs, gph ^ 1);
-            __syncwarp();
-            const int nst = D.nscat < PIPE_SG ? D.nscat : PIPE_SG;
-            for (int e = lane; e < nst; e += 32) {
-                sg_row[gs * PIPE_SG + e] = __ldg(a.scat_row + D.scat_begin + e);
-                sg_v[gs * PIPE_SG + e] = __ldg(a.scat_val + D.scat_begin + e);
-                sg_x[gs * PIPE_SG + e] = __ldg(a.x + __ldg(a.scat_col + D.scat_begin + e));
-            }
-            __syncwarp();
-            if (lane == 0) mbar_arrive(full_s + gs);  // release: the staged entries
-            if (++gs == nx) {
-                gs = 0;
-                gph ^= 1;
-            }
-        }
-        return;
-    }
     // ------------------------------ consumers ------------------------------
     // Q rows per consumer thread: local rows ct + q*C (conflict-free shared reads)
-    const int ct = threadIdx.x - 64;
+    const int ct = threadIdx.x - 32;
     const int lane = ct & 31;
     int xs = 0, vs = 0;
     uint32_t xph = 0, vph = 0;
@@ -620,6 +576,26 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
         const int32_t *xoff = plan + 2 + 2 * nwin;
         const int32_t *offs = a.pat_offs + P.off_begin;
         const T *xb = xbuf + (int64_t)xs * xmax_elems + ct;
+        // scatter points: each warp gathers the entries owned by its threads
+        // now (lane l takes entry l of the first 32 of the segment; a ballot
+        // keeps the ones whose row belongs to this warp), so the random x
+        // loads are in flight during the diagonal loop; entries beyond 32 are
+        // read at the end (rare)
+        int g_own = -1;
+        T g_v = T(0), g_x = T(0);
+        unsigned g_mask = 0u;
+        if (P.nscat > 0) {
+            if (lane < P.nscat) {
+                const int rr = __ldg(a.scat_row + P.scat_begin + lane);
+                g_own = (rr % C) * Q + rr / C;  // (thread, slot)
+            }
+            const bool mine = g_own >= 0 && (g_own / Q) / 32 == ct / 32;
+            g_mask = __ballot_sync(0xffffffffu, mine);
+            if (mine) {
+                g_v = __ldg(a.scat_val + P.scat_begin + lane);
+                g_x = __ldg(a.x + __ldg(a.scat_col + P.scat_begin + lane));
+            }
+        }
         T acc[Q];
 #pragma unroll
         for (int q = 0; q < Q; ++q) acc[q] = T(0);
@@ -658,21 +634,20 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(empty_x + xs);  // the x slot is no longer needed
-        // scatter points in (row, col) order: the ones the gatherer warp
-        // staged for this slot, then any beyond PIPE_SG from global memory
+        // scatter points in (row, col) order: the gathered ones (broadcast
+        // from the lane that holds them), then any beyond 32
         if (P.nscat > 0) {
-            mbar_wait(full_s + xs, xph);
-            const int nst = P.nscat < PIPE_SG ? P.nscat : PIPE_SG;
-            for (int e = 0; e < nst; ++e) {
-                const int rr = sg_row[xs * PIPE_SG + e];
-                if (rr % C != ct) continue;
-                const int qq = rr / C;
+            for (unsigned m = g_mask; m; m &= m - 1) {
+                const int j = __ffs(m) - 1;
+                const int own = __shfl_sync(0xffffffffu, g_own, j);
+                const T v = __shfl_sync(0xffffffffu, g_v, j);
+                const T xv = __shfl_sync(0xffffffffu, g_x, j);
 #pragma unroll
                 for (int q = 0; q < Q; ++q)
-                    if (qq == q) acc[q] = fma(sg_v[xs * PIPE_SG + e], sg_x[xs * PIPE_SG + e], acc[q]);
+                    if (own == ct * Q + q) acc[q] = fma(v, xv, acc[q]);
             }
             const int32_t *sr = a.scat_row + P.scat_begin;
-            for (int64_t e = PIPE_SG; e < P.nscat; ++e) {
+            for (int64_t e = 32; e < P.nscat; ++e) {
                 const int rr = __ldg(sr + e);
                 if (rr % C != ct) continue;
                 const T v = __ldg(a.scat_val + P.scat_begin + e);
@@ -683,8 +658,6 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
                     if (qq == q) acc[q] = fma(v, xv, acc[q]);
             }
         }
-        __syncwarp();
-        if (lane == 0) mbar_arrive(empty_s + xs);  // every segment: keeps the phases in step
 #pragma unroll
         for (int q = 0; q < Q; ++q) {
             const int64_t row = P.row0 + ct + q * C;
@@ -702,10 +675,9 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
 
 // shared memory of the PIPE variant for nx x slots and ns value stages
 inline int64_t pipe_smem(int ns, int nx, int kch, int mrows, int elem, int64_t xmax_elems) {
-    const int64_t bars = ((8 * (4 * nx + 2 * ns) + 127) / 128) * 128;
+    const int64_t bars = ((8 * (2 * nx + 2 * ns) + 127) / 128) * 128;
     const int64_t segs = ((nx * (int64_t)sizeof(PipeSeg) + 127) / 128) * 128;
-    const int64_t stage = 2 * nx * PIPE_SG * elem + ((nx * PIPE_SG * 4 + 127) / 128) * 128;
-    return bars + segs + stage + nx * xmax_elems * elem + (int64_t)ns * kch * mrows * elem;
+    return bars + segs + nx * xmax_elems * elem + (int64_t)ns * kch * mrows * elem;
 }
 
 static int env_int(const char *k, int d) {
@@ -766,7 +738,7 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
         }
         int64_t g = (int64_t)sm_count * per_sm;
         if (g > a.seg_count) g = a.seg_count;
-        kern<<<(unsigned)g, C + 64, sm, (cudaStream_t)stream>>>(a, ns, nx, (int)xmax);
+        kern<<<(unsigned)g, C + 32, sm, (cudaStream_t)stream>>>(a, ns, nx, (int)xmax);
     } else {
         crsd_spmv_ldg<T, 4><<<(unsigned)grid, threads, 0, (cudaStream_t)stream>>>(a);
     }
