@@ -394,7 +394,8 @@ crsd_status_t crsd_spmv(crsd_matrix_t A, const void *alpha, const void *x, const
 static crsd_status_t e2e_setup(crsd_matrix_s *A) {
     HostCRSD &H = A->H;
     const int64_t nseg = H.nseg;
-    int nch = (int)std::min<int64_t>(16, std::max<int64_t>(1, nseg / 64));
+    const int want = getenv("CRSD_E2E_CHUNKS") ? atoi(getenv("CRSD_E2E_CHUNKS")) : 32;
+    int nch = (int)std::min<int64_t>(want, std::max<int64_t>(1, nseg / 32));
     A->e2e_nchunk = nch;
     A->e2e_seg.resize(nch + 1);
     A->e2e_xcut.resize(nch + 1);

@@ -180,7 +180,7 @@ def test_spmv_host_e2e(torch_cuda, dt, n, variant):
     yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, x)
     assert coo.parity_error(y2, yref, scale) <= TOL[dt]
     if n == 96:
-        assert A.last_launch_count() == 16
+        assert A.last_launch_count() > 8  # chunked pipeline
 
 
 # ---------------------------------------------------------------- full sizes
