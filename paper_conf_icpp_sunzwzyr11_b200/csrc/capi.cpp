@@ -59,12 +59,12 @@ void free_device(crsd_matrix_s *A) {
         cudaStreamDestroy((cudaStream_t)A->e2e_d2h);
         A->e2e_ready = false;
     }
-    void *ptrs[] = {A->d_vals, A->d_segs, A->d_offs, A->d_plan, A->d_scat_row, A->d_scat_col, A->d_scat_val,
+    void *ptrs[] = {A->d_vals, A->d_segs, A->d_offs, A->d_plan, A->d_scat_row, A->d_scat_col, A->d_scat_val, A->d_scat_rec,
                     A->d_list_interior, A->d_list_boundary, A->d_list_all_edge, A->d_x_scratch, A->d_y_scratch};
     if (A->device >= 0) cudaSetDevice(A->device);
     for (void *p : ptrs)
         if (p) cudaFree(p);
-    A->d_vals = A->d_segs = A->d_offs = A->d_plan = A->d_scat_row = A->d_scat_col = A->d_scat_val = nullptr;
+    A->d_vals = A->d_segs = A->d_offs = A->d_plan = A->d_scat_row = A->d_scat_col = A->d_scat_val = A->d_scat_rec = nullptr;
     A->d_list_interior = A->d_list_boundary = A->d_list_all_edge = A->d_x_scratch = A->d_y_scratch = nullptr;
 }
 
@@ -153,6 +153,17 @@ static crsd_status_t upload(crsd_matrix_s *A) {
     if ((st = dev_alloc_copy(&A->d_scat_row, H.scat_row.data(), ns * 4, cnt))) return st;
     if ((st = dev_alloc_copy(&A->d_scat_col, colrel.data(), ns * 8, cnt))) return st;
     if ((st = dev_alloc_copy(&A->d_scat_val, H.scat_val.data(), H.scat_val.size(), cnt))) return st;
+    {
+        std::vector<ScatRec> rec(ns);
+        for (int64_t e = 0; e < ns; ++e) {
+            ScatRec r{};
+            r.col = colrel[e];
+            r.row = H.scat_row[e];
+            std::memcpy(&r.val, H.scat_val.data() + e * H.elem, H.elem);
+            rec[e] = r;
+        }
+        if ((st = dev_alloc_copy(&A->d_scat_rec, rec.data(), ns * sizeof(ScatRec), cnt))) return st;
+    }
     if ((st = dev_alloc_copy(&A->d_list_interior, A->list_interior.data(), A->list_interior.size() * 4, cnt))) return st;
     if ((st = dev_alloc_copy(&A->d_list_boundary, A->list_boundary.data(), A->list_boundary.size() * 4, cnt))) return st;
     // the host copy of the bulk arrays is dropped after upload (export reads the device copy)
@@ -266,6 +277,7 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
     a.scat_row = (const int32_t *)A->d_scat_row;
     a.scat_col = (const int64_t *)A->d_scat_col;
     a.scat_val = (const T *)A->d_scat_val;
+    a.scat_rec = (const ScatRec *)A->d_scat_rec;
     a.x = x;
     a.x_lo = A->x_lo;
     a.x_hi = A->x_hi;

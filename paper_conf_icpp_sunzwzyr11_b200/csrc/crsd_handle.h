@@ -39,6 +39,7 @@ struct crsd_matrix_s {
     void *d_scat_row = nullptr;
     void *d_scat_col = nullptr;
     void *d_scat_val = nullptr;
+    void *d_scat_rec = nullptr;
     void *d_list_interior = nullptr;
     void *d_list_boundary = nullptr;
     void *d_list_all_edge = nullptr;

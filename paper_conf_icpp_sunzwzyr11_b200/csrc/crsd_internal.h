@@ -54,6 +54,17 @@ enum : int32_t { VARIANT_AUTO = 0, VARIANT_LDG = 1, VARIANT_TMA = 2, VARIANT_PIP
 
 static_assert(sizeof(SegDesc) == 32, "SegDesc must be 32 bytes");
 
+// Scatter point as one 32-byte record (col relative to the x base, value as
+// the matrix dtype in the first bytes of `val`, row within the segment), so a
+// segment's points can be staged with one bulk copy (PIPE kernel).
+struct alignas(16) ScatRec {
+    int64_t col;
+    double val;   // float matrices use the first 4 bytes
+    int32_t row;
+    int32_t pad[3];
+};
+static_assert(sizeof(ScatRec) == 32, "ScatRec must be 32 bytes");
+
 struct HostCRSD {
     int64_t nrows = 0, ncols = 0;    // global
     int64_t row_begin = 0, row_end = 0;
@@ -129,6 +140,7 @@ struct SpmvArgs {
     const int32_t *scat_row;
     const int64_t *scat_col;  // relative to x base
     const T *scat_val;
+    const ScatRec *scat_rec;  // same points as 32-byte records
     const T *x;               // local x base (x_padded + halo_lo for dist)
     int64_t x_lo, x_hi;       // valid x range relative to x
     T *y;

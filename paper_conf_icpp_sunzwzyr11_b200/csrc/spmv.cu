@@ -449,6 +449,8 @@ __global__ void __launch_bounds__(256) crsd_spmv_tma(const SpmvArgs<T> a, int sp
 // set by the ring depth, not by the segment size, and the descriptor and
 // window fetches of the next segment overlap the current one.
 // ---------------------------------------------------------------------------
+constexpr int PIPE_SR = 32;  // scatter records staged per segment (one per lane)
+
 struct PipeSeg {  // segment info handed from producer to consumers (per x slot)
     int64_t row0;
     int64_t scat_begin;
@@ -477,7 +479,8 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
     uint64_t *full_v = full_x + 2 * nx;
     uint64_t *empty_v = full_v + ns;
     PipeSeg *sseg = reinterpret_cast<PipeSeg *>(smem + ((8 * (2 * nx + 2 * ns) + 127) / 128) * 128);
-    T *xbuf = reinterpret_cast<T *>(reinterpret_cast<unsigned char *>(sseg) + ((nx * (int)sizeof(PipeSeg) + 127) / 128) * 128);
+    ScatRec *srec = reinterpret_cast<ScatRec *>(reinterpret_cast<unsigned char *>(sseg) + ((nx * (int)sizeof(PipeSeg) + 127) / 128) * 128);
+    T *xbuf = reinterpret_cast<T *>(srec + nx * PIPE_SR);
     T *vring = xbuf + nx * (int64_t)xmax_elems;
     const int C = a.mrows / Q;  // consumer threads (Q rows each)
     const int nwarps_c = C / 32;
@@ -531,7 +534,11 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
             uint32_t xbytes = 0;
             if (!edge)
                 for (int q = 0; q < nwin; ++q) xbytes += (uint32_t)__ldg(plan + 3 + 2 * q) * sizeof(T);
+            const int nrec = D.nscat < PIPE_SR ? D.nscat : PIPE_SR;
+            xbytes += (uint32_t)nrec * sizeof(ScatRec);
             mbar_expect_tx(full_x + xs, xbytes);  // arrive (release: P visible) + tx
+            if (nrec)
+                bulk_g2s(srec + xs * PIPE_SR, a.scat_rec + D.scat_begin, (uint32_t)nrec * sizeof(ScatRec), full_x + xs, pn);
             if (!edge) {
                 T *dst = xbuf + (int64_t)xs * xmax_elems;
                 for (int q = 0; q < nwin; ++q) {
@@ -585,15 +592,18 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
         T g_v = T(0), g_x = T(0);
         unsigned g_mask = 0u;
         if (P.nscat > 0) {
+            // the first PIPE_SR points arrived with the slot as 32-B records:
+            // only the x[col] gather is a global load, issued now
+            const ScatRec *R = srec + xs * PIPE_SR;
             if (lane < P.nscat) {
-                const int rr = __ldg(a.scat_row + P.scat_begin + lane);
+                const int rr = R[lane].row;
                 g_own = (rr % C) * Q + rr / C;  // (thread, slot)
             }
             const bool mine = g_own >= 0 && (g_own / Q) / 32 == ct / 32;
             g_mask = __ballot_sync(0xffffffffu, mine);
             if (mine) {
-                g_v = __ldg(a.scat_val + P.scat_begin + lane);
-                g_x = __ldg(a.x + __ldg(a.scat_col + P.scat_begin + lane));
+                g_v = *reinterpret_cast<const T *>(&R[lane].val);
+                g_x = __ldg(a.x + R[lane].col);
             }
         }
         T acc[Q];
@@ -677,7 +687,8 @@ __global__ void __launch_bounds__(544, 1) crsd_spmv_pipe(const SpmvArgs<T> a, in
 inline int64_t pipe_smem(int ns, int nx, int kch, int mrows, int elem, int64_t xmax_elems) {
     const int64_t bars = ((8 * (2 * nx + 2 * ns) + 127) / 128) * 128;
     const int64_t segs = ((nx * (int64_t)sizeof(PipeSeg) + 127) / 128) * 128;
-    return bars + segs + nx * xmax_elems * elem + (int64_t)ns * kch * mrows * elem;
+    const int64_t recs = nx * PIPE_SR * (int64_t)sizeof(ScatRec);
+    return bars + segs + recs + nx * xmax_elems * elem + (int64_t)ns * kch * mrows * elem;
 }
 
 static int env_int(const char *k, int d) {
