@@ -25,20 +25,21 @@ from __future__ import annotations
 import numpy as np
 
 
-def _coords(dims):
+def _coords(dims, row_begin=0, row_end=None):
     dims = list(dims) + [1] * (3 - len(dims))
     n = dims[0] * dims[1] * dims[2]
-    idx = np.arange(n, dtype=np.int64)
+    idx = np.arange(row_begin, n if row_end is None else row_end, dtype=np.int64)
     g = [idx % dims[0], (idx // dims[0]) % dims[1], idx // (dims[0] * dims[1])]
     p = [(g[k] + 1 < dims[k]).astype(np.int64) for k in range(3)]
     m = [(g[k] >= 1).astype(np.int64) for k in range(3)]
     return dims, g, p, m
 
 
-def stencil_apply(dims, kind: str, xkind: str, coef=None) -> np.ndarray:
+def stencil_apply(dims, kind: str, xkind: str, coef=None, row_begin=0, row_end=None) -> np.ndarray:
     """Exact A*x (float64) for the Dirichlet stencil of ``kind`` and
-    x = 'ones' | 'linear' (a + sum b_k g_k) | 'quadratic' (sum g_k^2)."""
-    dims, g, p, m = _coords(dims)
+    x = 'ones' | 'linear' (a + sum b_k g_k) | 'quadratic' (sum g_k^2),
+    for rows [row_begin, row_end) (default: all)."""
+    dims, g, p, m = _coords(dims, row_begin, row_end)
     if kind in ("5pt", "7pt"):
         c = 4 if kind == "5pt" else 6
         active = [0, 1] if kind == "5pt" else [0, 1, 2]

@@ -302,3 +302,80 @@ def test_nccl_comm_world1(torch_cuda):
         comm.close()
     finally:
         dist.destroy_process_group()
+
+
+def _host_ram_gb():
+    try:
+        import psutil
+
+        return psutil.virtual_memory().available / 2**30
+    except Exception:
+        return 0.0
+
+
+@pytest.mark.slow
+def test_c4_full_sampled(torch_cuda):
+    """BASELINE config 4 at full size (100M rows, 19 offsets / 4 patterns,
+    fp32) on one GPU in the AUTO variant, checked on a row sample that the
+    oracle evaluates one by one (plus every pattern boundary row)."""
+    if _host_ram_gb() < 120:
+        pytest.skip("needs ~120 GB of host RAM for the 1.19e9-entry COO")
+    torch = torch_cuda
+    n = 100_000_000
+    a = gen.config4(n=n).astype(np.float32)
+    A = _mat(a)
+    inf = A.info()
+    assert inf["nnz"] == a.nnz and inf["nscatter"] == 0
+    x = np.random.default_rng(9).uniform(-1, 1, n).astype(np.float32)
+    y = _run(torch, A, x, 1.0, 0.0, None, n)
+    del A
+    # row sample: random rows + the ends of every pattern range
+    rng = np.random.default_rng(10)
+    bounds = [r for lo, hi, _ in gen.matrices.c4_ranges(n) for r in (lo, hi - 1)]
+    rows = np.unique(np.concatenate([rng.integers(0, n, 20000), np.array(bounds), np.arange(0, 64), np.arange(n - 64, n)]))
+    ptr = np.zeros(n + 1, np.int64)
+    ptr[1:] = np.cumsum(np.bincount(a.row, minlength=n))
+    yref, scale = coo.rows_spmv(rows, ptr, a.col, a.val.astype(np.float64), x.astype(np.float64))
+    err = coo.parity_error(y[rows], yref, scale)
+    assert err <= TOL[np.float32], err
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("rank", [0, 3])
+def test_c5_rank_block_closed_form(torch_cuda, rank):
+    """BASELINE config 5 (7-pt 768^3, fp64) split into 8 row blocks as the
+    8-GPU run would: one rank's block is built with its global row range, its
+    x halo filled from the global x, and every row of the block is compared
+    with the closed form (exact integers) -- the full-size multi-GPU layout on
+    one GPU, without NCCL."""
+    if _host_ram_gb() < 48:
+        pytest.skip("needs ~48 GB of host RAM for a 56.6M-row block")
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, partition_rows
+
+    torch = torch_cuda
+    nn = 768
+    dims = (nn, nn, nn)
+    n = nn**3
+    bounds = partition_rows(n, 256, 8)
+    rb, re = int(bounds[rank]), int(bounds[rank + 1])
+    a = gen.config5(n=nn, values="exact", row_begin=rb, row_end=re)
+    A = CRSDMatrix.from_coo(n, n, a.row, a.col, a.val, row_range=(rb, re))
+    del a
+    inf = A.info()
+    lo, nloc, hi = A.x_layout()
+    hlv, hhv = inf["halo_lo_valid"], inf["halo_hi_valid"]
+    # halos: the +-768^2 diagonals (plus the vector-window slack of a few elements)
+    assert (hlv == 0 if rank == 0 else nn * nn <= hlv <= nn * nn + 8) and nn * nn <= hhv <= nn * nn + 8
+    coef = (3.0, (1.0, -2.0, 5.0))
+    g = gen.matrices.grid_coords(dims, rb - hlv, re + hhv)
+    xp = np.zeros(lo + nloc + hi)
+    xp[lo - hlv : lo + nloc + hhv] = coef[0] + coef[1][0] * g[0] + coef[1][1] * g[1] + coef[1][2] * g[2]
+    del g
+    xd = torch.from_numpy(xp).to("cuda")
+    del xp
+    yd = torch.full((nloc,), float("nan"), device="cuda", dtype=torch.float64)
+    A.spmv_dist(xd, yd, 1.0, 0.0, None)
+    torch.cuda.synchronize()
+    y = yd.cpu().numpy()
+    ref = closed_forms.stencil_apply(dims, "7pt", "linear", coef, rb, re)
+    assert np.array_equal(y, ref)
