@@ -406,7 +406,7 @@ crsd_status_t crsd_spmv(crsd_matrix_t A, const void *alpha, const void *x, const
 static crsd_status_t e2e_setup(crsd_matrix_s *A) {
     HostCRSD &H = A->H;
     const int64_t nseg = H.nseg;
-    const int want = getenv("CRSD_E2E_CHUNKS") ? atoi(getenv("CRSD_E2E_CHUNKS")) : 12;
+    const int want = getenv("CRSD_E2E_CHUNKS") ? atoi(getenv("CRSD_E2E_CHUNKS")) : 16;
     int nch = (int)std::min<int64_t>(want, std::max<int64_t>(1, nseg / 32));
     A->e2e_nchunk = nch;
     A->e2e_seg.resize(nch + 1);
