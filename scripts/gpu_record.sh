@@ -9,7 +9,7 @@ timeout 300 python __graft_entry__.py --smoke > gpurun_out/smoke.log 2>&1; echo 
 timeout 1200 python -m pytest tests -m gpu -q > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
 timeout 900 python bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_default.err
 timeout 900 python bench.py --impl reference --steps 5 --warmup 3 > gpurun_out/bench_reference.json 2> gpurun_out/bench_reference.err
-for cfg in "c2 f32" "c3 f64" "c3 f32"; do
+for cfg in "c2 f32" "c3 f64" "c3 f32" "c4 f32"; do
   set -- $cfg
   timeout 600 python bench.py --no-cpu --config $1 --dtype $2 > gpurun_out/bench_$1_$2.json 2> gpurun_out/bench_$1_$2.err
 done
