@@ -312,7 +312,7 @@ def run_crsd(args):
     kw = dict(device=dev)
     if args.mrows:
         kw["mrows"] = args.mrows
-    kw["variant"] = {"auto": 0, "ldg": 1, "tma": 2, "pipe": 3}[args.variant]
+    kw["variant"] = {"auto": 0, "ldg": 1, "tma": 2, "pipe": 3, "jit": 4}[args.variant]
     if world > 1:
         kw["row_range"] = (rb, re)
     t0 = time.perf_counter()
@@ -498,7 +498,7 @@ def run_crsd(args):
             "workload": desc,
             "nnz": int(nnz_all),
             "mrows": info["mrows"],
-            "kernel_variant": {1: "ldg", 2: "tma", 3: "pipe"}[info["variant"]],
+            "kernel_variant": {1: "ldg", 2: "tma", 3: "pipe", 4: "jit"}[info["variant"]],
             "alpha": 1.0,
             "beta": 0.0,
             "patterns": info["npat"],
@@ -512,7 +512,7 @@ def run_crsd(args):
         "hbm_frac_of_peak": round(ub_all / (ms * 1e-3) / 1e9 / (peak * world), 4),
         "roofline": {
             "bound": "hbm",
-            "kernel": {1: "crsd_spmv_ldg", 2: "crsd_spmv_tma", 3: "crsd_spmv_pipe"}[info["variant"]],
+            "kernel": {1: "crsd_spmv_ldg", 2: "crsd_spmv_tma", 3: "crsd_spmv_pipe", 4: "crsd_jit"}[info["variant"]],
             "achieved": round(achieved, 1),
             "peak": peak,
             "peak_source": peak_src,
@@ -546,7 +546,7 @@ def main():
     ap.add_argument("--config", default="c2", choices=["c2", "c3", "c3ns", "c4"])
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
     ap.add_argument("--mrows", type=int, default=0)
-    ap.add_argument("--variant", default="auto", choices=["auto", "ldg", "tma", "pipe"])
+    ap.add_argument("--variant", default="auto", choices=["auto", "ldg", "tma", "pipe", "jit"])
     ap.add_argument("--impl", default="crsd", choices=["crsd", "reference"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()

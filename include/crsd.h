@@ -86,8 +86,11 @@ typedef enum { CRSD_R32F = 0, CRSD_R64F = 1 } crsd_dtype_t;
  *             per segment, bulk copies of its values and x windows into
  *             shared memory) or CRSD_VARIANT_PIPE (3: persistent CTAs, a
  *             producer warp streams value chunks through a shared-memory
- *             ring with TMA bulk copies). AUTO picks PIPE when the largest
- *             pattern's x windows fit in shared memory, else LDG. DESIGN.md
+ *             ring with TMA bulk copies) or CRSD_VARIANT_JIT (4: the TMA
+ *             data movement with every pattern quantity baked into a
+ *             runtime-generated codelet, NVRTC; the paper's code generator,
+ *             P:L131-143). AUTO picks TMA for small segments, PIPE for large
+ *             ones, LDG when neither staging fits in shared memory. DESIGN.md
  *             "Kernels".
  */
 typedef struct {
@@ -105,6 +108,7 @@ typedef struct {
 #define CRSD_VARIANT_LDG 1
 #define CRSD_VARIANT_TMA 2
 #define CRSD_VARIANT_PIPE 3
+#define CRSD_VARIANT_JIT 4
 
 typedef struct crsd_matrix_s *crsd_matrix_t;
 typedef struct crsd_comm_s *crsd_comm_t;
@@ -278,6 +282,14 @@ crsd_status_t crsd_partition_rows(int64_t nrows, int32_t mrows, int world, const
 /* Introspection */
 crsd_status_t crsd_get_info(crsd_matrix_t A, crsd_info_t *info);
 crsd_status_t crsd_export(crsd_matrix_t A, crsd_export_t *out);
+
+/* The CUDA source of the per-pattern codelets the JIT variant compiles for A
+ * (the paper's generated codelets): one `case` per distinct
+ * pattern with offsets, x windows and shapes as literals. buf (HOST, may be
+ * NULL) receives up to cap-1 bytes plus a NUL; *len the full length. Works on
+ * host-only handles (no GPU needed). UNSUPPORTED if a segment's staging
+ * (values + x windows) exceeds 200 KB of shared memory. */
+crsd_status_t crsd_jit_source(crsd_matrix_t A, char *buf, int64_t cap, int64_t *len);
 
 /* Number of kernel launches the last crsd_spmv / crsd_spmv_dist call made. */
 crsd_status_t crsd_last_launch_count(crsd_matrix_t A, int32_t *count);

@@ -75,6 +75,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         "-Xlinker",
         f"-rpath,{libdir}",
         "-lgomp",
+        "-ldl",
     ]
     subprocess.check_call(link)
     return LIB

@@ -27,7 +27,7 @@ STATUS = {
 }
 CRSD_R32F, CRSD_R64F = 0, 1
 CRSD_SUM_DUPLICATES, CRSD_HOST_ONLY, CRSD_DROP_ZEROS = 0x1, 0x2, 0x4
-VARIANT_AUTO, VARIANT_LDG, VARIANT_TMA, VARIANT_PIPE = 0, 1, 2, 3
+VARIANT_AUTO, VARIANT_LDG, VARIANT_TMA, VARIANT_PIPE, VARIANT_JIT = 0, 1, 2, 3, 4
 
 # every symbol include/crsd.h declares
 EXPORTED = [
@@ -50,6 +50,7 @@ EXPORTED = [
     "crsd_get_info",
     "crsd_export",
     "crsd_last_launch_count",
+    "crsd_jit_source",
 ]
 
 
@@ -133,6 +134,7 @@ def _load():
         "crsd_get_info": ([P, P], ctypes.c_int),
         "crsd_export": ([P, P], ctypes.c_int),
         "crsd_last_launch_count": ([P, P], ctypes.c_int),
+        "crsd_jit_source": ([P, P, I64, P], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)
@@ -318,6 +320,14 @@ class CRSDMatrix:
         lo, n, hi = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
         _check(lib.crsd_dist_x_layout(self._h, ctypes.byref(lo), ctypes.byref(n), ctypes.byref(hi)))
         return lo.value, n.value, hi.value
+
+    def jit_source(self) -> str:
+        """CUDA source of the JIT variant's per-pattern codelets."""
+        n = ctypes.c_int64()
+        _check(lib.crsd_jit_source(self._h, None, 0, ctypes.byref(n)))
+        buf = ctypes.create_string_buffer(n.value + 1)
+        _check(lib.crsd_jit_source(self._h, buf, n.value + 1, ctypes.byref(n)))
+        return buf.value.decode()
 
     def last_launch_count(self) -> int:
         c = ctypes.c_int32()

@@ -47,6 +47,7 @@ static crsd_status_t dev_alloc_copy(void **dptr, const void *src, size_t bytes, 
 }
 
 void free_device(crsd_matrix_s *A) {
+    jit_free(A);
     if (A->e2e_ready) {
         if (A->device >= 0) cudaSetDevice(A->device);
         cudaStreamSynchronize((cudaStream_t)A->e2e_h2d);
@@ -201,7 +202,8 @@ static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_
         delete A;
         return fail(CRSD_ERR_UNSUPPORTED, "PIPE variant: mrows must be <= 1024");
     }
-    if (o.variant == CRSD_VARIANT_LDG) A->variant = VARIANT_LDG;
+    if (o.variant == CRSD_VARIANT_JIT) A->variant = VARIANT_JIT;
+    else if (o.variant == CRSD_VARIANT_LDG) A->variant = VARIANT_LDG;
     else if (o.variant == CRSD_VARIANT_TMA) A->variant = VARIANT_TMA;
     else if (o.variant == CRSD_VARIANT_PIPE) A->variant = VARIANT_PIPE;
     else {
@@ -226,6 +228,7 @@ static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_
                                                   std::to_string(o.mrows) + " (use CRSD_HOST_ONLY for inspection)");
         }
         crsd_status_t st = upload(A);
+        if (!st && A->variant == VARIANT_JIT) st = jit_build(A);
         if (st) {
             free_device(A);
             delete A;
@@ -289,7 +292,7 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
     a.mrows = A->H.mrows;
     a.alpha = alpha;
     a.beta = beta;
-    int n = launch_spmv<T>(a, A->sm_count, stream);
+    int n = A->variant == VARIANT_JIT ? jit_launch<T>(A, a, stream) : launch_spmv<T>(a, A->sm_count, stream);
     if (n <= -10000)
         return fail(CRSD_ERR_CUDA, std::string("cudaFuncSetAttribute(MaxDynamicSharedMemorySize=") +
                                        std::to_string(a.smem_bytes) + "): " + cudaGetErrorString((cudaError_t)(-n - 10000)));

@@ -2,6 +2,7 @@
 #pragma once
 
 #include <cstdint>
+#include <string>
 #include <vector>
 
 #include "crsd_internal.h"
@@ -17,6 +18,10 @@ struct crsd_matrix_s {
     int64_t smem_bytes = 0;
     int64_t xmax_elems = 0;
     int tma_split = 1, tma_q = 2;
+    // JIT variant: generated source, loaded module and kernel (CUmodule / CUfunction)
+    std::string jit_source;
+    void *jit_module = nullptr;
+    void *jit_function = nullptr;
     int64_t tma_smem = 0;
     std::vector<int32_t> plan;
     int32_t last_launches = 0;
@@ -64,6 +69,11 @@ struct crsd_matrix_s {
 
 namespace crsd {
 void free_device(crsd_matrix_s *A);
+std::string jit_generate(const crsd_matrix_s *A);
+crsd_status_t jit_build(crsd_matrix_s *A);
+void jit_free(crsd_matrix_s *A);
+template <typename T>
+int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &a, void *stream);
 // Run the SpMV kernel over a device list of segments (list == nullptr: all
 // segments [0, count)). x_base is the local x base (x_padded + halo_lo).
 crsd_status_t run_lists(crsd_matrix_s *A, const void *alpha, const void *x_base, const void *beta, void *y,

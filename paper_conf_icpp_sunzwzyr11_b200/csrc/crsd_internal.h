@@ -42,7 +42,7 @@ struct alignas(16) SegDesc {
 constexpr int MAX_NDIAS = 4096;
 
 // Kernel variants
-enum : int32_t { VARIANT_AUTO = 0, VARIANT_LDG = 1, VARIANT_TMA = 2, VARIANT_PIPE = 3 };
+enum : int32_t { VARIANT_AUTO = 0, VARIANT_LDG = 1, VARIANT_TMA = 2, VARIANT_PIPE = 3, VARIANT_JIT = 4 };
 
 // TMA staging plan of one distinct pattern (int32 words at plan_begin):
 //   [0] nwin  [1] smem bytes (values + windows)

@@ -1,0 +1,335 @@
+// Runtime code generation of per-pattern SpMV codelets (variant JIT).
+//
+// The paper's mechanism: after
+// the matrix is stored in CRSD, a generator emits one `case` of a `switch` per
+// diagonal pattern with the index information baked into the code, and the
+// kernel is compiled at runtime (OpenCL there, NVRTC here). Only the values
+// (and x, y) are read at SpMV time.
+//
+// The generated kernel has the data movement of the TMA variant (one CTA per
+// segment, thread 0 bulk-copies the segment's value block, warp 0 the x
+// windows, one mbarrier), but every pattern-dependent quantity is a literal:
+// the diagonal count, the window starts/lengths, each diagonal's offset into
+// the staged x, the offsets for the guarded edge path. The codelet for a
+// pattern is fully unrolled. NVRTC (libnvrtc.so.12) and the CUDA
+// driver API are resolved at runtime (dlopen / cudaGetDriverEntryPoint), so
+// libcrsd.so loads on machines without them.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <nvrtc.h>
+
+#include <algorithm>
+#include <cstring>
+#include <mutex>
+#include <sstream>
+#include <string>
+#include <vector>
+
+#include "crsd_handle.h"
+#include "crsd_internal.h"
+
+namespace crsd {
+
+namespace {
+
+struct NvrtcApi {
+    bool ok = false;
+    std::string err;
+    nvrtcResult (*create)(nvrtcProgram *, const char *, const char *, int, const char *const *, const char *const *);
+    nvrtcResult (*compile)(nvrtcProgram, int, const char *const *);
+    nvrtcResult (*cubin_size)(nvrtcProgram, size_t *);
+    nvrtcResult (*cubin)(nvrtcProgram, char *);
+    nvrtcResult (*log_size)(nvrtcProgram, size_t *);
+    nvrtcResult (*log)(nvrtcProgram, char *);
+    nvrtcResult (*destroy)(nvrtcProgram *);
+};
+
+struct DriverApi {
+    bool ok = false;
+    std::string err;
+    CUresult (*load)(CUmodule *, const void *);
+    CUresult (*get_function)(CUfunction *, CUmodule, const char *);
+    CUresult (*launch)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, CUstream,
+                       void **, void **);
+    CUresult (*set_attr)(CUfunction, CUfunction_attribute, int);
+    CUresult (*unload)(CUmodule);
+};
+
+NvrtcApi &nvrtc() {
+    static NvrtcApi api;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        const char *names[] = {"libnvrtc.so.12", "/usr/local/cuda/lib64/libnvrtc.so.12", "libnvrtc.so"};
+        void *h = nullptr;
+        for (const char *n : names)
+            if ((h = dlopen(n, RTLD_NOW | RTLD_GLOBAL))) break;
+        if (!h) {
+            api.err = "libnvrtc.so.12 not found";
+            return;
+        }
+#define SYM(field, name)                                         \
+    api.field = reinterpret_cast<decltype(api.field)>(dlsym(h, name)); \
+    if (!api.field) {                                            \
+        api.err = std::string("missing ") + name;                \
+        return;                                                  \
+    }
+        SYM(create, "nvrtcCreateProgram");
+        SYM(compile, "nvrtcCompileProgram");
+        SYM(cubin_size, "nvrtcGetCUBINSize");
+        SYM(cubin, "nvrtcGetCUBIN");
+        SYM(log_size, "nvrtcGetProgramLogSize");
+        SYM(log, "nvrtcGetProgramLog");
+        SYM(destroy, "nvrtcDestroyProgram");
+#undef SYM
+        api.ok = true;
+    });
+    return api;
+}
+
+DriverApi &driver() {
+    static DriverApi api;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        auto get = [&](const char *name, void **fn) {
+            cudaDriverEntryPointQueryResult q;
+            return cudaGetDriverEntryPoint(name, fn, cudaEnableDefault, &q) == cudaSuccess &&
+                   q == cudaDriverEntryPointSuccess && *fn;
+        };
+        void *p;
+        if (!get("cuModuleLoadData", &p)) { api.err = "cuModuleLoadData"; return; }
+        api.load = reinterpret_cast<decltype(api.load)>(p);
+        if (!get("cuModuleGetFunction", &p)) { api.err = "cuModuleGetFunction"; return; }
+        api.get_function = reinterpret_cast<decltype(api.get_function)>(p);
+        if (!get("cuLaunchKernel", &p)) { api.err = "cuLaunchKernel"; return; }
+        api.launch = reinterpret_cast<decltype(api.launch)>(p);
+        if (!get("cuFuncSetAttribute", &p)) { api.err = "cuFuncSetAttribute"; return; }
+        api.set_attr = reinterpret_cast<decltype(api.set_attr)>(p);
+        if (!get("cuModuleUnload", &p)) { api.err = "cuModuleUnload"; return; }
+        api.unload = reinterpret_cast<decltype(api.unload)>(p);
+        api.ok = true;
+    });
+    return api;
+}
+
+// Arguments of the generated kernel (mirrored in the generated source).
+template <typename T>
+struct JitArgs {
+    const T *vals;
+    const SegDesc *segs;
+    const int32_t *seg_list;
+    int64_t seg_begin, seg_count;
+    const T *x;
+    int64_t x_lo, x_hi;
+    T *y;
+    int64_t nrows;
+    const int32_t *scat_row;
+    const int64_t *scat_col;
+    const T *scat_val;
+    T alpha, beta;
+};
+
+const char *kPrelude = R"(
+typedef long long i64;
+typedef unsigned long long u64;
+typedef unsigned int u32;
+typedef unsigned short u16;
+struct SegDesc { i64 val_base; i64 scat_begin; int off_begin; int nscat; u16 flags; u16 ndias; int plan_begin; };
+struct Args { const T *vals; const SegDesc *segs; const int *seg_list; i64 seg_begin, seg_count;
+              const T *x; i64 x_lo, x_hi; T *y; i64 nrows;
+              const int *scat_row; const i64 *scat_col; const T *scat_val; T alpha, beta; };
+__device__ __forceinline__ u32 su32(const void *p) { return (u32)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void bar_init(u64 *b) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(su32(b)) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
+__device__ __forceinline__ void bar_expect(u64 *b, u32 n) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(su32(b)), "r"(n) : "memory"); }
+__device__ __forceinline__ void bar_wait(u64 *b) {
+  u32 done = 0;
+  while (!done) asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0; selp.u32 %0, 1, 0, p; }"
+                             : "=r"(done) : "r"(su32(b)) : "memory"); }
+__device__ __forceinline__ u64 pol_first() { u64 p; asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p)); return p; }
+__device__ __forceinline__ u64 pol_normal() { u64 p; asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p)); return p; }
+__device__ __forceinline__ void g2s(void *dst, const void *src, u32 bytes, u64 *b, u64 pol) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+               :: "r"(su32(dst)), "l"(src), "r"(bytes), "r"(su32(b)), "l"(pol) : "memory"); }
+)";
+
+}  // namespace
+
+// Generate the codelets of every distinct pattern of A (TMA data movement,
+// whole segment per CTA, Q rows per thread).
+static std::string generate(const crsd_matrix_s *A, int Q) {
+    const HostCRSD &H = A->H;
+    const bool f64 = H.dtype == CRSD_R64F;
+    const int m = H.mrows, nt = m / Q, es = H.elem;
+    std::ostringstream o;
+    o << "typedef " << (f64 ? "double" : "float") << " T;\n" << kPrelude;
+    o << "#define MROWS " << m << "\n#define NT " << nt << "\n#define Q " << Q << "\n";
+    // one __device__ codelet per distinct pattern
+    std::vector<int32_t> seen;
+    for (const Instance &I : H.inst) {
+        const int32_t off_begin = (int32_t)H.pat_ptr[I.pattern];
+        bool dup = false;
+        for (int32_t v : seen) dup |= (v == off_begin);
+        if (dup) continue;
+        seen.push_back(off_begin);
+        const int32_t *pl = A->plan.data() + A->segdesc[I.first_seg].plan_begin;
+        const int nd = (int)H.ndias(I.pattern), nwin = pl[0];
+        const int64_t *offs = H.pat_offsets.data() + H.pat_ptr[I.pattern];
+        o << "// pattern offsets:";
+        for (int d = 0; d < nd; ++d) o << " " << offs[d];
+        o << "\n__device__ __forceinline__ void codelet_" << off_begin
+          << "(const Args &a, const SegDesc &D, i64 row0, bool edge, T *vs, u64 *bar, int t) {\n";
+        int64_t xb = 0;
+        for (int w = 0; w < nwin; ++w) xb += pl[3 + 2 * w];
+        o << "  T *xs = vs + " << (int64_t)nd * m << ";\n";
+        o << "  if (t == 0) { bar_init(bar); bar_expect(bar, " << (int64_t)nd * m * es << "u + (edge ? 0u : "
+          << xb * es << "u));\n";
+        if (nd) o << "    g2s(vs, a.vals + D.val_base, " << (int64_t)nd * m * es << "u, bar, pol_first()); }\n";
+        else o << "  }\n";
+        o << "  __syncthreads();\n";
+        if (nwin) {
+            o << "  if (!edge && t < 32) { const u64 pn = pol_normal();\n";
+            int64_t base = 0;
+            for (int w = 0; w < nwin; ++w) {
+                o << "    if (t == " << (w % 32) << ") g2s(xs + " << base << ", a.x + row0 + (" << pl[2 + 2 * w] << "), "
+                  << (int64_t)pl[3 + 2 * w] * es << "u, bar, pn);\n";
+                base += pl[3 + 2 * w];
+            }
+            o << "  }\n";
+        }
+        o << "  T acc[Q];\n#pragma unroll\n  for (int q = 0; q < Q; ++q) acc[q] = T(0);\n";
+        o << "  bar_wait(bar);\n";
+        const int32_t *xoff = pl + 2 + 2 * nwin;
+        o << "  if (!edge) {\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n      const int r = t + q * NT;\n";
+        for (int d = 0; d < nd; ++d)
+            o << "      acc[q] = fma(vs[" << (int64_t)d * m << " + r], xs[" << xoff[d] << " + r], acc[q]);\n";
+        o << "    }\n  } else {\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n      const i64 r = row0 + t + q * NT;\n";
+        for (int d = 0; d < nd; ++d)
+            o << "      { const i64 i = r + (" << offs[d] << "); acc[q] = fma(vs[" << (int64_t)d * m
+              << " + t + q * NT], (i >= a.x_lo && i < a.x_hi) ? __ldg(a.x + i) : T(0), acc[q]); }\n";
+        o << "    }\n  }\n";
+        // scatter points (owner thread, (row, col) order) and the epilogue
+        o << "  for (int e = 0; e < D.nscat; ++e) {\n"
+             "    const int rr = __ldg(a.scat_row + D.scat_begin + e);\n"
+             "    if (rr % NT != t) continue;\n"
+             "    const T v = __ldg(a.scat_val + D.scat_begin + e), xv = __ldg(a.x + __ldg(a.scat_col + D.scat_begin + e));\n"
+             "#pragma unroll\n    for (int q = 0; q < Q; ++q) if (rr / NT == q) acc[q] = fma(v, xv, acc[q]);\n  }\n";
+        o << "#pragma unroll\n  for (int q = 0; q < Q; ++q) {\n    const i64 r = row0 + t + q * NT;\n"
+             "    if (!edge || r < a.nrows) { T *yp = a.y + r; __stcs(yp, (a.beta != T(0)) ? fma(a.alpha, acc[q], a.beta * *yp) : a.alpha * acc[q]); }\n"
+             "  }\n}\n";
+    }
+    o << "extern \"C\" __global__ void __launch_bounds__(NT) crsd_jit(const Args a) {\n"
+         "  extern __shared__ __align__(128) unsigned char smem[];\n  __shared__ u64 bar;\n"
+         "  const i64 s = a.seg_list ? (i64)__ldg(a.seg_list + blockIdx.x) : a.seg_begin + blockIdx.x;\n"
+         "  const SegDesc D = a.segs[s];\n  const i64 row0 = s * MROWS;\n  const bool edge = (D.flags & 1) != 0;\n"
+         "  T *vs = reinterpret_cast<T *>(smem);\n  switch (D.off_begin) {\n";
+    for (int32_t v : seen) o << "  case " << v << ": codelet_" << v << "(a, D, row0, edge, vs, &bar, threadIdx.x); break;\n";
+    o << "  }\n}\n";
+    return o.str();
+}
+
+// rows per thread of the generated kernel: <= 256 threads per CTA
+static int jit_q(const crsd_matrix_s *A) {
+    int q = 1;
+    while (A->H.mrows / q > 256) q *= 2;
+    return q;
+}
+
+std::string jit_generate(const crsd_matrix_s *A) { return generate(A, jit_q(A)); }
+
+crsd_status_t jit_build(crsd_matrix_s *A) {
+    NvrtcApi &nv = nvrtc();
+    if (!nv.ok) return fail(CRSD_ERR_UNSUPPORTED, "JIT variant: " + nv.err);
+    DriverApi &dr = driver();
+    if (!dr.ok) return fail(CRSD_ERR_UNSUPPORTED, "JIT variant: driver entry point " + dr.err);
+    if (A->smem_bytes > 200 * 1024) return fail(CRSD_ERR_UNSUPPORTED, "JIT variant: a segment's staging exceeds 200 KB");
+    if (A->H.npat() > 256) return fail(CRSD_ERR_UNSUPPORTED, "JIT variant: more than 256 distinct patterns");
+    const int Q = jit_q(A);
+    A->jit_source = generate(A, Q);
+    nvrtcProgram prog;
+    if (nv.create(&prog, A->jit_source.c_str(), "crsd_jit.cu", 0, nullptr, nullptr) != NVRTC_SUCCESS)
+        return fail(CRSD_ERR_CUDA, "nvrtcCreateProgram failed");
+    const char *opts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-default-device", "-lineinfo"};
+    nvrtcResult r = nv.compile(prog, 4, opts);
+    if (r != NVRTC_SUCCESS) {
+        size_t n = 0;
+        nv.log_size(prog, &n);
+        std::string log(n, '\0');
+        nv.log(prog, &log[0]);
+        nv.destroy(&prog);
+        return fail(CRSD_ERR_CUDA, "NVRTC compile failed: " + log.substr(0, 2000));
+    }
+    size_t n = 0;
+    nv.cubin_size(prog, &n);
+    std::vector<char> cubin(n);
+    nv.cubin(prog, cubin.data());
+    nv.destroy(&prog);
+    CUmodule mod;
+    CUfunction fn;
+    if (dr.load(&mod, cubin.data()) != CUDA_SUCCESS) return fail(CRSD_ERR_CUDA, "cuModuleLoadData failed");
+    if (dr.get_function(&fn, mod, "crsd_jit") != CUDA_SUCCESS) {
+        dr.unload(mod);
+        return fail(CRSD_ERR_CUDA, "cuModuleGetFunction(crsd_jit) failed");
+    }
+    if (A->smem_bytes > 48 * 1024 &&
+        dr.set_attr(fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)A->smem_bytes) != CUDA_SUCCESS) {
+        dr.unload(mod);
+        return fail(CRSD_ERR_CUDA, "cuFuncSetAttribute failed");
+    }
+    A->jit_module = mod;
+    A->jit_function = fn;
+    return CRSD_OK;
+}
+
+void jit_free(crsd_matrix_s *A) {
+    if (A->jit_module && driver().ok) driver().unload((CUmodule)A->jit_module);
+    A->jit_module = nullptr;
+    A->jit_function = nullptr;
+}
+
+template <typename T>
+int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
+    if (s.seg_count <= 0) return 0;
+    JitArgs<T> j;
+    j.vals = s.vals;
+    j.segs = s.segs;
+    j.seg_list = s.seg_list;
+    j.seg_begin = s.seg_begin;
+    j.seg_count = s.seg_count;
+    j.x = s.x;
+    j.x_lo = s.x_lo;
+    j.x_hi = s.x_hi;
+    j.y = s.y;
+    j.nrows = s.nrows;
+    j.scat_row = s.scat_row;
+    j.scat_col = s.scat_col;
+    j.scat_val = s.scat_val;
+    j.alpha = s.alpha;
+    j.beta = s.beta;
+    void *params[] = {&j};
+    const unsigned nt = (unsigned)(A->H.mrows / jit_q(A));
+    CUresult r = driver().launch((CUfunction)A->jit_function, (unsigned)s.seg_count, 1, 1, nt, 1, 1,
+                                 (unsigned)A->smem_bytes, (CUstream)stream, params, nullptr);
+    return r == CUDA_SUCCESS ? 1 : -(int)cudaErrorLaunchFailure;
+}
+
+template int jit_launch<double>(const crsd_matrix_s *, const SpmvArgs<double> &, void *);
+template int jit_launch<float>(const crsd_matrix_s *, const SpmvArgs<float> &, void *);
+
+}  // namespace crsd
+
+extern "C" crsd_status_t crsd_jit_source(crsd_matrix_t A, char *buf, int64_t cap, int64_t *len) {
+    if (!A || !len) return crsd::fail(CRSD_ERR_INVALID_ARG, "NULL argument");
+    if (A->smem_bytes > 200 * 1024)
+        return crsd::fail(CRSD_ERR_UNSUPPORTED, "JIT codelets need a segment's staging <= 200 KB");
+    const std::string src = A->jit_source.empty() ? crsd::jit_generate(A) : A->jit_source;
+    *len = (int64_t)src.size();
+    if (buf && cap > 0) {
+        const int64_t n = std::min<int64_t>(cap - 1, (int64_t)src.size());
+        std::memcpy(buf, src.data(), n);
+        buf[n] = 0;
+    }
+    return CRSD_OK;
+}

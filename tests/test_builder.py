@@ -185,3 +185,32 @@ def test_unique_bytes_accounting():
     n = a.nrows
     assert inf["unique_bytes_beta0"] == inf["nslots"] * 8 + n * 8 + n * 8
     assert inf["unique_bytes_beta1"] == inf["unique_bytes_beta0"] + n * 8
+
+
+@pytest.mark.parametrize("case", ["c1", "c2s", "c3s", "rand"])
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_jit_codelets_compile_for_sm100a(case, dt, tmp_path):
+    """The JIT variant's generated per-pattern codelets (the paper's code
+    generator, P:L131-143, P:L687-701) compile for sm_100a, with one case per
+    distinct pattern and the pattern offsets baked in as literals."""
+    import subprocess
+
+    if case == "c1":
+        a = gen.config1()
+    elif case == "c2s":
+        a = gen.config2(n=24)
+    elif case == "c3s":
+        a = gen.config3(n=20)
+    else:
+        a = gen.random_diagonal(3000, 3000, 3, ndiag=8, max_off=400, n_scatter=40)
+    a = a.astype(dt)
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, host_only=True, variant=4)
+    src = A.jit_source()
+    P = A.export()
+    assert src.count("case ") == A.info()["npat"]
+    for offs in P["inst_offsets"]:
+        assert "// pattern offsets: " + " ".join(str(o) for o in offs) in src
+    f = tmp_path / "k.cu"
+    f.write_text(src)
+    r = subprocess.run(["/usr/local/cuda/bin/nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-std=c++17", "-c", str(f), "-o", str(tmp_path / "k.o")], capture_output=True, text=True)
+    assert r.returncode == 0, r.stderr[-2000:]

@@ -22,7 +22,7 @@ from tests.conftest import have_gpu
 pytestmark = pytest.mark.gpu
 
 TOL = {np.float64: 1e-12, np.float32: 1e-5}
-VARIANTS = [1, 2, 3]  # CRSD_VARIANT_LDG, CRSD_VARIANT_TMA, CRSD_VARIANT_PIPE
+VARIANTS = [1, 2, 3, 4]  # CRSD_VARIANT_LDG, _TMA, _PIPE, _JIT
 
 _CACHE = {}
 
@@ -45,9 +45,15 @@ def torch_cuda():
 
 
 def _mat(a, **kw):
-    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, CRSDError
 
-    return CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, **kw)
+    try:
+        return CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, **kw)
+    except CRSDError as e:
+        # the JIT codelets need a whole segment per CTA (staging <= 200 KB)
+        if kw.get("variant") == 4 and "UNSUPPORTED" in str(e):
+            pytest.skip(f"JIT variant not applicable: {e}")
+        raise
 
 
 def _run(torch, A, x, alpha=1.0, beta=0.0, y0=None, nrows=None):
