@@ -49,7 +49,7 @@ def main():
         tdt = torch.float64 if dt == "f64" else torch.float32
         x = torch.rand(a.ncols, dtype=tdt, device="cuda")
         y = torch.empty(a.nrows, dtype=tdt, device="cuda")
-        runs = [("ldg", 1, None)] + [("tma", 2, t) for t in TMA] + [("pipe", 3, sh) for sh in SHAPES]
+        runs = [("ldg", 1, None)] + [("tma", 2, t) for t in TMA] + [("pipe", 3, sh) for sh in SHAPES] + [("jit", 4, None)]
         for name, v, sh in runs:
             for k in ("CRSD_PIPE_PERSM", "CRSD_PIPE_NX", "CRSD_PIPE_NS", "CRSD_TMA_Q", "CRSD_TMA_SPLIT"):
                 os.environ.pop(k, None)
