@@ -60,13 +60,21 @@ void free_device(crsd_matrix_s *A) {
         cudaStreamDestroy((cudaStream_t)A->e2e_d2h);
         A->e2e_ready = false;
     }
-    void *ptrs[] = {A->d_vals, A->d_segs, A->d_offs, A->d_plan, A->d_scat_row, A->d_scat_col, A->d_scat_val, A->d_scat_rec,
-                    A->d_list_interior, A->d_list_boundary, A->d_list_all_edge, A->d_x_scratch, A->d_y_scratch};
     if (A->device >= 0) cudaSetDevice(A->device);
+    if (A->cg_stream) {
+        cudaStreamSynchronize((cudaStream_t)A->cg_stream);
+        cudaStreamDestroy((cudaStream_t)A->cg_stream);
+        cudaEventDestroy((cudaEvent_t)A->cg_ev_in);
+        cudaEventDestroy((cudaEvent_t)A->cg_ev_out);
+        A->cg_stream = A->cg_ev_in = A->cg_ev_out = nullptr;
+    }
+    void *ptrs[] = {A->d_vals, A->d_segs, A->d_offs, A->d_plan, A->d_scat_row, A->d_scat_col, A->d_scat_val, A->d_scat_rec,
+                    A->d_list_interior, A->d_list_boundary, A->d_list_all_edge, A->d_x_scratch, A->d_y_scratch, A->d_cg};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     A->d_vals = A->d_segs = A->d_offs = A->d_plan = A->d_scat_row = A->d_scat_col = A->d_scat_val = A->d_scat_rec = nullptr;
-    A->d_list_interior = A->d_list_boundary = A->d_list_all_edge = A->d_x_scratch = A->d_y_scratch = nullptr;
+    A->d_list_interior = A->d_list_boundary = A->d_list_all_edge = A->d_x_scratch = A->d_y_scratch = A->d_cg = nullptr;
+    A->cg_bytes = 0;
 }
 
 // Layout of x for this handle: valid range and halo widths (DESIGN.md
@@ -174,6 +182,13 @@ static crsd_status_t upload(crsd_matrix_s *A) {
     return CRSD_OK;
 }
 
+static int auto_variant(const crsd_matrix_s *A, bool jit, bool pipe_fits) {
+    if (jit && A->smem_bytes <= 75 * 1024) return VARIANT_JIT;
+    if (A->tma_split == 1 && A->tma_smem <= 32 * 1024) return VARIANT_TMA;
+    if (pipe_fits && A->H.mrows <= 1024) return VARIANT_PIPE;
+    return VARIANT_LDG;
+}
+
 static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_matrix_t *out) {
     A->rpt = (A->H.dtype == CRSD_R64F) ? 2 : 4;
     int64_t maxnd = 0;
@@ -202,20 +217,23 @@ static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_
         delete A;
         return fail(CRSD_ERR_UNSUPPORTED, "PIPE variant: mrows must be <= 1024");
     }
+    const bool auto_jit = !getenv("CRSD_NO_JIT");
     if (o.variant == CRSD_VARIANT_JIT) A->variant = VARIANT_JIT;
     else if (o.variant == CRSD_VARIANT_LDG) A->variant = VARIANT_LDG;
     else if (o.variant == CRSD_VARIANT_TMA) A->variant = VARIANT_TMA;
     else if (o.variant == CRSD_VARIANT_PIPE) A->variant = VARIANT_PIPE;
     else {
-        // AUTO, from the variant sweeps in profiles/r01_sweep*.jsonl: the
-        // one-shot TMA kernel when a whole segment stages in <= 32 KB (enough
-        // CTAs per SM to keep ~200 KB in flight: C2 ~98 % fp64 / ~92 % fp32 of
-        // the measured copy bandwidth); otherwise the persistent chunked ring
-        // (PIPE: C3 83-87 % fp64, 81 % fp32); the register variant when
-        // neither staging fits in shared memory.
-        if (A->tma_split == 1 && A->tma_smem <= 32 * 1024) A->variant = VARIANT_TMA;
-        else if (pipe_need <= smem_cap && A->H.mrows <= 1024) A->variant = VARIANT_PIPE;
-        else A->variant = VARIANT_LDG;
+        // AUTO, from the variant sweeps in profiles/r01_sweep*.jsonl. The
+        // runtime-generated one-shot kernel (JIT: every pattern quantity a
+        // literal, a whole segment staged per CTA, scatter points gathered
+        // while the bulk copies fly) leads wherever a segment stages in <= 75
+        // KB (>= 3 CTAs per SM): C2 1.05 / 1.02, C3 0.95 / 0.99 of the
+        // measured copy peak (fp64 / fp32, sweep18), ahead of the table-driven
+        // TMA (C2 0.98 / 0.90) and of the persistent ring (PIPE, C3 0.90 /
+        // 0.85), which remains the choice for bigger segments; the register
+        // variant when neither staging fits in shared memory. Without NVRTC
+        // the JIT falls back to TMA (small segments) below.
+        A->variant = auto_variant(A, auto_jit, pipe_need <= smem_cap);
     }
     if (!A->host_only) {
         if (A->H.mrows / A->rpt > 256) {
@@ -228,7 +246,13 @@ static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_
                                                   std::to_string(o.mrows) + " (use CRSD_HOST_ONLY for inspection)");
         }
         crsd_status_t st = upload(A);
-        if (!st && A->variant == VARIANT_JIT) st = jit_build(A);
+        if (!st && A->variant == VARIANT_JIT) {
+            st = jit_build(A);
+            if (st == CRSD_ERR_UNSUPPORTED && o.variant == CRSD_VARIANT_AUTO) {
+                A->variant = auto_variant(A, false, pipe_need <= smem_cap);  // no NVRTC
+                st = CRSD_OK;
+            }
+        }
         if (st) {
             free_device(A);
             delete A;

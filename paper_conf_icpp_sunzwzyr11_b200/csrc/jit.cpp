@@ -126,6 +126,7 @@ struct JitArgs {
     const int32_t *scat_row;
     const int64_t *scat_col;
     const T *scat_val;
+    const ScatRec *scat_rec;
     T alpha, beta;
 };
 
@@ -135,9 +136,10 @@ typedef unsigned long long u64;
 typedef unsigned int u32;
 typedef unsigned short u16;
 struct SegDesc { i64 val_base; i64 scat_begin; int off_begin; int nscat; u16 flags; u16 ndias; int plan_begin; };
+struct __align__(16) ScatRec { i64 col; double val; int row; int pad[3]; };
 struct Args { const T *vals; const SegDesc *segs; const int *seg_list; i64 seg_begin, seg_count;
               const T *x; i64 x_lo, x_hi; T *y; i64 nrows;
-              const int *scat_row; const i64 *scat_col; const T *scat_val; T alpha, beta; };
+              const int *scat_row; const i64 *scat_col; const T *scat_val; const ScatRec *scat_rec; T alpha, beta; };
 __device__ __forceinline__ u32 su32(const void *p) { return (u32)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void bar_init(u64 *b) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(su32(b)) : "memory");
@@ -163,23 +165,27 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
     const HostCRSD &H = A->H;
     const bool f64 = H.dtype == CRSD_R64F;
     const int m = H.mrows, nt = m / Q, es = H.elem;
+    const bool scat = H.nscatter() > 0;  // scatter code only for matrices that have scatter points
     std::ostringstream o;
     o << "typedef " << (f64 ? "double" : "float") << " T;\n" << kPrelude;
     o << "#define MROWS " << m << "\n#define NT " << nt << "\n#define Q " << Q << "\n";
     // one __device__ codelet per distinct pattern
+    // codelets are keyed by the pattern's plan_begin, which is unique per
+    // distinct pattern (off_begin is not: a pattern without diagonals shares
+    // it with the next pattern)
     std::vector<int32_t> seen;
     for (const Instance &I : H.inst) {
-        const int32_t off_begin = (int32_t)H.pat_ptr[I.pattern];
+        const int32_t key = A->segdesc[I.first_seg].plan_begin;
         bool dup = false;
-        for (int32_t v : seen) dup |= (v == off_begin);
+        for (int32_t v : seen) dup |= (v == key);
         if (dup) continue;
-        seen.push_back(off_begin);
-        const int32_t *pl = A->plan.data() + A->segdesc[I.first_seg].plan_begin;
+        seen.push_back(key);
+        const int32_t *pl = A->plan.data() + key;
         const int nd = (int)H.ndias(I.pattern), nwin = pl[0];
         const int64_t *offs = H.pat_offsets.data() + H.pat_ptr[I.pattern];
         o << "// pattern offsets:";
         for (int d = 0; d < nd; ++d) o << " " << offs[d];
-        o << "\n__device__ __forceinline__ void codelet_" << off_begin
+        o << "\n__device__ __forceinline__ void codelet_" << key
           << "(const Args &a, const SegDesc &D, i64 row0, bool edge, T *vs, u64 *bar, int t) {\n";
         int64_t xb = 0;
         for (int w = 0; w < nwin; ++w) xb += pl[3 + 2 * w];
@@ -199,6 +205,21 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
             }
             o << "  }\n";
         }
+        if (scat) {
+            // scatter points are gathered while the bulk copies are in flight:
+            // lane l of every warp reads record l of the segment's first 32
+            // (row, col, value in one 32-B record); a ballot keeps those whose
+            // row belongs to this warp, which alone load x[col]
+            o << "  int g_own = -1; T g_v = T(0), g_x = T(0); unsigned g_mask = 0u;\n"
+                 "  if (D.nscat > 0) {\n"
+                 "    const int lane = t & 31;\n"
+                 "    ScatRec R; R.col = 0; R.val = 0; R.row = 0;\n"
+                 "    if (lane < D.nscat) { R = a.scat_rec[D.scat_begin + lane]; g_own = (R.row % NT) * Q + R.row / NT; }\n"
+                 "    const bool mine = g_own >= 0 && (g_own / Q) / 32 == t / 32;\n"
+                 "    g_mask = __ballot_sync(0xffffffffu, mine);\n"
+                 "    if (mine) { g_v = *reinterpret_cast<const T *>(&R.val); g_x = __ldg(a.x + R.col); }\n"
+                 "  }\n";
+        }
         o << "  T acc[Q];\n#pragma unroll\n  for (int q = 0; q < Q; ++q) acc[q] = T(0);\n";
         o << "  bar_wait(bar);\n";
         const int32_t *xoff = pl + 2 + 2 * nwin;
@@ -210,12 +231,23 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
             o << "      { const i64 i = r + (" << offs[d] << "); acc[q] = fma(vs[" << (int64_t)d * m
               << " + t + q * NT], (i >= a.x_lo && i < a.x_hi) ? __ldg(a.x + i) : T(0), acc[q]); }\n";
         o << "    }\n  }\n";
-        // scatter points (owner thread, (row, col) order) and the epilogue
-        o << "  for (int e = 0; e < D.nscat; ++e) {\n"
-             "    const int rr = __ldg(a.scat_row + D.scat_begin + e);\n"
-             "    if (rr % NT != t) continue;\n"
-             "    const T v = __ldg(a.scat_val + D.scat_begin + e), xv = __ldg(a.x + __ldg(a.scat_col + D.scat_begin + e));\n"
-             "#pragma unroll\n    for (int q = 0; q < Q; ++q) if (rr / NT == q) acc[q] = fma(v, xv, acc[q]);\n  }\n";
+        // scatter points in (row, col) order by their owner thread: the
+        // gathered ones (broadcast from the lane holding them), then any
+        // beyond the first 32; then the epilogue
+        if (scat)
+            o << "  if (D.nscat > 0) {\n"
+                 "    for (unsigned mm = g_mask; mm; mm &= mm - 1) {\n"
+                 "      const int j = __ffs(mm) - 1;\n"
+                 "      const int own = __shfl_sync(0xffffffffu, g_own, j);\n"
+                 "      const T v = __shfl_sync(0xffffffffu, g_v, j), xv = __shfl_sync(0xffffffffu, g_x, j);\n"
+                 "#pragma unroll\n      for (int q = 0; q < Q; ++q) if (own == t * Q + q) acc[q] = fma(v, xv, acc[q]);\n"
+                 "    }\n"
+                 "    for (int e = 32; e < D.nscat; ++e) {\n"
+                 "      const int rr = __ldg(a.scat_row + D.scat_begin + e);\n"
+                 "      if (rr % NT != t) continue;\n"
+                 "      const T v = __ldg(a.scat_val + D.scat_begin + e), xv = __ldg(a.x + __ldg(a.scat_col + D.scat_begin + e));\n"
+                 "#pragma unroll\n      for (int q = 0; q < Q; ++q) if (rr / NT == q) acc[q] = fma(v, xv, acc[q]);\n"
+                 "    }\n  }\n";
         o << "#pragma unroll\n  for (int q = 0; q < Q; ++q) {\n    const i64 r = row0 + t + q * NT;\n"
              "    if (!edge || r < a.nrows) { T *yp = a.y + r; __stcs(yp, (a.beta != T(0)) ? fma(a.alpha, acc[q], a.beta * *yp) : a.alpha * acc[q]); }\n"
              "  }\n}\n";
@@ -224,7 +256,7 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
          "  extern __shared__ __align__(128) unsigned char smem[];\n  __shared__ u64 bar;\n"
          "  const i64 s = a.seg_list ? (i64)__ldg(a.seg_list + blockIdx.x) : a.seg_begin + blockIdx.x;\n"
          "  const SegDesc D = a.segs[s];\n  const i64 row0 = s * MROWS;\n  const bool edge = (D.flags & 1) != 0;\n"
-         "  T *vs = reinterpret_cast<T *>(smem);\n  switch (D.off_begin) {\n";
+         "  T *vs = reinterpret_cast<T *>(smem);\n  switch (D.plan_begin) {\n";
     for (int32_t v : seen) o << "  case " << v << ": codelet_" << v << "(a, D, row0, edge, vs, &bar, threadIdx.x); break;\n";
     o << "  }\n}\n";
     return o.str();
@@ -306,6 +338,7 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
     j.scat_row = s.scat_row;
     j.scat_col = s.scat_col;
     j.scat_val = s.scat_val;
+    j.scat_rec = s.scat_rec;
     j.alpha = s.alpha;
     j.beta = s.beta;
     void *params[] = {&j};

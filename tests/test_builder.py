@@ -187,7 +187,7 @@ def test_unique_bytes_accounting():
     assert inf["unique_bytes_beta1"] == inf["unique_bytes_beta0"] + n * 8
 
 
-@pytest.mark.parametrize("case", ["c1", "c2s", "c3s", "rand"])
+@pytest.mark.parametrize("case", ["c1", "c2s", "c3s", "rand", "empty"])
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
 def test_jit_codelets_compile_for_sm100a(case, dt, tmp_path):
     """The JIT variant's generated per-pattern codelets (the paper's code
@@ -201,6 +201,12 @@ def test_jit_codelets_compile_for_sm100a(case, dt, tmp_path):
         a = gen.config2(n=24)
     elif case == "c3s":
         a = gen.config3(n=20)
+    elif case == "empty":
+        # segments without any diagonal: that pattern has no offsets, so its
+        # offset-table start equals the next pattern's (A11)
+        a = gen.config2(n=24)
+        keep = (a.row < 1024) | (a.row >= 2048)
+        a = gen.COO(a.nrows, a.ncols, a.row[keep], a.col[keep], a.val[keep])
     else:
         a = gen.random_diagonal(3000, 3000, 3, ndiag=8, max_off=400, n_scatter=40)
     a = a.astype(dt)
