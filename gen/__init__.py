@@ -22,4 +22,5 @@ from .matrices import (  # noqa: F401
     random_diagonal,
     vectors,
     nonzero_uniform,
+    spd_stencil_scatter,
 )

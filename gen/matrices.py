@@ -436,3 +436,45 @@ def vectors(n: int, kind: str = "random", seed: int = 0, dims=None, coef=None) -
             return a + b[0] * g[0] + b[1] * g[1] + b[2] * g[2]
         return (g[0] * g[0] + g[1] * g[1] + g[2] * g[2]).astype(np.float64)
     raise ValueError(kind)
+
+
+# ---------------------------------------------------------------------------
+# symmetric positive definite inputs for the CG iteration
+# ---------------------------------------------------------------------------
+def spd_stencil_scatter(dims: Sequence[int], kind: str = "7pt", n_pairs: int = 0, seed: int = 0, shift: float = 0.0) -> COO:
+    """Dirichlet stencil (center = number of stencil neighbours, couplings -1:
+    symmetric, irreducibly diagonally dominant => SPD) plus ``n_pairs``
+    symmetric off-stencil pairs (r, c), (c, r) with one value v in U(-1,1)\\{0};
+    each pair adds |v| to both diagonal entries (and ``shift`` to every
+    diagonal entry), which keeps the matrix diagonally dominant, hence SPD.
+    The pairs exercise the scatter-point path inside CG."""
+    a = stencil(dims, kind)
+    n = a.nrows
+    rng = np.random.default_rng(seed)
+    diag_add = np.full(n, float(shift))
+    pr, pc, pv = [], [], []
+    if n_pairs:
+        taken = set((a.row * np.int64(n) + a.col).tolist())
+        while len(pr) < n_pairs:
+            r = int(rng.integers(0, n))
+            c = int(rng.integers(0, n))
+            if r == c or r * n + c in taken:
+                continue
+            taken.add(r * n + c)
+            taken.add(c * n + r)
+            v = float(nonzero_uniform(rng, 1)[0])
+            pr += [r, c]
+            pc += [c, r]
+            pv += [v, v]
+            diag_add[r] += abs(v)
+            diag_add[c] += abs(v)
+    val = a.val.astype(np.float64).copy()
+    on_diag = a.row == a.col
+    val[on_diag] += diag_add[a.row[on_diag]]
+    return COO(
+        n,
+        n,
+        np.concatenate([a.row, np.array(pr, np.int64)]),
+        np.concatenate([a.col, np.array(pc, np.int64)]),
+        np.concatenate([val, np.array(pv, np.float64)]),
+    )
