@@ -190,12 +190,15 @@ def sustained_copy_bandwidth(dev, seconds):
     return round(gbs, 1)
 
 
-def load_traffic(cfg, dtype):
+def load_traffic(cfg, dtype, kernel):
+    """ncu dram bytes (read + write) per launch of `kernel` on this workload,
+    from one `ncu --set full` capture (profiles/traffic.json, keyed
+    "<config>_<dtype>_<kernel>"); None when that kernel was not captured."""
     p = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(p):
         with open(p) as f:
             j = json.load(f)
-        return j.get(f"{cfg}_{dtype}")
+        return j.get(f"{cfg}_{dtype}_{kernel}")
     return None
 
 
@@ -480,7 +483,8 @@ def run_crsd(args):
     cpu = None if (world > 1 or args.no_cpu) else cpu_baseline(a)
     box_copy = copy_bandwidth(dev)
     box_copy_sus = sustained_copy_bandwidth(dev, total_ms * 1e-3)
-    traffic = load_traffic(args.config, args.dtype)
+    kname = {1: "crsd_spmv_ldg", 2: "crsd_spmv_tma", 3: "crsd_spmv_pipe", 4: "crsd_jit"}[info["variant"]]
+    traffic = None if args.mrows else load_traffic(args.config, args.dtype, kname)
     line = {
         "metric": "CRSD SpMV GFLOP/s (2*nnz/t) with achieved HBM GB/s (% of B200 peak)",
         "value": round(gflops, 3),
@@ -512,7 +516,7 @@ def run_crsd(args):
         "hbm_frac_of_peak": round(ub_all / (ms * 1e-3) / 1e9 / (peak * world), 4),
         "roofline": {
             "bound": "hbm",
-            "kernel": {1: "crsd_spmv_ldg", 2: "crsd_spmv_tma", 3: "crsd_spmv_pipe", 4: "crsd_jit"}[info["variant"]],
+            "kernel": kname,
             "achieved": round(achieved, 1),
             "peak": peak,
             "peak_source": peak_src,

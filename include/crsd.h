@@ -291,7 +291,53 @@ crsd_status_t crsd_export(crsd_matrix_t A, crsd_export_t *out);
  * (values + x windows) exceeds 200 KB of shared memory. */
 crsd_status_t crsd_jit_source(crsd_matrix_t A, char *buf, int64_t cap, int64_t *len);
 
-/* Number of kernel launches the last crsd_spmv / crsd_spmv_dist call made. */
+/* ------------------------------------------------------------------------
+ * Conjugate gradient on a CRSD matrix (the paper
+ * motivates CRSD with FDM/FVM coefficient matrices of PDEs, and
+ * cites Saad [2], for the iterative methods built on SpMV).
+ * Textbook CG (Hestenes & Stiefel; Saad Algorithm 6.18):
+ *     r0 = b - A x0; p0 = r0
+ *     q = A p; alpha = (r,r)/(p,q); x += alpha p; r -= alpha q;
+ *     beta = (r,r)_new/(r,r); p = r + beta p
+ * A must be symmetric positive definite (not checked) and square.
+ * ---------------------------------------------------------------------- */
+typedef struct {
+    int32_t iterations; /* CG steps taken */
+    int32_t converged;  /* 1 if sqrt((r,r)) <= rtol * sqrt((b,b)) was reached */
+    double rr0;         /* (r_0, r_0) */
+    double rr;          /* (r_k, r_k) at exit (recurrence residual) */
+    double bb;          /* (b, b) */
+    int64_t launches;   /* kernel launches of the solve (graph nodes included) */
+} crsd_cg_result_t;
+
+/*
+ * Solve A x = b.
+ *   b          DEVICE dtype[n_local], 16-byte aligned, read-only.
+ *   x          DEVICE dtype[n_local], 16-byte aligned: x0 on entry, the
+ *              iterate on exit. n_local = nrows for a one-GPU handle, the
+ *              owned rows of a row-partitioned handle.
+ *   max_iter   >= 0 steps at most.
+ *   rtol       stop when sqrt((r,r)) <= rtol * sqrt((b,b)) (0 => run
+ *              max_iter steps, or until (r,r) == 0). Evaluated on the device
+ *              after every step.
+ *   check_every steps per host poll (and per CUDA graph on one GPU); <= 0 => 16.
+ *   comm       NULL for a one-GPU handle; the bound communicator of a
+ *              row-partitioned handle (halo exchange through crsd_spmv_dist,
+ *              dot products as NCCL allreduces).
+ *   rr_history HOST double[max_iter+1] or NULL: (r_j, r_j), j = 0..iterations.
+ *   res        HOST, may be NULL.
+ *   stream     the work is ordered after prior work on `stream`; the call
+ *              returns when the solve has finished (it polls the device).
+ * Arithmetic: vectors in the matrix dtype; dot products accumulated in fp64
+ * and reduced deterministically; alpha, beta in fp64 (applied in the dtype).
+ * The handle owns a workspace (3 vectors + O(SMs) scalars) kept between calls.
+ * Errors: INVALID_ARG, UNSUPPORTED (not square / host-only), ALLOC, CUDA, NCCL.
+ */
+crsd_status_t crsd_cg(crsd_matrix_t A, const void *b, void *x, int32_t max_iter, double rtol,
+                      int32_t check_every, crsd_comm_t comm, double *rr_history, crsd_cg_result_t *res,
+                      void *stream);
+
+/* Number of kernel launches the last crsd_spmv / crsd_spmv_dist / crsd_cg call made. */
 crsd_status_t crsd_last_launch_count(crsd_matrix_t A, int32_t *count);
 
 #ifdef __cplusplus

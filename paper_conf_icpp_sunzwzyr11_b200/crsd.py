@@ -51,6 +51,7 @@ EXPORTED = [
     "crsd_export",
     "crsd_last_launch_count",
     "crsd_jit_source",
+    "crsd_cg",
 ]
 
 
@@ -109,6 +110,17 @@ class Export(ctypes.Structure):
     ]
 
 
+class CGResult(ctypes.Structure):
+    _fields_ = [
+        ("iterations", ctypes.c_int32),
+        ("converged", ctypes.c_int32),
+        ("rr0", ctypes.c_double),
+        ("rr", ctypes.c_double),
+        ("bb", ctypes.c_double),
+        ("launches", ctypes.c_int64),
+    ]
+
+
 def _load():
     if not os.path.exists(LIB_PATH):
         raise ImportError(f"{LIB_PATH} is not built; run `python -c 'import __graft_entry__ as g; g.build()'`")
@@ -135,6 +147,7 @@ def _load():
         "crsd_export": ([P, P], ctypes.c_int),
         "crsd_last_launch_count": ([P, P], ctypes.c_int),
         "crsd_jit_source": ([P, P, I64, P], ctypes.c_int),
+        "crsd_cg": ([P, P, P, I32, ctypes.c_double, I32, P, P, P, P], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)
@@ -306,6 +319,31 @@ class CRSDMatrix:
             )
         )
         return y_local
+
+    def cg(self, b, x, max_iter, rtol=0.0, check_every=16, comm=None, history=False, stream=None) -> dict:
+        """Conjugate gradient A x = b (crsd_cg): b, x torch CUDA tensors of the
+        owned rows; x holds x0 on entry and the iterate on exit. Returns the
+        crsd_cg_result_t fields (+ "rr_history" when history=True)."""
+        res = CGResult()
+        hist = np.zeros(max_iter + 1, np.float64) if history else None
+        _check(
+            lib.crsd_cg(
+                self._h,
+                ctypes.c_void_p(b.data_ptr()),
+                ctypes.c_void_p(x.data_ptr()),
+                int(max_iter),
+                float(rtol),
+                int(check_every),
+                comm._h if comm is not None else None,
+                _p(hist) if hist is not None else None,
+                ctypes.byref(res),
+                _stream_ptr(stream),
+            )
+        )
+        out = {k: getattr(res, k) for k, _ in CGResult._fields_}
+        if history:
+            out["rr_history"] = hist[: res.iterations + 1]
+        return out
 
     def dist_bind(self, comm, stream=None):
         _check(lib.crsd_dist_bind(self._h, comm._h, _stream_ptr(stream)))

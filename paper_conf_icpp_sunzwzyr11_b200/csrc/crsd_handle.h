@@ -61,6 +61,12 @@ struct crsd_matrix_s {
     std::vector<void *> e2e_ev_x, e2e_ev_y;         // cudaEvent_t
     void *e2e_ev_start = nullptr, *e2e_ev_done = nullptr;
 
+    // CG workspace (crsd_cg): state, partials, history, r, q, halo-padded p
+    void *d_cg = nullptr;
+    int64_t cg_bytes = 0;
+    void *cg_stream = nullptr;                  // cudaStream_t (graph capture / replay)
+    void *cg_ev_in = nullptr, *cg_ev_out = nullptr;  // cudaEvent_t
+
     // multi-GPU plan (crsd_dist_bind)
     bool bound = false;
     std::vector<int64_t> recv_peer, recv_off, recv_count;  // offsets into x_padded

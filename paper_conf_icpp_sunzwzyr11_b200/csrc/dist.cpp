@@ -21,12 +21,7 @@
 #include "crsd_handle.h"
 #include "crsd_internal.h"
 
-struct crsd_comm_s {
-    ncclComm_t comm = nullptr;
-    int rank = 0, world = 1, device = 0;
-    cudaStream_t cs = nullptr;
-    cudaEvent_t ev_x = nullptr, ev_halo = nullptr;
-};
+#include "crsd_comm.h"
 
 namespace {
 crsd_status_t nccl_fail(ncclResult_t r, const char *what) {

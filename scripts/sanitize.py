@@ -28,7 +28,7 @@ def main():
             x = np.random.default_rng(1).uniform(-1, 1, b.ncols).astype(dt)
             y0 = np.random.default_rng(2).uniform(-1, 1, b.nrows).astype(dt)
             yref, sc = coo.coo_spmv(b.nrows, b.ncols, b.row, b.col, b.val, x, -0.75, 0.5, y0)
-            for v in (1, 2, 3):
+            for v in (1, 2, 3, 4):
                 A = CRSDMatrix.from_coo(b.nrows, b.ncols, b.row, b.col, b.val, variant=v)
                 tdt = torch.float64 if dt == np.float64 else torch.float32
                 xd = torch.from_numpy(x).to("cuda", tdt)
@@ -39,6 +39,21 @@ def main():
                 ok = err <= (1e-12 if dt == np.float64 else 1e-5)
                 bad += not ok
                 print(f"{name} {np.dtype(dt).name} variant {v}: parity {err:.2e} {'ok' if ok else 'FAIL'}", flush=True)
+    # CG (vector kernels, grid reductions, graph replay) on an SPD stencil
+    from oracle import cg_ref
+
+    a = gen.spd_stencil_scatter((12, 12, 12), "7pt", n_pairs=30, seed=2)
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val)
+    rng = np.random.default_rng(3)
+    b = rng.uniform(-1, 1, a.nrows)
+    bd = torch.from_numpy(b).to("cuda")
+    xd = torch.zeros(a.nrows, dtype=torch.float64, device="cuda")
+    res = A.cg(bd, xd, 20, 0.0, check_every=6, history=True)
+    xr, _, hr = cg_ref.cg(a, b, np.zeros(a.nrows), 20)
+    ex = np.max(np.abs(xd.cpu().numpy() - xr)) / np.max(np.abs(xr))
+    ok = res["iterations"] == 20 and ex <= 1e-12
+    bad += not ok
+    print(f"cg f64: 20 steps, x deviation {ex:.2e} {'ok' if ok else 'FAIL'}", flush=True)
     sys.exit(1 if bad else 0)
 
 

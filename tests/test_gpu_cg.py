@@ -1,0 +1,177 @@
+"""GPU parity of crsd_cg (CG on the CRSD SpMV)
+against the CG oracle (oracle/cg_ref.py) and against closed forms.
+
+Tolerances: CG iterates are not backward-stable step
+by step -- two admissible evaluation orders of the same step drift apart by
+O(u * kappa) per step. scripts/cg_sensitivity.py runs the same CG with another
+admissible evaluation order (scipy CSR SpMV, vectors in the matrix precision,
+fp64 dots: the GPU path's arithmetic) against the oracle on these matrices;
+over 60 steps the largest differences are (r,r): 1.2e-14 (fp64) / 3.4e-6
+(fp32) relative, x: 7.9e-15 / 3.6e-6 of max|x|. The bars below leave >= 100x
+(fp64) / >= 25x (fp32) over those, and compare (r,r) only while the oracle
+residual is above the precision's floor (rr_j / rr_0 >= 1e-20 fp64, 1e-8 fp32).
+"""
+import numpy as np
+import pytest
+
+import gen
+from oracle import cg_ref, coo
+
+pytestmark = pytest.mark.gpu
+
+RR_TOL = {np.float64: 1e-11, np.float32: 1e-3}
+X_TOL = {np.float64: 1e-12, np.float32: 1e-4}
+RR_FLOOR = {np.float64: 1e-20, np.float32: 1e-8}
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+
+    if not torch.cuda.is_available():
+        pytest.fail("no CUDA device: -m gpu tests need a B200")
+    return torch
+
+
+def _solve(torch, a, dt, b, x0, iters, rtol=0.0, check_every=16, variant=0, mrows=0):
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix
+
+    a = a.astype(dt)
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, variant=variant, mrows=mrows)
+    tdt = torch.float64 if dt == np.float64 else torch.float32
+    bd = torch.from_numpy(b.astype(dt)).to("cuda")
+    xd = torch.from_numpy(x0.astype(dt)).to("cuda")
+    res = A.cg(bd, xd, iters, rtol, check_every=check_every, history=True)
+    torch.cuda.synchronize()
+    return A, res, xd.cpu().numpy()
+
+
+def _compare(a, dt, b, x0, res, x):
+    k = res["iterations"]
+    xr, _, hr = cg_ref.cg(a.astype(dt), b.astype(dt).astype(np.float64), x0.astype(dt).astype(np.float64), k)
+    h = res["rr_history"]
+    assert h.shape[0] == k + 1
+    live = hr / hr[0] >= RR_FLOOR[dt]
+    rel = np.abs(h[live] - hr[live]) / hr[live]
+    assert rel.max() <= RR_TOL[dt], f"rr history deviates by {rel.max():.3e}"
+    ex = np.max(np.abs(x - xr)) / np.max(np.abs(xr))
+    assert ex <= X_TOL[dt], f"x deviates by {ex:.3e}"
+    return rel.max(), ex
+
+
+CASES = {
+    "7pt": lambda: gen.spd_stencil_scatter((40, 40, 40), "7pt"),
+    "27pt": lambda: gen.spd_stencil_scatter((24, 24, 24), "27pt"),
+    "7pt+scatter": lambda: gen.spd_stencil_scatter((30, 30, 30), "7pt", n_pairs=500, seed=3),
+    "5pt-ragged": lambda: gen.spd_stencil_scatter((61, 67), "5pt", n_pairs=40, seed=4),
+}
+
+
+@pytest.mark.parametrize("variant", [0, 1, 2, 3, 4])
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+@pytest.mark.parametrize("case", list(CASES))
+def test_cg_parity_fixed_steps(torch_cuda, case, dt, variant):
+    """60 CG steps (rtol 0) on SPD stencil matrices, every kernel variant,
+    compared step by step with the oracle. check_every 7 does not divide 60:
+    the last graph batch overshoots and must be a no-op (device-side stop)."""
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDError
+
+    a = CASES[case]()
+    rng = np.random.default_rng(11)
+    b = rng.uniform(-1, 1, a.nrows)
+    x0 = rng.uniform(-0.5, 0.5, a.nrows)
+    try:
+        A, res, x = _solve(torch_cuda, a, dt, b, x0, 60, check_every=7, variant=variant)
+    except CRSDError as e:
+        if variant in (2, 3, 4) and "UNSUPPORTED" in str(e):
+            pytest.skip(f"variant not applicable: {e}")
+        raise
+    assert res["iterations"] == 60 and res["converged"] in (0, 1)
+    _compare(a, dt, b, x0, res, x)
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_cg_converges_and_true_residual(torch_cuda, dt):
+    """rtol stopping test on the device: the reported step count is the first
+    at which sqrt(rr) <= rtol * |b|, the recurrence residual matches the true
+    residual b - A x (oracle SpMV), and the history agrees with the oracle."""
+    a = gen.spd_stencil_scatter((32, 32, 32), "7pt", n_pairs=200, seed=5)
+    rng = np.random.default_rng(12)
+    b = rng.uniform(-1, 1, a.nrows)
+    x0 = np.zeros(a.nrows)
+    rtol = 1e-8 if dt == np.float64 else 1e-4
+    A, res, x = _solve(torch_cuda, a, dt, b, x0, 2000, rtol=rtol, check_every=16)
+    assert res["converged"] == 1
+    k = res["iterations"]
+    h = res["rr_history"]
+    bb = float(np.dot(b.astype(dt).astype(np.float64), b.astype(dt).astype(np.float64)))
+    assert res["bb"] == pytest.approx(bb, rel=1e-12)
+    assert h[k] <= rtol**2 * res["bb"] and np.all(h[:k] > rtol**2 * res["bb"])
+    ad = a.astype(dt)
+    ax, _ = coo.coo_spmv(ad.nrows, ad.ncols, ad.row, ad.col, ad.val.astype(np.float64), x.astype(np.float64))
+    true_r = np.linalg.norm(b.astype(dt).astype(np.float64) - ax)
+    assert true_r <= 2.0 * rtol * np.sqrt(bb) + (1e-12 if dt == np.float64 else 1e-4) * np.sqrt(bb)
+
+
+def test_cg_1d_laplacian_closed_form(torch_cuda):
+    """tridiag(-1, 2, -1) x = 1 has x_i = i (n+1-i) / 2 (i = 1..n): CG on the
+    GPU reaches it (fp64, kappa ~ 4 n^2 / pi^2)."""
+    n = 1000
+    r = np.concatenate([np.arange(n), np.arange(1, n), np.arange(n - 1)])
+    c = np.concatenate([np.arange(n), np.arange(n - 1), np.arange(1, n)])
+    v = np.concatenate([np.full(n, 2.0), np.full(n - 1, -1.0), np.full(n - 1, -1.0)])
+    a = gen.COO(n, n, r.astype(np.int64), c.astype(np.int64), v)
+    A, res, x = _solve(torch_cuda, a, np.float64, np.ones(n), np.zeros(n), 4 * n, rtol=1e-13, check_every=50, mrows=64)
+    i = np.arange(1, n + 1, dtype=np.float64)
+    xe = i * (n + 1 - i) / 2.0
+    assert res["converged"] == 1
+    assert np.max(np.abs(x - xe)) <= 1e-7 * np.max(xe)
+
+
+def test_cg_zero_rhs_and_zero_iters(torch_cuda):
+    import torch
+
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix
+
+    a = gen.spd_stencil_scatter((16, 16, 16), "7pt")
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val)
+    b = torch.zeros(a.nrows, dtype=torch.float64, device="cuda")
+    x = torch.zeros(a.nrows, dtype=torch.float64, device="cuda")
+    res = A.cg(b, x, 50, 1e-10, history=True)
+    assert res["iterations"] == 0 and res["converged"] == 1 and torch.all(x == 0)
+    b.uniform_(-1, 1)
+    x0 = torch.rand(a.nrows, dtype=torch.float64, device="cuda")
+    x.copy_(x0)
+    res = A.cg(b, x, 0, 0.0)
+    assert res["iterations"] == 0 and torch.equal(x, x0)
+
+
+def test_cg_one_rank_communicator(torch_cuda):
+    """The multi-GPU code path of crsd_cg (row-partitioned handle, bound NCCL
+    communicator, crsd_spmv_dist halo exchange, allreduced dots) with one rank
+    owning every row: must agree with the oracle like the one-GPU path."""
+    import os
+
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_icpp_sunzwzyr11_b200 import Comm, CRSDMatrix
+
+    if not dist.is_initialized():
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29611")
+        dist.init_process_group("gloo", rank=0, world_size=1)
+    a = gen.spd_stencil_scatter((24, 24, 24), "7pt", n_pairs=100, seed=6)
+    n = a.nrows
+    A = CRSDMatrix.from_coo(n, n, a.row, a.col, a.val, row_range=(0, n))
+    comm = Comm(0, 1, 0)
+    A.dist_bind(comm)
+    rng = np.random.default_rng(13)
+    b = rng.uniform(-1, 1, n)
+    x0 = rng.uniform(-1, 1, n)
+    bd = torch.from_numpy(b).to("cuda")
+    xd = torch.from_numpy(x0).to("cuda")
+    res = A.cg(bd, xd, 40, 0.0, check_every=8, comm=comm, history=True)
+    torch.cuda.synchronize()
+    _compare(a, np.float64, b, x0, res, xd.cpu().numpy())
+    comm.close()
