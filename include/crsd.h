@@ -63,6 +63,13 @@ typedef enum { CRSD_R32F = 0, CRSD_R64F = 1 } crsd_dtype_t;
 #define CRSD_SUM_DUPLICATES 0x1u /* duplicates are summed (in input order) instead of rejected */
 #define CRSD_HOST_ONLY 0x2u      /* build the CRSD structure on the host only (export/inspection); no device memory is touched and crsd_spmv* return CRSD_ERR_UNSUPPORTED */
 #define CRSD_DROP_ZEROS 0x4u     /* explicit zero entries are dropped instead of kept in the scatter list (R10) */
+#define CRSD_PAPER_ELL 0x8u      /* paper-exact scatter handling: every row holding a
+                                    scatter point is also stored whole in ELL and, after the diagonal part, its
+                                    y is OVERWRITTEN by the ELL row product, accumulated in ascending column
+                                    order with separately rounded multiplies and adds (CSR order). crsd_spmv
+                                    then needs beta == 0 (the paper computes y = A x; UNSUPPORTED otherwise);
+                                    one-GPU handles only; crsd_spmv_host / _dist / crsd_cg return UNSUPPORTED.
+                                    DESIGN.md R5/R6, §8(f) NEXT 3. */
 
 /*
  * Build options. Call crsd_opts_init() for defaults (NULL opts == defaults).
@@ -279,6 +286,16 @@ crsd_status_t crsd_dist_plan(int world, int rank, const int64_t *ranges4, int64_
 crsd_status_t crsd_partition_rows(int64_t nrows, int32_t mrows, int world, const double *weights,
                                   int64_t *bounds);
 
+/* The paper's scatter-row ELL arrays of a CRSD_PAPER_ELL handle (Fig. 4
+ * `num_scatter_rows`, `scatter_rowno`, `num_scatter_width`, `scatter_colval`,
+ * `scatter_val`). Two-call protocol: pass NULL
+ * arrays to get *nrows_s and *width; then HOST buffers rowno[nrows_s] (global
+ * rows), colval[width*nrows_s] and val[width*nrows_s] (dtype), column-major
+ * (entry k of row i at k*nrows_s + i), padding col -1 / value 0.
+ * UNSUPPORTED if the handle was built without CRSD_PAPER_ELL. */
+crsd_status_t crsd_export_paper_ell(crsd_matrix_t A, int64_t *nrows_s, int64_t *width, int64_t *rowno,
+                                    int64_t *colval, void *val);
+
 /* Introspection */
 crsd_status_t crsd_get_info(crsd_matrix_t A, crsd_info_t *info);
 crsd_status_t crsd_export(crsd_matrix_t A, crsd_export_t *out);
@@ -336,6 +353,21 @@ typedef struct {
 crsd_status_t crsd_cg(crsd_matrix_t A, const void *b, void *x, int32_t max_iter, double rtol,
                       int32_t check_every, crsd_comm_t comm, double *rr_history, crsd_cg_result_t *res,
                       void *stream);
+
+/*
+ * Runtime autotuning of the kernel variant (the paper
+ * leaves such choices to "the property of matrices"). Times
+ * y = A x for every variant whose staging fits (LDG, TMA, PIPE, JIT; the JIT
+ * codelets are compiled here if needed) over `reps` launches each (<= 0 =>
+ * 20, after 3 warm-ups) and makes the fastest the handle's variant.
+ *   x, y     DEVICE vectors as for crsd_spmv (y is overwritten).
+ *   ms_out   HOST double[5] or NULL: ms_out[v] = mean ms per launch of
+ *            variant v (1..4), -1 if not applicable; ms_out[0] = the best.
+ *   chosen   HOST or NULL: the variant chosen (CRSD_VARIANT_*).
+ * Synchronous. One-GPU (non-partitioned) handles only.
+ */
+crsd_status_t crsd_autotune(crsd_matrix_t A, const void *x, void *y, int32_t reps, double *ms_out,
+                            int32_t *chosen, void *stream);
 
 /* Number of kernel launches the last crsd_spmv / crsd_spmv_dist / crsd_cg call made. */
 crsd_status_t crsd_last_launch_count(crsd_matrix_t A, int32_t *count);

@@ -288,3 +288,25 @@ def to_layout(R: CRSDRef) -> dict:
         scat_col=np.array(cs, dtype=np.int64),
         scat_val=np.array(vs, dtype=R.crsd_dia_val.dtype),
     )
+
+
+def paper_ell_rows(R: CRSDRef, x, alpha=1.0, dtype=np.float64):
+    """Second part of the paper's SpMV kernel ("the final kernel is
+    composed of two parts"; the ELL part computes the scatter rows, stored
+    whole): for every stored row i, y[scatter_rowno[i]] =
+    alpha * (((0 + v_0 x_0) + v_1 x_1) + ...), entries in stored (ascending
+    column) order, each product and sum rounded to `dtype` separately (the
+    CSR evaluation order). Returns {row: value} in `dtype`."""
+    dt = np.dtype(dtype).type
+    N, W = R.num_scatter_rows, R.num_scatter_width
+    x = np.asarray(x, dtype=dt)
+    out = {}
+    for i, r in enumerate(R.scatter_rowno):
+        s = dt(0)
+        for k in range(W):
+            c = R.scatter_colval[k * N + i]
+            if c < 0:
+                break
+            s = dt(s + dt(dt(R.scatter_val[k * N + i]) * x[c]))
+        out[r] = dt(dt(alpha) * s)
+    return out

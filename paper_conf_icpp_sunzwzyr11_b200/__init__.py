@@ -13,4 +13,6 @@ from .crsd import (  # noqa: F401
     CRSD_SUM_DUPLICATES,
     CRSD_HOST_ONLY,
     CRSD_DROP_ZEROS,
+    CRSD_PAPER_ELL,
+    CGResult,
 )

@@ -26,7 +26,7 @@ STATUS = {
     7: "CRSD_ERR_NCCL",
 }
 CRSD_R32F, CRSD_R64F = 0, 1
-CRSD_SUM_DUPLICATES, CRSD_HOST_ONLY, CRSD_DROP_ZEROS = 0x1, 0x2, 0x4
+CRSD_SUM_DUPLICATES, CRSD_HOST_ONLY, CRSD_DROP_ZEROS, CRSD_PAPER_ELL = 0x1, 0x2, 0x4, 0x8
 VARIANT_AUTO, VARIANT_LDG, VARIANT_TMA, VARIANT_PIPE, VARIANT_JIT = 0, 1, 2, 3, 4
 
 # every symbol include/crsd.h declares
@@ -52,6 +52,8 @@ EXPORTED = [
     "crsd_last_launch_count",
     "crsd_jit_source",
     "crsd_cg",
+    "crsd_autotune",
+    "crsd_export_paper_ell",
 ]
 
 
@@ -148,6 +150,8 @@ def _load():
         "crsd_last_launch_count": ([P, P], ctypes.c_int),
         "crsd_jit_source": ([P, P, I64, P], ctypes.c_int),
         "crsd_cg": ([P, P, P, I32, ctypes.c_double, I32, P, P, P, P], ctypes.c_int),
+        "crsd_autotune": ([P, P, P, I32, P, P, P], ctypes.c_int),
+        "crsd_export_paper_ell": ([P, P, P, P, P, P], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)
@@ -344,6 +348,24 @@ class CRSDMatrix:
         if history:
             out["rr_history"] = hist[: res.iterations + 1]
         return out
+
+    def autotune(self, x, y, reps=20, stream=None) -> dict:
+        """Time every applicable kernel variant on (x, y) and keep the fastest
+        (crsd_autotune). Returns {"chosen": v, "ms": {variant: ms or None}}."""
+        ms = np.zeros(5, np.float64)
+        ch = ctypes.c_int32()
+        _check(lib.crsd_autotune(self._h, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(y.data_ptr()), int(reps), _p(ms), ctypes.byref(ch), _stream_ptr(stream)))
+        return {"chosen": ch.value, "ms": {v: (None if ms[v] < 0 else float(ms[v])) for v in range(1, 5)}}
+
+    def export_paper_ell(self) -> dict:
+        """The paper's scatter-row ELL arrays of a CRSD_PAPER_ELL handle (Fig. 4 names)."""
+        n, w = ctypes.c_int64(), ctypes.c_int64()
+        _check(lib.crsd_export_paper_ell(self._h, ctypes.byref(n), ctypes.byref(w), None, None, None))
+        rowno = np.zeros(n.value, np.int64)
+        colval = np.zeros(n.value * w.value, np.int64)
+        val = np.zeros(n.value * w.value, self.dtype)
+        _check(lib.crsd_export_paper_ell(self._h, None, None, _p(rowno), _p(colval), _p(val)))
+        return {"num_scatter_rows": n.value, "num_scatter_width": w.value, "scatter_rowno": rowno, "scatter_colval": colval, "scatter_val": val}
 
     def dist_bind(self, comm, stream=None):
         _check(lib.crsd_dist_bind(self._h, comm._h, _stream_ptr(stream)))

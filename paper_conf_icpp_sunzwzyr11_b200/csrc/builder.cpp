@@ -441,6 +441,43 @@ crsd_status_t build_from_csr_t(int64_t nrows, int64_t ncols, CSR<T> &C, const Bu
             }
         }
     }
+    // pass C (CRSD_PAPER_ELL): the paper's scatter storage --
+    // every row with a scatter point, whole (all its entries, ascending
+    // columns), in ELL: column-major, width = the longest such row, padding
+    // col -1 / value 0 (Bell & Garland ELL; R6)
+    H.paper_ell = (o.flags & CRSD_PAPER_ELL) != 0;
+    if (H.paper_ell) {
+        std::vector<int64_t> rows;
+        for (int64_t s = 0; s < nseg; ++s)
+            for (int64_t e = H.scat_ptr[s]; e < H.scat_ptr[s + 1]; ++e) {
+                const int64_t r = s * m + H.scat_row[e];
+                if (rows.empty() || rows.back() != r) rows.push_back(r);
+            }
+        auto row_len = [&](int64_t r) {
+            int64_t k = 0;
+            for (int64_t e = ptr[r]; e < ptr[r + 1]; ++e) k += !(drop_zeros && is_zero(val[e]));
+            return k;
+        };
+        int64_t W = 0;
+        for (int64_t r : rows) W = std::max(W, row_len(r));
+        const int64_t N = (int64_t)rows.size();
+        H.ell_nrows = N;
+        H.ell_width = W;
+        H.ell_rowno = rows;
+        H.ell_col.assign((size_t)(N * W), -1);
+        H.ell_val.assign((size_t)(N * W) * sizeof(T), 0);
+        T *EV = reinterpret_cast<T *>(H.ell_val.data());
+        for (int64_t i = 0; i < N; ++i) {
+            const int64_t r = rows[i];
+            int64_t k = 0;
+            for (int64_t e = ptr[r]; e < ptr[r + 1]; ++e) {
+                if (drop_zeros && is_zero(val[e])) continue;
+                H.ell_col[k * N + i] = col[e];
+                EV[k * N + i] = val[e];
+                ++k;
+            }
+        }
+    }
     return CRSD_OK;
 }
 

@@ -69,11 +69,13 @@ void free_device(crsd_matrix_s *A) {
         A->cg_stream = A->cg_ev_in = A->cg_ev_out = nullptr;
     }
     void *ptrs[] = {A->d_vals, A->d_segs, A->d_offs, A->d_plan, A->d_scat_row, A->d_scat_col, A->d_scat_val, A->d_scat_rec,
-                    A->d_list_interior, A->d_list_boundary, A->d_list_all_edge, A->d_x_scratch, A->d_y_scratch, A->d_cg};
+                    A->d_list_interior, A->d_list_boundary, A->d_list_all_edge, A->d_x_scratch, A->d_y_scratch, A->d_cg,
+                    A->d_ell_rowno, A->d_ell_col, A->d_ell_val};
     for (void *p : ptrs)
         if (p) cudaFree(p);
     A->d_vals = A->d_segs = A->d_offs = A->d_plan = A->d_scat_row = A->d_scat_col = A->d_scat_val = A->d_scat_rec = nullptr;
     A->d_list_interior = A->d_list_boundary = A->d_list_all_edge = A->d_x_scratch = A->d_y_scratch = A->d_cg = nullptr;
+    A->d_ell_rowno = A->d_ell_col = A->d_ell_val = nullptr;
     A->cg_bytes = 0;
 }
 
@@ -175,6 +177,11 @@ static crsd_status_t upload(crsd_matrix_s *A) {
     }
     if ((st = dev_alloc_copy(&A->d_list_interior, A->list_interior.data(), A->list_interior.size() * 4, cnt))) return st;
     if ((st = dev_alloc_copy(&A->d_list_boundary, A->list_boundary.data(), A->list_boundary.size() * 4, cnt))) return st;
+    if (H.paper_ell && H.ell_nrows > 0) {
+        if ((st = dev_alloc_copy(&A->d_ell_rowno, H.ell_rowno.data(), H.ell_rowno.size() * 8, cnt))) return st;
+        if ((st = dev_alloc_copy(&A->d_ell_col, H.ell_col.data(), H.ell_col.size() * 8, cnt))) return st;
+        if ((st = dev_alloc_copy(&A->d_ell_val, H.ell_val.data(), H.ell_val.size(), cnt))) return st;
+    }
     // the host copy of the bulk arrays is dropped after upload (export reads the device copy)
     std::vector<uint8_t>().swap(H.vals);
     std::vector<uint8_t>().swap(H.scat_val);
@@ -282,9 +289,13 @@ static crsd_status_t resolve_opts(int64_t nrows, crsd_dtype_t dtype, const crsd_
 
 template <typename T>
 static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *y, const int32_t *list,
-                              int64_t seg_begin, int64_t count, void *stream, int &launches) {
+                              int64_t seg_begin, int64_t count, void *stream, int &launches, const DotArgs *dot) {
     if (count <= 0) return CRSD_OK;
+    if (dot && A->variant != VARIANT_JIT) return fail(CRSD_ERR_UNSUPPORTED, "fused dot needs the JIT variant");
     SpmvArgs<T> a;
+    a.dot_part = dot ? dot->part : nullptr;
+    a.dot_cnt = dot ? dot->cnt : nullptr;
+    a.dot_out = dot ? dot->out : nullptr;
     a.vals = (const T *)A->d_vals;
     a.segs = (const SegDesc *)A->d_segs;
     a.pat_offs = (const int32_t *)A->d_offs;
@@ -330,12 +341,13 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
 }
 
 crsd_status_t run_lists(crsd_matrix_s *A, const void *alpha, const void *x_base, const void *beta, void *y,
-                        const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches) {
+                        const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches,
+                        const DotArgs *dot) {
     if (A->H.dtype == CRSD_R64F)
         return run_spmv<double>(A, *(const double *)alpha, (const double *)x_base, *(const double *)beta, (double *)y,
-                                list, seg_begin, count, stream, launches);
+                                list, seg_begin, count, stream, launches, dot);
     return run_spmv<float>(A, *(const float *)alpha, (const float *)x_base, *(const float *)beta, (float *)y, list,
-                           seg_begin, count, stream, launches);
+                           seg_begin, count, stream, launches, dot);
 }
 
 }  // namespace crsd
@@ -378,6 +390,10 @@ static crsd_status_t create_common(int64_t nrows, int64_t ncols, crsd_dtype_t dt
         return st;
     }
     A->H.partitioned = !(o.row_begin == 0 && o.row_end == nrows);
+    if (A->H.partitioned && (o.flags & CRSD_PAPER_ELL)) {
+        delete A;
+        return fail(CRSD_ERR_UNSUPPORTED, "CRSD_PAPER_ELL needs a one-GPU (non-partitioned) handle");
+    }
     if (A->H.partitioned && nrows != ncols) {
         delete A;
         return fail(CRSD_ERR_UNSUPPORTED, "row-partitioned handles need a square matrix");
@@ -416,10 +432,26 @@ crsd_status_t crsd_spmv(crsd_matrix_t A, const void *alpha, const void *x, const
     crsd_status_t st;
     if ((st = check_vec(x, "x")) || (st = check_vec(y, "y"))) return st;
     if (x == y) return fail(CRSD_ERR_INVALID_ARG, "x and y must not alias");
+    const bool beta_nz = (A->H.dtype == CRSD_R64F) ? (*(const double *)beta != 0.0) : (*(const float *)beta != 0.0f);
+    if (A->H.paper_ell && beta_nz)
+        return fail(CRSD_ERR_UNSUPPORTED, "CRSD_PAPER_ELL handles compute y = alpha*A*x (beta must be 0): the ELL part overwrites y");
     int launches = 0;
     cudaSetDevice(A->device);
     const int64_t nseg = A->H.nseg;
     st = run_lists(A, alpha, x, beta, y, nullptr, 0, nseg, stream, launches);
+    if (!st && A->H.paper_ell && A->H.ell_nrows > 0) {
+        // second part of the paper's kernel: the scatter rows,
+        // stored whole in ELL, overwrite what the diagonal part wrote
+        const int e = A->H.dtype == CRSD_R64F
+                          ? launch_paper_ell<double>((const int64_t *)A->d_ell_rowno, (const int64_t *)A->d_ell_col,
+                                                     (const double *)A->d_ell_val, A->H.ell_nrows, A->H.ell_width,
+                                                     (const double *)x, (double *)y, *(const double *)alpha, stream)
+                          : launch_paper_ell<float>((const int64_t *)A->d_ell_rowno, (const int64_t *)A->d_ell_col,
+                                                    (const float *)A->d_ell_val, A->H.ell_nrows, A->H.ell_width,
+                                                    (const float *)x, (float *)y, *(const float *)alpha, stream);
+        if (e) st = fail(CRSD_ERR_CUDA, std::string("paper ELL kernel launch: ") + cudaGetErrorString((cudaError_t)e));
+        else ++launches;
+    }
     A->last_launches = launches;
     return st;
 }
@@ -486,6 +518,7 @@ crsd_status_t crsd_spmv_host(crsd_matrix_t A, const void *alpha, const void *x_h
     if (!A) return fail(CRSD_ERR_INVALID_ARG, "A is NULL");
     if (A->host_only) return fail(CRSD_ERR_UNSUPPORTED, "host-only handle");
     if (A->H.partitioned) return fail(CRSD_ERR_UNSUPPORTED, "row-partitioned handle");
+    if (A->H.paper_ell) return fail(CRSD_ERR_UNSUPPORTED, "CRSD_PAPER_ELL handle: use crsd_spmv");
     if (!x_host || !y_host || !alpha || !beta) return fail(CRSD_ERR_INVALID_ARG, "NULL argument");
     CUDA_TRY(cudaSetDevice(A->device));
     const size_t es = A->H.elem;
@@ -608,6 +641,87 @@ crsd_status_t crsd_export(crsd_matrix_t A, crsd_export_t *E) {
         if (E->vals && vb) std::memcpy(E->vals, H.vals.data(), vb);
         if (E->scat_val && sb) std::memcpy(E->scat_val, H.scat_val.data(), sb);
     }
+    return CRSD_OK;
+}
+
+// Runtime autotuning of the kernel variant (the
+// paper leaves such choices to "the property of matrices"):
+// every variant whose staging fits is timed on the caller's vectors and the
+// fastest becomes the handle's variant.
+crsd_status_t crsd_autotune(crsd_matrix_t A, const void *x, void *y, int32_t reps, double *ms_out, int32_t *chosen,
+                            void *stream) {
+    if (!A) return fail(CRSD_ERR_INVALID_ARG, "A is NULL");
+    if (A->host_only) return fail(CRSD_ERR_UNSUPPORTED, "host-only handle");
+    if (A->H.partitioned) return fail(CRSD_ERR_UNSUPPORTED, "row-partitioned handle");
+    crsd_status_t st;
+    if ((st = check_vec(x, "x")) || (st = check_vec(y, "y"))) return st;
+    if (x == y) return fail(CRSD_ERR_INVALID_ARG, "x and y must not alias");
+    if (reps <= 0) reps = 20;
+    // (CRSD_PAPER_ELL: only the diagonal-part kernel is tuned; the ELL pass is fixed)
+    CUDA_TRY(cudaSetDevice(A->device));
+    cudaStream_t s = (cudaStream_t)stream;
+    const int64_t smem_cap = 200 * 1024;
+    const int64_t pipe_need = 2 * A->xmax_elems * A->H.elem + 2 * 8 * (int64_t)A->H.mrows * A->H.elem + 1024;
+    const int original = A->variant;
+    double best = 1e300;
+    int best_v = original;
+    cudaEvent_t e0, e1;
+    CUDA_TRY(cudaEventCreate(&e0));
+    CUDA_TRY(cudaEventCreate(&e1));
+    const double one_d = 1.0, zero_d = 0.0;
+    const float one_f = 1.0f, zero_f = 0.0f;
+    const bool f64 = A->H.dtype == CRSD_R64F;
+    const void *one = f64 ? (const void *)&one_d : (const void *)&one_f;
+    const void *zero = f64 ? (const void *)&zero_d : (const void *)&zero_f;
+    for (int v = VARIANT_LDG; v <= VARIANT_JIT; ++v) {
+        double ms = -1.0;
+        bool ok = true;
+        if (v == VARIANT_TMA) ok = A->tma_smem <= smem_cap;
+        if (v == VARIANT_PIPE) ok = pipe_need <= smem_cap && A->H.mrows <= 1024;
+        if (v == VARIANT_JIT) {
+            ok = A->smem_bytes <= smem_cap;
+            if (ok && !A->jit_function) ok = jit_build(A) == CRSD_OK;
+        }
+        if (ok) {
+            A->variant = v;
+            int l = 0;
+            st = CRSD_OK;
+            for (int i = 0; i < 3 && !st; ++i) st = run_lists(A, one, x, zero, y, nullptr, 0, A->H.nseg, s, l);
+            if (!st) CUDA_TRY(cudaEventRecord(e0, s));
+            for (int i = 0; i < reps && !st; ++i) st = run_lists(A, one, x, zero, y, nullptr, 0, A->H.nseg, s, l);
+            if (!st) {
+                CUDA_TRY(cudaEventRecord(e1, s));
+                CUDA_TRY(cudaEventSynchronize(e1));
+                float t = 0.f;
+                CUDA_TRY(cudaEventElapsedTime(&t, e0, e1));
+                ms = t / reps;
+                if (ms < best) {
+                    best = ms;
+                    best_v = v;
+                }
+            }
+        }
+        if (ms_out) ms_out[v] = ms;
+    }
+    if (ms_out) ms_out[0] = best;
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    A->variant = best_v;
+    if (chosen) *chosen = best_v;
+    return CRSD_OK;
+}
+
+crsd_status_t crsd_export_paper_ell(crsd_matrix_t A, int64_t *nrows_s, int64_t *width, int64_t *rowno,
+                                    int64_t *colval, void *val) {
+    if (!A) return fail(CRSD_ERR_INVALID_ARG, "A is NULL");
+    const HostCRSD &H = A->H;
+    if (!H.paper_ell) return fail(CRSD_ERR_UNSUPPORTED, "handle built without CRSD_PAPER_ELL");
+    if (nrows_s) *nrows_s = H.ell_nrows;
+    if (width) *width = H.ell_width;
+    if (rowno)
+        for (int64_t i = 0; i < H.ell_nrows; ++i) rowno[i] = H.ell_rowno[i] + H.row_begin;
+    if (colval && !H.ell_col.empty()) std::memcpy(colval, H.ell_col.data(), H.ell_col.size() * 8);
+    if (val && !H.ell_val.empty()) std::memcpy(val, H.ell_val.data(), H.ell_val.size());
     return CRSD_OK;
 }
 

@@ -48,6 +48,9 @@ struct crsd_matrix_s {
     void *d_list_interior = nullptr;
     void *d_list_boundary = nullptr;
     void *d_list_all_edge = nullptr;
+    void *d_ell_rowno = nullptr;  // CRSD_PAPER_ELL: scatter rows stored whole (int64 local rows)
+    void *d_ell_col = nullptr;    // int64, column-major, -1 padded
+    void *d_ell_val = nullptr;
     void *d_x_scratch = nullptr;
     void *d_y_scratch = nullptr;
 
@@ -82,6 +85,13 @@ template <typename T>
 int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &a, void *stream);
 // Run the SpMV kernel over a device list of segments (list == nullptr: all
 // segments [0, count)). x_base is the local x base (x_padded + halo_lo).
+// dot != null (JIT variant only, one launch): also *dot->out = sum_rows x[row] * y[row].
+struct DotArgs {
+    double *part;   // >= count partials
+    uint32_t *cnt;  // zero between launches
+    double *out;
+};
 crsd_status_t run_lists(crsd_matrix_s *A, const void *alpha, const void *x_base, const void *beta, void *y,
-                        const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches);
+                        const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches,
+                        const DotArgs *dot = nullptr);
 }  // namespace crsd

@@ -89,6 +89,15 @@ struct HostCRSD {
     std::vector<int64_t> scat_col;    // global column
     std::vector<uint8_t> scat_val;    // nscatter * elem
 
+    // paper-exact scatter rows (flag CRSD_PAPER_ELL): every row
+    // holding a scatter point, stored WHOLE in ELL (column-major, ascending
+    // columns, col -1 / value 0 padding); the SpMV overwrites those rows
+    bool paper_ell = false;
+    int64_t ell_nrows = 0, ell_width = 0;
+    std::vector<int64_t> ell_rowno;   // local row of each ELL row
+    std::vector<int64_t> ell_col;     // ell_width * ell_nrows, global column or -1
+    std::vector<uint8_t> ell_val;     // same, dtype
+
     // column extent actually referenced (global), over stored entries
     int64_t min_col_ref = 0, max_col_ref = -1;
 
@@ -157,7 +166,19 @@ struct SpmvArgs {
     int32_t has_scatter;      // the matrix has scatter points (selects the staging kernel)
     int32_t variant;          // VARIANT_LDG or VARIANT_TMA
     T alpha, beta;
+    // optional fused dot (JIT variant, CG): *dot_out = sum_rows x[row] * y[row]
+    // over the launch's rows, deterministic (per-CTA partials, last CTA sums)
+    double *dot_part;         // one per CTA, or null
+    uint32_t *dot_cnt;        // zero on entry, reset by the last CTA
+    double *dot_out;
 };
+
+// Paper-exact scatter rows (CRSD_PAPER_ELL): y[rowno[i]] = alpha * sum_k
+// val[k*n+i] * x[col[k*n+i]], ascending k, separately rounded mul and add.
+// Returns a cudaError_t value (0 = ok).
+template <typename T>
+int launch_paper_ell(const int64_t *rowno, const int64_t *col, const T *val, int64_t n, int64_t width, const T *x,
+                     T *y, T alpha, void *stream);
 
 // Launch the SpMV kernel for the given work (range or list) on `stream`.
 // Returns number of launches (0 if no work) or -1 on launch error.

@@ -184,6 +184,7 @@ crsd_status_t crsd_spmv_dist(crsd_matrix_t A, const void *alpha, void *x_padded,
                              crsd_comm_t c, void *stream) {
     if (!A) return crsd::fail(CRSD_ERR_INVALID_ARG, "A is NULL");
     if (A->host_only) return crsd::fail(CRSD_ERR_UNSUPPORTED, "host-only handle");
+    if (A->H.paper_ell) return crsd::fail(CRSD_ERR_UNSUPPORTED, "CRSD_PAPER_ELL handle: use crsd_spmv");
     if (!alpha || !beta || !x_padded || !y_local) return crsd::fail(CRSD_ERR_INVALID_ARG, "NULL argument");
     if (((uintptr_t)x_padded | (uintptr_t)y_local) & 15)
         return crsd::fail(CRSD_ERR_INVALID_ARG, "x_padded and y_local must be 16-byte aligned");

@@ -128,6 +128,9 @@ struct JitArgs {
     const T *scat_val;
     const ScatRec *scat_rec;
     T alpha, beta;
+    double *dot_part;
+    uint32_t *dot_cnt;
+    double *dot_out;
 };
 
 const char *kPrelude = R"(
@@ -139,7 +142,8 @@ struct SegDesc { i64 val_base; i64 scat_begin; int off_begin; int nscat; u16 fla
 struct __align__(16) ScatRec { i64 col; double val; int row; int pad[3]; };
 struct Args { const T *vals; const SegDesc *segs; const int *seg_list; i64 seg_begin, seg_count;
               const T *x; i64 x_lo, x_hi; T *y; i64 nrows;
-              const int *scat_row; const i64 *scat_col; const T *scat_val; const ScatRec *scat_rec; T alpha, beta; };
+              const int *scat_row; const i64 *scat_col; const T *scat_val; const ScatRec *scat_rec; T alpha, beta;
+              double *dot_part; u32 *dot_cnt; double *dot_out; };
 __device__ __forceinline__ u32 su32(const void *p) { return (u32)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void bar_init(u64 *b) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(su32(b)) : "memory");
@@ -185,7 +189,7 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
         const int64_t *offs = H.pat_offsets.data() + H.pat_ptr[I.pattern];
         o << "// pattern offsets:";
         for (int d = 0; d < nd; ++d) o << " " << offs[d];
-        o << "\n__device__ __forceinline__ void codelet_" << key
+        o << "\n__device__ __forceinline__ double codelet_" << key
           << "(const Args &a, const SegDesc &D, i64 row0, bool edge, T *vs, u64 *bar, int t) {\n";
         int64_t xb = 0;
         for (int w = 0; w < nwin; ++w) xb += pl[3 + 2 * w];
@@ -248,17 +252,38 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
                  "      const T v = __ldg(a.scat_val + D.scat_begin + e), xv = __ldg(a.x + __ldg(a.scat_col + D.scat_begin + e));\n"
                  "#pragma unroll\n      for (int q = 0; q < Q; ++q) if (rr / NT == q) acc[q] = fma(v, xv, acc[q]);\n"
                  "    }\n  }\n";
-        o << "#pragma unroll\n  for (int q = 0; q < Q; ++q) {\n    const i64 r = row0 + t + q * NT;\n"
-             "    if (!edge || r < a.nrows) { T *yp = a.y + r; __stcs(yp, (a.beta != T(0)) ? fma(a.alpha, acc[q], a.beta * *yp) : a.alpha * acc[q]); }\n"
-             "  }\n}\n";
+        // epilogue; with a fused dot (CG: (p, q) with p = x) each thread
+        // also accumulates x[row] * y[row] in fp64 (x[row] is an L2 hit: the
+        // window holding it was just bulk-copied)
+        o << "  double dsum = 0.0;\n#pragma unroll\n  for (int q = 0; q < Q; ++q) {\n    const i64 r = row0 + t + q * NT;\n"
+             "    if (!edge || r < a.nrows) {\n      T *yp = a.y + r;\n"
+             "      const T out = (a.beta != T(0)) ? fma(a.alpha, acc[q], a.beta * *yp) : a.alpha * acc[q];\n"
+             "      __stcs(yp, out);\n"
+             "      if (a.dot_part) dsum = fma((double)__ldg(a.x + r), (double)out, dsum);\n    }\n"
+             "  }\n  return dsum;\n}\n";
     }
     o << "extern \"C\" __global__ void __launch_bounds__(NT) crsd_jit(const Args a) {\n"
          "  extern __shared__ __align__(128) unsigned char smem[];\n  __shared__ u64 bar;\n"
          "  const i64 s = a.seg_list ? (i64)__ldg(a.seg_list + blockIdx.x) : a.seg_begin + blockIdx.x;\n"
          "  const SegDesc D = a.segs[s];\n  const i64 row0 = s * MROWS;\n  const bool edge = (D.flags & 1) != 0;\n"
-         "  T *vs = reinterpret_cast<T *>(smem);\n  switch (D.plan_begin) {\n";
-    for (int32_t v : seen) o << "  case " << v << ": codelet_" << v << "(a, D, row0, edge, vs, &bar, threadIdx.x); break;\n";
-    o << "  }\n}\n";
+         "  T *vs = reinterpret_cast<T *>(smem);\n  double d = 0.0;\n  switch (D.plan_begin) {\n";
+    for (int32_t v : seen) o << "  case " << v << ": d = codelet_" << v << "(a, D, row0, edge, vs, &bar, threadIdx.x); break;\n";
+    o << "  }\n";
+    // fused dot: per-CTA partial, the last CTA sums the partials in CTA order
+    o << "  if (a.dot_part) {\n"
+         "    __shared__ double red[NT / 32];\n    __shared__ bool last;\n"
+         "    for (int k = 16; k; k >>= 1) d += __shfl_down_sync(0xffffffffu, d, k);\n"
+         "    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = d;\n    __syncthreads();\n"
+         "    if (threadIdx.x == 0) {\n      double b = 0.0;\n      for (int k = 0; k < NT / 32; ++k) b += red[k];\n"
+         "      a.dot_part[blockIdx.x] = b;\n      __threadfence();\n"
+         "      last = atomicAdd(a.dot_cnt, 1u) == gridDim.x - 1;\n    }\n    __syncthreads();\n"
+         "    if (last) {\n      __threadfence();\n      double b = 0.0;\n"
+         "      for (unsigned k = threadIdx.x; k < gridDim.x; k += NT) b += *((volatile double *)a.dot_part + k);\n"
+         "      for (int k = 16; k; k >>= 1) b += __shfl_down_sync(0xffffffffu, b, k);\n"
+         "      __syncthreads();\n      if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = b;\n      __syncthreads();\n"
+         "      if (threadIdx.x == 0) {\n        double c = 0.0;\n        for (int k = 0; k < NT / 32; ++k) c += red[k];\n"
+         "        *a.dot_out = c;\n        *a.dot_cnt = 0u;\n      }\n    }\n  }\n";
+    o << "}\n";
     return o.str();
 }
 
@@ -339,6 +364,9 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
     j.scat_col = s.scat_col;
     j.scat_val = s.scat_val;
     j.scat_rec = s.scat_rec;
+    j.dot_part = s.dot_part;
+    j.dot_cnt = s.dot_cnt;
+    j.dot_out = s.dot_out;
     j.alpha = s.alpha;
     j.beta = s.beta;
     void *params[] = {&j};

@@ -13,6 +13,7 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -49,7 +50,7 @@ inline int64_t up256(int64_t b) { return (b + 255) / 256 * 256; }
 
 struct Ws {
     CgState *st;
-    double *partials, *hist;
+    double *partials, *hist, *dpart;  // dpart: one per segment (dot fused into the SpMV)
     char *r, *q, *p_pad;  // p_pad: halo_lo + n + halo_hi elements
 };
 
@@ -58,7 +59,8 @@ crsd_status_t workspace(crsd_matrix_s *A, int64_t max_iter, int grid, Ws &w) {
     const int64_t npad = A->halo_lo + n + A->halo_hi;
     const int64_t o_part = up256(sizeof(CgState));
     const int64_t o_hist = o_part + up256(8 * (int64_t)grid);
-    const int64_t o_r = o_hist + up256(8 * (max_iter + 1));
+    const int64_t o_dp = o_hist + up256(8 * (max_iter + 1));
+    const int64_t o_r = o_dp + up256(8 * std::max<int64_t>(1, A->H.nseg));
     const int64_t o_q = o_r + up256(es * n);
     const int64_t o_p = o_q + up256(es * n);
     const int64_t total = o_p + up256(es * npad);
@@ -83,6 +85,7 @@ crsd_status_t workspace(crsd_matrix_s *A, int64_t max_iter, int grid, Ws &w) {
     w.st = (CgState *)b;
     w.partials = (double *)(b + o_part);
     w.hist = (double *)(b + o_hist);
+    w.dpart = (double *)(b + o_dp);
     w.r = b + o_r;
     w.q = b + o_q;
     w.p_pad = b + o_p;
@@ -149,9 +152,18 @@ crsd_status_t cg_impl(crsd_matrix_s *A, const T *b, T *x, int32_t max_iter, doub
     if (comm) NC_TRY(ncclAllReduce(w.st->red + CG_RR, w.st->red + CG_RR, 2, f64, ncclSum, comm->comm, s));
     ST_TRY(kerr(cg_launch_init(w.st, s), "cg_init"));
 
+    // One GPU with the JIT variant: (p, q) is fused into the SpMV epilogue
+    // (saves one read of p and of q per step); otherwise a separate kernel.
+    const bool fused = !comm && A->variant == VARIANT_JIT && !getenv("CRSD_CG_NO_FUSED_DOT");
+    DotArgs dot{w.dpart, &w.st->dcounter, w.st->red + CG_PQ};
     auto step = [&]() -> crsd_status_t {
-        ST_TRY(spmv(T(1), T(0), q));  // q = A p
-        ST_TRY(kerr(cg_launch_dot<T>(p_own, q, n, w.st, CG_PQ, true, grid, s), "cg_dot(p,q)"));
+        if (fused) {
+            const T one(1), zero(0);
+            ST_TRY(run_lists(A, &one, p_own, &zero, q, nullptr, 0, nseg, s, launches, &dot));  // q = A p, (p, q)
+        } else {
+            ST_TRY(spmv(T(1), T(0), q));  // q = A p
+            ST_TRY(kerr(cg_launch_dot<T>(p_own, q, n, w.st, CG_PQ, true, grid, s), "cg_dot(p,q)"));
+        }
         if (comm) NC_TRY(ncclAllReduce(w.st->red + CG_PQ, w.st->red + CG_PQ, 1, f64, ncclSum, comm->comm, s));
         ST_TRY(kerr(cg_launch_update<T>(r, q, n, w.st, grid, s), "cg_update"));
         if (comm) NC_TRY(ncclAllReduce(w.st->red + CG_RR, w.st->red + CG_RR, 1, f64, ncclSum, comm->comm, s));
@@ -230,6 +242,7 @@ extern "C" crsd_status_t crsd_cg(crsd_matrix_t A, const void *b, void *x, int32_
     if (b == x) return fail(CRSD_ERR_INVALID_ARG, "b and x must not alias");
     if (max_iter < 0 || !(rtol >= 0.0)) return fail(CRSD_ERR_INVALID_ARG, "max_iter must be >= 0 and rtol >= 0");
     if (A->H.nrows != A->H.ncols) return fail(CRSD_ERR_UNSUPPORTED, "CG needs a square matrix");
+    if (A->H.paper_ell) return fail(CRSD_ERR_UNSUPPORTED, "CRSD_PAPER_ELL handle: CG needs y = alpha*A*x + beta*y");
     if (A->H.partitioned && !comm) return fail(CRSD_ERR_INVALID_ARG, "row-partitioned handle: pass its communicator");
     if (comm && !A->bound) return fail(CRSD_ERR_INVALID_ARG, "call crsd_dist_bind first");
     if (check_every <= 0) check_every = 16;

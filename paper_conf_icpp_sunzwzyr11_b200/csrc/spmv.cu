@@ -757,6 +757,47 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
     return e == cudaSuccess ? 1 : -(int)e;
 }
 
+// ---------------------------------------------------------------------------
+// Paper-exact scatter rows (CRSD_PAPER_ELL; P:L395-411 storage, P:L703-719
+// "the final kernel is composed of two parts": the ELL part runs after the
+// diagonal part and overwrites y for the rows it stores). One thread per
+// stored row, column-major ELL (coalesced across threads), the row product
+// accumulated in ascending column order with separately rounded multiply and
+// add -- the CSR evaluation order, reproducible bit for bit.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ double mul_rn(double a, double b) { return __dmul_rn(a, b); }
+__device__ __forceinline__ float mul_rn(float a, float b) { return __fmul_rn(a, b); }
+__device__ __forceinline__ double add_rn(double a, double b) { return __dadd_rn(a, b); }
+__device__ __forceinline__ float add_rn(float a, float b) { return __fadd_rn(a, b); }
+
+template <typename T>
+__global__ void __launch_bounds__(256) crsd_paper_ell(const int64_t *__restrict__ rowno, const int64_t *__restrict__ col,
+                                                      const T *__restrict__ val, int64_t n, int64_t width,
+                                                      const T *__restrict__ x, T *__restrict__ y, T alpha) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    T s = T(0);
+    for (int64_t k = 0; k < width; ++k) {
+        const int64_t c = __ldg(col + k * n + i);
+        if (c < 0) break;  // rows are left-packed: padding only at the end
+        s = add_rn(s, mul_rn(__ldg(val + k * n + i), __ldg(x + c)));
+    }
+    y[__ldg(rowno + i)] = mul_rn(alpha, s);
+}
+
+template <typename T>
+int launch_paper_ell(const int64_t *rowno, const int64_t *col, const T *val, int64_t n, int64_t width, const T *x,
+                     T *y, T alpha, void *stream) {
+    if (n <= 0) return 0;
+    crsd_paper_ell<T><<<(unsigned)((n + 255) / 256), 256, 0, (cudaStream_t)stream>>>(rowno, col, val, n, width, x, y, alpha);
+    return (int)cudaGetLastError();
+}
+
+template int launch_paper_ell<double>(const int64_t *, const int64_t *, const double *, int64_t, int64_t,
+                                      const double *, double *, double, void *);
+template int launch_paper_ell<float>(const int64_t *, const int64_t *, const float *, int64_t, int64_t, const float *,
+                                     float *, float, void *);
+
 template int launch_spmv<double>(const SpmvArgs<double> &, int, void *);
 template int launch_spmv<float>(const SpmvArgs<float> &, int, void *);
 

@@ -15,6 +15,7 @@ import gen
 from oracle import crsd_ref, decode
 from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, CRSDError, CRSD_SUM_DUPLICATES, CRSD_DROP_ZEROS
 from paper_conf_icpp_sunzwzyr11_b200 import crsd as C
+from tests.conftest import fig2_value
 
 
 def _bits(a):
@@ -220,3 +221,41 @@ def test_jit_codelets_compile_for_sm100a(case, dt, tmp_path):
     f.write_text(src)
     r = subprocess.run(["/usr/local/cuda/bin/nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-std=c++17", "-c", str(f), "-o", str(tmp_path / "k.o")], capture_output=True, text=True)
     assert r.returncode == 0, r.stderr[-2000:]
+
+
+def test_paper_ell_export_fig2_golden(fig2, fig2_expected):
+    """CRSD_PAPER_ELL: the product's scatter-row ELL arrays equal Fig. 4's
+    (num_scatter_rows, scatter_rowno, num_scatter_width, scatter_colval,
+    scatter_val; P:L503-511)."""
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSD_PAPER_ELL
+
+    n, m, r, c, v, _ = fig2
+    A = CRSDMatrix.from_coo(n, m, r, c, v, mrows=2, idle_max=1, host_only=True, flags=CRSD_PAPER_ELL)
+    E = A.export_paper_ell()
+    g = fig2_expected
+    assert E["num_scatter_rows"] == g["num_scatter_rows"]
+    assert E["num_scatter_width"] == g["num_scatter_width"]
+    assert E["scatter_rowno"].tolist() == g["scatter_rowno"]
+    assert E["scatter_colval"].tolist() == g["scatter_colval"]
+    assert E["scatter_val"].tolist() == [fig2_value(s) for s in g["scatter_val"]]
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_paper_ell_export_matches_oracle(seed):
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSD_PAPER_ELL
+
+    a = gen.random_diagonal(500, 460, seed, ndiag=7, n_scatter=60, n_zeros=5)
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, mrows=64, host_only=True, flags=CRSD_PAPER_ELL)
+    R = crsd_ref.build(a.nrows, a.ncols, a.row, a.col, a.val, mrows=64)
+    E = A.export_paper_ell()
+    assert E["num_scatter_rows"] == R.num_scatter_rows and E["num_scatter_width"] == R.num_scatter_width
+    assert E["scatter_rowno"].tolist() == R.scatter_rowno
+    assert E["scatter_colval"].tolist() == R.scatter_colval
+    assert np.array_equal(_bits(E["scatter_val"]), _bits(np.array(R.scatter_val, np.float64)))
+
+
+def test_paper_ell_needs_flag():
+    a = gen.config1()
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, host_only=True)
+    with pytest.raises(Exception, match="UNSUPPORTED"):
+        A.export_paper_ell()

@@ -394,3 +394,61 @@ def test_c5_rank_block_closed_form(torch_cuda, rank):
     y = yd.cpu().numpy()
     ref = closed_forms.stencil_apply(dims, "7pt", "linear", coef, rb, re)
     assert np.array_equal(y, ref)
+
+
+@pytest.mark.parametrize("case", ["c1", "c3s", "band"])
+def test_autotune_picks_fastest_and_keeps_parity(torch_cuda, case):
+    """crsd_autotune times every applicable variant and keeps the fastest;
+    the tuned handle still matches the oracle."""
+    a = {"c1": gen.config1, "c3s": lambda: gen.config3(n=36), "band": lambda: gen.config4(n=300_000)}[case]()
+    a = a.astype(np.float64)
+    A = _mat(a)
+    torch = torch_cuda
+    x = np.random.default_rng(3).uniform(-1, 1, a.ncols)
+    xd = torch.from_numpy(x).to("cuda")
+    yd = torch.empty(a.nrows, dtype=torch.float64, device="cuda")
+    r = A.autotune(xd, yd, reps=5)
+    ms = {v: t for v, t in r["ms"].items() if t is not None}
+    assert r["chosen"] in ms and ms[r["chosen"]] == min(ms.values())
+    assert A.info()["variant"] == r["chosen"]
+    y = _run(torch, A, x, -0.75, 0.0, None, a.nrows)
+    yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, x, -0.75, 0.0, None)
+    assert coo.parity_error(y, yref, scale) <= TOL[np.float64]
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+@pytest.mark.parametrize("case", ["fig2", "c1", "c3s", "rand"])
+def test_paper_ell_mode(torch_cuda, case, dt, variant):
+    """CRSD_PAPER_ELL (the paper's two-part kernel):
+    scatter rows are overwritten by the ELL part -- bit-exact against the
+    oracle's paper-order row products (separately rounded, ascending
+    columns); every other row matches the definition within tolerance."""
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSD_PAPER_ELL, CRSDError
+    from oracle import crsd_ref
+    from tests.conftest import load_fig2
+
+    mrows = None
+    if case == "fig2":
+        n, m, r, c, v, _ = load_fig2()
+        a = gen.COO(n, m, r, c, v)
+    elif case == "c1":
+        a = gen.config1()
+    elif case == "c3s":
+        a = gen.config3(n=24)
+    else:
+        a = gen.random_diagonal(3000, 2900, 7, ndiag=9, max_off=700, n_scatter=150)
+    a = a.astype(dt)
+    mrows = 64 if dt == np.float64 else 128
+    A = _mat(a, flags=CRSD_PAPER_ELL, variant=variant, mrows=mrows)
+    x = np.random.default_rng(21).uniform(-1, 1, a.ncols).astype(dt)
+    y = _run(torch_cuda, A, x, -0.75, 0.0, None, a.nrows)
+    R = crsd_ref.build(a.nrows, a.ncols, a.row, a.col, a.val, mrows=mrows)
+    ell = crsd_ref.paper_ell_rows(R, x, alpha=-0.75, dtype=dt)
+    assert len(ell) == R.num_scatter_rows > 0
+    rows = np.array(sorted(ell), np.int64)
+    assert np.array_equal(y[rows], np.array([ell[r] for r in rows], dtype=dt)), "ELL rows not bit-exact"
+    yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, x, -0.75, 0.0, None)
+    assert coo.parity_error(y, yref, scale) <= TOL[dt]
+    with pytest.raises(CRSDError, match="UNSUPPORTED"):
+        _run(torch_cuda, A, x, 1.0, 0.5, np.zeros(a.nrows, dt), a.nrows)

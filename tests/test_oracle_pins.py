@@ -269,3 +269,33 @@ def test_c3_present_center_rows_sum_to_zero():
     a = gen.config3(n=12, values="exact", scatter_frac=0.0)
     y, _ = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, np.ones(a.ncols))
     assert np.all(y == 0)
+
+
+def test_paper_ell_rows_fig2_exact(fig2):
+    """Fig. 2's scatter row 5 (scatter_rowno [5], colval [3,4,5,6])
+    computed by the paper's ELL part equals the row's dot product exactly
+    (small integers: every partial sum is exact)."""
+    n, m, r, c, v, _ = fig2
+    R = crsd_ref.build(n, m, r, c, v, mrows=2, idle_max=1)
+    x = np.arange(1, m + 1, dtype=np.float64)
+    out = crsd_ref.paper_ell_rows(R, x)
+    assert list(out) == [5]
+    row5 = [(cc, vv) for rr, cc, vv in zip(r, c, v) if rr == 5]
+    assert out[5] == sum(vv * x[cc] for cc, vv in row5)
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_paper_ell_rows_match_definition(dt):
+    """On random diagonal matrices with scatter points, the paper-order row
+    products of the scatter rows agree with the definition within the
+    recursive-summation bound (k u scale)."""
+    a = gen.random_diagonal(300, 280, 4, ndiag=6, n_scatter=40).astype(dt)
+    R = crsd_ref.build(a.nrows, a.ncols, a.row, a.col, a.val, mrows=32)
+    x = np.random.default_rng(5).uniform(-1, 1, a.ncols).astype(dt)
+    out = crsd_ref.paper_ell_rows(R, x, alpha=-0.75, dtype=dt)
+    yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, x, -0.75, 0.0, None)
+    assert len(out) == R.num_scatter_rows > 0
+    u = np.finfo(dt).eps
+    for row, val in out.items():
+        k = R.num_scatter_width + 2
+        assert abs(float(val) - yref[row]) <= k * u * scale[row]
