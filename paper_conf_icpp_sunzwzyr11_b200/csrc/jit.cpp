@@ -194,11 +194,16 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
         int64_t xb = 0;
         for (int w = 0; w < nwin; ++w) xb += pl[3 + 2 * w];
         o << "  T *xs = vs + " << (int64_t)nd * m << ";\n";
-        o << "  if (t == 0) { bar_init(bar); bar_expect(bar, " << (int64_t)nd * m * es << "u + (edge ? 0u : "
-          << xb * es << "u));\n";
-        if (nd) o << "    g2s(vs, a.vals + D.val_base, " << (int64_t)nd * m * es << "u, bar, pol_first()); }\n";
-        else o << "  }\n";
-        o << "  __syncthreads();\n";
+        // a pattern without diagonals (rows holding only scatter points, or
+        // nothing) stages nothing: no mbarrier at all
+        if (nd) {
+            o << "  if (t == 0) { bar_init(bar); bar_expect(bar, " << (int64_t)nd * m * es << "u + (edge ? 0u : "
+              << xb * es << "u));\n";
+            o << "    g2s(vs, a.vals + D.val_base, " << (int64_t)nd * m * es << "u, bar, pol_first()); }\n";
+            o << "  __syncthreads();\n";
+        } else {
+            o << "  (void)xs; (void)bar;\n";
+        }
         if (nwin) {
             o << "  if (!edge && t < 32) { const u64 pn = pol_normal();\n";
             int64_t base = 0;
@@ -225,7 +230,7 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
                  "  }\n";
         }
         o << "  T acc[Q];\n#pragma unroll\n  for (int q = 0; q < Q; ++q) acc[q] = T(0);\n";
-        o << "  bar_wait(bar);\n";
+        if (nd) o << "  bar_wait(bar);\n";
         const int32_t *xoff = pl + 2 + 2 * nwin;
         o << "  if (!edge) {\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n      const int r = t + q * NT;\n";
         for (int d = 0; d < nd; ++d)

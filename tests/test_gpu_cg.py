@@ -150,17 +150,29 @@ def test_cg_one_rank_communicator(torch_cuda):
     """The multi-GPU code path of crsd_cg (row-partitioned handle, bound NCCL
     communicator, crsd_spmv_dist halo exchange, allreduced dots) with one rank
     owning every row: must agree with the oracle like the one-GPU path."""
-    import os
-
     import torch
     import torch.distributed as dist
 
     from paper_conf_icpp_sunzwzyr11_b200 import Comm, CRSDMatrix
 
+    import socket
+
+    created = False
     if not dist.is_initialized():
-        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        os.environ.setdefault("MASTER_PORT", "29611")
-        dist.init_process_group("gloo", rank=0, world_size=1)
+        sk = socket.socket()
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+        sk.close()
+        dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=0, world_size=1)
+        created = True
+    try:
+        _one_rank_cg(torch, Comm, CRSDMatrix)
+    finally:
+        if created:
+            dist.destroy_process_group()
+
+
+def _one_rank_cg(torch, Comm, CRSDMatrix):
     a = gen.spd_stencil_scatter((24, 24, 24), "7pt", n_pairs=100, seed=6)
     n = a.nrows
     A = CRSDMatrix.from_coo(n, n, a.row, a.col, a.val, row_range=(0, n))
