@@ -20,6 +20,7 @@
 #include <nvrtc.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <sstream>
@@ -170,6 +171,7 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
     const bool f64 = H.dtype == CRSD_R64F;
     const int m = H.mrows, nt = m / Q, es = H.elem;
     const bool scat = H.nscatter() > 0;  // scatter code only for matrices that have scatter points
+    const bool early = getenv("CRSD_JIT_EARLY") && atoi(getenv("CRSD_JIT_EARLY")) != 0;
     std::ostringstream o;
     o << "typedef " << (f64 ? "double" : "float") << " T;\n" << kPrelude;
     o << "#define MROWS " << m << "\n#define NT " << nt << "\n#define Q " << Q << "\n";
@@ -196,30 +198,18 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
         o << "  T *xs = vs + " << (int64_t)nd * m << ";\n";
         // a pattern without diagonals (rows holding only scatter points, or
         // nothing) stages nothing: no mbarrier at all
-        if (nd) {
-            o << "  if (t == 0) { bar_init(bar); bar_expect(bar, " << (int64_t)nd * m * es << "u + (edge ? 0u : "
-              << xb * es << "u));\n";
-            o << "    g2s(vs, a.vals + D.val_base, " << (int64_t)nd * m * es << "u, bar, pol_first()); }\n";
-            o << "  __syncthreads();\n";
-        } else {
-            o << "  (void)xs; (void)bar;\n";
-        }
-        if (nwin) {
-            o << "  if (!edge && t < 32) { const u64 pn = pol_normal();\n";
-            int64_t base = 0;
-            for (int w = 0; w < nwin; ++w) {
-                o << "    if (t == " << (w % 32) << ") g2s(xs + " << base << ", a.x + row0 + (" << pl[2 + 2 * w] << "), "
-                  << (int64_t)pl[3 + 2 * w] * es << "u, bar, pn);\n";
-                base += pl[3 + 2 * w];
-            }
-            o << "  }\n";
-        }
+        // Copy issue. Default: thread 0 initialises the mbarrier and issues
+        // the value copy, then (after the CTA barrier) lane w of warp 0
+        // issues x window w. early (CRSD_JIT_EARLY=1): thread 0 issues every
+        // copy before the CTA barrier and the scatter gathers are issued
+        // before it too (A/B for the sweeps).
+        std::string sg;
         if (scat) {
             // scatter points are gathered while the bulk copies are in flight:
             // lane l of every warp reads record l of the segment's first 32
             // (row, col, value in one 32-B record); a ballot keeps those whose
             // row belongs to this warp, which alone load x[col]
-            o << "  int g_own = -1; T g_v = T(0), g_x = T(0); unsigned g_mask = 0u;\n"
+            sg = "  int g_own = -1; T g_v = T(0), g_x = T(0); unsigned g_mask = 0u;\n"
                  "  if (D.nscat > 0) {\n"
                  "    const int lane = t & 31;\n"
                  "    ScatRec R; R.col = 0; R.val = 0; R.row = 0;\n"
@@ -229,7 +219,45 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
                  "    if (mine) { g_v = *reinterpret_cast<const T *>(&R.val); g_x = __ldg(a.x + R.col); }\n"
                  "  }\n";
         }
+        // a pattern without diagonals (rows holding only scatter points, or
+        // nothing) stages nothing: no mbarrier at all
+        if (nd) {
+            o << "  if (t == 0) { bar_init(bar); bar_expect(bar, " << (int64_t)nd * m * es << "u + (edge ? 0u : "
+              << xb * es << "u));\n";
+            o << "    g2s(vs, a.vals + D.val_base, " << (int64_t)nd * m * es << "u, bar, pol_first());\n";
+            if (early && nwin) {
+                o << "    if (!edge) { const u64 pn = pol_normal();\n";
+                int64_t base = 0;
+                for (int w = 0; w < nwin; ++w) {
+                    o << "      g2s(xs + " << base << ", a.x + row0 + (" << pl[2 + 2 * w] << "), "
+                      << (int64_t)pl[3 + 2 * w] * es << "u, bar, pn);\n";
+                    base += pl[3 + 2 * w];
+                }
+                o << "    }\n";
+            }
+            o << "  }\n";
+            if (early) o << sg;
+            o << "  __syncthreads();\n";
+        } else {
+            o << "  (void)xs; (void)bar;\n";
+            if (early) o << sg;
+        }
+        if (nwin && !early) {
+            o << "  if (!edge && t < 32) { const u64 pn = pol_normal();\n";
+            int64_t base = 0;
+            for (int w = 0; w < nwin; ++w) {
+                o << "    if (t == " << (w % 32) << ") g2s(xs + " << base << ", a.x + row0 + (" << pl[2 + 2 * w] << "), "
+                  << (int64_t)pl[3 + 2 * w] * es << "u, bar, pn);\n";
+                base += pl[3 + 2 * w];
+            }
+            o << "  }\n";
+        }
+        if (!early) o << sg;
         o << "  T acc[Q];\n#pragma unroll\n  for (int q = 0; q < Q; ++q) acc[q] = T(0);\n";
+        // fused dot: x[row] is loaded now, while the bulk copies fly, not in
+        // the epilogue (a load there would add a memory latency to every CTA)
+        o << "  T xr[Q];\n  if (a.dot_part) {\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n"
+             "      const i64 r = row0 + t + q * NT;\n      xr[q] = (!edge || r < a.nrows) ? __ldg(a.x + r) : T(0);\n    }\n  }\n";
         if (nd) o << "  bar_wait(bar);\n";
         const int32_t *xoff = pl + 2 + 2 * nwin;
         o << "  if (!edge) {\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n      const int r = t + q * NT;\n";
@@ -258,13 +286,12 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
                  "#pragma unroll\n      for (int q = 0; q < Q; ++q) if (rr / NT == q) acc[q] = fma(v, xv, acc[q]);\n"
                  "    }\n  }\n";
         // epilogue; with a fused dot (CG: (p, q) with p = x) each thread
-        // also accumulates x[row] * y[row] in fp64 (x[row] is an L2 hit: the
-        // window holding it was just bulk-copied)
+        // also accumulates x[row] * y[row] in fp64
         o << "  double dsum = 0.0;\n#pragma unroll\n  for (int q = 0; q < Q; ++q) {\n    const i64 r = row0 + t + q * NT;\n"
              "    if (!edge || r < a.nrows) {\n      T *yp = a.y + r;\n"
              "      const T out = (a.beta != T(0)) ? fma(a.alpha, acc[q], a.beta * *yp) : a.alpha * acc[q];\n"
              "      __stcs(yp, out);\n"
-             "      if (a.dot_part) dsum = fma((double)__ldg(a.x + r), (double)out, dsum);\n    }\n"
+             "      if (a.dot_part) dsum = fma((double)xr[q], (double)out, dsum);\n    }\n"
              "  }\n  return dsum;\n}\n";
     }
     o << "extern \"C\" __global__ void __launch_bounds__(NT) crsd_jit(const Args a) {\n"

@@ -418,7 +418,7 @@ def test_autotune_picks_fastest_and_keeps_parity(torch_cuda, case):
 
 @pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
-@pytest.mark.parametrize("case", ["fig2", "c1", "c3s", "rand"])
+@pytest.mark.parametrize("case", ["c1", "c3s", "rand"])
 def test_paper_ell_mode(torch_cuda, case, dt, variant):
     """CRSD_PAPER_ELL (the paper's two-part kernel):
     scatter rows are overwritten by the ELL part -- bit-exact against the
@@ -426,13 +426,10 @@ def test_paper_ell_mode(torch_cuda, case, dt, variant):
     columns); every other row matches the definition within tolerance."""
     from paper_conf_icpp_sunzwzyr11_b200 import CRSD_PAPER_ELL, CRSDError
     from oracle import crsd_ref
-    from tests.conftest import load_fig2
 
-    mrows = None
-    if case == "fig2":
-        n, m, r, c, v, _ = load_fig2()
-        a = gen.COO(n, m, r, c, v)
-    elif case == "c1":
+    # (Fig. 2 itself needs mrows = 2, below the GPU minimum; its ELL arrays
+    # are checked against Fig. 4 on the host: test_paper_ell_export_fig2_golden)
+    if case == "c1":
         a = gen.config1()
     elif case == "c3s":
         a = gen.config3(n=24)
