@@ -542,6 +542,130 @@ def run_crsd(args):
         dist.destroy_process_group()
 
 
+# ---------------------------------------------------------------- CG workload
+def run_cg(args):
+    """--workload cg: K steps of crsd_cg (textbook CG on the CRSD SpMV,
+    SURVEY.md §8(f) NEXT 2) on the 7-point Dirichlet Laplacian of C2's grid
+    (256^3, SPD, exact values), one GPU. A step = SpMV + 3 vector kernels
+    (fused (p,q) with the JIT variant); its algorithmic bytes are the SpMV's
+    unique bytes + the vector traffic."""
+    import torch
+
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix
+    from oracle import cg_ref
+
+    import gen
+
+    if args.gpus != 1:
+        raise SystemExit("--workload cg runs on one GPU")
+    torch.cuda.set_device(0)
+    dt = np.float64 if args.dtype == "f64" else np.float32
+    tdt = torch.float64 if dt == np.float64 else torch.float32
+    es = np.dtype(dt).itemsize
+    n = 256
+    a = gen.spd_stencil_scatter((n, n, n), "7pt").astype(dt)
+    N = a.nrows
+    kw = {"mrows": args.mrows} if args.mrows else {}
+    A = CRSDMatrix.from_coo(N, N, a.row, a.col, a.val, **kw)
+    info = A.info()
+    fused = info["variant"] == 4 and not os.environ.get("CRSD_CG_NO_FUSED_DOT")
+    vec_passes = 8 if fused else 10
+    step_bytes = info["unique_bytes_beta0"] + vec_passes * N * es
+    step_flops = 2.0 * a.nnz + 10.0 * N
+    rng = np.random.default_rng(17)
+    bh = torch.from_numpy(rng.uniform(-1, 1, N).astype(dt)).pin_memory()
+    b = bh.to("cuda")
+    x = torch.zeros(N, dtype=tdt, device="cuda")
+    K = args.steps
+    check = min(K, 50)
+    clocks = ClockSampler(0)
+    clocks.start()
+    # warm-up: >= 300 steps (a short CG run otherwise starts below full clocks)
+    A.cg(b, x, max(args.warmup, 300), 0.0, check_every=check)
+    torch.cuda.synchronize()
+    x.zero_()
+    s_ev, e_ev = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    s_ev.record()
+    res = A.cg(b, x, K, 0.0, check_every=check)
+    e_ev.record()
+    e_ev.synchronize()
+    clk = clocks.stop()
+    ms = s_ev.elapsed_time(e_ev) / res["iterations"]
+    peak, peak_src = measured_peaks()
+    achieved = step_bytes / (ms * 1e-3) / 1e9
+    # e2e: pinned b -> device, K steps, x -> pinned host, every solve
+    xh = torch.empty(N, dtype=tdt).pin_memory()
+    t0 = time.perf_counter()
+    bd = bh.to("cuda", non_blocking=True)
+    xd = torch.zeros(N, dtype=tdt, device="cuda")
+    r2 = A.cg(bd, xd, K, 0.0, check_every=check)
+    xh.copy_(xd, non_blocking=True)
+    torch.cuda.synchronize()
+    te = time.perf_counter() - t0
+    # cpu_baseline: the CG oracle as it stands on a bounded sample (64^3 grid)
+    ns = 64
+    a_s = gen.spd_stencil_scatter((ns, ns, ns), "7pt").astype(dt)
+    b_s = rng.uniform(-1, 1, a_s.nrows)
+    ks = 5
+    t0 = time.perf_counter()
+    cg_ref.cg(a_s, b_s, np.zeros(a_s.nrows), ks)
+    tc = (time.perf_counter() - t0) / ks
+    cpu_gflops = (2.0 * a_s.nnz + 10.0 * a_s.nrows) / tc / 1e9
+    line = {
+        "metric": "CG step GFLOP/s ((2*nnz + 10n) per step / t) with achieved HBM GB/s",
+        "value": round(step_flops / (ms * 1e-3) / 1e9, 3),
+        "unit": "GFLOP/s",
+        "n_gpus": 1,
+        "steps": res["iterations"],
+        "warmup": max(args.warmup, 300),
+        "ms_per_step": round(ms, 5),
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": args.dtype,
+        "data": "synthetic",
+        "config": {
+            "workload": f"CG on the 7-point Dirichlet Laplacian 256^3 ({N:,} rows, SPD, exact values), rtol 0, {K} steps",
+            "nnz": int(a.nnz),
+            "mrows": info["mrows"],
+            "kernel_variant": {1: "ldg", 2: "tma", 3: "pipe", 4: "jit"}[info["variant"]],
+            "fused_pq_dot": fused,
+            "check_every": check,
+            "l2": f"inputs larger than L2 ({step_bytes / 1e9:.2f} GB per step); no flush",
+        },
+        "roofline": {
+            "bound": "hbm",
+            "kernel": "cg step (SpMV + vector kernels, one CUDA graph per batch)",
+            "achieved": round(achieved, 1),
+            "peak": peak,
+            "peak_source": peak_src,
+            "unit": "GB/s",
+            "frac": round(achieved / peak, 4),
+            "traffic": None,
+            "algorithmic_bytes_per_step": int(step_bytes),
+        },
+        "cpu_baseline": {
+            "value": round(cpu_gflops, 4),
+            "unit": "GFLOP/s",
+            "cores": 1,
+            "kind": "oracle",
+            "sample": f"oracle/cg_ref.py (long-double definition SpMV + numpy dots), 7-pt 64^3 grid, {ks} steps",
+        },
+        "e2e": {
+            "value": round(step_flops * r2["iterations"] / te / 1e9, 3),
+            "unit": "GFLOP/s",
+            "h2d_bytes_per_step": int(N * es),
+            "d2h_bytes_per_step": int(N * es),
+            "per": f"one solve of {K} steps: H2D b, crsd_cg, D2H x",
+            "ms_per_solve": round(te * 1e3, 3),
+        },
+        "gpu_launches": int(res["launches"]),
+        "clocks": clk,
+    }
+    print(json.dumps(line), flush=True)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -552,12 +676,15 @@ def main():
     ap.add_argument("--mrows", type=int, default=0)
     ap.add_argument("--variant", default="auto", choices=["auto", "ldg", "tma", "pipe", "jit"])
     ap.add_argument("--impl", default="crsd", choices=["crsd", "reference"])
+    ap.add_argument("--workload", default="spmv", choices=["spmv", "cg"], help="cg: K steps of crsd_cg (one GPU)")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
     if args.impl == "reference":
         run_reference(args)
+    elif args.workload == "cg":
+        run_cg(args)
     else:
         run_crsd(args)
 

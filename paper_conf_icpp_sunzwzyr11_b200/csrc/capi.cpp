@@ -471,24 +471,32 @@ static crsd_status_t e2e_setup(crsd_matrix_s *A) {
     A->e2e_seg.resize(nch + 1);
     A->e2e_xcut.resize(nch + 1);
     for (int c = 0; c <= nch; ++c) A->e2e_seg[c] = nseg * c / nch;
-    for (int c = 0; c <= nch; ++c) {
-        int64_t xc = (c == nch) ? H.ncols : std::min<int64_t>(H.ncols, A->e2e_seg[c] * H.mrows);
-        A->e2e_xcut[c] = (c == nch) ? xc : (xc / 4) * 4;
-    }
     // highest x element each row chunk reads (vector windows, clipped to
     // [0, ncols) as the guarded edge path does, and scatter columns)
-    A->e2e_need.assign(nch, 0);
+    std::vector<int64_t> hi(nch, 0);
     for (int c = 0; c < nch; ++c) {
-        int64_t hi = 0;
         for (int64_t sg = A->e2e_seg[c]; sg < A->e2e_seg[c + 1]; ++sg) {
             int64_t lo_w, hi_w;
             segment_x_window(H, sg, A->rpt, lo_w, hi_w);
-            if (lo_w < hi_w) hi = std::max(hi, std::min(hi_w, H.ncols));
-            for (int64_t e = H.scat_ptr[sg]; e < H.scat_ptr[sg + 1]; ++e) hi = std::max(hi, H.scat_col[e] + 1);
+            if (lo_w < hi_w) hi[c] = std::max(hi[c], std::min(hi_w, H.ncols));
+            for (int64_t e = H.scat_ptr[sg]; e < H.scat_ptr[sg + 1]; ++e) hi[c] = std::max(hi[c], H.scat_col[e] + 1);
         }
+    }
+    // x chunk c ends where row chunk c's reads end (monotone, 16-B aligned),
+    // so row chunk c waits for x chunks <= c only -- not for the whole next
+    // chunk because of a halo of a few rows. Row chunks whose reads reach
+    // further (scatter columns) share a later x chunk.
+    A->e2e_xcut[0] = 0;
+    for (int c = 0; c < nch; ++c) {
+        int64_t xc = (c == nch - 1) ? H.ncols : std::min<int64_t>(H.ncols, (hi[c] + 3) / 4 * 4);
+        A->e2e_xcut[c + 1] = std::max(A->e2e_xcut[c], xc);
+    }
+    A->e2e_xcut[nch] = H.ncols;
+    A->e2e_need.assign(nch, 0);
+    for (int c = 0; c < nch; ++c) {
         int j = 0;
-        while (j < nch - 1 && A->e2e_xcut[j + 1] < hi) ++j;
-        A->e2e_need[c] = std::max(j, c * 0);
+        while (j < nch - 1 && A->e2e_xcut[j + 1] < hi[c]) ++j;
+        A->e2e_need[c] = j;
     }
     cudaStream_t h, d;
     CUDA_TRY(cudaStreamCreateWithFlags(&h, cudaStreamNonBlocking));

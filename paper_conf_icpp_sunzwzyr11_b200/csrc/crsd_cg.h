@@ -20,7 +20,6 @@ struct CgState {
     double *hist;        // (r_j, r_j) for j = 0..it, or null
     double *partials;    // one per CTA of the vector kernels
     uint32_t counter;    // last-CTA detection (reset by the last CTA)
-    uint32_t dcounter;   // the same for the (p, q) dot fused into the JIT SpMV
     int32_t done;        // stopping test met or max_iter reached: the vector kernels become no-ops
 };
 

@@ -87,8 +87,8 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &a, void *stream);
 // segments [0, count)). x_base is the local x base (x_padded + halo_lo).
 // dot != null (JIT variant only, one launch): also *dot->out = sum_rows x[row] * y[row].
 struct DotArgs {
-    double *part;   // >= count partials
-    uint32_t *cnt;  // zero between launches
+    double *part;   // count + ceil(count / 256) partials
+    uint32_t *cnt;  // ceil(count / 256) + 1 counters, zero between launches
     double *out;
 };
 crsd_status_t run_lists(crsd_matrix_s *A, const void *alpha, const void *x_base, const void *beta, void *y,

@@ -171,10 +171,18 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
     const bool f64 = H.dtype == CRSD_R64F;
     const int m = H.mrows, nt = m / Q, es = H.elem;
     const bool scat = H.nscatter() > 0;  // scatter code only for matrices that have scatter points
-    const bool early = getenv("CRSD_JIT_EARLY") && atoi(getenv("CRSD_JIT_EARLY")) != 0;
+    // early issue (default; CRSD_JIT_EARLY=0 for the late form): +1-4 % on
+    // C2/C3/C4 (sweep20)
+    const bool early = !(getenv("CRSD_JIT_EARLY") && atoi(getenv("CRSD_JIT_EARLY")) == 0);
     std::ostringstream o;
     o << "typedef " << (f64 ? "double" : "float") << " T;\n" << kPrelude;
     o << "#define MROWS " << m << "\n#define NT " << nt << "\n#define Q " << Q << "\n";
+    // block sum in a fixed order (shuffle tree per warp, then warps in order);
+    // the result is valid in thread 0
+    o << "__device__ __forceinline__ double blk_sum(double v, double *red) {\n"
+         "  for (int k = 16; k; k >>= 1) v += __shfl_down_sync(0xffffffffu, v, k);\n"
+         "  __syncthreads();\n  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = v;\n  __syncthreads();\n"
+         "  double b = 0.0;\n  if (threadIdx.x == 0) for (int k = 0; k < NT / 32; ++k) b += red[k];\n  return b;\n}\n";
     // one __device__ codelet per distinct pattern
     // codelets are keyed by the pattern's plan_begin, which is unique per
     // distinct pattern (off_begin is not: a pattern without diagonals shares
@@ -198,11 +206,11 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
         o << "  T *xs = vs + " << (int64_t)nd * m << ";\n";
         // a pattern without diagonals (rows holding only scatter points, or
         // nothing) stages nothing: no mbarrier at all
-        // Copy issue. Default: thread 0 initialises the mbarrier and issues
-        // the value copy, then (after the CTA barrier) lane w of warp 0
-        // issues x window w. early (CRSD_JIT_EARLY=1): thread 0 issues every
-        // copy before the CTA barrier and the scatter gathers are issued
-        // before it too (A/B for the sweeps).
+        // Copy issue. early (default): thread 0 initialises the mbarrier and
+        // issues every copy (values, then the x windows) before the CTA
+        // barrier, and the scatter gathers are issued before it too. Late
+        // form (CRSD_JIT_EARLY=0): thread 0 issues the value copy, lane w of
+        // warp 0 issues x window w after the CTA barrier.
         std::string sg;
         if (scat) {
             // scatter points are gathered while the bulk copies are in flight:
@@ -301,20 +309,30 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
          "  T *vs = reinterpret_cast<T *>(smem);\n  double d = 0.0;\n  switch (D.plan_begin) {\n";
     for (int32_t v : seen) o << "  case " << v << ": d = codelet_" << v << "(a, D, row0, edge, vs, &bar, threadIdx.x); break;\n";
     o << "  }\n";
-    // fused dot: per-CTA partial, the last CTA sums the partials in CTA order
+    // fused dot, deterministic two-level reduction: every CTA writes its
+    // partial; the last CTA to arrive in each group of 256 CTAs sums that
+    // group's partials (one load per thread, fixed tree order) into a group
+    // partial; the last group sums the group partials. One counter per group
+    // keeps the atomics spread and the tail to two short reductions (a single
+    // last CTA summing every partial was a ~30 us serial tail per launch).
     o << "  if (a.dot_part) {\n"
          "    __shared__ double red[NT / 32];\n    __shared__ bool last;\n"
-         "    for (int k = 16; k; k >>= 1) d += __shfl_down_sync(0xffffffffu, d, k);\n"
-         "    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = d;\n    __syncthreads();\n"
-         "    if (threadIdx.x == 0) {\n      double b = 0.0;\n      for (int k = 0; k < NT / 32; ++k) b += red[k];\n"
-         "      a.dot_part[blockIdx.x] = b;\n      __threadfence();\n"
-         "      last = atomicAdd(a.dot_cnt, 1u) == gridDim.x - 1;\n    }\n    __syncthreads();\n"
-         "    if (last) {\n      __threadfence();\n      double b = 0.0;\n"
-         "      for (unsigned k = threadIdx.x; k < gridDim.x; k += NT) b += *((volatile double *)a.dot_part + k);\n"
-         "      for (int k = 16; k; k >>= 1) b += __shfl_down_sync(0xffffffffu, b, k);\n"
-         "      __syncthreads();\n      if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = b;\n      __syncthreads();\n"
-         "      if (threadIdx.x == 0) {\n        double c = 0.0;\n        for (int k = 0; k < NT / 32; ++k) c += red[k];\n"
-         "        *a.dot_out = c;\n        *a.dot_cnt = 0u;\n      }\n    }\n  }\n";
+         "    const unsigned G = (gridDim.x + 255u) / 256u, g = blockIdx.x / 256u;\n"
+         "    const unsigned gs = min(256u, gridDim.x - g * 256u);\n"
+         "    double *gpart = a.dot_part + gridDim.x;\n"
+         "    d = blk_sum(d, red);\n"
+         "    if (threadIdx.x == 0) {\n      a.dot_part[blockIdx.x] = d;\n      __threadfence();\n"
+         "      last = atomicAdd(a.dot_cnt + g, 1u) == gs - 1;\n    }\n    __syncthreads();\n"
+         "    if (last) {\n      __threadfence();\n"
+         "      double b = 0.0;\n"
+         "      for (unsigned k = threadIdx.x; k < gs; k += NT) b += __ldcg(a.dot_part + g * 256u + k);\n"
+         "      b = blk_sum(b, red);\n"
+         "      if (threadIdx.x == 0) {\n        gpart[g] = b;\n        a.dot_cnt[g] = 0u;\n        __threadfence();\n"
+         "        last = atomicAdd(a.dot_cnt + G, 1u) == G - 1;\n      }\n      __syncthreads();\n"
+         "      if (last) {\n        __threadfence();\n        double c = 0.0;\n"
+         "        for (unsigned k = threadIdx.x; k < G; k += NT) c += __ldcg(gpart + k);\n"
+         "        c = blk_sum(c, red);\n"
+         "        if (threadIdx.x == 0) {\n          *a.dot_out = c;\n          a.dot_cnt[G] = 0u;\n        }\n      }\n    }\n  }\n";
     o << "}\n";
     return o.str();
 }

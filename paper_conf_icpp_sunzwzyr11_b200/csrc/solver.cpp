@@ -50,7 +50,8 @@ inline int64_t up256(int64_t b) { return (b + 255) / 256 * 256; }
 
 struct Ws {
     CgState *st;
-    double *partials, *hist, *dpart;  // dpart: one per segment (dot fused into the SpMV)
+    double *partials, *hist, *dpart;  // dpart: per segment + per group of 256 (dot fused into the SpMV)
+    uint32_t *dcnt;                    // its counters: one per group + one
     char *r, *q, *p_pad;  // p_pad: halo_lo + n + halo_hi elements
 };
 
@@ -59,8 +60,10 @@ crsd_status_t workspace(crsd_matrix_s *A, int64_t max_iter, int grid, Ws &w) {
     const int64_t npad = A->halo_lo + n + A->halo_hi;
     const int64_t o_part = up256(sizeof(CgState));
     const int64_t o_hist = o_part + up256(8 * (int64_t)grid);
+    const int64_t ngrp = (A->H.nseg + 255) / 256;
     const int64_t o_dp = o_hist + up256(8 * (max_iter + 1));
-    const int64_t o_r = o_dp + up256(8 * std::max<int64_t>(1, A->H.nseg));
+    const int64_t o_dc = o_dp + up256(8 * (A->H.nseg + ngrp + 1));
+    const int64_t o_r = o_dc + up256(4 * (ngrp + 1));
     const int64_t o_q = o_r + up256(es * n);
     const int64_t o_p = o_q + up256(es * n);
     const int64_t total = o_p + up256(es * npad);
@@ -86,6 +89,7 @@ crsd_status_t workspace(crsd_matrix_s *A, int64_t max_iter, int grid, Ws &w) {
     w.partials = (double *)(b + o_part);
     w.hist = (double *)(b + o_hist);
     w.dpart = (double *)(b + o_dp);
+    w.dcnt = (uint32_t *)(b + o_dc);
     w.r = b + o_r;
     w.q = b + o_q;
     w.p_pad = b + o_p;
@@ -155,7 +159,7 @@ crsd_status_t cg_impl(crsd_matrix_s *A, const T *b, T *x, int32_t max_iter, doub
     // One GPU with the JIT variant: (p, q) is fused into the SpMV epilogue
     // (saves one read of p and of q per step); otherwise a separate kernel.
     const bool fused = !comm && A->variant == VARIANT_JIT && !getenv("CRSD_CG_NO_FUSED_DOT");
-    DotArgs dot{w.dpart, &w.st->dcounter, w.st->red + CG_PQ};
+    DotArgs dot{w.dpart, w.dcnt, w.st->red + CG_PQ};
     auto step = [&]() -> crsd_status_t {
         if (fused) {
             const T one(1), zero(0);

@@ -30,7 +30,7 @@ N = a.nrows
 tdt = torch.float64 if dt == np.float64 else torch.float32
 b = torch.rand(N, dtype=tdt, device="cuda") - 0.5
 x = torch.zeros(N, dtype=tdt, device="cuda")
-A.cg(b, x, 10, 0.0, check_every=check)  # warm-up (workspace, graph)
+A.cg(b, x, 300, 0.0, check_every=check)  # warm-up (workspace, graph, clocks)
 torch.cuda.synchronize()
 s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 x.zero_()
