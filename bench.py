@@ -568,7 +568,7 @@ def run_cg(args):
     kw = {"mrows": args.mrows} if args.mrows else {}
     A = CRSDMatrix.from_coo(N, N, a.row, a.col, a.val, **kw)
     info = A.info()
-    fused = info["variant"] == 4 and not os.environ.get("CRSD_CG_NO_FUSED_DOT")
+    fused = info["variant"] == 4 and os.environ.get("CRSD_CG_FUSED_DOT", "0") != "0"
     vec_passes = 8 if fused else 10
     step_bytes = info["unique_bytes_beta0"] + vec_passes * N * es
     step_flops = 2.0 * a.nnz + 10.0 * N

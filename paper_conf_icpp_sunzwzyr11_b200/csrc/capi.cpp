@@ -482,13 +482,17 @@ static crsd_status_t e2e_setup(crsd_matrix_s *A) {
             for (int64_t e = H.scat_ptr[sg]; e < H.scat_ptr[sg + 1]; ++e) hi[c] = std::max(hi[c], H.scat_col[e] + 1);
         }
     }
-    // x chunk c ends where row chunk c's reads end (monotone, 16-B aligned),
-    // so row chunk c waits for x chunks <= c only -- not for the whole next
-    // chunk because of a halo of a few rows. Row chunks whose reads reach
-    // further (scatter columns) share a later x chunk.
+    // x chunks are aligned with the row chunks, so row chunk c usually waits
+    // for x chunk c+1 (its far diagonals reach a few rows into it). Cutting x
+    // where each row chunk's reads end instead (CRSD_E2E_CUT=needs) lets
+    // y copies start one chunk earlier but measured slower: the earlier D2H
+    // overlaps more of the H2D stream and slows it (C2 f64, 12-16 chunks:
+    // 3.38 vs 3.56-3.59 ms; profiles/r01_e2e_cut_ab.txt).
+    const bool cut_rows = !(getenv("CRSD_E2E_CUT") && std::string(getenv("CRSD_E2E_CUT")) == "needs");
     A->e2e_xcut[0] = 0;
     for (int c = 0; c < nch; ++c) {
         int64_t xc = (c == nch - 1) ? H.ncols : std::min<int64_t>(H.ncols, (hi[c] + 3) / 4 * 4);
+        if (cut_rows) xc = std::min<int64_t>(H.ncols, A->e2e_seg[c + 1] * H.mrows) / 4 * 4;
         A->e2e_xcut[c + 1] = std::max(A->e2e_xcut[c], xc);
     }
     A->e2e_xcut[nch] = H.ncols;

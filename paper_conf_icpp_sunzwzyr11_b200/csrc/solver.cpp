@@ -158,7 +158,12 @@ crsd_status_t cg_impl(crsd_matrix_s *A, const T *b, T *x, int32_t max_iter, doub
 
     // One GPU with the JIT variant: (p, q) is fused into the SpMV epilogue
     // (saves one read of p and of q per step); otherwise a separate kernel.
-    const bool fused = !comm && A->variant == VARIANT_JIT && !getenv("CRSD_CG_NO_FUSED_DOT");
+    // Off by default: the reduction epilogue lengthens every SpMV CTA's life
+    // (fewer bytes in flight), which costs more than the two vector passes it
+    // saves (C2 f64 0.417 vs 0.407 ms/step, f32 equal; profiles/r01_cg_ab.jsonl).
+    // CRSD_CG_FUSED_DOT=1 enables it.
+    const bool fused = !comm && A->variant == VARIANT_JIT && getenv("CRSD_CG_FUSED_DOT") &&
+                       atoi(getenv("CRSD_CG_FUSED_DOT")) != 0;
     DotArgs dot{w.dpart, w.dcnt, w.st->red + CG_PQ};
     auto step = [&]() -> crsd_status_t {
         if (fused) {

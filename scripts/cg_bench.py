@@ -41,7 +41,7 @@ e.synchronize()
 ms = s.elapsed_time(e)
 es = np.dtype(dt).itemsize
 inf = A.info()
-fused = inf["variant"] == 4 and not os.environ.get("CRSD_CG_NO_FUSED_DOT")
+fused = inf["variant"] == 4 and os.environ.get("CRSD_CG_FUSED_DOT", "0") != "0"
 step_bytes = inf["unique_bytes_beta0"] + (8 if fused else 10) * N * es
 per = ms / res["iterations"]
 print(json.dumps({"workload": f"CG 7-pt {n}^3 {np.dtype(dt).name}", "variant": inf["variant"], "steps": res["iterations"],

@@ -449,3 +449,21 @@ def test_paper_ell_mode(torch_cuda, case, dt, variant):
     assert coo.parity_error(y, yref, scale) <= TOL[dt]
     with pytest.raises(CRSDError, match="UNSUPPORTED"):
         _run(torch_cuda, A, x, 1.0, 0.5, np.zeros(a.nrows, dt), a.nrows)
+
+
+@pytest.mark.slow
+@SLOW
+@pytest.mark.parametrize("case", ["c2", "c3"])
+def test_full_size_device_roundtrip(torch_cuda, case):
+    """BASELINE configs 2 and 3 at full size: the CRSD structure as it sits in
+    HBM (crsd_export reads the device arrays back; the host copy of the
+    values is dropped after upload) decodes to the canonical COO bit for bit
+    (north star: "CRSD construction must round-trip bit-exact to COO")."""
+    from oracle import decode
+
+    a = cached(case, gen.config2 if case == "c2" else gen.config3)
+    A = _mat(a)
+    P = A.export()
+    assert decode.roundtrip_equal(P, a.nrows, a.ncols, a.row, a.col, a.val)
+    inf = A.info()
+    assert inf["nnz"] == a.nnz
