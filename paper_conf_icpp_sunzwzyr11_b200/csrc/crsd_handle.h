@@ -22,6 +22,8 @@ struct crsd_matrix_s {
     std::string jit_source;
     void *jit_module = nullptr;
     void *jit_function = nullptr;
+    void *jitp_function = nullptr;  // persistent double-buffered form (crsd_jitp), or null
+    bool jit_persist = false;       // launch the persistent form by default
     int64_t tma_smem = 0;
     std::vector<int32_t> plan;
     int32_t last_launches = 0;

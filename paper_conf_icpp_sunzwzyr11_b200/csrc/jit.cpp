@@ -155,6 +155,10 @@ __device__ __forceinline__ void bar_wait(u64 *b) {
   u32 done = 0;
   while (!done) asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0; selp.u32 %0, 1, 0, p; }"
                              : "=r"(done) : "r"(su32(b)) : "memory"); }
+__device__ __forceinline__ void bar_wait_ph(u64 *b, u32 ph) {
+  u32 done = 0;
+  while (!done) asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+                             : "=r"(done) : "r"(su32(b)), "r"(ph) : "memory"); }
 __device__ __forceinline__ u64 pol_first() { u64 p; asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p)); return p; }
 __device__ __forceinline__ u64 pol_normal() { u64 p; asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p)); return p; }
 __device__ __forceinline__ void g2s(void *dst, const void *src, u32 bytes, u64 *b, u64 pol) {
@@ -337,6 +341,121 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
     return o.str();
 }
 
+// Persistent, double-buffered form of the codelets (kernel crsd_jitp): a
+// CTA per SM slot loops over its segments (w, w + G, ...) with two staging
+// buffers. Warp 0 refills a buffer as soon as every thread is done with it:
+// lane 0 copies the segment descriptor into the buffer's header and issues
+// the bulk copies (values, x windows) with every pattern quantity a literal;
+// the 32 lanes read the segment's first 32 scatter records and gather their
+// x[col] into the header. The segment after next is therefore in flight
+// while the current one computes, and no CTA start-up (launch, descriptor
+// load, scatter gather) sits between a buffer's reuse and its next copy.
+static void generate_persistent(const crsd_matrix_s *A, int Q, std::ostringstream &o) {
+    const HostCRSD &H = A->H;
+    const int m = H.mrows, es = H.elem;
+    const bool scat = H.nscatter() > 0;
+    o << "\n// ---- persistent double-buffered form ----\n"
+         "struct __align__(16) StageHdr { SegDesc D; i64 row0; int nsg; int pad; int own[32]; T v[32]; T xv[32]; };\n"
+         "#define HDR ((int)((sizeof(StageHdr) + 127) / 128 * 128))\n";
+    std::vector<int32_t> seen;
+    std::ostringstream issue_sw, comp_sw;
+    for (const Instance &I : H.inst) {
+        const int32_t key = A->segdesc[I.first_seg].plan_begin;
+        bool dup = false;
+        for (int32_t v : seen) dup |= (v == key);
+        if (dup) continue;
+        seen.push_back(key);
+        const int32_t *pl = A->plan.data() + key;
+        const int nd = (int)H.ndias(I.pattern), nwin = pl[0];
+        const int64_t *offs = H.pat_offsets.data() + H.pat_ptr[I.pattern];
+        int64_t xb = 0;
+        for (int w = 0; w < nwin; ++w) xb += pl[3 + 2 * w];
+        // issue (lane 0 of warp 0)
+        o << "__device__ __forceinline__ void pissue_" << key
+          << "(const Args &a, const SegDesc &D, i64 row0, bool edge, T *vs, u64 *bar) {\n";
+        o << "  bar_expect(bar, " << (int64_t)nd * m * es << "u + (edge ? 0u : " << xb * es << "u));\n";
+        if (nd) o << "  g2s(vs, a.vals + D.val_base, " << (int64_t)nd * m * es << "u, bar, pol_first());\n";
+        if (nwin) {
+            o << "  if (!edge) {\n    T *xs = vs + " << (int64_t)nd * m << ";\n    const u64 pn = pol_normal();\n";
+            int64_t base = 0;
+            for (int w = 0; w < nwin; ++w) {
+                o << "    g2s(xs + " << base << ", a.x + row0 + (" << pl[2 + 2 * w] << "), " << (int64_t)pl[3 + 2 * w] * es
+                  << "u, bar, pn);\n";
+                base += pl[3 + 2 * w];
+            }
+            o << "  }\n";
+        }
+        o << "}\n";
+        // compute (all threads)
+        const int32_t *xoff = pl + 2 + 2 * nwin;
+        o << "__device__ __forceinline__ void pcomp_" << key
+          << "(const Args &a, const StageHdr &S, bool edge, const T *vs, u64 *bar, u32 ph, int t) {\n";
+        o << "  const T *xs = vs + " << (int64_t)nd * m << ";\n  const i64 row0 = S.row0;\n  (void)xs;\n";
+        o << "  T acc[Q];\n#pragma unroll\n  for (int q = 0; q < Q; ++q) acc[q] = T(0);\n";
+        o << "  bar_wait_ph(bar, ph);\n";
+        o << "  if (!edge) {\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n      const int r = t + q * NT;\n";
+        for (int d = 0; d < nd; ++d)
+            o << "      acc[q] = fma(vs[" << (int64_t)d * m << " + r], xs[" << xoff[d] << " + r], acc[q]);\n";
+        o << "    }\n  } else {\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n      const i64 r = row0 + t + q * NT;\n";
+        for (int d = 0; d < nd; ++d)
+            o << "      { const i64 i = r + (" << offs[d] << "); acc[q] = fma(vs[" << (int64_t)d * m
+              << " + t + q * NT], (i >= a.x_lo && i < a.x_hi) ? __ldg(a.x + i) : T(0), acc[q]); }\n";
+        o << "    }\n  }\n";
+        if (scat)
+            o << "  if (S.D.nscat > 0) {\n"
+                 "    for (int e = 0; e < S.nsg; ++e) {\n"
+                 "      const int own = S.own[e];\n"
+                 "      if (own / Q != t) continue;\n"
+                 "#pragma unroll\n      for (int q = 0; q < Q; ++q) if (own == t * Q + q) acc[q] = fma(S.v[e], S.xv[e], acc[q]);\n"
+                 "    }\n"
+                 "    for (int e = 32; e < S.D.nscat; ++e) {\n"
+                 "      const int rr = __ldg(a.scat_row + S.D.scat_begin + e);\n"
+                 "      if (rr % NT != t) continue;\n"
+                 "      const T v = __ldg(a.scat_val + S.D.scat_begin + e), xv = __ldg(a.x + __ldg(a.scat_col + S.D.scat_begin + e));\n"
+                 "#pragma unroll\n      for (int q = 0; q < Q; ++q) if (rr / NT == q) acc[q] = fma(v, xv, acc[q]);\n"
+                 "    }\n  }\n";
+        o << "#pragma unroll\n  for (int q = 0; q < Q; ++q) {\n    const i64 r = row0 + t + q * NT;\n"
+             "    if (!edge || r < a.nrows) { T *yp = a.y + r; __stcs(yp, (a.beta != T(0)) ? fma(a.alpha, acc[q], a.beta * *yp) : a.alpha * acc[q]); }\n"
+             "  }\n}\n";
+        issue_sw << "      case " << key << ": pissue_" << key << "(a, D, row0, edge, vs, bar); break;\n";
+        comp_sw << "    case " << key << ": pcomp_" << key << "(a, S, edge, vk, bar + k, ph, t); break;\n";
+    }
+    // stage fill by warp 0 (lane = t < 32)
+    o << "__device__ __forceinline__ void pfill(const Args &a, i64 w, StageHdr *S, T *vs, u64 *bar, int lane) {\n"
+         "  const i64 s = a.seg_list ? (i64)__ldg(a.seg_list + w) : a.seg_begin + w;\n"
+         "  const SegDesc D = a.segs[s];\n  const i64 row0 = s * MROWS;\n  const bool edge = (D.flags & 1) != 0;\n"
+         "  if (lane == 0) {\n    S->D = D;\n    S->row0 = row0;\n    S->nsg = D.nscat < 32 ? D.nscat : 32;\n"
+         "    switch (D.plan_begin) {\n" << issue_sw.str() << "    }\n  }\n";
+    if (scat)
+        o << "  if (D.nscat > 0 && lane < D.nscat) {\n"
+             "    const ScatRec R = a.scat_rec[D.scat_begin + lane];\n"
+             "    S->own[lane] = (R.row % NT) * Q + R.row / NT;\n"
+             "    S->v[lane] = *reinterpret_cast<const T *>(&R.val);\n"
+             "    S->xv[lane] = __ldg(a.x + R.col);\n  }\n";
+    o << "}\n";
+    o << "extern \"C\" __global__ void __launch_bounds__(NT) crsd_jitp(const Args a, int stage_bytes) {\n"
+         "  extern __shared__ __align__(128) unsigned char smem[];\n  __shared__ u64 bar[2];\n"
+         "  const int t = threadIdx.x;\n"
+         "  if (t == 0) { bar_init(&bar[0]); bar_init(&bar[1]); }\n  __syncthreads();\n"
+         "  const i64 G = gridDim.x;\n"
+         "  if (t < 32)\n    for (int k = 0; k < 2; ++k) {\n      const i64 w = blockIdx.x + k * G;\n"
+         "      unsigned char *b = smem + k * stage_bytes;\n"
+         "      if (w < a.seg_count) pfill(a, w, reinterpret_cast<StageHdr *>(b), reinterpret_cast<T *>(b + HDR), bar + k, t);\n    }\n"
+         "  __syncthreads();\n"
+         "  u32 phs = 0u;  // bit k: phase of buffer k\n  int k = 0;\n"
+         "  for (i64 w = blockIdx.x; w < a.seg_count; w += G) {\n"
+         "    unsigned char *b = smem + k * stage_bytes;\n"
+         "    const StageHdr &S = *reinterpret_cast<const StageHdr *>(b);\n"
+         "    const T *vk = reinterpret_cast<const T *>(b + HDR);\n"
+         "    const u32 ph = (phs >> k) & 1u;\n"
+         "    const bool edge = (S.D.flags & 1) != 0;\n"
+         "    switch (S.D.plan_begin) {\n" << comp_sw.str() << "    }\n"
+         "    phs ^= 1u << k;\n    __syncthreads();\n"
+         "    if (t < 32 && w + 2 * G < a.seg_count)\n"
+         "      pfill(a, w + 2 * G, reinterpret_cast<StageHdr *>(b), reinterpret_cast<T *>(b + HDR), bar + k, t);\n"
+         "    k ^= 1;\n  }\n}\n";
+}
+
 // rows per thread of the generated kernel: <= 256 threads per CTA
 static int jit_q(const crsd_matrix_s *A) {
     int q = 1;
@@ -344,7 +463,18 @@ static int jit_q(const crsd_matrix_s *A) {
     return q;
 }
 
-std::string jit_generate(const crsd_matrix_s *A) { return generate(A, jit_q(A)); }
+// staging buffer of the persistent kernel: header + the largest staging
+static int64_t jitp_stage_bytes(const crsd_matrix_s *A) {
+    const int64_t hdr = (32 + 8 + 8 + 4 * 32 + 2 * 32 * (int64_t)A->H.elem + 127) / 128 * 128;
+    return (hdr + A->smem_bytes + 127) / 128 * 128;
+}
+
+std::string jit_generate(const crsd_matrix_s *A) {
+    std::string src = generate(A, jit_q(A));
+    std::ostringstream o;
+    generate_persistent(A, jit_q(A), o);
+    return src + o.str();
+}
 
 crsd_status_t jit_build(crsd_matrix_s *A) {
     NvrtcApi &nv = nvrtc();
@@ -353,8 +483,7 @@ crsd_status_t jit_build(crsd_matrix_s *A) {
     if (!dr.ok) return fail(CRSD_ERR_UNSUPPORTED, "JIT variant: driver entry point " + dr.err);
     if (A->smem_bytes > 200 * 1024) return fail(CRSD_ERR_UNSUPPORTED, "JIT variant: a segment's staging exceeds 200 KB");
     if (A->H.npat() > 256) return fail(CRSD_ERR_UNSUPPORTED, "JIT variant: more than 256 distinct patterns");
-    const int Q = jit_q(A);
-    A->jit_source = generate(A, Q);
+    A->jit_source = jit_generate(A);
     nvrtcProgram prog;
     if (nv.create(&prog, A->jit_source.c_str(), "crsd_jit.cu", 0, nullptr, nullptr) != NVRTC_SUCCESS)
         return fail(CRSD_ERR_CUDA, "nvrtcCreateProgram failed");
@@ -385,8 +514,19 @@ crsd_status_t jit_build(crsd_matrix_s *A) {
         dr.unload(mod);
         return fail(CRSD_ERR_CUDA, "cuFuncSetAttribute failed");
     }
+    // persistent form: usable when two staging buffers fit one CTA
+    CUfunction fnp = nullptr;
+    const int64_t pbytes = 2 * jitp_stage_bytes(A);
+    if (pbytes <= 220 * 1024 && dr.get_function(&fnp, mod, "crsd_jitp") == CUDA_SUCCESS) {
+        if (pbytes > 48 * 1024 &&
+            dr.set_attr(fnp, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)pbytes) != CUDA_SUCCESS)
+            fnp = nullptr;
+    } else {
+        fnp = nullptr;
+    }
     A->jit_module = mod;
     A->jit_function = fn;
+    A->jitp_function = fnp;
     return CRSD_OK;
 }
 
@@ -394,6 +534,7 @@ void jit_free(crsd_matrix_s *A) {
     if (A->jit_module && driver().ok) driver().unload((CUmodule)A->jit_module);
     A->jit_module = nullptr;
     A->jit_function = nullptr;
+    A->jitp_function = nullptr;
 }
 
 template <typename T>
@@ -419,10 +560,27 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
     j.dot_out = s.dot_out;
     j.alpha = s.alpha;
     j.beta = s.beta;
-    void *params[] = {&j};
     const unsigned nt = (unsigned)(A->H.mrows / jit_q(A));
-    CUresult r = driver().launch((CUfunction)A->jit_function, (unsigned)s.seg_count, 1, 1, nt, 1, 1,
-                                 (unsigned)A->smem_bytes, (CUstream)stream, params, nullptr);
+    CUresult r;
+    // persistent form (CRSD_JIT_MODE=persist, or A->jit_persist): no fused dot
+    const char *mode = getenv("CRSD_JIT_MODE");
+    const bool persist = A->jitp_function && !s.dot_part &&
+                         (mode ? std::string(mode) == "persist" : A->jit_persist);
+    if (persist) {
+        int stage = (int)jitp_stage_bytes(A);
+        const int64_t per_cta = 2 * (int64_t)stage + 1024 + 64;
+        int64_t per_sm = std::min<int64_t>(2048 / nt, (228 * 1024) / per_cta);
+        per_sm = std::min<int64_t>(per_sm, 65536 / (32 * (int64_t)nt));
+        if (per_sm < 1) per_sm = 1;
+        int64_t grid = std::min<int64_t>(s.seg_count, per_sm * A->sm_count);
+        void *pp[] = {&j, &stage};
+        r = driver().launch((CUfunction)A->jitp_function, (unsigned)grid, 1, 1, nt, 1, 1, (unsigned)(2 * stage),
+                            (CUstream)stream, pp, nullptr);
+    } else {
+        void *params[] = {&j};
+        r = driver().launch((CUfunction)A->jit_function, (unsigned)s.seg_count, 1, 1, nt, 1, 1,
+                            (unsigned)A->smem_bytes, (CUstream)stream, params, nullptr);
+    }
     return r == CUDA_SUCCESS ? 1 : -(int)cudaErrorLaunchFailure;
 }
 

@@ -49,15 +49,17 @@ def main():
         tdt = torch.float64 if dt == "f64" else torch.float32
         x = torch.rand(a.ncols, dtype=tdt, device="cuda")
         y = torch.empty(a.nrows, dtype=tdt, device="cuda")
-        runs = [("ldg", 1, None)] + [("tma", 2, t) for t in TMA] + [("pipe", 3, sh) for sh in SHAPES] + [("jit", 4, None), ("jit_late", 4, None)]
+        runs = [("ldg", 1, None)] + [("tma", 2, t) for t in TMA] + [("pipe", 3, sh) for sh in SHAPES] + [("jit", 4, None), ("jit_late", 4, None), ("jitp", 4, None)]
         only = os.environ.get("SWEEP_VARIANTS")
         if only:
             runs = [r for r in runs if r[0] in only.split(",")]
         for name, v, sh in runs:
-            for k in ("CRSD_PIPE_PERSM", "CRSD_PIPE_NX", "CRSD_PIPE_NS", "CRSD_TMA_Q", "CRSD_TMA_SPLIT", "CRSD_JIT_EARLY"):
+            for k in ("CRSD_PIPE_PERSM", "CRSD_PIPE_NX", "CRSD_PIPE_NS", "CRSD_TMA_Q", "CRSD_TMA_SPLIT", "CRSD_JIT_EARLY", "CRSD_JIT_MODE"):
                 os.environ.pop(k, None)
             if name == "jit_late":
                 os.environ["CRSD_JIT_EARLY"] = "0"
+            if name == "jitp":
+                os.environ["CRSD_JIT_MODE"] = "persist"
             if sh and name == "tma":
                 os.environ["CRSD_TMA_" + sh[0]] = str(sh[1])
             elif sh:

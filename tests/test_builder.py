@@ -214,7 +214,13 @@ def test_jit_codelets_compile_for_sm100a(case, dt, tmp_path):
     A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, host_only=True, variant=4)
     src = A.jit_source()
     P = A.export()
-    assert src.count("case ") == A.info()["npat"]
+    npat = A.info()["npat"]
+    # one-shot kernel: one codelet + case per pattern; persistent kernel: an
+    # issue and a compute function per pattern, each dispatched by a case
+    assert src.count("__device__ __forceinline__ double codelet_") == npat
+    assert src.count("__device__ __forceinline__ void pissue_") == npat
+    assert src.count("__device__ __forceinline__ void pcomp_") == npat
+    assert src.count("case ") == 3 * npat
     for offs in P["inst_offsets"]:
         assert "// pattern offsets: " + " ".join(str(o) for o in offs) in src
     f = tmp_path / "k.cu"

@@ -467,3 +467,26 @@ def test_full_size_device_roundtrip(torch_cuda, case):
     assert decode.roundtrip_equal(P, a.nrows, a.ncols, a.row, a.col, a.val)
     inf = A.info()
     assert inf["nnz"] == a.nnz
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+@pytest.mark.parametrize("case", ["c1", "c2s", "c3s", "c4s", "rand0", "rand1", "rand2", "dense_scatter"])
+def test_jit_persistent_parity(torch_cuda, case, dt, monkeypatch):
+    """The persistent double-buffered JIT form (crsd_jitp, CRSD_JIT_MODE=persist):
+    every CTA loops over several segments through two staging buffers."""
+    monkeypatch.setenv("CRSD_JIT_MODE", "persist")
+    if case == "c1":
+        a = gen.config1()
+    elif case == "c2s":
+        a = gen.config2(n=40)
+    elif case == "c3s":
+        a = gen.config3(n=36)
+    elif case == "c4s":
+        a = gen.config4(n=300_000)
+    elif case == "dense_scatter":
+        a = gen.random_diagonal(2048, 2048, 5, ndiag=3, n_scatter=3000, max_off=64)
+    else:
+        s = int(case[-1])
+        a = gen.random_diagonal(4000 + 97 * s, 3900, 30 + s, ndiag=12, max_off=900, p_break=0.02, max_break=400, n_scatter=200)
+    for alpha, beta in ((1.0, 0.0), (-0.75, 0.5)):
+        _parity(torch_cuda, a, dt, alpha, beta, seed=3, variant=4)
