@@ -369,6 +369,24 @@ crsd_status_t crsd_cg(crsd_matrix_t A, const void *b, void *x, int32_t max_iter,
 crsd_status_t crsd_autotune(crsd_matrix_t A, const void *x, void *y, int32_t reps, double *ms_out,
                             int32_t *chosen, void *stream);
 
+/*
+ * Build-time autotuning: the row-segment height
+ * `mrows` shapes the layout itself, so each candidate in
+ * mrows_cand[ncand] (HOST; NULL or ncand <= 0 => the default only) is built
+ * like crsd_create_from_coo with opts (NULL => defaults; one-GPU handles
+ * only), its variant chosen by crsd_autotune on scratch vectors (reps per
+ * variant), and the handle with the fastest SpMV is returned in *out; the
+ * others are destroyed as soon as they lose. Candidates the GPU path rejects
+ * (e.g. mrows not a multiple of 32*RPT) are skipped. ms_out HOST double[ncand]
+ * or NULL: best ms per launch of each candidate (-1 if skipped).
+ * Synchronous; peak memory = two candidates' device arrays. Errors as
+ * crsd_create_from_coo, plus UNSUPPORTED if no candidate is valid.
+ */
+crsd_status_t crsd_create_autotuned(int64_t nrows, int64_t ncols, int64_t nnz, const int64_t *row,
+                                    const int64_t *col, const void *val, crsd_dtype_t dtype,
+                                    const crsd_opts_t *opts, const int32_t *mrows_cand, int32_t ncand,
+                                    int32_t reps, crsd_matrix_t *out, double *ms_out);
+
 /* Number of kernel launches the last crsd_spmv / crsd_spmv_dist / crsd_cg call made. */
 crsd_status_t crsd_last_launch_count(crsd_matrix_t A, int32_t *count);
 

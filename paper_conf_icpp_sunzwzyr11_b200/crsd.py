@@ -54,6 +54,7 @@ EXPORTED = [
     "crsd_cg",
     "crsd_autotune",
     "crsd_export_paper_ell",
+    "crsd_create_autotuned",
 ]
 
 
@@ -152,6 +153,7 @@ def _load():
         "crsd_cg": ([P, P, P, I32, ctypes.c_double, I32, P, P, P, P], ctypes.c_int),
         "crsd_autotune": ([P, P, P, I32, P, P, P], ctypes.c_int),
         "crsd_export_paper_ell": ([P, P, P, P, P, P], ctypes.c_int),
+        "crsd_create_autotuned": ([I64, I64, I64, P, P, P, ctypes.c_int, P, P, I32, I32, P, P], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)
@@ -243,6 +245,29 @@ class CRSDMatrix:
             )
         )
         return cls(h.value, val.dtype)
+
+    @classmethod
+    def autotuned(cls, nrows, ncols, row, col, val, *, mrows_candidates=(0,), idle_max=-1, flags=0, device=-1, reps=20):
+        """crsd_create_autotuned: build each mrows candidate, autotune its kernel
+        variant, keep the fastest handle. Returns (matrix, {mrows: ms or None})."""
+        row = np.ascontiguousarray(row, dtype=np.int64)
+        col = np.ascontiguousarray(col, dtype=np.int64)
+        val = np.ascontiguousarray(val)
+        if val.dtype not in (np.float32, np.float64):
+            val = val.astype(np.float64)
+        o = Opts()
+        lib.crsd_opts_init(ctypes.byref(o))
+        o.idle_max, o.flags, o.device = idle_max, flags, device
+        cand = np.ascontiguousarray(mrows_candidates, dtype=np.int32)
+        ms = np.zeros(cand.shape[0], np.float64)
+        h = ctypes.c_void_p()
+        _check(
+            lib.crsd_create_autotuned(
+                nrows, ncols, row.shape[0], _p(row), _p(col), _p(val), _dtype_code(val.dtype), ctypes.byref(o),
+                _p(cand), int(cand.shape[0]), int(reps), ctypes.byref(h), _p(ms),
+            )
+        )
+        return cls(h.value, val.dtype), {int(m): (None if t < 0 else float(t)) for m, t in zip(cand, ms)}
 
     @classmethod
     def from_csr(cls, nrows, ncols, row_ptr, col, val, *, mrows=0, idle_max=-1, flags=0, host_only=False, device=-1):

@@ -723,6 +723,75 @@ crsd_status_t crsd_autotune(crsd_matrix_t A, const void *x, void *y, int32_t rep
     return CRSD_OK;
 }
 
+// Build-time autotuning: the row-segment height changes the layout itself
+// (P:L351-361), so every candidate is built, its kernel variant autotuned on
+// scratch vectors, and the fastest handle kept (one candidate resident at a
+// time besides the best so far).
+crsd_status_t crsd_create_autotuned(int64_t nrows, int64_t ncols, int64_t nnz, const int64_t *row, const int64_t *col,
+                                    const void *val, crsd_dtype_t dtype, const crsd_opts_t *opts,
+                                    const int32_t *mrows_cand, int32_t ncand, int32_t reps, crsd_matrix_t *out,
+                                    double *ms_out) {
+    if (!out) return fail(CRSD_ERR_INVALID_ARG, "out is NULL");
+    *out = nullptr;
+    crsd_opts_t o;
+    if (opts) o = *opts;
+    else crsd_opts_init(&o);
+    if (o.flags & CRSD_HOST_ONLY) return fail(CRSD_ERR_UNSUPPORTED, "autotuning needs a GPU handle");
+    if (o.row_begin != 0 || (o.row_end != 0 && o.row_end != nrows))
+        return fail(CRSD_ERR_UNSUPPORTED, "autotuning is for one-GPU (non-partitioned) handles");
+    const int32_t dflt[] = {0};
+    if (!mrows_cand || ncand <= 0) {
+        mrows_cand = dflt;
+        ncand = 1;
+    }
+    const size_t es = dtype == CRSD_R64F ? 8 : 4;
+    void *x = nullptr, *y = nullptr;
+    crsd_matrix_t best = nullptr;
+    double best_ms = 1e300;
+    crsd_status_t st = CRSD_OK;
+    for (int32_t c = 0; c < ncand; ++c) {
+        crsd_opts_t oc = o;
+        oc.mrows = mrows_cand[c];
+        crsd_matrix_t A = nullptr;
+        crsd_status_t sc = crsd_create_from_coo(nrows, ncols, nnz, row, col, val, dtype, &oc, &A);
+        if (ms_out) ms_out[c] = -1.0;
+        if (sc) continue;  // this candidate is not valid for the GPU path (e.g. mrows alignment)
+        if (!x) {
+            cudaError_t e1 = cudaMalloc(&x, es * (size_t)ncols), e2 = cudaMalloc(&y, es * (size_t)nrows);
+            if (e1 != cudaSuccess || e2 != cudaSuccess) {
+                crsd_destroy(A);
+                st = fail(CRSD_ERR_ALLOC, "autotune scratch vectors");
+                break;
+            }
+            cudaMemset(x, 0, es * (size_t)ncols);  // values do not change the timing
+        }
+        double ms[5];
+        int32_t chosen = 0;
+        sc = crsd_autotune(A, x, y, reps, ms, &chosen, nullptr);
+        if (sc) {
+            crsd_destroy(A);
+            continue;
+        }
+        if (ms_out) ms_out[c] = ms[0];
+        if (ms[0] < best_ms) {
+            if (best) crsd_destroy(best);
+            best = A;
+            best_ms = ms[0];
+        } else {
+            crsd_destroy(A);
+        }
+    }
+    if (x) cudaFree(x);
+    if (y) cudaFree(y);
+    if (st) {
+        if (best) crsd_destroy(best);
+        return st;
+    }
+    if (!best) return fail(CRSD_ERR_UNSUPPORTED, "no mrows candidate is valid for the GPU path");
+    *out = best;
+    return CRSD_OK;
+}
+
 crsd_status_t crsd_export_paper_ell(crsd_matrix_t A, int64_t *nrows_s, int64_t *width, int64_t *rowno,
                                     int64_t *colval, void *val) {
     if (!A) return fail(CRSD_ERR_INVALID_ARG, "A is NULL");

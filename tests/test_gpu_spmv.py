@@ -490,3 +490,21 @@ def test_jit_persistent_parity(torch_cuda, case, dt, monkeypatch):
         a = gen.random_diagonal(4000 + 97 * s, 3900, 30 + s, ndiag=12, max_off=900, p_break=0.02, max_break=400, n_scatter=200)
     for alpha, beta in ((1.0, 0.0), (-0.75, 0.5)):
         _parity(torch_cuda, a, dt, alpha, beta, seed=3, variant=4)
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_create_autotuned(torch_cuda, dt):
+    """crsd_create_autotuned: every valid mrows candidate is built and timed,
+    invalid ones (not a multiple of 32*RPT) are skipped, the fastest handle is
+    returned and matches the oracle."""
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix
+
+    a = gen.config3(n=40).astype(dt)
+    cands = (64, 128, 256, 100) if dt == np.float64 else (128, 256, 512, 100)
+    A, ms = CRSDMatrix.autotuned(a.nrows, a.ncols, a.row, a.col, a.val, mrows_candidates=cands, reps=3)
+    assert ms[100] is None and all(ms[m] is not None for m in cands[:3])
+    assert A.info()["mrows"] == min(cands[:3], key=lambda m: ms[m])
+    x = np.random.default_rng(8).uniform(-1, 1, a.ncols).astype(dt)
+    y = _run(torch_cuda, A, x, 1.0, 0.0, None, a.nrows)
+    yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, x)
+    assert coo.parity_error(y, yref, scale) <= TOL[dt]
