@@ -96,9 +96,10 @@ typedef enum { CRSD_R32F = 0, CRSD_R64F = 1 } crsd_dtype_t;
  *             ring with TMA bulk copies) or CRSD_VARIANT_JIT (4: the TMA
  *             data movement with every pattern quantity baked into a
  *             runtime-generated codelet, NVRTC; the paper's code generator,
- *             P:L131-143). AUTO picks TMA for small segments, PIPE for large
- *             ones, LDG when neither staging fits in shared memory. DESIGN.md
- *             "Kernels".
+ *             P:L131-143). AUTO picks JIT when a segment stages in <= 75 KB
+ *             (TMA for <= 32 KB unsplit segments if NVRTC is unavailable),
+ *             PIPE for larger ones, LDG when neither staging fits in shared
+ *             memory. DESIGN.md "Kernels".
  */
 typedef struct {
     int32_t mrows;
@@ -142,7 +143,7 @@ typedef struct {
     int64_t halo_lo, halo_hi;       /* x halo pads (elements) of a row-partitioned handle; halo_lo is a multiple of 4 */
     int64_t halo_lo_valid, halo_hi_valid; /* halo elements actually exchanged (<= the pads; clipped at the matrix edges) */
     int64_t device_bytes;           /* device memory held by the handle */
-    int32_t variant;                /* kernel variant in use (CRSD_VARIANT_LDG / _TMA / _PIPE) */
+    int32_t variant;                /* kernel variant in use (CRSD_VARIANT_LDG / _TMA / _PIPE / _JIT) */
     int32_t smem_bytes;             /* dynamic shared memory per CTA of the TMA variant */
     int64_t unique_bytes_beta0;     /* algorithmic bytes of one SpMV with beta == 0 */
     int64_t unique_bytes_beta1;     /* ... with beta != 0 (y also read) */

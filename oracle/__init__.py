@@ -14,7 +14,12 @@ Modules
                   paper-layout arrays (Fig. 4) and the B200 layout      [pinned]
   decode       -- independent CRSD decoder + structural invariants I1-I8 [pinned]
   closed_forms -- analytic A*x for 5/7/27-point stencils                [pinned]
+  cg_ref       -- textbook conjugate gradient (Hestenes-Stiefel / Saad
+                  Alg. 6.18) on the definition SpMV                    [pinned]
+  crsd_ref.paper_ell_rows -- the paper's ELL scatter-row pass
+                  (P:L395-411), paper evaluation order       [pinned]
 
-Every function is pinned by ``tests/test_oracle_pins.py`` (``-m "not gpu"``);
+Every function is pinned by ``tests/test_oracle_pins.py`` and
+``tests/test_oracle_cg_pins.py`` (``-m "not gpu"``);
 none is "parity unpinned".
 """

@@ -157,14 +157,14 @@ struct SpmvArgs {
     const int32_t *seg_list;  // if non-null: CTA work = seg_list[i]
     int64_t seg_begin, seg_count;
     int32_t mrows;
-    int32_t smem_bytes;       // TMA variant: dynamic shared memory per CTA
+    int32_t smem_bytes;       // largest whole-segment staging (values + x windows), bytes
     int32_t pipe_xmax_elems;  // PIPE variant: largest x staging of a pattern (elements)
     int32_t max_ndias;        // largest NDias over patterns
     int32_t tma_split;        // TMA variant: CTAs per segment (each covers mrows/split rows)
     int32_t tma_q;            // TMA variant: rows per thread
     int64_t tma_smem;         // TMA variant: dynamic shared memory per CTA
     int32_t has_scatter;      // the matrix has scatter points (selects the staging kernel)
-    int32_t variant;          // VARIANT_LDG or VARIANT_TMA
+    int32_t variant;          // VARIANT_LDG / _TMA / _PIPE / _JIT
     T alpha, beta;
     // optional fused dot (JIT variant, CG): *dot_out = sum_rows x[row] * y[row]
     // over the launch's rows, deterministic (per-CTA partials, last CTA sums)
