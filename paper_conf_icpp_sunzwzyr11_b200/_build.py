@@ -81,5 +81,26 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB
 
 
+EXAMPLE_SRC = os.path.join(ROOT, "examples", "crsd_example.c")
+EXAMPLE_BIN = os.path.join(ROOT, "examples", "crsd_example")
+
+
+def build_example() -> str:
+    """Plain-C consumer of the C-ABI (examples/crsd_example.c), linked
+    against the in-tree libcrsd.so: proves the boundary needs no Python."""
+    if os.path.exists(EXAMPLE_BIN) and os.path.getmtime(EXAMPLE_BIN) > max(
+        os.path.getmtime(EXAMPLE_SRC), os.path.getmtime(LIB)
+    ):
+        return EXAMPLE_BIN
+    cuda = os.path.dirname(os.path.dirname(NVCC))
+    cmd = [
+        "gcc", "-O2", "-Wall", f"-I{os.path.join(ROOT, 'include')}", f"-I{os.path.join(cuda, 'include')}",
+        EXAMPLE_SRC, "-o", EXAMPLE_BIN, f"-L{HERE}", "-lcrsd", f"-L{os.path.join(cuda, 'lib64')}", "-lcudart",
+        "-lm", f"-Wl,-rpath,{HERE}", f"-Wl,-rpath,{os.path.join(cuda, 'lib64')}",
+    ]
+    subprocess.check_call(cmd)
+    return EXAMPLE_BIN
+
+
 if __name__ == "__main__":
     print(build(force="--force" in sys.argv, verbose=True))

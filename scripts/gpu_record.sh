@@ -14,7 +14,9 @@ for cfg in "c2 f32" "c3 f64" "c3 f32" "c4 f32"; do
   set -- $cfg
   timeout 900 python bench.py --no-cpu --config $1 --dtype $2 > gpurun_out/bench_$1_$2.json 2> gpurun_out/bench_$1_$2.err
 done
-for d in f64 f32; do timeout 300 python scripts/cg_bench.py 256 400 $d; done > gpurun_out/cg_bench.jsonl 2>&1
+timeout 900 python bench.py --no-cpu --config c3 --dtype f32 --mrows 256 > gpurun_out/bench_c3_f32_m256.json 2> gpurun_out/bench_c3_f32_m256.err
+for d in f64 f32; do timeout 600 python bench.py --workload cg --dtype $d > gpurun_out/bench_cg_$d.json 2> gpurun_out/bench_cg_$d.err; done
+timeout 600 ncu --set full --clock-control none -k regex:cg_ -s 12 -c 3 -o gpurun_out/prof_cg_f64 -f python bench.py --workload cg --steps 20 --warmup 3 > gpurun_out/ncu_cg.log 2>&1
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 40 --csv --log-file gpurun_out/launches_default.csv python bench.py --steps 20 --warmup 3 --no-cpu > /dev/null 2>&1
 for cfg in "c2 f64" "c2 f32" "c3 f64" "c3 f32" "c4 f32"; do
   set -- $cfg

@@ -265,3 +265,18 @@ def test_paper_ell_needs_flag():
     A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, host_only=True)
     with pytest.raises(Exception, match="UNSUPPORTED"):
         A.export_paper_ell()
+
+
+def test_c_example_links_against_the_c_abi():
+    """examples/crsd_example.c (plain C, no Python) compiles and links against
+    libcrsd.so through include/crsd.h alone; it runs on the GPU in
+    tests/test_gpu_spmv.py::test_c_example_runs."""
+    import os
+    import subprocess
+
+    from paper_conf_icpp_sunzwzyr11_b200 import _build
+
+    exe = _build.build_example()
+    assert os.access(exe, os.X_OK)
+    out = subprocess.run(["ldd", exe], capture_output=True, text=True).stdout
+    assert "libcrsd.so" in out and "not found" not in out

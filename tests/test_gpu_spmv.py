@@ -508,3 +508,16 @@ def test_create_autotuned(torch_cuda, dt):
     y = _run(torch_cuda, A, x, 1.0, 0.0, None, a.nrows)
     yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, x)
     assert coo.parity_error(y, yref, scale) <= TOL[dt]
+
+
+def test_c_example_runs(torch_cuda):
+    """The plain-C consumer of the C-ABI: CRSD build, SpMV vs the A*1 closed
+    form (exact), CG to 1e-10 -- exit code 0."""
+    import subprocess
+
+    from paper_conf_icpp_sunzwzyr11_b200 import _build
+
+    exe = _build.build_example()
+    r = subprocess.run([exe, "40"], capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stdout + r.stderr
+    assert "closed-form mismatches 0" in r.stdout
