@@ -296,17 +296,25 @@ def run_crsd(args):
     import torch
     import torch.distributed as dist
 
-    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, Comm
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, Comm, P2PComm
 
     world = args.gpus
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    # --share-gpu: every rank on cuda:0 (functional check of the multi-rank
+    # path on a one-GPU box; NCCL refuses two ranks per GPU, so the torch
+    # plumbing uses gloo and the transport must be p2p). Not a scaling number.
+    if args.share_gpu:
+        local_rank = 0
+        if args.transport != "p2p":
+            raise SystemExit("--share-gpu needs --transport p2p")
     if world > 1:
-        dist.init_process_group("nccl", init_method="env://")
+        dist.init_process_group("gloo" if args.share_gpu else "nccl", init_method="env://")
         world = dist.get_world_size()
         rank = dist.get_rank()
     torch.cuda.set_device(local_rank)
     dev = local_rank
+    red_dev = "cpu" if args.share_gpu else f"cuda:{dev}"
 
     a, desc, (rb, re), N = workload(args.config, args.dtype, world, rank)
     dt = a.val.dtype
@@ -333,7 +341,10 @@ def run_crsd(args):
         xp = torch.zeros(lo + nloc + hi, dtype=tdt, device=f"cuda:{dev}")
         xp[lo : lo + nloc] = x_full
         y = torch.empty(nloc, dtype=tdt, device=f"cuda:{dev}")
-        comm = Comm(rank, world, dev)
+        if args.transport == "p2p":
+            comm = P2PComm(rank, world, dev, mailbox_bytes=max(1 << 20, 4 * (lo + hi) * es))
+        else:
+            comm = Comm(rank, world, dev)
         A.dist_bind(comm)
 
         def step():
@@ -375,10 +386,10 @@ def run_crsd(args):
     total_ms = t_all0.elapsed_time(t_all1)
     step_ms = [s.elapsed_time(e) for s, e in ev]
     if world > 1:
-        tt = torch.tensor([total_ms], dtype=torch.float64, device=f"cuda:{dev}")
+        tt = torch.tensor([total_ms], dtype=torch.float64, device=red_dev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         total_ms = float(tt.item())
-        nn = torch.tensor([nnz_local, ub], dtype=torch.float64, device=f"cuda:{dev}")
+        nn = torch.tensor([nnz_local, ub], dtype=torch.float64, device=red_dev)
         dist.all_reduce(nn)
         nnz_all, ub_all = float(nn[0].item()), float(nn[1].item())
     else:
@@ -463,7 +474,7 @@ def run_crsd(args):
         t0 = time.perf_counter()
         for _ in range(ke):
             e2e_step()
-        te = torch.tensor([(time.perf_counter() - t0) / ke], dtype=torch.float64, device=f"cuda:{dev}")
+        te = torch.tensor([(time.perf_counter() - t0) / ke], dtype=torch.float64, device=red_dev)
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
         te = float(te.item())
         e2e = {
@@ -472,7 +483,7 @@ def run_crsd(args):
             "h2d_bytes_per_step": int((re - rb) * es) * world,
             "d2h_bytes_per_step": int((re - rb) * es) * world,
             "ms_per_step": round(te * 1e3, 4),
-            "path": "per rank: H2D of the owned x slice, crsd_spmv_dist (NCCL halo + SpMV), D2H of the y slice; max over ranks",
+            "path": f"per rank: H2D of the owned x slice, crsd_spmv_dist ({args.transport} halo + SpMV), D2H of the y slice; max over ranks",
         }
     if rank != 0:
         if comm is not None:
@@ -511,6 +522,7 @@ def run_crsd(args):
             "scatter": info["nscatter"],
             "l2": f"inputs larger than L2 ({ub / 1e9:.2f} GB streamed per step vs {L2_BYTES / 2**20:.0f} MiB L2); no flush",
             "build_s": round(build_s, 2),
+            "parallelism": f"row-partitioned x{world}" + (f", {args.transport} halo" if world > 1 else "") + (", ranks share cuda:0 (functional only)" if args.share_gpu else ""),
         },
         "hbm_gbs": round(ub_all / (ms * 1e-3) / 1e9, 1),
         "hbm_frac_of_peak": round(ub_all / (ms * 1e-3) / 1e9 / (peak * world), 4),
@@ -678,6 +690,8 @@ def main():
     ap.add_argument("--impl", default="crsd", choices=["crsd", "reference"])
     ap.add_argument("--workload", default="spmv", choices=["spmv", "cg"], help="cg: K steps of crsd_cg (one GPU)")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p"], help="N>1 halo exchange: NCCL send/recv or the library's peer-memory kernels")
+    ap.add_argument("--share-gpu", action="store_true", help="N>1 ranks all on cuda:0 (functional check only; needs --transport p2p)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

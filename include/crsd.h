@@ -248,6 +248,54 @@ crsd_status_t crsd_comm_unique_id(void *id128);
 crsd_status_t crsd_comm_init_rank(const void *id128, int rank, int world, int device, crsd_comm_t *out);
 crsd_status_t crsd_comm_destroy(crsd_comm_t comm);
 
+/*
+ * Peer-memory communicator: the library's own transport (csrc/p2p.cu) in
+ * place of NCCL for the halo exchange (north_star (3))
+ * and the CG's scalar allreduce. Each rank allocates one device region
+ * [flags 64 KB | mailbox parity 0 | mailbox parity 1] and exports it with
+ * CUDA IPC; after crsd_comm_p2p_open every rank maps every peer's region
+ * (NVLink/NVSwitch loads and stores between GPUs; also works for several
+ * processes sharing one GPU). The halo moves by our kernels: the sender
+ * packs its send slices into its mailbox and raises a flag in each
+ * receiver's region; the receiver waits for the flag and pulls the slices
+ * from the peer's mailbox straight into the pads of x_padded, then raises a
+ * "consumed" flag so the sender may reuse that parity. Epochs live on the
+ * device, so the exchange can be captured into a CUDA graph (crsd_cg does).
+ * Every wait is bounded (10 s): on timeout the kernel returns and
+ * crsd_comm_error reports a non-zero code instead of the GPU hanging.
+ *
+ *   crsd_comm_init_p2p(rank, world, device, mailbox_bytes, handle64, &c)
+ *       mailbox_bytes: capacity per parity, >= the bytes this rank sends per
+ *       exchange (slices rounded up to 256 B; crsd_dist_bind_ranges checks).
+ *       handle64: HOST 64 bytes out, this rank's cudaIpcMemHandle_t.
+ *       world <= 64. Not collective.
+ *   crsd_comm_p2p_open(c, handles)
+ *       handles: HOST world*64 bytes, every rank's handle in rank order
+ *       (allgathered by the caller, e.g. through torch.distributed).
+ *       Must be called on every rank after every rank's init.
+ *   crsd_dist_bind_ranges(A, c, ranges4)
+ *       The bind of crsd_dist_bind with the range table supplied by the
+ *       caller: HOST int64[world][4] = every rank's crsd_dist_ranges() row.
+ *       Required for peer-memory communicators (crsd_dist_bind returns
+ *       INVALID_ARG for them); also accepted with NCCL communicators.
+ *   crsd_comm_allreduce_f64(c, dev, n, stream)
+ *       In-place sum of n <= 4 DEVICE doubles over all ranks, stream-ordered.
+ *       Peer memory: every rank sums the W contributions in rank order, so
+ *       all ranks get bit-identical results. NCCL: ncclAllReduce.
+ *   crsd_comm_error(c, &err)
+ *       Synchronous. err = 0, or 1/2/3 when a send / recv / allreduce wait
+ *       timed out (a peer never arrived); the results are then invalid.
+ */
+crsd_status_t crsd_comm_init_p2p(int rank, int world, int device, int64_t mailbox_bytes, void *ipc_handle64,
+                                 crsd_comm_t *out);
+crsd_status_t crsd_comm_p2p_open(crsd_comm_t comm, const void *ipc_handles);
+crsd_status_t crsd_dist_bind_ranges(crsd_matrix_t A_local, crsd_comm_t comm, const int64_t *ranges4);
+crsd_status_t crsd_comm_allreduce_f64(crsd_comm_t comm, double *dev, int n, void *stream);
+crsd_status_t crsd_comm_error(crsd_comm_t comm, int32_t *err);
+/* This handle's row of the range table: {row_begin, row_end, halo_lo_valid,
+ * halo_hi_valid} (the halo widths actually needed, without alignment). */
+crsd_status_t crsd_dist_ranges(crsd_matrix_t A_local, int64_t *ranges4);
+
 /* Exchange row ranges and halo widths with every rank (collective, once per
  * handle and communicator) and derive the send/recv plan. */
 crsd_status_t crsd_dist_bind(crsd_matrix_t A_local, crsd_comm_t comm, void *stream);

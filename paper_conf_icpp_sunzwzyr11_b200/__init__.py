@@ -6,6 +6,7 @@ include/crsd.h, sm_100a kernels in csrc/); this package is its binding.
 from .crsd import (  # noqa: F401
     CRSDMatrix,
     Comm,
+    P2PComm,
     CRSDError,
     dist_plan,
     partition_rows,

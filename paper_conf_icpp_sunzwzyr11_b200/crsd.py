@@ -55,6 +55,12 @@ EXPORTED = [
     "crsd_autotune",
     "crsd_export_paper_ell",
     "crsd_create_autotuned",
+    "crsd_comm_init_p2p",
+    "crsd_comm_p2p_open",
+    "crsd_dist_bind_ranges",
+    "crsd_comm_allreduce_f64",
+    "crsd_comm_error",
+    "crsd_dist_ranges",
 ]
 
 
@@ -154,6 +160,12 @@ def _load():
         "crsd_autotune": ([P, P, P, I32, P, P, P], ctypes.c_int),
         "crsd_export_paper_ell": ([P, P, P, P, P, P], ctypes.c_int),
         "crsd_create_autotuned": ([I64, I64, I64, P, P, P, ctypes.c_int, P, P, I32, I32, P, P], ctypes.c_int),
+        "crsd_comm_init_p2p": ([ctypes.c_int, ctypes.c_int, ctypes.c_int, I64, P, P], ctypes.c_int),
+        "crsd_comm_p2p_open": ([P, P], ctypes.c_int),
+        "crsd_dist_bind_ranges": ([P, P, P], ctypes.c_int),
+        "crsd_comm_allreduce_f64": ([P, P, ctypes.c_int, P], ctypes.c_int),
+        "crsd_comm_error": ([P, P], ctypes.c_int),
+        "crsd_dist_ranges": ([P, P], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)
@@ -392,8 +404,21 @@ class CRSDMatrix:
         _check(lib.crsd_export_paper_ell(self._h, None, None, _p(rowno), _p(colval), _p(val)))
         return {"num_scatter_rows": n.value, "num_scatter_width": w.value, "scatter_rowno": rowno, "scatter_colval": colval, "scatter_val": val}
 
-    def dist_bind(self, comm, stream=None):
-        _check(lib.crsd_dist_bind(self._h, comm._h, _stream_ptr(stream)))
+    def dist_bind(self, comm, stream=None, pg=None):
+        """Derive the halo plan. NCCL communicators exchange the range table
+        themselves (crsd_dist_bind); peer-memory ones get it allgathered here
+        over torch.distributed (crsd_dist_bind_ranges)."""
+        if isinstance(comm, P2PComm):
+            table = comm.allgather_i64(self.dist_ranges())
+            _check(lib.crsd_dist_bind_ranges(self._h, comm._h, _p(table)))
+        else:
+            _check(lib.crsd_dist_bind(self._h, comm._h, _stream_ptr(stream)))
+
+    def dist_ranges(self) -> np.ndarray:
+        """{row_begin, row_end, halo_lo_valid, halo_hi_valid} of this handle (crsd_dist_ranges)."""
+        r = np.zeros(4, np.int64)
+        _check(lib.crsd_dist_ranges(self._h, _p(r)))
+        return r
 
     # ------------------------------------------------------------ introspection
     def info(self) -> dict:
@@ -464,6 +489,67 @@ class Comm:
         h = ctypes.c_void_p()
         _check(lib.crsd_comm_init_rank(_p(uid), rank, world, device, ctypes.byref(h)))
         self._h = h
+
+    def allreduce_f64(self, dev_tensor, stream=None):
+        """In-place sum over ranks of a CUDA float64 tensor (crsd_comm_allreduce_f64: ncclAllReduce)."""
+        _check(lib.crsd_comm_allreduce_f64(self._h, ctypes.c_void_p(dev_tensor.data_ptr()), dev_tensor.numel(), _stream_ptr(stream)))
+        return dev_tensor
+
+    def error(self) -> int:
+        return 0
+
+    def close(self):
+        if self._h is not None and self._h.value:
+            lib.crsd_comm_destroy(self._h)
+        self._h = None
+
+
+class P2PComm:
+    """Peer-memory communicator owned by libcrsd (crsd_comm_init_p2p /
+    crsd_comm_p2p_open): the halo exchange and the CG's scalar allreduce run
+    as the library's own kernels over CUDA-IPC-mapped regions. Only the
+    64-byte IPC handles and the range table travel over torch.distributed
+    (any backend: gloo works, so several processes may share one GPU)."""
+
+    def __init__(self, rank: int, world: int, device: int, mailbox_bytes: int = 64 << 20, pg=None):
+        import torch
+        import torch.distributed as dist
+
+        self.rank, self.world, self.device, self._pg = rank, world, device, pg
+        self._h = None
+        handle = np.zeros(64, np.uint8)
+        h = ctypes.c_void_p()
+        _check(lib.crsd_comm_init_p2p(rank, world, device, int(mailbox_bytes), _p(handle), ctypes.byref(h)))
+        self._h = h
+        allh = self._allgather(torch.from_numpy(handle.copy()))
+        _check(lib.crsd_comm_p2p_open(self._h, _p(np.ascontiguousarray(allh))))
+        dist.barrier(group=pg)
+
+    def _allgather(self, t):
+        import torch
+        import torch.distributed as dist
+
+        dev = torch.device("cuda", self.device) if dist.get_backend(self._pg) == "nccl" else torch.device("cpu")
+        t = t.to(dev)
+        out = [torch.empty_like(t) for _ in range(self.world)]
+        dist.all_gather(out, t, group=self._pg)
+        return torch.stack(out).cpu().numpy()
+
+    def allgather_i64(self, row: np.ndarray) -> np.ndarray:
+        import torch
+
+        return np.ascontiguousarray(self._allgather(torch.from_numpy(np.asarray(row, np.int64).copy())), np.int64)
+
+    def allreduce_f64(self, dev_tensor, stream=None):
+        """In-place sum over ranks of a CUDA float64 tensor with <= 4 elements (crsd_comm_allreduce_f64)."""
+        _check(lib.crsd_comm_allreduce_f64(self._h, ctypes.c_void_p(dev_tensor.data_ptr()), dev_tensor.numel(), _stream_ptr(stream)))
+        return dev_tensor
+
+    def error(self) -> int:
+        """0, or 1/2/3 when a send / recv / allreduce wait timed out (crsd_comm_error)."""
+        e = ctypes.c_int32()
+        _check(lib.crsd_comm_error(self._h, ctypes.byref(e)))
+        return e.value
 
     def close(self):
         if self._h is not None and self._h.value:

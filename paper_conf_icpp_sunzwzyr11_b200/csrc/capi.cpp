@@ -820,6 +820,15 @@ crsd_status_t crsd_dist_x_layout(crsd_matrix_t A, int64_t *halo_lo, int64_t *n_l
     return CRSD_OK;
 }
 
+crsd_status_t crsd_dist_ranges(crsd_matrix_t A, int64_t *r4) {
+    if (!A || !r4) return fail(CRSD_ERR_INVALID_ARG, "NULL argument");
+    r4[0] = A->H.row_begin;
+    r4[1] = A->H.row_end;
+    r4[2] = A->halo_lo_valid;
+    r4[3] = A->halo_hi_valid;
+    return CRSD_OK;
+}
+
 crsd_status_t crsd_partition_rows(int64_t nrows, int32_t mrows, int world, const double *weights, int64_t *bounds) {
     if (nrows <= 0 || mrows <= 0 || world <= 0 || !bounds) return fail(CRSD_ERR_INVALID_ARG, "bad argument");
     const int64_t nseg = (nrows + mrows - 1) / mrows;

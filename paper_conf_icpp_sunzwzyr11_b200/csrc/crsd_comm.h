@@ -1,12 +1,30 @@
-// NCCL communicator behind crsd_comm_t (dist.cpp, solver.cpp).
+// Communicator behind crsd_comm_t (dist.cpp, solver.cpp): NCCL, or the
+// library's own peer-memory transport (p2p.cu) over CUDA-IPC-mapped regions.
 #pragma once
 
 #include <cuda_runtime.h>
 #include <nccl.h>
 
+#include <vector>
+
+#include "crsd.h"
+#include "crsd_p2p.h"
+
 struct crsd_comm_s {
+    enum Kind { NCCL = 0, P2P = 1 };
+    int kind = NCCL;
     ncclComm_t comm = nullptr;
     int rank = 0, world = 1, device = 0;
     cudaStream_t cs = nullptr;                         // halo exchange stream
     cudaEvent_t ev_x = nullptr, ev_halo = nullptr;
+    // P2P: own symmetric region [P2PFlags | mailbox parity 0 | parity 1] and the peers' (IPC-opened)
+    void *sym = nullptr;
+    int64_t cap = 0;                  // bytes per mailbox parity
+    std::vector<void *> peer_sym;     // world entries, nullptr for self / not opened
+    bool opened = false;
 };
+
+namespace crsd {
+// Sum n doubles (device pointer) over every rank of comm, in place, on stream.
+crsd_status_t comm_allreduce_f64(crsd_comm_s *c, double *dev, int n, cudaStream_t stream);
+}  // namespace crsd

@@ -76,6 +76,9 @@ struct crsd_matrix_s {
     bool bound = false;
     std::vector<int64_t> recv_peer, recv_off, recv_count;  // offsets into x_padded
     std::vector<int64_t> send_peer, send_off, send_count;
+    // peer-memory transport: byte offsets into my mailbox (sends) / the sender's mailbox (recvs)
+    std::vector<int64_t> send_mb_off, recv_mb_off;
+    const void *bound_comm = nullptr;
 };
 
 namespace crsd {

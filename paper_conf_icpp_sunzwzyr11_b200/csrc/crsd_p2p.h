@@ -1,0 +1,51 @@
+// Peer-memory transport (p2p.cu): symmetric flag block and launch records.
+#pragma once
+
+#include <cstdint>
+
+namespace crsd {
+
+constexpr int P2P_MAX_WORLD = 64;
+constexpr int P2P_MAX_ITEMS = 16;  // slices per rank and direction (2 per peer; multi-hop)
+constexpr int P2P_MAX_RED = 4;     // doubles per scalar allreduce
+constexpr int64_t P2P_FLAGS_BYTES = 65536;
+
+// Head of every rank's symmetric region. Slots indexed by the WRITING rank.
+struct P2PFlags {
+    uint64_t ready[P2P_MAX_WORLD];      // written by sender q: its mailbox holds epoch ready[q]
+    uint64_t consumed[P2P_MAX_WORLD];   // written by receiver q: it has read my epoch consumed[q]
+    uint64_t red_ready[P2P_MAX_WORLD];  // written by q: red[.][q] holds its epoch red_ready[q]
+    double red[2][P2P_MAX_WORLD][P2P_MAX_RED];
+    uint64_t halo_epoch;  // own: last completed halo exchange
+    uint64_t red_epoch;   // own: last completed allreduce
+    uint32_t counter[2];  // own: grid arrival counters (send, recv)
+    uint32_t err;         // own: 0, or 1/2/3 = send/recv/allreduce wait timed out
+};
+static_assert(sizeof(P2PFlags) <= P2P_FLAGS_BYTES, "P2PFlags too large");
+
+struct P2PItem {
+    const void *src;
+    void *dst;
+    int64_t bytes;
+};
+
+struct P2PLaunch {
+    P2PFlags *local;
+    P2PFlags *peer_flags[P2P_MAX_ITEMS];  // per distinct peer of this direction
+    int32_t peer[P2P_MAX_ITEMS];
+    int32_t npeer, nitems, rank, pad_;
+    int64_t cap;  // bytes per mailbox parity
+    P2PItem items[P2P_MAX_ITEMS];
+};
+
+struct P2PReduce {
+    P2PFlags *local;
+    P2PFlags *peer_flags[P2P_MAX_WORLD];
+    int32_t rank, world;
+};
+
+int p2p_launch_send(const P2PLaunch &L, int grid, void *stream);
+int p2p_launch_recv(const P2PLaunch &L, int grid, void *stream);
+int p2p_launch_allreduce(const P2PReduce &R, double *val, int n, void *stream);
+
+}  // namespace crsd

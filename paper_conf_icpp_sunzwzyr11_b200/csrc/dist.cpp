@@ -10,10 +10,16 @@
 // scatter columns stay inside the owned range) run on the compute stream;
 // the boundary segments run after the halo event. y stays row-distributed:
 // no reduction.
+//
+// Two transports behind crsd_comm_t: NCCL (grouped send/recv), or the
+// library's own peer-memory kernels (p2p.cu) over CUDA-IPC-mapped symmetric
+// regions — loads over NVLink/NVSwitch from the neighbour's mailbox straight
+// into the pads, flag handshakes in peer memory, no NCCL on the data path.
 #include <cuda_runtime.h>
 #include <nccl.h>
 
 #include <algorithm>
+#include <cstddef>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -41,6 +47,11 @@ crsd_status_t cu_fail(cudaError_t e, const char *what) {
     do {                                                    \
         cudaError_t _e = (expr);                            \
         if (_e != cudaSuccess) return cu_fail(_e, #expr); \
+    } while (0)
+#define ST_TRY(expr)                  \
+    do {                              \
+        crsd_status_t _s = (expr);    \
+        if (_s != CRSD_OK) return _s; \
     } while (0)
 
 extern "C" {
@@ -80,6 +91,9 @@ crsd_status_t crsd_comm_destroy(crsd_comm_t c) {
     cudaSetDevice(c->device);
     if (c->cs) cudaStreamSynchronize(c->cs);
     if (c->comm) ncclCommDestroy(c->comm);
+    for (void *p : c->peer_sym)
+        if (p) cudaIpcCloseMemHandle(p);
+    if (c->sym) cudaFree(c->sym);
     if (c->ev_x) cudaEventDestroy(c->ev_x);
     if (c->ev_halo) cudaEventDestroy(c->ev_halo);
     if (c->cs) cudaStreamDestroy(c->cs);
@@ -143,9 +157,205 @@ crsd_status_t crsd_dist_plan(int world, int rank, const int64_t *rg, int64_t *re
     return CRSD_OK;
 }
 
+crsd_status_t crsd_comm_init_p2p(int rank, int world, int device, int64_t mailbox_bytes, void *ipc_handle64,
+                                 crsd_comm_t *out) {
+    if (!out || !ipc_handle64 || world <= 0 || world > crsd::P2P_MAX_WORLD || rank < 0 || rank >= world ||
+        mailbox_bytes < 0)
+        return crsd::fail(CRSD_ERR_INVALID_ARG, "bad peer-memory communicator arguments");
+    *out = nullptr;
+    static_assert(sizeof(cudaIpcMemHandle_t) == 64, "cudaIpcMemHandle_t must be 64 bytes");
+    CU_TRY(cudaSetDevice(device));
+    crsd_comm_s *c = new crsd_comm_s();
+    c->kind = crsd_comm_s::P2P;
+    c->rank = rank;
+    c->world = world;
+    c->device = device;
+    c->cap = (mailbox_bytes + 255) / 256 * 256;
+    c->peer_sym.assign(world, nullptr);
+    const size_t bytes = crsd::P2P_FLAGS_BYTES + 2 * c->cap;
+    cudaError_t e = cudaMalloc(&c->sym, bytes);
+    if (e == cudaSuccess) e = cudaMemset(c->sym, 0, crsd::P2P_FLAGS_BYTES);
+    if (e == cudaSuccess) e = cudaIpcGetMemHandle((cudaIpcMemHandle_t *)ipc_handle64, c->sym);
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->cs, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_x, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_halo, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaDeviceSynchronize();
+    if (e != cudaSuccess) {
+        crsd_comm_destroy(c);
+        return cu_fail(e, "peer-memory communicator setup");
+    }
+    *out = c;
+    return CRSD_OK;
+}
+
+crsd_status_t crsd_comm_p2p_open(crsd_comm_t c, const void *ipc_handles) {
+    if (!c || !ipc_handles) return crsd::fail(CRSD_ERR_INVALID_ARG, "NULL argument");
+    if (c->kind != crsd_comm_s::P2P) return crsd::fail(CRSD_ERR_INVALID_ARG, "not a peer-memory communicator");
+    if (c->opened) return crsd::fail(CRSD_ERR_INVALID_ARG, "communicator already opened");
+    CU_TRY(cudaSetDevice(c->device));
+    for (int q = 0; q < c->world; ++q) {
+        if (q == c->rank) continue;
+        cudaIpcMemHandle_t h;
+        std::memcpy(&h, (const char *)ipc_handles + 64 * q, 64);
+        void *p = nullptr;
+        CU_TRY(cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess));
+        c->peer_sym[q] = p;
+    }
+    c->opened = true;
+    return CRSD_OK;
+}
+
+crsd_status_t crsd_comm_error(crsd_comm_t c, int32_t *err) {
+    if (!c || !err) return crsd::fail(CRSD_ERR_INVALID_ARG, "NULL argument");
+    *err = 0;
+    if (c->kind != crsd_comm_s::P2P) return CRSD_OK;
+    CU_TRY(cudaSetDevice(c->device));
+    uint32_t v = 0;
+    CU_TRY(cudaMemcpy(&v, (char *)c->sym + offsetof(crsd::P2PFlags, err), sizeof(v), cudaMemcpyDeviceToHost));
+    *err = (int32_t)v;
+    return CRSD_OK;
+}
+
+crsd_status_t crsd_comm_allreduce_f64(crsd_comm_t c, double *dev, int n, void *stream) {
+    if (!c || !dev || n <= 0) return crsd::fail(CRSD_ERR_INVALID_ARG, "bad allreduce arguments");
+    CU_TRY(cudaSetDevice(c->device));
+    return crsd::comm_allreduce_f64(c, dev, n, (cudaStream_t)stream);
+}
+
+}  // extern "C"
+
+namespace crsd {
+crsd_status_t comm_allreduce_f64(crsd_comm_s *c, double *dev, int n, cudaStream_t s) {
+    if (c->world == 1) return CRSD_OK;
+    if (c->kind == crsd_comm_s::NCCL) {
+        NCCL_TRY(ncclAllReduce(dev, dev, n, ncclFloat64, ncclSum, c->comm, s));
+        return CRSD_OK;
+    }
+    if (!c->opened) return fail(CRSD_ERR_INVALID_ARG, "call crsd_comm_p2p_open first");
+    if (n > P2P_MAX_RED) return fail(CRSD_ERR_INVALID_ARG, "peer-memory allreduce: at most 4 values");
+    P2PReduce R{};
+    R.local = (P2PFlags *)c->sym;
+    R.rank = c->rank;
+    R.world = c->world;
+    for (int q = 0; q < c->world; ++q) R.peer_flags[q] = (P2PFlags *)c->peer_sym[q];
+    CU_TRY((cudaError_t)p2p_launch_allreduce(R, dev, n, s));
+    return CRSD_OK;
+}
+
+namespace {
+// Derive A's send/recv plan from every rank's [row_begin, row_end,
+// halo_lo_valid, halo_hi_valid]; for the peer-memory transport also where
+// each slice sits in the sender's mailbox (its send slices in plan order,
+// 256-B aligned) and check that it fits.
+crsd_status_t mailbox_layout(int W, int q, const int64_t *all, int64_t es, std::vector<int64_t> &peer,
+                             std::vector<int64_t> &begin, std::vector<int64_t> &off, int64_t &total) {
+    std::vector<int64_t> p(2 * W), b(2 * W), cnt(2 * W), d0(2 * W), d1(2 * W), d2(2 * W);
+    int64_t n_r, n_s;
+    ST_TRY(crsd_dist_plan(W, q, all, d0.data(), d1.data(), d2.data(), &n_r, p.data(), b.data(), cnt.data(), &n_s));
+    peer.assign(p.begin(), p.begin() + n_s);
+    begin.assign(b.begin(), b.begin() + n_s);
+    off.resize(n_s);
+    total = 0;
+    for (int64_t k = 0; k < n_s; ++k) {
+        off[k] = total;
+        total += (cnt[k] * es + 255) / 256 * 256;
+    }
+    return CRSD_OK;
+}
+
+crsd_status_t bind_table(crsd_matrix_t A, crsd_comm_t c, const int64_t *all) {
+    const int W = c->world;
+    if (all[4 * c->rank] != A->H.row_begin || all[4 * c->rank + 1] != A->H.row_end)
+        return fail(CRSD_ERR_INVALID_ARG, "range table does not match this handle's rows");
+    std::vector<int64_t> rp(2 * W), rb(2 * W), rc(2 * W), sp(2 * W), sb(2 * W), sc(2 * W);
+    int64_t nr, ns;
+    ST_TRY(crsd_dist_plan(W, c->rank, all, rp.data(), rb.data(), rc.data(), &nr, sp.data(), sb.data(), sc.data(),
+                          &ns));
+    const int64_t es = A->H.elem;
+    std::vector<int64_t> send_mb(ns), recv_mb(nr);
+    if (c->kind == crsd_comm_s::P2P) {
+        if (nr > P2P_MAX_ITEMS || ns > P2P_MAX_ITEMS)
+            return fail(CRSD_ERR_UNSUPPORTED, "peer-memory transport: more than 16 halo slices per direction");
+        std::vector<int64_t> peer, begin, off;
+        int64_t total = 0;
+        ST_TRY(mailbox_layout(W, c->rank, all, es, peer, begin, off, total));
+        if (total > c->cap)
+            return fail(CRSD_ERR_INVALID_ARG, "peer-memory mailbox too small: need " + std::to_string(total) +
+                                                  " bytes per parity, have " + std::to_string(c->cap));
+        for (int64_t k = 0; k < ns; ++k) send_mb[k] = off[k];
+        for (int64_t k = 0; k < nr; ++k) {
+            ST_TRY(mailbox_layout(W, (int)rp[k], all, es, peer, begin, off, total));
+            int64_t found = -1;
+            for (size_t j = 0; j < peer.size(); ++j)
+                if (peer[j] == c->rank && begin[j] == rb[k]) found = off[j];
+            if (found < 0) return fail(CRSD_ERR_INVALID_ARG, "inconsistent halo plan between ranks");
+            recv_mb[k] = found;
+        }
+    }
+    // global column -> index into x_padded
+    const int64_t origin = A->H.row_begin - A->halo_lo;
+    A->recv_peer.assign(rp.begin(), rp.begin() + nr);
+    A->recv_count.assign(rc.begin(), rc.begin() + nr);
+    A->recv_off.resize(nr);
+    for (int64_t k = 0; k < nr; ++k) A->recv_off[k] = rb[k] - origin;
+    A->send_peer.assign(sp.begin(), sp.begin() + ns);
+    A->send_count.assign(sc.begin(), sc.begin() + ns);
+    A->send_off.resize(ns);
+    for (int64_t k = 0; k < ns; ++k) A->send_off[k] = sb[k] - origin;
+    A->send_mb_off = send_mb;
+    A->recv_mb_off = recv_mb;
+    A->bound = true;
+    A->bound_comm = c;
+    return CRSD_OK;
+}
+
+// One halo exchange through peer memory, on the comm stream: p2p_send packs
+// my send slices into my mailbox and flags the receivers; p2p_recv waits for
+// the senders' flags and pulls their slices into the pads of x_padded.
+crsd_status_t p2p_exchange(crsd_matrix_t A, crsd_comm_t c, char *xp) {
+    if (!c->opened) return fail(CRSD_ERR_INVALID_ARG, "call crsd_comm_p2p_open first");
+    const int64_t es = A->H.elem;
+    char *mb = (char *)c->sym + P2P_FLAGS_BYTES;
+    auto fill = [&](P2PLaunch &L, const std::vector<int64_t> &peers) {
+        L.local = (P2PFlags *)c->sym;
+        L.rank = c->rank;
+        L.cap = c->cap;
+        L.npeer = 0;
+        for (int64_t q : peers) {
+            bool seen = false;
+            for (int k = 0; k < L.npeer; ++k) seen |= (L.peer[k] == q);
+            if (!seen) {
+                L.peer[L.npeer] = (int32_t)q;
+                L.peer_flags[L.npeer] = (P2PFlags *)c->peer_sym[q];
+                ++L.npeer;
+            }
+        }
+    };
+    P2PLaunch S{}, R{};
+    fill(S, A->send_peer);
+    S.nitems = (int32_t)A->send_peer.size();
+    for (int k = 0; k < S.nitems; ++k)
+        S.items[k] = P2PItem{xp + es * A->send_off[k], mb + A->send_mb_off[k], es * A->send_count[k]};
+    fill(R, A->recv_peer);
+    R.nitems = (int32_t)A->recv_peer.size();
+    for (int k = 0; k < R.nitems; ++k)
+        R.items[k] = P2PItem{(char *)c->peer_sym[A->recv_peer[k]] + P2P_FLAGS_BYTES + A->recv_mb_off[k],
+                             xp + es * A->recv_off[k], es * A->recv_count[k]};
+    const int grid = 32;
+    CU_TRY((cudaError_t)p2p_launch_send(S, grid, c->cs));
+    CU_TRY((cudaError_t)p2p_launch_recv(R, grid, c->cs));
+    return CRSD_OK;
+}
+}  // namespace
+}  // namespace crsd
+
+extern "C" {
+
 crsd_status_t crsd_dist_bind(crsd_matrix_t A, crsd_comm_t c, void *stream) {
     if (!A || !c) return crsd::fail(CRSD_ERR_INVALID_ARG, "NULL argument");
     if (A->host_only) return crsd::fail(CRSD_ERR_UNSUPPORTED, "host-only handle");
+    if (c->kind != crsd_comm_s::NCCL)
+        return crsd::fail(CRSD_ERR_INVALID_ARG, "peer-memory communicator: use crsd_dist_bind_ranges");
     CU_TRY(cudaSetDevice(A->device));
     const int W = c->world;
     int64_t mine[4] = {A->H.row_begin, A->H.row_end, A->halo_lo_valid, A->halo_hi_valid};
@@ -161,23 +371,13 @@ crsd_status_t crsd_dist_bind(crsd_matrix_t A, crsd_comm_t c, void *stream) {
     cudaFree(d);
     if (r != ncclSuccess) return nccl_fail(r, "ncclAllGather");
     if (e != cudaSuccess) return cu_fail(e, "allgather copy");
-    std::vector<int64_t> rp(2 * W), rb(2 * W), rc(2 * W), sp(2 * W), sb(2 * W), sc(2 * W);
-    int64_t nr, ns;
-    crsd_status_t st = crsd_dist_plan(W, c->rank, all.data(), rp.data(), rb.data(), rc.data(), &nr, sp.data(),
-                                      sb.data(), sc.data(), &ns);
-    if (st) return st;
-    // global column -> index into x_padded
-    const int64_t origin = A->H.row_begin - A->halo_lo;
-    A->recv_peer.assign(rp.begin(), rp.begin() + nr);
-    A->recv_count.assign(rc.begin(), rc.begin() + nr);
-    A->recv_off.resize(nr);
-    for (int64_t k = 0; k < nr; ++k) A->recv_off[k] = rb[k] - origin;
-    A->send_peer.assign(sp.begin(), sp.begin() + ns);
-    A->send_count.assign(sc.begin(), sc.begin() + ns);
-    A->send_off.resize(ns);
-    for (int64_t k = 0; k < ns; ++k) A->send_off[k] = sb[k] - origin;
-    A->bound = true;
-    return CRSD_OK;
+    return crsd::bind_table(A, c, all.data());
+}
+
+crsd_status_t crsd_dist_bind_ranges(crsd_matrix_t A, crsd_comm_t c, const int64_t *ranges4) {
+    if (!A || !c || !ranges4) return crsd::fail(CRSD_ERR_INVALID_ARG, "NULL argument");
+    if (A->host_only) return crsd::fail(CRSD_ERR_UNSUPPORTED, "host-only handle");
+    return crsd::bind_table(A, c, ranges4);
 }
 
 crsd_status_t crsd_spmv_dist(crsd_matrix_t A, const void *alpha, void *x_padded, const void *beta, void *y_local,
@@ -189,6 +389,7 @@ crsd_status_t crsd_spmv_dist(crsd_matrix_t A, const void *alpha, void *x_padded,
     if (((uintptr_t)x_padded | (uintptr_t)y_local) & 15)
         return crsd::fail(CRSD_ERR_INVALID_ARG, "x_padded and y_local must be 16-byte aligned");
     if (c && !A->bound) return crsd::fail(CRSD_ERR_INVALID_ARG, "call crsd_dist_bind first");
+    if (c && A->bound_comm != c) return crsd::fail(CRSD_ERR_INVALID_ARG, "handle was bound to another communicator");
     CU_TRY(cudaSetDevice(A->device));
     const size_t es = A->H.elem;
     char *xp = (char *)x_padded;
@@ -197,15 +398,22 @@ crsd_status_t crsd_spmv_dist(crsd_matrix_t A, const void *alpha, void *x_padded,
     int launches = 0;
     crsd_status_t st;
     if (c) {
-        const ncclDataType_t ty = (A->H.dtype == CRSD_R64F) ? ncclFloat64 : ncclFloat32;
         CU_TRY(cudaEventRecord(c->ev_x, s));
         CU_TRY(cudaStreamWaitEvent(c->cs, c->ev_x, 0));
-        NCCL_TRY(ncclGroupStart());
-        for (size_t k = 0; k < A->recv_peer.size(); ++k)
-            NCCL_TRY(ncclRecv(xp + es * A->recv_off[k], A->recv_count[k], ty, (int)A->recv_peer[k], c->comm, c->cs));
-        for (size_t k = 0; k < A->send_peer.size(); ++k)
-            NCCL_TRY(ncclSend(xp + es * A->send_off[k], A->send_count[k], ty, (int)A->send_peer[k], c->comm, c->cs));
-        NCCL_TRY(ncclGroupEnd());
+        if (c->kind == crsd_comm_s::P2P) {
+            ST_TRY(crsd::p2p_exchange(A, c, xp));
+            launches += 2;
+        } else {
+            const ncclDataType_t ty = (A->H.dtype == CRSD_R64F) ? ncclFloat64 : ncclFloat32;
+            NCCL_TRY(ncclGroupStart());
+            for (size_t k = 0; k < A->recv_peer.size(); ++k)
+                NCCL_TRY(ncclRecv(xp + es * A->recv_off[k], A->recv_count[k], ty, (int)A->recv_peer[k], c->comm,
+                                  c->cs));
+            for (size_t k = 0; k < A->send_peer.size(); ++k)
+                NCCL_TRY(ncclSend(xp + es * A->send_off[k], A->send_count[k], ty, (int)A->send_peer[k], c->comm,
+                                  c->cs));
+            NCCL_TRY(ncclGroupEnd());
+        }
         CU_TRY(cudaEventRecord(c->ev_halo, c->cs));
     }
     st = crsd::run_lists(A, alpha, xbase, beta, y_local, (const int32_t *)A->d_list_interior, 0,

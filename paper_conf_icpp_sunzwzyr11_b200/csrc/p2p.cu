@@ -1,0 +1,211 @@
+// Peer-memory transport for the row-partitioned SpMV (BASELINE.json
+// north_star (3)): the x halo exchange and the
+// CG's scalar allreduce done by our own kernels through CUDA-IPC-mapped
+// device memory (NVLink / NVSwitch loads and stores between GPUs; plain HBM
+// when two ranks share one GPU), instead of NCCL calls.
+//
+// Each rank owns one symmetric region (cudaMalloc, exported with
+// cudaIpcGetMemHandle, opened by every peer):
+//
+//   [P2PFlags (4 KB)] [mailbox parity 0 (cap bytes)] [mailbox parity 1 (cap bytes)]
+//
+// Halo exchange of call e (epoch, device-resident, so the kernels can be
+// captured into a CUDA graph):
+//   p2p_send: wait until every peer I send to has consumed epoch e-2 from
+//             mailbox[e&1] (my flags.consumed[q] >= e-2); copy my send
+//             slices of x into mailbox[e&1]; last CTA: system fence, then
+//             flags.ready[me] = e in each receiver's region.
+//   p2p_recv: wait until every peer I receive from has published e (my
+//             flags.ready[q] >= e); copy the slices from the peers'
+//             mailbox[e&1] straight into the pads of x_padded; last CTA:
+//             system fence, flags.consumed[me] = e in each sender's region,
+//             my halo epoch = e.
+// Two parities let a sender run one call ahead of a slow receiver without
+// overwriting what the receiver has not read yet.
+//
+// Scalar allreduce (CG dots, n <= 4 doubles): one thread writes its values
+// into every peer's red[e&1][me] slot, fences, publishes red_ready[me] = e,
+// waits for red_ready[q] >= e from every peer and sums the W slots in rank
+// order 0..W-1 — the same operands in the same order on every rank, so every
+// rank gets the bit-identical result (deterministic, unlike a ring).
+//
+// Every wait is bounded (10 s on %globaltimer): on timeout the kernel sets
+// flags.err and returns instead of hanging the GPU; crsd_comm_check reports it.
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "crsd_p2p.h"
+
+namespace crsd {
+
+namespace {
+
+__device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t *p) {
+    uint64_t v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_sys(uint64_t *p, uint64_t v) {
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t globaltimer() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
+constexpr uint64_t kTimeoutNs = 10ull * 1000 * 1000 * 1000;
+
+// Spin until *p >= want (acquire, system scope). Returns false on timeout.
+__device__ bool wait_geq(const uint64_t *p, uint64_t want) {
+    if (ld_acquire_sys(p) >= want) return true;
+    const uint64_t t0 = globaltimer();
+    while (ld_acquire_sys(p) < want) {
+        __nanosleep(200);
+        if (globaltimer() - t0 > kTimeoutNs) return false;
+    }
+    return true;
+}
+
+// Byte copy of one item, split over the grid in 4-byte words (element sizes
+// are 4 or 8; slices start at arbitrary elements, so 16-B alignment is not
+// guaranteed and the halo is ~2 % of a rank's bytes).
+__device__ void copy_items(const P2PItem *items, int nitems, int64_t gtid, int64_t gsz) {
+    for (int k = 0; k < nitems; ++k) {
+        const uint32_t *s = (const uint32_t *)items[k].src;
+        uint32_t *d = (uint32_t *)items[k].dst;
+        const int64_t nw = items[k].bytes >> 2;
+        if ((((uintptr_t)s | (uintptr_t)d) & 15) == 0) {
+            const int64_t nv = nw >> 2;
+            const uint4 *s4 = (const uint4 *)s;
+            uint4 *d4 = (uint4 *)d;
+            for (int64_t i = gtid; i < nv; i += gsz) d4[i] = __ldcv(s4 + i);
+            for (int64_t i = (nv << 2) + gtid; i < nw; i += gsz) d[i] = __ldcv(s + i);
+        } else {
+            for (int64_t i = gtid; i < nw; i += gsz) d[i] = __ldcv(s + i);
+        }
+    }
+}
+
+// Grid arrival: returns true in exactly one CTA (the last to arrive), after
+// every CTA's writes are fenced at system scope.
+__device__ bool last_cta(uint32_t *counter) {
+    __shared__ bool last;
+    __threadfence_system();
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        const uint32_t prev = atomicAdd(counter, 1u);
+        last = (prev == gridDim.x - 1);
+        if (last) *counter = 0;  // reset for the next launch (stream-ordered)
+    }
+    __syncthreads();
+    if (last) __threadfence_system();
+    return last;
+}
+
+__global__ void p2p_send_kernel(P2PLaunch L) {
+    P2PFlags *me = L.local;
+    const uint64_t e = *(volatile uint64_t *)&me->halo_epoch + 1;
+    __shared__ int ok;
+    if (threadIdx.x == 0) {
+        ok = 1;
+        if (e > 2)
+            for (int k = 0; k < L.npeer; ++k)
+                if (!wait_geq(&me->consumed[L.peer[k]], e - 2)) {
+                    ok = 0;
+                    me->err = 1;
+                }
+    }
+    __syncthreads();
+    if (!ok) return;
+    const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
+    // mailbox parity: items carry parity-0 destinations; parity 1 is cap bytes further
+    P2PItem it[P2P_MAX_ITEMS];
+    const int64_t shift = (e & 1) ? L.cap : 0;
+    for (int k = 0; k < L.nitems; ++k) {
+        it[k] = L.items[k];
+        it[k].dst = (char *)it[k].dst + shift;
+    }
+    copy_items(it, L.nitems, gtid, gsz);
+    if (last_cta(&me->counter[0]) && threadIdx.x == 0)
+        for (int k = 0; k < L.npeer; ++k) st_release_sys(&L.peer_flags[k]->ready[L.rank], e);
+}
+
+__global__ void p2p_recv_kernel(P2PLaunch L) {
+    P2PFlags *me = L.local;
+    const uint64_t e = *(volatile uint64_t *)&me->halo_epoch + 1;
+    __shared__ int ok;
+    if (threadIdx.x == 0) {
+        ok = 1;
+        for (int k = 0; k < L.npeer; ++k)
+            if (!wait_geq(&me->ready[L.peer[k]], e)) {
+                ok = 0;
+                me->err = 2;
+            }
+    }
+    __syncthreads();
+    if (!ok) return;
+    const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
+    P2PItem it[P2P_MAX_ITEMS];
+    const int64_t shift = (e & 1) ? L.cap : 0;
+    for (int k = 0; k < L.nitems; ++k) {
+        it[k] = L.items[k];
+        it[k].src = (const char *)it[k].src + shift;
+    }
+    copy_items(it, L.nitems, gtid, gsz);
+    if (last_cta(&me->counter[1]) && threadIdx.x == 0) {
+        for (int k = 0; k < L.npeer; ++k) st_release_sys(&L.peer_flags[k]->consumed[L.rank], e);
+        me->halo_epoch = e;
+    }
+}
+
+__global__ void p2p_allreduce_kernel(P2PReduce R, double *val, int n) {
+    if (threadIdx.x != 0) return;
+    P2PFlags *me = R.local;
+    const uint64_t e = me->red_epoch + 1;
+    const int par = (int)(e & 1);
+    double v[P2P_MAX_RED];
+    for (int i = 0; i < n; ++i) v[i] = val[i];
+    for (int q = 0; q < R.world; ++q) {
+        if (q == R.rank) continue;
+        P2PFlags *pf = R.peer_flags[q];
+        for (int i = 0; i < n; ++i) *(volatile double *)&pf->red[par][R.rank][i] = v[i];
+    }
+    __threadfence_system();
+    for (int q = 0; q < R.world; ++q)
+        if (q != R.rank) st_release_sys(&R.peer_flags[q]->red_ready[R.rank], e);
+    bool ok = true;
+    for (int q = 0; q < R.world; ++q)
+        if (q != R.rank && !wait_geq(&me->red_ready[q], e)) ok = false;
+    if (!ok) {
+        me->err = 3;
+        me->red_epoch = e;
+        return;
+    }
+    double s[P2P_MAX_RED];
+    for (int i = 0; i < n; ++i) s[i] = 0.0;
+    for (int q = 0; q < R.world; ++q)
+        for (int i = 0; i < n; ++i) s[i] += (q == R.rank) ? v[i] : *(volatile double *)&me->red[par][q][i];
+    for (int i = 0; i < n; ++i) val[i] = s[i];
+    me->red_epoch = e;
+}
+
+}  // namespace
+
+int p2p_launch_send(const P2PLaunch &L, int grid, void *stream) {
+    p2p_send_kernel<<<grid, 256, 0, (cudaStream_t)stream>>>(L);
+    return (int)cudaGetLastError();
+}
+int p2p_launch_recv(const P2PLaunch &L, int grid, void *stream) {
+    p2p_recv_kernel<<<grid, 256, 0, (cudaStream_t)stream>>>(L);
+    return (int)cudaGetLastError();
+}
+int p2p_launch_allreduce(const P2PReduce &R, double *val, int n, void *stream) {
+    p2p_allreduce_kernel<<<1, 32, 0, (cudaStream_t)stream>>>(R, val, n);
+    return (int)cudaGetLastError();
+}
+
+}  // namespace crsd

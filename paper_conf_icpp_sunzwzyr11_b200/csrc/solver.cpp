@@ -120,7 +120,6 @@ crsd_status_t cg_impl(crsd_matrix_s *A, const T *b, T *x, int32_t max_iter, doub
 
     T *r = (T *)w.r, *q = (T *)w.q;
     T *p_own = (T *)w.p_pad + A->halo_lo;
-    const ncclDataType_t f64 = ncclFloat64;
     int launches = 0;
     auto spmv = [&](T al, T be, T *y) -> crsd_status_t {
         if (comm) {
@@ -153,7 +152,7 @@ crsd_status_t cg_impl(crsd_matrix_s *A, const T *b, T *x, int32_t max_iter, doub
     CU_TRY(cudaMemcpyAsync(p_own, r, es * n, cudaMemcpyDeviceToDevice, s));
     ST_TRY(kerr(cg_launch_dot<T>(r, r, n, w.st, CG_RR, false, grid, s), "cg_dot(r,r)"));
     ST_TRY(kerr(cg_launch_dot<T>(b, b, n, w.st, CG_BB, false, grid, s), "cg_dot(b,b)"));
-    if (comm) NC_TRY(ncclAllReduce(w.st->red + CG_RR, w.st->red + CG_RR, 2, f64, ncclSum, comm->comm, s));
+    if (comm) ST_TRY(comm_allreduce_f64(comm, w.st->red + CG_RR, 2, s));
     ST_TRY(kerr(cg_launch_init(w.st, s), "cg_init"));
 
     // One GPU with the JIT variant: (p, q) is fused into the SpMV epilogue
@@ -173,9 +172,9 @@ crsd_status_t cg_impl(crsd_matrix_s *A, const T *b, T *x, int32_t max_iter, doub
             ST_TRY(spmv(T(1), T(0), q));  // q = A p
             ST_TRY(kerr(cg_launch_dot<T>(p_own, q, n, w.st, CG_PQ, true, grid, s), "cg_dot(p,q)"));
         }
-        if (comm) NC_TRY(ncclAllReduce(w.st->red + CG_PQ, w.st->red + CG_PQ, 1, f64, ncclSum, comm->comm, s));
+        if (comm) ST_TRY(comm_allreduce_f64(comm, w.st->red + CG_PQ, 1, s));
         ST_TRY(kerr(cg_launch_update<T>(r, q, n, w.st, grid, s), "cg_update"));
-        if (comm) NC_TRY(ncclAllReduce(w.st->red + CG_RR, w.st->red + CG_RR, 1, f64, ncclSum, comm->comm, s));
+        if (comm) ST_TRY(comm_allreduce_f64(comm, w.st->red + CG_RR, 1, s));
         ST_TRY(kerr(cg_launch_pupdate<T>(p_own, r, x, n, w.st, grid, s), "cg_pupdate"));
         return CRSD_OK;
     };
@@ -187,9 +186,12 @@ crsd_status_t cg_impl(crsd_matrix_s *A, const T *b, T *x, int32_t max_iter, doub
     cudaGraphExec_t exec = nullptr;
     int graph_launches = 0;
     for (int64_t issued = 0; !done && issued < max_iter; issued += batch) {
-        if (!comm) {
+        // One batch of steps as a CUDA graph: one GPU, or the peer-memory
+        // transport (its exchange and allreduce kernels keep their epochs on
+        // the device, so a replay is a new exchange). NCCL calls are issued
+        // directly.
+        if (!comm || comm->kind == crsd_comm_s::P2P) {
             if (!exec) {
-                // one batch of steps as a CUDA graph (no NCCL inside: one GPU)
                 const int l0 = launches;
                 cudaGraph_t g;
                 CU_TRY(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
