@@ -306,8 +306,8 @@ def run_crsd(args):
     # plumbing uses gloo and the transport must be p2p). Not a scaling number.
     if args.share_gpu:
         local_rank = 0
-        if args.transport != "p2p":
-            raise SystemExit("--share-gpu needs --transport p2p")
+        if args.transport == "nccl":
+            raise SystemExit("--share-gpu needs the p2p transport")
     if world > 1:
         dist.init_process_group("gloo" if args.share_gpu else "nccl", init_method="env://")
         world = dist.get_world_size()
@@ -334,6 +334,7 @@ def run_crsd(args):
     ub = info["unique_bytes_beta0"]
     stream = torch.cuda.current_stream()
 
+    transport = None
     x_full = torch.from_numpy(np.random.default_rng(7 + rank).uniform(-1, 1, re - rb).astype(dt)).to(f"cuda:{dev}")
     comm = None
     if world > 1:
@@ -341,10 +342,18 @@ def run_crsd(args):
         xp = torch.zeros(lo + nloc + hi, dtype=tdt, device=f"cuda:{dev}")
         xp[lo : lo + nloc] = x_full
         y = torch.empty(nloc, dtype=tdt, device=f"cuda:{dev}")
-        if args.transport == "p2p":
-            comm = P2PComm(rank, world, dev, mailbox_bytes=max(1 << 20, 4 * (lo + hi) * es))
-        else:
+        comm = None
+        if args.transport in ("auto", "p2p"):
+            try:
+                comm = P2PComm(rank, world, dev, mailbox_bytes=max(1 << 20, 4 * (lo + hi) * es))
+                transport = "p2p"
+            except Exception as e:  # collective: every rank lands here together
+                if args.transport == "p2p":
+                    raise
+                print(f"[bench] peer-memory transport unavailable ({e}); using NCCL", file=sys.stderr)
+        if comm is None:
             comm = Comm(rank, world, dev)
+            transport = "nccl"
         A.dist_bind(comm)
 
         def step():
@@ -483,7 +492,7 @@ def run_crsd(args):
             "h2d_bytes_per_step": int((re - rb) * es) * world,
             "d2h_bytes_per_step": int((re - rb) * es) * world,
             "ms_per_step": round(te * 1e3, 4),
-            "path": f"per rank: H2D of the owned x slice, crsd_spmv_dist ({args.transport} halo + SpMV), D2H of the y slice; max over ranks",
+            "path": f"per rank: H2D of the owned x slice, crsd_spmv_dist ({transport} halo + SpMV), D2H of the y slice; max over ranks",
         }
     if rank != 0:
         if comm is not None:
@@ -522,7 +531,7 @@ def run_crsd(args):
             "scatter": info["nscatter"],
             "l2": f"inputs larger than L2 ({ub / 1e9:.2f} GB streamed per step vs {L2_BYTES / 2**20:.0f} MiB L2); no flush",
             "build_s": round(build_s, 2),
-            "parallelism": f"row-partitioned x{world}" + (f", {args.transport} halo" if world > 1 else "") + (", ranks share cuda:0 (functional only)" if args.share_gpu else ""),
+            "parallelism": f"row-partitioned x{world}" + (f", {transport} halo" if world > 1 else "") + (", ranks share cuda:0 (functional only)" if args.share_gpu else ""),
         },
         "hbm_gbs": round(ub_all / (ms * 1e-3) / 1e9, 1),
         "hbm_frac_of_peak": round(ub_all / (ms * 1e-3) / 1e9 / (peak * world), 4),
@@ -690,7 +699,7 @@ def main():
     ap.add_argument("--impl", default="crsd", choices=["crsd", "reference"])
     ap.add_argument("--workload", default="spmv", choices=["spmv", "cg"], help="cg: K steps of crsd_cg (one GPU)")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
-    ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p"], help="N>1 halo exchange: NCCL send/recv or the library's peer-memory kernels")
+    ap.add_argument("--transport", default="auto", choices=["auto", "nccl", "p2p"], help="N>1 halo exchange: the library's peer-memory kernels (p2p), NCCL send/recv, or auto (p2p if every rank can map its peers, else NCCL)")
     ap.add_argument("--share-gpu", action="store_true", help="N>1 ranks all on cuda:0 (functional check only; needs --transport p2p)")
     args = ap.parse_args()
     if args.warmup < 3:

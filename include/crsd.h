@@ -261,8 +261,9 @@ crsd_status_t crsd_comm_destroy(crsd_comm_t comm);
  * from the peer's mailbox straight into the pads of x_padded, then raises a
  * "consumed" flag so the sender may reuse that parity. Epochs live on the
  * device, so the exchange can be captured into a CUDA graph (crsd_cg does).
- * Every wait is bounded (10 s): on timeout the kernel returns and
- * crsd_comm_error reports a non-zero code instead of the GPU hanging.
+ * Every wait is bounded (30 s, env CRSD_P2P_TIMEOUT_S read at init): on
+ * timeout the kernel returns and crsd_comm_error reports a non-zero code
+ * instead of the GPU hanging.
  *
  *   crsd_comm_init_p2p(rank, world, device, mailbox_bytes, handle64, &c)
  *       mailbox_bytes: capacity per parity, >= the bytes this rank sends per

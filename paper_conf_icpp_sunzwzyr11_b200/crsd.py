@@ -522,8 +522,17 @@ class P2PComm:
         _check(lib.crsd_comm_init_p2p(rank, world, device, int(mailbox_bytes), _p(handle), ctypes.byref(h)))
         self._h = h
         allh = self._allgather(torch.from_numpy(handle.copy()))
-        _check(lib.crsd_comm_p2p_open(self._h, _p(np.ascontiguousarray(allh))))
-        dist.barrier(group=pg)
+        # open collectively: if any rank cannot map its peers (e.g. no IPC
+        # between the visible devices) every rank raises, none waits forever
+        err = None
+        try:
+            _check(lib.crsd_comm_p2p_open(self._h, _p(np.ascontiguousarray(allh))))
+        except CRSDError as e:
+            err = e
+        ok = self._allgather(torch.tensor([0 if err else 1], dtype=torch.int64))
+        if not ok.all():
+            self.close()
+            raise err if err is not None else CRSDError(1, "peer-memory open failed on another rank")
 
     def _allgather(self, t):
         import torch

@@ -21,7 +21,9 @@ struct crsd_comm_s {
     void *sym = nullptr;
     int64_t cap = 0;                  // bytes per mailbox parity
     std::vector<void *> peer_sym;     // world entries, nullptr for self / not opened
+    std::vector<int64_t> peer_cap;    // each peer's mailbox bytes per parity (read from its flags)
     bool opened = false;
+    uint64_t timeout_ns = 30ull * 1000 * 1000 * 1000;  // peer-memory waits (CRSD_P2P_TIMEOUT_S)
 };
 
 namespace crsd {

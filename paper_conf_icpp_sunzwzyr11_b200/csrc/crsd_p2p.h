@@ -20,6 +20,7 @@ struct P2PFlags {
     uint64_t red_epoch;   // own: last completed allreduce
     uint32_t counter[2];  // own: grid arrival counters (send, recv)
     uint32_t err;         // own: 0, or 1/2/3 = send/recv/allreduce wait timed out
+    int64_t cap;          // own mailbox bytes per parity (read by peers at open)
 };
 static_assert(sizeof(P2PFlags) <= P2P_FLAGS_BYTES, "P2PFlags too large");
 
@@ -27,6 +28,7 @@ struct P2PItem {
     const void *src;
     void *dst;
     int64_t bytes;
+    int64_t parity_shift;  // bytes from mailbox parity 0 to parity 1 of the mailbox this item touches
 };
 
 struct P2PLaunch {
@@ -34,7 +36,7 @@ struct P2PLaunch {
     P2PFlags *peer_flags[P2P_MAX_ITEMS];  // per distinct peer of this direction
     int32_t peer[P2P_MAX_ITEMS];
     int32_t npeer, nitems, rank, pad_;
-    int64_t cap;  // bytes per mailbox parity
+    uint64_t timeout_ns;
     P2PItem items[P2P_MAX_ITEMS];
 };
 
@@ -42,6 +44,7 @@ struct P2PReduce {
     P2PFlags *local;
     P2PFlags *peer_flags[P2P_MAX_WORLD];
     int32_t rank, world;
+    uint64_t timeout_ns;
 };
 
 int p2p_launch_send(const P2PLaunch &L, int grid, void *stream);

@@ -20,6 +20,7 @@
 
 #include <algorithm>
 #include <cstddef>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -172,9 +173,17 @@ crsd_status_t crsd_comm_init_p2p(int rank, int world, int device, int64_t mailbo
     c->device = device;
     c->cap = (mailbox_bytes + 255) / 256 * 256;
     c->peer_sym.assign(world, nullptr);
+    c->peer_cap.assign(world, 0);
+    if (const char *t = getenv("CRSD_P2P_TIMEOUT_S")) {
+        const double sec = atof(t);
+        if (sec > 0) c->timeout_ns = (uint64_t)(sec * 1e9);
+    }
     const size_t bytes = crsd::P2P_FLAGS_BYTES + 2 * c->cap;
     cudaError_t e = cudaMalloc(&c->sym, bytes);
     if (e == cudaSuccess) e = cudaMemset(c->sym, 0, crsd::P2P_FLAGS_BYTES);
+    if (e == cudaSuccess)
+        e = cudaMemcpy((char *)c->sym + offsetof(crsd::P2PFlags, cap), &c->cap, sizeof(int64_t),
+                       cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaIpcGetMemHandle((cudaIpcMemHandle_t *)ipc_handle64, c->sym);
     if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->cs, cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_x, cudaEventDisableTiming);
@@ -200,6 +209,9 @@ crsd_status_t crsd_comm_p2p_open(crsd_comm_t c, const void *ipc_handles) {
         void *p = nullptr;
         CU_TRY(cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess));
         c->peer_sym[q] = p;
+        // the peer wrote its capacity before exporting the handle
+        CU_TRY(cudaMemcpy(&c->peer_cap[q], (char *)p + offsetof(crsd::P2PFlags, cap), sizeof(int64_t),
+                          cudaMemcpyDeviceToHost));
     }
     c->opened = true;
     return CRSD_OK;
@@ -237,6 +249,7 @@ crsd_status_t comm_allreduce_f64(crsd_comm_s *c, double *dev, int n, cudaStream_
     R.local = (P2PFlags *)c->sym;
     R.rank = c->rank;
     R.world = c->world;
+    R.timeout_ns = c->timeout_ns;
     for (int q = 0; q < c->world; ++q) R.peer_flags[q] = (P2PFlags *)c->peer_sym[q];
     CU_TRY((cudaError_t)p2p_launch_allreduce(R, dev, n, s));
     return CRSD_OK;
@@ -319,7 +332,7 @@ crsd_status_t p2p_exchange(crsd_matrix_t A, crsd_comm_t c, char *xp) {
     auto fill = [&](P2PLaunch &L, const std::vector<int64_t> &peers) {
         L.local = (P2PFlags *)c->sym;
         L.rank = c->rank;
-        L.cap = c->cap;
+        L.timeout_ns = c->timeout_ns;
         L.npeer = 0;
         for (int64_t q : peers) {
             bool seen = false;
@@ -335,12 +348,12 @@ crsd_status_t p2p_exchange(crsd_matrix_t A, crsd_comm_t c, char *xp) {
     fill(S, A->send_peer);
     S.nitems = (int32_t)A->send_peer.size();
     for (int k = 0; k < S.nitems; ++k)
-        S.items[k] = P2PItem{xp + es * A->send_off[k], mb + A->send_mb_off[k], es * A->send_count[k]};
+        S.items[k] = P2PItem{xp + es * A->send_off[k], mb + A->send_mb_off[k], es * A->send_count[k], c->cap};
     fill(R, A->recv_peer);
     R.nitems = (int32_t)A->recv_peer.size();
     for (int k = 0; k < R.nitems; ++k)
         R.items[k] = P2PItem{(char *)c->peer_sym[A->recv_peer[k]] + P2P_FLAGS_BYTES + A->recv_mb_off[k],
-                             xp + es * A->recv_off[k], es * A->recv_count[k]};
+                             xp + es * A->recv_off[k], es * A->recv_count[k], c->peer_cap[A->recv_peer[k]]};
     const int grid = 32;
     CU_TRY((cudaError_t)p2p_launch_send(S, grid, c->cs));
     CU_TRY((cudaError_t)p2p_launch_recv(R, grid, c->cs));

@@ -7,7 +7,7 @@
 // Each rank owns one symmetric region (cudaMalloc, exported with
 // cudaIpcGetMemHandle, opened by every peer):
 //
-//   [P2PFlags (4 KB)] [mailbox parity 0 (cap bytes)] [mailbox parity 1 (cap bytes)]
+//   [P2PFlags (64 KB slot)] [mailbox parity 0 (cap bytes)] [mailbox parity 1 (cap bytes)]
 //
 // Halo exchange of call e (epoch, device-resident, so the kernels can be
 // captured into a CUDA graph):
@@ -29,8 +29,9 @@
 // order 0..W-1 — the same operands in the same order on every rank, so every
 // rank gets the bit-identical result (deterministic, unlike a ring).
 //
-// Every wait is bounded (10 s on %globaltimer): on timeout the kernel sets
-// flags.err and returns instead of hanging the GPU; crsd_comm_check reports it.
+// Every wait is bounded (%globaltimer; 30 s unless CRSD_P2P_TIMEOUT_S says
+// otherwise): on timeout the kernel sets flags.err and returns instead of
+// hanging the GPU; crsd_comm_error reports it.
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -55,15 +56,14 @@ __device__ __forceinline__ uint64_t globaltimer() {
     return t;
 }
 
-constexpr uint64_t kTimeoutNs = 10ull * 1000 * 1000 * 1000;
-
-// Spin until *p >= want (acquire, system scope). Returns false on timeout.
-__device__ bool wait_geq(const uint64_t *p, uint64_t want) {
+// Spin until *p >= want (acquire, system scope). Returns false after
+// timeout_ns (crsd_comm_s::timeout_ns, CRSD_P2P_TIMEOUT_S, default 30 s).
+__device__ bool wait_geq(const uint64_t *p, uint64_t want, uint64_t timeout_ns) {
     if (ld_acquire_sys(p) >= want) return true;
     const uint64_t t0 = globaltimer();
     while (ld_acquire_sys(p) < want) {
         __nanosleep(200);
-        if (globaltimer() - t0 > kTimeoutNs) return false;
+        if (globaltimer() - t0 > timeout_ns) return false;
     }
     return true;
 }
@@ -112,7 +112,7 @@ __global__ void p2p_send_kernel(P2PLaunch L) {
         ok = 1;
         if (e > 2)
             for (int k = 0; k < L.npeer; ++k)
-                if (!wait_geq(&me->consumed[L.peer[k]], e - 2)) {
+                if (!wait_geq(&me->consumed[L.peer[k]], e - 2, L.timeout_ns)) {
                     ok = 0;
                     me->err = 1;
                 }
@@ -121,12 +121,11 @@ __global__ void p2p_send_kernel(P2PLaunch L) {
     if (!ok) return;
     const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
-    // mailbox parity: items carry parity-0 destinations; parity 1 is cap bytes further
+    // mailbox parity: items carry parity-0 destinations; parity 1 is my cap further
     P2PItem it[P2P_MAX_ITEMS];
-    const int64_t shift = (e & 1) ? L.cap : 0;
     for (int k = 0; k < L.nitems; ++k) {
         it[k] = L.items[k];
-        it[k].dst = (char *)it[k].dst + shift;
+        if (e & 1) it[k].dst = (char *)it[k].dst + it[k].parity_shift;
     }
     copy_items(it, L.nitems, gtid, gsz);
     if (last_cta(&me->counter[0]) && threadIdx.x == 0)
@@ -140,7 +139,7 @@ __global__ void p2p_recv_kernel(P2PLaunch L) {
     if (threadIdx.x == 0) {
         ok = 1;
         for (int k = 0; k < L.npeer; ++k)
-            if (!wait_geq(&me->ready[L.peer[k]], e)) {
+            if (!wait_geq(&me->ready[L.peer[k]], e, L.timeout_ns)) {
                 ok = 0;
                 me->err = 2;
             }
@@ -149,11 +148,11 @@ __global__ void p2p_recv_kernel(P2PLaunch L) {
     if (!ok) return;
     const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
+    // parity 1 of the SENDER's mailbox is the sender's cap further (caps may differ per rank)
     P2PItem it[P2P_MAX_ITEMS];
-    const int64_t shift = (e & 1) ? L.cap : 0;
     for (int k = 0; k < L.nitems; ++k) {
         it[k] = L.items[k];
-        it[k].src = (const char *)it[k].src + shift;
+        if (e & 1) it[k].src = (const char *)it[k].src + it[k].parity_shift;
     }
     copy_items(it, L.nitems, gtid, gsz);
     if (last_cta(&me->counter[1]) && threadIdx.x == 0) {
@@ -179,7 +178,7 @@ __global__ void p2p_allreduce_kernel(P2PReduce R, double *val, int n) {
         if (q != R.rank) st_release_sys(&R.peer_flags[q]->red_ready[R.rank], e);
     bool ok = true;
     for (int q = 0; q < R.world; ++q)
-        if (q != R.rank && !wait_geq(&me->red_ready[q], e)) ok = false;
+        if (q != R.rank && !wait_geq(&me->red_ready[q], e, R.timeout_ns)) ok = false;
     if (!ok) {
         me->err = 3;
         me->red_epoch = e;

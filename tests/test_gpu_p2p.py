@@ -72,10 +72,26 @@ def _worker(rank, world, port, case, variant, q):
         bounds = partition_rows(n, mrows, world, np.bincount(a.row, minlength=n).astype(np.float64))
         rb, re = int(bounds[rank]), int(bounds[rank + 1])
         m = (a.row >= rb) & (a.row < re)
-        A = CRSDMatrix.from_coo(n, n, a.row[m], a.col[m], a.val[m], mrows=mrows, row_range=(rb, re), variant=variant, device=0)
-        comm = P2PComm(rank, world, 0, mailbox_bytes=1 << 20)
+        A = CRSDMatrix.from_coo(n, n, a.row[m], a.col[m], a.val[m], mrows=mrows, row_range=(rb, re), variant=0 if variant == "timeout" else variant, device=0)
+        if variant == "timeout":
+            os.environ["CRSD_P2P_TIMEOUT_S"] = "2"
+        # capacities differ per rank on purpose: a receiver must address the
+        # sender's parity-1 mailbox with the sender's capacity, not its own
+        comm = P2PComm(rank, world, 0, mailbox_bytes=(1 << 20) * (rank + 1))
         A.dist_bind(comm)
         lo, nloc, hi = A.x_layout()
+        if variant == "timeout":
+            # rank 1 never joins the exchange: rank 0's receive must give up
+            # after 2 s and report it instead of hanging the GPU
+            if rank == 0:
+                xd = torch.zeros(lo + nloc + hi, device="cuda:0", dtype=tdt)
+                yd = torch.empty(nloc, device="cuda:0", dtype=tdt)
+                A.spmv_dist(xd, yd, 1.0, 0.0, comm)
+                torch.cuda.synchronize()
+            dist.barrier()
+            out["err"] = comm.error()
+            comm.close()
+            return
         if case.startswith("cg"):
             rng = np.random.default_rng(11)
             b = rng.uniform(-1, 1, n)
@@ -126,7 +142,7 @@ def _worker(rank, world, port, case, variant, q):
         dist.destroy_process_group()
 
 
-def _run(case, world, variant=0):
+def _run(case, world, variant=0, check_err=True):
     import torch.multiprocessing as mp
 
     ctx = mp.get_context("spawn")
@@ -141,7 +157,7 @@ def _run(case, world, variant=0):
     res.sort(key=lambda r: r["rank"])
     for r in res:
         assert "exc" not in r, r["exc"]
-        assert r["err"] == 0, f"rank {r['rank']}: a peer-memory wait timed out (code {r['err']})"
+        assert not check_err or r["err"] == 0, f"rank {r['rank']}: a peer-memory wait timed out (code {r['err']})"
     return res
 
 
@@ -186,3 +202,11 @@ def test_p2p_cg(torch_cuda, case, world):
         assert r["rr_rel"] <= rr_tol, r
         assert r["x_rel"] <= x_tol, r
     assert len({r["rr_bits"] for r in res}) == 1
+
+
+def test_p2p_wait_is_bounded(torch_cuda):
+    """A peer that never arrives: the waiting kernel gives up after
+    CRSD_P2P_TIMEOUT_S (2 s here) and crsd_comm_error reports the receive
+    timeout (2) on that rank; the other rank saw nothing wrong."""
+    res = _run("c2", 2, "timeout", check_err=False)
+    assert res[0]["err"] == 2 and res[1]["err"] == 0, res
