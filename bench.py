@@ -58,7 +58,13 @@ def workload(cfg: str, dtype: str, world: int = 1, rank: int = 0):
     import gen
 
     dt = np.float64 if dtype == "f64" else np.float32
-    if cfg == "c2":
+    if cfg == "c1":
+        if world != 1:
+            raise SystemExit("config c1 is a single-GPU latency workload")
+        a = gen.config1()
+        N, rb, re = a.nrows, 0, a.nrows
+        desc = f"C1: 2D 5-point Laplacian 64x64 ({N:,} rows) + 16 scatter points, {dtype} (L2-resident: latency, L2 flushed before every step)"
+    elif cfg == "c2":
         n = 256
         nz = n * world
         N = n * n * nz
@@ -382,7 +388,12 @@ def run_crsd(args):
     t_all1 = torch.cuda.Event(enable_timing=True)
     t_all0.record(stream)
     launches = 0
+    # C1 fits in L2 (0.23 MB): flush it (write a buffer > L2) before every
+    # step, outside the step's events; the metric is then the per-step time
+    flush = torch.empty(2 * L2_BYTES // 4, dtype=torch.int32, device=f"cuda:{dev}") if args.config == "c1" else None
     for i in range(args.steps):
+        if flush is not None:
+            flush.zero_()
         ev[i][0].record(stream)
         step()
         ev[i][1].record(stream)
@@ -404,6 +415,8 @@ def run_crsd(args):
     else:
         nnz_all, ub_all = float(nnz_local), float(ub)
     ms = total_ms / args.steps
+    if flush is not None:
+        ms = statistics.median(step_ms)
     gflops = 2.0 * nnz_all / (ms * 1e-3) / 1e9
     kern_ms = statistics.mean(step_ms)
     peak, peak_src = measured_peaks()
@@ -529,10 +542,11 @@ def run_crsd(args):
             "instances": info["ninst"],
             "fills": info["nfills"],
             "scatter": info["nscatter"],
-            "l2": f"inputs larger than L2 ({ub / 1e9:.2f} GB streamed per step vs {L2_BYTES / 2**20:.0f} MiB L2); no flush",
+            "l2": (f"inputs larger than L2 ({ub / 1e9:.2f} GB streamed per step vs {L2_BYTES / 2**20:.0f} MiB L2); no flush" if flush is None else f"L2 flushed (252 MiB written) before every step; ms_per_step = median per-step CUDA-event time"),
             "build_s": round(build_s, 2),
             "parallelism": f"row-partitioned x{world}" + (f", {transport} halo" if world > 1 else "") + (", ranks share cuda:0 (functional only)" if args.share_gpu else ""),
         },
+        "latency_us": round(ms * 1e3, 2) if flush is not None else None,
         "hbm_gbs": round(ub_all / (ms * 1e-3) / 1e9, 1),
         "hbm_frac_of_peak": round(ub_all / (ms * 1e-3) / 1e9 / (peak * world), 4),
         "roofline": {
@@ -567,77 +581,136 @@ def run_crsd(args):
 def run_cg(args):
     """--workload cg: K steps of crsd_cg (textbook CG on the CRSD SpMV,
     SURVEY.md §8(f) NEXT 2) on the 7-point Dirichlet Laplacian of C2's grid
-    (256^3, SPD, exact values), one GPU. A step = SpMV + 3 vector kernels
-    (fused (p,q) with the JIT variant); its algorithmic bytes are the SpMV's
-    unique bytes + the vector traffic."""
+    (256^3 per GPU, SPD, exact values). A step = SpMV + 3 vector kernels; its
+    algorithmic bytes are the SpMV's unique bytes + the vector traffic
+    (DESIGN.md §13). N > 1: weak scaling, grid 256 x 256 x 256N cut into
+    z-slabs, halo exchange + allreduced dots through the communicator
+    (peer-memory kernels: graph batches; NCCL fallback: direct calls)."""
     import torch
+    import torch.distributed as dist
 
-    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, Comm, P2PComm
     from oracle import cg_ref
 
     import gen
 
-    if args.gpus != 1:
-        raise SystemExit("--workload cg runs on one GPU")
-    torch.cuda.set_device(0)
+    world = args.gpus
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = 0 if args.share_gpu else int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        dist.init_process_group("gloo" if args.share_gpu else "nccl", init_method="env://")
+        world, rank = dist.get_world_size(), dist.get_rank()
+    torch.cuda.set_device(local_rank)
+    dev = f"cuda:{local_rank}"
+    red_dev = "cpu" if args.share_gpu else dev
     dt = np.float64 if args.dtype == "f64" else np.float32
     tdt = torch.float64 if dt == np.float64 else torch.float32
     es = np.dtype(dt).itemsize
     n = 256
-    a = gen.spd_stencil_scatter((n, n, n), "7pt").astype(dt)
-    N = a.nrows
+    nloc = n * n * n
+    rb, re = rank * nloc, (rank + 1) * nloc
+    N = nloc * world
+    if world == 1:
+        a = gen.spd_stencil_scatter((n, n, n), "7pt").astype(dt)
+    else:
+        a = gen.stencil((n, n, n * world), "7pt", row_begin=rb, row_end=re)
+        a = gen.COO(N, N, a.row, a.col, a.val.astype(dt))
     kw = {"mrows": args.mrows} if args.mrows else {}
-    A = CRSDMatrix.from_coo(N, N, a.row, a.col, a.val, **kw)
+    if world > 1:
+        kw["row_range"] = (rb, re)
+    A = CRSDMatrix.from_coo(N, N, a.row, a.col, a.val, device=local_rank, **kw)
     info = A.info()
-    fused = info["variant"] == 4 and os.environ.get("CRSD_CG_FUSED_DOT", "0") != "0"
+    comm, transport = None, None
+    if world > 1:
+        lo, _, hi = A.x_layout()
+        if args.transport in ("auto", "p2p"):
+            try:
+                comm, transport = P2PComm(rank, world, local_rank, mailbox_bytes=max(1 << 20, 4 * (lo + hi) * es)), "p2p"
+            except Exception as e:
+                if args.transport == "p2p":
+                    raise
+                print(f"[bench] peer-memory transport unavailable ({e}); using NCCL", file=sys.stderr)
+        if comm is None:
+            comm, transport = Comm(rank, world, local_rank), "nccl"
+        A.dist_bind(comm)
+    fused = world == 1 and info["variant"] == 4 and os.environ.get("CRSD_CG_FUSED_DOT", "0") != "0"
     vec_passes = 8 if fused else 10
-    step_bytes = info["unique_bytes_beta0"] + vec_passes * N * es
-    step_flops = 2.0 * a.nnz + 10.0 * N
-    rng = np.random.default_rng(17)
-    bh = torch.from_numpy(rng.uniform(-1, 1, N).astype(dt)).pin_memory()
-    b = bh.to("cuda")
-    x = torch.zeros(N, dtype=tdt, device="cuda")
+    step_bytes = info["unique_bytes_beta0"] + vec_passes * nloc * es
+    nnz_local = int(a.nnz)
+    step_flops = 2.0 * nnz_local + 10.0 * nloc
+    rng = np.random.default_rng(17 + rank)
+    bh = torch.from_numpy(rng.uniform(-1, 1, nloc).astype(dt)).pin_memory()
+    b = bh.to(dev)
+    x = torch.zeros(nloc, dtype=tdt, device=dev)
     K = args.steps
     check = min(K, 50)
-    clocks = ClockSampler(0)
+    clocks = ClockSampler(local_rank)
     clocks.start()
     # warm-up: >= 300 steps (a short CG run otherwise starts below full clocks)
-    A.cg(b, x, max(args.warmup, 300), 0.0, check_every=check)
+    A.cg(b, x, max(args.warmup, 300), 0.0, check_every=check, comm=comm)
     torch.cuda.synchronize()
     x.zero_()
     s_ev, e_ev = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    if world > 1:
+        dist.barrier()
     torch.cuda.synchronize()
     s_ev.record()
-    res = A.cg(b, x, K, 0.0, check_every=check)
+    res = A.cg(b, x, K, 0.0, check_every=check, comm=comm)
     e_ev.record()
     e_ev.synchronize()
+    if world > 1:
+        dist.barrier()
     clk = clocks.stop()
     ms = s_ev.elapsed_time(e_ev) / res["iterations"]
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=red_dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
     peak, peak_src = measured_peaks()
     achieved = step_bytes / (ms * 1e-3) / 1e9
     # e2e: pinned b -> device, K steps, x -> pinned host, every solve
-    xh = torch.empty(N, dtype=tdt).pin_memory()
+    xh = torch.empty(nloc, dtype=tdt).pin_memory()
+    if world > 1:
+        dist.barrier()
     t0 = time.perf_counter()
-    bd = bh.to("cuda", non_blocking=True)
-    xd = torch.zeros(N, dtype=tdt, device="cuda")
-    r2 = A.cg(bd, xd, K, 0.0, check_every=check)
+    bd = bh.to(dev, non_blocking=True)
+    xd = torch.zeros(nloc, dtype=tdt, device=dev)
+    r2 = A.cg(bd, xd, K, 0.0, check_every=check, comm=comm)
     xh.copy_(xd, non_blocking=True)
     torch.cuda.synchronize()
     te = time.perf_counter() - t0
-    # cpu_baseline: the CG oracle as it stands on a bounded sample (64^3 grid)
-    ns = 64
-    a_s = gen.spd_stencil_scatter((ns, ns, ns), "7pt").astype(dt)
-    b_s = rng.uniform(-1, 1, a_s.nrows)
-    ks = 5
-    t0 = time.perf_counter()
-    cg_ref.cg(a_s, b_s, np.zeros(a_s.nrows), ks)
-    tc = (time.perf_counter() - t0) / ks
-    cpu_gflops = (2.0 * a_s.nnz + 10.0 * a_s.nrows) / tc / 1e9
+    if world > 1:
+        t = torch.tensor([te], dtype=torch.float64, device=red_dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        te = float(t.item())
+        if comm is not None and comm.error():
+            raise SystemExit("peer-memory wait timed out")
+    if rank != 0:
+        comm.close()
+        dist.destroy_process_group()
+        return
+    cpu = None
+    if world == 1:
+        # cpu_baseline: the CG oracle as it stands on a bounded sample (64^3 grid)
+        ns = 64
+        a_s = gen.spd_stencil_scatter((ns, ns, ns), "7pt").astype(dt)
+        b_s = rng.uniform(-1, 1, a_s.nrows)
+        ks = 5
+        t0 = time.perf_counter()
+        cg_ref.cg(a_s, b_s, np.zeros(a_s.nrows), ks)
+        tc = (time.perf_counter() - t0) / ks
+        cpu = {
+            "value": round((2.0 * a_s.nnz + 10.0 * a_s.nrows) / tc / 1e9, 4),
+            "unit": "GFLOP/s",
+            "cores": 1,
+            "kind": "oracle",
+            "sample": f"oracle/cg_ref.py (long-double definition SpMV + numpy dots), 7-pt 64^3 grid, {ks} steps",
+        }
     line = {
         "metric": "CG step GFLOP/s ((2*nnz + 10n) per step / t) with achieved HBM GB/s",
-        "value": round(step_flops / (ms * 1e-3) / 1e9, 3),
+        "value": round(world * step_flops / (ms * 1e-3) / 1e9, 3),
         "unit": "GFLOP/s",
-        "n_gpus": 1,
+        "n_gpus": world,
         "steps": res["iterations"],
         "warmup": max(args.warmup, 300),
         "ms_per_step": round(ms, 5),
@@ -647,12 +720,13 @@ def run_cg(args):
         "dtype": args.dtype,
         "data": "synthetic",
         "config": {
-            "workload": f"CG on the 7-point Dirichlet Laplacian 256^3 ({N:,} rows, SPD, exact values), rtol 0, {K} steps",
-            "nnz": int(a.nnz),
+            "workload": f"CG on the 7-point Dirichlet Laplacian 256x256x{256 * world} ({N:,} rows, SPD, exact values), rtol 0, {K} steps",
+            "nnz": int(nnz_local * world),
             "mrows": info["mrows"],
             "kernel_variant": {1: "ldg", 2: "tma", 3: "pipe", 4: "jit"}[info["variant"]],
             "fused_pq_dot": fused,
             "check_every": check,
+            "parallelism": f"row-partitioned x{world}" + (f", {transport} halo + allreduce" if world > 1 else "") + (", ranks share cuda:0 (functional only)" if args.share_gpu else ""),
             "l2": f"inputs larger than L2 ({step_bytes / 1e9:.2f} GB per step); no flush",
         },
         "roofline": {
@@ -666,15 +740,9 @@ def run_cg(args):
             "traffic": None,
             "algorithmic_bytes_per_step": int(step_bytes),
         },
-        "cpu_baseline": {
-            "value": round(cpu_gflops, 4),
-            "unit": "GFLOP/s",
-            "cores": 1,
-            "kind": "oracle",
-            "sample": f"oracle/cg_ref.py (long-double definition SpMV + numpy dots), 7-pt 64^3 grid, {ks} steps",
-        },
+        "cpu_baseline": cpu,
         "e2e": {
-            "value": round(step_flops * r2["iterations"] / te / 1e9, 3),
+            "value": round(world * step_flops * r2["iterations"] / te / 1e9, 3),
             "unit": "GFLOP/s",
             "h2d_bytes_per_step": int(N * es),
             "d2h_bytes_per_step": int(N * es),
@@ -685,6 +753,10 @@ def run_cg(args):
         "clocks": clk,
     }
     print(json.dumps(line), flush=True)
+    if comm is not None:
+        comm.close()
+    if world > 1:
+        dist.destroy_process_group()
 
 
 def main():
@@ -692,12 +764,12 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=20)
-    ap.add_argument("--config", default="c2", choices=["c2", "c3", "c3ns", "c4"])
+    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c3ns", "c4"])
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
     ap.add_argument("--mrows", type=int, default=0)
     ap.add_argument("--variant", default="auto", choices=["auto", "ldg", "tma", "pipe", "jit"])
     ap.add_argument("--impl", default="crsd", choices=["crsd", "reference"])
-    ap.add_argument("--workload", default="spmv", choices=["spmv", "cg"], help="cg: K steps of crsd_cg (one GPU)")
+    ap.add_argument("--workload", default="spmv", choices=["spmv", "cg"], help="cg: K steps of crsd_cg (N>1: row-partitioned, halo + allreduce)")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--transport", default="auto", choices=["auto", "nccl", "p2p"], help="N>1 halo exchange: the library's peer-memory kernels (p2p), NCCL send/recv, or auto (p2p if every rank can map its peers, else NCCL)")
     ap.add_argument("--share-gpu", action="store_true", help="N>1 ranks all on cuda:0 (functional check only; needs --transport p2p)")

@@ -80,7 +80,9 @@ crsd_status_t crsd_comm_init_rank(const void *id128, int rank, int world, int de
         delete c;
         return nccl_fail(r, "ncclCommInitRank");
     }
-    CU_TRY(cudaStreamCreateWithFlags(&c->cs, cudaStreamNonBlocking));
+    int prio_lo = 0, prio_hi = 0;
+    CU_TRY(cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi));
+    CU_TRY(cudaStreamCreateWithPriority(&c->cs, cudaStreamNonBlocking, prio_hi));
     CU_TRY(cudaEventCreateWithFlags(&c->ev_x, cudaEventDisableTiming));
     CU_TRY(cudaEventCreateWithFlags(&c->ev_halo, cudaEventDisableTiming));
     *out = c;
@@ -185,7 +187,9 @@ crsd_status_t crsd_comm_init_p2p(int rank, int world, int device, int64_t mailbo
         e = cudaMemcpy((char *)c->sym + offsetof(crsd::P2PFlags, cap), &c->cap, sizeof(int64_t),
                        cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaIpcGetMemHandle((cudaIpcMemHandle_t *)ipc_handle64, c->sym);
-    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&c->cs, cudaStreamNonBlocking);
+    int prio_lo = 0, prio_hi = 0;
+    if (e == cudaSuccess) e = cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+    if (e == cudaSuccess) e = cudaStreamCreateWithPriority(&c->cs, cudaStreamNonBlocking, prio_hi);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_x, cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&c->ev_halo, cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaDeviceSynchronize();
@@ -354,7 +358,9 @@ crsd_status_t p2p_exchange(crsd_matrix_t A, crsd_comm_t c, char *xp) {
     for (int k = 0; k < R.nitems; ++k)
         R.items[k] = P2PItem{(char *)c->peer_sym[A->recv_peer[k]] + P2P_FLAGS_BYTES + A->recv_mb_off[k],
                              xp + es * A->recv_off[k], es * A->recv_count[k], c->peer_cap[A->recv_peer[k]]};
-    const int grid = 32;
+    // a few CTAs suffice for the halo (~2 % of a rank's bytes); every CTA of
+    // p2p_recv holds an SM slot while it waits for the peers
+    static const int grid = getenv("CRSD_P2P_GRID") ? std::max(1, atoi(getenv("CRSD_P2P_GRID"))) : 16;
     CU_TRY((cudaError_t)p2p_launch_send(S, grid, c->cs));
     CU_TRY((cudaError_t)p2p_launch_recv(R, grid, c->cs));
     return CRSD_OK;
@@ -410,8 +416,15 @@ crsd_status_t crsd_spmv_dist(crsd_matrix_t A, const void *alpha, void *x_padded,
     cudaStream_t s = (cudaStream_t)stream;
     int launches = 0;
     crsd_status_t st;
-    if (c) {
-        CU_TRY(cudaEventRecord(c->ev_x, s));
+    // The exchange runs on the comm stream (created at the highest stream
+    // priority, so its CTAs take the next free SM slots ahead of queued SpMV
+    // CTAs). Default order: interior segments launched first, then the
+    // exchange — the interior fills the GPU at once and the small exchange
+    // kernels slot in as CTAs retire; CRSD_DIST_EXCHANGE_FIRST=1 launches the
+    // exchange first.
+    static const bool exchange_first = getenv("CRSD_DIST_EXCHANGE_FIRST") && atoi(getenv("CRSD_DIST_EXCHANGE_FIRST"));
+    if (c) CU_TRY(cudaEventRecord(c->ev_x, s));
+    auto exchange = [&]() -> crsd_status_t {
         CU_TRY(cudaStreamWaitEvent(c->cs, c->ev_x, 0));
         if (c->kind == crsd_comm_s::P2P) {
             ST_TRY(crsd::p2p_exchange(A, c, xp));
@@ -428,10 +441,13 @@ crsd_status_t crsd_spmv_dist(crsd_matrix_t A, const void *alpha, void *x_padded,
             NCCL_TRY(ncclGroupEnd());
         }
         CU_TRY(cudaEventRecord(c->ev_halo, c->cs));
-    }
+        return CRSD_OK;
+    };
+    if (c && exchange_first) ST_TRY(exchange());
     st = crsd::run_lists(A, alpha, xbase, beta, y_local, (const int32_t *)A->d_list_interior, 0,
                          (int64_t)A->list_interior.size(), stream, launches);
     if (st) return st;
+    if (c && !exchange_first) ST_TRY(exchange());
     if (c) CU_TRY(cudaStreamWaitEvent(s, c->ev_halo, 0));
     st = crsd::run_lists(A, alpha, xbase, beta, y_local, (const int32_t *)A->d_list_boundary, 0,
                          (int64_t)A->list_boundary.size(), stream, launches);
