@@ -517,16 +517,24 @@ class P2PComm:
 
         self.rank, self.world, self.device, self._pg = rank, world, device, pg
         self._h = None
-        handle = np.zeros(64, np.uint8)
+        # every step is collective: if any rank fails (no memory, no IPC
+        # between the visible devices, ...) every rank raises, none waits
+        # forever in the next exchange
+        handle = np.zeros(65, np.uint8)  # 64-byte IPC handle + ok flag
         h = ctypes.c_void_p()
-        _check(lib.crsd_comm_init_p2p(rank, world, device, int(mailbox_bytes), _p(handle), ctypes.byref(h)))
-        self._h = h
-        allh = self._allgather(torch.from_numpy(handle.copy()))
-        # open collectively: if any rank cannot map its peers (e.g. no IPC
-        # between the visible devices) every rank raises, none waits forever
         err = None
         try:
-            _check(lib.crsd_comm_p2p_open(self._h, _p(np.ascontiguousarray(allh))))
+            _check(lib.crsd_comm_init_p2p(rank, world, device, int(mailbox_bytes), _p(handle), ctypes.byref(h)))
+            self._h = h
+            handle[64] = 1
+        except CRSDError as e:
+            err = e
+        allh = self._allgather(torch.from_numpy(handle.copy()))
+        if not allh[:, 64].all():
+            self.close()
+            raise err if err is not None else CRSDError(1, "peer-memory init failed on another rank")
+        try:
+            _check(lib.crsd_comm_p2p_open(self._h, _p(np.ascontiguousarray(allh[:, :64]))))
         except CRSDError as e:
             err = e
         ok = self._allgather(torch.tensor([0 if err else 1], dtype=torch.int64))
