@@ -24,6 +24,9 @@ struct crsd_matrix_s {
     void *jit_function = nullptr;
     void *jitp_function = nullptr;  // persistent double-buffered form (crsd_jitp), or null
     bool jit_persist = false;       // launch the persistent form by default
+    // one-GPU launches of the one-shot codelets split into contiguous segment
+    // ranges of equal occupancy class: {seg_begin, seg_count, dynamic smem}
+    std::vector<std::vector<int64_t>> jit_ranges;
     int64_t tma_smem = 0;
     std::vector<int32_t> plan;
     int32_t last_launches = 0;

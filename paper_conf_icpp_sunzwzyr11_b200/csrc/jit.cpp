@@ -476,6 +476,54 @@ std::string jit_generate(const crsd_matrix_s *A) {
     return src + o.str();
 }
 
+// The kernel's dynamic shared memory is one number per launch, so a single
+// launch reserves the LARGEST pattern's staging for every CTA: on C4 the
+// 19-diagonal rows (56 KB, 4 CTAs/SM) set the reservation for the 9- and
+// 11-diagonal rows too, which alone would fit 7-8 CTAs per SM. Instances are
+// contiguous segment ranges, so the one-GPU launch is split into runs of
+// instances with the same occupancy class, each launched with its own
+// staging size (at most 8 launches; more runs, or one class, keep one
+// launch). CRSD_JIT_RANGES=0 disables the split.
+static void jit_plan_ranges(crsd_matrix_s *A) {
+    const HostCRSD &H = A->H;
+    A->jit_ranges.clear();
+    const int64_t nseg = H.nseg;
+    const int64_t nt = H.mrows / jit_q(A);
+    const bool off = getenv("CRSD_JIT_RANGES") && atoi(getenv("CRSD_JIT_RANGES")) == 0;
+    std::vector<int64_t> whole = {0, nseg, A->smem_bytes};
+    if (off || H.inst.empty()) {
+        A->jit_ranges.push_back(whole);
+        return;
+    }
+    auto staging = [&](const Instance &I) {
+        const int32_t *pl = A->plan.data() + A->segdesc[I.first_seg].plan_begin;
+        int64_t el = H.ndias(I.pattern) * H.mrows;
+        for (int w = 0; w < pl[0]; ++w) el += pl[3 + 2 * w];
+        return el * H.elem;
+    };
+    auto occupancy = [&](int64_t b) {
+        const int64_t per_cta = (b + 127) / 128 * 128 + 1024 + 128;  // + driver reserve + static smem
+        return std::min<int64_t>(2048 / nt, (228 * 1024) / per_cta);
+    };
+    std::vector<std::vector<int64_t>> runs;
+    int64_t run_occ = -1;
+    for (const Instance &I : H.inst) {
+        const int64_t b = staging(I), occ = occupancy(b);
+        if (!runs.empty() && occ == run_occ) {
+            runs.back()[1] = I.first_seg + I.nseg - runs.back()[0];
+            runs.back()[2] = std::max(runs.back()[2], b);
+        } else {
+            runs.push_back({I.first_seg, I.nseg, b});
+            run_occ = occ;
+        }
+    }
+    if (runs.size() <= 1 || runs.size() > 8) {
+        A->jit_ranges.push_back(whole);
+        return;
+    }
+    A->jit_ranges = runs;
+}
+
 crsd_status_t jit_build(crsd_matrix_s *A) {
     NvrtcApi &nv = nvrtc();
     if (!nv.ok) return fail(CRSD_ERR_UNSUPPORTED, "JIT variant: " + nv.err);
@@ -527,6 +575,7 @@ crsd_status_t jit_build(crsd_matrix_s *A) {
     A->jit_module = mod;
     A->jit_function = fn;
     A->jitp_function = fnp;
+    jit_plan_ranges(A);
     return CRSD_OK;
 }
 
@@ -576,6 +625,20 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
         void *pp[] = {&j, &stage};
         r = driver().launch((CUfunction)A->jitp_function, (unsigned)grid, 1, 1, nt, 1, 1, (unsigned)(2 * stage),
                             (CUstream)stream, pp, nullptr);
+    } else if (!s.seg_list && !s.dot_part && s.seg_begin == 0 && s.seg_count == A->H.nseg &&
+               A->jit_ranges.size() > 1) {
+        // whole matrix, one launch per occupancy class (jit_plan_ranges)
+        int n = 0;
+        for (const std::vector<int64_t> &rg : A->jit_ranges) {
+            j.seg_begin = rg[0];
+            j.seg_count = rg[1];
+            void *params[] = {&j};
+            r = driver().launch((CUfunction)A->jit_function, (unsigned)rg[1], 1, 1, nt, 1, 1, (unsigned)rg[2],
+                                (CUstream)stream, params, nullptr);
+            if (r != CUDA_SUCCESS) return -(int)cudaErrorLaunchFailure;
+            ++n;
+        }
+        return n;
     } else {
         void *params[] = {&j};
         r = driver().launch((CUfunction)A->jit_function, (unsigned)s.seg_count, 1, 1, nt, 1, 1,

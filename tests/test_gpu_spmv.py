@@ -107,6 +107,28 @@ def test_c4_reduced_parity(torch_cuda, variant):
     _parity(torch_cuda, gen.config4(n=300_000), np.float32, 1.0, 0.0, variant=variant)
 
 
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+@pytest.mark.parametrize("alpha,beta", [(1.0, 0.0), (-0.75, 0.5)])
+def test_jit_occupancy_ranges(torch_cuda, dt, alpha, beta, monkeypatch):
+    """C4's four row-range patterns (19 / 11 / 9 / 9 diagonals) need 4, 7 and
+    8 CTAs-per-SM staging sizes: the one-GPU JIT launch is split into one
+    launch per occupancy class (jit_plan_ranges), each with its own dynamic
+    shared memory. Every range must reproduce the oracle, with alpha/beta;
+    CRSD_JIT_RANGES=0 (one launch) must give the same bits."""
+    a = gen.config4(n=300_000)
+    A, _ = _parity(torch_cuda, a, dt, alpha, beta, variant=4, mrows=512)
+    assert A.last_launch_count() > 1
+    rng = np.random.default_rng(0)
+    x = rng.uniform(-1, 1, a.ncols).astype(dt)
+    y0 = rng.uniform(-1, 1, a.nrows).astype(dt)
+    y1 = _run(torch_cuda, A, x, alpha, beta, y0, a.nrows)
+    monkeypatch.setenv("CRSD_JIT_RANGES", "0")
+    B = _mat(a.astype(dt), variant=4, mrows=512)
+    y2 = _run(torch_cuda, B, x, alpha, beta, y0, a.nrows)
+    assert B.last_launch_count() == 1
+    assert np.array_equal(y1, y2)
+
+
 @pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("seed", range(12))
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
