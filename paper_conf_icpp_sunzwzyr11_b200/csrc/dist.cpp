@@ -444,8 +444,17 @@ crsd_status_t crsd_spmv_dist(crsd_matrix_t A, const void *alpha, void *x_padded,
         return CRSD_OK;
     };
     if (c && exchange_first) ST_TRY(exchange());
-    st = crsd::run_lists(A, alpha, xbase, beta, y_local, (const int32_t *)A->d_list_interior, 0,
-                         (int64_t)A->list_interior.size(), stream, launches);
+    // a contiguous interior (no scatter column reaching outside: C2, C4, C5)
+    // launches as a segment range: no per-CTA list load before the
+    // descriptor, and the JIT occupancy classes apply
+    const std::vector<int32_t> &li = A->list_interior;
+    const bool contig = !li.empty() && (int64_t)li.back() - li.front() + 1 == (int64_t)li.size();
+    if (contig)
+        st = crsd::run_lists(A, alpha, xbase, beta, y_local, nullptr, li.front(), (int64_t)li.size(), stream,
+                             launches);
+    else
+        st = crsd::run_lists(A, alpha, xbase, beta, y_local, (const int32_t *)A->d_list_interior, 0,
+                             (int64_t)li.size(), stream, launches);
     if (st) return st;
     if (c && !exchange_first) ST_TRY(exchange());
     if (c) CU_TRY(cudaStreamWaitEvent(s, c->ev_halo, 0));

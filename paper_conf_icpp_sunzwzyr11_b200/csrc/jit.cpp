@@ -482,8 +482,8 @@ std::string jit_generate(const crsd_matrix_s *A) {
 // 11-diagonal rows too, which alone would fit 7-8 CTAs per SM. Instances are
 // contiguous segment ranges, so the one-GPU launch is split into runs of
 // instances with the same occupancy class, each launched with its own
-// staging size (at most 8 launches; more runs, or one class, keep one
-// launch). CRSD_JIT_RANGES=0 disables the split.
+// staging size (runs shorter than 4 waves folded into their predecessor; at
+// most 8 launches, else one). CRSD_JIT_RANGES=0 disables the split.
 static void jit_plan_ranges(crsd_matrix_s *A) {
     const HostCRSD &H = A->H;
     A->jit_ranges.clear();
@@ -517,11 +517,56 @@ static void jit_plan_ranges(crsd_matrix_s *A) {
             run_occ = occ;
         }
     }
-    if (runs.size() <= 1 || runs.size() > 8) {
+    // runs shorter than a few waves (C3's idle sub-block B2 leaves ~48
+    // segments per z-plane) would be launches of mostly tail: fold each into
+    // a neighbour whose staging is at least as large (that neighbour's class
+    // does not change), then merge equal-class neighbours
+    const int64_t min_run = 4 * (int64_t)A->sm_count;
+    for (bool changed = true; changed;) {
+        changed = false;
+        for (size_t i = 0; i < runs.size(); ++i) {
+            if (runs[i][1] >= min_run) continue;
+            size_t into = runs.size();
+            if (i > 0 && runs[i - 1][2] >= runs[i][2]) into = i - 1;
+            else if (i + 1 < runs.size() && runs[i + 1][2] >= runs[i][2]) into = i + 1;
+            if (into == runs.size()) continue;
+            runs[into][0] = std::min(runs[into][0], runs[i][0]);
+            runs[into][1] += runs[i][1];
+            runs.erase(runs.begin() + i);
+            changed = true;
+            break;
+        }
+    }
+    std::vector<std::vector<int64_t>> merged;
+    for (const std::vector<int64_t> &r : runs) {
+        if (!merged.empty() && occupancy(merged.back()[2]) == occupancy(r[2])) {
+            merged.back()[1] += r[1];
+            merged.back()[2] = std::max(merged.back()[2], r[2]);
+        } else {
+            merged.push_back(r);
+        }
+    }
+    if (merged.size() <= 1 || merged.size() > 8) {
         A->jit_ranges.push_back(whole);
         return;
     }
-    A->jit_ranges = runs;
+    // Split only if it pays: the staging bytes that get extra CTA slots,
+    // sum over runs of nseg * staging * (1 - occ_whole / occ_run), must
+    // exceed what the extra launch boundaries cost, taken as one wave of the
+    // single launch each (sm_count * occ_whole CTAs of the largest staging).
+    // C4: ~2 GB gained vs 33 MB per boundary -> split; C3 (idle blocks B1 and
+    // B3 only, 16 % of the rows): ~32 MB vs ~130 MB -> one launch (measured:
+    // the split form ran at 0.90 against 0.96, sweep24b).
+    const int64_t occ_whole = occupancy(A->smem_bytes);
+    double gain = 0.0;
+    for (const std::vector<int64_t> &r : merged)
+        gain += (double)r[1] * (double)r[2] * (1.0 - (double)occ_whole / (double)occupancy(r[2]));
+    const double wave = (double)A->sm_count * (double)occ_whole * (double)A->smem_bytes;
+    if (gain <= (double)(merged.size() - 1) * wave) {
+        A->jit_ranges.push_back(whole);
+        return;
+    }
+    A->jit_ranges = merged;
 }
 
 crsd_status_t jit_build(crsd_matrix_s *A) {
@@ -625,15 +670,18 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
         void *pp[] = {&j, &stage};
         r = driver().launch((CUfunction)A->jitp_function, (unsigned)grid, 1, 1, nt, 1, 1, (unsigned)(2 * stage),
                             (CUstream)stream, pp, nullptr);
-    } else if (!s.seg_list && !s.dot_part && s.seg_begin == 0 && s.seg_count == A->H.nseg &&
-               A->jit_ranges.size() > 1) {
-        // whole matrix, one launch per occupancy class (jit_plan_ranges)
+    } else if (!s.seg_list && !s.dot_part && A->jit_ranges.size() > 1) {
+        // a segment range (the whole matrix, or a contiguous interior):
+        // one launch per occupancy class it meets (jit_plan_ranges)
         int n = 0;
+        const int64_t b0 = s.seg_begin, b1 = s.seg_begin + s.seg_count;
         for (const std::vector<int64_t> &rg : A->jit_ranges) {
-            j.seg_begin = rg[0];
-            j.seg_count = rg[1];
+            const int64_t lo = std::max(b0, rg[0]), hi = std::min(b1, rg[0] + rg[1]);
+            if (lo >= hi) continue;
+            j.seg_begin = lo;
+            j.seg_count = hi - lo;
             void *params[] = {&j};
-            r = driver().launch((CUfunction)A->jit_function, (unsigned)rg[1], 1, 1, nt, 1, 1, (unsigned)rg[2],
+            r = driver().launch((CUfunction)A->jit_function, (unsigned)(hi - lo), 1, 1, nt, 1, 1, (unsigned)rg[2],
                                 (CUstream)stream, params, nullptr);
             if (r != CUDA_SUCCESS) return -(int)cudaErrorLaunchFailure;
             ++n;

@@ -72,7 +72,7 @@ def main():
             ub = A.info()["unique_bytes_beta0"]
             ms = time_it(A, x, y)
             gbs = ub / (ms * 1e-3) / 1e9
-            print(json.dumps({"case": case, "mrows": mrows, "variant": name, "shape": sh, "ms": round(ms, 5), "GBps": round(gbs, 1), "frac": round(gbs / PEAK, 4), "smem": A.info()["smem_bytes"], "unique_bytes": ub}), flush=True)
+            print(json.dumps({"case": case, "mrows": mrows, "variant": name, "shape": sh, "ms": round(ms, 5), "GBps": round(gbs, 1), "frac": round(gbs / PEAK, 4), "smem": A.info()["smem_bytes"], "unique_bytes": ub, "launches": A.last_launch_count()}), flush=True)
             del A
         del a
         torch.cuda.empty_cache()

@@ -107,15 +107,16 @@ def test_c4_reduced_parity(torch_cuda, variant):
     _parity(torch_cuda, gen.config4(n=300_000), np.float32, 1.0, 0.0, variant=variant)
 
 
-@pytest.mark.parametrize("dt", [np.float64, np.float32])
-@pytest.mark.parametrize("alpha,beta", [(1.0, 0.0), (-0.75, 0.5)])
+@pytest.mark.parametrize("dt,alpha,beta", [(np.float32, 1.0, 0.0), (np.float64, -0.75, 0.5)])
 def test_jit_occupancy_ranges(torch_cuda, dt, alpha, beta, monkeypatch):
     """C4's four row-range patterns (19 / 11 / 9 / 9 diagonals) need 4, 7 and
     8 CTAs-per-SM staging sizes: the one-GPU JIT launch is split into one
     launch per occupancy class (jit_plan_ranges), each with its own dynamic
     shared memory. Every range must reproduce the oracle, with alpha/beta;
     CRSD_JIT_RANGES=0 (one launch) must give the same bits."""
-    a = gen.config4(n=300_000)
+    # 8M rows: long enough that the split pays under jit_plan_ranges' rule
+    # (the gain grows with the rows, the boundary cost is one wave)
+    a = gen.config4(n=8_000_000)
     A, _ = _parity(torch_cuda, a, dt, alpha, beta, variant=4, mrows=512)
     assert A.last_launch_count() > 1
     rng = np.random.default_rng(0)
@@ -293,7 +294,7 @@ def test_dist_compute_single_gpu(torch_cuda, case, world, variant):
         torch.cuda.synchronize()
         err = coo.parity_error(yd.cpu().numpy(), yref[rb:re], scale[rb:re])
         assert err <= TOL[dt], (r, err)
-        assert A.last_launch_count() in (1, 2)
+        assert 1 <= A.last_launch_count() <= 10  # interior range (one launch per occupancy class) + boundary list
 
 
 def test_nccl_comm_world1(torch_cuda):
