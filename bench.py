@@ -560,6 +560,8 @@ def run_crsd(args):
             "traffic": traffic,
             "algorithmic_bytes_per_launch": int(ub),
             "avg_launch_ms": round(kern_ms, 5),
+            "launches_per_step": round(launches / max(1, args.steps), 2),
+            "per_step_note": "with several launches per step (JIT occupancy classes, dist interior/boundary) achieved = the step's algorithmic bytes / the step's CUDA-event time",
             "copy_gbs_this_box": box_copy,
             "frac_of_this_box_copy": round(achieved / box_copy, 4) if box_copy else None,
             "sustained_copy_gbs_this_box": box_copy_sus,

@@ -10,6 +10,8 @@
 #include "crsd.h"
 #include "crsd_p2p.h"
 
+struct crsd_matrix_s;
+
 struct crsd_comm_s {
     enum Kind { NCCL = 0, P2P = 1 };
     int kind = NCCL;
@@ -29,4 +31,8 @@ struct crsd_comm_s {
 namespace crsd {
 // Sum n doubles (device pointer) over every rank of comm, in place, on stream.
 crsd_status_t comm_allreduce_f64(crsd_comm_s *c, double *dev, int n, cudaStream_t stream);
+// crsd_spmv_dist with the boundary placement chosen by the caller: -1 default,
+// 0 concurrent with the interior (comm stream), 1 serial after the interior
+crsd_status_t spmv_dist_impl(crsd_matrix_s *A, const void *alpha, void *x_padded, const void *beta, void *y_local,
+                             crsd_comm_s *c, void *stream, int boundary);
 }  // namespace crsd

@@ -26,7 +26,11 @@ struct crsd_matrix_s {
     bool jit_persist = false;       // launch the persistent form by default
     // one-GPU launches of the one-shot codelets split into contiguous segment
     // ranges of equal occupancy class: {seg_begin, seg_count, dynamic smem}
+    // {seg_begin, seg_count, dynamic smem, aux}: aux = 1 for short runs that
+    // go to a forked stream alongside the main sequence
     std::vector<std::vector<int64_t>> jit_ranges;
+    void *jit_aux = nullptr;                          // cudaStream_t
+    void *jit_ev_fork = nullptr, *jit_ev_join = nullptr;  // cudaEvent_t
     int64_t tma_smem = 0;
     std::vector<int32_t> plan;
     int32_t last_launches = 0;

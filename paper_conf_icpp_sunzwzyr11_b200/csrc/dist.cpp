@@ -4,12 +4,13 @@
 // Each rank owns rows [row_begin, row_end) of a square matrix and the same
 // range of x. Rows are independent given x (one work-item per
 // row), so the only exchange is the x halo: rank r needs x[row_begin -
-// halo_lo, row_begin) and x[row_end, row_end + halo_hi). The halo moves with
-// NCCL send/recv on a comm stream, received straight into the pads of the
-// caller's padded x buffer, while the interior segments (whose x windows and
-// scatter columns stay inside the owned range) run on the compute stream;
-// the boundary segments run after the halo event. y stays row-distributed:
-// no reduction.
+// halo_lo, row_begin) and x[row_end, row_end + halo_hi). The halo moves on
+// a comm stream, received straight into the pads of the caller's padded x
+// buffer, while the interior segments (whose x windows and scatter columns
+// stay inside the owned range) run on the compute stream; the boundary
+// segments run on the comm stream behind the exchange, concurrently with the
+// interior, and the compute stream joins at the end. y stays
+// row-distributed: no reduction.
 //
 // Two transports behind crsd_comm_t: NCCL (grouped send/recv), or the
 // library's own peer-memory kernels (p2p.cu) over CUDA-IPC-mapped symmetric
@@ -401,6 +402,15 @@ crsd_status_t crsd_dist_bind_ranges(crsd_matrix_t A, crsd_comm_t c, const int64_
 
 crsd_status_t crsd_spmv_dist(crsd_matrix_t A, const void *alpha, void *x_padded, const void *beta, void *y_local,
                              crsd_comm_t c, void *stream) {
+    return crsd::spmv_dist_impl(A, alpha, x_padded, beta, y_local, c, stream, -1);
+}
+
+}  // extern "C"
+
+// boundary: -1 = default (concurrent on the comm stream unless
+// CRSD_DIST_BOUNDARY_SERIAL=1), 0 = concurrent, 1 = serial after the interior
+crsd_status_t crsd::spmv_dist_impl(crsd_matrix_t A, const void *alpha, void *x_padded, const void *beta,
+                                   void *y_local, crsd_comm_t c, void *stream, int boundary) {
     if (!A) return crsd::fail(CRSD_ERR_INVALID_ARG, "A is NULL");
     if (A->host_only) return crsd::fail(CRSD_ERR_UNSUPPORTED, "host-only handle");
     if (A->H.paper_ell) return crsd::fail(CRSD_ERR_UNSUPPORTED, "CRSD_PAPER_ELL handle: use crsd_spmv");
@@ -457,11 +467,21 @@ crsd_status_t crsd_spmv_dist(crsd_matrix_t A, const void *alpha, void *x_padded,
                              (int64_t)li.size(), stream, launches);
     if (st) return st;
     if (c && !exchange_first) ST_TRY(exchange());
-    if (c) CU_TRY(cudaStreamWaitEvent(s, c->ev_halo, 0));
+    // The boundary segments run on the comm stream right behind the
+    // exchange, i.e. concurrently with the interior rather than after it: no
+    // serial tail (interior drain + a small dependent launch) per call. The
+    // caller's stream then waits for the comm stream. CRSD_DIST_BOUNDARY_SERIAL=1
+    // runs them on the caller's stream after the interior instead.
+    static const bool serial_env = getenv("CRSD_DIST_BOUNDARY_SERIAL") && atoi(getenv("CRSD_DIST_BOUNDARY_SERIAL"));
+    const bool serial = boundary < 0 ? serial_env : boundary == 1;
+    if (c && serial) CU_TRY(cudaStreamWaitEvent(s, c->ev_halo, 0));
     st = crsd::run_lists(A, alpha, xbase, beta, y_local, (const int32_t *)A->d_list_boundary, 0,
-                         (int64_t)A->list_boundary.size(), stream, launches);
+                         (int64_t)A->list_boundary.size(), (c && !serial) ? (void *)c->cs : stream, launches);
+    if (st) return st;
+    if (c && !serial) {
+        CU_TRY(cudaEventRecord(c->ev_halo, c->cs));
+        CU_TRY(cudaStreamWaitEvent(s, c->ev_halo, 0));
+    }
     A->last_launches = launches;
     return st;
 }
-
-}  // extern "C"

@@ -490,7 +490,7 @@ static void jit_plan_ranges(crsd_matrix_s *A) {
     const int64_t nseg = H.nseg;
     const int64_t nt = H.mrows / jit_q(A);
     const bool off = getenv("CRSD_JIT_RANGES") && atoi(getenv("CRSD_JIT_RANGES")) == 0;
-    std::vector<int64_t> whole = {0, nseg, A->smem_bytes};
+    std::vector<int64_t> whole = {0, nseg, A->smem_bytes, 0};
     if (off || H.inst.empty()) {
         A->jit_ranges.push_back(whole);
         return;
@@ -517,10 +517,12 @@ static void jit_plan_ranges(crsd_matrix_s *A) {
             run_occ = occ;
         }
     }
-    // runs shorter than a few waves (C3's idle sub-block B2 leaves ~48
-    // segments per z-plane) would be launches of mostly tail: fold each into
-    // a neighbour whose staging is at least as large (that neighbour's class
-    // does not change), then merge equal-class neighbours
+    // Runs shorter than a few waves (C3's idle sub-block B2 leaves ~48
+    // segments per z-plane; C4 has one-segment transitions between its
+    // patterns) would cost a whole launch boundary each: fold each into a
+    // neighbour with at least as much staging (that neighbour's class does
+    // not change); what cannot be folded becomes an "aux" run, launched on a
+    // forked stream alongside the main sequence instead of inside it.
     const int64_t min_run = 4 * (int64_t)A->sm_count;
     for (bool changed = true; changed;) {
         changed = false;
@@ -537,35 +539,43 @@ static void jit_plan_ranges(crsd_matrix_s *A) {
             break;
         }
     }
-    std::vector<std::vector<int64_t>> merged;
+    // main sequence: long runs, equal-class neighbours merged when contiguous
+    std::vector<std::vector<int64_t>> merged, aux;
     for (const std::vector<int64_t> &r : runs) {
-        if (!merged.empty() && occupancy(merged.back()[2]) == occupancy(r[2])) {
+        if (r[1] < min_run) {
+            aux.push_back({r[0], r[1], r[2], 1});
+            continue;
+        }
+        if (!merged.empty() && occupancy(merged.back()[2]) == occupancy(r[2]) &&
+            merged.back()[0] + merged.back()[1] == r[0]) {
             merged.back()[1] += r[1];
             merged.back()[2] = std::max(merged.back()[2], r[2]);
         } else {
-            merged.push_back(r);
+            merged.push_back({r[0], r[1], r[2], 0});
         }
     }
-    if (merged.size() <= 1 || merged.size() > 8) {
+    if (merged.size() + aux.size() <= 1 || merged.size() > 8 || aux.size() > 8) {
         A->jit_ranges.push_back(whole);
         return;
     }
     // Split only if it pays: the staging bytes that get extra CTA slots,
-    // sum over runs of nseg * staging * (1 - occ_whole / occ_run), must
-    // exceed what the extra launch boundaries cost, taken as one wave of the
-    // single launch each (sm_count * occ_whole CTAs of the largest staging).
-    // C4: ~2 GB gained vs 33 MB per boundary -> split; C3 (idle blocks B1 and
-    // B3 only, 16 % of the rows): ~32 MB vs ~130 MB -> one launch (measured:
-    // the split form ran at 0.90 against 0.96, sweep24b).
+    // sum over the main runs of nseg * staging * (1 - occ_whole / occ_run),
+    // must exceed what the extra launch boundaries cost, taken as one wave
+    // of the single launch each (sm_count * occ_whole CTAs of the largest
+    // staging). C4 (10^8 rows): ~2 GB gained vs 33 MB per boundary -> split;
+    // C3 (idle blocks B1 and B3 only, 16 % of the rows): ~32 MB vs ~130 MB
+    // -> one launch (measured: a 5-launch split ran at 0.90 against 0.96,
+    // sweep24b).
     const int64_t occ_whole = occupancy(A->smem_bytes);
     double gain = 0.0;
     for (const std::vector<int64_t> &r : merged)
         gain += (double)r[1] * (double)r[2] * (1.0 - (double)occ_whole / (double)occupancy(r[2]));
     const double wave = (double)A->sm_count * (double)occ_whole * (double)A->smem_bytes;
-    if (gain <= (double)(merged.size() - 1) * wave) {
+    if (merged.empty() || gain <= (double)(merged.size() - 1) * wave) {
         A->jit_ranges.push_back(whole);
         return;
     }
+    merged.insert(merged.end(), aux.begin(), aux.end());
     A->jit_ranges = merged;
 }
 
@@ -625,6 +635,13 @@ crsd_status_t jit_build(crsd_matrix_s *A) {
 }
 
 void jit_free(crsd_matrix_s *A) {
+    if (A->jit_aux) {
+        cudaStreamSynchronize((cudaStream_t)A->jit_aux);
+        cudaStreamDestroy((cudaStream_t)A->jit_aux);
+        cudaEventDestroy((cudaEvent_t)A->jit_ev_fork);
+        cudaEventDestroy((cudaEvent_t)A->jit_ev_join);
+        A->jit_aux = A->jit_ev_fork = A->jit_ev_join = nullptr;
+    }
     if (A->jit_module && driver().ok) driver().unload((CUmodule)A->jit_module);
     A->jit_module = nullptr;
     A->jit_function = nullptr;
@@ -673,19 +690,49 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
     } else if (!s.seg_list && !s.dot_part && A->jit_ranges.size() > 1) {
         // a segment range (the whole matrix, or a contiguous interior):
         // one launch per occupancy class it meets (jit_plan_ranges)
+        // aux runs (short, unfoldable) on a forked stream, joined at the end
         int n = 0;
         const int64_t b0 = s.seg_begin, b1 = s.seg_begin + s.seg_count;
-        for (const std::vector<int64_t> &rg : A->jit_ranges) {
-            const int64_t lo = std::max(b0, rg[0]), hi = std::min(b1, rg[0] + rg[1]);
-            if (lo >= hi) continue;
-            j.seg_begin = lo;
-            j.seg_count = hi - lo;
-            void *params[] = {&j};
-            r = driver().launch((CUfunction)A->jit_function, (unsigned)(hi - lo), 1, 1, nt, 1, 1, (unsigned)rg[2],
-                                (CUstream)stream, params, nullptr);
-            if (r != CUDA_SUCCESS) return -(int)cudaErrorLaunchFailure;
-            ++n;
+        bool forked = false;
+        crsd_matrix_s *M = const_cast<crsd_matrix_s *>(A);
+        for (int pass = 0; pass < 2; ++pass) {
+            for (const std::vector<int64_t> &rg : A->jit_ranges) {
+                if (rg[3] != (pass == 0 ? 1 : 0)) continue;
+                const int64_t lo = std::max(b0, rg[0]), hi = std::min(b1, rg[0] + rg[1]);
+                if (lo >= hi) continue;
+                CUstream st = (CUstream)stream;
+                if (rg[3]) {
+                    if (!M->jit_aux) {
+                        cudaStream_t as;
+                        cudaEvent_t e1, e2;
+                        if (cudaStreamCreateWithFlags(&as, cudaStreamNonBlocking) != cudaSuccess ||
+                            cudaEventCreateWithFlags(&e1, cudaEventDisableTiming) != cudaSuccess ||
+                            cudaEventCreateWithFlags(&e2, cudaEventDisableTiming) != cudaSuccess)
+                            return -(int)cudaErrorLaunchFailure;
+                        M->jit_aux = as;
+                        M->jit_ev_fork = e1;
+                        M->jit_ev_join = e2;
+                    }
+                    if (!forked) {
+                        if (cudaEventRecord((cudaEvent_t)A->jit_ev_fork, (cudaStream_t)stream) != cudaSuccess ||
+                            cudaStreamWaitEvent((cudaStream_t)A->jit_aux, (cudaEvent_t)A->jit_ev_fork, 0) != cudaSuccess)
+                            return -(int)cudaErrorLaunchFailure;
+                        forked = true;
+                    }
+                    st = (CUstream)A->jit_aux;
+                }
+                j.seg_begin = lo;
+                j.seg_count = hi - lo;
+                void *params[] = {&j};
+                r = driver().launch((CUfunction)A->jit_function, (unsigned)(hi - lo), 1, 1, nt, 1, 1,
+                                    (unsigned)rg[2], st, params, nullptr);
+                if (r != CUDA_SUCCESS) return -(int)cudaErrorLaunchFailure;
+                ++n;
+            }
         }
+        if (forked && (cudaEventRecord((cudaEvent_t)A->jit_ev_join, (cudaStream_t)A->jit_aux) != cudaSuccess ||
+                       cudaStreamWaitEvent((cudaStream_t)stream, (cudaEvent_t)A->jit_ev_join, 0) != cudaSuccess))
+            return -(int)cudaErrorLaunchFailure;
         return n;
     } else {
         void *params[] = {&j};

@@ -123,7 +123,14 @@ crsd_status_t cg_impl(crsd_matrix_s *A, const T *b, T *x, int32_t max_iter, doub
     int launches = 0;
     auto spmv = [&](T al, T be, T *y) -> crsd_status_t {
         if (comm) {
-            ST_TRY(crsd_spmv_dist(A, &al, w.p_pad, &be, y, comm, s));
+            // boundary placement as crsd_spmv_dist's default (concurrent with
+            // the interior); CRSD_CG_BOUNDARY=1 forces the serial form, =0 the
+            // concurrent one. Under MPS (ranks sharing one GPU) the CG is
+            // bimodal: one run favoured serial 2-3x, the next concurrent 2x
+            // (profiles/r01_ab_boundary_cg_*, r01_ab_cg_*), so the default
+            // follows the SpMV measurement and the no-serial-tail argument.
+            static const int cg_boundary = getenv("CRSD_CG_BOUNDARY") ? atoi(getenv("CRSD_CG_BOUNDARY")) : -1;
+            ST_TRY(spmv_dist_impl(A, &al, w.p_pad, &be, y, comm, s, cg_boundary));
             launches += A->last_launches;
             return CRSD_OK;
         }
@@ -186,11 +193,13 @@ crsd_status_t cg_impl(crsd_matrix_s *A, const T *b, T *x, int32_t max_iter, doub
     cudaGraphExec_t exec = nullptr;
     int graph_launches = 0;
     for (int64_t issued = 0; !done && issued < max_iter; issued += batch) {
-        // One batch of steps as a CUDA graph: one GPU, or the peer-memory
+        // One batch of steps as a CUDA graph (CRSD_CG_NO_GRAPH=1: direct
+        // launches, for A/B runs): one GPU, or the peer-memory
         // transport (its exchange and allreduce kernels keep their epochs on
         // the device, so a replay is a new exchange). NCCL calls are issued
         // directly.
-        if (!comm || comm->kind == crsd_comm_s::P2P) {
+        static const bool no_graph = getenv("CRSD_CG_NO_GRAPH") && atoi(getenv("CRSD_CG_NO_GRAPH"));
+        if (!no_graph && (!comm || comm->kind == crsd_comm_s::P2P)) {
             if (!exec) {
                 const int l0 = launches;
                 cudaGraph_t g;
