@@ -471,6 +471,23 @@ static crsd_status_t e2e_setup(crsd_matrix_s *A) {
     A->e2e_seg.resize(nch + 1);
     A->e2e_xcut.resize(nch + 1);
     for (int c = 0; c <= nch; ++c) A->e2e_seg[c] = nseg * c / nch;
+    // CRSD_E2E_RAMP=1: the first and last three chunks 1/8, 1/4, 1/2 of the
+    // others (shorter pipeline fill before the first y copy and drain after
+    // the last kernel)
+    if (getenv("CRSD_E2E_RAMP") && atoi(getenv("CRSD_E2E_RAMP")) && nch >= 8) {
+        std::vector<double> w(nch, 1.0);
+        const double r[3] = {0.125, 0.25, 0.5};
+        for (int k = 0; k < 3; ++k) w[k] = w[nch - 1 - k] = r[k];
+        double tot = 0.0;
+        for (double v : w) tot += v;
+        double acc = 0.0;
+        for (int c = 0; c < nch; ++c) {
+            A->e2e_seg[c] = std::min<int64_t>(nseg, (int64_t)(nseg * acc / tot));
+            acc += w[c];
+        }
+        A->e2e_seg[nch] = nseg;
+        for (int c = 1; c <= nch; ++c) A->e2e_seg[c] = std::max(A->e2e_seg[c], A->e2e_seg[c - 1]);
+    }
     // highest x element each row chunk reads (vector windows, clipped to
     // [0, ncols) as the guarded edge path does, and scatter columns)
     std::vector<int64_t> hi(nch, 0);

@@ -482,14 +482,16 @@ std::string jit_generate(const crsd_matrix_s *A) {
 // 11-diagonal rows too, which alone would fit 7-8 CTAs per SM. Instances are
 // contiguous segment ranges, so the one-GPU launch is split into runs of
 // instances with the same occupancy class, each launched with its own
-// staging size (runs shorter than 4 waves folded into their predecessor; at
-// most 8 launches, else one). CRSD_JIT_RANGES=0 disables the split.
+// staging size (see below for when it pays). CRSD_JIT_RANGES=0 disables
+// the split, =2 forces it at every class change (tests, sanitizer runs).
 static void jit_plan_ranges(crsd_matrix_s *A) {
     const HostCRSD &H = A->H;
     A->jit_ranges.clear();
     const int64_t nseg = H.nseg;
     const int64_t nt = H.mrows / jit_q(A);
-    const bool off = getenv("CRSD_JIT_RANGES") && atoi(getenv("CRSD_JIT_RANGES")) == 0;
+    const int mode = getenv("CRSD_JIT_RANGES") ? atoi(getenv("CRSD_JIT_RANGES")) : 1;
+    const bool off = mode == 0;
+    const bool force = mode == 2;  // testing: split at every class change, no folding, no cost rule
     std::vector<int64_t> whole = {0, nseg, A->smem_bytes, 0};
     if (off || H.inst.empty()) {
         A->jit_ranges.push_back(whole);
@@ -523,7 +525,7 @@ static void jit_plan_ranges(crsd_matrix_s *A) {
     // neighbour with at least as much staging (that neighbour's class does
     // not change); what cannot be folded becomes an "aux" run, launched on a
     // forked stream alongside the main sequence instead of inside it.
-    const int64_t min_run = 4 * (int64_t)A->sm_count;
+    const int64_t min_run = force ? 0 : 4 * (int64_t)A->sm_count;
     for (bool changed = true; changed;) {
         changed = false;
         for (size_t i = 0; i < runs.size(); ++i) {
@@ -554,7 +556,8 @@ static void jit_plan_ranges(crsd_matrix_s *A) {
             merged.push_back({r[0], r[1], r[2], 0});
         }
     }
-    if (merged.size() + aux.size() <= 1 || merged.size() > 8 || aux.size() > 8) {
+    const size_t max_runs = force ? 64 : 8;
+    if (merged.size() + aux.size() <= 1 || merged.size() > max_runs || aux.size() > max_runs) {
         A->jit_ranges.push_back(whole);
         return;
     }
@@ -571,7 +574,7 @@ static void jit_plan_ranges(crsd_matrix_s *A) {
     for (const std::vector<int64_t> &r : merged)
         gain += (double)r[1] * (double)r[2] * (1.0 - (double)occ_whole / (double)occupancy(r[2]));
     const double wave = (double)A->sm_count * (double)occ_whole * (double)A->smem_bytes;
-    if (merged.empty() || gain <= (double)(merged.size() - 1) * wave) {
+    if (merged.empty() || (!force && gain <= (double)(merged.size() - 1) * wave)) {
         A->jit_ranges.push_back(whole);
         return;
     }
