@@ -579,6 +579,150 @@ def run_crsd(args):
         dist.destroy_process_group()
 
 
+# ---------------------------------------------------------------- C5 on one GPU
+def run_c5(args):
+    """--config c5: BASELINE config 5 (3D 7-point Laplacian 768^3, fp64,
+    452,984,832 rows, 3.17e9 nonzeros, 32.6 GB) on ONE B200. The host builds
+    it as 8 row blocks (the 8-GPU partition: a single 3.17e9-entry COO would
+    need ~76 GB of host RAM plus the builder's copies), every block resident
+    on the GPU; the blocks share one global x (each block's padded x is a
+    view of it: its halos are the neighbours' owned x, no exchange) and write
+    disjoint slices of one global y. A step = the 8 blocks' crsd_spmv_dist
+    calls (comm = NULL)."""
+    import torch
+
+    import gen
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, partition_rows
+
+    if args.gpus != 1:
+        raise SystemExit("--config c5 here is the one-GPU form; N > 1 uses c2 weak or c4 strong scaling")
+    if args.dtype != "f64":
+        raise SystemExit("config c5 is fp64")
+    torch.cuda.set_device(0)
+    nn, nb = 768, 8
+    N = nn**3
+    bounds = partition_rows(N, 256, nb)
+    blocks, t0 = [], time.perf_counter()
+    cpu = None
+    for k in range(nb):
+        rb, re = int(bounds[k]), int(bounds[k + 1])
+        a = gen.config5(n=nn, values="exact", row_begin=rb, row_end=re)
+        if k == 0 and not args.no_cpu:
+            cpu = cpu_baseline(gen.COO(re, N, a.row, a.col, a.val))
+            cpu["sample"] += " (block 0 of the 8 host-built blocks)"
+        A = CRSDMatrix.from_coo(N, N, a.row, a.col, a.val, row_range=(rb, re), device=0)
+        del a
+        blocks.append((rb, re, A))
+    build_s = time.perf_counter() - t0
+    pad = (max(max(A.x_layout()[0], A.x_layout()[2]) for _, _, A in blocks) + 64 + 3) // 4 * 4  # keeps views 16-B aligned
+    x_ext = torch.zeros(N + 2 * pad, dtype=torch.float64, device="cuda:0")
+    x = x_ext[pad : pad + N]
+    x.copy_(torch.from_numpy(np.random.default_rng(7).uniform(-1, 1, N)))
+    y = torch.empty(N, dtype=torch.float64, device="cuda:0")
+    views = []
+    for rb, re, A in blocks:
+        lo, nloc, hi = A.x_layout()
+        views.append((A, x_ext[pad + rb - lo : pad + re + hi], y[rb:re]))
+    infos = [A.info() for _, _, A in blocks]
+    nnz = sum(i["nnz"] for i in infos)
+    ub = sum(i["unique_bytes_beta0"] for i in infos)
+
+    def step():
+        for A, xv, yv in views:
+            A.spmv_dist(xv, yv, 1.0, 0.0, None)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    stream = torch.cuda.current_stream()
+    clocks = ClockSampler(0)
+    clocks.start()
+    time.sleep(0.3)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    launches = 0
+    torch.cuda.synchronize()
+    for i in range(args.steps):
+        ev[i][0].record(stream)
+        step()
+        ev[i][1].record(stream)
+        launches += sum(A.last_launch_count() for A, _, _ in views)
+    torch.cuda.synchronize()
+    clk = clocks.stop()
+    step_ms = [s_.elapsed_time(e_) for s_, e_ in ev]
+    ms = statistics.mean(step_ms)
+    peak, peak_src = measured_peaks()
+    achieved = ub / (ms * 1e-3) / 1e9
+    # e2e: pinned host x -> device, the 8 block SpMVs, device y -> pinned host
+    xh = torch.from_numpy(np.random.default_rng(7).uniform(-1, 1, N)).pin_memory()
+    yh = torch.empty(N, dtype=torch.float64).pin_memory()
+
+    def e2e_step():
+        x.copy_(xh, non_blocking=True)
+        step()
+        yh.copy_(y, non_blocking=True)
+        torch.cuda.synchronize()
+
+    e2e_step()
+    ke = 5
+    t0 = time.perf_counter()
+    for _ in range(ke):
+        e2e_step()
+    te = (time.perf_counter() - t0) / ke
+    line = {
+        "metric": "CRSD SpMV GFLOP/s (2*nnz/t) with achieved HBM GB/s (% of B200 peak)",
+        "value": round(2.0 * nnz / (ms * 1e-3) / 1e9, 3),
+        "unit": "GFLOP/s",
+        "n_gpus": 1,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": round(ms, 5),
+        "higher_is_better": True,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": "f64",
+        "data": "synthetic",
+        "config": {
+            "workload": f"C5: 3D 7-point Laplacian 768^3 ({N:,} rows), fp64, one B200, 8 resident row blocks sharing one x",
+            "nnz": int(nnz),
+            "mrows": infos[0]["mrows"],
+            "kernel_variant": {1: "ldg", 2: "tma", 3: "pipe", 4: "jit"}[infos[0]["variant"]],
+            "alpha": 1.0,
+            "beta": 0.0,
+            "device_bytes": int(sum(i["device_bytes"] for i in infos) + (N + 2 * pad + N) * 8),
+            "l2": f"inputs larger than L2 ({ub / 1e9:.1f} GB per step); no flush",
+            "build_s": round(build_s, 1),
+            "parallelism": "one GPU",
+        },
+        "hbm_gbs": round(achieved, 1),
+        "hbm_frac_of_peak": round(achieved / peak, 4),
+        "roofline": {
+            "bound": "hbm",
+            "kernel": "crsd_jit (8 blocks x interior range + boundary list per step)",
+            "achieved": round(achieved, 1),
+            "peak": peak,
+            "peak_source": peak_src,
+            "unit": "GB/s",
+            "frac": round(achieved / peak, 4),
+            "traffic": None,
+            "algorithmic_bytes_per_step": int(ub),
+            "avg_step_ms": round(ms, 5),
+            "launches_per_step": round(launches / max(1, args.steps), 2),
+        },
+        "cpu_baseline": cpu,
+        "e2e": {
+            "value": round(2.0 * nnz / te / 1e9, 3),
+            "unit": "GFLOP/s",
+            "h2d_bytes_per_step": int(N * 8),
+            "d2h_bytes_per_step": int(N * 8),
+            "ms_per_step": round(te * 1e3, 3),
+            "path": "pinned H2D of x (3.6 GB), the 8 block SpMVs, pinned D2H of y (3.6 GB); serial",
+        },
+        "gpu_launches": int(launches),
+        "clocks": clk,
+    }
+    print(json.dumps(line), flush=True)
+
+
 # ---------------------------------------------------------------- CG workload
 def run_cg(args):
     """--workload cg: K steps of crsd_cg (textbook CG on the CRSD SpMV,
@@ -766,7 +910,7 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=20)
-    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c3ns", "c4"])
+    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c3ns", "c4", "c5"])
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
     ap.add_argument("--mrows", type=int, default=0)
     ap.add_argument("--variant", default="auto", choices=["auto", "ldg", "tma", "pipe", "jit"])
@@ -782,6 +926,8 @@ def main():
         run_reference(args)
     elif args.workload == "cg":
         run_cg(args)
+    elif args.config == "c5":
+        run_c5(args)
     else:
         run_crsd(args)
 

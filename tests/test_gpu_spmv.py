@@ -335,6 +335,49 @@ def test_nccl_comm_world1(torch_cuda):
         dist.destroy_process_group()
 
 
+def test_p2p_comm_world1_nccl_plumbing(torch_cuda):
+    """The peer-memory communicator bootstrapped over an NCCL process group
+    (the plumbing bench.py uses under torchrun: handles and range table
+    allgathered as CUDA tensors), one rank: empty halo plan, exchange kernels
+    with no peers, allreduce of one rank, CG graph batches through it."""
+    import os
+    import socket
+
+    import torch.distributed as dist
+
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, P2PComm
+
+    torch = torch_cuda
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK="0", WORLD_SIZE="1")
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda:0"))
+    try:
+        a = gen.config2(n=40)
+        n = a.nrows
+        A = CRSDMatrix.from_coo(n, n, a.row, a.col, a.val, row_range=(0, n), device=0)
+        comm = P2PComm(0, 1, 0)
+        A.dist_bind(comm)
+        x = np.random.default_rng(4).uniform(-1, 1, n)
+        xd = torch.from_numpy(x).to("cuda:0")
+        yd = torch.full((n,), float("nan"), device="cuda:0", dtype=torch.float64)
+        for _ in range(3):
+            A.spmv_dist(xd, yd, 1.0, 0.0, comm)
+        torch.cuda.synchronize()
+        yref, scale = coo.coo_spmv(n, n, a.row, a.col, a.val, x)
+        assert coo.parity_error(yd.cpu().numpy(), yref, scale) <= 1e-12
+        v = torch.tensor([1.5, -2.0], dtype=torch.float64, device="cuda:0")
+        comm.allreduce_f64(v)
+        torch.cuda.synchronize()
+        assert v.cpu().tolist() == [1.5, -2.0]
+        assert comm.error() == 0
+        comm.close()
+    finally:
+        dist.destroy_process_group()
+
+
 def _host_ram_gb():
     try:
         import psutil
