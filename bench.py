@@ -78,10 +78,30 @@ def workload(cfg: str, dtype: str, world: int = 1, rank: int = 0):
         a = gen.config3(scatter_frac=0.001 if cfg == "c3" else 0.0)
         N, rb, re = a.nrows, 0, a.nrows
         desc = f"C3: 3D 27-point FVM stencil 192^3 with idle sub-blocks and 0.1% scatter points ({N:,} rows), {dtype}"
+    elif cfg == "c5":
+        # N > 1: each rank builds its row block of C5 (strong scaling; N = 1 runs run_c5)
+        from paper_conf_icpp_sunzwzyr11_b200 import partition_rows
+
+        nn = 768
+        N = nn**3
+        bounds = partition_rows(N, 256, world)
+        rb, re = int(bounds[rank]), int(bounds[rank + 1])
+        a = gen.config5(n=nn, values="exact", row_begin=rb, row_end=re)
+        desc = f"C5: 3D 7-point Laplacian 768^3 ({N:,} rows), fp64, row-partitioned"
     elif cfg == "c4":
         n = 100_000_000
-        bounds = np.linspace(0, n, world + 1).astype(np.int64) // 512 * 512
-        bounds[-1] = n
+        if world == 1:
+            bounds = np.array([0, n], np.int64)
+        else:
+            # byte-balanced row blocks (equal rows give
+            # max/avg 1.52 on C4): weight per row = its stored diagonals + x + y
+            from paper_conf_icpp_sunzwzyr11_b200 import partition_rows
+
+            w = np.empty(n, np.float64)
+            for r0, r1, offs in gen.matrices.c4_ranges(n):
+                w[r0:r1] = len(offs) + 2
+            bounds = partition_rows(n, 512, world, w)
+            del w
         rb, re = int(bounds[rank]), int(bounds[rank + 1])
         a = gen.config4(n=n, row_begin=rb, row_end=re)
         N = n
@@ -527,7 +547,7 @@ def run_crsd(args):
         "warmup": args.warmup,
         "ms_per_step": round(ms, 5),
         "higher_is_better": True,
-        "scaling": "weak",
+        "scaling": "strong" if args.config in ("c4", "c5") else "weak",
         "vs_baseline": None,
         "dtype": args.dtype,
         "data": "synthetic",
@@ -595,7 +615,7 @@ def run_c5(args):
     from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, partition_rows
 
     if args.gpus != 1:
-        raise SystemExit("--config c5 here is the one-GPU form; N > 1 uses c2 weak or c4 strong scaling")
+        raise SystemExit("run_c5 is the one-GPU form")
     if args.dtype != "f64":
         raise SystemExit("config c5 is fp64")
     torch.cuda.set_device(0)
@@ -926,7 +946,7 @@ def main():
         run_reference(args)
     elif args.workload == "cg":
         run_cg(args)
-    elif args.config == "c5":
+    elif args.config == "c5" and args.gpus == 1:
         run_c5(args)
     else:
         run_crsd(args)
