@@ -302,8 +302,13 @@ crsd_status_t crsd_dist_ranges(crsd_matrix_t A_local, int64_t *ranges4);
 crsd_status_t crsd_dist_bind(crsd_matrix_t A_local, crsd_comm_t comm, void *stream);
 
 /*
- * Distributed SpMV: halo exchange (NCCL send/recv on the comm stream) in
- * parallel with the interior segments, then the boundary segments.
+ * Distributed SpMV (north_star (3)): the halo exchange
+ * (peer-memory kernels or NCCL send/recv, per the communicator) runs on the
+ * communicator's highest-priority stream in parallel with the interior
+ * segments on `stream`; the boundary segments follow the exchange on the
+ * comm stream (concurrently with the interior; CRSD_DIST_BOUNDARY_SERIAL=1
+ * runs them on `stream` after it) and `stream` joins the comm stream before
+ * the call returns, so y_local is complete in `stream` order. Asynchronous.
  *   x_padded  DEVICE dtype[halo_lo+n_local+halo_hi], 16-byte aligned; the
  *             owned part must be written before the call (stream-ordered);
  *             the halo parts are overwritten.
