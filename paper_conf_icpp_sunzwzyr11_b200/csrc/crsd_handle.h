@@ -29,8 +29,9 @@ struct crsd_matrix_s {
     // {seg_begin, seg_count, dynamic smem, aux}: aux = 1 for short runs that
     // go to a forked stream alongside the main sequence
     std::vector<std::vector<int64_t>> jit_ranges;
-    void *jit_aux = nullptr;                          // cudaStream_t
-    void *jit_ev_fork = nullptr, *jit_ev_join = nullptr;  // cudaEvent_t
+    std::vector<void *> jit_pool;       // cudaStream_t: forked streams for range launches
+    std::vector<void *> jit_ev_join;    // cudaEvent_t, one per pool stream
+    void *jit_ev_fork = nullptr;        // cudaEvent_t
     int64_t tma_smem = 0;
     std::vector<int32_t> plan;
     int32_t last_launches = 0;

@@ -476,6 +476,13 @@ std::string jit_generate(const crsd_matrix_s *A) {
     return src + o.str();
 }
 
+// Range launches on forked streams, concurrently (default), or one after the
+// other on the caller's stream (CRSD_JIT_CONCURRENT=0).
+static bool jit_concurrent() {
+    static const bool v = !(getenv("CRSD_JIT_CONCURRENT") && atoi(getenv("CRSD_JIT_CONCURRENT")) == 0);
+    return v;
+}
+
 // The kernel's dynamic shared memory is one number per launch, so a single
 // launch reserves the LARGEST pattern's staging for every CTA: on C4 the
 // 19-diagonal rows (56 KB, 4 CTAs/SM) set the reservation for the 9- and
@@ -574,7 +581,15 @@ static void jit_plan_ranges(crsd_matrix_s *A) {
     for (const std::vector<int64_t> &r : merged)
         gain += (double)r[1] * (double)r[2] * (1.0 - (double)occ_whole / (double)occupancy(r[2]));
     const double wave = (double)A->sm_count * (double)occ_whole * (double)A->smem_bytes;
-    if (merged.empty() || (!force && gain <= (double)(merged.size() - 1) * wave)) {
+    // Concurrent range launches have no boundary to drain; what a split still
+    // costs (launches that do not fully overlap, fork/join) is taken as 3/4
+    // of a wave in total -- a threshold fitted to sweep25, not derived: C3
+    // f64 gains 30.6 MB against a 33.2 MB wave (0.92) and measured 0.960 ->
+    // 1.005 split; C3 f32 (mrows 256) gains 15.3 MB against 33.3 MB (0.46)
+    // and measured 1.044 -> 0.992 split, so it stays one launch; C4 f32
+    // gains ~2 GB (1.013 -> 1.022 against the sequential split).
+    const double boundary_cost = jit_concurrent() ? 0.75 * wave : (double)(merged.size() - 1) * wave;
+    if (merged.empty() || (!force && gain <= boundary_cost)) {
         A->jit_ranges.push_back(whole);
         return;
     }
@@ -638,13 +653,15 @@ crsd_status_t jit_build(crsd_matrix_s *A) {
 }
 
 void jit_free(crsd_matrix_s *A) {
-    if (A->jit_aux) {
-        cudaStreamSynchronize((cudaStream_t)A->jit_aux);
-        cudaStreamDestroy((cudaStream_t)A->jit_aux);
-        cudaEventDestroy((cudaEvent_t)A->jit_ev_fork);
-        cudaEventDestroy((cudaEvent_t)A->jit_ev_join);
-        A->jit_aux = A->jit_ev_fork = A->jit_ev_join = nullptr;
+    for (size_t i = 0; i < A->jit_pool.size(); ++i) {
+        cudaStreamSynchronize((cudaStream_t)A->jit_pool[i]);
+        cudaStreamDestroy((cudaStream_t)A->jit_pool[i]);
+        cudaEventDestroy((cudaEvent_t)A->jit_ev_join[i]);
     }
+    if (A->jit_ev_fork) cudaEventDestroy((cudaEvent_t)A->jit_ev_fork);
+    A->jit_pool.clear();
+    A->jit_ev_join.clear();
+    A->jit_ev_fork = nullptr;
     if (A->jit_module && driver().ok) driver().unload((CUmodule)A->jit_module);
     A->jit_module = nullptr;
     A->jit_function = nullptr;
@@ -693,36 +710,53 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
     } else if (!s.seg_list && !s.dot_part && A->jit_ranges.size() > 1) {
         // a segment range (the whole matrix, or a contiguous interior):
         // one launch per occupancy class it meets (jit_plan_ranges)
-        // aux runs (short, unfoldable) on a forked stream, joined at the end
+        // Concurrent mode (default, CRSD_JIT_CONCURRENT=1): every range on
+        // its own forked stream, all joined at the end -- the ranges are
+        // independent (disjoint rows), so no launch waits for another's
+        // drain and their tails overlap. Sequential mode (=0): the main
+        // ranges one after the other on `stream`, aux runs on a forked stream.
         int n = 0;
         const int64_t b0 = s.seg_begin, b1 = s.seg_begin + s.seg_count;
-        bool forked = false;
         crsd_matrix_s *M = const_cast<crsd_matrix_s *>(A);
+        const bool conc = jit_concurrent();
+        int next = 0, nstreams = 0;
+        auto pool_stream = [&](int i) -> CUstream {
+            while ((int)M->jit_pool.size() <= i) {
+                cudaStream_t as;
+                cudaEvent_t ej;
+                if (cudaStreamCreateWithFlags(&as, cudaStreamNonBlocking) != cudaSuccess ||
+                    cudaEventCreateWithFlags(&ej, cudaEventDisableTiming) != cudaSuccess)
+                    return nullptr;
+                M->jit_pool.push_back(as);
+                M->jit_ev_join.push_back(ej);
+            }
+            if (!M->jit_ev_fork) {
+                cudaEvent_t ef;
+                if (cudaEventCreateWithFlags(&ef, cudaEventDisableTiming) != cudaSuccess) return nullptr;
+                M->jit_ev_fork = ef;
+            }
+            if (i == 0 && cudaEventRecord((cudaEvent_t)M->jit_ev_fork, (cudaStream_t)stream) != cudaSuccess)
+                return nullptr;
+            if (cudaStreamWaitEvent((cudaStream_t)M->jit_pool[i], (cudaEvent_t)M->jit_ev_fork, 0) != cudaSuccess)
+                return nullptr;
+            return (CUstream)M->jit_pool[i];
+        };
         for (int pass = 0; pass < 2; ++pass) {
             for (const std::vector<int64_t> &rg : A->jit_ranges) {
                 if (rg[3] != (pass == 0 ? 1 : 0)) continue;
                 const int64_t lo = std::max(b0, rg[0]), hi = std::min(b1, rg[0] + rg[1]);
                 if (lo >= hi) continue;
                 CUstream st = (CUstream)stream;
-                if (rg[3]) {
-                    if (!M->jit_aux) {
-                        cudaStream_t as;
-                        cudaEvent_t e1, e2;
-                        if (cudaStreamCreateWithFlags(&as, cudaStreamNonBlocking) != cudaSuccess ||
-                            cudaEventCreateWithFlags(&e1, cudaEventDisableTiming) != cudaSuccess ||
-                            cudaEventCreateWithFlags(&e2, cudaEventDisableTiming) != cudaSuccess)
-                            return -(int)cudaErrorLaunchFailure;
-                        M->jit_aux = as;
-                        M->jit_ev_fork = e1;
-                        M->jit_ev_join = e2;
+                if (conc || rg[3]) {
+                    // concurrent: one stream per range (pool of 8, reused
+                    // round-robin); sequential: the aux runs share stream 0
+                    const int i = conc ? (next++) % 8 : 0;
+                    if (i < nstreams) {
+                        st = (CUstream)M->jit_pool[i];
+                    } else {
+                        if ((st = pool_stream(i)) == nullptr) return -(int)cudaErrorLaunchFailure;
+                        nstreams = i + 1;
                     }
-                    if (!forked) {
-                        if (cudaEventRecord((cudaEvent_t)A->jit_ev_fork, (cudaStream_t)stream) != cudaSuccess ||
-                            cudaStreamWaitEvent((cudaStream_t)A->jit_aux, (cudaEvent_t)A->jit_ev_fork, 0) != cudaSuccess)
-                            return -(int)cudaErrorLaunchFailure;
-                        forked = true;
-                    }
-                    st = (CUstream)A->jit_aux;
                 }
                 j.seg_begin = lo;
                 j.seg_count = hi - lo;
@@ -733,9 +767,10 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
                 ++n;
             }
         }
-        if (forked && (cudaEventRecord((cudaEvent_t)A->jit_ev_join, (cudaStream_t)A->jit_aux) != cudaSuccess ||
-                       cudaStreamWaitEvent((cudaStream_t)stream, (cudaEvent_t)A->jit_ev_join, 0) != cudaSuccess))
-            return -(int)cudaErrorLaunchFailure;
+        for (int i = 0; i < nstreams; ++i)
+            if (cudaEventRecord((cudaEvent_t)M->jit_ev_join[i], (cudaStream_t)M->jit_pool[i]) != cudaSuccess ||
+                cudaStreamWaitEvent((cudaStream_t)stream, (cudaEvent_t)M->jit_ev_join[i], 0) != cudaSuccess)
+                return -(int)cudaErrorLaunchFailure;
         return n;
     } else {
         void *params[] = {&j};
