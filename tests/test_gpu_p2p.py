@@ -119,6 +119,10 @@ def _worker(rank, world, port, case, variant, q):
                 xp[lo : lo + nloc] = x[rb:re]
                 xd = torch.from_numpy(xp).to("cuda:0", tdt)
                 yd = torch.full((nloc,), float("nan"), device="cuda:0", dtype=tdt)
+                # xd / yd were written on the default stream; the side stream
+                # (non-blocking) must not start before those writes land, or
+                # the NaN pads of xd could overwrite the received halo
+                stream.wait_stream(torch.cuda.current_stream())
                 with torch.cuda.stream(stream):
                     A.spmv_dist(xd, yd, 1.0, 0.0, comm, stream=stream)
                 stream.synchronize()
