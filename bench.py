@@ -394,6 +394,8 @@ def run_crsd(args):
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
+    if comm is not None and comm.error():
+        raise SystemExit(f"[bench] rank {rank}: a peer-memory wait timed out during warm-up (code {comm.error()}); no valid number")
 
     # timed region: K steps, per-step CUDA events on the launching stream
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
@@ -423,6 +425,8 @@ def run_crsd(args):
     if world > 1:
         dist.barrier()
     clk = clocks.stop()
+    if comm is not None and comm.error():
+        raise SystemExit(f"[bench] rank {rank}: a peer-memory wait timed out in the timed region (code {comm.error()}); no valid number")
     total_ms = t_all0.elapsed_time(t_all1)
     step_ms = [s.elapsed_time(e) for s, e in ev]
     if world > 1:
