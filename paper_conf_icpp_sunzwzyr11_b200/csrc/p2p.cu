@@ -68,13 +68,16 @@ __device__ bool wait_geq(const uint64_t *p, uint64_t want, uint64_t timeout_ns) 
     return true;
 }
 
-// Byte copy of one item, split over the grid in 4-byte words (element sizes
-// are 4 or 8; slices start at arbitrary elements, so 16-B alignment is not
-// guaranteed and the halo is ~2 % of a rank's bytes).
-__device__ void copy_items(const P2PItem *items, int nitems, int64_t gtid, int64_t gsz) {
+// Byte copy of the items, split over the grid in 4-byte words (element
+// sizes are 4 or 8; slices start at arbitrary elements, so 16-B alignment is
+// not guaranteed and the halo is ~2 % of a rank's bytes). Parity 1 of a
+// mailbox lies parity_shift bytes after parity 0: added to the destination
+// (send: my mailbox) or to the source (recv: the sender's mailbox).
+__device__ void copy_items(const P2PItem *items, int nitems, bool odd, bool shift_dst, int64_t gtid, int64_t gsz) {
     for (int k = 0; k < nitems; ++k) {
-        const uint32_t *s = (const uint32_t *)items[k].src;
-        uint32_t *d = (uint32_t *)items[k].dst;
+        const int64_t sh = odd ? items[k].parity_shift : 0;
+        const uint32_t *s = (const uint32_t *)((const char *)items[k].src + (shift_dst ? 0 : sh));
+        uint32_t *d = (uint32_t *)((char *)items[k].dst + (shift_dst ? sh : 0));
         const int64_t nw = items[k].bytes >> 2;
         if ((((uintptr_t)s | (uintptr_t)d) & 15) == 0) {
             const int64_t nv = nw >> 2;
@@ -121,13 +124,8 @@ __global__ void p2p_send_kernel(P2PLaunch L) {
     if (!ok) return;
     const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
-    // mailbox parity: items carry parity-0 destinations; parity 1 is my cap further
-    P2PItem it[P2P_MAX_ITEMS];
-    for (int k = 0; k < L.nitems; ++k) {
-        it[k] = L.items[k];
-        if (e & 1) it[k].dst = (char *)it[k].dst + it[k].parity_shift;
-    }
-    copy_items(it, L.nitems, gtid, gsz);
+    // items carry parity-0 mailbox destinations (my mailbox, my capacity)
+    copy_items(L.items, L.nitems, (e & 1) != 0, true, gtid, gsz);
     if (last_cta(&me->counter[0]) && threadIdx.x == 0)
         for (int k = 0; k < L.npeer; ++k) st_release_sys(&L.peer_flags[k]->ready[L.rank], e);
 }
@@ -148,13 +146,9 @@ __global__ void p2p_recv_kernel(P2PLaunch L) {
     if (!ok) return;
     const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
-    // parity 1 of the SENDER's mailbox is the sender's cap further (caps may differ per rank)
-    P2PItem it[P2P_MAX_ITEMS];
-    for (int k = 0; k < L.nitems; ++k) {
-        it[k] = L.items[k];
-        if (e & 1) it[k].src = (const char *)it[k].src + it[k].parity_shift;
-    }
-    copy_items(it, L.nitems, gtid, gsz);
+    // items carry parity-0 sources in the SENDER's mailbox, shifted by the
+    // sender's capacity for parity 1 (capacities may differ per rank)
+    copy_items(L.items, L.nitems, (e & 1) != 0, false, gtid, gsz);
     if (last_cta(&me->counter[1]) && threadIdx.x == 0) {
         for (int k = 0; k < L.npeer; ++k) st_release_sys(&L.peer_flags[k]->consumed[L.rank], e);
         me->halo_epoch = e;
