@@ -163,6 +163,24 @@ def test_dense_scatter_segments(torch_cuda, dt, variant):
     assert A.info()["nscatter"] > 1000 and np.max(np.diff(P["scat_ptr"])) > 32
 
 
+@pytest.mark.parametrize("variant", VARIANTS)
+@pytest.mark.parametrize("idle_max", [1, 8, 63])
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_idle_max_sweep_device(torch_cuda, dt, idle_max, variant):
+    """The idle threshold decides which gaps are bridged by fills
+    and which nonzeros fall to the scatter list. On the device path the built
+    layout must equal the oracle's paper-order build for every threshold, and
+    every kernel variant must stay within tolerance of the definition."""
+    from oracle import crsd_ref
+    from tests.test_builder import assert_layout_equal
+
+    a = gen.random_diagonal(3000, 3100, 11 + idle_max, ndiag=9, max_off=700, p_break=0.05,
+                            max_break=80, n_scatter=150).astype(dt)
+    A, _ = _parity(torch_cuda, a, dt, -0.75, 0.5, seed=idle_max, mrows=64, idle_max=idle_max, variant=variant)
+    R = crsd_ref.build(a.nrows, a.ncols, a.row, a.col, a.val, mrows=64, idle_max=idle_max, dtype=dt)
+    assert_layout_equal(A.export(), crsd_ref.to_layout(R))
+
+
 def test_beta_zero_never_reads_y(torch_cuda):
     a = gen.config1()
     A = _mat(a)
