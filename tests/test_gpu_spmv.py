@@ -176,8 +176,8 @@ def test_idle_max_sweep_device(torch_cuda, dt, idle_max, variant):
 
     a = gen.random_diagonal(3000, 3100, 11 + idle_max, ndiag=9, max_off=700, p_break=0.05,
                             max_break=80, n_scatter=150).astype(dt)
-    A, _ = _parity(torch_cuda, a, dt, -0.75, 0.5, seed=idle_max, mrows=64, idle_max=idle_max, variant=variant)
-    R = crsd_ref.build(a.nrows, a.ncols, a.row, a.col, a.val, mrows=64, idle_max=idle_max, dtype=dt)
+    A, _ = _parity(torch_cuda, a, dt, -0.75, 0.5, seed=idle_max, mrows=128, idle_max=idle_max, variant=variant)
+    R = crsd_ref.build(a.nrows, a.ncols, a.row, a.col, a.val, mrows=128, idle_max=idle_max, dtype=dt)
     assert_layout_equal(A.export(), crsd_ref.to_layout(R))
 
 
