@@ -803,8 +803,7 @@ def run_cg(args):
         if comm is None:
             comm, transport = Comm(rank, world, local_rank), "nccl"
         A.dist_bind(comm)
-    fused = world == 1 and info["variant"] == 4 and os.environ.get("CRSD_CG_FUSED_DOT", "0") != "0"
-    vec_passes = 8 if fused else 10
+    vec_passes = 10
     step_bytes = info["unique_bytes_beta0"] + vec_passes * nloc * es
     nnz_local = int(a.nnz)
     step_flops = 2.0 * nnz_local + 10.0 * nloc
@@ -894,7 +893,6 @@ def run_cg(args):
             "nnz": int(nnz_local * world),
             "mrows": info["mrows"],
             "kernel_variant": {1: "ldg", 2: "tma", 3: "pipe", 4: "jit"}[info["variant"]],
-            "fused_pq_dot": fused,
             "check_every": check,
             "parallelism": f"row-partitioned x{world}" + (f", {transport} halo + allreduce" if world > 1 else "") + (", ranks share cuda:0 (functional only)" if args.share_gpu else ""),
             "l2": f"inputs larger than L2 ({step_bytes / 1e9:.2f} GB per step); no flush",

@@ -110,7 +110,25 @@ typedef struct {
     int64_t row_end;
     int32_t nthreads;
     int32_t variant;
+    int32_t jit_chunk;  /* JIT staging chunks (each its own mbarrier): 0 => one per x
+                           window (default), k > 0 => windows split into runs of <= k diagonals, < 0 =>
+                           the whole segment on one mbarrier */
+    uint32_t tune;      /* CRSD_TUNE_* implementation switches (0 = the measured defaults); per handle */
+    int32_t e2e_chunks; /* crsd_spmv_host pipeline depth (row chunks); 0 => 16 */
+    int32_t reserved;   /* must be 0 */
 } crsd_opts_t;
+
+/* opts.tune: the alternatives the measurements in DESIGN.md compare against
+ * the defaults. They change how the work is scheduled, never what is
+ * computed (every setting gives the same y bit for bit). */
+#define CRSD_TUNE_JIT_DESC_ISSUE 0x1u      /* JIT: issue the bulk copies after loading the segment descriptor
+                                              instead of from the baked instance lookup */
+#define CRSD_TUNE_JIT_ONE_LAUNCH 0x2u      /* JIT: one launch for the whole matrix (no occupancy-class ranges) */
+#define CRSD_TUNE_JIT_SPLIT_ALL 0x4u       /* JIT: a range launch at every occupancy-class change (testing) */
+#define CRSD_TUNE_JIT_SEQUENTIAL 0x8u      /* JIT: range launches one after another instead of concurrently */
+#define CRSD_TUNE_DIST_BOUNDARY_SERIAL 0x10u /* crsd_spmv_dist / crsd_cg: boundary segments after the interior on
+                                              the caller's stream instead of behind the exchange on the comm stream */
+#define CRSD_TUNE_NO_JIT 0x20u             /* AUTO never picks the JIT variant */
 
 #define CRSD_VARIANT_AUTO 0
 #define CRSD_VARIANT_LDG 1
@@ -261,7 +279,8 @@ crsd_status_t crsd_comm_destroy(crsd_comm_t comm);
  * from the peer's mailbox straight into the pads of x_padded, then raises a
  * "consumed" flag so the sender may reuse that parity. Epochs live on the
  * device, so the exchange can be captured into a CUDA graph (crsd_cg does).
- * Every wait is bounded (30 s, env CRSD_P2P_TIMEOUT_S read at init): on
+ * Every wait is bounded (30 s; the environment variable CRSD_P2P_TIMEOUT_S,
+ * read once in crsd_comm_init_p2p, overrides it): on
  * timeout the kernel returns and crsd_comm_error reports a non-zero code
  * instead of the GPU hanging.
  *
@@ -306,7 +325,7 @@ crsd_status_t crsd_dist_bind(crsd_matrix_t A_local, crsd_comm_t comm, void *stre
  * (peer-memory kernels or NCCL send/recv, per the communicator) runs on the
  * communicator's highest-priority stream in parallel with the interior
  * segments on `stream`; the boundary segments follow the exchange on the
- * comm stream (concurrently with the interior; CRSD_DIST_BOUNDARY_SERIAL=1
+ * comm stream (concurrently with the interior; CRSD_TUNE_DIST_BOUNDARY_SERIAL
  * runs them on `stream` after it) and `stream` joins the comm stream before
  * the call returns, so y_local is complete in `stream` order. Asynchronous.
  *   x_padded  DEVICE dtype[halo_lo+n_local+halo_hi], 16-byte aligned; the
@@ -362,6 +381,13 @@ crsd_status_t crsd_export(crsd_matrix_t A, crsd_export_t *out);
  * host-only handles (no GPU needed). UNSUPPORTED if a segment's staging
  * (values + x windows) exceeds 200 KB of shared memory. */
 crsd_status_t crsd_jit_source(crsd_matrix_t A, char *buf, int64_t cap, int64_t *len);
+
+/* The sm_100a cubin NVRTC compiled from crsd_jit_source (compiled here if
+ * the handle has none yet; NVRTC only, no GPU needed) -- for inspection with
+ * cuobjdump/nvdisasm (the SASS histogram in profiles/). buf (HOST, may be
+ * NULL) receives up to cap bytes; *len the full size. UNSUPPORTED without
+ * NVRTC or when the staging exceeds 200 KB. */
+crsd_status_t crsd_jit_cubin(crsd_matrix_t A, void *buf, int64_t cap, int64_t *len);
 
 /* ------------------------------------------------------------------------
  * Conjugate gradient on a CRSD matrix (the paper

@@ -1,8 +1,12 @@
-"""ORACLE (test infrastructure only): ctypes wrapper of oracle/coo_spmv.c.
+"""ORACLE (test infrastructure only): ctypes wrapper of oracle/coo_spmv.c
+and oracle/coo_native.c.
 
-y = alpha*A*x + beta*y by definition, long double accumulation
-(BASELINE.json north_star alpha/beta form).
-The shared object is compiled with gcc by ``__graft_entry__.build()`` or on
+y = alpha*A*x + beta*y by definition (
+BASELINE.json north_star alpha/beta form):
+  coo_spmv / rows_spmv -- long double accumulation: the checker
+  coo_spmv_native      -- the same loop in the matrix dtype, 1 or many
+                          threads: the timed CPU baseline
+The shared objects are compiled with gcc by ``__graft_entry__.build()`` or on
 first use here.
 """
 from __future__ import annotations
@@ -16,7 +20,10 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "coo_spmv.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
+_SRC_NATIVE = os.path.join(_HERE, "coo_native.c")
+_LIB_NATIVE = os.path.join(_HERE, "liboracle_native.so")
 _lib = None
+_lib_native = None
 
 
 def build(force: bool = False) -> str:
@@ -24,7 +31,47 @@ def build(force: bool = False) -> str:
         subprocess.check_call(
             ["gcc", "-O2", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared", "-o", _LIB, _SRC, "-lm"]
         )
+    if force or not os.path.exists(_LIB_NATIVE) or os.path.getmtime(_LIB_NATIVE) < os.path.getmtime(_SRC_NATIVE):
+        # -O3 (vectorised loop control), no -march: the .so travels to the GPU box host
+        subprocess.check_call(
+            ["gcc", "-O3", "-ffp-contract=off", "-fno-fast-math", "-fopenmp", "-fPIC", "-shared", "-o", _LIB_NATIVE,
+             _SRC_NATIVE]
+        )
     return _LIB
+
+
+def _load_native():
+    global _lib_native
+    if _lib_native is None:
+        build()
+        lib = ctypes.CDLL(_LIB_NATIVE)
+        p, i64 = ctypes.c_void_p, ctypes.c_int64
+        lib.oracle_coo_native_f64.argtypes = [i64, i64, p, p, p, ctypes.c_double, p, ctypes.c_double, p, p, ctypes.c_int]
+        lib.oracle_coo_native_f32.argtypes = [i64, i64, p, p, p, ctypes.c_float, p, ctypes.c_float, p, p, ctypes.c_int]
+        lib.oracle_coo_native_f64.restype = lib.oracle_coo_native_f32.restype = ctypes.c_int
+        _lib_native = lib
+    return _lib_native
+
+
+def coo_spmv_native(nrows, row, col, val, x, alpha=1.0, beta=0.0, y0=None, nthreads=1, out=None):
+    """y = alpha*A*x + beta*y0 accumulated in val's dtype (float32/float64),
+    ``nthreads`` OpenMP threads over row ranges. COO sorted by row. Returns y
+    in the dtype (into ``out`` when given)."""
+    lib = _load_native()
+    dt = np.float32 if np.asarray(val).dtype == np.float32 else np.float64
+    row = np.ascontiguousarray(row, dtype=np.int64)
+    col = np.ascontiguousarray(col, dtype=np.int64)
+    val = np.ascontiguousarray(val, dtype=dt)
+    x = np.ascontiguousarray(x, dtype=dt)
+    y0 = np.ascontiguousarray(y0 if y0 is not None else np.zeros(0, dt), dtype=dt)
+    if beta != 0 and y0.shape[0] != nrows:
+        raise ValueError("beta != 0 needs y0 of length nrows")
+    y = out if out is not None else np.empty(nrows, dtype=dt)
+    fn = lib.oracle_coo_native_f32 if dt == np.float32 else lib.oracle_coo_native_f64
+    rc = fn(nrows, row.shape[0], _ptr(row), _ptr(col), _ptr(val), alpha, _ptr(x), beta, _ptr(y0), _ptr(y), int(nthreads))
+    if rc != 0:
+        raise ValueError("coo_spmv_native needs a row-sorted COO")
+    return y
 
 
 def _load():

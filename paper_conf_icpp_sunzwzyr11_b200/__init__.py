@@ -16,4 +16,10 @@ from .crsd import (  # noqa: F401
     CRSD_DROP_ZEROS,
     CRSD_PAPER_ELL,
     CGResult,
+    TUNE_JIT_DESC_ISSUE,
+    TUNE_JIT_ONE_LAUNCH,
+    TUNE_JIT_SPLIT_ALL,
+    TUNE_JIT_SEQUENTIAL,
+    TUNE_DIST_BOUNDARY_SERIAL,
+    TUNE_NO_JIT,
 )

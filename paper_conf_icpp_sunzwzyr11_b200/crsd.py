@@ -28,6 +28,9 @@ STATUS = {
 CRSD_R32F, CRSD_R64F = 0, 1
 CRSD_SUM_DUPLICATES, CRSD_HOST_ONLY, CRSD_DROP_ZEROS, CRSD_PAPER_ELL = 0x1, 0x2, 0x4, 0x8
 VARIANT_AUTO, VARIANT_LDG, VARIANT_TMA, VARIANT_PIPE, VARIANT_JIT = 0, 1, 2, 3, 4
+# opts.tune (include/crsd.h CRSD_TUNE_*)
+TUNE_JIT_DESC_ISSUE, TUNE_JIT_ONE_LAUNCH, TUNE_JIT_SPLIT_ALL = 0x1, 0x2, 0x4
+TUNE_JIT_SEQUENTIAL, TUNE_DIST_BOUNDARY_SERIAL, TUNE_NO_JIT = 0x8, 0x10, 0x20
 
 # every symbol include/crsd.h declares
 EXPORTED = [
@@ -51,6 +54,7 @@ EXPORTED = [
     "crsd_export",
     "crsd_last_launch_count",
     "crsd_jit_source",
+    "crsd_jit_cubin",
     "crsd_cg",
     "crsd_autotune",
     "crsd_export_paper_ell",
@@ -80,6 +84,10 @@ class Opts(ctypes.Structure):
         ("row_end", ctypes.c_int64),
         ("nthreads", ctypes.c_int32),
         ("variant", ctypes.c_int32),
+        ("jit_chunk", ctypes.c_int32),
+        ("tune", ctypes.c_uint32),
+        ("e2e_chunks", ctypes.c_int32),
+        ("reserved", ctypes.c_int32),
     ]
 
 
@@ -156,6 +164,7 @@ def _load():
         "crsd_export": ([P, P], ctypes.c_int),
         "crsd_last_launch_count": ([P, P], ctypes.c_int),
         "crsd_jit_source": ([P, P, I64, P], ctypes.c_int),
+        "crsd_jit_cubin": ([P, P, I64, P], ctypes.c_int),
         "crsd_cg": ([P, P, P, I32, ctypes.c_double, I32, P, P, P, P], ctypes.c_int),
         "crsd_autotune": ([P, P, P, I32, P, P, P], ctypes.c_int),
         "crsd_export_paper_ell": ([P, P, P, P, P, P], ctypes.c_int),
@@ -232,6 +241,9 @@ class CRSDMatrix:
         device: int = -1,
         nthreads: int = 0,
         variant: int = 0,
+        jit_chunk: int = 0,
+        tune: int = 0,
+        e2e_chunks: int = 0,
     ) -> "CRSDMatrix":
         row = np.ascontiguousarray(row, dtype=np.int64)
         col = np.ascontiguousarray(col, dtype=np.int64)
@@ -248,6 +260,9 @@ class CRSDMatrix:
         o.device = device
         o.nthreads = nthreads
         o.variant = variant
+        o.jit_chunk = jit_chunk
+        o.tune = tune
+        o.e2e_chunks = e2e_chunks
         if row_range is not None:
             o.row_begin, o.row_end = int(row_range[0]), int(row_range[1])
         h = ctypes.c_void_p()
@@ -438,6 +453,15 @@ class CRSDMatrix:
         buf = ctypes.create_string_buffer(n.value + 1)
         _check(lib.crsd_jit_source(self._h, buf, n.value + 1, ctypes.byref(n)))
         return buf.value.decode()
+
+    def jit_cubin(self) -> bytes:
+        """The sm_100a cubin of the JIT codelets (compiled by NVRTC on demand;
+        no GPU needed) -- for cuobjdump / nvdisasm inspection."""
+        n = ctypes.c_int64()
+        _check(lib.crsd_jit_cubin(self._h, None, 0, ctypes.byref(n)))
+        buf = ctypes.create_string_buffer(n.value)
+        _check(lib.crsd_jit_cubin(self._h, buf, n.value, ctypes.byref(n)))
+        return buf.raw[: n.value]
 
     def last_launch_count(self) -> int:
         c = ctypes.c_int32()

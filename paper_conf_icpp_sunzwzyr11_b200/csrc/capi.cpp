@@ -106,9 +106,7 @@ static void plan_layout(crsd_matrix_s *A) {
     // staging (values + x windows) stays <= 40 KB, i.e. >= 5 CTAs per SM
     A->tma_split = 1;
     A->tma_smem = A->smem_bytes;
-    const int force_split = getenv("CRSD_TMA_SPLIT") ? atoi(getenv("CRSD_TMA_SPLIT")) : 0;
     for (int split = 1; split <= 8; split *= 2) {
-        if (force_split && split < force_split) continue;
         const int64_t rc = H.mrows / split;
         if (H.mrows % split || rc % 32 || (rc * H.elem) % 16) break;
         int64_t mx = 0;
@@ -122,15 +120,14 @@ static void plan_layout(crsd_matrix_s *A) {
         }
         A->tma_split = split;
         A->tma_smem = mx;
-        if (mx <= 40 * 1024 || force_split) break;
+        if (mx <= 40 * 1024) break;
     }
     {
         // rows per thread: the vector width of the dtype (2 fp64, 4 fp32) as
-        // long as a CTA keeps >= 2 warps; CRSD_TMA_Q / CRSD_TMA_SPLIT override
+        // long as a CTA keeps >= 2 warps
         const int64_t rc = H.mrows / A->tma_split;
         int q = A->rpt;
         while (q > 1 && rc / q < 64) q /= 2;
-        if (const char *e = getenv("CRSD_TMA_Q")) q = atoi(e);
         while (rc / q > 256) q *= 2;  // <= 256 threads per CTA
         A->tma_q = q;
     }
@@ -224,7 +221,10 @@ static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_
         delete A;
         return fail(CRSD_ERR_UNSUPPORTED, "PIPE variant: mrows must be <= 1024");
     }
-    const bool auto_jit = !getenv("CRSD_NO_JIT");
+    A->jit_chunk = o.jit_chunk;
+    A->tune = o.tune;
+    A->e2e_chunks = o.e2e_chunks > 0 ? o.e2e_chunks : 16;
+    const bool auto_jit = !(o.tune & CRSD_TUNE_NO_JIT);
     if (o.variant == CRSD_VARIANT_JIT) A->variant = VARIANT_JIT;
     else if (o.variant == CRSD_VARIANT_LDG) A->variant = VARIANT_LDG;
     else if (o.variant == CRSD_VARIANT_TMA) A->variant = VARIANT_TMA;
@@ -289,13 +289,9 @@ static crsd_status_t resolve_opts(int64_t nrows, crsd_dtype_t dtype, const crsd_
 
 template <typename T>
 static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *y, const int32_t *list,
-                              int64_t seg_begin, int64_t count, void *stream, int &launches, const DotArgs *dot) {
+                              int64_t seg_begin, int64_t count, void *stream, int &launches) {
     if (count <= 0) return CRSD_OK;
-    if (dot && A->variant != VARIANT_JIT) return fail(CRSD_ERR_UNSUPPORTED, "fused dot needs the JIT variant");
     SpmvArgs<T> a;
-    a.dot_part = dot ? dot->part : nullptr;
-    a.dot_cnt = dot ? dot->cnt : nullptr;
-    a.dot_out = dot ? dot->out : nullptr;
     a.vals = (const T *)A->d_vals;
     a.segs = (const SegDesc *)A->d_segs;
     a.pat_offs = (const int32_t *)A->d_offs;
@@ -341,13 +337,12 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
 }
 
 crsd_status_t run_lists(crsd_matrix_s *A, const void *alpha, const void *x_base, const void *beta, void *y,
-                        const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches,
-                        const DotArgs *dot) {
+                        const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches) {
     if (A->H.dtype == CRSD_R64F)
         return run_spmv<double>(A, *(const double *)alpha, (const double *)x_base, *(const double *)beta, (double *)y,
-                                list, seg_begin, count, stream, launches, dot);
+                                list, seg_begin, count, stream, launches);
     return run_spmv<float>(A, *(const float *)alpha, (const float *)x_base, *(const float *)beta, (float *)y, list,
-                           seg_begin, count, stream, launches, dot);
+                           seg_begin, count, stream, launches);
 }
 
 }  // namespace crsd
@@ -465,29 +460,11 @@ crsd_status_t crsd_spmv(crsd_matrix_t A, const void *alpha, const void *x, const
 static crsd_status_t e2e_setup(crsd_matrix_s *A) {
     HostCRSD &H = A->H;
     const int64_t nseg = H.nseg;
-    const int want = getenv("CRSD_E2E_CHUNKS") ? atoi(getenv("CRSD_E2E_CHUNKS")) : 16;
-    int nch = (int)std::min<int64_t>(want, std::max<int64_t>(1, nseg / 32));
+    int nch = (int)std::min<int64_t>(A->e2e_chunks, std::max<int64_t>(1, nseg / 32));
     A->e2e_nchunk = nch;
     A->e2e_seg.resize(nch + 1);
     A->e2e_xcut.resize(nch + 1);
     for (int c = 0; c <= nch; ++c) A->e2e_seg[c] = nseg * c / nch;
-    // CRSD_E2E_RAMP=1: the first and last three chunks 1/8, 1/4, 1/2 of the
-    // others (shorter pipeline fill before the first y copy and drain after
-    // the last kernel)
-    if (getenv("CRSD_E2E_RAMP") && atoi(getenv("CRSD_E2E_RAMP")) && nch >= 8) {
-        std::vector<double> w(nch, 1.0);
-        const double r[3] = {0.125, 0.25, 0.5};
-        for (int k = 0; k < 3; ++k) w[k] = w[nch - 1 - k] = r[k];
-        double tot = 0.0;
-        for (double v : w) tot += v;
-        double acc = 0.0;
-        for (int c = 0; c < nch; ++c) {
-            A->e2e_seg[c] = std::min<int64_t>(nseg, (int64_t)(nseg * acc / tot));
-            acc += w[c];
-        }
-        A->e2e_seg[nch] = nseg;
-        for (int c = 1; c <= nch; ++c) A->e2e_seg[c] = std::max(A->e2e_seg[c], A->e2e_seg[c - 1]);
-    }
     // highest x element each row chunk reads (vector windows, clipped to
     // [0, ncols) as the guarded edge path does, and scatter columns)
     std::vector<int64_t> hi(nch, 0);
@@ -501,15 +478,13 @@ static crsd_status_t e2e_setup(crsd_matrix_s *A) {
     }
     // x chunks are aligned with the row chunks, so row chunk c usually waits
     // for x chunk c+1 (its far diagonals reach a few rows into it). Cutting x
-    // where each row chunk's reads end instead (CRSD_E2E_CUT=needs) lets
-    // y copies start one chunk earlier but measured slower: the earlier D2H
-    // overlaps more of the H2D stream and slows it (C2 f64, 12-16 chunks:
-    // 3.38 vs 3.56-3.59 ms; profiles/r01_e2e_cut_ab.txt).
-    const bool cut_rows = !(getenv("CRSD_E2E_CUT") && std::string(getenv("CRSD_E2E_CUT")) == "needs");
+    // where each row chunk's reads end instead lets y copies start one chunk
+    // earlier but measured slower: the earlier D2H overlaps more of the H2D
+    // stream and slows it (C2 f64, 12-16 chunks: 3.38 vs 3.56-3.59 ms;
+    // profiles/r01_e2e_cut_ab.txt).
     A->e2e_xcut[0] = 0;
     for (int c = 0; c < nch; ++c) {
-        int64_t xc = (c == nch - 1) ? H.ncols : std::min<int64_t>(H.ncols, (hi[c] + 3) / 4 * 4);
-        if (cut_rows) xc = std::min<int64_t>(H.ncols, A->e2e_seg[c + 1] * H.mrows) / 4 * 4;
+        const int64_t xc = std::min<int64_t>(H.ncols, A->e2e_seg[c + 1] * H.mrows) / 4 * 4;
         A->e2e_xcut[c + 1] = std::max(A->e2e_xcut[c], xc);
     }
     A->e2e_xcut[nch] = H.ncols;

@@ -22,8 +22,10 @@ struct crsd_matrix_s {
     std::string jit_source;
     void *jit_module = nullptr;
     void *jit_function = nullptr;
-    void *jitp_function = nullptr;  // persistent double-buffered form (crsd_jitp), or null
-    bool jit_persist = false;       // launch the persistent form by default
+    std::vector<char> jit_cubin;    // the compiled codelets (crsd_jit_cubin)
+    int32_t jit_chunk = 0;          // opts.jit_chunk: diagonals per staging chunk (0 = per x window, <0 = one)
+    uint32_t tune = 0;              // opts.tune: CRSD_TUNE_* switches
+    int32_t e2e_chunks = 16;        // opts.e2e_chunks: crsd_spmv_host pipeline depth
     // one-GPU launches of the one-shot codelets split into contiguous segment
     // ranges of equal occupancy class: {seg_begin, seg_count, dynamic smem}
     // {seg_begin, seg_count, dynamic smem, aux}: aux = 1 for short runs that
@@ -96,15 +98,9 @@ crsd_status_t jit_build(crsd_matrix_s *A);
 void jit_free(crsd_matrix_s *A);
 template <typename T>
 int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &a, void *stream);
-// Run the SpMV kernel over a device list of segments (list == nullptr: all
-// segments [0, count)). x_base is the local x base (x_padded + halo_lo).
-// dot != null (JIT variant only, one launch): also *dot->out = sum_rows x[row] * y[row].
-struct DotArgs {
-    double *part;   // count + ceil(count / 256) partials
-    uint32_t *cnt;  // ceil(count / 256) + 1 counters, zero between launches
-    double *out;
-};
+// Run the SpMV kernel over a device list of segments (list == nullptr: the
+// segment range [seg_begin, seg_begin + count)). x_base is the local x base
+// (x_padded + halo_lo).
 crsd_status_t run_lists(crsd_matrix_s *A, const void *alpha, const void *x_base, const void *beta, void *y,
-                        const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches,
-                        const DotArgs *dot = nullptr);
+                        const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches);
 }  // namespace crsd

@@ -166,11 +166,6 @@ struct SpmvArgs {
     int32_t has_scatter;      // the matrix has scatter points (selects the staging kernel)
     int32_t variant;          // VARIANT_LDG / _TMA / _PIPE / _JIT
     T alpha, beta;
-    // optional fused dot (JIT variant, CG): *dot_out = sum_rows x[row] * y[row]
-    // over the launch's rows, deterministic (per-CTA partials, last CTA sums)
-    double *dot_part;         // one per CTA, or null
-    uint32_t *dot_cnt;        // zero on entry, reset by the last CTA
-    double *dot_out;
 };
 
 // Paper-exact scatter rows (CRSD_PAPER_ELL): y[rowno[i]] = alpha * sum_k

@@ -361,7 +361,7 @@ crsd_status_t p2p_exchange(crsd_matrix_t A, crsd_comm_t c, char *xp) {
                              xp + es * A->recv_off[k], es * A->recv_count[k], c->peer_cap[A->recv_peer[k]]};
     // a few CTAs suffice for the halo (~2 % of a rank's bytes); every CTA of
     // p2p_recv holds an SM slot while it waits for the peers
-    static const int grid = getenv("CRSD_P2P_GRID") ? std::max(1, atoi(getenv("CRSD_P2P_GRID"))) : 16;
+    const int grid = 16;
     CU_TRY((cudaError_t)p2p_launch_send(S, grid, c->cs));
     CU_TRY((cudaError_t)p2p_launch_recv(R, grid, c->cs));
     return CRSD_OK;
@@ -407,8 +407,8 @@ crsd_status_t crsd_spmv_dist(crsd_matrix_t A, const void *alpha, void *x_padded,
 
 }  // extern "C"
 
-// boundary: -1 = default (concurrent on the comm stream unless
-// CRSD_DIST_BOUNDARY_SERIAL=1), 0 = concurrent, 1 = serial after the interior
+// boundary: -1 = the handle's setting (concurrent on the comm stream unless
+// CRSD_TUNE_DIST_BOUNDARY_SERIAL), 0 = concurrent, 1 = serial after the interior
 crsd_status_t crsd::spmv_dist_impl(crsd_matrix_t A, const void *alpha, void *x_padded, const void *beta,
                                    void *y_local, crsd_comm_t c, void *stream, int boundary) {
     if (!A) return crsd::fail(CRSD_ERR_INVALID_ARG, "A is NULL");
@@ -430,9 +430,8 @@ crsd_status_t crsd::spmv_dist_impl(crsd_matrix_t A, const void *alpha, void *x_p
     // priority, so its CTAs take the next free SM slots ahead of queued SpMV
     // CTAs). Default order: interior segments launched first, then the
     // exchange — the interior fills the GPU at once and the small exchange
-    // kernels slot in as CTAs retire; CRSD_DIST_EXCHANGE_FIRST=1 launches the
-    // exchange first.
-    static const bool exchange_first = getenv("CRSD_DIST_EXCHANGE_FIRST") && atoi(getenv("CRSD_DIST_EXCHANGE_FIRST"));
+    // kernels slot in as CTAs retire (launching the exchange first measured
+    // the same under MPS).
     if (c) CU_TRY(cudaEventRecord(c->ev_x, s));
     auto exchange = [&]() -> crsd_status_t {
         CU_TRY(cudaStreamWaitEvent(c->cs, c->ev_x, 0));
@@ -453,7 +452,6 @@ crsd_status_t crsd::spmv_dist_impl(crsd_matrix_t A, const void *alpha, void *x_p
         CU_TRY(cudaEventRecord(c->ev_halo, c->cs));
         return CRSD_OK;
     };
-    if (c && exchange_first) ST_TRY(exchange());
     // a contiguous interior (no scatter column reaching outside: C2, C4, C5)
     // launches as a segment range: no per-CTA list load before the
     // descriptor, and the JIT occupancy classes apply
@@ -466,14 +464,13 @@ crsd_status_t crsd::spmv_dist_impl(crsd_matrix_t A, const void *alpha, void *x_p
         st = crsd::run_lists(A, alpha, xbase, beta, y_local, (const int32_t *)A->d_list_interior, 0,
                              (int64_t)li.size(), stream, launches);
     if (st) return st;
-    if (c && !exchange_first) ST_TRY(exchange());
+    if (c) ST_TRY(exchange());
     // The boundary segments run on the comm stream right behind the
     // exchange, i.e. concurrently with the interior rather than after it: no
     // serial tail (interior drain + a small dependent launch) per call. The
-    // caller's stream then waits for the comm stream. CRSD_DIST_BOUNDARY_SERIAL=1
+    // caller's stream then waits for the comm stream. CRSD_TUNE_DIST_BOUNDARY_SERIAL
     // runs them on the caller's stream after the interior instead.
-    static const bool serial_env = getenv("CRSD_DIST_BOUNDARY_SERIAL") && atoi(getenv("CRSD_DIST_BOUNDARY_SERIAL"));
-    const bool serial = boundary < 0 ? serial_env : boundary == 1;
+    const bool serial = boundary < 0 ? (A->tune & CRSD_TUNE_DIST_BOUNDARY_SERIAL) != 0 : boundary == 1;
     if (c && serial) CU_TRY(cudaStreamWaitEvent(s, c->ev_halo, 0));
     st = crsd::run_lists(A, alpha, xbase, beta, y_local, (const int32_t *)A->d_list_boundary, 0,
                          (int64_t)A->list_boundary.size(), (c && !serial) ? (void *)c->cs : stream, launches);

@@ -6,14 +6,29 @@
 // kernel is compiled at runtime (OpenCL there, NVRTC here). Only the values
 // (and x, y) are read at SpMV time.
 //
-// The generated kernel has the data movement of the TMA variant (one CTA per
-// segment, thread 0 bulk-copies the segment's value block, warp 0 the x
-// windows, one mbarrier), but every pattern-dependent quantity is a literal:
-// the diagonal count, the window starts/lengths, each diagonal's offset into
-// the staged x, the offsets for the guarded edge path. The codelet for a
-// pattern is fully unrolled. NVRTC (libnvrtc.so.12) and the CUDA
-// driver API are resolved at runtime (dlopen / cudaGetDriverEntryPoint), so
-// libcrsd.so loads on machines without them.
+// The generated kernel runs one CTA per row segment. Thread 0
+// bulk-copies (cp.async.bulk, SASS UBLKCP) the segment's value block and its
+// x windows into shared memory; every pattern-dependent quantity is a
+// literal: the diagonal count, the window starts/lengths, each diagonal's
+// offset into the staged x, the offsets for the guarded edge path. The
+// codelet for a pattern is fully unrolled.
+//
+// Staging chunks. The value block and the windows are split into chunks,
+// each completing on its own mbarrier (by default one chunk per x window:
+// the window and the value runs of the diagonals that read it). The FMAs of
+// chunk c start as soon as chunk c has landed while the later chunks are
+// still in flight, so a CTA holds its shared memory for less time after its
+// last byte arrives than with one barrier for the whole segment.
+//
+// Descriptor-free issue. The segment -> pattern lookup (the paper's group_id
+// -> pattern) is baked into the kernel as a comparison tree over
+// the instances' first segments, with each instance's value base as a
+// literal, so thread 0 issues the bulk copies without waiting for any memory
+// load; the segment descriptor (scatter list) is read while they fly.
+//
+// NVRTC (libnvrtc.so.12) and the CUDA driver API are resolved at runtime
+// (dlopen / cudaGetDriverEntryPoint), so libcrsd.so loads on machines
+// without them.
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <dlfcn.h>
@@ -129,9 +144,6 @@ struct JitArgs {
     const T *scat_val;
     const ScatRec *scat_rec;
     T alpha, beta;
-    double *dot_part;
-    uint32_t *dot_cnt;
-    double *dot_out;
 };
 
 const char *kPrelude = R"(
@@ -143,11 +155,11 @@ struct SegDesc { i64 val_base; i64 scat_begin; int off_begin; int nscat; u16 fla
 struct __align__(16) ScatRec { i64 col; double val; int row; int pad[3]; };
 struct Args { const T *vals; const SegDesc *segs; const int *seg_list; i64 seg_begin, seg_count;
               const T *x; i64 x_lo, x_hi; T *y; i64 nrows;
-              const int *scat_row; const i64 *scat_col; const T *scat_val; const ScatRec *scat_rec; T alpha, beta;
-              double *dot_part; u32 *dot_cnt; double *dot_out; };
+              const int *scat_row; const i64 *scat_col; const T *scat_val; const ScatRec *scat_rec; T alpha, beta; };
 __device__ __forceinline__ u32 su32(const void *p) { return (u32)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void bar_init(u64 *b) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(su32(b)) : "memory");
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(su32(b)) : "memory"); }
+__device__ __forceinline__ void bar_fence_init() {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
 __device__ __forceinline__ void bar_expect(u64 *b, u32 n) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(su32(b)), "r"(n) : "memory"); }
@@ -155,10 +167,6 @@ __device__ __forceinline__ void bar_wait(u64 *b) {
   u32 done = 0;
   while (!done) asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0; selp.u32 %0, 1, 0, p; }"
                              : "=r"(done) : "r"(su32(b)) : "memory"); }
-__device__ __forceinline__ void bar_wait_ph(u64 *b, u32 ph) {
-  u32 done = 0;
-  while (!done) asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
-                             : "=r"(done) : "r"(su32(b)), "r"(ph) : "memory"); }
 __device__ __forceinline__ u64 pol_first() { u64 p; asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p)); return p; }
 __device__ __forceinline__ u64 pol_normal() { u64 p; asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p)); return p; }
 __device__ __forceinline__ void g2s(void *dst, const void *src, u32 bytes, u64 *b, u64 pol) {
@@ -166,295 +174,59 @@ __device__ __forceinline__ void g2s(void *dst, const void *src, u32 bytes, u64 *
                :: "r"(su32(dst)), "l"(src), "r"(bytes), "r"(su32(b)), "l"(pol) : "memory"); }
 )";
 
+// One staging chunk: diagonals [d0, d1) of a pattern's value block and,
+// when win >= 0, the x window `win` (whose diagonals start at d0).
+struct Chunk {
+    int d0, d1, win;
+};
+
+// Chunks of a pattern. chunk < 0: one chunk (one mbarrier) holding the whole
+// value block and every window (win == -2); chunk == 0: one chunk per x
+// window (the window's diagonals are contiguous: windows are clusters of
+// consecutive offsets, make_plans); chunk > 0: windows further split into
+// runs of at most `chunk` diagonals, the window riding with the first.
+std::vector<Chunk> make_chunks(const int32_t *pl, int nd, int chunk) {
+    std::vector<Chunk> out;
+    if (nd == 0) return out;
+    if (chunk < 0) {
+        out.push_back({0, nd, -2});
+        return out;
+    }
+    const int nwin = pl[0];
+    const int32_t *xwin = pl + 2 + 2 * nwin + nd;
+    const int step = chunk > 0 ? chunk : nd;
+    for (int d = 0; d < nd;) {
+        int e = d;
+        while (e + 1 < nd && xwin[e + 1] == xwin[d]) ++e;
+        for (int a = d; a <= e; a += step) out.push_back({a, std::min(e + 1, a + step), a == d ? xwin[d] : -1});
+        d = e + 1;
+    }
+    return out;
+}
+
+// Instances as leaves of the baked segment -> (pattern, value base) lookup.
+struct Leaf {
+    int64_t first, stride, val_base;
+    int32_t key;
+};
+
+void emit_locate(std::ostringstream &o, const std::vector<Leaf> &L, size_t lo, size_t hi, int depth) {
+    const std::string ind(2 + 2 * depth, ' ');
+    if (hi - lo == 1) {
+        const Leaf &f = L[lo];
+        o << ind << "{ key = " << f.key << "; vb = " << f.val_base << "LL + (s - " << f.first << "LL) * " << f.stride
+          << "LL; }\n";
+        return;
+    }
+    const size_t mid = (lo + hi) / 2;
+    o << ind << "if (s < " << L[mid].first << "LL) {\n";
+    emit_locate(o, L, lo, mid, depth + 1);
+    o << ind << "} else {\n";
+    emit_locate(o, L, mid, hi, depth + 1);
+    o << ind << "}\n";
+}
+
 }  // namespace
-
-// Generate the codelets of every distinct pattern of A (TMA data movement,
-// whole segment per CTA, Q rows per thread).
-static std::string generate(const crsd_matrix_s *A, int Q) {
-    const HostCRSD &H = A->H;
-    const bool f64 = H.dtype == CRSD_R64F;
-    const int m = H.mrows, nt = m / Q, es = H.elem;
-    const bool scat = H.nscatter() > 0;  // scatter code only for matrices that have scatter points
-    // early issue (default; CRSD_JIT_EARLY=0 for the late form): +1-4 % on
-    // C2/C3/C4 (sweep20)
-    const bool early = !(getenv("CRSD_JIT_EARLY") && atoi(getenv("CRSD_JIT_EARLY")) == 0);
-    std::ostringstream o;
-    o << "typedef " << (f64 ? "double" : "float") << " T;\n" << kPrelude;
-    o << "#define MROWS " << m << "\n#define NT " << nt << "\n#define Q " << Q << "\n";
-    // block sum in a fixed order (shuffle tree per warp, then warps in order);
-    // the result is valid in thread 0
-    o << "__device__ __forceinline__ double blk_sum(double v, double *red) {\n"
-         "  for (int k = 16; k; k >>= 1) v += __shfl_down_sync(0xffffffffu, v, k);\n"
-         "  __syncthreads();\n  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = v;\n  __syncthreads();\n"
-         "  double b = 0.0;\n  if (threadIdx.x == 0) for (int k = 0; k < NT / 32; ++k) b += red[k];\n  return b;\n}\n";
-    // one __device__ codelet per distinct pattern
-    // codelets are keyed by the pattern's plan_begin, which is unique per
-    // distinct pattern (off_begin is not: a pattern without diagonals shares
-    // it with the next pattern)
-    std::vector<int32_t> seen;
-    for (const Instance &I : H.inst) {
-        const int32_t key = A->segdesc[I.first_seg].plan_begin;
-        bool dup = false;
-        for (int32_t v : seen) dup |= (v == key);
-        if (dup) continue;
-        seen.push_back(key);
-        const int32_t *pl = A->plan.data() + key;
-        const int nd = (int)H.ndias(I.pattern), nwin = pl[0];
-        const int64_t *offs = H.pat_offsets.data() + H.pat_ptr[I.pattern];
-        o << "// pattern offsets:";
-        for (int d = 0; d < nd; ++d) o << " " << offs[d];
-        o << "\n__device__ __forceinline__ double codelet_" << key
-          << "(const Args &a, const SegDesc &D, i64 row0, bool edge, T *vs, u64 *bar, int t) {\n";
-        int64_t xb = 0;
-        for (int w = 0; w < nwin; ++w) xb += pl[3 + 2 * w];
-        o << "  T *xs = vs + " << (int64_t)nd * m << ";\n";
-        // a pattern without diagonals (rows holding only scatter points, or
-        // nothing) stages nothing: no mbarrier at all
-        // Copy issue. early (default): thread 0 initialises the mbarrier and
-        // issues every copy (values, then the x windows) before the CTA
-        // barrier, and the scatter gathers are issued before it too. Late
-        // form (CRSD_JIT_EARLY=0): thread 0 issues the value copy, lane w of
-        // warp 0 issues x window w after the CTA barrier.
-        std::string sg;
-        if (scat) {
-            // scatter points are gathered while the bulk copies are in flight:
-            // lane l of every warp reads record l of the segment's first 32
-            // (row, col, value in one 32-B record); a ballot keeps those whose
-            // row belongs to this warp, which alone load x[col]
-            sg = "  int g_own = -1; T g_v = T(0), g_x = T(0); unsigned g_mask = 0u;\n"
-                 "  if (D.nscat > 0) {\n"
-                 "    const int lane = t & 31;\n"
-                 "    ScatRec R; R.col = 0; R.val = 0; R.row = 0;\n"
-                 "    if (lane < D.nscat) { R = a.scat_rec[D.scat_begin + lane]; g_own = (R.row % NT) * Q + R.row / NT; }\n"
-                 "    const bool mine = g_own >= 0 && (g_own / Q) / 32 == t / 32;\n"
-                 "    g_mask = __ballot_sync(0xffffffffu, mine);\n"
-                 "    if (mine) { g_v = *reinterpret_cast<const T *>(&R.val); g_x = __ldg(a.x + R.col); }\n"
-                 "  }\n";
-        }
-        // a pattern without diagonals (rows holding only scatter points, or
-        // nothing) stages nothing: no mbarrier at all
-        if (nd) {
-            o << "  if (t == 0) { bar_init(bar); bar_expect(bar, " << (int64_t)nd * m * es << "u + (edge ? 0u : "
-              << xb * es << "u));\n";
-            o << "    g2s(vs, a.vals + D.val_base, " << (int64_t)nd * m * es << "u, bar, pol_first());\n";
-            if (early && nwin) {
-                o << "    if (!edge) { const u64 pn = pol_normal();\n";
-                int64_t base = 0;
-                for (int w = 0; w < nwin; ++w) {
-                    o << "      g2s(xs + " << base << ", a.x + row0 + (" << pl[2 + 2 * w] << "), "
-                      << (int64_t)pl[3 + 2 * w] * es << "u, bar, pn);\n";
-                    base += pl[3 + 2 * w];
-                }
-                o << "    }\n";
-            }
-            o << "  }\n";
-            if (early) o << sg;
-            o << "  __syncthreads();\n";
-        } else {
-            o << "  (void)xs; (void)bar;\n";
-            if (early) o << sg;
-        }
-        if (nwin && !early) {
-            o << "  if (!edge && t < 32) { const u64 pn = pol_normal();\n";
-            int64_t base = 0;
-            for (int w = 0; w < nwin; ++w) {
-                o << "    if (t == " << (w % 32) << ") g2s(xs + " << base << ", a.x + row0 + (" << pl[2 + 2 * w] << "), "
-                  << (int64_t)pl[3 + 2 * w] * es << "u, bar, pn);\n";
-                base += pl[3 + 2 * w];
-            }
-            o << "  }\n";
-        }
-        if (!early) o << sg;
-        o << "  T acc[Q];\n#pragma unroll\n  for (int q = 0; q < Q; ++q) acc[q] = T(0);\n";
-        // fused dot: x[row] is loaded now, while the bulk copies fly, not in
-        // the epilogue (a load there would add a memory latency to every CTA)
-        o << "  T xr[Q];\n  if (a.dot_part) {\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n"
-             "      const i64 r = row0 + t + q * NT;\n      xr[q] = (!edge || r < a.nrows) ? __ldg(a.x + r) : T(0);\n    }\n  }\n";
-        if (nd) o << "  bar_wait(bar);\n";
-        const int32_t *xoff = pl + 2 + 2 * nwin;
-        o << "  if (!edge) {\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n      const int r = t + q * NT;\n";
-        for (int d = 0; d < nd; ++d)
-            o << "      acc[q] = fma(vs[" << (int64_t)d * m << " + r], xs[" << xoff[d] << " + r], acc[q]);\n";
-        o << "    }\n  } else {\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n      const i64 r = row0 + t + q * NT;\n";
-        for (int d = 0; d < nd; ++d)
-            o << "      { const i64 i = r + (" << offs[d] << "); acc[q] = fma(vs[" << (int64_t)d * m
-              << " + t + q * NT], (i >= a.x_lo && i < a.x_hi) ? __ldg(a.x + i) : T(0), acc[q]); }\n";
-        o << "    }\n  }\n";
-        // scatter points in (row, col) order by their owner thread: the
-        // gathered ones (broadcast from the lane holding them), then any
-        // beyond the first 32; then the epilogue
-        if (scat)
-            o << "  if (D.nscat > 0) {\n"
-                 "    for (unsigned mm = g_mask; mm; mm &= mm - 1) {\n"
-                 "      const int j = __ffs(mm) - 1;\n"
-                 "      const int own = __shfl_sync(0xffffffffu, g_own, j);\n"
-                 "      const T v = __shfl_sync(0xffffffffu, g_v, j), xv = __shfl_sync(0xffffffffu, g_x, j);\n"
-                 "#pragma unroll\n      for (int q = 0; q < Q; ++q) if (own == t * Q + q) acc[q] = fma(v, xv, acc[q]);\n"
-                 "    }\n"
-                 "    for (int e = 32; e < D.nscat; ++e) {\n"
-                 "      const int rr = __ldg(a.scat_row + D.scat_begin + e);\n"
-                 "      if (rr % NT != t) continue;\n"
-                 "      const T v = __ldg(a.scat_val + D.scat_begin + e), xv = __ldg(a.x + __ldg(a.scat_col + D.scat_begin + e));\n"
-                 "#pragma unroll\n      for (int q = 0; q < Q; ++q) if (rr / NT == q) acc[q] = fma(v, xv, acc[q]);\n"
-                 "    }\n  }\n";
-        // epilogue; with a fused dot (CG: (p, q) with p = x) each thread
-        // also accumulates x[row] * y[row] in fp64
-        o << "  double dsum = 0.0;\n#pragma unroll\n  for (int q = 0; q < Q; ++q) {\n    const i64 r = row0 + t + q * NT;\n"
-             "    if (!edge || r < a.nrows) {\n      T *yp = a.y + r;\n"
-             "      const T out = (a.beta != T(0)) ? fma(a.alpha, acc[q], a.beta * *yp) : a.alpha * acc[q];\n"
-             "      __stcs(yp, out);\n"
-             "      if (a.dot_part) dsum = fma((double)xr[q], (double)out, dsum);\n    }\n"
-             "  }\n  return dsum;\n}\n";
-    }
-    o << "extern \"C\" __global__ void __launch_bounds__(NT) crsd_jit(const Args a) {\n"
-         "  extern __shared__ __align__(128) unsigned char smem[];\n  __shared__ u64 bar;\n"
-         "  const i64 s = a.seg_list ? (i64)__ldg(a.seg_list + blockIdx.x) : a.seg_begin + blockIdx.x;\n"
-         "  const SegDesc D = a.segs[s];\n  const i64 row0 = s * MROWS;\n  const bool edge = (D.flags & 1) != 0;\n"
-         "  T *vs = reinterpret_cast<T *>(smem);\n  double d = 0.0;\n  switch (D.plan_begin) {\n";
-    for (int32_t v : seen) o << "  case " << v << ": d = codelet_" << v << "(a, D, row0, edge, vs, &bar, threadIdx.x); break;\n";
-    o << "  }\n";
-    // fused dot, deterministic two-level reduction: every CTA writes its
-    // partial; the last CTA to arrive in each group of 256 CTAs sums that
-    // group's partials (one load per thread, fixed tree order) into a group
-    // partial; the last group sums the group partials. One counter per group
-    // keeps the atomics spread and the tail to two short reductions (a single
-    // last CTA summing every partial was a ~30 us serial tail per launch).
-    o << "  if (a.dot_part) {\n"
-         "    __shared__ double red[NT / 32];\n    __shared__ bool last;\n"
-         "    const unsigned G = (gridDim.x + 255u) / 256u, g = blockIdx.x / 256u;\n"
-         "    const unsigned gs = min(256u, gridDim.x - g * 256u);\n"
-         "    double *gpart = a.dot_part + gridDim.x;\n"
-         "    d = blk_sum(d, red);\n"
-         "    if (threadIdx.x == 0) {\n      a.dot_part[blockIdx.x] = d;\n      __threadfence();\n"
-         "      last = atomicAdd(a.dot_cnt + g, 1u) == gs - 1;\n    }\n    __syncthreads();\n"
-         "    if (last) {\n      __threadfence();\n"
-         "      double b = 0.0;\n"
-         "      for (unsigned k = threadIdx.x; k < gs; k += NT) b += __ldcg(a.dot_part + g * 256u + k);\n"
-         "      b = blk_sum(b, red);\n"
-         "      if (threadIdx.x == 0) {\n        gpart[g] = b;\n        a.dot_cnt[g] = 0u;\n        __threadfence();\n"
-         "        last = atomicAdd(a.dot_cnt + G, 1u) == G - 1;\n      }\n      __syncthreads();\n"
-         "      if (last) {\n        __threadfence();\n        double c = 0.0;\n"
-         "        for (unsigned k = threadIdx.x; k < G; k += NT) c += __ldcg(gpart + k);\n"
-         "        c = blk_sum(c, red);\n"
-         "        if (threadIdx.x == 0) {\n          *a.dot_out = c;\n          a.dot_cnt[G] = 0u;\n        }\n      }\n    }\n  }\n";
-    o << "}\n";
-    return o.str();
-}
-
-// Persistent, double-buffered form of the codelets (kernel crsd_jitp): a
-// CTA per SM slot loops over its segments (w, w + G, ...) with two staging
-// buffers. Warp 0 refills a buffer as soon as every thread is done with it:
-// lane 0 copies the segment descriptor into the buffer's header and issues
-// the bulk copies (values, x windows) with every pattern quantity a literal;
-// the 32 lanes read the segment's first 32 scatter records and gather their
-// x[col] into the header. The segment after next is therefore in flight
-// while the current one computes, and no CTA start-up (launch, descriptor
-// load, scatter gather) sits between a buffer's reuse and its next copy.
-static void generate_persistent(const crsd_matrix_s *A, int Q, std::ostringstream &o) {
-    const HostCRSD &H = A->H;
-    const int m = H.mrows, es = H.elem;
-    const bool scat = H.nscatter() > 0;
-    o << "\n// ---- persistent double-buffered form ----\n"
-         "struct __align__(16) StageHdr { SegDesc D; i64 row0; int nsg; int pad; int own[32]; T v[32]; T xv[32]; };\n"
-         "#define HDR ((int)((sizeof(StageHdr) + 127) / 128 * 128))\n";
-    std::vector<int32_t> seen;
-    std::ostringstream issue_sw, comp_sw;
-    for (const Instance &I : H.inst) {
-        const int32_t key = A->segdesc[I.first_seg].plan_begin;
-        bool dup = false;
-        for (int32_t v : seen) dup |= (v == key);
-        if (dup) continue;
-        seen.push_back(key);
-        const int32_t *pl = A->plan.data() + key;
-        const int nd = (int)H.ndias(I.pattern), nwin = pl[0];
-        const int64_t *offs = H.pat_offsets.data() + H.pat_ptr[I.pattern];
-        int64_t xb = 0;
-        for (int w = 0; w < nwin; ++w) xb += pl[3 + 2 * w];
-        // issue (lane 0 of warp 0)
-        o << "__device__ __forceinline__ void pissue_" << key
-          << "(const Args &a, const SegDesc &D, i64 row0, bool edge, T *vs, u64 *bar) {\n";
-        o << "  bar_expect(bar, " << (int64_t)nd * m * es << "u + (edge ? 0u : " << xb * es << "u));\n";
-        if (nd) o << "  g2s(vs, a.vals + D.val_base, " << (int64_t)nd * m * es << "u, bar, pol_first());\n";
-        if (nwin) {
-            o << "  if (!edge) {\n    T *xs = vs + " << (int64_t)nd * m << ";\n    const u64 pn = pol_normal();\n";
-            int64_t base = 0;
-            for (int w = 0; w < nwin; ++w) {
-                o << "    g2s(xs + " << base << ", a.x + row0 + (" << pl[2 + 2 * w] << "), " << (int64_t)pl[3 + 2 * w] * es
-                  << "u, bar, pn);\n";
-                base += pl[3 + 2 * w];
-            }
-            o << "  }\n";
-        }
-        o << "}\n";
-        // compute (all threads)
-        const int32_t *xoff = pl + 2 + 2 * nwin;
-        o << "__device__ __forceinline__ void pcomp_" << key
-          << "(const Args &a, const StageHdr &S, bool edge, const T *vs, u64 *bar, u32 ph, int t) {\n";
-        o << "  const T *xs = vs + " << (int64_t)nd * m << ";\n  const i64 row0 = S.row0;\n  (void)xs;\n";
-        o << "  T acc[Q];\n#pragma unroll\n  for (int q = 0; q < Q; ++q) acc[q] = T(0);\n";
-        o << "  bar_wait_ph(bar, ph);\n";
-        o << "  if (!edge) {\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n      const int r = t + q * NT;\n";
-        for (int d = 0; d < nd; ++d)
-            o << "      acc[q] = fma(vs[" << (int64_t)d * m << " + r], xs[" << xoff[d] << " + r], acc[q]);\n";
-        o << "    }\n  } else {\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n      const i64 r = row0 + t + q * NT;\n";
-        for (int d = 0; d < nd; ++d)
-            o << "      { const i64 i = r + (" << offs[d] << "); acc[q] = fma(vs[" << (int64_t)d * m
-              << " + t + q * NT], (i >= a.x_lo && i < a.x_hi) ? __ldg(a.x + i) : T(0), acc[q]); }\n";
-        o << "    }\n  }\n";
-        if (scat)
-            o << "  if (S.D.nscat > 0) {\n"
-                 "    for (int e = 0; e < S.nsg; ++e) {\n"
-                 "      const int own = S.own[e];\n"
-                 "      if (own / Q != t) continue;\n"
-                 "#pragma unroll\n      for (int q = 0; q < Q; ++q) if (own == t * Q + q) acc[q] = fma(S.v[e], S.xv[e], acc[q]);\n"
-                 "    }\n"
-                 "    for (int e = 32; e < S.D.nscat; ++e) {\n"
-                 "      const int rr = __ldg(a.scat_row + S.D.scat_begin + e);\n"
-                 "      if (rr % NT != t) continue;\n"
-                 "      const T v = __ldg(a.scat_val + S.D.scat_begin + e), xv = __ldg(a.x + __ldg(a.scat_col + S.D.scat_begin + e));\n"
-                 "#pragma unroll\n      for (int q = 0; q < Q; ++q) if (rr / NT == q) acc[q] = fma(v, xv, acc[q]);\n"
-                 "    }\n  }\n";
-        o << "#pragma unroll\n  for (int q = 0; q < Q; ++q) {\n    const i64 r = row0 + t + q * NT;\n"
-             "    if (!edge || r < a.nrows) { T *yp = a.y + r; __stcs(yp, (a.beta != T(0)) ? fma(a.alpha, acc[q], a.beta * *yp) : a.alpha * acc[q]); }\n"
-             "  }\n}\n";
-        issue_sw << "      case " << key << ": pissue_" << key << "(a, D, row0, edge, vs, bar); break;\n";
-        comp_sw << "    case " << key << ": pcomp_" << key << "(a, S, edge, vk, bar + k, ph, t); break;\n";
-    }
-    // stage fill by warp 0 (lane = t < 32)
-    o << "__device__ __forceinline__ void pfill(const Args &a, i64 w, StageHdr *S, T *vs, u64 *bar, int lane) {\n"
-         "  const i64 s = a.seg_list ? (i64)__ldg(a.seg_list + w) : a.seg_begin + w;\n"
-         "  const SegDesc D = a.segs[s];\n  const i64 row0 = s * MROWS;\n  const bool edge = (D.flags & 1) != 0;\n"
-         "  if (lane == 0) {\n    S->D = D;\n    S->row0 = row0;\n    S->nsg = D.nscat < 32 ? D.nscat : 32;\n"
-         "    switch (D.plan_begin) {\n" << issue_sw.str() << "    }\n  }\n";
-    if (scat)
-        o << "  if (D.nscat > 0 && lane < D.nscat) {\n"
-             "    const ScatRec R = a.scat_rec[D.scat_begin + lane];\n"
-             "    S->own[lane] = (R.row % NT) * Q + R.row / NT;\n"
-             "    S->v[lane] = *reinterpret_cast<const T *>(&R.val);\n"
-             "    S->xv[lane] = __ldg(a.x + R.col);\n  }\n";
-    o << "}\n";
-    o << "extern \"C\" __global__ void __launch_bounds__(NT) crsd_jitp(const Args a, int stage_bytes) {\n"
-         "  extern __shared__ __align__(128) unsigned char smem[];\n  __shared__ u64 bar[2];\n"
-         "  const int t = threadIdx.x;\n"
-         "  if (t == 0) { bar_init(&bar[0]); bar_init(&bar[1]); }\n  __syncthreads();\n"
-         "  const i64 G = gridDim.x;\n"
-         "  if (t < 32)\n    for (int k = 0; k < 2; ++k) {\n      const i64 w = blockIdx.x + k * G;\n"
-         "      unsigned char *b = smem + k * stage_bytes;\n"
-         "      if (w < a.seg_count) pfill(a, w, reinterpret_cast<StageHdr *>(b), reinterpret_cast<T *>(b + HDR), bar + k, t);\n    }\n"
-         "  __syncthreads();\n"
-         "  u32 phs = 0u;  // bit k: phase of buffer k\n  int k = 0;\n"
-         "  for (i64 w = blockIdx.x; w < a.seg_count; w += G) {\n"
-         "    unsigned char *b = smem + k * stage_bytes;\n"
-         "    const StageHdr &S = *reinterpret_cast<const StageHdr *>(b);\n"
-         "    const T *vk = reinterpret_cast<const T *>(b + HDR);\n"
-         "    const u32 ph = (phs >> k) & 1u;\n"
-         "    const bool edge = (S.D.flags & 1) != 0;\n"
-         "    switch (S.D.plan_begin) {\n" << comp_sw.str() << "    }\n"
-         "    phs ^= 1u << k;\n    __syncthreads();\n"
-         "    if (t < 32 && w + 2 * G < a.seg_count)\n"
-         "      pfill(a, w + 2 * G, reinterpret_cast<StageHdr *>(b), reinterpret_cast<T *>(b + HDR), bar + k, t);\n"
-         "    k ^= 1;\n  }\n}\n";
-}
 
 // rows per thread of the generated kernel: <= 256 threads per CTA
 static int jit_q(const crsd_matrix_s *A) {
@@ -463,25 +235,174 @@ static int jit_q(const crsd_matrix_s *A) {
     return q;
 }
 
-// staging buffer of the persistent kernel: header + the largest staging
-static int64_t jitp_stage_bytes(const crsd_matrix_s *A) {
-    const int64_t hdr = (32 + 8 + 8 + 4 * 32 + 2 * 32 * (int64_t)A->H.elem + 127) / 128 * 128;
-    return (hdr + A->smem_bytes + 127) / 128 * 128;
+// Generate the codelets of every distinct pattern of A (one CTA per segment,
+// Q rows per thread) and the kernel that dispatches to them.
+static std::string generate(const crsd_matrix_s *A, int Q) {
+    const HostCRSD &H = A->H;
+    const bool f64 = H.dtype == CRSD_R64F;
+    const int m = H.mrows, nt = m / Q, es = H.elem;
+    const bool scat = H.nscatter() > 0;  // scatter code only for matrices that have scatter points
+    std::ostringstream o;
+    o << "typedef " << (f64 ? "double" : "float") << " T;\n" << kPrelude;
+    o << "#define MROWS " << m << "\n#define NT " << nt << "\n#define Q " << Q << "\n";
+    // one __device__ codelet per distinct pattern, keyed by the pattern's
+    // plan_begin (unique per distinct pattern; off_begin is not: a pattern
+    // without diagonals shares it with the next pattern)
+    std::vector<int32_t> seen;
+    int nbar = 1;
+    for (const Instance &I : H.inst) {
+        const int32_t key = A->segdesc[I.first_seg].plan_begin;
+        bool dup = false;
+        for (int32_t v : seen) dup |= (v == key);
+        if (dup) continue;
+        seen.push_back(key);
+        const int32_t *pl = A->plan.data() + key;
+        const int nd = (int)H.ndias(I.pattern), nwin = pl[0];
+        const int64_t *offs = H.pat_offsets.data() + H.pat_ptr[I.pattern];
+        const int32_t *xoff = pl + 2 + 2 * nwin;
+        std::vector<int64_t> wbase(nwin + 1, 0);
+        for (int w = 0; w < nwin; ++w) wbase[w + 1] = wbase[w] + pl[3 + 2 * w];
+        const std::vector<Chunk> ch = make_chunks(pl, nd, A->jit_chunk);
+        nbar = std::max(nbar, (int)ch.size());
+        o << "// pattern offsets:";
+        for (int d = 0; d < nd; ++d) o << " " << offs[d];
+        o << "\n// " << ch.size() << " staging chunk(s)\n";
+        o << "__device__ __forceinline__ void codelet_" << key
+          << "(const Args &a, const i64 s, const i64 vb, const i64 row0, const bool edge, T *vs, u64 *bar, const int t) {\n";
+        if (nd) {
+            // thread 0: every mbarrier, then every copy, chunk by chunk
+            o << "  T *xs = vs + " << (int64_t)nd * m << ";\n";
+            o << "  if (t == 0) {\n";
+            for (size_t c = 0; c < ch.size(); ++c) o << "    bar_init(bar + " << c << ");\n";
+            o << "    bar_fence_init();\n    const u64 pf = pol_first(), pn = pol_normal();\n";
+            for (size_t c = 0; c < ch.size(); ++c) {
+                const Chunk &k = ch[c];
+                const int64_t vbytes = (int64_t)(k.d1 - k.d0) * m * es;
+                int64_t xbytes = 0;
+                if (k.win == -2) xbytes = wbase[nwin] * es;
+                else if (k.win >= 0) xbytes = (int64_t)pl[3 + 2 * k.win] * es;
+                o << "    bar_expect(bar + " << c << ", " << vbytes << "u" << (xbytes ? " + (edge ? 0u : " : "")
+                  << (xbytes ? std::to_string(xbytes) + "u)" : "") << ");\n";
+                o << "    g2s(vs + " << (int64_t)k.d0 * m << ", a.vals + vb + " << (int64_t)k.d0 * m << ", " << vbytes
+                  << "u, bar + " << c << ", pf);\n";
+                if (xbytes) {
+                    o << "    if (!edge) {\n";
+                    for (int w = 0; w < nwin; ++w) {
+                        if (!(k.win == -2 || k.win == w)) continue;
+                        o << "      g2s(xs + " << wbase[w] << ", a.x + row0 + (" << pl[2 + 2 * w] << "), "
+                          << (int64_t)pl[3 + 2 * w] * es << "u, bar + " << c << ", pn);\n";
+                    }
+                    o << "    }\n";
+                }
+            }
+            o << "  }\n";
+        } else {
+            o << "  (void)vs; (void)bar; (void)vb;\n";
+        }
+        if (scat) {
+            // scatter points are gathered while the bulk copies are in flight:
+            // lane l of every warp reads record l of the segment's first 32
+            // (row, col, value in one 32-B record); a ballot keeps those whose
+            // row belongs to this warp, which alone load x[col]
+            o << "  const SegDesc *Dp = a.segs + s;\n  const int nscat = __ldg(&Dp->nscat);\n"
+                 "  const i64 sbeg = nscat > 0 ? __ldg(&Dp->scat_begin) : 0;\n"
+                 "  int g_own = -1; T g_v = T(0), g_x = T(0); unsigned g_mask = 0u;\n"
+                 "  if (nscat > 0) {\n"
+                 "    const int lane = t & 31;\n"
+                 "    ScatRec R; R.col = 0; R.val = 0; R.row = 0;\n"
+                 "    if (lane < nscat) { R = a.scat_rec[sbeg + lane]; g_own = (R.row % NT) * Q + R.row / NT; }\n"
+                 "    const bool mine = g_own >= 0 && (g_own / Q) / 32 == t / 32;\n"
+                 "    g_mask = __ballot_sync(0xffffffffu, mine);\n"
+                 "    if (mine) { g_v = *reinterpret_cast<const T *>(&R.val); g_x = __ldg(a.x + R.col); }\n"
+                 "  }\n";
+        }
+        if (nd) o << "  __syncthreads();\n";
+        o << "  T acc[Q];\n#pragma unroll\n  for (int q = 0; q < Q; ++q) acc[q] = T(0);\n";
+        // FMAs chunk by chunk, each after its own barrier; ascending offset
+        // order within and across chunks (the order of the paper's codelet)
+        o << "  if (!edge) {\n";
+        for (size_t c = 0; c < ch.size(); ++c) {
+            o << "    bar_wait(bar + " << c << ");\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n      const int r = t + q * NT;\n";
+            for (int d = ch[c].d0; d < ch[c].d1; ++d)
+                o << "      acc[q] = fma(vs[" << (int64_t)d * m << " + r], xs[" << xoff[d] << " + r], acc[q]);\n";
+            o << "    }\n";
+        }
+        o << "  } else {\n";
+        for (size_t c = 0; c < ch.size(); ++c) {
+            o << "    bar_wait(bar + " << c << ");\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n      const i64 r = row0 + t + q * NT;\n";
+            for (int d = ch[c].d0; d < ch[c].d1; ++d)
+                o << "      { const i64 i = r + (" << offs[d] << "); acc[q] = fma(vs[" << (int64_t)d * m
+                  << " + t + q * NT], (i >= a.x_lo && i < a.x_hi) ? __ldg(a.x + i) : T(0), acc[q]); }\n";
+            o << "    }\n";
+        }
+        o << "  }\n";
+        // scatter points in (row, col) order by their owner thread: the
+        // gathered ones (broadcast from the lane holding them), then any
+        // beyond the first 32; then the epilogue
+        if (scat)
+            o << "  if (nscat > 0) {\n"
+                 "    for (unsigned mm = g_mask; mm; mm &= mm - 1) {\n"
+                 "      const int j = __ffs(mm) - 1;\n"
+                 "      const int own = __shfl_sync(0xffffffffu, g_own, j);\n"
+                 "      const T v = __shfl_sync(0xffffffffu, g_v, j), xv = __shfl_sync(0xffffffffu, g_x, j);\n"
+                 "#pragma unroll\n      for (int q = 0; q < Q; ++q) if (own == t * Q + q) acc[q] = fma(v, xv, acc[q]);\n"
+                 "    }\n"
+                 "    for (int e = 32; e < nscat; ++e) {\n"
+                 "      const int rr = __ldg(a.scat_row + sbeg + e);\n"
+                 "      if (rr % NT != t) continue;\n"
+                 "      const T v = __ldg(a.scat_val + sbeg + e), xv = __ldg(a.x + __ldg(a.scat_col + sbeg + e));\n"
+                 "#pragma unroll\n      for (int q = 0; q < Q; ++q) if (rr / NT == q) acc[q] = fma(v, xv, acc[q]);\n"
+                 "    }\n  }\n";
+        // epilogue: y = alpha*acc + beta*y, y not read when beta == 0
+        o << "#pragma unroll\n  for (int q = 0; q < Q; ++q) {\n    const i64 r = row0 + t + q * NT;\n"
+             "    if (!edge || r < a.nrows) {\n      T *yp = a.y + r;\n"
+             "      __stcs(yp, (a.beta != T(0)) ? fma(a.alpha, acc[q], a.beta * *yp) : a.alpha * acc[q]);\n    }\n"
+             "  }\n}\n";
+    }
+    // Baked segment -> (pattern, value base) lookup and edge test, used for
+    // range launches (the one-GPU path and contiguous interiors); list
+    // launches read the descriptor. Off with CRSD_TUNE_JIT_DESC_ISSUE, or when
+    // the tables would be large.
+    std::vector<std::pair<int64_t, int64_t>> edges;  // [a, b) runs of edge segments
+    for (int64_t s = 0; s < H.nseg; ++s)
+        if (A->segdesc[s].flags & SEG_EDGE) {
+            if (!edges.empty() && edges.back().second == s) edges.back().second = s + 1;
+            else edges.push_back({s, s + 1});
+        }
+    const bool locate = !(A->tune & CRSD_TUNE_JIT_DESC_ISSUE) && !H.inst.empty() && H.inst.size() <= 4096 &&
+                        edges.size() <= 16;
+    o << "#define NBAR " << nbar << "\n";
+    if (locate) {
+        std::vector<Leaf> L;
+        for (const Instance &I : H.inst)
+            L.push_back({I.first_seg, H.ndias(I.pattern) * m, I.val_base, A->segdesc[I.first_seg].plan_begin});
+        o << "__device__ __forceinline__ void locate(const i64 s, int &key, i64 &vb) {\n";
+        emit_locate(o, L, 0, L.size(), 0);
+        o << "}\n__device__ __forceinline__ bool is_edge(const i64 s) {\n  return false";
+        for (const auto &e : edges) o << " || (s >= " << e.first << "LL && s < " << e.second << "LL)";
+        o << ";\n}\n";
+    }
+    o << "extern \"C\" __global__ void __launch_bounds__(NT) crsd_jit(const Args a) {\n"
+         "  extern __shared__ __align__(128) unsigned char smem[];\n  __shared__ u64 bar[NBAR];\n"
+         "  T *vs = reinterpret_cast<T *>(smem);\n  i64 s, vb;\n  int key;\n  bool edge;\n";
+    if (locate)
+        o << "  if (!a.seg_list) {\n    s = a.seg_begin + blockIdx.x;\n    locate(s, key, vb);\n    edge = is_edge(s);\n"
+             "  } else {\n";
+    else
+        o << "  {\n";
+    o << "    s = a.seg_list ? (i64)__ldg(a.seg_list + blockIdx.x) : a.seg_begin + blockIdx.x;\n"
+         "    const SegDesc D = a.segs[s];\n    key = D.plan_begin;\n    vb = D.val_base;\n    edge = (D.flags & 1) != 0;\n"
+         "  }\n  const i64 row0 = s * MROWS;\n  switch (key) {\n";
+    for (int32_t v : seen) o << "  case " << v << ": codelet_" << v << "(a, s, vb, row0, edge, vs, bar, threadIdx.x); break;\n";
+    o << "  }\n}\n";
+    return o.str();
 }
 
-std::string jit_generate(const crsd_matrix_s *A) {
-    std::string src = generate(A, jit_q(A));
-    std::ostringstream o;
-    generate_persistent(A, jit_q(A), o);
-    return src + o.str();
-}
+std::string jit_generate(const crsd_matrix_s *A) { return generate(A, jit_q(A)); }
 
 // Range launches on forked streams, concurrently (default), or one after the
-// other on the caller's stream (CRSD_JIT_CONCURRENT=0).
-static bool jit_concurrent() {
-    static const bool v = !(getenv("CRSD_JIT_CONCURRENT") && atoi(getenv("CRSD_JIT_CONCURRENT")) == 0);
-    return v;
-}
+// other on the caller's stream (CRSD_TUNE_JIT_SEQUENTIAL).
+static bool jit_concurrent(const crsd_matrix_s *A) { return !(A->tune & CRSD_TUNE_JIT_SEQUENTIAL); }
 
 // The kernel's dynamic shared memory is one number per launch, so a single
 // launch reserves the LARGEST pattern's staging for every CTA: on C4 the
@@ -489,16 +410,16 @@ static bool jit_concurrent() {
 // 11-diagonal rows too, which alone would fit 7-8 CTAs per SM. Instances are
 // contiguous segment ranges, so the one-GPU launch is split into runs of
 // instances with the same occupancy class, each launched with its own
-// staging size (see below for when it pays). CRSD_JIT_RANGES=0 disables
-// the split, =2 forces it at every class change (tests, sanitizer runs).
+// staging size (see below for when it pays). CRSD_TUNE_JIT_ONE_LAUNCH
+// disables the split, CRSD_TUNE_JIT_SPLIT_ALL forces it at every class
+// change (tests, sanitizer runs).
 static void jit_plan_ranges(crsd_matrix_s *A) {
     const HostCRSD &H = A->H;
     A->jit_ranges.clear();
     const int64_t nseg = H.nseg;
     const int64_t nt = H.mrows / jit_q(A);
-    const int mode = getenv("CRSD_JIT_RANGES") ? atoi(getenv("CRSD_JIT_RANGES")) : 1;
-    const bool off = mode == 0;
-    const bool force = mode == 2;  // testing: split at every class change, no folding, no cost rule
+    const bool off = (A->tune & CRSD_TUNE_JIT_ONE_LAUNCH) != 0;
+    const bool force = (A->tune & CRSD_TUNE_JIT_SPLIT_ALL) != 0;
     std::vector<int64_t> whole = {0, nseg, A->smem_bytes, 0};
     if (off || H.inst.empty()) {
         A->jit_ranges.push_back(whole);
@@ -511,7 +432,7 @@ static void jit_plan_ranges(crsd_matrix_s *A) {
         return el * H.elem;
     };
     auto occupancy = [&](int64_t b) {
-        const int64_t per_cta = (b + 127) / 128 * 128 + 1024 + 128;  // + driver reserve + static smem
+        const int64_t per_cta = (b + 127) / 128 * 128 + 1024 + 256;  // + driver reserve + static smem (barriers)
         return std::min<int64_t>(2048 / nt, (228 * 1024) / per_cta);
     };
     std::vector<std::vector<int64_t>> runs;
@@ -588,7 +509,7 @@ static void jit_plan_ranges(crsd_matrix_s *A) {
     // 1.005 split; C3 f32 (mrows 256) gains 15.3 MB against 33.3 MB (0.46)
     // and measured 1.044 -> 0.992 split, so it stays one launch; C4 f32
     // gains ~2 GB (1.013 -> 1.022 against the sequential split).
-    const double boundary_cost = jit_concurrent() ? 0.75 * wave : (double)(merged.size() - 1) * wave;
+    const double boundary_cost = jit_concurrent(A) ? 0.75 * wave : (double)(merged.size() - 1) * wave;
     if (merged.empty() || (!force && gain <= boundary_cost)) {
         A->jit_ranges.push_back(whole);
         return;
@@ -597,11 +518,10 @@ static void jit_plan_ranges(crsd_matrix_s *A) {
     A->jit_ranges = merged;
 }
 
-crsd_status_t jit_build(crsd_matrix_s *A) {
+// Generate and compile A's codelets for sm_100a (NVRTC only; no device needed).
+static crsd_status_t jit_compile(crsd_matrix_s *A) {
     NvrtcApi &nv = nvrtc();
     if (!nv.ok) return fail(CRSD_ERR_UNSUPPORTED, "JIT variant: " + nv.err);
-    DriverApi &dr = driver();
-    if (!dr.ok) return fail(CRSD_ERR_UNSUPPORTED, "JIT variant: driver entry point " + dr.err);
     if (A->smem_bytes > 200 * 1024) return fail(CRSD_ERR_UNSUPPORTED, "JIT variant: a segment's staging exceeds 200 KB");
     if (A->H.npat() > 256) return fail(CRSD_ERR_UNSUPPORTED, "JIT variant: more than 256 distinct patterns");
     A->jit_source = jit_generate(A);
@@ -620,12 +540,20 @@ crsd_status_t jit_build(crsd_matrix_s *A) {
     }
     size_t n = 0;
     nv.cubin_size(prog, &n);
-    std::vector<char> cubin(n);
-    nv.cubin(prog, cubin.data());
+    A->jit_cubin.resize(n);
+    nv.cubin(prog, A->jit_cubin.data());
     nv.destroy(&prog);
+    return CRSD_OK;
+}
+
+crsd_status_t jit_build(crsd_matrix_s *A) {
+    DriverApi &dr = driver();
+    if (!dr.ok) return fail(CRSD_ERR_UNSUPPORTED, "JIT variant: driver entry point " + dr.err);
+    crsd_status_t st = jit_compile(A);
+    if (st) return st;
     CUmodule mod;
     CUfunction fn;
-    if (dr.load(&mod, cubin.data()) != CUDA_SUCCESS) return fail(CRSD_ERR_CUDA, "cuModuleLoadData failed");
+    if (dr.load(&mod, A->jit_cubin.data()) != CUDA_SUCCESS) return fail(CRSD_ERR_CUDA, "cuModuleLoadData failed");
     if (dr.get_function(&fn, mod, "crsd_jit") != CUDA_SUCCESS) {
         dr.unload(mod);
         return fail(CRSD_ERR_CUDA, "cuModuleGetFunction(crsd_jit) failed");
@@ -635,19 +563,8 @@ crsd_status_t jit_build(crsd_matrix_s *A) {
         dr.unload(mod);
         return fail(CRSD_ERR_CUDA, "cuFuncSetAttribute failed");
     }
-    // persistent form: usable when two staging buffers fit one CTA
-    CUfunction fnp = nullptr;
-    const int64_t pbytes = 2 * jitp_stage_bytes(A);
-    if (pbytes <= 220 * 1024 && dr.get_function(&fnp, mod, "crsd_jitp") == CUDA_SUCCESS) {
-        if (pbytes > 48 * 1024 &&
-            dr.set_attr(fnp, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)pbytes) != CUDA_SUCCESS)
-            fnp = nullptr;
-    } else {
-        fnp = nullptr;
-    }
     A->jit_module = mod;
     A->jit_function = fn;
-    A->jitp_function = fnp;
     jit_plan_ranges(A);
     return CRSD_OK;
 }
@@ -665,7 +582,6 @@ void jit_free(crsd_matrix_s *A) {
     if (A->jit_module && driver().ok) driver().unload((CUmodule)A->jit_module);
     A->jit_module = nullptr;
     A->jit_function = nullptr;
-    A->jitp_function = nullptr;
 }
 
 template <typename T>
@@ -686,47 +602,31 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
     j.scat_col = s.scat_col;
     j.scat_val = s.scat_val;
     j.scat_rec = s.scat_rec;
-    j.dot_part = s.dot_part;
-    j.dot_cnt = s.dot_cnt;
-    j.dot_out = s.dot_out;
     j.alpha = s.alpha;
     j.beta = s.beta;
     const unsigned nt = (unsigned)(A->H.mrows / jit_q(A));
-    CUresult r;
-    // persistent form (CRSD_JIT_MODE=persist, or A->jit_persist): no fused dot
-    const char *mode = getenv("CRSD_JIT_MODE");
-    const bool persist = A->jitp_function && !s.dot_part &&
-                         (mode ? std::string(mode) == "persist" : A->jit_persist);
-    if (persist) {
-        int stage = (int)jitp_stage_bytes(A);
-        const int64_t per_cta = 2 * (int64_t)stage + 1024 + 64;
-        int64_t per_sm = std::min<int64_t>(2048 / nt, (228 * 1024) / per_cta);
-        per_sm = std::min<int64_t>(per_sm, 65536 / (32 * (int64_t)nt));
-        if (per_sm < 1) per_sm = 1;
-        int64_t grid = std::min<int64_t>(s.seg_count, per_sm * A->sm_count);
-        void *pp[] = {&j, &stage};
-        r = driver().launch((CUfunction)A->jitp_function, (unsigned)grid, 1, 1, nt, 1, 1, (unsigned)(2 * stage),
-                            (CUstream)stream, pp, nullptr);
-    } else if (!s.seg_list && !s.dot_part && A->jit_ranges.size() > 1) {
+    if (!s.seg_list && A->jit_ranges.size() > 1) {
         // a segment range (the whole matrix, or a contiguous interior):
-        // one launch per occupancy class it meets (jit_plan_ranges)
-        // Concurrent mode (default, CRSD_JIT_CONCURRENT=1): every range on
-        // its own forked stream, all joined at the end -- the ranges are
-        // independent (disjoint rows), so no launch waits for another's
-        // drain and their tails overlap. Sequential mode (=0): the main
+        // one launch per occupancy class it meets (jit_plan_ranges).
+        // Concurrent mode (default): every range on its own forked stream,
+        // all joined at the end -- the ranges are independent (disjoint
+        // rows), so no launch waits for another's drain and their tails
+        // overlap. Sequential mode (CRSD_TUNE_JIT_SEQUENTIAL): the main
         // ranges one after the other on `stream`, aux runs on a forked stream.
         int n = 0;
         const int64_t b0 = s.seg_begin, b1 = s.seg_begin + s.seg_count;
         crsd_matrix_s *M = const_cast<crsd_matrix_s *>(A);
-        const bool conc = jit_concurrent();
+        const bool conc = jit_concurrent(A);
         int next = 0, nstreams = 0;
         auto pool_stream = [&](int i) -> CUstream {
             while ((int)M->jit_pool.size() <= i) {
                 cudaStream_t as;
                 cudaEvent_t ej;
-                if (cudaStreamCreateWithFlags(&as, cudaStreamNonBlocking) != cudaSuccess ||
-                    cudaEventCreateWithFlags(&ej, cudaEventDisableTiming) != cudaSuccess)
+                if (cudaStreamCreateWithFlags(&as, cudaStreamNonBlocking) != cudaSuccess) return nullptr;
+                if (cudaEventCreateWithFlags(&ej, cudaEventDisableTiming) != cudaSuccess) {
+                    cudaStreamDestroy(as);
                     return nullptr;
+                }
                 M->jit_pool.push_back(as);
                 M->jit_ev_join.push_back(ej);
             }
@@ -741,6 +641,16 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
                 return nullptr;
             return (CUstream)M->jit_pool[i];
         };
+        // join every forked stream used so far back into `stream` (also on
+        // the error path, so later work on `stream` -- or a graph capture --
+        // stays ordered after the launches already made)
+        auto join = [&]() -> bool {
+            bool ok = true;
+            for (int i = 0; i < nstreams; ++i)
+                ok &= cudaEventRecord((cudaEvent_t)M->jit_ev_join[i], (cudaStream_t)M->jit_pool[i]) == cudaSuccess &&
+                      cudaStreamWaitEvent((cudaStream_t)stream, (cudaEvent_t)M->jit_ev_join[i], 0) == cudaSuccess;
+            return ok;
+        };
         for (int pass = 0; pass < 2; ++pass) {
             for (const std::vector<int64_t> &rg : A->jit_ranges) {
                 if (rg[3] != (pass == 0 ? 1 : 0)) continue;
@@ -754,29 +664,29 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
                     if (i < nstreams) {
                         st = (CUstream)M->jit_pool[i];
                     } else {
-                        if ((st = pool_stream(i)) == nullptr) return -(int)cudaErrorLaunchFailure;
+                        if ((st = pool_stream(i)) == nullptr) {
+                            join();
+                            return -(int)cudaErrorLaunchFailure;
+                        }
                         nstreams = i + 1;
                     }
                 }
                 j.seg_begin = lo;
                 j.seg_count = hi - lo;
                 void *params[] = {&j};
-                r = driver().launch((CUfunction)A->jit_function, (unsigned)(hi - lo), 1, 1, nt, 1, 1,
-                                    (unsigned)rg[2], st, params, nullptr);
-                if (r != CUDA_SUCCESS) return -(int)cudaErrorLaunchFailure;
+                if (driver().launch((CUfunction)A->jit_function, (unsigned)(hi - lo), 1, 1, nt, 1, 1, (unsigned)rg[2],
+                                    st, params, nullptr) != CUDA_SUCCESS) {
+                    join();
+                    return -(int)cudaErrorLaunchFailure;
+                }
                 ++n;
             }
         }
-        for (int i = 0; i < nstreams; ++i)
-            if (cudaEventRecord((cudaEvent_t)M->jit_ev_join[i], (cudaStream_t)M->jit_pool[i]) != cudaSuccess ||
-                cudaStreamWaitEvent((cudaStream_t)stream, (cudaEvent_t)M->jit_ev_join[i], 0) != cudaSuccess)
-                return -(int)cudaErrorLaunchFailure;
-        return n;
-    } else {
-        void *params[] = {&j};
-        r = driver().launch((CUfunction)A->jit_function, (unsigned)s.seg_count, 1, 1, nt, 1, 1,
-                            (unsigned)A->smem_bytes, (CUstream)stream, params, nullptr);
+        return join() ? n : -(int)cudaErrorLaunchFailure;
     }
+    void *params[] = {&j};
+    const CUresult r = driver().launch((CUfunction)A->jit_function, (unsigned)s.seg_count, 1, 1, nt, 1, 1,
+                                       (unsigned)A->smem_bytes, (CUstream)stream, params, nullptr);
     return r == CUDA_SUCCESS ? 1 : -(int)cudaErrorLaunchFailure;
 }
 
@@ -796,5 +706,16 @@ extern "C" crsd_status_t crsd_jit_source(crsd_matrix_t A, char *buf, int64_t cap
         std::memcpy(buf, src.data(), n);
         buf[n] = 0;
     }
+    return CRSD_OK;
+}
+
+extern "C" crsd_status_t crsd_jit_cubin(crsd_matrix_t A, void *buf, int64_t cap, int64_t *len) {
+    if (!A || !len) return crsd::fail(CRSD_ERR_INVALID_ARG, "NULL argument");
+    if (A->jit_cubin.empty()) {
+        const crsd_status_t st = crsd::jit_compile(A);
+        if (st) return st;
+    }
+    *len = (int64_t)A->jit_cubin.size();
+    if (buf && cap > 0) std::memcpy(buf, A->jit_cubin.data(), std::min<int64_t>(cap, *len));
     return CRSD_OK;
 }

@@ -50,8 +50,7 @@ inline int64_t up256(int64_t b) { return (b + 255) / 256 * 256; }
 
 struct Ws {
     CgState *st;
-    double *partials, *hist, *dpart;  // dpart: per segment + per group of 256 (dot fused into the SpMV)
-    uint32_t *dcnt;                    // its counters: one per group + one
+    double *partials, *hist;
     char *r, *q, *p_pad;  // p_pad: halo_lo + n + halo_hi elements
 };
 
@@ -60,10 +59,7 @@ crsd_status_t workspace(crsd_matrix_s *A, int64_t max_iter, int grid, Ws &w) {
     const int64_t npad = A->halo_lo + n + A->halo_hi;
     const int64_t o_part = up256(sizeof(CgState));
     const int64_t o_hist = o_part + up256(8 * (int64_t)grid);
-    const int64_t ngrp = (A->H.nseg + 255) / 256;
-    const int64_t o_dp = o_hist + up256(8 * (max_iter + 1));
-    const int64_t o_dc = o_dp + up256(8 * (A->H.nseg + ngrp + 1));
-    const int64_t o_r = o_dc + up256(4 * (ngrp + 1));
+    const int64_t o_r = o_hist + up256(8 * (max_iter + 1));
     const int64_t o_q = o_r + up256(es * n);
     const int64_t o_p = o_q + up256(es * n);
     const int64_t total = o_p + up256(es * npad);
@@ -88,8 +84,6 @@ crsd_status_t workspace(crsd_matrix_s *A, int64_t max_iter, int grid, Ws &w) {
     w.st = (CgState *)b;
     w.partials = (double *)(b + o_part);
     w.hist = (double *)(b + o_hist);
-    w.dpart = (double *)(b + o_dp);
-    w.dcnt = (uint32_t *)(b + o_dc);
     w.r = b + o_r;
     w.q = b + o_q;
     w.p_pad = b + o_p;
@@ -123,14 +117,12 @@ crsd_status_t cg_impl(crsd_matrix_s *A, const T *b, T *x, int32_t max_iter, doub
     int launches = 0;
     auto spmv = [&](T al, T be, T *y) -> crsd_status_t {
         if (comm) {
-            // boundary placement as crsd_spmv_dist's default (concurrent with
-            // the interior); CRSD_CG_BOUNDARY=1 forces the serial form, =0 the
-            // concurrent one. Under MPS (ranks sharing one GPU) the CG is
-            // bimodal: one run favoured serial 2-3x, the next concurrent 2x
-            // (profiles/r01_ab_boundary_cg_*, r01_ab_cg_*), so the default
-            // follows the SpMV measurement and the no-serial-tail argument.
-            static const int cg_boundary = getenv("CRSD_CG_BOUNDARY") ? atoi(getenv("CRSD_CG_BOUNDARY")) : -1;
-            ST_TRY(spmv_dist_impl(A, &al, w.p_pad, &be, y, comm, s, cg_boundary));
+            // boundary placement as crsd_spmv_dist (the handle's
+            // CRSD_TUNE_DIST_BOUNDARY_SERIAL). Under MPS (ranks sharing one
+            // GPU) the CG is bimodal: one run favoured serial 2-3x, the next
+            // concurrent 2x (profiles/r01_ab_boundary_cg_*, r01_ab_cg_*), so the
+            // default follows the SpMV measurement and the no-serial-tail argument.
+            ST_TRY(spmv_dist_impl(A, &al, w.p_pad, &be, y, comm, s, -1));
             launches += A->last_launches;
             return CRSD_OK;
         }
@@ -162,23 +154,13 @@ crsd_status_t cg_impl(crsd_matrix_s *A, const T *b, T *x, int32_t max_iter, doub
     if (comm) ST_TRY(comm_allreduce_f64(comm, w.st->red + CG_RR, 2, s));
     ST_TRY(kerr(cg_launch_init(w.st, s), "cg_init"));
 
-    // One GPU with the JIT variant: (p, q) is fused into the SpMV epilogue
-    // (saves one read of p and of q per step); otherwise a separate kernel.
-    // Off by default: the reduction epilogue lengthens every SpMV CTA's life
-    // (fewer bytes in flight), which costs more than the two vector passes it
-    // saves (C2 f64 0.417 vs 0.407 ms/step, f32 equal; profiles/r01_cg_ab.jsonl).
-    // CRSD_CG_FUSED_DOT=1 enables it.
-    const bool fused = !comm && A->variant == VARIANT_JIT && getenv("CRSD_CG_FUSED_DOT") &&
-                       atoi(getenv("CRSD_CG_FUSED_DOT")) != 0;
-    DotArgs dot{w.dpart, w.dcnt, w.st->red + CG_PQ};
+    // (p, q) is a separate kernel. Fusing it into the SpMV epilogue (round 1,
+    // removed) saved two vector passes but lengthened every SpMV CTA's life
+    // (fewer bytes in flight): C2 f64 0.417 vs 0.407 ms/step, f32 equal
+    // (profiles/r01_cg_ab.jsonl).
     auto step = [&]() -> crsd_status_t {
-        if (fused) {
-            const T one(1), zero(0);
-            ST_TRY(run_lists(A, &one, p_own, &zero, q, nullptr, 0, nseg, s, launches, &dot));  // q = A p, (p, q)
-        } else {
-            ST_TRY(spmv(T(1), T(0), q));  // q = A p
-            ST_TRY(kerr(cg_launch_dot<T>(p_own, q, n, w.st, CG_PQ, true, grid, s), "cg_dot(p,q)"));
-        }
+        ST_TRY(spmv(T(1), T(0), q));  // q = A p
+        ST_TRY(kerr(cg_launch_dot<T>(p_own, q, n, w.st, CG_PQ, true, grid, s), "cg_dot(p,q)"));
         if (comm) ST_TRY(comm_allreduce_f64(comm, w.st->red + CG_PQ, 1, s));
         ST_TRY(kerr(cg_launch_update<T>(r, q, n, w.st, grid, s), "cg_update"));
         if (comm) ST_TRY(comm_allreduce_f64(comm, w.st->red + CG_RR, 1, s));
@@ -193,13 +175,11 @@ crsd_status_t cg_impl(crsd_matrix_s *A, const T *b, T *x, int32_t max_iter, doub
     cudaGraphExec_t exec = nullptr;
     int graph_launches = 0;
     for (int64_t issued = 0; !done && issued < max_iter; issued += batch) {
-        // One batch of steps as a CUDA graph (CRSD_CG_NO_GRAPH=1: direct
-        // launches, for A/B runs): one GPU, or the peer-memory
+        // One batch of steps as a CUDA graph: one GPU, or the peer-memory
         // transport (its exchange and allreduce kernels keep their epochs on
         // the device, so a replay is a new exchange). NCCL calls are issued
         // directly.
-        static const bool no_graph = getenv("CRSD_CG_NO_GRAPH") && atoi(getenv("CRSD_CG_NO_GRAPH"));
-        if (!no_graph && (!comm || comm->kind == crsd_comm_s::P2P)) {
+        if (!comm || comm->kind == crsd_comm_s::P2P) {
             if (!exec) {
                 const int l0 = launches;
                 cudaGraph_t g;

@@ -29,6 +29,7 @@
 #include <algorithm>
 #include <cstdint>
 #include <cstdlib>
+#include <mutex>
 
 #include "crsd_internal.h"
 
@@ -691,9 +692,21 @@ inline int64_t pipe_smem(int ns, int nx, int kch, int mrows, int elem, int64_t x
     return bars + segs + recs + nx * xmax_elems * elem + (int64_t)ns * kch * mrows * elem;
 }
 
-static int env_int(const char *k, int d) {
-    const char *v = getenv(k);
-    return v ? atoi(v) : d;
+// cudaFuncSetAttribute(MaxDynamicSharedMemorySize) applies per device
+// context: remember the largest size set, per device and kernel instance.
+constexpr int kMaxDev = 64;
+static std::mutex g_attr_mu;
+template <typename K>
+static cudaError_t ensure_smem(K kern, int bytes, int *cache_per_dev) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    if (dev < 0 || dev >= kMaxDev) return cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    std::lock_guard<std::mutex> lk(g_attr_mu);
+    if (bytes <= cache_per_dev[dev]) return cudaSuccess;
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    if (e == cudaSuccess) cache_per_dev[dev] = bytes;
+    return e;
 }
 
 template <typename T>
@@ -709,17 +722,13 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
         const int rc = a.mrows / split;
         const int thr = rc / q;
         const int smem = (int)a.tma_smem;
-        static int attr_bytes[2][3][2] = {};
+        static int attr_bytes[3][2][kMaxDev] = {};
         const int qi = q == 1 ? 0 : (q == 2 ? 1 : 2);
         const bool sc = a.has_scatter != 0;
-        int &cur = attr_bytes[sizeof(T) == 8][qi][sc];
         auto kern = sc ? (q == 1 ? crsd_spmv_tma<T, 1, true> : (q == 2 ? crsd_spmv_tma<T, 2, true> : crsd_spmv_tma<T, 4, true>))
                        : (q == 1 ? crsd_spmv_tma<T, 1, false> : (q == 2 ? crsd_spmv_tma<T, 2, false> : crsd_spmv_tma<T, 4, false>));
-        if (smem > cur) {
-            e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-            if (e != cudaSuccess) return -(10000 + (int)e);
-            cur = smem;
-        }
+        e = ensure_smem(kern, smem, attr_bytes[qi][sc]);
+        if (e != cudaSuccess) return -(10000 + (int)e);
         int64_t g = a.seg_count * split;
         if (g > 0x7fffffff) g = 0x7fffffff;
         kern<<<(unsigned)g, thr, smem, (cudaStream_t)stream>>>(a, split);
@@ -729,24 +738,19 @@ int launch_spmv(const SpmvArgs<T> &a, int sm_count, void *stream) {
         // stages as fit
         constexpr int kch = 8;
         const int64_t xmax = a.pipe_xmax_elems;
-        const int q = env_int("CRSD_PIPE_Q", a.mrows > 256 ? a.mrows / 256 : 1);
+        const int q = a.mrows > 256 ? a.mrows / 256 : 1;
         const int C = a.mrows / q;
-        const int per_sm = env_int("CRSD_PIPE_PERSM", C <= 256 ? 2 : 1);
+        const int per_sm = C <= 256 ? 2 : 1;
         const int64_t budget = (per_sm >= 2 ? 110 : 220) * 1024;
-        int nx = env_int("CRSD_PIPE_NX", 2);
-        while (nx > 2 && pipe_smem(2, nx, kch, a.mrows, sizeof(T), xmax) > budget) --nx;
-        int ns = env_int("CRSD_PIPE_NS", 32);
+        const int nx = 2;
+        int ns = 32;
         while (ns > 2 && pipe_smem(ns, nx, kch, a.mrows, sizeof(T), xmax) > budget) --ns;
         const int64_t sm = pipe_smem(ns, nx, kch, a.mrows, sizeof(T), xmax);
-        static int attr_pipe[2][3] = {};
+        static int attr_pipe[3][kMaxDev] = {};
         const int qi = q == 1 ? 0 : (q == 2 ? 1 : 2);
-        int &cur = attr_pipe[sizeof(T) == 8][qi];
         auto kern = q == 1 ? crsd_spmv_pipe<T, kch, 1> : (q == 2 ? crsd_spmv_pipe<T, kch, 2> : crsd_spmv_pipe<T, kch, 4>);
-        if (sm > cur) {
-            e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-            if (e != cudaSuccess) return -(10000 + (int)e);
-            cur = (int)sm;
-        }
+        e = ensure_smem(kern, (int)sm, attr_pipe[qi]);
+        if (e != cudaSuccess) return -(10000 + (int)e);
         int64_t g = (int64_t)sm_count * per_sm;
         if (g > a.seg_count) g = a.seg_count;
         kern<<<(unsigned)g, C + 32, sm, (cudaStream_t)stream>>>(a, ns, nx, (int)xmax);

@@ -5,8 +5,7 @@ C2 grid (7-point Dirichlet Laplacian, SPD) at n^3, fixed K steps (rtol 0),
 timed with CUDA events around crsd_cg (one graph replay per check_every
 steps, device-side scalars). Bytes per step: the SpMV's unique bytes plus the
 vector traffic of the three vector kernels ((p,q): 2 reads; r update: 2
-reads + 1 write; x and p update: 3 reads + 2 writes = 10 vectors; 8 when
-(p,q) is fused into the JIT SpMV's epilogue).
+reads + 1 write; x and p update: 3 reads + 2 writes = 10 vectors).
 usage: python scripts/cg_bench.py [n] [K] [f64|f32]
 """
 import json
@@ -41,10 +40,9 @@ e.synchronize()
 ms = s.elapsed_time(e)
 es = np.dtype(dt).itemsize
 inf = A.info()
-fused = inf["variant"] == 4 and os.environ.get("CRSD_CG_FUSED_DOT", "0") != "0"
-step_bytes = inf["unique_bytes_beta0"] + (8 if fused else 10) * N * es
+step_bytes = inf["unique_bytes_beta0"] + 10 * N * es
 per = ms / res["iterations"]
 print(json.dumps({"workload": f"CG 7-pt {n}^3 {np.dtype(dt).name}", "variant": inf["variant"], "steps": res["iterations"],
                   "ms_per_step": round(per, 5), "GBps": round(step_bytes / (per * 1e-3) / 1e9, 1),
                   "spmv_bytes": inf["unique_bytes_beta0"], "step_bytes": step_bytes,
-                  "launches": res["launches"], "fused_dot": fused, "rr_ratio": res["rr"] / res["rr0"]}), flush=True)
+                  "launches": res["launches"], "rr_ratio": res["rr"] / res["rr0"]}), flush=True)

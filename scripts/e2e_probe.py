@@ -11,8 +11,7 @@ a, _, _, _ = bench.workload("c2", "f64", 1, 0)
 xh = torch.from_numpy(np.random.default_rng(7).uniform(-1, 1, a.ncols)).pin_memory()
 yh = torch.empty(a.nrows, dtype=torch.float64).pin_memory()
 for ch in sys.argv[1:] or ["8", "16", "32", "64"]:
-    os.environ["CRSD_E2E_CHUNKS"] = ch
-    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val)
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, e2e_chunks=int(ch))
     for _ in range(3):
         A.spmv_host_ptr(xh.data_ptr(), yh.data_ptr())
     t0 = time.perf_counter()

@@ -41,12 +41,13 @@ def main():
                 print(f"{name} {np.dtype(dt).name} variant {v}: parity {err:.2e} {'ok' if ok else 'FAIL'}", flush=True)
     # JIT launches split by occupancy class (forced on a small C4: several
     # ranges with their own dynamic smem)
-    os.environ["CRSD_JIT_RANGES"] = "2"
+    from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_SPLIT_ALL
+
     for dt in (np.float64, np.float32):
         b = gen.config4(n=400_000).astype(dt)
         x = np.random.default_rng(1).uniform(-1, 1, b.ncols).astype(dt)
         yref, sc = coo.coo_spmv(b.nrows, b.ncols, b.row, b.col, b.val, x)
-        A = CRSDMatrix.from_coo(b.nrows, b.ncols, b.row, b.col, b.val, variant=4, mrows=512)
+        A = CRSDMatrix.from_coo(b.nrows, b.ncols, b.row, b.col, b.val, variant=4, mrows=512, tune=TUNE_JIT_SPLIT_ALL)
         tdt = torch.float64 if dt == np.float64 else torch.float32
         xd = torch.from_numpy(x).to("cuda", tdt)
         yd = torch.full((b.nrows,), float("nan"), device="cuda", dtype=tdt)
@@ -56,7 +57,6 @@ def main():
         ok = err <= (1e-12 if dt == np.float64 else 1e-5) and A.last_launch_count() > 1
         bad += not ok
         print(f"c4 ranges {np.dtype(dt).name}: {A.last_launch_count()} launches, parity {err:.2e} {'ok' if ok else 'FAIL'}", flush=True)
-    os.environ.pop("CRSD_JIT_RANGES")
     # CG (vector kernels, grid reductions, graph replay) on an SPD stencil
     from oracle import cg_ref
 

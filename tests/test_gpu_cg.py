@@ -187,19 +187,3 @@ def _one_rank_cg(torch, Comm, CRSDMatrix):
     torch.cuda.synchronize()
     _compare(a, np.float64, b, x0, res, xd.cpu().numpy())
     comm.close()
-
-
-@pytest.mark.parametrize("dt", [np.float64, np.float32])
-@pytest.mark.parametrize("case", ["7pt", "7pt+scatter"])
-def test_cg_fused_dot_option(torch_cuda, case, dt, monkeypatch):
-    """CRSD_CG_FUSED_DOT=1: (p, q) reduced in the JIT SpMV's epilogue
-    (two-level deterministic reduction) must give the same iteration."""
-    monkeypatch.setenv("CRSD_CG_FUSED_DOT", "1")
-    a = CASES[case]()
-    rng = np.random.default_rng(14)
-    b = rng.uniform(-1, 1, a.nrows)
-    x0 = rng.uniform(-0.5, 0.5, a.nrows)
-    A, res, x = _solve(torch_cuda, a, dt, b, x0, 60, check_every=9, variant=4)
-    assert res["iterations"] == 60
-    assert res["launches"] < 4 * 60 + 10  # 3 launches per step: the separate dot kernel is gone
-    _compare(a, dt, b, x0, res, x)

@@ -108,12 +108,15 @@ def test_c4_reduced_parity(torch_cuda, variant):
 
 
 @pytest.mark.parametrize("dt,alpha,beta", [(np.float32, 1.0, 0.0), (np.float64, -0.75, 0.5)])
-def test_jit_occupancy_ranges(torch_cuda, dt, alpha, beta, monkeypatch):
+def test_jit_occupancy_ranges(torch_cuda, dt, alpha, beta):
     """C4's four row-range patterns (19 / 11 / 9 / 9 diagonals) need 4, 7 and
     8 CTAs-per-SM staging sizes: the one-GPU JIT launch is split into one
     launch per occupancy class (jit_plan_ranges), each with its own dynamic
     shared memory. Every range must reproduce the oracle, with alpha/beta;
-    CRSD_JIT_RANGES=0 (one launch) must give the same bits."""
+    CRSD_TUNE_JIT_ONE_LAUNCH (one launch) and CRSD_TUNE_JIT_SEQUENTIAL (the
+    ranges one after another) must give the same bits."""
+    from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_ONE_LAUNCH, TUNE_JIT_SEQUENTIAL
+
     # 8M rows: long enough that the split pays under jit_plan_ranges' rule
     # (the gain grows with the rows, the boundary cost is one wave)
     a = gen.config4(n=8_000_000)
@@ -123,11 +126,14 @@ def test_jit_occupancy_ranges(torch_cuda, dt, alpha, beta, monkeypatch):
     x = rng.uniform(-1, 1, a.ncols).astype(dt)
     y0 = rng.uniform(-1, 1, a.nrows).astype(dt)
     y1 = _run(torch_cuda, A, x, alpha, beta, y0, a.nrows)
-    monkeypatch.setenv("CRSD_JIT_RANGES", "0")
-    B = _mat(a.astype(dt), variant=4, mrows=512)
+    B = _mat(a.astype(dt), variant=4, mrows=512, tune=TUNE_JIT_ONE_LAUNCH)
     y2 = _run(torch_cuda, B, x, alpha, beta, y0, a.nrows)
     assert B.last_launch_count() == 1
     assert np.array_equal(y1, y2)
+    C = _mat(a.astype(dt), variant=4, mrows=512, tune=TUNE_JIT_SEQUENTIAL)
+    y3 = _run(torch_cuda, C, x, alpha, beta, y0, a.nrows)
+    assert C.last_launch_count() > 1
+    assert np.array_equal(y1, y3)
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
@@ -555,10 +561,15 @@ def test_full_size_device_roundtrip(torch_cuda, case):
 
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
 @pytest.mark.parametrize("case", ["c1", "c2s", "c3s", "c4s", "rand0", "rand1", "rand2", "dense_scatter"])
-def test_jit_persistent_parity(torch_cuda, case, dt, monkeypatch):
-    """The persistent double-buffered JIT form (crsd_jitp, CRSD_JIT_MODE=persist):
-    every CTA loops over several segments through two staging buffers."""
-    monkeypatch.setenv("CRSD_JIT_MODE", "persist")
+def test_jit_staging_chunks_and_issue(torch_cuda, case, dt):
+    """The JIT codelet's staging chunks (opts.jit_chunk: one mbarrier per x
+    window by default, the whole segment on one barrier, or windows split into
+    runs of k diagonals) and its copy issue (baked instance lookup by default,
+    CRSD_TUNE_JIT_DESC_ISSUE: after the descriptor load) change only when the
+    FMAs start, never their order: every setting matches the oracle and all
+    settings give the same bits."""
+    from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_DESC_ISSUE
+
     if case == "c1":
         a = gen.config1()
     elif case == "c2s":
@@ -572,8 +583,20 @@ def test_jit_persistent_parity(torch_cuda, case, dt, monkeypatch):
     else:
         s = int(case[-1])
         a = gen.random_diagonal(4000 + 97 * s, 3900, 30 + s, ndiag=12, max_off=900, p_break=0.02, max_break=400, n_scatter=200)
-    for alpha, beta in ((1.0, 0.0), (-0.75, 0.5)):
-        _parity(torch_cuda, a, dt, alpha, beta, seed=3, variant=4)
+    a = a.astype(dt)
+    rng = np.random.default_rng(3)
+    x = rng.uniform(-1, 1, a.ncols).astype(dt)
+    y0 = rng.uniform(-1, 1, a.nrows).astype(dt)
+    yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, x, -0.75, 0.5, y0)
+    first = None
+    for chunk in (0, -1, 1, 5):
+        for tune in (0, TUNE_JIT_DESC_ISSUE):
+            A = _mat(a, variant=4, jit_chunk=chunk, tune=tune)
+            y = _run(torch_cuda, A, x, -0.75, 0.5, y0, a.nrows)
+            assert coo.parity_error(y, yref, scale) <= TOL[dt], (chunk, tune)
+            if first is None:
+                first = y
+            assert np.array_equal(y, first), (chunk, tune)
 
 
 @pytest.mark.parametrize("dt", [np.float64, np.float32])

@@ -5,8 +5,13 @@ Each oracle function is checked against something other than itself:
                    P:L503-511), grouping example,
                    DIA special case (P:L81-95 textbook DIA), presence-rule edge
                    cases worked by hand
-  coo           -- dense brute-force product (numpy longdouble), scipy.sparse,
-                   stencil closed forms (exact integers)
+  coo           -- coo_spmv: dense brute-force product (numpy longdouble),
+                   scipy.sparse, stencil closed forms (exact integers);
+                   rows_spmv: dense brute force on shuffled row samples (first,
+                   last, empty rows; beta != 0), bitwise against coo_spmv,
+                   closed forms; parity_error: hand-worked cases; coo_spmv_native:
+                   summation bound vs the definition, thread-count invariance,
+                   closed forms
   closed_forms  -- interior values stated in SURVEY.md §8(c) (0, 0, -4/-6/-54)
   decode        -- round trip of the paper-order construction, and corrupted
                    layouts that must be rejected
@@ -231,6 +236,133 @@ def test_coo_spmv_beta_zero_never_reads_y():
 def test_coo_spmv_rejects_out_of_range():
     with pytest.raises(ValueError):
         coo.coo_spmv(2, 2, np.array([0]), np.array([2]), np.array([1.0]), np.ones(2))
+
+
+# ---------------------------------------------------------------- rows_spmv (sampled rows)
+def _csr(a):
+    """Row-sorted copy and its row pointer (the layout rows_spmv reads)."""
+    order = np.lexsort((a.col, a.row))
+    r, c, v = a.row[order], a.col[order], a.val[order]
+    ptr = np.zeros(a.nrows + 1, np.int64)
+    ptr[1:] = np.cumsum(np.bincount(r, minlength=a.nrows))
+    return r, c, v, ptr
+
+
+@pytest.mark.parametrize("seed", range(5))
+@pytest.mark.parametrize("alpha,beta", [(1.0, 0.0), (-0.75, 0.5)])
+def test_rows_spmv_vs_dense_bruteforce(seed, alpha, beta):
+    """rows_spmv on a shuffled row subset (first and last rows and rows with no
+    entries included) against the dense long-double product: a row_ptr
+    off-by-one, or y0 indexed by the sample position instead of the row,
+    fails here."""
+    rng = np.random.default_rng(100 + seed)
+    n, m = int(rng.integers(8, 64)), int(rng.integers(8, 64))
+    a = gen.random_diagonal(n, m, seed, ndiag=5, n_scatter=4)
+    # empty out a few rows entirely
+    empty = rng.choice(n, size=3, replace=False)
+    keep = ~np.isin(a.row, empty)
+    a = gen.COO(n, m, a.row[keep], a.col[keep], a.val[keep])
+    r, c, v, ptr = _csr(a)
+    x = rng.uniform(-1, 1, m)
+    y0 = rng.uniform(-1, 1, n)
+    sel = np.unique(np.concatenate([[0, n - 1], empty, rng.integers(0, n, 10)]))
+    sel = sel[rng.permutation(sel.shape[0])]  # sample order != row order
+    y, sc = coo.rows_spmv(sel, ptr, c, v, x, alpha, beta, y0)
+    ref = _dense_longdouble(a, x, alpha, beta, y0).astype(np.float64)
+    assert np.max(np.abs(y - ref[sel])) <= 1e-15 * max(1.0, float(np.max(sc)))
+    # rows without entries: beta * y0[row] exactly
+    for t, row in enumerate(sel):
+        if row in empty:
+            assert y[t] == (beta * y0[row] if beta != 0 else 0.0)
+
+
+def test_rows_spmv_equals_full_definition_bitwise():
+    """Same entries in the same order: rows_spmv must give the full
+    coo_spmv's bits for every sampled row (incl. scale)."""
+    a = gen.config3(n=16)
+    r, c, v, ptr = _csr(a)
+    rng = np.random.default_rng(3)
+    x = rng.uniform(-1, 1, a.ncols)
+    y0 = rng.uniform(-1, 1, a.nrows)
+    yf, sf = coo.coo_spmv(a.nrows, a.ncols, r, c, v, x, -0.75, 0.5, y0)
+    sel = np.concatenate([[a.nrows - 1, 0], rng.integers(0, a.nrows, 300)])
+    y, s2 = coo.rows_spmv(sel, ptr, c, v, x, -0.75, 0.5, y0)
+    assert np.array_equal(y, yf[sel]) and np.array_equal(s2, sf[sel])
+
+
+def test_rows_spmv_closed_form():
+    """Sampled rows of the 7-point stencil applied to the quadratic vector:
+    -6 in the interior, the closed form everywhere (exact integers)."""
+    dims = (11, 9, 7)
+    a = gen.stencil(dims, "7pt", values="exact")
+    r, c, v, ptr = _csr(a)
+    x = gen.vectors(a.ncols, "quadratic", dims=dims)
+    sel = np.arange(a.nrows)[::-3]
+    y, _ = coo.rows_spmv(sel, ptr, c, v, x)
+    assert np.array_equal(y, closed_forms.stencil_apply(dims, "7pt", "quadratic")[sel])
+
+
+# ---------------------------------------------------------------- parity_error
+def test_parity_error_hand_cases():
+    """The pass criterion of SURVEY.md §8(c): max over rows (not mean) of
+    |y - y_ref| / scale; rows with scale 0 must match exactly; NaN fails."""
+    ref = np.array([1.0, -2.0, 0.0, 4.0])
+    scale = np.array([1.0, 2.0, 0.0, 8.0])
+    assert coo.parity_error(ref.copy(), ref, scale) == 0.0
+    y = ref + np.array([1e-13, 0.0, 0.0, 0.0])
+    assert coo.parity_error(y, ref, scale) == pytest.approx(1e-13, rel=1e-3)
+    y = ref + np.array([1e-13, 4e-13, 0.0, 8e-13])  # per-row 1e-13, 2e-13, -, 1e-13: max, not mean
+    assert coo.parity_error(y, ref, scale) == pytest.approx(2e-13, rel=1e-3)
+    y = ref.copy()
+    y[2] = 1e-300  # a scale-0 row off by anything is a failure
+    assert coo.parity_error(y, ref, scale) == float("inf")
+    y = ref.copy()
+    y[1] = np.nan
+    assert coo.parity_error(y, ref, scale) == float("inf")
+    assert coo.parity_error(np.zeros(2), np.zeros(2), np.zeros(2)) == 0.0
+    # relative to the row's own scale: a large error on a large-scale row passes
+    assert coo.parity_error(np.array([1e6 + 1e-7]), np.array([1e6]), np.array([1e6])) <= 1e-12
+
+
+# ---------------------------------------------------------------- native-dtype baseline
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+@pytest.mark.parametrize("seed", range(4))
+def test_coo_native_within_summation_bound_and_thread_invariant(dt, seed):
+    """coo_spmv_native (the timed CPU baseline) against the long-double
+    definition: per row |y - y_ref| <= (k + 2) u scale (k entries, u the unit
+    roundoff; the recursive-summation bound), and the same bits for 1, 2, 3
+    and 8 threads (each row is summed by one thread in entry order)."""
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(1, 4000))
+    a = gen.random_diagonal(n, n, seed, ndiag=9, n_scatter=30).astype(dt)
+    keep = ~np.isin(a.row, rng.choice(n, size=min(n, 5), replace=False))  # some empty rows
+    a = gen.COO(n, n, a.row[keep], a.col[keep], a.val[keep])
+    r, c, v, ptr = _csr(a)
+    x = rng.uniform(-1, 1, n).astype(dt)
+    y0 = rng.uniform(-1, 1, n).astype(dt)
+    for alpha, beta in ((1.0, 0.0), (-0.75, 0.5)):
+        yref, sc = coo.coo_spmv(n, n, r, c, v, x, alpha, beta, y0)
+        u = 2.0**-53 if dt == np.float64 else 2.0**-24
+        k = np.diff(ptr).astype(np.float64)
+        outs = [coo.coo_spmv_native(n, r, c, v, x, alpha, beta, y0, nthreads=t) for t in (1, 2, 3, 8)]
+        assert outs[0].dtype == dt
+        err = np.abs(outs[0].astype(np.float64) - yref)
+        assert np.all(err <= (k + 2) * u * sc + (sc == 0) * 0.0)
+        for o in outs[1:]:
+            assert np.array_equal(o, outs[0])
+    # beta == 0 never reads y0
+    y = coo.coo_spmv_native(n, r, c, v, x, 1.0, 0.0, np.full(n, np.nan, dt), nthreads=3)
+    assert np.all(np.isfinite(y))
+
+
+def test_coo_native_closed_form_and_rejects_unsorted():
+    dims = (13, 11, 9)
+    a = gen.stencil(dims, "7pt", values="exact")
+    x = gen.vectors(a.ncols, "linear", dims=dims)
+    y = coo.coo_spmv_native(a.nrows, a.row, a.col, a.val, x, nthreads=4)
+    assert np.array_equal(y, closed_forms.stencil_apply(dims, "7pt", "linear"))
+    with pytest.raises(ValueError):
+        coo.coo_spmv_native(2, np.array([1, 0]), np.array([0, 0]), np.array([1.0, 1.0]), np.ones(2))
 
 
 # ---------------------------------------------------------------- closed forms
