@@ -17,6 +17,8 @@ from typing import Callable, Iterable, Optional, Sequence
 
 import numpy as np
 
+from . import fast as _fast
+
 _M64 = np.uint64(0xFFFFFFFFFFFFFFFF)
 
 
@@ -89,6 +91,37 @@ def _disps(kind: str):
 
 
 def stencil(
+    dims: Sequence[int],
+    kind: str,
+    *,
+    center: str = "dirichlet",
+    values: str = "exact",
+    seed: int = 0,
+    drop: Optional[Callable] = None,
+    row_begin: int = 0,
+    row_end: Optional[int] = None,
+) -> COO:
+    """Stencil matrix (see ``stencil_numpy``, the definition). Large grids go
+    through gen/fastgen.c, which produces the same COO bit for bit
+    (tests/test_gen.py); ``drop`` must then be a ``c3_drop`` mask."""
+    d3 = [int(d) for d in list(dims) + [1] * (3 - len(dims))]
+    if row_end is None:
+        row_end = d3[0] * d3[1] * d3[2]
+    if (row_end - row_begin) >= 200_000 and (drop is None or hasattr(drop, "c3_params")) and _fast.available():
+        if center not in ("dirichlet", "present") or values not in ("exact", "random"):
+            raise ValueError((center, values))
+        disps = _disps(kind)
+        lin = [di + d3[0] * (dj + d3[1] * dk) for (di, dj, dk) in disps]
+        disps = [disps[q] for q in np.argsort(lin, kind="stable")]
+        r, c, v = _fast.stencil(d3, disps, center == "present", values == "random", seed,
+                                None if drop is None else drop.c3_params, row_begin, row_end)
+        n = d3[0] * d3[1] * d3[2]
+        return COO(n, n, r, c, v)
+    return stencil_numpy(dims, kind, center=center, values=values, seed=seed, drop=drop, row_begin=row_begin,
+                         row_end=row_end)
+
+
+def stencil_numpy(
     dims: Sequence[int],
     kind: str,
     *,
@@ -258,6 +291,17 @@ def c4_ranges(n: int):
 
 
 def band(n: int, ranges, seed: int, row_begin: int = 0, row_end: Optional[int] = None) -> COO:
+    """Banded matrix (see ``band_numpy``, the definition); large row ranges
+    through gen/fastgen.c, bit for bit the same (tests/test_gen.py)."""
+    if row_end is None:
+        row_end = n
+    if row_end - row_begin >= 200_000 and _fast.available():
+        r, c, v = _fast.band(n, ranges, seed, row_begin, row_end)
+        return COO(n, n, r, c, v)
+    return band_numpy(n, ranges, seed, row_begin, row_end)
+
+
+def band_numpy(n: int, ranges, seed: int, row_begin: int = 0, row_end: Optional[int] = None) -> COO:
     """Banded matrix: rows [a,b) carry the offsets of their range; entries with
     columns outside [0,n) are omitted. Values U(-1,1)\\{0} from a counter hash
     of (row, offset) so row ranges agree with the global matrix."""
@@ -319,6 +363,7 @@ def c3_drop(n: int):
         m |= (k >= k3a) & (k < k3b)
         return m
 
+    drop.c3_params = (k1a, k1b, j2a, j2b, k2a, k2b, k3a, k3b)  # the same rule in gen/fastgen.c
     return drop
 
 
