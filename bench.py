@@ -1,27 +1,37 @@
 #!/usr/bin/env python
 """Benchmark of the CRSD SpMV hot path on B200 (driver contract: one JSON line).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2|c3|c4]
-                    [--dtype f64|f32] [--impl crsd|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c1..c5]
+                    [--dtype f64|f32] [--impl crsd|reference] [--workload spmv|cg]
 
-A step is one y = A*x (alpha 1, beta 0, the paper's SpMV) over the
-whole workload, inputs resident in HBM. Workload at N=1: BASELINE.json
-configs[1] (C2, 3D 7-point Laplacian 256^3, fp64) unless --config says
-otherwise. N>1 (torchrun): weak scaling, rank r owns a 256^3 slab of a
-256 x 256 x (256 N) 7-point grid; x halos move with NCCL send/recv over
-NVLink inside crsd_spmv_dist, overlapped with the interior segments.
+Metric (BASELINE.json): CRSD SpMV GFLOP/s (2 nnz / t, whole job) with the
+achieved HBM GB/s on algorithmic bytes and its fraction of the measured B200
+copy bandwidth (MEASURED_PEAKS.json), at 1/2/4/8 GPUs.
 
-Metric (BASELINE.json): CRSD SpMV GFLOP/s (= 2 nnz / t, whole job) with
-achieved HBM GB/s on algorithmic ("unique") bytes and its fraction of the
-measured B200 copy bandwidth (MEASURED_PEAKS.json).
---impl reference times the oracle (oracle/coo_spmv.c, long double, 1 thread)
-on the host cores on the same workload (the tier's reference arm).
+A step is one y = A x (alpha 1, beta 0: the paper's SpMV) over
+the whole workload, inputs resident in HBM. Default workload at EVERY N:
+BASELINE.json config 5, the 3D 7-point Laplacian on 768^3 (452,984,832 rows,
+3.17e9 nonzeros, fp64) -- strong scaling: N ranks own N row blocks of the one
+matrix, x halos move between ranks inside crsd_spmv_dist (the library's
+peer-memory kernels over NVLink, NCCL send/recv fallback), overlapped with
+the interior segments. At N = 1 the same run also times the north-star
+matrix, config 3 (27-point 192^3 with idle sections and 0.1 % scatter
+points) in fp64 and fp32, each with its own roofline record.
+
+When N > 1 and WORLD_SIZE is unset the script re-launches itself under
+torch.distributed.run with N ranks (one per GPU, rendezvous on 127.0.0.1).
+
+--impl reference times the oracle (oracle/coo_native.c: the definition
+accumulated in the matrix dtype, OpenMP over row ranges of the row-sorted
+COO, all host cores) on a bounded row sample of the same workload: the tier's
+reference arm. Under torchrun only rank 0 runs it.
 """
 from __future__ import annotations
 
 import argparse
 import json
 import os
+import socket
 import statistics
 import subprocess
 import sys
@@ -33,14 +43,11 @@ import numpy as np
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
+METRIC = "CRSD SpMV GFLOP/s and achieved HBM GB/s (% of B200 peak) at 1/2/4/8 GPUs"
 L2_BYTES = 126 * 1024 * 1024
-
-
-def _env_int(k, d):
-    try:
-        return int(os.environ.get(k, d))
-    except ValueError:
-        return d
+VARIANTS = {"auto": 0, "ldg": 1, "tma": 2, "pipe": 3, "jit": 4}
+VNAME = {1: "ldg", 2: "tma", 3: "pipe", 4: "jit"}
+KNAME = {1: "crsd_spmv_ldg", 2: "crsd_spmv_tma", 3: "crsd_spmv_pipe", 4: "crsd_jit"}
 
 
 def measured_peaks():
@@ -52,64 +59,122 @@ def measured_peaks():
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+def _affinity():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
+# read once at import: OMP_PROC_BIND later pins the main thread to one core
+_HOST_CORES = _affinity()
+
+
+def host_cores():
+    return _HOST_CORES
+
+
+def host_cpu_info():
+    info = {"nproc": host_cores()}
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            k, _, v = line.partition(":")
+            k, v = k.strip(), v.strip()
+            if k == "Model name":
+                info["model"] = v
+            elif k == "Socket(s)":
+                info["sockets"] = int(v) if v.isdigit() else v
+            elif k == "Thread(s) per core":
+                info["threads_per_core"] = int(v) if v.isdigit() else v
+    except Exception:
+        pass
+    return info
+
+
 # ---------------------------------------------------------------- workloads
-def workload(cfg: str, dtype: str, world: int = 1, rank: int = 0):
-    """Returns (COO of this rank's rows, description dict, row range or None, global nrows)."""
-    import gen
+def _stencil_disps(kind, dims):
+    from gen import matrices
 
-    dt = np.float64 if dtype == "f64" else np.float32
-    if cfg == "c1":
-        if world != 1:
-            raise SystemExit("config c1 is a single-GPU latency workload")
-        a = gen.config1()
-        N, rb, re = a.nrows, 0, a.nrows
-        desc = f"C1: 2D 5-point Laplacian 64x64 ({N:,} rows) + 16 scatter points, {dtype} (L2-resident: latency, L2 flushed before every step)"
+    disps = matrices._disps(kind)
+    lin = [di + dims[0] * (dj + dims[1] * dk) for (di, dj, dk) in disps]
+    return [disps[q] for q in np.argsort(lin, kind="stable")]
+
+
+def rank_rows(cfg, world, rank, mrows=256):
+    """Global size and this rank's row block [rb, re)."""
+    from paper_conf_icpp_sunzwzyr11_b200 import partition_rows
+
+    if cfg == "c5":
+        N = 768**3
+        b = partition_rows(N, mrows, world)  # uniform rows: equal blocks are byte-balanced
     elif cfg == "c2":
-        n = 256
-        nz = n * world
-        N = n * n * nz
-        rb, re = rank * n * n * n, (rank + 1) * n * n * n
-        a = gen.stencil((n, n, nz), "7pt", values="random", seed=2, row_begin=rb, row_end=re)
-        desc = f"C2: 3D 7-point FDM Laplacian 256^3 per GPU (grid 256x256x{nz}, {N:,} rows), {dtype}"
-    elif cfg in ("c3", "c3ns"):
-        if world != 1:
-            raise SystemExit("config c3 is a single-GPU workload")
-        # c3ns: the same matrix without its scatter points (diagnostic only)
-        a = gen.config3(scatter_frac=0.001 if cfg == "c3" else 0.0)
-        N, rb, re = a.nrows, 0, a.nrows
-        desc = f"C3: 3D 27-point FVM stencil 192^3 with idle sub-blocks and 0.1% scatter points ({N:,} rows), {dtype}"
-    elif cfg == "c5":
-        # N > 1: each rank builds its row block of C5 (strong scaling; N = 1 runs run_c5)
-        from paper_conf_icpp_sunzwzyr11_b200 import partition_rows
-
-        nn = 768
-        N = nn**3
-        bounds = partition_rows(N, 256, world)
-        rb, re = int(bounds[rank]), int(bounds[rank + 1])
-        a = gen.config5(n=nn, values="exact", row_begin=rb, row_end=re)
-        desc = f"C5: 3D 7-point Laplacian 768^3 ({N:,} rows), fp64, row-partitioned"
+        N = 256**3 * world  # weak: a 256^3 slab per rank
+        b = [k * 256**3 for k in range(world + 1)]
     elif cfg == "c4":
-        n = 100_000_000
+        import gen
+
+        N = 100_000_000
         if world == 1:
-            bounds = np.array([0, n], np.int64)
+            b = [0, N]
         else:
             # byte-balanced row blocks (SURVEY.md §8(e): equal rows give
             # max/avg 1.52 on C4): weight per row = its stored diagonals + x + y
-            from paper_conf_icpp_sunzwzyr11_b200 import partition_rows
-
-            w = np.empty(n, np.float64)
-            for r0, r1, offs in gen.matrices.c4_ranges(n):
+            w = np.empty(N, np.float64)
+            for r0, r1, offs in gen.matrices.c4_ranges(N):
                 w[r0:r1] = len(offs) + 2
-            bounds = partition_rows(n, 512, world, w)
+            b = partition_rows(N, 512, world, w)
             del w
-        rb, re = int(bounds[rank]), int(bounds[rank + 1])
-        a = gen.config4(n=n, row_begin=rb, row_end=re)
-        N = n
-        desc = f"C4: banded, 19 offsets in 9 groups / 4 patterns, 100M rows, {dtype}"
     else:
-        raise SystemExit(f"unknown config {cfg}")
-    a = gen.COO(N, N, a.row, a.col, a.val.astype(dt))
-    return a, desc, (rb, re), N
+        raise SystemExit(f"config {cfg} is one-GPU only")
+    return N, int(b[rank]), int(b[rank + 1])
+
+
+def build(cfg, dtype, world, rank, dev, mrows=0, variant=0, nthreads=0):
+    """Build this rank's CRSD handle for config `cfg`. Large configs are
+    generated as CSR by gen/fastgen.c and handed to crsd_create_from_csr,
+    which reads canonical CSR in place (C5 holds 3.17e9 entries).
+    Returns (A, description, (rb, re), N global rows, build seconds)."""
+    import gen
+    from gen import fast
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix
+
+    dt = np.float64 if dtype == "f64" else np.float32
+    kw = dict(device=dev, mrows=mrows, variant=variant, nthreads=nthreads)
+    t0 = time.perf_counter()
+    if cfg in ("c1", "c3", "c3ns"):
+        if world != 1:
+            raise SystemExit(f"config {cfg} is a single-GPU workload")
+        if cfg == "c1":
+            a = gen.config1()
+            desc = f"C1: 2D 5-point Laplacian 64x64 (4,096 rows) + 16 scatter points, {dtype} (L2-resident: latency, L2 flushed before every step)"
+        else:
+            # c3ns: the same matrix without its scatter points (diagnostic only)
+            a = gen.config3(scatter_frac=0.001 if cfg == "c3" else 0.0)
+            desc = f"C3: 3D 27-point FVM stencil 192^3 with idle sub-blocks and {'0.1% scatter points' if cfg == 'c3' else 'no scatter points'} ({a.nrows:,} rows), {dtype}"
+        A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val.astype(dt), **kw)
+        N, rb, re = a.nrows, 0, a.nrows
+        del a
+    else:
+        N, rb, re = rank_rows(cfg, world, rank)
+        if cfg == "c4":
+            ptr, col, val = fast.band(N, gen.matrices.c4_ranges(N), 4, rb, re, nthreads=nthreads, csr=True)
+            desc = f"C4: banded, 19 offsets in 9 groups / 4 patterns, 100M rows, {dtype}"
+        elif cfg == "c5":
+            if dtype != "f64":
+                raise SystemExit("config c5 is fp64")
+            d = (768, 768, 768)
+            ptr, col, val = fast.stencil(d, _stencil_disps("7pt", d), False, False, 5, None, rb, re, nthreads=nthreads, csr=True)
+            desc = f"C5: 3D 7-point Laplacian 768^3 ({N:,} rows, 3,167,354,880 nonzeros), fp64"
+        else:  # c2
+            d = (256, 256, 256 * world)
+            ptr, col, val = fast.stencil(d, _stencil_disps("7pt", d), False, True, 2, None, rb, re, nthreads=nthreads, csr=True)
+            desc = f"C2: 3D 7-point FDM Laplacian 256^3 per GPU (grid 256x256x{256 * world}, {N:,} rows), {dtype}"
+        if dt != np.float64:
+            val = val.astype(dt)
+        A = CRSDMatrix.from_csr(N, N, ptr, col, val, row_range=None if (rb, re) == (0, N) else (rb, re), **kw)
+        del ptr, col, val
+    return A, desc, (rb, re), N, time.perf_counter() - t0
 
 
 # ---------------------------------------------------------------- clocks
@@ -133,8 +198,10 @@ class ClockSampler:
             )
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
+            time.sleep(0.3)
         except Exception:
             self.proc = None
+        return self
 
     def _read(self):
         for line in self.proc.stdout:
@@ -159,12 +226,8 @@ class ClockSampler:
             for nm, v in zip(names, s[3:]):
                 if v.lower() == "active":
                     reasons.add(nm)
-        return {
-            "sm_mhz": statistics.median(sm) if sm else None,
-            "sm_max_mhz": max(mx) if mx else None,
-            "reasons": sorted(reasons),
-            "samples": len(self.samples),
-        }
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.samples)}
 
 
 def copy_bandwidth(dev, reps=5):
@@ -187,146 +250,217 @@ def copy_bandwidth(dev, reps=5):
     return round(best, 1)
 
 
-def sustained_copy_bandwidth(dev, seconds):
-    """Copy bandwidth sustained over about as long as the timed region
-    (back-to-back 1 Gi bf16 copies): the power-capped counterpart of the
-    burst figure in MEASURED_PEAKS.json."""
-    import torch
-
-    a = torch.empty(1 << 30, dtype=torch.bfloat16, device=f"cuda:{dev}")
-    b = torch.empty_like(a)
-    b.copy_(a)
-    torch.cuda.synchronize()
-    n = 0
-    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    t0 = time.perf_counter()
-    s.record()
-    while True:
-        for _ in range(10):
-            b.copy_(a)
-        n += 10
-        torch.cuda.synchronize()
-        if time.perf_counter() - t0 >= max(seconds, 0.05):
-            break
-    e.record()
-    e.synchronize()
-    gbs = n * 2 * a.numel() * 2 / (s.elapsed_time(e) * 1e-3) / 1e9
-    del a, b
-    torch.cuda.empty_cache()
-    return round(gbs, 1)
-
-
-def load_traffic(cfg, dtype, kernel):
-    """ncu dram bytes (read + write) per launch of `kernel` on this workload,
-    from one `ncu --set full` capture (profiles/traffic.json, keyed
+def load_traffic(key):
+    """ncu dram bytes (read + write) per launch of the dominant kernel on this
+    workload, from one `ncu --set full` capture (profiles/traffic.json, keyed
     "<config>_<dtype>_<kernel>"); None when that kernel was not captured."""
     p = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(p):
         with open(p) as f:
-            j = json.load(f)
-        return j.get(f"{cfg}_{dtype}_{kernel}")
+            return json.load(f).get(key)
     return None
+
+
+# ---------------------------------------------------------------- timing
+def timed_steps(step, steps, stream, count):
+    """K steps back to back between two CUDA events on the launching stream
+    (no per-step host work besides the launches themselves). Returns (ms per
+    step, whole-region ms, kernel launches)."""
+    import torch
+
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    t0.record(stream)
+    for _ in range(steps):
+        step()
+    t1.record(stream)
+    launches = steps * count()  # every step launches the same kernels
+    torch.cuda.synchronize()
+    total = t0.elapsed_time(t1)
+    return total / steps, total, launches
+
+
+def sub_record(cfg, dtype, args, dev):
+    """One-GPU timing of another BASELINE matrix inside the same run (the
+    north-star C3 records at N = 1): value, ms, roofline of its own."""
+    import torch
+
+    A, desc, _, N, bs = build(cfg, dtype, 1, 0, dev, mrows=0, variant=VARIANTS[args.variant])
+    info = A.info()
+    tdt = torch.float64 if dtype == "f64" else torch.float32
+    x = torch.from_numpy(np.random.default_rng(7).uniform(-1, 1, N)).to(f"cuda:{dev}", tdt)
+    y = torch.empty(N, dtype=tdt, device=f"cuda:{dev}")
+    stream = torch.cuda.current_stream()
+
+    def step():
+        A.spmv(x, y, 1.0, 0.0)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    clk = ClockSampler(dev).start()
+    ms, total_ms, launches = timed_steps(step, args.steps, stream, A.last_launch_count)
+    clocks = clk.stop()
+    ub = info["unique_bytes_beta0"]
+    peak, _ = measured_peaks()
+    achieved = ub / (ms * 1e-3) / 1e9
+    kname = KNAME[info["variant"]]
+    rec = {
+        "workload": desc,
+        "value": round(2.0 * info["nnz"] / (ms * 1e-3) / 1e9, 3),
+        "unit": "GFLOP/s",
+        "ms_per_step": round(ms, 5),
+        "dtype": dtype,
+        "nnz": info["nnz"],
+        "mrows": info["mrows"],
+        "kernel_variant": VNAME[info["variant"]],
+        "scatter": info["nscatter"],
+        "fills": info["nfills"],
+        "launches_per_step": round(launches / args.steps, 2),
+        "roofline": {
+            "bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+            "frac": round(achieved / peak, 4), "traffic": load_traffic(f"{cfg}_{dtype}_{kname}"),
+            "algorithmic_bytes_per_launch": int(ub), "avg_step_ms": round(ms, 5),
+        },
+        "l2": f"inputs larger than L2 ({ub / 1e9:.2f} GB per step); no flush",
+        "build_s": round(bs, 1),
+        "clocks": clocks,
+    }
+    A.close()
+    del x, y
+    torch.cuda.empty_cache()
+    return rec
+
+
+# ---------------------------------------------------------------- CPU baseline
+def cpu_sample(cfg, dtype, cap_nnz):
+    """Rows [0, cut) of the workload with about cap_nnz entries, as a
+    row-sorted COO (the reference arm and cpu_baseline generate only these).
+    Returns (nrows, ncols, cut, row, col, val, nnz of the whole matrix)."""
+    import gen
+    from gen import fast
+
+    dt = np.float64 if dtype == "f64" else np.float32
+    if cfg in ("c1", "c3", "c3ns"):
+        a = gen.config1() if cfg == "c1" else gen.config3(scatter_frac=0.001 if cfg == "c3" else 0.0)
+        a = a.sorted()
+        N = a.nrows
+        cut = N if a.nnz <= cap_nnz else max(1, int(N * cap_nnz // a.nnz))
+        m = a.row < cut
+        return N, N, cut, a.row[m], a.col[m], a.val[m].astype(dt), a.nnz
+    N, _, _ = rank_rows(cfg, 1, 0)
+    per_row = {"c5": 7.0, "c2": 7.0, "c4": 11.9}[cfg]
+    cut = int(min(N, max(1024, cap_nnz / per_row)))
+    if cfg == "c4":
+        r, c, v = fast.band(N, gen.matrices.c4_ranges(N), 4, 0, cut)
+        total = 1_186_000_000
+    else:
+        d = (768, 768, 768) if cfg == "c5" else (256, 256, 256)
+        r, c, v = fast.stencil(d, _stencil_disps("7pt", d), False, cfg == "c2", 5 if cfg == "c5" else 2, None, 0, cut)
+        total = 3_167_354_880 if cfg == "c5" else 117_047_296
+    return N, N, cut, r, c, v.astype(dt), total
+
+
+def time_native(nrows, r, c, v, x, nthreads, reps=5):
+    """Median of `reps` runs of the oracle's native-dtype loop (after one warm-up)."""
+    from oracle import coo as oracle_coo
+
+    y = np.empty(nrows, dtype=v.dtype)
+    oracle_coo.coo_spmv_native(nrows, r, c, v, x, nthreads=nthreads, out=y)
+    ts = []
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        oracle_coo.coo_spmv_native(nrows, r, c, v, x, nthreads=nthreads, out=y)
+        ts.append(time.perf_counter() - t0)
+    return statistics.median(ts)
+
+
+def cpu_baseline(cfg, dtype, cap_nnz=200_000_000):
+    """The oracle's plain COO SpMV in the matrix dtype (oracle/coo_native.c,
+    as it stands) on the host cores, on a bounded row sample of the workload:
+    1 thread and all cores (OpenMP over row ranges, OMP_PROC_BIND=spread),
+    median of 5 each."""
+    N, ncols, cut, r, c, v, total = cpu_sample(cfg, dtype, cap_nnz)
+    x = np.random.default_rng(7).uniform(-1, 1, ncols).astype(v.dtype)
+    k = r.shape[0]
+    cores = host_cores()
+    t1 = time_native(cut, r, c, v, x, 1)
+    tn = time_native(cut, r, c, v, x, cores)
+    return {
+        "value": round(2.0 * k / tn / 1e9, 3),
+        "unit": "GFLOP/s",
+        "cores": cores,
+        "kind": "oracle",
+        "sample": f"rows [0,{cut:,}) of the workload ({k:,} nonzeros, {k / total:.1%} of the matrix); oracle/coo_native.c "
+                  f"(definition in the matrix dtype, OpenMP over row ranges of the row-sorted COO, OMP_PROC_BIND=spread), median of 5",
+        "value_1_thread": round(2.0 * k / t1 / 1e9, 3),
+        "host": host_cpu_info(),
+    }
 
 
 # ---------------------------------------------------------------- reference arm
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
-        return
+        return  # the oracle arm runs on rank 0 alone; the other ranks exit without work
     from oracle import coo as oracle_coo
 
-    a, desc, _, N = workload(args.config, args.dtype, 1, 0)
-    dt = a.val.dtype
-    x = np.random.default_rng(7).uniform(-1, 1, a.ncols).astype(dt)
-    # bounded sample: calibrate the oracle's rate, then size each step so the
-    # whole --steps/--warmup run stays within ~2 minutes of CPU time
-    n0, r0_, c0_, v0_ = row_sample(a, 2_000_000)
-    t0 = time.perf_counter()
-    oracle_coo.coo_spmv(n0, a.ncols, r0_, c0_, v0_, x)
-    rate = r0_.shape[0] / max(time.perf_counter() - t0, 1e-6)
+    cores = host_cores()
+    # bounded sample: calibrate the oracle's rate on a small sample, then size
+    # each step so the whole --steps/--warmup run stays within ~2 minutes
     budget = float(os.environ.get("CRSD_REF_BUDGET_S", "120"))
-    cap = int(min(a.nnz, max(1_000_000, rate * budget / (args.steps + args.warmup))))
-    sample_rows, row, col, val = row_sample(a, cap)
-    nnz_s = row.shape[0]
+    N, ncols, cut, r, c, v, total = cpu_sample(args.config, args.dtype, 20_000_000)
+    x = np.random.default_rng(7).uniform(-1, 1, ncols).astype(v.dtype)
+    t = time_native(cut, r, c, v, x, cores, reps=2)
+    rate = r.shape[0] / max(t, 1e-6)
+    cap = int(min(total, 500_000_000, max(10_000_000, rate * budget / (args.steps + args.warmup))))
+    if cap > r.shape[0]:
+        del r, c, v
+        N, ncols, cut, r, c, v, total = cpu_sample(args.config, args.dtype, cap)
+        x = np.random.default_rng(7).uniform(-1, 1, ncols).astype(v.dtype)
+    k = r.shape[0]
+    y = np.empty(cut, dtype=v.dtype)
     for _ in range(args.warmup):
-        oracle_coo.coo_spmv(sample_rows, a.ncols, row, col, val, x)
+        oracle_coo.coo_spmv_native(cut, r, c, v, x, nthreads=cores, out=y)
     ts = []
     for _ in range(args.steps):
         t0 = time.perf_counter()
-        oracle_coo.coo_spmv(sample_rows, a.ncols, row, col, val, x)
+        oracle_coo.coo_spmv_native(cut, r, c, v, x, nthreads=cores, out=y)
         ts.append(time.perf_counter() - t0)
-    t = sum(ts) / len(ts)
-    gflops = 2.0 * nnz_s / t / 1e9
-    sample = f"rows [0,{sample_rows:,}) of the workload, {nnz_s:,} nonzeros per step ({nnz_s / a.nnz:.1%} of the matrix)"
+    tm = statistics.mean(ts)
+    gflops = 2.0 * k / tm / 1e9
+    sample = (f"rows [0,{cut:,}) of the workload, {k:,} nonzeros per step ({k / total:.1%} of the matrix); "
+              f"oracle/coo_native.c on {cores} host threads")
     line = {
         "impl": "reference",
-        "metric": "CRSD SpMV GFLOP/s (2*nnz/t)",
+        "metric": METRIC,
         "value": round(gflops, 4),
         "unit": "GFLOP/s",
         "n_gpus": args.gpus,
         "steps": args.steps,
         "warmup": args.warmup,
-        "ms_per_step": round(t * 1e3, 3),
+        "ms_per_step": round(tm * 1e3, 3),
         "higher_is_better": True,
-        "scaling": "weak",
+        "scaling": "strong" if args.config in ("c4", "c5") else "weak",
         "vs_baseline": None,
-        "dtype": "f64" if dt == np.float64 else "f32",
+        "dtype": args.dtype,
         "data": "synthetic",
-        "config": {"workload": desc, "alpha": 1.0, "beta": 0.0},
-        "cpu_baseline": {"value": round(gflops, 4), "unit": "GFLOP/s", "cores": 1, "kind": "oracle", "sample": sample},
+        "config": {"workload": args.config.upper() + " (row sample, see cpu_baseline.sample)", "alpha": 1.0, "beta": 0.0},
+        "cpu_baseline": {"value": round(gflops, 4), "unit": "GFLOP/s", "cores": cores, "kind": "oracle", "sample": sample,
+                         "host": host_cpu_info()},
         "e2e": {"value": round(gflops, 4), "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
 
 
-def row_sample(a, cap=None):
-    """Rows [0, cut) of the workload, sized to ~cap nonzeros (bounded CPU
-    work); entries selected by mask, so input order is irrelevant."""
-    if cap is None:
-        cap = int(os.environ.get("CRSD_REF_SAMPLE_NNZ", "60000000"))
-    if a.nnz <= cap:
-        return a.nrows, a.row, a.col, a.val
-    cut = max(1, int(a.nrows * cap // a.nnz))
-    m = a.row < cut
-    return cut, a.row[m], a.col[m], a.val[m]
-
-
 # ---------------------------------------------------------------- CRSD arm
-def cpu_baseline(a, seconds_target=10.0):
-    """The oracle as it stands (1 thread, long double) on a bounded row sample."""
-    from oracle import coo as oracle_coo
-
-    dt = a.val.dtype
-    x = np.random.default_rng(7).uniform(-1, 1, a.ncols).astype(dt)
-    nr, row, col, val = row_sample(a)
-    k = row.shape[0]
-    ts = []
-    t_start = time.perf_counter()
-    while True:
-        t0 = time.perf_counter()
-        oracle_coo.coo_spmv(nr, a.ncols, row, col, val, x)
-        ts.append(time.perf_counter() - t0)
-        if time.perf_counter() - t_start > seconds_target or len(ts) >= 20:
-            break
-    t = statistics.median(ts)
-    return {
-        "value": round(2.0 * k / t / 1e9, 4),
-        "unit": "GFLOP/s",
-        "cores": 1,
-        "kind": "oracle",
-        "sample": f"rows [0,{nr:,}) ({k:,} nonzeros, {k / a.nnz:.1%} of the workload), median of {len(ts)} runs, long-double accumulation, 1 thread",
-    }
-
-
-def run_crsd(args):
+def init_dist(args):
     import torch
     import torch.distributed as dist
-
-    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, Comm, P2PComm
 
     world = args.gpus
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    local_world = int(os.environ.get("LOCAL_WORLD_SIZE", str(world)))
     # --share-gpu: every rank on cuda:0 (functional check of the multi-rank
     # path on a one-GPU box; NCCL refuses two ranks per GPU, so the torch
     # plumbing uses gloo and the transport must be p2p). Not a scaling number.
@@ -336,60 +470,59 @@ def run_crsd(args):
             raise SystemExit("--share-gpu needs the p2p transport")
     if world > 1:
         dist.init_process_group("gloo" if args.share_gpu else "nccl", init_method="env://")
-        world = dist.get_world_size()
-        rank = dist.get_rank()
+        world, rank = dist.get_world_size(), dist.get_rank()
     torch.cuda.set_device(local_rank)
-    dev = local_rank
+    nthreads = max(1, host_cores() // max(1, local_world))
+    return world, rank, local_rank, nthreads
+
+
+def make_comm(args, A, rank, world, dev, es):
+    from paper_conf_icpp_sunzwzyr11_b200 import Comm, P2PComm
+
+    lo, _, hi = A.x_layout()
+    comm, transport = None, None
+    if args.transport in ("auto", "p2p"):
+        try:
+            comm, transport = P2PComm(rank, world, dev, mailbox_bytes=max(1 << 20, 4 * (lo + hi) * es)), "p2p"
+        except Exception as e:  # collective: every rank lands here together
+            if args.transport == "p2p":
+                raise
+            print(f"[bench] peer-memory transport unavailable ({e}); using NCCL", file=sys.stderr)
+    if comm is None:
+        comm, transport = Comm(rank, world, dev), "nccl"
+    A.dist_bind(comm)
+    return comm, transport
+
+
+def run_spmv(args):
+    import torch
+    import torch.distributed as dist
+
+    world, rank, dev, nthreads = init_dist(args)
     red_dev = "cpu" if args.share_gpu else f"cuda:{dev}"
-
-    a, desc, (rb, re), N = workload(args.config, args.dtype, world, rank)
-    dt = a.val.dtype
-    tdt = torch.float64 if dt == np.float64 else torch.float32
-    es = np.dtype(dt).itemsize
-    kw = dict(device=dev)
-    if args.mrows:
-        kw["mrows"] = args.mrows
-    kw["variant"] = {"auto": 0, "ldg": 1, "tma": 2, "pipe": 3, "jit": 4}[args.variant]
-    if world > 1:
-        kw["row_range"] = (rb, re)
-    t0 = time.perf_counter()
-    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, **kw)
-    build_s = time.perf_counter() - t0
+    A, desc, (rb, re), N, build_s = build(args.config, args.dtype, world, rank, dev, args.mrows, VARIANTS[args.variant], nthreads)
     info = A.info()
-    nnz_local = info["nnz"]
-    ub = info["unique_bytes_beta0"]
+    dt = np.float64 if args.dtype == "f64" else np.float32
+    tdt = torch.float64 if args.dtype == "f64" else torch.float32
+    es = np.dtype(dt).itemsize
     stream = torch.cuda.current_stream()
-
-    transport = None
-    x_full = torch.from_numpy(np.random.default_rng(7 + rank).uniform(-1, 1, re - rb).astype(dt)).to(f"cuda:{dev}")
-    comm = None
+    nloc = re - rb
+    x_own = torch.from_numpy(np.random.default_rng(7 + rank).uniform(-1, 1, nloc).astype(dt)).to(f"cuda:{dev}")
+    comm, transport = None, None
     if world > 1:
-        lo, nloc, hi = A.x_layout()
+        comm, transport = make_comm(args, A, rank, world, dev, es)
+        lo, _, hi = A.x_layout()
         xp = torch.zeros(lo + nloc + hi, dtype=tdt, device=f"cuda:{dev}")
-        xp[lo : lo + nloc] = x_full
+        xp[lo : lo + nloc] = x_own
         y = torch.empty(nloc, dtype=tdt, device=f"cuda:{dev}")
-        comm = None
-        if args.transport in ("auto", "p2p"):
-            try:
-                comm = P2PComm(rank, world, dev, mailbox_bytes=max(1 << 20, 4 * (lo + hi) * es))
-                transport = "p2p"
-            except Exception as e:  # collective: every rank lands here together
-                if args.transport == "p2p":
-                    raise
-                print(f"[bench] peer-memory transport unavailable ({e}); using NCCL", file=sys.stderr)
-        if comm is None:
-            comm = Comm(rank, world, dev)
-            transport = "nccl"
-        A.dist_bind(comm)
 
         def step():
             A.spmv_dist(xp, y, 1.0, 0.0, comm)
     else:
-        x = x_full
-        y = torch.empty(a.nrows, dtype=tdt, device=f"cuda:{dev}")
+        y = torch.empty(N, dtype=tdt, device=f"cuda:{dev}")
 
         def step():
-            A.spmv(x, y, 1.0, 0.0)
+            A.spmv(x_own, y, 1.0, 0.0)
 
     for _ in range(args.warmup):
         step()
@@ -397,153 +530,73 @@ def run_crsd(args):
     if comm is not None and comm.error():
         raise SystemExit(f"[bench] rank {rank}: a peer-memory wait timed out during warm-up (code {comm.error()}); no valid number")
 
-    # timed region: K steps, per-step CUDA events on the launching stream
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    clocks = ClockSampler(dev)
-    if not os.environ.get("CRSD_BENCH_NO_CLOCKS"):  # diagnostic switch only
-        clocks.start()
-        time.sleep(0.3)
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
-    t_all0 = torch.cuda.Event(enable_timing=True)
-    t_all1 = torch.cuda.Event(enable_timing=True)
-    t_all0.record(stream)
-    launches = 0
+    # timed region: K steps, per-step CUDA events on the launching stream,
+    # barrier + synchronize on both sides
     # C1 fits in L2 (0.23 MB): flush it (write a buffer > L2) before every
     # step, outside the step's events; the metric is then the per-step time
     flush = torch.empty(2 * L2_BYTES // 4, dtype=torch.int32, device=f"cuda:{dev}") if args.config == "c1" else None
-    for i in range(args.steps):
-        if flush is not None:
-            flush.zero_()
-        ev[i][0].record(stream)
-        step()
-        ev[i][1].record(stream)
-        launches += A.last_launch_count()
-    t_all1.record(stream)
-    torch.cuda.synchronize()
+    clk = ClockSampler(dev).start()
     if world > 1:
         dist.barrier()
-    clk = clocks.stop()
+    torch.cuda.synchronize()
+    if flush is None:
+        step_ms, total_ms, launches = timed_steps(step, args.steps, stream, A.last_launch_count)
+        step_ms = [step_ms]
+    else:  # per-step events, the flush outside them
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        for i in range(args.steps):
+            flush.zero_()
+            ev[i][0].record(stream)
+            step()
+            ev[i][1].record(stream)
+        torch.cuda.synchronize()
+        step_ms = [s_.elapsed_time(e_) for s_, e_ in ev]
+        total_ms, launches = sum(step_ms), args.steps * A.last_launch_count()
+    if world > 1:
+        dist.barrier()
+    clocks = clk.stop()
     if comm is not None and comm.error():
         raise SystemExit(f"[bench] rank {rank}: a peer-memory wait timed out in the timed region (code {comm.error()}); no valid number")
-    total_ms = t_all0.elapsed_time(t_all1)
-    step_ms = [s.elapsed_time(e) for s, e in ev]
+    nnz_local, ub = info["nnz"], info["unique_bytes_beta0"]
     if world > 1:
-        tt = torch.tensor([total_ms], dtype=torch.float64, device=red_dev)
+        tt = torch.tensor([total_ms, statistics.mean(step_ms)], dtype=torch.float64, device=red_dev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        total_ms = float(tt.item())
-        nn = torch.tensor([nnz_local, ub], dtype=torch.float64, device=red_dev)
+        total_ms, kern_ms = float(tt[0].item()), float(tt[1].item())
+        nn = torch.tensor([nnz_local, ub, launches], dtype=torch.float64, device=red_dev)
         dist.all_reduce(nn)
-        nnz_all, ub_all = float(nn[0].item()), float(nn[1].item())
+        nnz_all, ub_all, launches_all = (float(v) for v in nn.tolist())
     else:
-        nnz_all, ub_all = float(nnz_local), float(ub)
+        kern_ms = statistics.mean(step_ms)
+        nnz_all, ub_all, launches_all = float(nnz_local), float(ub), float(launches)
     ms = total_ms / args.steps
     if flush is not None:
-        ms = statistics.median(step_ms)
+        ms = kern_ms = statistics.median(step_ms)
     gflops = 2.0 * nnz_all / (ms * 1e-3) / 1e9
-    kern_ms = statistics.mean(step_ms)
     peak, peak_src = measured_peaks()
-    achieved = ub / (kern_ms * 1e-3) / 1e9
+    achieved = ub_all / world / (kern_ms * 1e-3) / 1e9  # per GPU: whole-job bytes / N / max-over-ranks step time
 
-    # e2e through the public C-ABI with host buffers (pinned), N = 1 path
-    e2e = None
-    if world == 1:
-        xh = torch.from_numpy(np.random.default_rng(7).uniform(-1, 1, a.ncols).astype(dt)).pin_memory()
-        yh = torch.empty(a.nrows, dtype=tdt).pin_memory()
-        for _ in range(2):
-            A.spmv_host_ptr(xh.data_ptr(), yh.data_ptr(), 1.0, 0.0)
-        ke = max(3, min(args.steps, 50))
-        t0 = time.perf_counter()
-        for _ in range(ke):
-            A.spmv_host_ptr(xh.data_ptr(), yh.data_ptr(), 1.0, 0.0)
-        te = (time.perf_counter() - t0) / ke
-        # transfer bound of the e2e step: pinned H2D / D2H bandwidth alone
-        xd_tmp = torch.empty(a.ncols, dtype=tdt, device=f"cuda:{dev}")
-        yd_tmp = torch.empty(a.nrows, dtype=tdt, device=f"cuda:{dev}")
-
-        def bw(fn, nbytes):
-            fn()
-            torch.cuda.synchronize()
-            t0 = time.perf_counter()
-            for _ in range(5):
-                fn()
-            torch.cuda.synchronize()
-            return nbytes * 5 / (time.perf_counter() - t0) / 1e9
-
-        h2d = bw(lambda: xd_tmp.copy_(xh, non_blocking=True), a.ncols * es)
-        d2h = bw(lambda: yh.copy_(yd_tmp, non_blocking=True), a.nrows * es)
-        s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
-
-        def both():  # H2D and D2H at the same time on two streams
-            with torch.cuda.stream(s1):
-                xd_tmp.copy_(xh, non_blocking=True)
-            with torch.cuda.stream(s2):
-                yh.copy_(yd_tmp, non_blocking=True)
-
-        bidir_ms = bw(both, 1e6) and None
-        torch.cuda.synchronize()
-        t0 = time.perf_counter()
-        for _ in range(5):
-            both()
-        torch.cuda.synchronize()
-        bidir_ms = (time.perf_counter() - t0) / 5 * 1e3
-        del xd_tmp, yd_tmp
-        e2e = {
-            "value": round(2.0 * nnz_all / te / 1e9, 3),
-            "unit": "GFLOP/s",
-            "h2d_bytes_per_step": int(a.ncols * es),
-            "d2h_bytes_per_step": int(a.nrows * es),
-            "ms_per_step": round(te * 1e3, 4),
-            "pinned_h2d_gbs": round(h2d, 1),
-            "pinned_d2h_gbs": round(d2h, 1),
-            "transfer_bound_ms": round(max(a.ncols * es / h2d, a.nrows * es / d2h) / 1e6, 4),
-            "concurrent_h2d_d2h_ms": round(bidir_ms, 4),
-            "path": "crsd_spmv_host: chunked H2D(x) / kernel / D2H(y) pipeline on three streams",
-        }
-    if world > 1:
-        # e2e through crsd_spmv_dist: pinned host x slice -> owned part of
-        # x_padded, halo exchange + SpMV, y slice -> pinned host; max over ranks
-        xh = torch.from_numpy(np.random.default_rng(7 + rank).uniform(-1, 1, re - rb).astype(dt)).pin_memory()
-        yh = torch.empty(re - rb, dtype=tdt).pin_memory()
-
-        def e2e_step():
-            xp[lo : lo + nloc].copy_(xh, non_blocking=True)
-            A.spmv_dist(xp, y, 1.0, 0.0, comm)
-            yh.copy_(y, non_blocking=True)
-            torch.cuda.current_stream().synchronize()
-
-        for _ in range(2):
-            e2e_step()
-        ke = max(3, min(args.steps, 50))
-        dist.barrier()
-        t0 = time.perf_counter()
-        for _ in range(ke):
-            e2e_step()
-        te = torch.tensor([(time.perf_counter() - t0) / ke], dtype=torch.float64, device=red_dev)
-        dist.all_reduce(te, op=dist.ReduceOp.MAX)
-        te = float(te.item())
-        e2e = {
-            "value": round(2.0 * nnz_all / te / 1e9, 3),
-            "unit": "GFLOP/s",
-            "h2d_bytes_per_step": int((re - rb) * es) * world,
-            "d2h_bytes_per_step": int((re - rb) * es) * world,
-            "ms_per_step": round(te * 1e3, 4),
-            "path": f"per rank: H2D of the owned x slice, crsd_spmv_dist ({transport} halo + SpMV), D2H of the y slice; max over ranks",
-        }
+    # e2e through the public C-ABI with host buffers (pinned)
+    e2e = run_e2e(args, A, world, rank, dev, dt, tdt, N, rb, re, nnz_all, red_dev, comm, transport)
     if rank != 0:
         if comm is not None:
             comm.close()
         dist.destroy_process_group()
         return
 
-    cpu = None if (world > 1 or args.no_cpu) else cpu_baseline(a)
+    subs = None
+    cpu = None
+    if world == 1 and args.config == "c5" and not args.no_sub:
+        # the north-star matrix (BASELINE config 3) in both precisions
+        A.close()
+        del x_own, y
+        torch.cuda.empty_cache()
+        subs = {"f64": sub_record("c3", "f64", args, dev), "f32": sub_record("c3", "f32", args, dev)}
+    if world == 1 and not args.no_cpu:
+        cpu = cpu_baseline(args.config, args.dtype)
     box_copy = copy_bandwidth(dev)
-    box_copy_sus = sustained_copy_bandwidth(dev, total_ms * 1e-3)
-    kname = {1: "crsd_spmv_ldg", 2: "crsd_spmv_tma", 3: "crsd_spmv_pipe", 4: "crsd_jit"}[info["variant"]]
-    traffic = None if args.mrows else load_traffic(args.config, args.dtype, kname)
+    kname = KNAME[info["variant"]]
     line = {
-        "metric": "CRSD SpMV GFLOP/s (2*nnz/t) with achieved HBM GB/s (% of B200 peak)",
+        "metric": METRIC,
         "value": round(gflops, 3),
         "unit": "GFLOP/s",
         "n_gpus": world,
@@ -558,16 +611,17 @@ def run_crsd(args):
         "config": {
             "workload": desc,
             "nnz": int(nnz_all),
+            "rows_per_rank": int(re - rb),
             "mrows": info["mrows"],
-            "kernel_variant": {1: "ldg", 2: "tma", 3: "pipe", 4: "jit"}[info["variant"]],
+            "kernel_variant": VNAME[info["variant"]],
             "alpha": 1.0,
             "beta": 0.0,
             "patterns": info["npat"],
             "instances": info["ninst"],
             "fills": info["nfills"],
             "scatter": info["nscatter"],
-            "l2": (f"inputs larger than L2 ({ub / 1e9:.2f} GB streamed per step vs {L2_BYTES / 2**20:.0f} MiB L2); no flush" if flush is None else f"L2 flushed (252 MiB written) before every step; ms_per_step = median per-step CUDA-event time"),
-            "build_s": round(build_s, 2),
+            "l2": (f"inputs larger than L2 ({ub_all / 1e9:.2f} GB streamed per step vs {L2_BYTES / 2**20:.0f} MiB L2); no flush" if flush is None else f"L2 flushed (252 MiB written) before every step; ms_per_step = median per-step CUDA-event time"),
+            "build_s": round(build_s, 1),
             "parallelism": f"row-partitioned x{world}" + (f", {transport} halo" if world > 1 else "") + (", ranks share cuda:0 (functional only)" if args.share_gpu else ""),
         },
         "latency_us": round(ms * 1e3, 2) if flush is not None else None,
@@ -581,20 +635,18 @@ def run_crsd(args):
             "peak_source": peak_src,
             "unit": "GB/s",
             "frac": round(achieved / peak, 4),
-            "traffic": traffic,
-            "algorithmic_bytes_per_launch": int(ub),
+            "traffic": load_traffic(f"{args.config}_{args.dtype}_{kname}") if (world == 1 and not args.mrows) else None,
+            "algorithmic_bytes_per_launch": int(ub_all / world),
             "avg_launch_ms": round(kern_ms, 5),
-            "launches_per_step": round(launches / max(1, args.steps), 2),
-            "per_step_note": "with several launches per step (JIT occupancy classes, dist interior/boundary) achieved = the step's algorithmic bytes / the step's CUDA-event time",
+            "launches_per_step": round(launches_all / world / max(1, args.steps), 2),
+            "scope": "per GPU: whole-job algorithmic bytes / N / the max-over-ranks CUDA-event step time; with several launches per step (occupancy-class ranges, interior/boundary) the step's bytes / the step's time",
             "copy_gbs_this_box": box_copy,
-            "frac_of_this_box_copy": round(achieved / box_copy, 4) if box_copy else None,
-            "sustained_copy_gbs_this_box": box_copy_sus,
-            "sustained_copy_note": "copies for as long as the timed region; long runs hit the 1 kW power cap",
         },
+        "north_star_c3": subs,
         "cpu_baseline": cpu,
         "e2e": e2e,
-        "gpu_launches": int(launches),
-        "clocks": clk,
+        "gpu_launches": int(launches_all),
+        "clocks": clocks,
     }
     print(json.dumps(line), flush=True)
     if comm is not None:
@@ -603,148 +655,80 @@ def run_crsd(args):
         dist.destroy_process_group()
 
 
-# ---------------------------------------------------------------- C5 on one GPU
-def run_c5(args):
-    """--config c5: BASELINE config 5 (3D 7-point Laplacian 768^3, fp64,
-    452,984,832 rows, 3.17e9 nonzeros, 32.6 GB) on ONE B200. The host builds
-    it as 8 row blocks (the 8-GPU partition: a single 3.17e9-entry COO would
-    need ~76 GB of host RAM plus the builder's copies), every block resident
-    on the GPU; the blocks share one global x (each block's padded x is a
-    view of it: its halos are the neighbours' owned x, no exchange) and write
-    disjoint slices of one global y. A step = the 8 blocks' crsd_spmv_dist
-    calls (comm = NULL)."""
+def run_e2e(args, A, world, rank, dev, dt, tdt, N, rb, re, nnz_all, red_dev, comm, transport):
+    """The metric end to end through the public C-ABI: every step copies the
+    step's x from pinned host memory and its y back (N = 1: crsd_spmv_host,
+    the library's chunked H2D / SpMV / D2H pipeline; N > 1: per rank the
+    owned x slice in, crsd_spmv_dist, the y slice out, max over ranks)."""
     import torch
+    import torch.distributed as dist
 
-    import gen
-    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, partition_rows
-
-    if args.gpus != 1:
-        raise SystemExit("run_c5 is the one-GPU form")
-    if args.dtype != "f64":
-        raise SystemExit("config c5 is fp64")
-    torch.cuda.set_device(0)
-    nn, nb = 768, 8
-    N = nn**3
-    bounds = partition_rows(N, 256, nb)
-    blocks, t0 = [], time.perf_counter()
-    cpu = None
-    for k in range(nb):
-        rb, re = int(bounds[k]), int(bounds[k + 1])
-        a = gen.config5(n=nn, values="exact", row_begin=rb, row_end=re)
-        if k == 0 and not args.no_cpu:
-            cpu = cpu_baseline(gen.COO(re, N, a.row, a.col, a.val))
-            cpu["sample"] += " (block 0 of the 8 host-built blocks)"
-        A = CRSDMatrix.from_coo(N, N, a.row, a.col, a.val, row_range=(rb, re), device=0)
-        del a
-        blocks.append((rb, re, A))
-    build_s = time.perf_counter() - t0
-    pad = (max(max(A.x_layout()[0], A.x_layout()[2]) for _, _, A in blocks) + 64 + 3) // 4 * 4  # keeps views 16-B aligned
-    x_ext = torch.zeros(N + 2 * pad, dtype=torch.float64, device="cuda:0")
-    x = x_ext[pad : pad + N]
-    x.copy_(torch.from_numpy(np.random.default_rng(7).uniform(-1, 1, N)))
-    y = torch.empty(N, dtype=torch.float64, device="cuda:0")
-    views = []
-    for rb, re, A in blocks:
-        lo, nloc, hi = A.x_layout()
-        views.append((A, x_ext[pad + rb - lo : pad + re + hi], y[rb:re]))
-    infos = [A.info() for _, _, A in blocks]
-    nnz = sum(i["nnz"] for i in infos)
-    ub = sum(i["unique_bytes_beta0"] for i in infos)
-
-    def step():
-        for A, xv, yv in views:
-            A.spmv_dist(xv, yv, 1.0, 0.0, None)
-
-    for _ in range(args.warmup):
-        step()
-    torch.cuda.synchronize()
-    stream = torch.cuda.current_stream()
-    clocks = ClockSampler(0)
-    clocks.start()
-    time.sleep(0.3)
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    launches = 0
-    torch.cuda.synchronize()
-    for i in range(args.steps):
-        ev[i][0].record(stream)
-        step()
-        ev[i][1].record(stream)
-        launches += sum(A.last_launch_count() for A, _, _ in views)
-    torch.cuda.synchronize()
-    clk = clocks.stop()
-    step_ms = [s_.elapsed_time(e_) for s_, e_ in ev]
-    ms = statistics.mean(step_ms)
-    peak, peak_src = measured_peaks()
-    achieved = ub / (ms * 1e-3) / 1e9
-    # e2e: pinned host x -> device, the 8 block SpMVs, device y -> pinned host
-    xh = torch.from_numpy(np.random.default_rng(7).uniform(-1, 1, N)).pin_memory()
-    yh = torch.empty(N, dtype=torch.float64).pin_memory()
+    es = np.dtype(dt).itemsize
+    ke = max(3, min(args.steps, 10))
+    if world == 1:
+        xh = torch.from_numpy(np.random.default_rng(7).uniform(-1, 1, N).astype(dt)).pin_memory()
+        yh = torch.empty(N, dtype=tdt).pin_memory()
+        for _ in range(2):
+            A.spmv_host_ptr(xh.data_ptr(), yh.data_ptr(), 1.0, 0.0)
+        t0 = time.perf_counter()
+        for _ in range(ke):
+            A.spmv_host_ptr(xh.data_ptr(), yh.data_ptr(), 1.0, 0.0)
+        te = (time.perf_counter() - t0) / ke
+        # the copy bound of the e2e step: H2D and D2H at the same time on two streams
+        xd = torch.empty(N, dtype=tdt, device=f"cuda:{dev}")
+        yd = torch.empty(N, dtype=tdt, device=f"cuda:{dev}")
+        s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(3):
+            with torch.cuda.stream(s1):
+                xd.copy_(xh, non_blocking=True)
+            with torch.cuda.stream(s2):
+                yh.copy_(yd, non_blocking=True)
+        torch.cuda.synchronize()
+        bidir_ms = (time.perf_counter() - t0) / 3 * 1e3
+        del xd, yd, xh, yh
+        torch.cuda.empty_cache()
+        return {
+            "value": round(2.0 * nnz_all / te / 1e9, 3),
+            "unit": "GFLOP/s",
+            "h2d_bytes_per_step": int(N * es),
+            "d2h_bytes_per_step": int(N * es),
+            "ms_per_step": round(te * 1e3, 3),
+            "concurrent_h2d_d2h_ms": round(bidir_ms, 3),
+            "frac_of_copy_bound": round(bidir_ms / (te * 1e3), 3),
+            "path": "crsd_spmv_host: chunked H2D(x) / SpMV / D2H(y) pipeline on three streams",
+        }
+    nloc = re - rb
+    lo, _, hi = A.x_layout()
+    xp = torch.zeros(lo + nloc + hi, dtype=tdt, device=f"cuda:{dev}")
+    y = torch.empty(nloc, dtype=tdt, device=f"cuda:{dev}")
+    xh = torch.from_numpy(np.random.default_rng(7 + rank).uniform(-1, 1, nloc).astype(dt)).pin_memory()
+    yh = torch.empty(nloc, dtype=tdt).pin_memory()
 
     def e2e_step():
-        x.copy_(xh, non_blocking=True)
-        step()
+        xp[lo : lo + nloc].copy_(xh, non_blocking=True)
+        A.spmv_dist(xp, y, 1.0, 0.0, comm)
         yh.copy_(y, non_blocking=True)
-        torch.cuda.synchronize()
+        torch.cuda.current_stream().synchronize()
 
-    e2e_step()
-    ke = 5
+    for _ in range(2):
+        e2e_step()
+    dist.barrier()
     t0 = time.perf_counter()
     for _ in range(ke):
         e2e_step()
-    te = (time.perf_counter() - t0) / ke
-    line = {
-        "metric": "CRSD SpMV GFLOP/s (2*nnz/t) with achieved HBM GB/s (% of B200 peak)",
-        "value": round(2.0 * nnz / (ms * 1e-3) / 1e9, 3),
+    te = torch.tensor([(time.perf_counter() - t0) / ke], dtype=torch.float64, device=red_dev)
+    dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    te = float(te.item())
+    return {
+        "value": round(2.0 * nnz_all / te / 1e9, 3),
         "unit": "GFLOP/s",
-        "n_gpus": 1,
-        "steps": args.steps,
-        "warmup": args.warmup,
-        "ms_per_step": round(ms, 5),
-        "higher_is_better": True,
-        "scaling": "weak",
-        "vs_baseline": None,
-        "dtype": "f64",
-        "data": "synthetic",
-        "config": {
-            "workload": f"C5: 3D 7-point Laplacian 768^3 ({N:,} rows), fp64, one B200, 8 resident row blocks sharing one x",
-            "nnz": int(nnz),
-            "mrows": infos[0]["mrows"],
-            "kernel_variant": {1: "ldg", 2: "tma", 3: "pipe", 4: "jit"}[infos[0]["variant"]],
-            "alpha": 1.0,
-            "beta": 0.0,
-            "device_bytes": int(sum(i["device_bytes"] for i in infos) + (N + 2 * pad + N) * 8),
-            "l2": f"inputs larger than L2 ({ub / 1e9:.1f} GB per step); no flush",
-            "build_s": round(build_s, 1),
-            "parallelism": "one GPU",
-        },
-        "hbm_gbs": round(achieved, 1),
-        "hbm_frac_of_peak": round(achieved / peak, 4),
-        "roofline": {
-            "bound": "hbm",
-            "kernel": "crsd_jit (8 blocks x interior range + boundary list per step)",
-            "achieved": round(achieved, 1),
-            "peak": peak,
-            "peak_source": peak_src,
-            "unit": "GB/s",
-            "frac": round(achieved / peak, 4),
-            "traffic": None,
-            "algorithmic_bytes_per_step": int(ub),
-            "avg_step_ms": round(ms, 5),
-            "launches_per_step": round(launches / max(1, args.steps), 2),
-        },
-        "cpu_baseline": cpu,
-        "e2e": {
-            "value": round(2.0 * nnz / te / 1e9, 3),
-            "unit": "GFLOP/s",
-            "h2d_bytes_per_step": int(N * 8),
-            "d2h_bytes_per_step": int(N * 8),
-            "ms_per_step": round(te * 1e3, 3),
-            "path": "pinned H2D of x (3.6 GB), the 8 block SpMVs, pinned D2H of y (3.6 GB); serial",
-        },
-        "gpu_launches": int(launches),
-        "clocks": clk,
+        "h2d_bytes_per_step": int(N * es),
+        "d2h_bytes_per_step": int(N * es),
+        "ms_per_step": round(te * 1e3, 3),
+        "path": f"per rank: H2D of the owned x slice, crsd_spmv_dist ({transport} halo + SpMV), D2H of the y slice; max over ranks",
     }
-    print(json.dumps(line), flush=True)
 
 
 # ---------------------------------------------------------------- CG workload
@@ -759,18 +743,11 @@ def run_cg(args):
     import torch
     import torch.distributed as dist
 
-    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, Comm, P2PComm
-    from oracle import cg_ref
-
     import gen
+    from oracle import cg_ref
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix
 
-    world = args.gpus
-    rank = int(os.environ.get("RANK", "0"))
-    local_rank = 0 if args.share_gpu else int(os.environ.get("LOCAL_RANK", "0"))
-    if world > 1:
-        dist.init_process_group("gloo" if args.share_gpu else "nccl", init_method="env://")
-        world, rank = dist.get_world_size(), dist.get_rank()
-    torch.cuda.set_device(local_rank)
+    world, rank, local_rank, nthreads = init_dist(args)
     dev = f"cuda:{local_rank}"
     red_dev = "cpu" if args.share_gpu else dev
     dt = np.float64 if args.dtype == "f64" else np.float32
@@ -792,19 +769,8 @@ def run_cg(args):
     info = A.info()
     comm, transport = None, None
     if world > 1:
-        lo, _, hi = A.x_layout()
-        if args.transport in ("auto", "p2p"):
-            try:
-                comm, transport = P2PComm(rank, world, local_rank, mailbox_bytes=max(1 << 20, 4 * (lo + hi) * es)), "p2p"
-            except Exception as e:
-                if args.transport == "p2p":
-                    raise
-                print(f"[bench] peer-memory transport unavailable ({e}); using NCCL", file=sys.stderr)
-        if comm is None:
-            comm, transport = Comm(rank, world, local_rank), "nccl"
-        A.dist_bind(comm)
-    vec_passes = 10
-    step_bytes = info["unique_bytes_beta0"] + vec_passes * nloc * es
+        comm, transport = make_comm(args, A, rank, world, local_rank, es)
+    step_bytes = info["unique_bytes_beta0"] + 10 * nloc * es
     nnz_local = int(a.nnz)
     step_flops = 2.0 * nnz_local + 10.0 * nloc
     rng = np.random.default_rng(17 + rank)
@@ -813,8 +779,7 @@ def run_cg(args):
     x = torch.zeros(nloc, dtype=tdt, device=dev)
     K = args.steps
     check = min(K, 50)
-    clocks = ClockSampler(local_rank)
-    clocks.start()
+    clocks = ClockSampler(local_rank).start()
     # warm-up: >= 300 steps (a short CG run otherwise starts below full clocks)
     A.cg(b, x, max(args.warmup, 300), 0.0, check_every=check, comm=comm)
     torch.cuda.synchronize()
@@ -859,7 +824,7 @@ def run_cg(args):
         dist.destroy_process_group()
         return
     cpu = None
-    if world == 1:
+    if world == 1 and not args.no_cpu:
         # cpu_baseline: the CG oracle as it stands on a bounded sample (64^3 grid)
         ns = 64
         a_s = gen.spd_stencil_scatter((ns, ns, ns), "7pt").astype(dt)
@@ -892,7 +857,7 @@ def run_cg(args):
             "workload": f"CG on the 7-point Dirichlet Laplacian 256x256x{256 * world} ({N:,} rows, SPD, exact values), rtol 0, {K} steps",
             "nnz": int(nnz_local * world),
             "mrows": info["mrows"],
-            "kernel_variant": {1: "ldg", 2: "tma", 3: "pipe", 4: "jit"}[info["variant"]],
+            "kernel_variant": VNAME[info["variant"]],
             "check_every": check,
             "parallelism": f"row-partitioned x{world}" + (f", {transport} halo + allreduce" if world > 1 else "") + (", ranks share cuda:0 (functional only)" if args.share_gpu else ""),
             "l2": f"inputs larger than L2 ({step_bytes / 1e9:.2f} GB per step); no flush",
@@ -927,31 +892,55 @@ def run_cg(args):
         dist.destroy_process_group()
 
 
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def relaunch(args):
+    """N > 1 without a torchrun environment: start N ranks ourselves."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", f"--master-port={_free_port()}", os.path.abspath(__file__)] + sys.argv[1:]
+    env = dict(os.environ, OMP_NUM_THREADS=os.environ.get("OMP_NUM_THREADS", str(max(1, host_cores() // args.gpus))))
+    return subprocess.call(cmd, env=env)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=20)
-    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c3ns", "c4", "c5"])
-    ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
+    ap.add_argument("--config", default="c5", choices=["c1", "c2", "c3", "c3ns", "c4", "c5"])
+    ap.add_argument("--dtype", default=None, choices=["f64", "f32"], help="default: f64 (f32 for c4)")
     ap.add_argument("--mrows", type=int, default=0)
-    ap.add_argument("--variant", default="auto", choices=["auto", "ldg", "tma", "pipe", "jit"])
+    ap.add_argument("--variant", default="auto", choices=list(VARIANTS))
     ap.add_argument("--impl", default="crsd", choices=["crsd", "reference"])
     ap.add_argument("--workload", default="spmv", choices=["spmv", "cg"], help="cg: K steps of crsd_cg (N>1: row-partitioned, halo + allreduce)")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--no-sub", action="store_true", help="N=1 C5: skip the C3 f64/f32 sub-records")
     ap.add_argument("--transport", default="auto", choices=["auto", "nccl", "p2p"], help="N>1 halo exchange: the library's peer-memory kernels (p2p), NCCL send/recv, or auto (p2p if every rank can map its peers, else NCCL)")
     ap.add_argument("--share-gpu", action="store_true", help="N>1 ranks all on cuda:0 (functional check only; needs --transport p2p)")
     args = ap.parse_args()
+    if args.dtype is None:
+        args.dtype = "f32" if args.config == "c4" else "f64"
     if args.warmup < 3:
         args.warmup = 3
+    if args.gpus == 1 or args.impl == "reference":
+        # the CPU baseline's OpenMP threads spread over the host cores (read
+        # by libgomp at load, i.e. before any OpenMP code runs); not with
+        # several ranks per host, whose builders would share the same cores
+        os.environ.setdefault("OMP_PROC_BIND", "spread")
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ and args.impl != "reference":
+        sys.exit(relaunch(args))
     if args.impl == "reference":
         run_reference(args)
     elif args.workload == "cg":
         run_cg(args)
-    elif args.config == "c5" and args.gpus == 1:
-        run_c5(args)
     else:
-        run_crsd(args)
+        run_spmv(args)
 
 
 if __name__ == "__main__":

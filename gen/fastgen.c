@@ -84,12 +84,14 @@ static int stencil_row(const Stencil *S, int64_t idx, int64_t *col, double *val)
     return n;
 }
 
-/* disp: m x 3 int32 (di, dj, dk), in ascending linear-offset order. drop6:
- * k1a k1b j2a j2b k2a k2b k3a k3b or NULL. Two calls: with row == NULL it
- * returns the entry count; then fills row/col/val (int64, int64, double). */
+/* disp: m x 3 int32 (di, dj, dk), in ascending linear-offset order. drop8:
+ * k1a k1b j2a j2b k2a k2b k3a k3b or NULL. Two calls: with col == NULL it
+ * returns the entry count; then fills col/val (int64, double) and the COO
+ * rows (row, int64[count]) and/or the CSR pointers (ptr, int64[rows + 1],
+ * from 0), whichever is not NULL. */
 int64_t fg_stencil(int64_t n1, int64_t n2, int64_t n3, int32_t m, const int32_t *disp, int32_t present,
                    int32_t random, uint64_t seed, const int64_t *drop8, int64_t row_begin, int64_t row_end,
-                   int64_t *row, int64_t *col, double *val, int32_t nthreads) {
+                   int64_t *row, int64_t *ptr, int64_t *col, double *val, int32_t nthreads) {
     Stencil S;
     memset(&S, 0, sizeof(S));
     S.n1 = n1;
@@ -129,17 +131,20 @@ int64_t fg_stencil(int64_t n1, int64_t n2, int64_t n3, int32_t m, const int32_t 
     }
     for (int64_t b = 0; b < nb; ++b) cnt[b + 1] += cnt[b];
     const int64_t total = cnt[nb];
-    if (row) {
+    if (col) {
 #pragma omp parallel for schedule(dynamic, 1) num_threads(nthreads)
         for (int64_t b = 0; b < nb; ++b) {
             int64_t e = cnt[b];
             const int64_t r1 = row_begin + (b + 1 < nb ? (b + 1) * B : nr);
             for (int64_t r = row_begin + b * B; r < r1; ++r) {
                 const int n = stencil_row(&S, r, col + e, val + e);
-                for (int t = 0; t < n; ++t) row[e + t] = r;
+                if (row)
+                    for (int t = 0; t < n; ++t) row[e + t] = r;
+                if (ptr) ptr[r - row_begin] = e;
                 e += n;
             }
         }
+        if (ptr) ptr[nr] = total;
     }
     free(cnt);
     return total;
@@ -149,8 +154,8 @@ int64_t fg_stencil(int64_t n1, int64_t n2, int64_t n3, int32_t m, const int32_t 
  * (ascending); entries with columns outside [0, n) omitted; value 2u - 1
  * from counter row * 2^20 + (offset + 2^19), 0 replaced by 0.5. */
 int64_t fg_band(int64_t n, int32_t nranges, const int64_t *ra, const int64_t *rb, const int64_t *optr,
-                const int64_t *offs, uint64_t seed, int64_t row_begin, int64_t row_end, int64_t *row, int64_t *col,
-                double *val, int32_t nthreads) {
+                const int64_t *offs, uint64_t seed, int64_t row_begin, int64_t row_end, int64_t *row, int64_t *ptr,
+                int64_t *col, double *val, int32_t nthreads) {
     if (nthreads < 1) nthreads = omp_get_max_threads();
     int64_t total = 0;
     for (int32_t g = 0; g < nranges; ++g) {
@@ -172,26 +177,39 @@ int64_t fg_band(int64_t n, int32_t nranges, const int64_t *ra, const int64_t *rb
             cnt[k + 1] = c;
         }
         for (int64_t k = 0; k < nb; ++k) cnt[k + 1] += cnt[k];
-        if (row) {
+        if (col) {
 #pragma omp parallel for schedule(dynamic, 1) num_threads(nthreads)
             for (int64_t k = 0; k < nb; ++k) {
                 int64_t e = total + cnt[k];
                 const int64_t r1 = a + (k + 1 < nb ? (k + 1) * B : nr);
-                for (int64_t r = a + k * B; r < r1; ++r)
+                for (int64_t r = a + k * B; r < r1; ++r) {
+                    if (ptr) ptr[r - row_begin] = e;
                     for (int64_t q = 0; q < no; ++q) {
                         const int64_t c = r + o[q];
                         if (c < 0 || c >= n) continue;
                         double v = 2.0 * counter_uniform((uint64_t)(r * (int64_t)(1 << 20) + (o[q] + (1 << 19))), seed) - 1.0;
                         if (v == 0.0) v = 0.5;
-                        row[e] = r;
+                        if (row) row[e] = r;
                         col[e] = c;
                         val[e] = v;
                         ++e;
                     }
+                }
             }
         }
         total += cnt[nb];
         free(cnt);
+    }
+    /* rows of [row_begin, row_end) outside every range carry no entries */
+    if (col && ptr && row_end > row_begin) {
+        /* such a row starts where the next row in a range starts */
+        int64_t next = total;
+        for (int64_t r = row_end - row_begin - 1; r >= 0; --r) {
+            int in = 0;
+            for (int32_t g = 0; g < nranges; ++g) in |= (row_begin + r >= ra[g] && row_begin + r < rb[g]);
+            if (in) next = ptr[r]; else ptr[r] = next;
+        }
+        ptr[row_end - row_begin] = total;
     }
     return total;
 }

@@ -74,7 +74,9 @@ typedef enum { CRSD_R32F = 0, CRSD_R64F = 1 } crsd_dtype_t;
 /*
  * Build options. Call crsd_opts_init() for defaults (NULL opts == defaults).
  *   mrows     row-segment height (token `mrows`); 0 => 2 KB of
- *             values per diagonal run: 256 (fp64) / 512 (fp32). The
+ *             values per diagonal run: 256 (fp64) / 512 (fp32), except that
+ *             fp32 falls back to 256 when a segment's staging at 512 rows
+ *             would leave fewer than 4 CTAs per SM. The
  *             GPU path needs mrows % (32*RPT) == 0 and mrows <= 256*RPT,
  *             RPT = 2 rows per thread for fp64 and 4 for fp32 (one 128-bit
  *             vector per thread and diagonal; <= 256 threads per CTA); the
@@ -264,6 +266,12 @@ crsd_status_t crsd_dist_x_layout(crsd_matrix_t A, int64_t *halo_lo, int64_t *n_l
  * all ranks. The library creates the NCCL communicator and a comm stream. */
 crsd_status_t crsd_comm_unique_id(void *id128);
 crsd_status_t crsd_comm_init_rank(const void *id128, int rank, int world, int device, crsd_comm_t *out);
+/* Destroy a communicator. Collective for peer-memory communicators: every
+ * rank calls it; each rank first finishes all its device work, then tells
+ * every peer it is done with the peer's region and waits (bounded) for every
+ * peer to say the same before unmapping the peers' regions and freeing its
+ * own, so no rank frees memory a slower peer still reads or writes. Destroy
+ * the handles bound to it (crsd_destroy) after it. */
 crsd_status_t crsd_comm_destroy(crsd_comm_t comm);
 
 /*
@@ -303,8 +311,24 @@ crsd_status_t crsd_comm_destroy(crsd_comm_t comm);
  *       Peer memory: every rank sums the W contributions in rank order, so
  *       all ranks get bit-identical results. NCCL: ncclAllReduce.
  *   crsd_comm_error(c, &err)
- *       Synchronous. err = 0, or 1/2/3 when a send / recv / allreduce wait
- *       timed out (a peer never arrived); the results are then invalid.
+ *       Synchronous. err = 0, or 1/2/3/4 when a send / recv / allreduce /
+ *       close wait timed out (a peer never arrived); the results are then
+ *       invalid. A communicator with err != 0 is poisoned: its kernels skip
+ *       their copies and publish nothing, and once crsd_comm_error has seen
+ *       the error, crsd_spmv_dist / crsd_comm_allreduce_f64 / crsd_cg on it
+ *       return CRSD_ERR_CUDA. Recreate the communicator.
+ *   crsd_dist_x_alloc(A, c, &x_padded)
+ *       Collective over the ranks of c (peer-memory communicators; A bound
+ *       to c). Allocates this rank's padded x (halo_lo + n_local + halo_hi
+ *       elements of the dtype, zeroed, owned by A, freed by crsd_destroy) and
+ *       maps every peer's. crsd_spmv_dist called with this x_padded moves the
+ *       halo as ONE-SIDED PUTS: each rank stores its send slices straight
+ *       into the receivers' pads over NVLink (one crossing per halo byte, no
+ *       mailbox copy), signals, and the receivers release the pads after
+ *       their boundary segments. Any other x_padded uses the two-stage
+ *       mailbox path. crsd_cg over a peer-memory communicator uses this
+ *       buffer for p. Every rank must stop using it (crsd_comm_destroy, or a
+ *       barrier after its last crsd_spmv_dist) before any rank destroys A.
  */
 crsd_status_t crsd_comm_init_p2p(int rank, int world, int device, int64_t mailbox_bytes, void *ipc_handle64,
                                  crsd_comm_t *out);
@@ -312,6 +336,7 @@ crsd_status_t crsd_comm_p2p_open(crsd_comm_t comm, const void *ipc_handles);
 crsd_status_t crsd_dist_bind_ranges(crsd_matrix_t A_local, crsd_comm_t comm, const int64_t *ranges4);
 crsd_status_t crsd_comm_allreduce_f64(crsd_comm_t comm, double *dev, int n, void *stream);
 crsd_status_t crsd_comm_error(crsd_comm_t comm, int32_t *err);
+crsd_status_t crsd_dist_x_alloc(crsd_matrix_t A_local, crsd_comm_t comm, void **x_padded);
 /* This handle's row of the range table: {row_begin, row_end, halo_lo_valid,
  * halo_hi_valid} (the halo widths actually needed, without alignment). */
 crsd_status_t crsd_dist_ranges(crsd_matrix_t A_local, int64_t *ranges4);

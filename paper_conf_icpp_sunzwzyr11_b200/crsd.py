@@ -65,6 +65,7 @@ EXPORTED = [
     "crsd_comm_allreduce_f64",
     "crsd_comm_error",
     "crsd_dist_ranges",
+    "crsd_dist_x_alloc",
 ]
 
 
@@ -175,6 +176,7 @@ def _load():
         "crsd_comm_allreduce_f64": ([P, P, ctypes.c_int, P], ctypes.c_int),
         "crsd_comm_error": ([P, P], ctypes.c_int),
         "crsd_dist_ranges": ([P, P], ctypes.c_int),
+        "crsd_dist_x_alloc": ([P, P, P], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)
@@ -297,13 +299,40 @@ class CRSDMatrix:
         return cls(h.value, val.dtype), {int(m): (None if t < 0 else float(t)) for m, t in zip(cand, ms)}
 
     @classmethod
-    def from_csr(cls, nrows, ncols, row_ptr, col, val, *, mrows=0, idle_max=-1, flags=0, host_only=False, device=-1):
+    def from_csr(
+        cls,
+        nrows,
+        ncols,
+        row_ptr,
+        col,
+        val,
+        *,
+        mrows=0,
+        idle_max=-1,
+        flags=0,
+        host_only=False,
+        row_range: Optional[tuple] = None,
+        device=-1,
+        nthreads=0,
+        variant=0,
+        jit_chunk=0,
+        tune=0,
+        e2e_chunks=0,
+    ):
+        """crsd_create_from_csr: row_ptr over the owned rows (row_range, default
+        all rows). Canonical input (strictly increasing columns per row) is
+        read in place by the builder, without a copy of the entries."""
         row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
         col = np.ascontiguousarray(col, dtype=np.int64)
         val = np.ascontiguousarray(val)
+        if val.dtype not in (np.float32, np.float64):
+            val = val.astype(np.float64)
         o = Opts()
         lib.crsd_opts_init(ctypes.byref(o))
         o.mrows, o.idle_max, o.flags, o.device = mrows, idle_max, flags | (CRSD_HOST_ONLY if host_only else 0), device
+        o.nthreads, o.variant, o.jit_chunk, o.tune, o.e2e_chunks = nthreads, variant, jit_chunk, tune, e2e_chunks
+        if row_range is not None:
+            o.row_begin, o.row_end = int(row_range[0]), int(row_range[1])
         h = ctypes.c_void_p()
         _check(lib.crsd_create_from_csr(nrows, ncols, _p(row_ptr), _p(col), _p(val), _dtype_code(val.dtype), ctypes.byref(o), ctypes.byref(h)))
         return cls(h.value, val.dtype)
@@ -428,6 +457,30 @@ class CRSDMatrix:
             _check(lib.crsd_dist_bind_ranges(self._h, comm._h, _p(table)))
         else:
             _check(lib.crsd_dist_bind(self._h, comm._h, _stream_ptr(stream)))
+
+    def dist_x_alloc(self, comm):
+        """crsd_dist_x_alloc (collective): the library-owned padded x of this
+        rank, mapped by every peer, as a CUDA tensor view (halo_lo + n_local +
+        halo_hi elements; owned part at [halo_lo, halo_lo + n_local)).
+        crsd_spmv_dist with it moves the halo as one-sided puts into the
+        neighbours' pads. The view is valid while this handle lives."""
+        import torch
+
+        p = ctypes.c_void_p()
+        _check(lib.crsd_dist_x_alloc(self._h, comm._h, ctypes.byref(p)))
+        lo, n, hi = self.x_layout()
+
+        class _View:
+            __cuda_array_interface__ = {
+                "shape": (lo + n + hi,),
+                "typestr": "<f8" if self.dtype == np.float64 else "<f4",
+                "data": (p.value, False),
+                "version": 3,
+            }
+
+        t = torch.as_tensor(_View(), device=f"cuda:{torch.cuda.current_device()}")
+        self._dx = t
+        return t
 
     def dist_ranges(self) -> np.ndarray:
         """{row_begin, row_end, halo_lo_valid, halo_hi_valid} of this handle (crsd_dist_ranges)."""

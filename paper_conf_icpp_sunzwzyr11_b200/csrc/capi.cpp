@@ -68,6 +68,12 @@ void free_device(crsd_matrix_s *A) {
         cudaEventDestroy((cudaEvent_t)A->cg_ev_out);
         A->cg_stream = A->cg_ev_in = A->cg_ev_out = nullptr;
     }
+    // direct-mode padded x (crsd_dist_x_alloc): unmap the peers', free mine
+    for (void *p : A->dx_peer)
+        if (p) cudaIpcCloseMemHandle(p);
+    A->dx_peer.clear();
+    if (A->dx_own) cudaFree(A->dx_own);
+    A->dx_own = nullptr;
     void *ptrs[] = {A->d_vals, A->d_segs, A->d_offs, A->d_plan, A->d_scat_row, A->d_scat_col, A->d_scat_val, A->d_scat_rec,
                     A->d_list_interior, A->d_list_boundary, A->d_list_all_edge, A->d_x_scratch, A->d_y_scratch, A->d_cg,
                     A->d_ell_rowno, A->d_ell_col, A->d_ell_val};
@@ -380,6 +386,26 @@ static crsd_status_t create_common(int64_t nrows, int64_t ncols, crsd_dtype_t dt
     A->H.partitioned = !(o.row_begin == 0 && o.row_end == nrows);
     crsd_status_t st = csr ? build_from_csr(nrows, ncols, row_or_ptr, col, val, dtype, b, A->H)
                            : build_from_coo(nrows, ncols, nnz, row_or_ptr, col, val, dtype, b, A->H);
+    // AUTO height for fp32: 512 rows (2 KB per diagonal run) unless a
+    // segment's staging (values + x windows) would then leave fewer than 4
+    // CTAs per SM -- then 256. Measured (profiles/r02/sweep1*): C3 f32
+    // (27 diagonals, 70 KB at 512 -> 3 CTAs/SM) 1.06 of the copy peak at
+    // 256 against 1.02 at 512; C4 f32 (19 diagonals, 56 KB -> 4 CTAs/SM) and
+    // C2 f32 keep 512 (round 1 sweep19: 256 costs them 0.17-0.3).
+    const bool auto_m = (!opts || opts->mrows == 0) && dtype == CRSD_R32F && (o.row_begin % 256) == 0;
+    if (!st && auto_m && A->H.mrows == 512) {
+        std::vector<int32_t> pl;
+        std::vector<SegDesc> sg(A->H.nseg);
+        const int64_t mx = make_plans(A->H, A->H.mrows, pl, sg);
+        const int64_t per_cta = (mx + 127) / 128 * 128 + 1024 + 256;
+        if ((228 * 1024) / per_cta < 4) {
+            A->H = HostCRSD();
+            o.mrows = b.mrows = 256;
+            if (!opts || opts->idle_max < 0) o.idle_max = b.idle_max = 255;
+            st = csr ? build_from_csr(nrows, ncols, row_or_ptr, col, val, dtype, b, A->H)
+                     : build_from_coo(nrows, ncols, nnz, row_or_ptr, col, val, dtype, b, A->H);
+        }
+    }
     if (st) {
         delete A;
         return st;

@@ -25,6 +25,8 @@ struct crsd_comm_s {
     std::vector<void *> peer_sym;     // world entries, nullptr for self / not opened
     std::vector<int64_t> peer_cap;    // each peer's mailbox bytes per parity (read from its flags)
     bool opened = false;
+    bool poisoned = false;            // a wait timed out (seen by crsd_comm_error): refuse further exchanges
+    uint64_t xseq = 0;                // crsd_dist_x_alloc handshakes made
     uint64_t timeout_ns = 30ull * 1000 * 1000 * 1000;  // peer-memory waits (CRSD_P2P_TIMEOUT_S)
 };
 
@@ -33,6 +35,9 @@ namespace crsd {
 crsd_status_t comm_allreduce_f64(crsd_comm_s *c, double *dev, int n, cudaStream_t stream);
 // crsd_spmv_dist with the boundary placement chosen by the caller: -1 default,
 // 0 concurrent with the interior (comm stream), 1 serial after the interior
+// the handle's crsd_dist_x_alloc buffer (direct one-sided puts), collective
+crsd_status_t dist_x_alloc(crsd_matrix_s *A, crsd_comm_s *c);
+crsd_status_t release_halo(crsd_matrix_s *A, crsd_comm_s *c);
 crsd_status_t spmv_dist_impl(crsd_matrix_s *A, const void *alpha, void *x_padded, const void *beta, void *y_local,
                              crsd_comm_s *c, void *stream, int boundary);
 }  // namespace crsd

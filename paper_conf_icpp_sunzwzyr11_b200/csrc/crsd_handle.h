@@ -89,6 +89,12 @@ struct crsd_matrix_s {
     // peer-memory transport: byte offsets into my mailbox (sends) / the sender's mailbox (recvs)
     std::vector<int64_t> send_mb_off, recv_mb_off;
     const void *bound_comm = nullptr;
+    std::vector<int64_t> range_table;  // every rank's {row_begin, row_end, halo_lo_valid, halo_hi_valid}
+    // direct (one-sided put) mode: this rank's padded x from crsd_dist_x_alloc
+    // (IPC-exported) and every peer's, mapped; the sends land in the peers' pads
+    void *dx_own = nullptr;
+    std::vector<void *> dx_peer;
+    const void *dx_comm = nullptr;
 };
 
 namespace crsd {

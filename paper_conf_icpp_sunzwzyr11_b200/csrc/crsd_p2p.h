@@ -19,8 +19,13 @@ struct P2PFlags {
     uint64_t halo_epoch;  // own: last completed halo exchange
     uint64_t red_epoch;   // own: last completed allreduce
     uint32_t counter[2];  // own: grid arrival counters (send, recv)
-    uint32_t err;         // own: 0, or 1/2/3 = send/recv/allreduce wait timed out
+    uint32_t err;         // own: 0, or 1/2/3/4 = send/recv/allreduce/close wait timed out
     int64_t cap;          // own mailbox bytes per parity (read by peers at open)
+    uint64_t closing[P2P_MAX_WORLD];  // written by q at crsd_comm_destroy: q no longer touches my region
+    // crsd_dist_x_alloc handshake, written by q (host copies into peer memory):
+    // q's padded-x IPC handle, then xseq[q] = the allocation's sequence number
+    uint8_t xh[P2P_MAX_WORLD][64];
+    uint64_t xseq[P2P_MAX_WORLD];
 };
 static_assert(sizeof(P2PFlags) <= P2P_FLAGS_BYTES, "P2PFlags too large");
 
@@ -49,6 +54,10 @@ struct P2PReduce {
 
 int p2p_launch_send(const P2PLaunch &L, int grid, void *stream);
 int p2p_launch_recv(const P2PLaunch &L, int grid, void *stream);
+int p2p_launch_put(const P2PLaunch &L, int grid, void *stream);
+int p2p_launch_wait(const P2PLaunch &L, void *stream);
+int p2p_launch_release(const P2PLaunch &L, void *stream);
 int p2p_launch_allreduce(const P2PReduce &R, double *val, int n, void *stream);
+int p2p_launch_close(const P2PReduce &R, uint64_t token, void *stream);
 
 }  // namespace crsd

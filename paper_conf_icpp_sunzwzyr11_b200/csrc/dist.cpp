@@ -23,7 +23,9 @@
 #include <cstddef>
 #include <cstdlib>
 #include <cstring>
+#include <chrono>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "crsd_handle.h"
@@ -94,6 +96,22 @@ crsd_status_t crsd_comm_destroy(crsd_comm_t c) {
     if (!c) return CRSD_OK;
     cudaSetDevice(c->device);
     if (c->cs) cudaStreamSynchronize(c->cs);
+    if (c->kind == crsd_comm_s::P2P && c->opened && c->world > 1) {
+        // Collective close (every rank calls crsd_comm_destroy): a fast rank
+        // must not free (or let the allocator reuse) its region while a
+        // slower peer's last exchange still reads its mailbox or writes its
+        // flags. All this rank's work on the device is finished first; then
+        // every rank announces "done with your region" to every peer and
+        // waits (bounded) for all peers' announcements before unmapping.
+        cudaDeviceSynchronize();
+        crsd::P2PReduce R{};
+        R.local = (crsd::P2PFlags *)c->sym;
+        R.rank = c->rank;
+        R.world = c->world;
+        R.timeout_ns = c->timeout_ns;
+        for (int q = 0; q < c->world; ++q) R.peer_flags[q] = (crsd::P2PFlags *)c->peer_sym[q];
+        if (crsd::p2p_launch_close(R, 1, c->cs) == 0) cudaStreamSynchronize(c->cs);
+    }
     if (c->comm) ncclCommDestroy(c->comm);
     for (void *p : c->peer_sym)
         if (p) cudaIpcCloseMemHandle(p);
@@ -230,6 +248,7 @@ crsd_status_t crsd_comm_error(crsd_comm_t c, int32_t *err) {
     uint32_t v = 0;
     CU_TRY(cudaMemcpy(&v, (char *)c->sym + offsetof(crsd::P2PFlags, err), sizeof(v), cudaMemcpyDeviceToHost));
     *err = (int32_t)v;
+    if (v) c->poisoned = true;
     return CRSD_OK;
 }
 
@@ -249,6 +268,7 @@ crsd_status_t comm_allreduce_f64(crsd_comm_s *c, double *dev, int n, cudaStream_
         return CRSD_OK;
     }
     if (!c->opened) return fail(CRSD_ERR_INVALID_ARG, "call crsd_comm_p2p_open first");
+    if (c->poisoned) return fail(CRSD_ERR_CUDA, "peer-memory communicator poisoned by a timed-out wait (crsd_comm_error)");
     if (n > P2P_MAX_RED) return fail(CRSD_ERR_INVALID_ARG, "peer-memory allreduce: at most 4 values");
     P2PReduce R{};
     R.local = (P2PFlags *)c->sym;
@@ -322,51 +342,145 @@ crsd_status_t bind_table(crsd_matrix_t A, crsd_comm_t c, const int64_t *all) {
     for (int64_t k = 0; k < ns; ++k) A->send_off[k] = sb[k] - origin;
     A->send_mb_off = send_mb;
     A->recv_mb_off = recv_mb;
+    A->range_table.assign(all, all + 4 * W);
     A->bound = true;
     A->bound_comm = c;
     return CRSD_OK;
 }
 
-// One halo exchange through peer memory, on the comm stream: p2p_send packs
-// my send slices into my mailbox and flags the receivers; p2p_recv waits for
-// the senders' flags and pulls their slices into the pads of x_padded.
+// Launch record over the distinct peers of `peers` (send or receive side).
+void fill_launch(P2PLaunch &L, crsd_comm_t c, const std::vector<int64_t> &peers) {
+    L.local = (P2PFlags *)c->sym;
+    L.rank = c->rank;
+    L.timeout_ns = c->timeout_ns;
+    L.npeer = 0;
+    for (int64_t q : peers) {
+        bool seen = false;
+        for (int k = 0; k < L.npeer; ++k) seen |= (L.peer[k] == q);
+        if (!seen) {
+            L.peer[L.npeer] = (int32_t)q;
+            L.peer_flags[L.npeer] = (P2PFlags *)c->peer_sym[q];
+            ++L.npeer;
+        }
+    }
+}
+
+// One halo exchange through peer memory, on the comm stream. Direct mode
+// (x_padded is this handle's crsd_dist_x_alloc buffer): p2p_put stores my
+// send slices straight into the receivers' pads, p2p_wait waits for my
+// senders. Mailbox mode (any other x_padded): p2p_send packs my send slices
+// into my mailbox and flags the receivers; p2p_recv waits for the senders'
+// flags and pulls their slices into the pads. Either way p2p_release (after
+// the boundary segments, release_halo) frees the pads for the next epoch.
 crsd_status_t p2p_exchange(crsd_matrix_t A, crsd_comm_t c, char *xp) {
     if (!c->opened) return fail(CRSD_ERR_INVALID_ARG, "call crsd_comm_p2p_open first");
+    if (c->poisoned) return fail(CRSD_ERR_CUDA, "peer-memory communicator poisoned by a timed-out wait (crsd_comm_error)");
     const int64_t es = A->H.elem;
-    char *mb = (char *)c->sym + P2P_FLAGS_BYTES;
-    auto fill = [&](P2PLaunch &L, const std::vector<int64_t> &peers) {
-        L.local = (P2PFlags *)c->sym;
-        L.rank = c->rank;
-        L.timeout_ns = c->timeout_ns;
-        L.npeer = 0;
-        for (int64_t q : peers) {
-            bool seen = false;
-            for (int k = 0; k < L.npeer; ++k) seen |= (L.peer[k] == q);
-            if (!seen) {
-                L.peer[L.npeer] = (int32_t)q;
-                L.peer_flags[L.npeer] = (P2PFlags *)c->peer_sym[q];
-                ++L.npeer;
-            }
-        }
-    };
+    // a few CTAs suffice for the halo (~2 % of a rank's bytes); every CTA of
+    // p2p_recv / p2p_put holds an SM slot while it waits for the peers
+    const int grid = 16;
     P2PLaunch S{}, R{};
-    fill(S, A->send_peer);
+    fill_launch(S, c, A->send_peer);
+    fill_launch(R, c, A->recv_peer);
     S.nitems = (int32_t)A->send_peer.size();
+    R.nitems = (int32_t)A->recv_peer.size();
+    if (xp == (char *)A->dx_own && A->dx_comm == c) {
+        const int W = c->world;
+        for (int k = 0; k < S.nitems; ++k) {
+            const int64_t q = A->send_peer[k];
+            const int64_t gcol = A->send_off[k] + (A->H.row_begin - A->halo_lo);  // global column of the slice
+            const int64_t q_halo_lo = (A->range_table[4 * q + 2] + 3) / 4 * 4;
+            const int64_t q_origin = A->range_table[4 * q] - q_halo_lo;
+            (void)W;
+            S.items[k] = P2PItem{xp + es * A->send_off[k], (char *)A->dx_peer[q] + es * (gcol - q_origin),
+                                 es * A->send_count[k], 0};
+        }
+        CU_TRY((cudaError_t)p2p_launch_put(S, grid, c->cs));
+        CU_TRY((cudaError_t)p2p_launch_wait(R, c->cs));
+        return CRSD_OK;
+    }
+    char *mb = (char *)c->sym + P2P_FLAGS_BYTES;
     for (int k = 0; k < S.nitems; ++k)
         S.items[k] = P2PItem{xp + es * A->send_off[k], mb + A->send_mb_off[k], es * A->send_count[k], c->cap};
-    fill(R, A->recv_peer);
-    R.nitems = (int32_t)A->recv_peer.size();
     for (int k = 0; k < R.nitems; ++k)
         R.items[k] = P2PItem{(char *)c->peer_sym[A->recv_peer[k]] + P2P_FLAGS_BYTES + A->recv_mb_off[k],
                              xp + es * A->recv_off[k], es * A->recv_count[k], c->peer_cap[A->recv_peer[k]]};
-    // a few CTAs suffice for the halo (~2 % of a rank's bytes); every CTA of
-    // p2p_recv holds an SM slot while it waits for the peers
-    const int grid = 16;
     CU_TRY((cudaError_t)p2p_launch_send(S, grid, c->cs));
     CU_TRY((cudaError_t)p2p_launch_recv(R, grid, c->cs));
     return CRSD_OK;
 }
+
 }  // namespace
+
+// The boundary segments of this epoch are done with the pads: tell the senders.
+crsd_status_t release_halo(crsd_matrix_t A, crsd_comm_t c) {
+    P2PLaunch R{};
+    fill_launch(R, c, A->recv_peer);
+    CU_TRY((cudaError_t)p2p_launch_release(R, c->cs));
+    return CRSD_OK;
+}
+
+// crsd_dist_x_alloc: allocate this rank's padded x (IPC-exportable), hand
+// its IPC handle to every peer through the peers' flag regions (host copies
+// into peer memory), wait until every peer's handle has arrived in mine
+// (bounded), and map them.
+crsd_status_t dist_x_alloc(crsd_matrix_t A, crsd_comm_t c) {
+    if (c->kind != crsd_comm_s::P2P || !c->opened)
+        return fail(CRSD_ERR_INVALID_ARG, "crsd_dist_x_alloc needs an opened peer-memory communicator");
+    if (!A->bound || A->bound_comm != c) return fail(CRSD_ERR_INVALID_ARG, "bind the handle to this communicator first");
+    if (A->dx_own) return fail(CRSD_ERR_INVALID_ARG, "the handle already has a crsd_dist_x_alloc buffer");
+    const int64_t bytes = A->H.elem * (A->halo_lo + A->H.n_local + A->halo_hi);
+    void *p = nullptr;
+    CU_TRY(cudaMalloc(&p, std::max<int64_t>(bytes, 256)));
+    cudaError_t e = cudaMemset(p, 0, std::max<int64_t>(bytes, 256));
+    cudaIpcMemHandle_t h;
+    if (e == cudaSuccess) e = cudaIpcGetMemHandle(&h, p);
+    if (e != cudaSuccess) {
+        cudaFree(p);
+        return cu_fail(e, "crsd_dist_x_alloc");
+    }
+    const uint64_t seq = ++c->xseq;
+    const int W = c->world;
+    for (int q = 0; q < W && e == cudaSuccess; ++q) {
+        if (q == c->rank) continue;
+        char *pf = (char *)c->peer_sym[q];
+        e = cudaMemcpy(pf + offsetof(P2PFlags, xh) + 64 * c->rank, &h, 64, cudaMemcpyHostToDevice);
+        if (e == cudaSuccess)
+            e = cudaMemcpy(pf + offsetof(P2PFlags, xseq) + 8 * c->rank, &seq, 8, cudaMemcpyHostToDevice);
+    }
+    std::vector<void *> peer(W, nullptr);
+    const auto t0 = std::chrono::steady_clock::now();
+    for (int q = 0; q < W && e == cudaSuccess; ++q) {
+        if (q == c->rank) continue;
+        char *mine = (char *)c->sym;
+        uint64_t got = 0;
+        while (e == cudaSuccess) {
+            e = cudaMemcpy(&got, mine + offsetof(P2PFlags, xseq) + 8 * q, 8, cudaMemcpyDeviceToHost);
+            if (got >= seq) break;
+            if (std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count() * 1e9 > (double)c->timeout_ns) {
+                for (void *m : peer)
+                    if (m) cudaIpcCloseMemHandle(m);
+                cudaFree(p);
+                return fail(CRSD_ERR_CUDA, "crsd_dist_x_alloc: rank " + std::to_string(q) + " never published its buffer");
+            }
+            std::this_thread::sleep_for(std::chrono::microseconds(200));
+        }
+        cudaIpcMemHandle_t hq;
+        if (e == cudaSuccess) e = cudaMemcpy(&hq, mine + offsetof(P2PFlags, xh) + 64 * q, 64, cudaMemcpyDeviceToHost);
+        if (e == cudaSuccess) e = cudaIpcOpenMemHandle(&peer[q], hq, cudaIpcMemLazyEnablePeerAccess);
+    }
+    if (e != cudaSuccess) {
+        for (void *m : peer)
+            if (m) cudaIpcCloseMemHandle(m);
+        cudaFree(p);
+        return cu_fail(e, "crsd_dist_x_alloc handshake");
+    }
+    A->dx_own = p;
+    A->dx_peer = peer;
+    A->dx_comm = c;
+    A->device_bytes += bytes;
+    return CRSD_OK;
+}
 }  // namespace crsd
 
 extern "C" {
@@ -398,6 +512,15 @@ crsd_status_t crsd_dist_bind_ranges(crsd_matrix_t A, crsd_comm_t c, const int64_
     if (!A || !c || !ranges4) return crsd::fail(CRSD_ERR_INVALID_ARG, "NULL argument");
     if (A->host_only) return crsd::fail(CRSD_ERR_UNSUPPORTED, "host-only handle");
     return crsd::bind_table(A, c, ranges4);
+}
+
+crsd_status_t crsd_dist_x_alloc(crsd_matrix_t A, crsd_comm_t c, void **x_padded) {
+    if (!A || !c || !x_padded) return crsd::fail(CRSD_ERR_INVALID_ARG, "NULL argument");
+    *x_padded = nullptr;
+    CU_TRY(cudaSetDevice(A->device));
+    ST_TRY(crsd::dist_x_alloc(A, c));
+    *x_padded = A->dx_own;
+    return CRSD_OK;
 }
 
 crsd_status_t crsd_spmv_dist(crsd_matrix_t A, const void *alpha, void *x_padded, const void *beta, void *y_local,
@@ -437,7 +560,7 @@ crsd_status_t crsd::spmv_dist_impl(crsd_matrix_t A, const void *alpha, void *x_p
         CU_TRY(cudaStreamWaitEvent(c->cs, c->ev_x, 0));
         if (c->kind == crsd_comm_s::P2P) {
             ST_TRY(crsd::p2p_exchange(A, c, xp));
-            launches += 2;
+            launches += 2;  // send + recv, or put + wait
         } else {
             const ncclDataType_t ty = (A->H.dtype == CRSD_R64F) ? ncclFloat64 : ncclFloat32;
             NCCL_TRY(ncclGroupStart());
@@ -475,7 +598,16 @@ crsd_status_t crsd::spmv_dist_impl(crsd_matrix_t A, const void *alpha, void *x_p
     st = crsd::run_lists(A, alpha, xbase, beta, y_local, (const int32_t *)A->d_list_boundary, 0,
                          (int64_t)A->list_boundary.size(), (c && !serial) ? (void *)c->cs : stream, launches);
     if (st) return st;
-    if (c && !serial) {
+    if (c && c->kind == crsd_comm_s::P2P) {
+        // the pads are free once the boundary segments are done with them
+        if (serial) {
+            CU_TRY(cudaEventRecord(c->ev_x, s));
+            CU_TRY(cudaStreamWaitEvent(c->cs, c->ev_x, 0));
+        }
+        ST_TRY(crsd::release_halo(A, c));
+        ++launches;
+    }
+    if (c) {
         CU_TRY(cudaEventRecord(c->ev_halo, c->cs));
         CU_TRY(cudaStreamWaitEvent(s, c->ev_halo, 0));
     }

@@ -113,6 +113,14 @@ crsd_status_t cg_impl(crsd_matrix_s *A, const T *b, T *x, int32_t max_iter, doub
     CU_TRY(cudaStreamWaitEvent(s, (cudaEvent_t)A->cg_ev_in, 0));
 
     T *r = (T *)w.r, *q = (T *)w.q;
+    // peer-memory transport: p lives in the handle's crsd_dist_x_alloc
+    // buffer, so every halo moves as one-sided puts into the neighbours'
+    // pads (collective: every rank runs crsd_cg)
+    if (comm && comm->kind == crsd_comm_s::P2P && comm->world > 1) {
+        if (!A->dx_own) ST_TRY(dist_x_alloc(A, comm));
+        if (A->dx_comm != comm) return fail(CRSD_ERR_INVALID_ARG, "the handle's direct x buffer belongs to another communicator");
+        w.p_pad = (char *)A->dx_own;
+    }
     T *p_own = (T *)w.p_pad + A->halo_lo;
     int launches = 0;
     auto spmv = [&](T al, T be, T *y) -> crsd_status_t {

@@ -173,6 +173,38 @@ def test_csr_input_equals_coo():
     assert_layout_equal(A.export(), B.export())
 
 
+@pytest.mark.parametrize("mode", ["canonical", "unsorted_cols", "duplicates", "out_of_range", "row_range"])
+def test_csr_input_paths(mode):
+    """crsd_create_from_csr reads canonical CSR in place (no copy of the
+    entries); anything else goes through the COO canonicalisation. Both give
+    the COO build's layout, and the errors of the COO path."""
+    a = gen.random_diagonal(3000, 3000, 4, ndiag=9, max_off=500, n_scatter=40).sorted()
+    n = a.nrows
+    rb, re = (1024, 2560) if mode == "row_range" else (0, n)
+    m = (a.row >= rb) & (a.row < re)
+    r, c, v = a.row[m], a.col[m].copy(), a.val[m].copy()
+    ptr = np.zeros(re - rb + 1, np.int64)
+    ptr[1:] = np.cumsum(np.bincount(r - rb, minlength=re - rb))
+    A = CRSDMatrix.from_coo(n, n, r, c, v, mrows=128, host_only=True, row_range=(rb, re))
+    if mode == "unsorted_cols":
+        for q in range(0, re - rb, 7):  # reverse the columns of every 7th row
+            c[ptr[q]:ptr[q + 1]] = c[ptr[q]:ptr[q + 1]][::-1].copy()
+            v[ptr[q]:ptr[q + 1]] = v[ptr[q]:ptr[q + 1]][::-1].copy()
+    if mode == "duplicates":
+        q = int(np.argmax(np.diff(ptr) >= 2))
+        c[ptr[q] + 1] = c[ptr[q]]
+        with pytest.raises(CRSDError, match="DUPLICATE"):
+            CRSDMatrix.from_csr(n, n, ptr, c, v, mrows=128, host_only=True)
+        return
+    if mode == "out_of_range":
+        c[5] = n + 3
+        with pytest.raises(CRSDError, match="INDEX_RANGE"):
+            CRSDMatrix.from_csr(n, n, ptr, c, v, mrows=128, host_only=True)
+        return
+    B = CRSDMatrix.from_csr(n, n, ptr, c, v, mrows=128, host_only=True, row_range=(rb, re))
+    assert_layout_equal(A.export(), B.export())
+
+
 def test_gpu_handle_needs_aligned_mrows():
     a = gen.config1()
     with pytest.raises(CRSDError, match="UNSUPPORTED"):

@@ -60,3 +60,31 @@ def test_dispatch_uses_fast_path_for_large_grids():
     a = matrices.stencil((64, 64, 64), "7pt", values="random", seed=2, row_begin=10_000, row_end=260_000)
     b = matrices.stencil_numpy((64, 64, 64), "7pt", values="random", seed=2, row_begin=10_000, row_end=260_000)
     _same(b, a.row, a.col, a.val)
+
+
+@pytest.mark.parametrize("kind", ["band", "c3", "7pt"])
+def test_fast_csr_mode_matches_coo(kind):
+    """csr=True returns row pointers over the requested rows, consistent with
+    the COO rows (rows without entries included)."""
+    if kind == "band":
+        n = 300_000
+        ranges = [(1000, 90_000, [-5, 0, 7]), (120_000, 250_000, [-1, 0, 1, 40_000])]  # gaps: empty rows
+        r, c, v = fast.band(n, ranges, 4, 500, 260_000, nthreads=2)
+        p, c2, v2 = fast.band(n, ranges, 4, 500, 260_000, nthreads=2, csr=True)
+        rb, re = 500, 260_000
+    else:
+        nn = 24
+        drop = matrices.c3_drop(nn) if kind == "c3" else None
+        st = "27pt" if kind == "c3" else "7pt"
+        d3 = [nn, nn, nn]
+        disps = matrices._disps(st)
+        lin = [di + d3[0] * (dj + d3[1] * dk) for (di, dj, dk) in disps]
+        disps = [disps[q] for q in np.argsort(lin, kind="stable")]
+        rb, re = 100, nn**3 - 7
+        args = (d3, disps, kind == "c3", True, 3, None if drop is None else drop.c3_params, rb, re)
+        r, c, v = fast.stencil(*args, nthreads=2)
+        p, c2, v2 = fast.stencil(*args, nthreads=2, csr=True)
+    assert np.array_equal(c, c2) and np.array_equal(v, v2)
+    expect = np.zeros(re - rb + 1, np.int64)
+    expect[1:] = np.cumsum(np.bincount(r - rb, minlength=re - rb))
+    assert np.array_equal(p, expect)

@@ -54,7 +54,7 @@ def _matrix(case):
     raise ValueError(case)
 
 
-def _worker(rank, world, port, case, variant, q):
+def _worker(rank, world, port, case, variant, q, mode="mailbox"):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     import torch
     import torch.distributed as dist
@@ -112,12 +112,25 @@ def _worker(rank, world, port, case, variant, q):
         else:
             errs = []
             stream = torch.cuda.Stream()
+            if mode == "direct":
+                # the library-owned padded x, mapped by every peer: the halo
+                # arrives as one-sided puts. NaN pads once, before any rank
+                # can put (barrier): every call must overwrite them.
+                xdir = A.dist_x_alloc(comm)
+                xdir.fill_(float("nan"))
+                torch.cuda.synchronize()
+                dist.barrier()
             for call in range(5):  # epochs 1..5: both mailbox parities, reuse after consumed
                 x = np.random.default_rng(100 + call).uniform(-1, 1, n).astype(dt)
                 yref, scale = coo.coo_spmv(n, n, a.row, a.col, a.val, x)
-                xp = np.full(lo + nloc + hi, np.nan, dt)  # pads must be written by the exchange
-                xp[lo : lo + nloc] = x[rb:re]
-                xd = torch.from_numpy(xp).to("cuda:0", tdt)
+                if mode == "direct":
+                    # only the owned part is ours to write; peers write the pads
+                    xdir[lo : lo + nloc].copy_(torch.from_numpy(x[rb:re]).to("cuda:0", tdt))
+                    xd = xdir
+                else:
+                    xp = np.full(lo + nloc + hi, np.nan, dt)  # pads must be written by the exchange
+                    xp[lo : lo + nloc] = x[rb:re]
+                    xd = torch.from_numpy(xp).to("cuda:0", tdt)
                 yd = torch.full((nloc,), float("nan"), device="cuda:0", dtype=tdt)
                 # xd / yd were written on the default stream; the side stream
                 # (non-blocking) must not start before those writes land, or
@@ -146,13 +159,13 @@ def _worker(rank, world, port, case, variant, q):
         dist.destroy_process_group()
 
 
-def _run(case, world, variant=0, check_err=True):
+def _run(case, world, variant=0, check_err=True, mode="mailbox"):
     import torch.multiprocessing as mp
 
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    ps = [ctx.Process(target=_worker, args=(r, world, port, case, variant, q)) for r in range(world)]
+    ps = [ctx.Process(target=_worker, args=(r, world, port, case, variant, q, mode)) for r in range(world)]
     for p in ps:
         p.start()
     res = [q.get(timeout=400) for _ in range(world)]
@@ -175,12 +188,16 @@ def torch_cuda():
 
 
 @pytest.mark.parametrize(
-    "case,world,variant",
-    [("c2", 2, 0), ("c3", 2, 0), ("c4", 2, 0), ("c2", 3, 4), ("c3", 3, 3), ("multihop", 4, 0), ("c4", 4, 1)],
+    "case,world,variant,mode",
+    [("c2", 2, 0, "mailbox"), ("c3", 2, 0, "mailbox"), ("c4", 2, 0, "mailbox"), ("c2", 3, 4, "mailbox"),
+     ("c3", 3, 3, "mailbox"), ("multihop", 4, 0, "mailbox"), ("c4", 4, 1, "mailbox"),
+     ("c2", 2, 0, "direct"), ("c3", 3, 0, "direct"), ("c4", 2, 0, "direct"), ("multihop", 4, 0, "direct")],
 )
-def test_p2p_spmv_dist(torch_cuda, case, world, variant):
+def test_p2p_spmv_dist(torch_cuda, case, world, variant, mode):
+    """mailbox: caller-owned x_padded, two-stage exchange; direct: the
+    crsd_dist_x_alloc buffer, one-sided puts into the neighbours' pads."""
     _, dt, _ = _matrix(case)
-    res = _run(case, world, variant)
+    res = _run(case, world, variant, mode=mode)
     for r in res:
         assert max(r["errs"]) <= TOL[dt], (r["rank"], r["errs"])
     # bit-identical allreduce on every rank, equal to the rank-order sum

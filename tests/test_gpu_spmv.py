@@ -259,11 +259,14 @@ def test_c2_full_random_parity(torch_cuda):
 
 @pytest.mark.parametrize("variant", VARIANTS)
 @pytest.mark.parametrize("dt", [np.float64, np.float32])
-def test_c3_full_parity(torch_cuda, dt, variant):
-    """Config 3 at full size (192^3 27-pt, idle blocks, 0.1% scatter), every row."""
-    A, _ = _parity(torch_cuda, cached("c3", gen.config3), dt, 1.0, 0.0, variant=variant)
+@pytest.mark.parametrize("alpha,beta", [(1.0, 0.0), (-0.75, 0.5)])
+def test_c3_full_parity(torch_cuda, dt, variant, alpha, beta):
+    """Config 3 at full size (192^3 27-pt, idle blocks, 0.1% scatter), every
+    row, in the default height the bench uses (AUTO mrows: 256 for both
+    precisions), with and without alpha/beta."""
+    A, _ = _parity(torch_cuda, cached("c3", gen.config3), dt, alpha, beta, variant=variant)
     inf = A.info()
-    assert inf["nscatter"] > 100_000
+    assert inf["nscatter"] > 100_000 and inf["mrows"] == 256
 
 
 def test_c3_full_closed_form_ones(torch_cuda):
@@ -418,30 +421,73 @@ SLOW = pytest.mark.skipif(bool(os.environ.get("CRSD_SKIP_SLOW")), reason="CRSD_S
 
 @pytest.mark.slow
 @SLOW
-def test_c4_full_sampled(torch_cuda):
+def test_c4_full_every_row(torch_cuda):
     """BASELINE config 4 at full size (100M rows, 19 offsets / 4 patterns,
-    fp32) on one GPU in the AUTO variant, checked on a row sample that the
-    oracle evaluates one by one (plus every pattern boundary row)."""
-    if _host_ram_gb() < 120:
-        pytest.skip("needs ~120 GB of host RAM for the 1.19e9-entry COO")
+    fp32) on one GPU in the AUTO variant, alpha = -0.75, beta = 0.5: EVERY
+    row against the long-double definition (oracle.coo_spmv)."""
+    if _host_ram_gb() < 60:
+        pytest.skip("needs ~60 GB of host RAM for the 1.19e9-entry COO")
     torch = torch_cuda
     n = 100_000_000
-    a = gen.config4(n=n).astype(np.float32)
+    a = gen.config4(n=n)
+    a = gen.COO(n, n, a.row, a.col, a.val.astype(np.float32))
     A = _mat(a)
     inf = A.info()
-    assert inf["nnz"] == a.nnz and inf["nscatter"] == 0
-    x = np.random.default_rng(9).uniform(-1, 1, n).astype(np.float32)
-    y = _run(torch, A, x, 1.0, 0.0, None, n)
+    assert inf["nnz"] == a.nnz and inf["nscatter"] == 0 and inf["variant"] == 4
+    rng = np.random.default_rng(9)
+    x = rng.uniform(-1, 1, n).astype(np.float32)
+    y0 = rng.uniform(-1, 1, n).astype(np.float32)
+    y = _run(torch, A, x, -0.75, 0.5, y0, n)
+    assert A.last_launch_count() >= 1
     del A
-    # row sample: random rows + the ends of every pattern range
-    rng = np.random.default_rng(10)
-    bounds = [r for lo, hi, _ in gen.matrices.c4_ranges(n) for r in (lo, hi - 1)]
-    rows = np.unique(np.concatenate([rng.integers(0, n, 20000), np.array(bounds), np.arange(0, 64), np.arange(n - 64, n)]))
-    ptr = np.zeros(n + 1, np.int64)
-    ptr[1:] = np.cumsum(np.bincount(a.row, minlength=n))
-    yref, scale = coo.rows_spmv(rows, ptr, a.col, a.val.astype(np.float64), x.astype(np.float64))
-    err = coo.parity_error(y[rows], yref, scale)
+    yref, scale = coo.coo_spmv(n, n, a.row, a.col, a.val, x, -0.75, 0.5, y0)
+    err = coo.parity_error(y, yref, scale)
     assert err <= TOL[np.float32], err
+
+
+@pytest.mark.slow
+@SLOW
+def test_c5_full_single_handle_closed_form(torch_cuda):
+    """BASELINE config 5 at full size exactly as bench.py times it at N = 1:
+    one handle over all 452,984,832 rows, built by crsd_create_from_csr from
+    the C generator's CSR (read in place), AUTO variant. Every row of
+    y = A x and of y = -0.75 A x + 0.5 y0 is compared with the closed form
+    (x affine in the grid coordinates, y0 integer: every value exact)."""
+    if _host_ram_gb() < 110:
+        pytest.skip("needs ~110 GB of host RAM (50 GB CSR + 25 GB CRSD values + vectors)")
+    import bench
+    from gen import fast
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix
+
+    torch = torch_cuda
+    nn = 768
+    dims = (nn, nn, nn)
+    n = nn**3
+    ptr, col, val = fast.stencil(dims, bench._stencil_disps("7pt", dims), False, False, 5, None, 0, n, csr=True)
+    A = CRSDMatrix.from_csr(n, n, ptr, col, val, device=0)
+    del ptr, col, val
+    inf = A.info()
+    assert inf["nnz"] == 3_167_354_880 and inf["variant"] == 4
+    coef = (3.0, (1.0, -2.0, 5.0))
+    xd = torch.empty(n, dtype=torch.float64, device="cuda")
+    y0 = torch.empty(n, dtype=torch.float64, device="cuda")
+    ch = 1 << 26
+    for r0 in range(0, n, ch):
+        r1 = min(n, r0 + ch)
+        g = gen.matrices.grid_coords(dims, r0, r1)
+        xd[r0:r1] = torch.from_numpy(coef[0] + coef[1][0] * g[0] + coef[1][1] * g[1] + coef[1][2] * g[2])
+        y0[r0:r1] = torch.from_numpy((g[0] - 2 * g[1] + 3 * g[2]).astype(np.float64))
+    yd = torch.full((n,), float("nan"), dtype=torch.float64, device="cuda")
+    A.spmv(xd, yd, 1.0, 0.0)
+    y2 = y0.clone()
+    A.spmv(xd, y2, -0.75, 0.5)
+    torch.cuda.synchronize()
+    for r0 in range(0, n, ch):
+        r1 = min(n, r0 + ch)
+        ref = closed_forms.stencil_apply(dims, "7pt", "linear", coef, r0, r1)
+        assert np.array_equal(yd[r0:r1].cpu().numpy(), ref), r0
+        exp2 = -0.75 * ref + 0.5 * y0[r0:r1].cpu().numpy()
+        assert np.array_equal(y2[r0:r1].cpu().numpy(), exp2), r0
 
 
 @pytest.mark.slow
