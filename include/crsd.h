@@ -116,7 +116,7 @@ typedef struct {
                            window (default), k > 0 => windows split into runs of <= k diagonals, < 0 =>
                            the whole segment on one mbarrier */
     uint32_t tune;      /* CRSD_TUNE_* implementation switches (0 = the measured defaults); per handle */
-    int32_t e2e_chunks; /* crsd_spmv_host pipeline depth (row chunks); 0 => 16 */
+    int32_t e2e_chunks; /* crsd_spmv_host pipeline depth (row chunks); 0 => x bytes / 56 MB, within [16, 64] */
     int32_t reserved;   /* must be 0 */
 } crsd_opts_t;
 

@@ -229,7 +229,7 @@ static crsd_status_t finish_create(crsd_matrix_s *A, const crsd_opts_t &o, crsd_
     }
     A->jit_chunk = o.jit_chunk;
     A->tune = o.tune;
-    A->e2e_chunks = o.e2e_chunks > 0 ? o.e2e_chunks : 16;
+    A->e2e_chunks = o.e2e_chunks;  // 0: chosen from the vector size at the first crsd_spmv_host
     const bool auto_jit = !(o.tune & CRSD_TUNE_NO_JIT);
     if (o.variant == CRSD_VARIANT_JIT) A->variant = VARIANT_JIT;
     else if (o.variant == CRSD_VARIANT_LDG) A->variant = VARIANT_LDG;
@@ -486,7 +486,13 @@ crsd_status_t crsd_spmv(crsd_matrix_t A, const void *alpha, const void *x, const
 static crsd_status_t e2e_setup(crsd_matrix_s *A) {
     HostCRSD &H = A->H;
     const int64_t nseg = H.nseg;
-    int nch = (int)std::min<int64_t>(A->e2e_chunks, std::max<int64_t>(1, nseg / 32));
+    // pipeline depth: fill (the first x chunks) and drain (the last y chunk)
+    // cost ~2 chunks of transfer, every chunk ~17 us of per-copy overhead
+    // (profiles/r01_e2e_chunk_probe*: C2's 134 MB x is best at 12-16
+    // chunks); large vectors get chunks of ~56 MB, at most 64 (C5: 3.6 GB)
+    int64_t want = A->e2e_chunks;
+    if (want <= 0) want = std::min<int64_t>(64, std::max<int64_t>(16, (H.ncols * H.elem) / (56 << 20)));
+    int nch = (int)std::min<int64_t>(want, std::max<int64_t>(1, nseg / 32));
     A->e2e_nchunk = nch;
     A->e2e_seg.resize(nch + 1);
     A->e2e_xcut.resize(nch + 1);
@@ -850,6 +856,9 @@ crsd_status_t crsd_dist_ranges(crsd_matrix_t A, int64_t *r4) {
 crsd_status_t crsd_partition_rows(int64_t nrows, int32_t mrows, int world, const double *weights, int64_t *bounds) {
     if (nrows <= 0 || mrows <= 0 || world <= 0 || !bounds) return fail(CRSD_ERR_INVALID_ARG, "bad argument");
     const int64_t nseg = (nrows + mrows - 1) / mrows;
+    if (world > nseg)
+        return fail(CRSD_ERR_INVALID_ARG, "crsd_partition_rows: " + std::to_string(world) + " ranks but only " +
+                                              std::to_string(nseg) + " row segments (every rank needs one)");
     // per-segment weight prefix; cut where the prefix crosses k/world of the total
     std::vector<double> pre(nseg + 1, 0.0);
     for (int64_t s = 0; s < nseg; ++s) {
@@ -870,8 +879,11 @@ crsd_status_t crsd_partition_rows(int64_t nrows, int32_t mrows, int world, const
         // choose the nearer boundary
         int64_t cut = s;
         if (s < nseg && (pre[s + 1] - target) < (target - pre[s])) cut = s + 1;
-        int64_t prev = (bounds[k - 1] + mrows - 1) / mrows;
-        cut = std::max(cut, prev);
+        // every rank keeps at least one segment: after the previous cut, and
+        // early enough that each remaining rank still gets one
+        const int64_t prev = (bounds[k - 1] + mrows - 1) / mrows;
+        cut = std::max(cut, prev + 1);
+        cut = std::min<int64_t>(cut, nseg - (world - k));
         bounds[k] = std::min<int64_t>(nrows, cut * mrows);
     }
     bounds[world] = nrows;

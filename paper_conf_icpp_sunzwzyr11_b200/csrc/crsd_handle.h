@@ -25,7 +25,7 @@ struct crsd_matrix_s {
     std::vector<char> jit_cubin;    // the compiled codelets (crsd_jit_cubin)
     int32_t jit_chunk = 0;          // opts.jit_chunk: diagonals per staging chunk (0 = per x window, <0 = one)
     uint32_t tune = 0;              // opts.tune: CRSD_TUNE_* switches
-    int32_t e2e_chunks = 16;        // opts.e2e_chunks: crsd_spmv_host pipeline depth
+    int32_t e2e_chunks = 0;         // opts.e2e_chunks: crsd_spmv_host pipeline depth (0: from the size)
     // one-GPU launches of the one-shot codelets split into contiguous segment
     // ranges of equal occupancy class: {seg_begin, seg_count, dynamic smem}
     // {seg_begin, seg_count, dynamic smem, aux}: aux = 1 for short runs that

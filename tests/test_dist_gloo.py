@@ -133,3 +133,24 @@ def test_partition_rows_balanced():
     b = partition_rows(100_000, 512, 4, w)
     loads = [w[b[i] : b[i + 1]].sum() for i in range(4)]
     assert max(loads) / (sum(loads) / 4) < 1.02
+
+
+def test_partition_rows_never_empty():
+    """Every rank gets at least one segment, also when the weights are
+    concentrated or the ranks barely fit; more ranks than segments is an
+    error at the cause (not an 'empty row range' later)."""
+    from paper_conf_icpp_sunzwzyr11_b200 import CRSDError, partition_rows
+
+    b = partition_rows(1000, 256, 4)  # 4 segments, 4 ranks
+    assert list(b) == [0, 256, 512, 768, 1000]
+    w = np.zeros(10_000)
+    w[:10] = 1.0  # all the weight in the first segment
+    b = partition_rows(10_000, 256, 8, w)
+    assert np.all(np.diff(b) > 0) and b[0] == 0 and b[-1] == 10_000
+    assert np.all(b[1:-1] % 256 == 0)
+    w = np.zeros(10_000)
+    w[-10:] = 1.0  # all the weight in the last segment
+    b = partition_rows(10_000, 256, 8, w)
+    assert np.all(np.diff(b) > 0)
+    with pytest.raises(CRSDError, match="INVALID_ARG"):
+        partition_rows(1000, 256, 8)

@@ -54,7 +54,7 @@ def _matrix(case):
     raise ValueError(case)
 
 
-def _worker(rank, world, port, case, variant, q, mode="mailbox"):
+def _worker(rank, world, port, case, variant, q, mode="mailbox", distinct=False, transport="p2p"):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     import torch
     import torch.distributed as dist
@@ -62,9 +62,10 @@ def _worker(rank, world, port, case, variant, q, mode="mailbox"):
     dist.init_process_group("gloo", rank=rank, world_size=world)
     out = {"rank": rank}
     try:
-        from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix, P2PComm, partition_rows
+        from paper_conf_icpp_sunzwzyr11_b200 import Comm, CRSDMatrix, P2PComm, partition_rows
 
-        torch.cuda.set_device(0)
+        dev = rank if distinct else 0  # distinct: one GPU per rank (halos over NVLink)
+        torch.cuda.set_device(dev)
         a, dt, mrows = _matrix(case)
         a = a.astype(dt)
         n = a.nrows
@@ -72,20 +73,23 @@ def _worker(rank, world, port, case, variant, q, mode="mailbox"):
         bounds = partition_rows(n, mrows, world, np.bincount(a.row, minlength=n).astype(np.float64))
         rb, re = int(bounds[rank]), int(bounds[rank + 1])
         m = (a.row >= rb) & (a.row < re)
-        A = CRSDMatrix.from_coo(n, n, a.row[m], a.col[m], a.val[m], mrows=mrows, row_range=(rb, re), variant=0 if variant == "timeout" else variant, device=0)
+        A = CRSDMatrix.from_coo(n, n, a.row[m], a.col[m], a.val[m], mrows=mrows, row_range=(rb, re), variant=0 if variant == "timeout" else variant, device=dev)
         if variant == "timeout":
             os.environ["CRSD_P2P_TIMEOUT_S"] = "2"
         # capacities differ per rank on purpose: a receiver must address the
         # sender's parity-1 mailbox with the sender's capacity, not its own
-        comm = P2PComm(rank, world, 0, mailbox_bytes=(1 << 20) * (rank + 1))
+        if transport == "nccl":
+            comm = Comm(rank, world, dev)
+        else:
+            comm = P2PComm(rank, world, dev, mailbox_bytes=(1 << 20) * (rank + 1))
         A.dist_bind(comm)
         lo, nloc, hi = A.x_layout()
         if variant == "timeout":
             # rank 1 never joins the exchange: rank 0's receive must give up
             # after 2 s and report it instead of hanging the GPU
             if rank == 0:
-                xd = torch.zeros(lo + nloc + hi, device="cuda:0", dtype=tdt)
-                yd = torch.empty(nloc, device="cuda:0", dtype=tdt)
+                xd = torch.zeros(lo + nloc + hi, device=f"cuda:{dev}", dtype=tdt)
+                yd = torch.empty(nloc, device=f"cuda:{dev}", dtype=tdt)
                 A.spmv_dist(xd, yd, 1.0, 0.0, comm)
                 torch.cuda.synchronize()
             dist.barrier()
@@ -97,8 +101,8 @@ def _worker(rank, world, port, case, variant, q, mode="mailbox"):
             b = rng.uniform(-1, 1, n)
             x0 = np.zeros(n)
             iters = 40
-            bd = torch.from_numpy(b[rb:re].astype(dt)).to("cuda:0")
-            xd = torch.from_numpy(x0[rb:re].astype(dt)).to("cuda:0")
+            bd = torch.from_numpy(b[rb:re].astype(dt)).to(f"cuda:{dev}")
+            xd = torch.from_numpy(x0[rb:re].astype(dt)).to(f"cuda:{dev}")
             res = A.cg(bd, xd, iters, 0.0, check_every=7, comm=comm, history=True)
             torch.cuda.synchronize()
             xr, _, hr = cg_ref.cg(a, b.astype(dt).astype(np.float64), x0, res["iterations"])
@@ -125,13 +129,13 @@ def _worker(rank, world, port, case, variant, q, mode="mailbox"):
                 yref, scale = coo.coo_spmv(n, n, a.row, a.col, a.val, x)
                 if mode == "direct":
                     # only the owned part is ours to write; peers write the pads
-                    xdir[lo : lo + nloc].copy_(torch.from_numpy(x[rb:re]).to("cuda:0", tdt))
+                    xdir[lo : lo + nloc].copy_(torch.from_numpy(x[rb:re]).to(f"cuda:{dev}", tdt))
                     xd = xdir
                 else:
                     xp = np.full(lo + nloc + hi, np.nan, dt)  # pads must be written by the exchange
                     xp[lo : lo + nloc] = x[rb:re]
-                    xd = torch.from_numpy(xp).to("cuda:0", tdt)
-                yd = torch.full((nloc,), float("nan"), device="cuda:0", dtype=tdt)
+                    xd = torch.from_numpy(xp).to(f"cuda:{dev}", tdt)
+                yd = torch.full((nloc,), float("nan"), device=f"cuda:{dev}", dtype=tdt)
                 # xd / yd were written on the default stream; the side stream
                 # (non-blocking) must not start before those writes land, or
                 # the NaN pads of xd could overwrite the received halo
@@ -143,7 +147,7 @@ def _worker(rank, world, port, case, variant, q, mode="mailbox"):
             out["errs"] = errs
             out["launches"] = A.last_launch_count()
             # scalar allreduce: every rank contributes distinct values; results bit-identical
-            v = torch.tensor([0.1 * (rank + 1), 1e16 * (-1) ** rank, 3.0 + rank / 7.0], dtype=torch.float64, device="cuda:0")
+            v = torch.tensor([0.1 * (rank + 1), 1e16 * (-1) ** rank, 3.0 + rank / 7.0], dtype=torch.float64, device=f"cuda:{dev}")
             comm.allreduce_f64(v)
             torch.cuda.synchronize()
             out["red"] = v.cpu().numpy().tobytes().hex()
@@ -159,13 +163,13 @@ def _worker(rank, world, port, case, variant, q, mode="mailbox"):
         dist.destroy_process_group()
 
 
-def _run(case, world, variant=0, check_err=True, mode="mailbox"):
+def _run(case, world, variant=0, check_err=True, mode="mailbox", distinct=False, transport="p2p"):
     import torch.multiprocessing as mp
 
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    ps = [ctx.Process(target=_worker, args=(r, world, port, case, variant, q, mode)) for r in range(world)]
+    ps = [ctx.Process(target=_worker, args=(r, world, port, case, variant, q, mode, distinct, transport)) for r in range(world)]
     for p in ps:
         p.start()
     res = [q.get(timeout=400) for _ in range(world)]
@@ -231,3 +235,37 @@ def test_p2p_wait_is_bounded(torch_cuda):
     timeout (2) on that rank; the other rank saw nothing wrong."""
     res = _run("c2", 2, "timeout", check_err=False)
     assert res[0]["err"] == 2 and res[1]["err"] == 0, res
+
+
+def _ngpus():
+    import torch
+
+    return torch.cuda.device_count() if torch.cuda.is_available() else 0
+
+
+@pytest.mark.parametrize("transport,mode", [("p2p", "mailbox"), ("p2p", "direct"), ("nccl", "mailbox")])
+@pytest.mark.parametrize("case", ["c2", "c4", "multihop"])
+def test_distinct_devices_spmv_dist(torch_cuda, case, transport, mode):
+    """Ranks on DISTINCT GPUs (runs whenever >= 2 are visible; the gpurun
+    boxes have one): the halo crosses NVLink -- NCCL send/recv, or the
+    library's peer-memory kernels (mailbox pull or one-sided puts) -- and each
+    rank's rows match the oracle over 5 consecutive exchanges."""
+    world = min(_ngpus(), 4 if case == "multihop" else 2)
+    if world < 2:
+        pytest.skip("needs >= 2 visible GPUs")
+    _, dt, _ = _matrix(case)
+    res = _run(case, world, 0, mode=mode, distinct=True, transport=transport)
+    for r in res:
+        assert max(r["errs"]) <= TOL[dt], (r["rank"], r["errs"])
+
+
+@pytest.mark.parametrize("transport", ["p2p", "nccl"])
+def test_distinct_devices_cg(torch_cuda, transport):
+    """Distributed CG with one GPU per rank (>= 2 visible GPUs) against the CG oracle."""
+    if _ngpus() < 2:
+        pytest.skip("needs >= 2 visible GPUs")
+    res = _run("cg7pt", 2, distinct=True, transport=transport)
+    for r in res:
+        assert r["rr_rel"] <= 1e-11 and r["x_rel"] <= 1e-12, r
+    if transport == "p2p":
+        assert len({r["rr_bits"] for r in res}) == 1
