@@ -250,6 +250,26 @@ def copy_bandwidth(dev, reps=5):
     return round(best, 1)
 
 
+def read_bandwidth(dev, reps=5):
+    """Read-only HBM bandwidth on this box (torch sum over 4 GiB of fp32, best
+    of `reps`): context for a read-dominated stream such as SpMV, whose
+    fraction of the copy peak (read + write) can exceed 1."""
+    import torch
+
+    a = torch.ones(1 << 30, dtype=torch.float32, device=f"cuda:{dev}")
+    best = 0.0
+    for _ in range(reps + 1):
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s.record()
+        a.sum()
+        e.record()
+        e.synchronize()
+        best = max(best, a.numel() * 4 / (s.elapsed_time(e) * 1e-3) / 1e9)
+    del a
+    torch.cuda.empty_cache()
+    return round(best, 1)
+
+
 def load_traffic(key):
     """ncu dram bytes (read + write) per launch of the dominant kernel on this
     workload, from one `ncu --set full` capture (profiles/traffic.json, keyed
@@ -594,6 +614,7 @@ def run_spmv(args):
     if world == 1 and not args.no_cpu:
         cpu = cpu_baseline(args.config, args.dtype)
     box_copy = copy_bandwidth(dev)
+    box_read = read_bandwidth(dev)
     kname = KNAME[info["variant"]]
     line = {
         "metric": METRIC,
@@ -641,6 +662,8 @@ def run_spmv(args):
             "launches_per_step": round(launches_all / world / max(1, args.steps), 2),
             "scope": "per GPU: whole-job algorithmic bytes / N / the max-over-ranks CUDA-event step time; with several launches per step (occupancy-class ranges, interior/boundary) the step's bytes / the step's time",
             "copy_gbs_this_box": box_copy,
+            "read_gbs_this_box": box_read,
+            "frac_of_this_box_read": round(achieved / box_read, 4) if box_read else None,
         },
         "north_star_c3": subs,
         "cpu_baseline": cpu,

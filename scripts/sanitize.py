@@ -28,8 +28,10 @@ def main():
             x = np.random.default_rng(1).uniform(-1, 1, b.ncols).astype(dt)
             y0 = np.random.default_rng(2).uniform(-1, 1, b.nrows).astype(dt)
             yref, sc = coo.coo_spmv(b.nrows, b.ncols, b.row, b.col, b.val, x, -0.75, 0.5, y0)
-            for v in (1, 2, 3, 4):
-                A = CRSDMatrix.from_coo(b.nrows, b.ncols, b.row, b.col, b.val, variant=v)
+            # variants 1-4; the JIT codelet also with one barrier (-1), two
+            # diagonals per chunk (2) and descriptor-issued copies (tune 1)
+            for v, chunk, tune in ((1, 0, 0), (2, 0, 0), (3, 0, 0), (4, 0, 0), (4, -1, 0), (4, 2, 0), (4, 0, 1)):
+                A = CRSDMatrix.from_coo(b.nrows, b.ncols, b.row, b.col, b.val, variant=v, jit_chunk=chunk, tune=tune)
                 tdt = torch.float64 if dt == np.float64 else torch.float32
                 xd = torch.from_numpy(x).to("cuda", tdt)
                 yd = torch.from_numpy(y0).to("cuda", tdt)
@@ -38,7 +40,7 @@ def main():
                 err = coo.parity_error(yd.cpu().numpy(), yref, sc)
                 ok = err <= (1e-12 if dt == np.float64 else 1e-5)
                 bad += not ok
-                print(f"{name} {np.dtype(dt).name} variant {v}: parity {err:.2e} {'ok' if ok else 'FAIL'}", flush=True)
+                print(f"{name} {np.dtype(dt).name} variant {v} chunk {chunk} tune {tune}: parity {err:.2e} {'ok' if ok else 'FAIL'}", flush=True)
     # JIT launches split by occupancy class (forced on a small C4: several
     # ranges with their own dynamic smem)
     from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_SPLIT_ALL

@@ -17,15 +17,16 @@ from tests import test_gpu_p2p as t  # noqa: E402
 
 def main():
     bad = 0
-    for case, world, variant in (("c3", 2, 0), ("multihop", 3, 4), ("cg7pt", 2, 0)):
-        res = t._run(case, world, variant)
+    for case, world, variant, mode in (("c3", 2, 0, "mailbox"), ("multihop", 3, 4, "mailbox"), ("c3", 2, 0, "direct"),
+                                       ("multihop", 4, 0, "direct"), ("cg7pt", 2, 0, "direct")):
+        res = t._run(case, world, variant, mode=mode)
         for r in res:
             if "errs" in r:
                 ok = max(r["errs"]) <= 1e-12
             else:
                 ok = r["rr_rel"] <= 1e-11 and r["x_rel"] <= 1e-12
             bad += not ok
-            print(f"{case} world {world} rank {r['rank']}: {'ok' if ok else 'FAIL'}", flush=True)
+            print(f"{case} {mode} world {world} rank {r['rank']}: {'ok' if ok else 'FAIL'}", flush=True)
     sys.exit(1 if bad else 0)
 
 
