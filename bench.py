@@ -130,6 +130,23 @@ def rank_rows(cfg, world, rank, mrows=256):
     return N, int(b[rank]), int(b[rank + 1])
 
 
+def coo_matrix(cfg, dtype):
+    """The whole single-GPU workload `cfg` as a COO (gen.COO; values in the
+    dtype) -- for scripts that build several handles of one matrix."""
+    import gen
+
+    dt = np.float64 if dtype == "f64" else np.float32
+    a = {
+        "c1": gen.config1,
+        "c2": gen.config2,
+        "c3": gen.config3,
+        "c3ns": lambda: gen.config3(scatter_frac=0.0),
+        "c4": gen.config4,
+        "c5": gen.config5,
+    }[cfg]()
+    return gen.COO(a.nrows, a.ncols, a.row, a.col, a.val.astype(dt))
+
+
 def build(cfg, dtype, world, rank, dev, mrows=0, variant=0, nthreads=0):
     """Build this rank's CRSD handle for config `cfg`. Large configs are
     generated as CSR by gen/fastgen.c and handed to crsd_create_from_csr,

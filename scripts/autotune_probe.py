@@ -17,7 +17,7 @@ PEAK = bench.measured_peaks()[0]
 CANDS = {"f64": (128, 256, 512), "f32": (256, 512, 1024)}
 for case in sys.argv[1:] or ["c2:f64", "c2:f32", "c3:f64", "c3:f32", "c4:f32"]:
     cfg, dt = case.split(":")
-    a, _, _, _ = bench.workload(cfg, dt, 1, 0)
+    a = bench.coo_matrix(cfg, dt)
     A, ms = CRSDMatrix.autotuned(a.nrows, a.ncols, a.row, a.col, a.val, mrows_candidates=CANDS[dt], reps=50)
     inf = A.info()
     best = ms[inf["mrows"]]

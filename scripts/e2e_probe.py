@@ -7,7 +7,7 @@ sys.path.insert(0, ROOT)
 import bench
 from paper_conf_icpp_sunzwzyr11_b200 import CRSDMatrix
 torch.cuda.set_device(0)
-a, _, _, _ = bench.workload("c2", "f64", 1, 0)
+a = bench.coo_matrix("c2", "f64")
 xh = torch.from_numpy(np.random.default_rng(7).uniform(-1, 1, a.ncols)).pin_memory()
 yh = torch.empty(a.nrows, dtype=torch.float64).pin_memory()
 for ch in sys.argv[1:] or ["8", "16", "32", "64"]:

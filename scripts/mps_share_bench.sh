@@ -15,9 +15,9 @@ $MPS -d >> gpurun_out/mps.log 2>&1
 sleep 2
 for N in ${MPS_NS:-1 2 4}; do
   if [ "$N" = 1 ]; then
-    timeout 300 python bench.py --steps 100 --warmup 10 --no-cpu ${MPS_ARGS} > gpurun_out/bench_mps1.json 2> gpurun_out/bench_mps1.err
+    timeout 300 python bench.py --config c2 --steps 100 --warmup 10 --no-cpu ${MPS_ARGS} > gpurun_out/bench_mps1.json 2> gpurun_out/bench_mps1.err
   else
-    timeout 400 python -m torch.distributed.run --nnodes=1 --nproc-per-node $N --master-addr 127.0.0.1 --master-port 2966$N bench.py --gpus $N --share-gpu --steps 100 --warmup 10 --no-cpu ${MPS_ARGS} > gpurun_out/bench_mps$N.json 2> gpurun_out/bench_mps$N.err
+    timeout 400 python -m torch.distributed.run --nnodes=1 --nproc-per-node $N --master-addr 127.0.0.1 --master-port 2966$N bench.py --gpus $N --share-gpu --config c2 --steps 100 --warmup 10 --no-cpu ${MPS_ARGS} > gpurun_out/bench_mps$N.json 2> gpurun_out/bench_mps$N.err
   fi
   echo "N=$N rc=$?" >> gpurun_out/mps.log
 done

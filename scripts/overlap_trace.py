@@ -14,6 +14,7 @@ JSON summary line per rank.
 """
 import json
 import os
+import re
 import sys
 
 import numpy as np
@@ -66,45 +67,29 @@ def main():
     ks = [e for e in tr["traceEvents"] if e.get("cat") == "kernel"]
     ks.sort(key=lambda e: e["ts"])
     streams = sorted({e["args"].get("stream") for e in ks})
-    # the compute stream carries the interior crsd_jit launches (the most
-    # kernel time); the comm stream the p2p_* kernels
+    # the comm stream carries the p2p_* kernels and the boundary segments;
+    # the compute stream the interior segments (one crsd_jit launch per call
+    # for these matrices). A call = one interior launch and the comm-stream
+    # kernels that follow it up to the next interior launch.
     comm_stream = next(e["args"]["stream"] for e in ks if "p2p" in e["name"])
-    steps = []
-    cur = None
-    for e in ks:
-        nm, st = e["name"], e["args"].get("stream")
-        t0, t1 = e["ts"], e["ts"] + e["dur"]
-        is_first = ("p2p_put" in nm or "p2p_send" in nm)
-        if is_first:
-            cur = {"interior": [], "halo": []}
-            steps.append(cur)
-        if cur is None:
-            continue
-        if st == comm_stream:
-            cur["halo"].append((t0, t1, nm))
-        else:
-            cur["interior"].append((t0, t1, nm))
-    # interior launches were issued before the exchange of the same call:
-    # attach each interior kernel to the step whose halo starts within it
+    inter = [e for e in ks if e["args"].get("stream") != comm_stream]
+    comm_k = [e for e in ks if e["args"].get("stream") == comm_stream]
     recs = []
-    inter_all = [(e["ts"], e["ts"] + e["dur"]) for e in ks if e["args"].get("stream") != comm_stream]
-    for s in steps:
-        if not s["halo"]:
+    for i, e in enumerate(inter):
+        i0, i1 = e["ts"], e["ts"] + e["dur"]
+        nxt = inter[i + 1]["ts"] if i + 1 < len(inter) else float("inf")
+        mine = [c for c in comm_k if i0 <= c["ts"] < nxt]
+        if not mine:
             continue
-        h0 = min(a for a, _, _ in s["halo"])
-        h1 = max(b for _, b, _ in s["halo"])
-        spans = [(a, b) for a, b in inter_all if a <= h1 and b >= h0]
-        if not spans:
-            continue
-        i0, i1 = min(a for a, _ in spans), max(b for _, b in spans)
-        inside = sum(max(0.0, min(b, i1) - max(a, i0)) for a, b, _ in s["halo"])
-        total = sum(b - a for a, b, _ in s["halo"])
-        recs.append({"interior_us": round(i1 - i0, 1), "halo_path_us": round(h1 - h0, 1),
-                     "halo_kernel_us": round(total, 1), "halo_inside_interior": round(inside / total, 3) if total else None,
-                     "halo_ends_before_interior": h1 <= i1,
-                     "halo_kernels": [n.split("(")[0] for _, _, n in s["halo"]]})
+        tl = [(re.search(r"p2p_\w+", c["name"]).group(0) if "p2p" in c["name"] else "boundary " + c["name"],
+               round(c["ts"] - i0, 1), round(c["ts"] + c["dur"] - i0, 1)) for c in mine]
+        busy = sum(c["dur"] for c in mine)
+        inside = sum(max(0.0, min(c["ts"] + c["dur"], i1) - max(c["ts"], i0)) for c in mine)
+        recs.append({"interior_us": round(i1 - i0, 1), "comm_path_end_us": round(max(c["ts"] + c["dur"] for c in mine) - i0, 1),
+                     "comm_kernel_us_inside_interior": round(inside, 1), "comm_kernel_us": round(busy, 1),
+                     "timeline_us_from_interior_start": tl})
     print(json.dumps({"rank": rank, "world": world, "config": desc, "mode": mode, "streams": len(streams),
-                      "steps": recs[1:]}), flush=True)
+                      "calls": recs}), flush=True)
     comm.close()
     dist.destroy_process_group()
 

@@ -52,7 +52,7 @@ def main():
         parts = case.split(":")
         cfg, dt = parts[0], parts[1]
         mrows = int(parts[2]) if len(parts) > 2 else 0
-        a, desc, _, _ = bench.workload(cfg, dt, 1, 0)
+        a = bench.coo_matrix(cfg, dt)
         tdt = torch.float64 if dt == "f64" else torch.float32
         x = torch.rand(a.ncols, dtype=tdt, device="cuda")
         y = torch.empty(a.nrows, dtype=tdt, device="cuda")
