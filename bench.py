@@ -365,6 +365,9 @@ def sub_record(cfg, dtype, args, dev):
     A.close()
     del x, y
     torch.cuda.empty_cache()
+    if not args.no_cpu:
+        # the oracle's native loop on the WHOLE matrix (C1-C3 run in full)
+        rec["cpu_baseline"] = cpu_baseline(cfg, dtype, cap_nnz=1 << 62)
     return rec
 
 
