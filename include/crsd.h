@@ -131,6 +131,8 @@ typedef struct {
 #define CRSD_TUNE_DIST_BOUNDARY_SERIAL 0x10u /* crsd_spmv_dist / crsd_cg: boundary segments after the interior on
                                               the caller's stream instead of behind the exchange on the comm stream */
 #define CRSD_TUNE_NO_JIT 0x20u             /* AUTO never picks the JIT variant */
+#define CRSD_TUNE_HALO_UNFUSED 0x40u       /* crsd_spmv_dist direct mode: separate wait / release kernels instead of
+                                              the receive fused into the boundary kernel (crsd_jit_halo) */
 
 #define CRSD_VARIANT_AUTO 0
 #define CRSD_VARIANT_LDG 1

@@ -22,4 +22,5 @@ from .crsd import (  # noqa: F401
     TUNE_JIT_SEQUENTIAL,
     TUNE_DIST_BOUNDARY_SERIAL,
     TUNE_NO_JIT,
+    TUNE_HALO_UNFUSED,
 )

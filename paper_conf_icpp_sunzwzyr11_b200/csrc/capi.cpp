@@ -295,9 +295,10 @@ static crsd_status_t resolve_opts(int64_t nrows, crsd_dtype_t dtype, const crsd_
 
 template <typename T>
 static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *y, const int32_t *list,
-                              int64_t seg_begin, int64_t count, void *stream, int &launches) {
+                              int64_t seg_begin, int64_t count, void *stream, int &launches, const HaloSync *halo) {
     if (count <= 0) return CRSD_OK;
     SpmvArgs<T> a;
+    a.halo = halo;
     a.vals = (const T *)A->d_vals;
     a.segs = (const SegDesc *)A->d_segs;
     a.pat_offs = (const int32_t *)A->d_offs;
@@ -343,12 +344,14 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
 }
 
 crsd_status_t run_lists(crsd_matrix_s *A, const void *alpha, const void *x_base, const void *beta, void *y,
-                        const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches) {
+                        const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches,
+                        const HaloSync *halo) {
+    if (halo && A->variant != VARIANT_JIT) return fail(CRSD_ERR_UNSUPPORTED, "fused halo receive needs the JIT variant");
     if (A->H.dtype == CRSD_R64F)
         return run_spmv<double>(A, *(const double *)alpha, (const double *)x_base, *(const double *)beta, (double *)y,
-                                list, seg_begin, count, stream, launches);
+                                list, seg_begin, count, stream, launches, halo);
     return run_spmv<float>(A, *(const float *)alpha, (const float *)x_base, *(const float *)beta, (float *)y, list,
-                           seg_begin, count, stream, launches);
+                           seg_begin, count, stream, launches, halo);
 }
 
 }  // namespace crsd

@@ -22,6 +22,7 @@ struct crsd_matrix_s {
     std::string jit_source;
     void *jit_module = nullptr;
     void *jit_function = nullptr;
+    void *jit_halo_function = nullptr;  // the same codelets with the fused halo receive (crsd_jit_halo)
     std::vector<char> jit_cubin;    // the compiled codelets (crsd_jit_cubin)
     int32_t jit_chunk = 0;          // opts.jit_chunk: diagonals per staging chunk (0 = per x window, <0 = one)
     uint32_t tune = 0;              // opts.tune: CRSD_TUNE_* switches
@@ -107,6 +108,9 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &a, void *stream);
 // Run the SpMV kernel over a device list of segments (list == nullptr: the
 // segment range [seg_begin, seg_begin + count)). x_base is the local x base
 // (x_padded + halo_lo).
+// halo != null: the boundary launch of a direct-mode exchange with the
+// receive side fused into the JIT kernel (crsd_jit_halo).
 crsd_status_t run_lists(crsd_matrix_s *A, const void *alpha, const void *x_base, const void *beta, void *y,
-                        const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches);
+                        const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches,
+                        const HaloSync *halo = nullptr);
 }  // namespace crsd

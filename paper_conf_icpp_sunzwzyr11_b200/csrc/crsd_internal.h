@@ -140,6 +140,25 @@ void needed_halo(const HostCRSD &H, int rpt, int64_t &need_lo, int64_t &need_hi)
 // ----------------------------------------------------------------------------
 // device side
 // ----------------------------------------------------------------------------
+// Receive side of a one-sided halo exchange fused into the boundary
+// segments' kernel (JIT variant, peer-memory direct mode; dist.cpp): every
+// CTA's thread 0 waits (bounded) until each sender has published this
+// epoch's puts (ready[peer[k]] >= halo_epoch + 1) before it copies x windows
+// that reach into the pads; the last CTA to finish releases the pads to the
+// senders (*consumed[k] = epoch) and advances halo_epoch. Mirrored in the
+// generated source (jit.cpp).
+constexpr int HALO_MAX_PEERS = 16;
+struct HaloSync {
+    const uint64_t *ready;                 // my flags.ready[], indexed by peer rank
+    uint64_t *halo_epoch;                  // my flags.halo_epoch
+    uint32_t *counter;                     // my flags.counter[1] (grid arrival)
+    uint32_t *err;                         // my flags.err (set on timeout)
+    uint64_t *consumed[HALO_MAX_PEERS];    // &peer_flags(sender k)->consumed[me]
+    int32_t peer[HALO_MAX_PEERS];          // sender ranks
+    int32_t npeer, pad_;
+    uint64_t timeout_ns;
+};
+
 template <typename T>
 struct SpmvArgs {
     const T *vals;
@@ -166,6 +185,7 @@ struct SpmvArgs {
     int32_t has_scatter;      // the matrix has scatter points (selects the staging kernel)
     int32_t variant;          // VARIANT_LDG / _TMA / _PIPE / _JIT
     T alpha, beta;
+    const HaloSync *halo = nullptr;  // JIT boundary launch with the fused halo receive, or null
 };
 
 // Paper-exact scatter rows (CRSD_PAPER_ELL): y[rowno[i]] = alpha * sum_k

@@ -372,7 +372,7 @@ void fill_launch(P2PLaunch &L, crsd_comm_t c, const std::vector<int64_t> &peers)
 // into my mailbox and flags the receivers; p2p_recv waits for the senders'
 // flags and pulls their slices into the pads. Either way p2p_release (after
 // the boundary segments, release_halo) frees the pads for the next epoch.
-crsd_status_t p2p_exchange(crsd_matrix_t A, crsd_comm_t c, char *xp) {
+crsd_status_t p2p_exchange(crsd_matrix_t A, crsd_comm_t c, char *xp, bool fused_recv, int &launches) {
     if (!c->opened) return fail(CRSD_ERR_INVALID_ARG, "call crsd_comm_p2p_open first");
     if (c->poisoned) return fail(CRSD_ERR_CUDA, "peer-memory communicator poisoned by a timed-out wait (crsd_comm_error)");
     const int64_t es = A->H.elem;
@@ -396,7 +396,11 @@ crsd_status_t p2p_exchange(crsd_matrix_t A, crsd_comm_t c, char *xp) {
                                  es * A->send_count[k], 0};
         }
         CU_TRY((cudaError_t)p2p_launch_put(S, grid, c->cs));
-        CU_TRY((cudaError_t)p2p_launch_wait(R, c->cs));
+        ++launches;
+        if (!fused_recv) {  // else the boundary kernel waits itself (crsd_jit_halo)
+            CU_TRY((cudaError_t)p2p_launch_wait(R, c->cs));
+            ++launches;
+        }
         return CRSD_OK;
     }
     char *mb = (char *)c->sym + P2P_FLAGS_BYTES;
@@ -407,7 +411,29 @@ crsd_status_t p2p_exchange(crsd_matrix_t A, crsd_comm_t c, char *xp) {
                              xp + es * A->recv_off[k], es * A->recv_count[k], c->peer_cap[A->recv_peer[k]]};
     CU_TRY((cudaError_t)p2p_launch_send(S, grid, c->cs));
     CU_TRY((cudaError_t)p2p_launch_recv(R, grid, c->cs));
+    launches += 2;
     return CRSD_OK;
+}
+
+// The receive side of a direct-mode exchange for the boundary kernel
+// (crsd_jit_halo): my flags, the senders, where to release them.
+void make_halo_sync(crsd_matrix_t A, crsd_comm_t c, HaloSync &h) {
+    P2PFlags *me = (P2PFlags *)c->sym;
+    h = HaloSync{};
+    h.ready = me->ready;
+    h.halo_epoch = &me->halo_epoch;
+    h.counter = &me->counter[1];
+    h.err = &me->err;
+    h.timeout_ns = c->timeout_ns;
+    h.npeer = 0;
+    for (int64_t q : A->recv_peer) {
+        bool seen = false;
+        for (int k = 0; k < h.npeer; ++k) seen |= (h.peer[k] == q);
+        if (seen) continue;
+        h.peer[h.npeer] = (int32_t)q;
+        h.consumed[h.npeer] = &((P2PFlags *)c->peer_sym[q])->consumed[c->rank];
+        ++h.npeer;
+    }
 }
 
 }  // namespace
@@ -556,11 +582,19 @@ crsd_status_t crsd::spmv_dist_impl(crsd_matrix_t A, const void *alpha, void *x_p
     // kernels slot in as CTAs retire (launching the exchange first measured
     // the same under MPS).
     if (c) CU_TRY(cudaEventRecord(c->ev_x, s));
+    // Direct mode (one-sided puts into this handle's crsd_dist_x_alloc
+    // buffer) with the JIT kernel: the receive side is fused into the
+    // boundary segments' kernel -- each CTA waits for the senders' flags
+    // before copying its x windows, the last CTA releases the pads -- so a
+    // call is put + interior + boundary, no separate wait / release kernels
+    // (CRSD_TUNE_HALO_UNFUSED restores them).
+    const bool fused = c && c->kind == crsd_comm_s::P2P && xp == (char *)A->dx_own && A->dx_comm == c &&
+                       A->variant == VARIANT_JIT && A->jit_halo_function && !A->list_boundary.empty() &&
+                       !(A->tune & CRSD_TUNE_HALO_UNFUSED);
     auto exchange = [&]() -> crsd_status_t {
         CU_TRY(cudaStreamWaitEvent(c->cs, c->ev_x, 0));
         if (c->kind == crsd_comm_s::P2P) {
-            ST_TRY(crsd::p2p_exchange(A, c, xp));
-            launches += 2;  // send + recv, or put + wait
+            ST_TRY(crsd::p2p_exchange(A, c, xp, fused, launches));
         } else {
             const ncclDataType_t ty = (A->H.dtype == CRSD_R64F) ? ncclFloat64 : ncclFloat32;
             NCCL_TRY(ncclGroupStart());
@@ -595,10 +629,13 @@ crsd_status_t crsd::spmv_dist_impl(crsd_matrix_t A, const void *alpha, void *x_p
     // runs them on the caller's stream after the interior instead.
     const bool serial = boundary < 0 ? (A->tune & CRSD_TUNE_DIST_BOUNDARY_SERIAL) != 0 : boundary == 1;
     if (c && serial) CU_TRY(cudaStreamWaitEvent(s, c->ev_halo, 0));
+    crsd::HaloSync hs;
+    if (fused) crsd::make_halo_sync(A, c, hs);
     st = crsd::run_lists(A, alpha, xbase, beta, y_local, (const int32_t *)A->d_list_boundary, 0,
-                         (int64_t)A->list_boundary.size(), (c && !serial) ? (void *)c->cs : stream, launches);
+                         (int64_t)A->list_boundary.size(), (c && !serial) ? (void *)c->cs : stream, launches,
+                         fused ? &hs : nullptr);
     if (st) return st;
-    if (c && c->kind == crsd_comm_s::P2P) {
+    if (c && c->kind == crsd_comm_s::P2P && !fused) {
         // the pads are free once the boundary segments are done with them
         if (serial) {
             CU_TRY(cudaEventRecord(c->ev_x, s));

@@ -169,6 +169,27 @@ __device__ __forceinline__ void bar_wait(u64 *b) {
                              : "=r"(done) : "r"(su32(b)) : "memory"); }
 __device__ __forceinline__ u64 pol_first() { u64 p; asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p)); return p; }
 __device__ __forceinline__ u64 pol_normal() { u64 p; asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p)); return p; }
+struct HaloSync { const u64 *ready; u64 *halo_epoch; u32 *counter; u32 *err; u64 *consumed[16]; int peer[16];
+                  int npeer, pad_; u64 timeout_ns; };
+__device__ __forceinline__ u64 ld_acquire_sys(const u64 *p) {
+  u64 v; asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory"); return v; }
+__device__ __forceinline__ void st_release_sys(u64 *p, u64 v) {
+  asm volatile("st.release.sys.global.u64 [%0], %1;" :: "l"(p), "l"(v) : "memory"); }
+// thread 0: every sender has published epoch e (bounded wait; err = 2 on timeout);
+// then order the async-proxy (bulk copy) reads of the pads after the acquire
+__device__ __noinline__ void halo_wait(const HaloSync &h, u64 e) {
+  for (int k = 0; k < h.npeer; ++k) {
+    const u64 *f = h.ready + h.peer[k];
+    if (ld_acquire_sys(f) >= e) continue;
+    u64 t0; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+    while (ld_acquire_sys(f) < e) {
+      __nanosleep(128);
+      u64 t; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      if (t - t0 > h.timeout_ns) { atomicExch(h.err, 2u); break; }
+    }
+  }
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+}
 __device__ __forceinline__ void g2s(void *dst, const void *src, u32 bytes, u64 *b, u64 pol) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
                :: "r"(su32(dst)), "l"(src), "r"(bytes), "r"(su32(b)), "l"(pol) : "memory"); }
@@ -267,8 +288,14 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
         o << "// pattern offsets:";
         for (int d = 0; d < nd; ++d) o << " " << offs[d];
         o << "\n// " << ch.size() << " staging chunk(s)\n";
+        // halo (compile-time after inlining): the crsd_jit_halo kernel, whose
+        // x windows and scatter gathers may reach into pads written by the
+        // neighbours' one-sided puts -- thread 0 issues the value copies,
+        // waits for the senders, then issues the window copies; the scatter
+        // gathers move after the CTA barrier
         o << "__device__ __forceinline__ void codelet_" << key
-          << "(const Args &a, const i64 s, const i64 vb, const i64 row0, const bool edge, T *vs, u64 *bar, const int t) {\n";
+          << "(const Args &a, const i64 s, const i64 vb, const i64 row0, const bool edge, T *vs, u64 *bar, const int t,"
+             " const bool halo, const HaloSync &hs, const u64 he) {\n";
         if (nd) {
             // thread 0: every mbarrier, then every copy, chunk by chunk
             o << "  T *xs = vs + " << (int64_t)nd * m << ";\n";
@@ -286,7 +313,7 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
                 o << "    g2s(vs + " << (int64_t)k.d0 * m << ", a.vals + vb + " << (int64_t)k.d0 * m << ", " << vbytes
                   << "u, bar + " << c << ", pf);\n";
                 if (xbytes) {
-                    o << "    if (!edge) {\n";
+                    o << "    if (!edge && !halo) {\n";
                     for (int w = 0; w < nwin; ++w) {
                         if (!(k.win == -2 || k.win == w)) continue;
                         o << "      g2s(xs + " << wbase[w] << ", a.x + row0 + (" << pl[2 + 2 * w] << "), "
@@ -295,9 +322,22 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
                     o << "    }\n";
                 }
             }
+            // fused halo receive: the windows after the senders' flags
+            o << "    if (halo) {\n      halo_wait(hs, he);\n";
+            for (size_t c = 0; c < ch.size(); ++c) {
+                const Chunk &k = ch[c];
+                if (k.win == -1) continue;
+                for (int w = 0; w < nwin; ++w) {
+                    if (!(k.win == -2 || k.win == w)) continue;
+                    o << "      if (!edge) g2s(xs + " << wbase[w] << ", a.x + row0 + (" << pl[2 + 2 * w] << "), "
+                      << (int64_t)pl[3 + 2 * w] * es << "u, bar + " << c << ", pn);\n";
+                }
+            }
+            o << "    }\n";
             o << "  }\n";
         } else {
             o << "  (void)vs; (void)bar; (void)vb;\n";
+            o << "  if (halo) { if (t == 0) halo_wait(hs, he); __syncthreads(); }\n";
         }
         if (scat) {
             // scatter points are gathered while the bulk copies are in flight:
@@ -306,17 +346,20 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
             // row belongs to this warp, which alone load x[col]
             o << "  const SegDesc *Dp = a.segs + s;\n  const int nscat = __ldg(&Dp->nscat);\n"
                  "  const i64 sbeg = nscat > 0 ? __ldg(&Dp->scat_begin) : 0;\n"
-                 "  int g_own = -1; T g_v = T(0), g_x = T(0); unsigned g_mask = 0u;\n"
-                 "  if (nscat > 0) {\n"
-                 "    const int lane = t & 31;\n"
-                 "    ScatRec R; R.col = 0; R.val = 0; R.row = 0;\n"
-                 "    if (lane < nscat) { R = a.scat_rec[sbeg + lane]; g_own = (R.row % NT) * Q + R.row / NT; }\n"
-                 "    const bool mine = g_own >= 0 && (g_own / Q) / 32 == t / 32;\n"
-                 "    g_mask = __ballot_sync(0xffffffffu, mine);\n"
-                 "    if (mine) { g_v = *reinterpret_cast<const T *>(&R.val); g_x = __ldg(a.x + R.col); }\n"
-                 "  }\n";
+                 "  int g_own = -1; T g_v = T(0), g_x = T(0); unsigned g_mask = 0u;\n";
         }
+        const char *gather =
+            "  if (nscat > 0) {\n"
+            "    const int lane = t & 31;\n"
+            "    ScatRec R; R.col = 0; R.val = 0; R.row = 0;\n"
+            "    if (lane < nscat) { R = a.scat_rec[sbeg + lane]; g_own = (R.row % NT) * Q + R.row / NT; }\n"
+            "    const bool mine = g_own >= 0 && (g_own / Q) / 32 == t / 32;\n"
+            "    g_mask = __ballot_sync(0xffffffffu, mine);\n"
+            "    if (mine) { g_v = *reinterpret_cast<const T *>(&R.val); g_x = __ldg(a.x + R.col); }\n"
+            "  }\n";
+        if (scat) o << "  if (!halo) {\n" << gather << "  }\n";
         if (nd) o << "  __syncthreads();\n";
+        if (scat) o << "  if (halo) {\n" << gather << "  }\n";
         o << "  T acc[Q];\n#pragma unroll\n  for (int q = 0; q < Q; ++q) acc[q] = T(0);\n";
         // FMAs chunk by chunk, each after its own barrier; ascending offset
         // order within and across chunks (the order of the paper's codelet)
@@ -382,7 +425,8 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
         for (const auto &e : edges) o << " || (s >= " << e.first << "LL && s < " << e.second << "LL)";
         o << ";\n}\n";
     }
-    o << "extern \"C\" __global__ void __launch_bounds__(NT) crsd_jit(const Args a) {\n"
+    // the dispatch body shared by crsd_jit and crsd_jit_halo
+    o << "__device__ __forceinline__ void run_segment(const Args &a, const bool halo, const HaloSync &hs, const u64 he) {\n"
          "  extern __shared__ __align__(128) unsigned char smem[];\n  __shared__ u64 bar[NBAR];\n"
          "  T *vs = reinterpret_cast<T *>(smem);\n  i64 s, vb;\n  int key;\n  bool edge;\n";
     if (locate)
@@ -393,8 +437,22 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
     o << "    s = a.seg_list ? (i64)__ldg(a.seg_list + blockIdx.x) : a.seg_begin + blockIdx.x;\n"
          "    const SegDesc D = a.segs[s];\n    key = D.plan_begin;\n    vb = D.val_base;\n    edge = (D.flags & 1) != 0;\n"
          "  }\n  const i64 row0 = s * MROWS;\n  switch (key) {\n";
-    for (int32_t v : seen) o << "  case " << v << ": codelet_" << v << "(a, s, vb, row0, edge, vs, bar, threadIdx.x); break;\n";
+    for (int32_t v : seen)
+        o << "  case " << v << ": codelet_" << v << "(a, s, vb, row0, edge, vs, bar, threadIdx.x, halo, hs, he); break;\n";
     o << "  }\n}\n";
+    o << "extern \"C\" __global__ void __launch_bounds__(NT) crsd_jit(const Args a) {\n"
+         "  const HaloSync hs{};\n  run_segment(a, false, hs, 0ull);\n}\n";
+    // boundary segments of a direct-mode exchange: the receive side fused in
+    // (wait per CTA before the window copies; the last CTA to finish releases
+    // the pads to the senders and advances the epoch)
+    o << "extern \"C\" __global__ void __launch_bounds__(NT) crsd_jit_halo(const Args a, const HaloSync hs) {\n"
+         "  const u64 he = *(volatile u64 *)hs.halo_epoch + 1;\n"
+         "  run_segment(a, true, hs, he);\n"
+         "  __shared__ bool last;\n  __threadfence();\n  __syncthreads();\n"
+         "  if (threadIdx.x == 0) {\n    last = atomicAdd(hs.counter, 1u) == gridDim.x - 1;\n"
+         "    if (last) {\n      *hs.counter = 0u;\n      __threadfence_system();\n"
+         "      if (*(volatile u32 *)hs.err == 0u)\n        for (int k = 0; k < hs.npeer; ++k) st_release_sys(hs.consumed[k], he);\n"
+         "      *(volatile u64 *)hs.halo_epoch = he;\n    }\n  }\n}\n";
     return o.str();
 }
 
@@ -563,8 +621,16 @@ crsd_status_t jit_build(crsd_matrix_s *A) {
         dr.unload(mod);
         return fail(CRSD_ERR_CUDA, "cuFuncSetAttribute failed");
     }
+    CUfunction fh = nullptr;
+    if (dr.get_function(&fh, mod, "crsd_jit_halo") != CUDA_SUCCESS ||
+        (A->smem_bytes > 48 * 1024 &&
+         dr.set_attr(fh, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)A->smem_bytes) != CUDA_SUCCESS)) {
+        dr.unload(mod);
+        return fail(CRSD_ERR_CUDA, "crsd_jit_halo: cuModuleGetFunction / cuFuncSetAttribute failed");
+    }
     A->jit_module = mod;
     A->jit_function = fn;
+    A->jit_halo_function = fh;
     jit_plan_ranges(A);
     return CRSD_OK;
 }
@@ -582,6 +648,7 @@ void jit_free(crsd_matrix_s *A) {
     if (A->jit_module && driver().ok) driver().unload((CUmodule)A->jit_module);
     A->jit_module = nullptr;
     A->jit_function = nullptr;
+    A->jit_halo_function = nullptr;
 }
 
 template <typename T>
@@ -605,6 +672,14 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
     j.alpha = s.alpha;
     j.beta = s.beta;
     const unsigned nt = (unsigned)(A->H.mrows / jit_q(A));
+    if (s.halo) {
+        // boundary segments with the fused halo receive: one launch
+        static_assert(sizeof(HaloSync) == 8 * 4 + 8 * HALO_MAX_PEERS + 4 * HALO_MAX_PEERS + 8 + 8, "HaloSync layout");
+        void *params[] = {&j, const_cast<HaloSync *>(s.halo)};
+        const CUresult r = driver().launch((CUfunction)A->jit_halo_function, (unsigned)s.seg_count, 1, 1, nt, 1, 1,
+                                           (unsigned)A->smem_bytes, (CUstream)stream, params, nullptr);
+        return r == CUDA_SUCCESS ? 1 : -(int)cudaErrorLaunchFailure;
+    }
     if (!s.seg_list && A->jit_ranges.size() > 1) {
         // a segment range (the whole matrix, or a contiguous interior):
         // one launch per occupancy class it meets (jit_plan_ranges).

@@ -73,7 +73,11 @@ def _worker(rank, world, port, case, variant, q, mode="mailbox", distinct=False,
         bounds = partition_rows(n, mrows, world, np.bincount(a.row, minlength=n).astype(np.float64))
         rb, re = int(bounds[rank]), int(bounds[rank + 1])
         m = (a.row >= rb) & (a.row < re)
-        A = CRSDMatrix.from_coo(n, n, a.row[m], a.col[m], a.val[m], mrows=mrows, row_range=(rb, re), variant=0 if variant == "timeout" else variant, device=dev)
+        from paper_conf_icpp_sunzwzyr11_b200 import TUNE_HALO_UNFUSED
+
+        tune = TUNE_HALO_UNFUSED if mode == "direct-unfused" else 0
+        A = CRSDMatrix.from_coo(n, n, a.row[m], a.col[m], a.val[m], mrows=mrows, row_range=(rb, re),
+                                variant=0 if variant == "timeout" else variant, device=dev, tune=tune)
         if variant == "timeout":
             os.environ["CRSD_P2P_TIMEOUT_S"] = "2"
         # capacities differ per rank on purpose: a receiver must address the
@@ -116,7 +120,7 @@ def _worker(rank, world, port, case, variant, q, mode="mailbox", distinct=False,
         else:
             errs = []
             stream = torch.cuda.Stream()
-            if mode == "direct":
+            if mode.startswith("direct"):
                 # the library-owned padded x, mapped by every peer: the halo
                 # arrives as one-sided puts. NaN pads once, before any rank
                 # can put (barrier): every call must overwrite them.
@@ -127,7 +131,7 @@ def _worker(rank, world, port, case, variant, q, mode="mailbox", distinct=False,
             for call in range(5):  # epochs 1..5: both mailbox parities, reuse after consumed
                 x = np.random.default_rng(100 + call).uniform(-1, 1, n).astype(dt)
                 yref, scale = coo.coo_spmv(n, n, a.row, a.col, a.val, x)
-                if mode == "direct":
+                if mode.startswith("direct"):
                     # only the owned part is ours to write; peers write the pads
                     xdir[lo : lo + nloc].copy_(torch.from_numpy(x[rb:re]).to(f"cuda:{dev}", tdt))
                     xd = xdir
@@ -195,11 +199,14 @@ def torch_cuda():
     "case,world,variant,mode",
     [("c2", 2, 0, "mailbox"), ("c3", 2, 0, "mailbox"), ("c4", 2, 0, "mailbox"), ("c2", 3, 4, "mailbox"),
      ("c3", 3, 3, "mailbox"), ("multihop", 4, 0, "mailbox"), ("c4", 4, 1, "mailbox"),
-     ("c2", 2, 0, "direct"), ("c3", 3, 0, "direct"), ("c4", 2, 0, "direct"), ("multihop", 4, 0, "direct")],
+     ("c2", 2, 0, "direct"), ("c3", 3, 0, "direct"), ("c4", 2, 0, "direct"), ("multihop", 4, 0, "direct"),
+     ("c3", 2, 0, "direct-unfused"), ("multihop", 4, 0, "direct-unfused"), ("c3", 2, 3, "direct")],
 )
 def test_p2p_spmv_dist(torch_cuda, case, world, variant, mode):
     """mailbox: caller-owned x_padded, two-stage exchange; direct: the
-    crsd_dist_x_alloc buffer, one-sided puts into the neighbours' pads."""
+    crsd_dist_x_alloc buffer, one-sided puts into the neighbours' pads, the
+    receive fused into the boundary kernel (JIT variant; separate wait /
+    release kernels with CRSD_TUNE_HALO_UNFUSED or a table-driven variant)."""
     _, dt, _ = _matrix(case)
     res = _run(case, world, variant, mode=mode)
     for r in res:
