@@ -267,26 +267,6 @@ def copy_bandwidth(dev, reps=5):
     return round(best, 1)
 
 
-def read_bandwidth(dev, reps=5):
-    """Read-only HBM bandwidth on this box (torch sum over 4 GiB of fp32, best
-    of `reps`): context for a read-dominated stream such as SpMV, whose
-    fraction of the copy peak (read + write) can exceed 1."""
-    import torch
-
-    a = torch.ones(1 << 30, dtype=torch.float32, device=f"cuda:{dev}")
-    best = 0.0
-    for _ in range(reps + 1):
-        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        s.record()
-        a.sum()
-        e.record()
-        e.synchronize()
-        best = max(best, a.numel() * 4 / (s.elapsed_time(e) * 1e-3) / 1e9)
-    del a
-    torch.cuda.empty_cache()
-    return round(best, 1)
-
-
 def load_traffic(key):
     """ncu dram bytes (read + write) per launch of the dominant kernel on this
     workload, from one `ncu --set full` capture (profiles/traffic.json, keyed
@@ -552,7 +532,13 @@ def run_spmv(args):
     if world > 1:
         comm, transport = make_comm(args, A, rank, world, dev, es)
         lo, _, hi = A.x_layout()
-        xp = torch.zeros(lo + nloc + hi, dtype=tdt, device=f"cuda:{dev}")
+        if transport == "p2p":
+            # the library-owned padded x, mapped by the neighbours: halos
+            # arrive as one-sided puts, received inside the boundary kernel
+            xp = A.dist_x_alloc(comm)
+            transport = "p2p one-sided puts"
+        else:
+            xp = torch.zeros(lo + nloc + hi, dtype=tdt, device=f"cuda:{dev}")
         xp[lo : lo + nloc] = x_own
         y = torch.empty(nloc, dtype=tdt, device=f"cuda:{dev}")
 
@@ -616,7 +602,8 @@ def run_spmv(args):
     achieved = ub_all / world / (kern_ms * 1e-3) / 1e9  # per GPU: whole-job bytes / N / max-over-ranks step time
 
     # e2e through the public C-ABI with host buffers (pinned)
-    e2e = run_e2e(args, A, world, rank, dev, dt, tdt, N, rb, re, nnz_all, red_dev, comm, transport)
+    e2e = run_e2e(args, A, world, rank, dev, dt, tdt, N, rb, re, nnz_all, red_dev, comm, transport,
+                  xp if world > 1 else None)
     if rank != 0:
         if comm is not None:
             comm.close()
@@ -634,7 +621,6 @@ def run_spmv(args):
     if world == 1 and not args.no_cpu:
         cpu = cpu_baseline(args.config, args.dtype)
     box_copy = copy_bandwidth(dev)
-    box_read = read_bandwidth(dev)
     kname = KNAME[info["variant"]]
     line = {
         "metric": METRIC,
@@ -682,8 +668,6 @@ def run_spmv(args):
             "launches_per_step": round(launches_all / world / max(1, args.steps), 2),
             "scope": "per GPU: whole-job algorithmic bytes / N / the max-over-ranks CUDA-event step time; with several launches per step (occupancy-class ranges, interior/boundary) the step's bytes / the step's time",
             "copy_gbs_this_box": box_copy,
-            "read_gbs_this_box": box_read,
-            "frac_of_this_box_read": round(achieved / box_read, 4) if box_read else None,
         },
         "north_star_c3": subs,
         "cpu_baseline": cpu,
@@ -698,7 +682,7 @@ def run_spmv(args):
         dist.destroy_process_group()
 
 
-def run_e2e(args, A, world, rank, dev, dt, tdt, N, rb, re, nnz_all, red_dev, comm, transport):
+def run_e2e(args, A, world, rank, dev, dt, tdt, N, rb, re, nnz_all, red_dev, comm, transport, xp=None):
     """The metric end to end through the public C-ABI: every step copies the
     step's x from pinned host memory and its y back (N = 1: crsd_spmv_host,
     the library's chunked H2D / SpMV / D2H pipeline; N > 1: per rank the
@@ -744,7 +728,6 @@ def run_e2e(args, A, world, rank, dev, dt, tdt, N, rb, re, nnz_all, red_dev, com
         }
     nloc = re - rb
     lo, _, hi = A.x_layout()
-    xp = torch.zeros(lo + nloc + hi, dtype=tdt, device=f"cuda:{dev}")
     y = torch.empty(nloc, dtype=tdt, device=f"cuda:{dev}")
     xh = torch.from_numpy(np.random.default_rng(7 + rank).uniform(-1, 1, nloc).astype(dt)).pin_memory()
     yh = torch.empty(nloc, dtype=tdt).pin_memory()

@@ -355,6 +355,11 @@ crsd_status_t crsd_dist_bind(crsd_matrix_t A_local, crsd_comm_t comm, void *stre
  * comm stream (concurrently with the interior; CRSD_TUNE_DIST_BOUNDARY_SERIAL
  * runs them on `stream` after it) and `stream` joins the comm stream before
  * the call returns, so y_local is complete in `stream` order. Asynchronous.
+ * With a peer-memory communicator and x_padded from crsd_dist_x_alloc the
+ * halo moves as one-sided puts, and (JIT variant) the receive is fused into
+ * the boundary kernel: each boundary CTA waits for the senders' flags before
+ * copying its x windows and the last one releases the pads
+ * (CRSD_TUNE_HALO_UNFUSED: separate wait / release kernels).
  *   x_padded  DEVICE dtype[halo_lo+n_local+halo_hi], 16-byte aligned; the
  *             owned part must be written before the call (stream-ordered);
  *             the halo parts are overwritten.

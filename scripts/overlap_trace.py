@@ -34,7 +34,7 @@ def main():
     torch.cuda.set_device(0)
     from paper_conf_icpp_sunzwzyr11_b200 import P2PComm
 
-    A, desc, (rb, re), N, _ = bench.build(cfg, "f64", world, rank, 0, nthreads=max(1, bench.host_cores() // world))
+    A, desc, (rb, rend), N, _ = bench.build(cfg, "f64", world, rank, 0, nthreads=max(1, bench.host_cores() // world))
     lo, nloc, hi = A.x_layout()
     comm = P2PComm(rank, world, 0, mailbox_bytes=max(1 << 20, 4 * (lo + hi) * 8))
     A.dist_bind(comm)

@@ -252,6 +252,11 @@ def test_jit_codelets_compile_for_sm100a(case, dt, tmp_path):
     assert src.count("__device__ __forceinline__ void codelet_") == npat
     assert src.count("case ") == npat
     assert src.count("{ key = ") == A.info()["ninst"]
+    # two entry points: the plain kernel and the boundary kernel with the
+    # fused halo receive (wait on the senders' flags, proxy fence, release)
+    assert 'extern "C" __global__ void __launch_bounds__(NT) crsd_jit(' in src
+    assert 'extern "C" __global__ void __launch_bounds__(NT) crsd_jit_halo(' in src
+    assert "fence.proxy.async.global" in src and "st.release.sys" in src
     for offs in P["inst_offsets"]:
         assert "// pattern offsets: " + " ".join(str(o) for o in offs) in src
     f = tmp_path / "k.cu"
