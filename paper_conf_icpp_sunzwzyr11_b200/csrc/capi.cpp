@@ -376,6 +376,7 @@ crsd_status_t crsd_opts_init(crsd_opts_t *o) {
 static crsd_status_t create_common(int64_t nrows, int64_t ncols, crsd_dtype_t dtype, const crsd_opts_t *opts,
                                    crsd_matrix_t *out, bool csr, int64_t nnz, const int64_t *row_or_ptr,
                                    const int64_t *col, const void *val) {
+    NvtxRange nv("crsd_create");
     if (!out) return fail(CRSD_ERR_INVALID_ARG, "out is NULL");
     *out = nullptr;
     if (dtype != CRSD_R32F && dtype != CRSD_R64F) return fail(CRSD_ERR_INVALID_ARG, "bad dtype");
@@ -449,6 +450,7 @@ static crsd_status_t check_vec(const void *p, const char *name) {
 }
 
 crsd_status_t crsd_spmv(crsd_matrix_t A, const void *alpha, const void *x, const void *beta, void *y, void *stream) {
+    NvtxRange nv("crsd_spmv");
     if (!A) return fail(CRSD_ERR_INVALID_ARG, "A is NULL");
     if (A->host_only) return fail(CRSD_ERR_UNSUPPORTED, "host-only handle");
     if (A->H.partitioned) return fail(CRSD_ERR_UNSUPPORTED, "row-partitioned handle: use crsd_spmv_dist");
@@ -554,6 +556,7 @@ static crsd_status_t e2e_setup(crsd_matrix_s *A) {
 
 crsd_status_t crsd_spmv_host(crsd_matrix_t A, const void *alpha, const void *x_host, const void *beta, void *y_host,
                              void *stream) {
+    NvtxRange nv("crsd_spmv_host");
     if (!A) return fail(CRSD_ERR_INVALID_ARG, "A is NULL");
     if (A->host_only) return fail(CRSD_ERR_UNSUPPORTED, "host-only handle");
     if (A->H.partitioned) return fail(CRSD_ERR_UNSUPPORTED, "row-partitioned handle");

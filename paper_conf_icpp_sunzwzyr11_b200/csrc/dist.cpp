@@ -560,6 +560,7 @@ crsd_status_t crsd_spmv_dist(crsd_matrix_t A, const void *alpha, void *x_padded,
 // CRSD_TUNE_DIST_BOUNDARY_SERIAL), 0 = concurrent, 1 = serial after the interior
 crsd_status_t crsd::spmv_dist_impl(crsd_matrix_t A, const void *alpha, void *x_padded, const void *beta,
                                    void *y_local, crsd_comm_t c, void *stream, int boundary) {
+    crsd::NvtxRange nv("crsd_spmv_dist");
     if (!A) return crsd::fail(CRSD_ERR_INVALID_ARG, "A is NULL");
     if (A->host_only) return crsd::fail(CRSD_ERR_UNSUPPORTED, "host-only handle");
     if (A->H.paper_ell) return crsd::fail(CRSD_ERR_UNSUPPORTED, "CRSD_PAPER_ELL handle: use crsd_spmv");
@@ -592,6 +593,7 @@ crsd_status_t crsd::spmv_dist_impl(crsd_matrix_t A, const void *alpha, void *x_p
                        A->variant == VARIANT_JIT && A->jit_halo_function && !A->list_boundary.empty() &&
                        !(A->tune & CRSD_TUNE_HALO_UNFUSED);
     auto exchange = [&]() -> crsd_status_t {
+        crsd::NvtxRange nvx("halo exchange");
         CU_TRY(cudaStreamWaitEvent(c->cs, c->ev_x, 0));
         if (c->kind == crsd_comm_s::P2P) {
             ST_TRY(crsd::p2p_exchange(A, c, xp, fused, launches));

@@ -243,6 +243,7 @@ crsd_status_t cg_impl(crsd_matrix_s *A, const T *b, T *x, int32_t max_iter, doub
 extern "C" crsd_status_t crsd_cg(crsd_matrix_t A, const void *b, void *x, int32_t max_iter, double rtol,
                                  int32_t check_every, crsd_comm_t comm, double *rr_history, crsd_cg_result_t *res,
                                  void *stream) {
+    NvtxRange nv("crsd_cg");
     if (!A) return fail(CRSD_ERR_INVALID_ARG, "A is NULL");
     if (A->host_only) return fail(CRSD_ERR_UNSUPPORTED, "host-only handle");
     if (!b || !x) return fail(CRSD_ERR_INVALID_ARG, "b and x must not be NULL");
