@@ -311,11 +311,14 @@ def sub_record(cfg, dtype, args, dev):
     def step():
         A.spmv(x, y, 1.0, 0.0)
 
-    for _ in range(args.warmup):
+    # a sub-record's steps are short (0.1-0.8 ms): at least 200 of them, so
+    # the timed region is not dominated by its ramp-up
+    steps = max(args.steps, 200)
+    for _ in range(max(args.warmup, 10)):
         step()
     torch.cuda.synchronize()
     clk = ClockSampler(dev).start()
-    ms, total_ms, launches = timed_steps(step, args.steps, stream, A.last_launch_count)
+    ms, total_ms, launches = timed_steps(step, steps, stream, A.last_launch_count)
     clocks = clk.stop()
     ub = info["unique_bytes_beta0"]
     peak, _ = measured_peaks()
@@ -332,7 +335,8 @@ def sub_record(cfg, dtype, args, dev):
         "kernel_variant": VNAME[info["variant"]],
         "scatter": info["nscatter"],
         "fills": info["nfills"],
-        "launches_per_step": round(launches / args.steps, 2),
+        "steps": steps,
+        "launches_per_step": round(launches / steps, 2),
         "roofline": {
             "bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
             "frac": round(achieved / peak, 4), "traffic": load_traffic(f"{cfg}_{dtype}_{kname}"),
