@@ -331,6 +331,10 @@ crsd_status_t crsd_comm_destroy(crsd_comm_t comm);
  *       mailbox path. crsd_cg over a peer-memory communicator uses this
  *       buffer for p. Every rank must stop using it (crsd_comm_destroy, or a
  *       barrier after its last crsd_spmv_dist) before any rank destroys A.
+ *       Ranks must allocate for their handles in the same order (one handle
+ *       at a time); a peer that allocated for a different row block is
+ *       detected and refused (INVALID_ARG). Bounded by the communicator's
+ *       wait limit (CUDA error if a peer never arrives).
  */
 crsd_status_t crsd_comm_init_p2p(int rank, int world, int device, int64_t mailbox_bytes, void *ipc_handle64,
                                  crsd_comm_t *out);

@@ -471,6 +471,9 @@ crsd_status_t dist_x_alloc(crsd_matrix_t A, crsd_comm_t c) {
         if (q == c->rank) continue;
         char *pf = (char *)c->peer_sym[q];
         e = cudaMemcpy(pf + offsetof(P2PFlags, xh) + 64 * c->rank, &h, 64, cudaMemcpyHostToDevice);
+        const int64_t rng[2] = {A->H.row_begin, A->H.row_end};
+        if (e == cudaSuccess)
+            e = cudaMemcpy(pf + offsetof(P2PFlags, xrange) + 16 * c->rank, rng, 16, cudaMemcpyHostToDevice);
         if (e == cudaSuccess)
             e = cudaMemcpy(pf + offsetof(P2PFlags, xseq) + 8 * c->rank, &seq, 8, cudaMemcpyHostToDevice);
     }
@@ -492,7 +495,19 @@ crsd_status_t dist_x_alloc(crsd_matrix_t A, crsd_comm_t c) {
             std::this_thread::sleep_for(std::chrono::microseconds(200));
         }
         cudaIpcMemHandle_t hq;
+        int64_t rq[2] = {-1, -1};
         if (e == cudaSuccess) e = cudaMemcpy(&hq, mine + offsetof(P2PFlags, xh) + 64 * q, 64, cudaMemcpyDeviceToHost);
+        if (e == cudaSuccess) e = cudaMemcpy(rq, mine + offsetof(P2PFlags, xrange) + 16 * q, 16, cudaMemcpyDeviceToHost);
+        // the peer must have allocated for the handle this one is bound to
+        // (same row block as in the range table): a collective mismatch
+        // (ranks allocating for different matrices) is refused, not mapped
+        if (e == cudaSuccess && (rq[0] != A->range_table[4 * q] || rq[1] != A->range_table[4 * q + 1])) {
+            for (void *m : peer)
+                if (m) cudaIpcCloseMemHandle(m);
+            cudaFree(p);
+            return fail(CRSD_ERR_INVALID_ARG, "crsd_dist_x_alloc: rank " + std::to_string(q) +
+                                                  " allocated for a different row block (collective mismatch)");
+        }
         if (e == cudaSuccess) e = cudaIpcOpenMemHandle(&peer[q], hq, cudaIpcMemLazyEnablePeerAccess);
     }
     if (e != cudaSuccess) {
