@@ -69,11 +69,12 @@ void free_device(crsd_matrix_s *A) {
         A->cg_stream = A->cg_ev_in = A->cg_ev_out = nullptr;
     }
     // direct-mode padded x (crsd_dist_x_alloc): unmap the peers', free mine
-    for (void *p : A->dx_peer)
-        if (p) cudaIpcCloseMemHandle(p);
-    A->dx_peer.clear();
-    if (A->dx_own) cudaFree(A->dx_own);
-    A->dx_own = nullptr;
+    for (crsd_matrix_s::DirectX &d : A->dx) {
+        for (void *p : d.peer)
+            if (p) cudaIpcCloseMemHandle(p);
+        if (d.own) cudaFree(d.own);
+    }
+    A->dx.clear();
     void *ptrs[] = {A->d_vals, A->d_segs, A->d_offs, A->d_plan, A->d_scat_row, A->d_scat_col, A->d_scat_val, A->d_scat_rec,
                     A->d_list_interior, A->d_list_boundary, A->d_list_all_edge, A->d_x_scratch, A->d_y_scratch, A->d_cg,
                     A->d_ell_rowno, A->d_ell_col, A->d_ell_val};

@@ -36,7 +36,7 @@ crsd_status_t comm_allreduce_f64(crsd_comm_s *c, double *dev, int n, cudaStream_
 // crsd_spmv_dist with the boundary placement chosen by the caller: -1 default,
 // 0 concurrent with the interior (comm stream), 1 serial after the interior
 // the handle's crsd_dist_x_alloc buffer (direct one-sided puts), collective
-crsd_status_t dist_x_alloc(crsd_matrix_s *A, crsd_comm_s *c);
+crsd_status_t dist_x_alloc(crsd_matrix_s *A, crsd_comm_s *c, int purpose, void **out);
 crsd_status_t release_halo(crsd_matrix_s *A, crsd_comm_s *c);
 crsd_status_t spmv_dist_impl(crsd_matrix_s *A, const void *alpha, void *x_padded, const void *beta, void *y_local,
                              crsd_comm_s *c, void *stream, int boundary);

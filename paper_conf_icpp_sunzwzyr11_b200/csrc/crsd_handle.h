@@ -91,11 +91,22 @@ struct crsd_matrix_s {
     std::vector<int64_t> send_mb_off, recv_mb_off;
     const void *bound_comm = nullptr;
     std::vector<int64_t> range_table;  // every rank's {row_begin, row_end, halo_lo_valid, halo_hi_valid}
-    // direct (one-sided put) mode: this rank's padded x from crsd_dist_x_alloc
-    // (IPC-exported) and every peer's, mapped; the sends land in the peers' pads
-    void *dx_own = nullptr;
-    std::vector<void *> dx_peer;
-    const void *dx_comm = nullptr;
+    // direct (one-sided put) mode: padded x buffers allocated by the library
+    // (IPC-exported) with every peer's counterpart mapped; the sends land in
+    // the peers' pads. purpose 0: crsd_dist_x_alloc (the caller's x), 1: the
+    // CG's p (so a CG never writes into the caller's x)
+    struct DirectX {
+        void *own = nullptr;
+        std::vector<void *> peer;
+        const void *comm = nullptr;
+        int purpose = 0;
+    };
+    std::vector<DirectX> dx;
+    const DirectX *find_dx(const void *xp, const void *comm) const {
+        for (const DirectX &d : dx)
+            if (d.own == xp && d.comm == comm) return &d;
+        return nullptr;
+    }
 };
 
 namespace crsd {

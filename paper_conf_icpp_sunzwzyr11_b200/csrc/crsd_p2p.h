@@ -25,7 +25,7 @@ struct P2PFlags {
     // crsd_dist_x_alloc handshake, written by q (host copies into peer memory):
     // q's padded-x IPC handle, then xseq[q] = the allocation's sequence number
     uint8_t xh[P2P_MAX_WORLD][64];
-    int64_t xrange[P2P_MAX_WORLD][2];  // the row range of the handle q allocated it for
+    int64_t xrange[P2P_MAX_WORLD][4];  // {row_begin, row_end, purpose, 0} of the handle q allocated it for
     uint64_t xseq[P2P_MAX_WORLD];
 };
 static_assert(sizeof(P2PFlags) <= P2P_FLAGS_BYTES, "P2PFlags too large");

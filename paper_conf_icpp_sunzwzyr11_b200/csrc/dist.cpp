@@ -384,7 +384,7 @@ crsd_status_t p2p_exchange(crsd_matrix_t A, crsd_comm_t c, char *xp, bool fused_
     fill_launch(R, c, A->recv_peer);
     S.nitems = (int32_t)A->send_peer.size();
     R.nitems = (int32_t)A->recv_peer.size();
-    if (xp == (char *)A->dx_own && A->dx_comm == c) {
+    if (const crsd_matrix_s::DirectX *dx = A->find_dx(xp, c)) {
         const int W = c->world;
         for (int k = 0; k < S.nitems; ++k) {
             const int64_t q = A->send_peer[k];
@@ -392,7 +392,7 @@ crsd_status_t p2p_exchange(crsd_matrix_t A, crsd_comm_t c, char *xp, bool fused_
             const int64_t q_halo_lo = (A->range_table[4 * q + 2] + 3) / 4 * 4;
             const int64_t q_origin = A->range_table[4 * q] - q_halo_lo;
             (void)W;
-            S.items[k] = P2PItem{xp + es * A->send_off[k], (char *)A->dx_peer[q] + es * (gcol - q_origin),
+            S.items[k] = P2PItem{xp + es * A->send_off[k], (char *)dx->peer[q] + es * (gcol - q_origin),
                                  es * A->send_count[k], 0};
         }
         CU_TRY((cudaError_t)p2p_launch_put(S, grid, c->cs));
@@ -450,11 +450,14 @@ crsd_status_t release_halo(crsd_matrix_t A, crsd_comm_t c) {
 // its IPC handle to every peer through the peers' flag regions (host copies
 // into peer memory), wait until every peer's handle has arrived in mine
 // (bounded), and map them.
-crsd_status_t dist_x_alloc(crsd_matrix_t A, crsd_comm_t c) {
+crsd_status_t dist_x_alloc(crsd_matrix_t A, crsd_comm_t c, int purpose, void **out) {
     if (c->kind != crsd_comm_s::P2P || !c->opened)
         return fail(CRSD_ERR_INVALID_ARG, "crsd_dist_x_alloc needs an opened peer-memory communicator");
     if (!A->bound || A->bound_comm != c) return fail(CRSD_ERR_INVALID_ARG, "bind the handle to this communicator first");
-    if (A->dx_own) return fail(CRSD_ERR_INVALID_ARG, "the handle already has a crsd_dist_x_alloc buffer");
+    for (const crsd_matrix_s::DirectX &d : A->dx)
+        if (d.purpose == purpose)
+            return fail(CRSD_ERR_INVALID_ARG, purpose == 0 ? "the handle already has a crsd_dist_x_alloc buffer"
+                                                           : "the handle already has a CG direct buffer");
     const int64_t bytes = A->H.elem * (A->halo_lo + A->H.n_local + A->halo_hi);
     void *p = nullptr;
     CU_TRY(cudaMalloc(&p, std::max<int64_t>(bytes, 256)));
@@ -471,9 +474,9 @@ crsd_status_t dist_x_alloc(crsd_matrix_t A, crsd_comm_t c) {
         if (q == c->rank) continue;
         char *pf = (char *)c->peer_sym[q];
         e = cudaMemcpy(pf + offsetof(P2PFlags, xh) + 64 * c->rank, &h, 64, cudaMemcpyHostToDevice);
-        const int64_t rng[2] = {A->H.row_begin, A->H.row_end};
+        const int64_t rng[4] = {A->H.row_begin, A->H.row_end, purpose, 0};
         if (e == cudaSuccess)
-            e = cudaMemcpy(pf + offsetof(P2PFlags, xrange) + 16 * c->rank, rng, 16, cudaMemcpyHostToDevice);
+            e = cudaMemcpy(pf + offsetof(P2PFlags, xrange) + 32 * c->rank, rng, 32, cudaMemcpyHostToDevice);
         if (e == cudaSuccess)
             e = cudaMemcpy(pf + offsetof(P2PFlags, xseq) + 8 * c->rank, &seq, 8, cudaMemcpyHostToDevice);
     }
@@ -495,13 +498,15 @@ crsd_status_t dist_x_alloc(crsd_matrix_t A, crsd_comm_t c) {
             std::this_thread::sleep_for(std::chrono::microseconds(200));
         }
         cudaIpcMemHandle_t hq;
-        int64_t rq[2] = {-1, -1};
+        int64_t rq[4] = {-1, -1, -1, 0};
         if (e == cudaSuccess) e = cudaMemcpy(&hq, mine + offsetof(P2PFlags, xh) + 64 * q, 64, cudaMemcpyDeviceToHost);
-        if (e == cudaSuccess) e = cudaMemcpy(rq, mine + offsetof(P2PFlags, xrange) + 16 * q, 16, cudaMemcpyDeviceToHost);
+        if (e == cudaSuccess) e = cudaMemcpy(rq, mine + offsetof(P2PFlags, xrange) + 32 * q, 32, cudaMemcpyDeviceToHost);
         // the peer must have allocated for the handle this one is bound to
-        // (same row block as in the range table): a collective mismatch
-        // (ranks allocating for different matrices) is refused, not mapped
-        if (e == cudaSuccess && (rq[0] != A->range_table[4 * q] || rq[1] != A->range_table[4 * q + 1])) {
+        // (same row block as in the range table) and for the same purpose: a
+        // collective mismatch (ranks allocating for different matrices or in
+        // a different order) is refused, not mapped
+        if (e == cudaSuccess &&
+            (rq[0] != A->range_table[4 * q] || rq[1] != A->range_table[4 * q + 1] || rq[2] != purpose)) {
             for (void *m : peer)
                 if (m) cudaIpcCloseMemHandle(m);
             cudaFree(p);
@@ -516,10 +521,14 @@ crsd_status_t dist_x_alloc(crsd_matrix_t A, crsd_comm_t c) {
         cudaFree(p);
         return cu_fail(e, "crsd_dist_x_alloc handshake");
     }
-    A->dx_own = p;
-    A->dx_peer = peer;
-    A->dx_comm = c;
+    crsd_matrix_s::DirectX d;
+    d.own = p;
+    d.peer = peer;
+    d.comm = c;
+    d.purpose = purpose;
+    A->dx.push_back(d);
     A->device_bytes += bytes;
+    if (out) *out = p;
     return CRSD_OK;
 }
 }  // namespace crsd
@@ -559,9 +568,7 @@ crsd_status_t crsd_dist_x_alloc(crsd_matrix_t A, crsd_comm_t c, void **x_padded)
     if (!A || !c || !x_padded) return crsd::fail(CRSD_ERR_INVALID_ARG, "NULL argument");
     *x_padded = nullptr;
     CU_TRY(cudaSetDevice(A->device));
-    ST_TRY(crsd::dist_x_alloc(A, c));
-    *x_padded = A->dx_own;
-    return CRSD_OK;
+    return crsd::dist_x_alloc(A, c, 0, x_padded);
 }
 
 crsd_status_t crsd_spmv_dist(crsd_matrix_t A, const void *alpha, void *x_padded, const void *beta, void *y_local,
@@ -604,7 +611,7 @@ crsd_status_t crsd::spmv_dist_impl(crsd_matrix_t A, const void *alpha, void *x_p
     // before copying its x windows, the last CTA releases the pads -- so a
     // call is put + interior + boundary, no separate wait / release kernels
     // (CRSD_TUNE_HALO_UNFUSED restores them).
-    const bool fused = c && c->kind == crsd_comm_s::P2P && xp == (char *)A->dx_own && A->dx_comm == c &&
+    const bool fused = c && c->kind == crsd_comm_s::P2P && A->find_dx(xp, c) &&
                        A->variant == VARIANT_JIT && A->jit_halo_function && !A->list_boundary.empty() &&
                        !(A->tune & CRSD_TUNE_HALO_UNFUSED);
     auto exchange = [&]() -> crsd_status_t {

@@ -117,9 +117,14 @@ crsd_status_t cg_impl(crsd_matrix_s *A, const T *b, T *x, int32_t max_iter, doub
     // buffer, so every halo moves as one-sided puts into the neighbours'
     // pads (collective: every rank runs crsd_cg)
     if (comm && comm->kind == crsd_comm_s::P2P && comm->world > 1) {
-        if (!A->dx_own) ST_TRY(dist_x_alloc(A, comm));
-        if (A->dx_comm != comm) return fail(CRSD_ERR_INVALID_ARG, "the handle's direct x buffer belongs to another communicator");
-        w.p_pad = (char *)A->dx_own;
+        const crsd_matrix_s::DirectX *d = nullptr;
+        for (const crsd_matrix_s::DirectX &e : A->dx)
+            if (e.purpose == 1) d = &e;
+        if (d && d->comm != comm)
+            return fail(CRSD_ERR_INVALID_ARG, "the handle's CG direct buffer belongs to another communicator");
+        void *pp = d ? d->own : nullptr;
+        if (!d) ST_TRY(dist_x_alloc(A, comm, 1, &pp));
+        w.p_pad = (char *)pp;
     }
     T *p_own = (T *)w.p_pad + A->halo_lo;
     int launches = 0;

@@ -150,6 +150,22 @@ def _worker(rank, world, port, case, variant, q, mode="mailbox", distinct=False,
                 errs.append(coo.parity_error(yd.cpu().numpy(), yref[rb:re], scale[rb:re]))
             out["errs"] = errs
             out["launches"] = A.last_launch_count()
+            if mode.startswith("direct") and case == "c2":
+                # a CG on the same handle uses a direct buffer of its own for
+                # p: the caller's x_padded (owned part and halo) must survive
+                keep = xdir.clone()
+                y_before = yd.clone()
+                bd = torch.ones(nloc, dtype=tdt, device=f"cuda:{dev}")
+                xc = torch.zeros(nloc, dtype=tdt, device=f"cuda:{dev}")
+                A.cg(bd, xc, 3, 0.0, check_every=3, comm=comm)
+                torch.cuda.synchronize()
+                out["x_kept"] = bool(torch.equal(xdir[lo : lo + nloc], keep[lo : lo + nloc]))
+                y2 = torch.full((nloc,), float("nan"), device=f"cuda:{dev}", dtype=tdt)
+                stream.wait_stream(torch.cuda.current_stream())
+                with torch.cuda.stream(stream):
+                    A.spmv_dist(xdir, y2, 1.0, 0.0, comm, stream=stream)
+                stream.synchronize()
+                out["y_same_after_cg"] = bool(torch.equal(y2, y_before))
             # scalar allreduce: every rank contributes distinct values; results bit-identical
             v = torch.tensor([0.1 * (rank + 1), 1e16 * (-1) ** rank, 3.0 + rank / 7.0], dtype=torch.float64, device=f"cuda:{dev}")
             comm.allreduce_f64(v)
@@ -211,6 +227,8 @@ def test_p2p_spmv_dist(torch_cuda, case, world, variant, mode):
     res = _run(case, world, variant, mode=mode)
     for r in res:
         assert max(r["errs"]) <= TOL[dt], (r["rank"], r["errs"])
+        if "x_kept" in r:
+            assert r["x_kept"] and r["y_same_after_cg"], r
     # bit-identical allreduce on every rank, equal to the rank-order sum
     vals = [np.array([0.1 * (q + 1), 1e16 * (-1) ** q, 3.0 + q / 7.0]) for q in range(world)]
     expect = np.zeros(3)
