@@ -252,9 +252,10 @@ def test_c2_full_closed_form(torch_cuda, dt, xkind, variant):
     assert np.array_equal(y.astype(np.float64), closed_forms.stencil_apply(dims, "7pt", xkind))
 
 
-def test_c2_full_random_parity(torch_cuda):
-    """Config 2 at full size with perturbed values, fp64, every row vs the oracle."""
-    _parity(torch_cuda, cached("c2", gen.config2), np.float64, -0.75, 0.5)
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_c2_full_random_parity(torch_cuda, dt):
+    """Config 2 at full size with perturbed values, every row vs the oracle."""
+    _parity(torch_cuda, cached("c2", gen.config2), dt, -0.75, 0.5)
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
