@@ -267,6 +267,22 @@ def copy_bandwidth(dev, reps=5):
     return round(best, 1)
 
 
+def read_bandwidth(nbytes=16 << 30, reps=5):
+    """Read-only HBM bandwidth on this box (tools/hbm_read.cu: a grid-stride
+    stream of 128-bit loads, best of `reps` passes over 16 GiB) -- context for
+    a read-dominated kernel whose fraction of the read + write copy peak can
+    exceed 1. None when the probe is not built."""
+    import ctypes
+
+    lib = os.path.join(ROOT, "tools", "libhbmread.so")
+    if not os.path.exists(lib):
+        return None
+    f = ctypes.CDLL(lib).hbm_read_gbs
+    f.argtypes, f.restype = [ctypes.c_int64, ctypes.c_int], ctypes.c_double
+    g = f(nbytes, reps)
+    return round(g, 1) if g > 0 else None
+
+
 def load_traffic(key):
     """ncu dram bytes (read + write) per launch of the dominant kernel on this
     workload, from one `ncu --set full` capture (profiles/traffic.json, keyed
@@ -629,6 +645,7 @@ def run_spmv(args):
     if world == 1 and not args.no_cpu:
         cpu = cpu_baseline(args.config, args.dtype)
     box_copy = copy_bandwidth(dev)
+    box_read = read_bandwidth()
     kname = KNAME[info["variant"]]
     line = {
         "metric": METRIC,
@@ -676,6 +693,8 @@ def run_spmv(args):
             "launches_per_step": round(launches_all / world / max(1, args.steps), 2),
             "scope": "per GPU: whole-job algorithmic bytes / N / the max-over-ranks CUDA-event step time; with several launches per step (occupancy-class ranges, interior/boundary) the step's bytes / the step's time",
             "copy_gbs_this_box": box_copy,
+            "read_gbs_this_box": box_read,
+            "frac_of_this_box_read": round(achieved / box_read, 4) if box_read else None,
         },
         "north_star_c3": subs,
         "other_configs": other,

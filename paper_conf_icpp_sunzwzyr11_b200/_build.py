@@ -102,5 +102,17 @@ def build_example() -> str:
     return EXAMPLE_BIN
 
 
+TOOL_SRC = os.path.join(ROOT, "tools", "hbm_read.cu")
+TOOL_LIB = os.path.join(ROOT, "tools", "libhbmread.so")
+
+
+def build_tools() -> str:
+    """tools/libhbmread.so: the read-only HBM bandwidth probe bench.py reports
+    as roofline context (not part of the product library)."""
+    if not os.path.exists(TOOL_LIB) or os.path.getmtime(TOOL_LIB) < os.path.getmtime(TOOL_SRC):
+        subprocess.check_call([NVCC, "-O3"] + ARCH + ["-Xcompiler", "-fPIC", "-shared", "-o", TOOL_LIB, TOOL_SRC])
+    return TOOL_LIB
+
+
 if __name__ == "__main__":
     print(build(force="--force" in sys.argv, verbose=True))
