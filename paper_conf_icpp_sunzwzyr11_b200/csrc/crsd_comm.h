@@ -24,6 +24,7 @@ struct crsd_comm_s {
     int64_t cap = 0;                  // bytes per mailbox parity
     std::vector<void *> peer_sym;     // world entries, nullptr for self / not opened
     std::vector<int64_t> peer_cap;    // each peer's mailbox bytes per parity (read from its flags)
+    std::vector<uint8_t> peer_same_gpu;  // 1 if the peer's region lives on my GPU (ranks sharing a device)
     bool opened = false;
     bool poisoned = false;            // a wait timed out (seen by crsd_comm_error): refuse further exchanges
     uint64_t xseq = 0;                // crsd_dist_x_alloc handshakes made

@@ -21,6 +21,7 @@ struct P2PFlags {
     uint32_t counter[2];  // own: grid arrival counters (send, recv)
     uint32_t err;         // own: 0, or 1/2/3/4 = send/recv/allreduce/close wait timed out
     int64_t cap;          // own mailbox bytes per parity (read by peers at open)
+    uint8_t dev_uuid[16]; // own GPU's UUID (read by peers at open: who shares my GPU)
     uint64_t closing[P2P_MAX_WORLD];  // written by q at crsd_comm_destroy: q no longer touches my region
     // crsd_dist_x_alloc handshake, written by q (host copies into peer memory):
     // q's padded-x IPC handle, then xseq[q] = the allocation's sequence number

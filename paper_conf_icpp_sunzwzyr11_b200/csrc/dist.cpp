@@ -195,6 +195,7 @@ crsd_status_t crsd_comm_init_p2p(int rank, int world, int device, int64_t mailbo
     c->cap = (mailbox_bytes + 255) / 256 * 256;
     c->peer_sym.assign(world, nullptr);
     c->peer_cap.assign(world, 0);
+    c->peer_same_gpu.assign(world, 0);
     if (const char *t = getenv("CRSD_P2P_TIMEOUT_S")) {
         const double sec = atof(t);
         if (sec > 0) c->timeout_ns = (uint64_t)(sec * 1e9);
@@ -205,6 +206,10 @@ crsd_status_t crsd_comm_init_p2p(int rank, int world, int device, int64_t mailbo
     if (e == cudaSuccess)
         e = cudaMemcpy((char *)c->sym + offsetof(crsd::P2PFlags, cap), &c->cap, sizeof(int64_t),
                        cudaMemcpyHostToDevice);
+    cudaDeviceProp prop;
+    if (e == cudaSuccess) e = cudaGetDeviceProperties(&prop, device);
+    if (e == cudaSuccess)
+        e = cudaMemcpy((char *)c->sym + offsetof(crsd::P2PFlags, dev_uuid), &prop.uuid, 16, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaIpcGetMemHandle((cudaIpcMemHandle_t *)ipc_handle64, c->sym);
     int prio_lo = 0, prio_hi = 0;
     if (e == cudaSuccess) e = cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
@@ -235,6 +240,10 @@ crsd_status_t crsd_comm_p2p_open(crsd_comm_t c, const void *ipc_handles) {
         // the peer wrote its capacity before exporting the handle
         CU_TRY(cudaMemcpy(&c->peer_cap[q], (char *)p + offsetof(crsd::P2PFlags, cap), sizeof(int64_t),
                           cudaMemcpyDeviceToHost));
+        uint8_t uq[16], um[16];
+        CU_TRY(cudaMemcpy(uq, (char *)p + offsetof(crsd::P2PFlags, dev_uuid), 16, cudaMemcpyDeviceToHost));
+        CU_TRY(cudaMemcpy(um, (char *)c->sym + offsetof(crsd::P2PFlags, dev_uuid), 16, cudaMemcpyDeviceToHost));
+        c->peer_same_gpu[q] = std::memcmp(uq, um, 16) == 0;
     }
     c->opened = true;
     return CRSD_OK;
@@ -611,9 +620,18 @@ crsd_status_t crsd::spmv_dist_impl(crsd_matrix_t A, const void *alpha, void *x_p
     // before copying its x windows, the last CTA releases the pads -- so a
     // call is put + interior + boundary, no separate wait / release kernels
     // (CRSD_TUNE_HALO_UNFUSED restores them).
+    // Liveness: the boundary CTAs spin until the senders' puts land. A
+    // sender on another GPU always runs; a sender SHARING this GPU (ranks
+    // co-located, e.g. under MPS) needs an SM slot, which spinning CTAs
+    // could all hold -- so with a co-located sender the fused form is used
+    // only while the boundary launch fits in one CTA per SM.
+    bool colocated_sender = false;
+    if (c && c->kind == crsd_comm_s::P2P)
+        for (int64_t q : A->recv_peer) colocated_sender |= c->peer_same_gpu[q] != 0;
     const bool fused = c && c->kind == crsd_comm_s::P2P && A->find_dx(xp, c) &&
                        A->variant == VARIANT_JIT && A->jit_halo_function && !A->list_boundary.empty() &&
-                       !(A->tune & CRSD_TUNE_HALO_UNFUSED);
+                       !(A->tune & CRSD_TUNE_HALO_UNFUSED) &&
+                       (!colocated_sender || (int64_t)A->list_boundary.size() <= A->sm_count);
     auto exchange = [&]() -> crsd_status_t {
         crsd::NvtxRange nvx("halo exchange");
         CU_TRY(cudaStreamWaitEvent(c->cs, c->ev_x, 0));
