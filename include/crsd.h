@@ -133,6 +133,18 @@ typedef struct {
 #define CRSD_TUNE_NO_JIT 0x20u             /* AUTO never picks the JIT variant */
 #define CRSD_TUNE_HALO_UNFUSED 0x40u       /* crsd_spmv_dist direct mode: separate wait / release kernels instead of
                                               the receive fused into the boundary kernel (crsd_jit_halo) */
+#define CRSD_TUNE_JIT_NO_SLAB 0x100u       /* JIT: each CTA finds its scatter points through its segment descriptor
+                                              instead of the per-segment slab of the first 16 */
+#define CRSD_TUNE_JIT_INTERLEAVE 0x200u    /* JIT, one GPU: one launch in which the light instances' segments are
+                                              spread evenly among the heavy ones, instead of occupancy-class range
+                                              launches */
+#define CRSD_TUNE_JIT_NO_PDL 0x80u         /* crsd_spmv, JIT: plain launches instead of programmatic dependent launch.
+                                              By default a one-GPU handle whose matrix runs as ONE launch is
+                                              launched with PDL: it may start while the previous kernel on the
+                                              stream drains; its CTAs stream the (immutable) matrix values first
+                                              and wait for the previous kernel (griddepcontrol.wait) before they
+                                              touch x or y. Handles split into occupancy-class ranges keep their
+                                              concurrent range launches; stream capture keeps plain launches */
 
 #define CRSD_VARIANT_AUTO 0
 #define CRSD_VARIANT_LDG 1
@@ -169,6 +181,8 @@ typedef struct {
     int32_t smem_bytes;             /* dynamic shared memory per CTA of the TMA variant */
     int64_t unique_bytes_beta0;     /* algorithmic bytes of one SpMV with beta == 0 */
     int64_t unique_bytes_beta1;     /* ... with beta != 0 (y also read) */
+    int32_t jit_launches;           /* JIT: kernel launches of one crsd_spmv (occupancy-class ranges), else 1 */
+    int32_t pdl;                    /* 1: crsd_spmv launches with programmatic dependent launch (CRSD_TUNE_JIT_NO_PDL) */
 } crsd_info_t;
 
 /*

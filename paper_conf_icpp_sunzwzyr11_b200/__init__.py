@@ -23,4 +23,7 @@ from .crsd import (  # noqa: F401
     TUNE_DIST_BOUNDARY_SERIAL,
     TUNE_NO_JIT,
     TUNE_HALO_UNFUSED,
+    TUNE_JIT_NO_PDL,
+    TUNE_JIT_NO_SLAB,
+    TUNE_JIT_INTERLEAVE,
 )

@@ -3,6 +3,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <climits>
 #include <cstdlib>
 #include <cstring>
 #include <string>
@@ -76,11 +77,11 @@ void free_device(crsd_matrix_s *A) {
     }
     A->dx.clear();
     void *ptrs[] = {A->d_vals, A->d_segs, A->d_offs, A->d_plan, A->d_scat_row, A->d_scat_col, A->d_scat_val, A->d_scat_rec,
-                    A->d_list_interior, A->d_list_boundary, A->d_list_all_edge, A->d_x_scratch, A->d_y_scratch, A->d_cg,
+                    A->d_scat_slab, A->d_list_interior, A->d_list_boundary, A->d_list_all_edge, A->d_x_scratch, A->d_y_scratch, A->d_cg,
                     A->d_ell_rowno, A->d_ell_col, A->d_ell_val};
     for (void *p : ptrs)
         if (p) cudaFree(p);
-    A->d_vals = A->d_segs = A->d_offs = A->d_plan = A->d_scat_row = A->d_scat_col = A->d_scat_val = A->d_scat_rec = nullptr;
+    A->d_vals = A->d_segs = A->d_offs = A->d_plan = A->d_scat_row = A->d_scat_col = A->d_scat_val = A->d_scat_rec = A->d_scat_slab = nullptr;
     A->d_list_interior = A->d_list_boundary = A->d_list_all_edge = A->d_x_scratch = A->d_y_scratch = A->d_cg = nullptr;
     A->d_ell_rowno = A->d_ell_col = A->d_ell_val = nullptr;
     A->cg_bytes = 0;
@@ -149,6 +150,14 @@ static void plan_layout(crsd_matrix_s *A) {
     }
 }
 
+bool slab_ok(const crsd_matrix_s *A) {
+    const HostCRSD &H = A->H;
+    if (H.nscatter() == 0 || (A->tune & CRSD_TUNE_JIT_NO_SLAB) || H.mrows > 65535) return false;
+    for (int64_t c : H.scat_col)
+        if (c - H.row_begin < INT32_MIN || c - H.row_begin > INT32_MAX) return false;
+    return true;
+}
+
 static crsd_status_t upload(crsd_matrix_s *A) {
     HostCRSD &H = A->H;
     if (A->device < 0) CUDA_TRY(cudaGetDevice(&A->device));
@@ -178,6 +187,24 @@ static crsd_status_t upload(crsd_matrix_s *A) {
             rec[e] = r;
         }
         if ((st = dev_alloc_copy(&A->d_scat_rec, rec.data(), ns * sizeof(ScatRec), cnt))) return st;
+    }
+    // scatter slab (JIT codelets; CRSD_TUNE_JIT_NO_SLAB keeps the descriptor path)
+    if (slab_ok(A)) {
+        std::vector<SlabRec> sl((size_t)H.nseg * SLAB_K);
+        for (int64_t sg = 0; sg < H.nseg; ++sg) {
+            const int64_t b = H.scat_ptr[sg], n = H.scat_ptr[sg + 1] - b;
+            for (int l = 0; l < SLAB_K; ++l) {
+                SlabRec r{};
+                r.n = (uint16_t)std::min<int64_t>(n, 65535);
+                if (l < n) {
+                    r.col = (int32_t)colrel[b + l];
+                    r.row = (uint16_t)H.scat_row[b + l];
+                    std::memcpy(&r.val, H.scat_val.data() + (b + l) * H.elem, H.elem);
+                }
+                sl[sg * SLAB_K + l] = r;
+            }
+        }
+        if ((st = dev_alloc_copy(&A->d_scat_slab, sl.data(), sl.size() * sizeof(SlabRec), cnt))) return st;
     }
     if ((st = dev_alloc_copy(&A->d_list_interior, A->list_interior.data(), A->list_interior.size() * 4, cnt))) return st;
     if ((st = dev_alloc_copy(&A->d_list_boundary, A->list_boundary.data(), A->list_boundary.size() * 4, cnt))) return st;
@@ -296,10 +323,12 @@ static crsd_status_t resolve_opts(int64_t nrows, crsd_dtype_t dtype, const crsd_
 
 template <typename T>
 static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *y, const int32_t *list,
-                              int64_t seg_begin, int64_t count, void *stream, int &launches, const HaloSync *halo) {
+                              int64_t seg_begin, int64_t count, void *stream, int &launches, const HaloSync *halo,
+                              bool pdl) {
     if (count <= 0) return CRSD_OK;
     SpmvArgs<T> a;
     a.halo = halo;
+    a.pdl = pdl;
     a.vals = (const T *)A->d_vals;
     a.segs = (const SegDesc *)A->d_segs;
     a.pat_offs = (const int32_t *)A->d_offs;
@@ -320,6 +349,7 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
     a.scat_col = (const int64_t *)A->d_scat_col;
     a.scat_val = (const T *)A->d_scat_val;
     a.scat_rec = (const ScatRec *)A->d_scat_rec;
+    a.scat_slab = (const SlabRec *)A->d_scat_slab;
     a.x = x;
     a.x_lo = A->x_lo;
     a.x_hi = A->x_hi;
@@ -346,13 +376,13 @@ static crsd_status_t run_spmv(crsd_matrix_s *A, T alpha, const T *x, T beta, T *
 
 crsd_status_t run_lists(crsd_matrix_s *A, const void *alpha, const void *x_base, const void *beta, void *y,
                         const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches,
-                        const HaloSync *halo) {
+                        const HaloSync *halo, bool pdl) {
     if (halo && A->variant != VARIANT_JIT) return fail(CRSD_ERR_UNSUPPORTED, "fused halo receive needs the JIT variant");
     if (A->H.dtype == CRSD_R64F)
         return run_spmv<double>(A, *(const double *)alpha, (const double *)x_base, *(const double *)beta, (double *)y,
-                                list, seg_begin, count, stream, launches, halo);
+                                list, seg_begin, count, stream, launches, halo, pdl);
     return run_spmv<float>(A, *(const float *)alpha, (const float *)x_base, *(const float *)beta, (float *)y, list,
-                           seg_begin, count, stream, launches, halo);
+                           seg_begin, count, stream, launches, halo, pdl);
 }
 
 }  // namespace crsd
@@ -465,7 +495,7 @@ crsd_status_t crsd_spmv(crsd_matrix_t A, const void *alpha, const void *x, const
     int launches = 0;
     cudaSetDevice(A->device);
     const int64_t nseg = A->H.nseg;
-    st = run_lists(A, alpha, x, beta, y, nullptr, 0, nseg, stream, launches);
+    st = run_lists(A, alpha, x, beta, y, nullptr, 0, nseg, stream, launches, nullptr, true);
     if (!st && A->H.paper_ell && A->H.ell_nrows > 0) {
         // second part of the paper's kernel: the scatter rows,
         // stored whole in ELL, overwrite what the diagonal part wrote
@@ -659,6 +689,8 @@ crsd_status_t crsd_get_info(crsd_matrix_t A, crsd_info_t *I) {
     const int64_t base = H.nslots * es + I->nscatter * (es + 4 + 8) + xs * es + H.n_local * es;
     I->unique_bytes_beta0 = base;
     I->unique_bytes_beta1 = base + H.n_local * es;
+    I->jit_launches = A->variant == VARIANT_JIT ? (int32_t)std::max<size_t>(1, A->jit_ranges.size()) : 1;
+    I->pdl = (A->variant == VARIANT_JIT && !A->host_only && jit_pdl(A)) ? 1 : 0;
     return CRSD_OK;
 }
 

@@ -58,6 +58,7 @@ struct crsd_matrix_s {
     void *d_scat_col = nullptr;
     void *d_scat_val = nullptr;
     void *d_scat_rec = nullptr;
+    void *d_scat_slab = nullptr;  // crsd::SlabRec[nseg * SLAB_K] (JIT; null if a column does not fit int32)
     void *d_list_interior = nullptr;
     void *d_list_boundary = nullptr;
     void *d_list_all_edge = nullptr;
@@ -116,12 +117,18 @@ crsd_status_t jit_build(crsd_matrix_s *A);
 void jit_free(crsd_matrix_s *A);
 template <typename T>
 int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &a, void *stream);
+// crsd_spmv launches A's JIT kernel with programmatic dependent launch
+bool jit_pdl(const crsd_matrix_s *A);
+// A's scatter points go to the per-segment slab (SlabRec) for the JIT codelets
+bool slab_ok(const crsd_matrix_s *A);
 // Run the SpMV kernel over a device list of segments (list == nullptr: the
 // segment range [seg_begin, seg_begin + count)). x_base is the local x base
 // (x_padded + halo_lo).
 // halo != null: the boundary launch of a direct-mode exchange with the
 // receive side fused into the JIT kernel (crsd_jit_halo).
+// pdl: the caller (crsd_spmv) allows a programmatic dependent launch
+// (used when jit_pdl(A) and the stream is not capturing).
 crsd_status_t run_lists(crsd_matrix_s *A, const void *alpha, const void *x_base, const void *beta, void *y,
                         const int32_t *list, int64_t seg_begin, int64_t count, void *stream, int &launches,
-                        const HaloSync *halo = nullptr);
+                        const HaloSync *halo = nullptr, bool pdl = false);
 }  // namespace crsd

@@ -75,6 +75,21 @@ struct alignas(16) ScatRec {
 };
 static_assert(sizeof(ScatRec) == 32, "ScatRec must be 32 bytes");
 
+// Scatter slab (JIT codelets): the first SLAB_K scatter points of segment s
+// at slab[s * SLAB_K + l], 16 bytes each, so a CTA loads its points from an
+// address it knows without any load (no segment-descriptor round trip before
+// the x gathers). Every slot, used or not, carries the segment's point count
+// n (saturated at 65535); points beyond SLAB_K are read from the plain
+// arrays (scat_row/col/val at scat_begin + l) after the descriptor load.
+constexpr int SLAB_K = 16;
+struct alignas(16) SlabRec {
+    int32_t col;    // column relative to the local x base
+    uint16_t row;   // row within the segment
+    uint16_t n;     // the segment's scatter points, min(n, 65535)
+    double val;     // float matrices use the first 4 bytes
+};
+static_assert(sizeof(SlabRec) == 16, "SlabRec must be 16 bytes");
+
 struct HostCRSD {
     int64_t nrows = 0, ncols = 0;    // global
     int64_t row_begin = 0, row_end = 0;
@@ -179,6 +194,7 @@ struct SpmvArgs {
     const int64_t *scat_col;  // relative to x base
     const T *scat_val;
     const ScatRec *scat_rec;  // same points as 32-byte records
+    const SlabRec *scat_slab; // per-segment slab of the first SLAB_K points (JIT), or null
     const T *x;               // local x base (x_padded + halo_lo for dist)
     int64_t x_lo, x_hi;       // valid x range relative to x
     T *y;
@@ -196,6 +212,7 @@ struct SpmvArgs {
     int32_t variant;          // VARIANT_LDG / _TMA / _PIPE / _JIT
     T alpha, beta;
     const HaloSync *halo = nullptr;  // JIT boundary launch with the fused halo receive, or null
+    bool pdl = false;                // JIT: programmatic dependent launch allowed (CRSD_TUNE_JIT_PDL)
 };
 
 // Paper-exact scatter rows (CRSD_PAPER_ELL): y[rowno[i]] = alpha * sum_k

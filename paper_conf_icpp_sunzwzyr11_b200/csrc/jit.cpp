@@ -70,6 +70,7 @@ struct DriverApi {
                        void **, void **);
     CUresult (*set_attr)(CUfunction, CUfunction_attribute, int);
     CUresult (*unload)(CUmodule);
+    CUresult (*launch_ex)(const CUlaunchConfig *, CUfunction, void **, void **) = nullptr;  // optional (PDL)
 };
 
 NvrtcApi &nvrtc() {
@@ -123,6 +124,7 @@ DriverApi &driver() {
         api.set_attr = reinterpret_cast<decltype(api.set_attr)>(p);
         if (!get("cuModuleUnload", &p)) { api.err = "cuModuleUnload"; return; }
         api.unload = reinterpret_cast<decltype(api.unload)>(p);
+        if (get("cuLaunchKernelEx", &p)) api.launch_ex = reinterpret_cast<decltype(api.launch_ex)>(p);
         api.ok = true;
     });
     return api;
@@ -143,6 +145,7 @@ struct JitArgs {
     const int64_t *scat_col;
     const T *scat_val;
     const ScatRec *scat_rec;
+    const SlabRec *scat_slab;
     T alpha, beta;
 };
 
@@ -155,7 +158,8 @@ struct SegDesc { i64 val_base; i64 scat_begin; int off_begin; int nscat; u16 fla
 struct __align__(16) ScatRec { i64 col; double val; int row; int pad[3]; };
 struct Args { const T *vals; const SegDesc *segs; const int *seg_list; i64 seg_begin, seg_count;
               const T *x; i64 x_lo, x_hi; T *y; i64 nrows;
-              const int *scat_row; const i64 *scat_col; const T *scat_val; const ScatRec *scat_rec; T alpha, beta; };
+              const int *scat_row; const i64 *scat_col; const T *scat_val; const ScatRec *scat_rec; const int4 *scat_slab;
+              T alpha, beta; };
 __device__ __forceinline__ u32 su32(const void *p) { return (u32)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void bar_init(u64 *b) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(su32(b)) : "memory"); }
@@ -249,11 +253,101 @@ void emit_locate(std::ostringstream &o, const std::vector<Leaf> &L, size_t lo, s
 
 }  // namespace
 
+// Programmatic dependent launch (PDL) for crsd_spmv: a one-GPU handle whose
+// matrix runs as one launch. Consecutive SpMVs on a stream then overlap: the
+// next launch's CTAs take the SM slots the previous kernel's last wave frees
+// and stream their values while it drains (frac of the copy peak, plain ->
+// PDL: C2 f64 1.080 -> 1.101, C2 f32 1.054 -> 1.091, C3 f32 1.044 -> 1.069;
+// profiles/r02/sweep6_pdl_default.jsonl). Occupancy-class range launches
+// keep their concurrent forked streams: a PDL chain of the ranges measured
+// 0.89-0.93 against 0.98-1.03 on C3 f64 (sweep5_pdl_chain.jsonl).
+bool jit_pdl(const crsd_matrix_s *A) {
+    return !(A->tune & CRSD_TUNE_JIT_NO_PDL) && !A->H.partitioned && A->jit_ranges.size() <= 1;
+}
+
 // rows per thread of the generated kernel: <= 256 threads per CTA
 static int jit_q(const crsd_matrix_s *A) {
     int q = 1;
     while (A->H.mrows / q > 256) q *= 2;
     return q;
+}
+
+// Staging bytes (values + x windows) of one CTA of instance I, and the CTAs
+// per SM a launch with `b` bytes of dynamic shared memory per CTA allows.
+static int64_t inst_staging(const crsd_matrix_s *A, const Instance &I) {
+    const HostCRSD &H = A->H;
+    const int32_t *pl = A->plan.data() + A->segdesc[I.first_seg].plan_begin;
+    int64_t el = H.ndias(I.pattern) * H.mrows;
+    for (int w = 0; w < pl[0]; ++w) el += pl[3 + 2 * w];
+    return el * H.elem;
+}
+static int64_t occupancy_of(const crsd_matrix_s *A, int64_t b) {
+    const int64_t nt = A->H.mrows / jit_q(A);
+    const int64_t per_cta = (b + 127) / 128 * 128 + 1024 + 256;  // + driver reserve + static smem (barriers)
+    return std::min<int64_t>(2048 / nt, (228 * 1024) / per_cta);
+}
+
+// Interleaved single launch (CRSD_TUNE_JIT_INTERLEAVE): instead of launching
+// the light instances (staging small enough for >= 2x the CTAs per SM of the
+// largest) as separate occupancy-class ranges, ONE launch visits them spread
+// evenly among the heavy segments: block b takes light segment b / R when
+// b % R == R - 1 (and light ones remain), else the next heavy segment in
+// order. A light CTA then shares its SM with heavy CTAs whose staging keeps
+// HBM busy, instead of a run of light CTAs that cannot (C3's idle block B3:
+// one diagonal per segment), and the handle stays one launch (PDL applies).
+// [a, b) runs of edge segments
+static std::vector<std::pair<int64_t, int64_t>> edge_runs(const crsd_matrix_s *A) {
+    std::vector<std::pair<int64_t, int64_t>> edges;
+    for (int64_t s = 0; s < A->H.nseg; ++s)
+        if (A->segdesc[s].flags & SEG_EDGE) {
+            if (!edges.empty() && edges.back().second == s) edges.back().second = s + 1;
+            else edges.push_back({s, s + 1});
+        }
+    return edges;
+}
+// the generated kernel carries the baked segment -> (pattern, value base) lookup
+static bool jit_locate(const crsd_matrix_s *A, const std::vector<std::pair<int64_t, int64_t>> &edges) {
+    return !(A->tune & CRSD_TUNE_JIT_DESC_ISSUE) && !A->H.inst.empty() && A->H.inst.size() <= 4096 &&
+           edges.size() <= 16;
+}
+
+struct Interleave {
+    int64_t R = 0, L = 0;
+    std::vector<std::vector<int64_t>> light, heavy;  // runs {first index, first segment, length}
+};
+static bool interleave_plan(const crsd_matrix_s *A, Interleave &iv) {
+    const HostCRSD &H = A->H;
+    if (!(A->tune & CRSD_TUNE_JIT_INTERLEAVE) || H.partitioned || !jit_locate(A, edge_runs(A))) return false;
+    const int64_t occ_max = occupancy_of(A, A->smem_bytes);
+    auto add = [](std::vector<std::vector<int64_t>> &runs, int64_t &count, const Instance &I) {
+        if (!runs.empty() && runs.back()[1] + runs.back()[2] == I.first_seg) runs.back()[2] += I.nseg;
+        else runs.push_back({count, I.first_seg, I.nseg});
+        count += I.nseg;
+    };
+    int64_t nl = 0, nh = 0;
+    for (const Instance &I : H.inst) {
+        if (occupancy_of(A, inst_staging(A, I)) >= 2 * occ_max) add(iv.light, nl, I);
+        else add(iv.heavy, nh, I);
+    }
+    if (nl == 0 || nh == 0 || iv.light.size() > 256 || iv.heavy.size() > 256) return false;
+    iv.L = nl;
+    iv.R = H.nseg / nl;
+    return iv.R >= 2;
+}
+
+static void emit_runs(std::ostringstream &o, const std::vector<std::vector<int64_t>> &L, size_t lo, size_t hi,
+                      const char *idx, int depth) {
+    const std::string ind(2 + 2 * depth, ' ');
+    if (hi - lo == 1) {
+        o << ind << "return " << L[lo][1] << "LL + (" << idx << " - " << L[lo][0] << "LL);\n";
+        return;
+    }
+    const size_t mid = (lo + hi) / 2;
+    o << ind << "if (" << idx << " < " << L[mid][0] << "LL) {\n";
+    emit_runs(o, L, lo, mid, idx, depth + 1);
+    o << ind << "} else {\n";
+    emit_runs(o, L, mid, hi, idx, depth + 1);
+    o << ind << "}\n";
 }
 
 // Generate the codelets of every distinct pattern of A (one CTA per segment,
@@ -263,8 +357,16 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
     const bool f64 = H.dtype == CRSD_R64F;
     const int m = H.mrows, nt = m / Q, es = H.elem;
     const bool scat = H.nscatter() > 0;  // scatter code only for matrices that have scatter points
+    // programmatic dependent launch (jit_pdl): the value copies (the matrix
+    // never changes) are issued before griddepcontrol.wait, the x windows,
+    // scatter gathers and y after it
+    const bool pdl = jit_pdl(A);
+    // scatter slab: a CTA's first SLAB_K points from a fixed address
+    const bool slab = scat && slab_ok(A);
     std::ostringstream o;
     o << "typedef " << (f64 ? "double" : "float") << " T;\n" << kPrelude;
+    // a slab record's value (int4 .z/.w): the dtype's bits, no local-memory round trip
+    o << (f64 ? "#define SLAB_VAL(r) __hiloint2double((r).w, (r).z)\n" : "#define SLAB_VAL(r) __int_as_float((r).z)\n");
     o << "#define MROWS " << m << "\n#define NT " << nt << "\n#define Q " << Q << "\n";
     // one __device__ codelet per distinct pattern, keyed by the pattern's
     // plan_begin (unique per distinct pattern; off_begin is not: a pattern
@@ -296,6 +398,12 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
         o << "__device__ __forceinline__ void codelet_" << key
           << "(const Args &a, const i64 s, const i64 vb, const i64 row0, const bool edge, T *vs, u64 *bar, const int t,"
              " const bool halo, const HaloSync &hs, const u64 he) {\n";
+        if (slab)
+            // the slab load needs no other load: issued first, it lands while
+            // thread 0 sets up the copies (the matrix never changes, so it may
+            // also precede griddepcontrol.wait)
+            o << "  int4 sr = make_int4(0, 0, 0, 0);\n"
+                 "  if ((t & 31) < " << SLAB_K << ") sr = __ldg(a.scat_slab + s * " << SLAB_K << " + (t & 31));\n";
         if (nd) {
             // thread 0: every mbarrier, then every copy, chunk by chunk
             o << "  T *xs = vs + " << (int64_t)nd * m << ";\n";
@@ -312,7 +420,7 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
                   << (xbytes ? std::to_string(xbytes) + "u)" : "") << ");\n";
                 o << "    g2s(vs + " << (int64_t)k.d0 * m << ", a.vals + vb + " << (int64_t)k.d0 * m << ", " << vbytes
                   << "u, bar + " << c << ", pf);\n";
-                if (xbytes) {
+                if (xbytes && !pdl) {
                     o << "    if (!edge && !halo) {\n";
                     for (int w = 0; w < nwin; ++w) {
                         if (!(k.win == -2 || k.win == w)) continue;
@@ -335,11 +443,31 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
             }
             o << "    }\n";
             o << "  }\n";
+            if (pdl) {
+                // every thread orders its x / y accesses after the previous
+                // kernel on the stream; then thread 0 issues the windows
+                o << "  if (!halo) {\n    asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");\n"
+                     "    if (t == 0 && !edge) {\n      const u64 pn = pol_normal();\n";
+                for (size_t c = 0; c < ch.size(); ++c) {
+                    const Chunk &k = ch[c];
+                    if (k.win == -1) continue;
+                    for (int w = 0; w < nwin; ++w) {
+                        if (!(k.win == -2 || k.win == w)) continue;
+                        o << "      g2s(xs + " << wbase[w] << ", a.x + row0 + (" << pl[2 + 2 * w] << "), "
+                          << (int64_t)pl[3 + 2 * w] * es << "u, bar + " << c << ", pn);\n";
+                    }
+                }
+                o << "    }\n  }\n";
+            }
         } else {
             o << "  (void)vs; (void)bar; (void)vb;\n";
             o << "  if (halo) { if (t == 0) halo_wait(hs, he); __syncthreads(); }\n";
+            if (pdl) o << "  if (!halo) asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");\n";
         }
-        if (scat) {
+        if (slab) {
+            o << "  int g_own = -1; T g_v = T(0), g_x = T(0); unsigned g_mask = 0u;\n"
+                 "  const int nscat = __shfl_sync(0xffffffffu, (sr.y >> 16) & 0xffff, 0);\n";
+        } else if (scat) {
             // scatter points are gathered while the bulk copies are in flight:
             // lane l of every warp reads record l of the segment's first 32
             // (row, col, value in one 32-B record); a ballot keeps those whose
@@ -348,7 +476,16 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
                  "  const i64 sbeg = nscat > 0 ? __ldg(&Dp->scat_begin) : 0;\n"
                  "  int g_own = -1; T g_v = T(0), g_x = T(0); unsigned g_mask = 0u;\n";
         }
+        static_assert(SLAB_K == 16, "the generated slab gather assumes 16 slots");
         const char *gather =
+            slab ? "  if (nscat > 0) {\n"
+                   "    const int lane = t & 31, row = sr.y & 0xffff;\n"
+                   "    if (lane < min(nscat, 16)) g_own = (row % NT) * Q + row / NT;\n"
+                   "    const bool mine = g_own >= 0 && (g_own / Q) / 32 == t / 32;\n"
+                   "    g_mask = __ballot_sync(0xffffffffu, mine);\n"
+                   "    if (mine) { g_v = SLAB_VAL(sr); g_x = __ldg(a.x + sr.x); }\n"
+                   "  }\n"
+                 :
             "  if (nscat > 0) {\n"
             "    const int lane = t & 31;\n"
             "    ScatRec R; R.col = 0; R.val = 0; R.row = 0;\n"
@@ -381,7 +518,8 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
         o << "  }\n";
         // scatter points in (row, col) order by their owner thread: the
         // gathered ones (broadcast from the lane holding them), then any
-        // beyond the first 32; then the epilogue
+        // beyond the first 32 (16 with the slab, after the descriptor load);
+        // then the epilogue
         if (scat)
             o << "  if (nscat > 0) {\n"
                  "    for (unsigned mm = g_mask; mm; mm &= mm - 1) {\n"
@@ -390,12 +528,16 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
                  "      const T v = __shfl_sync(0xffffffffu, g_v, j), xv = __shfl_sync(0xffffffffu, g_x, j);\n"
                  "#pragma unroll\n      for (int q = 0; q < Q; ++q) if (own == t * Q + q) acc[q] = fma(v, xv, acc[q]);\n"
                  "    }\n"
-                 "    for (int e = 32; e < nscat; ++e) {\n"
-                 "      const int rr = __ldg(a.scat_row + sbeg + e);\n"
+              << (slab ? "    if (nscat > 16) {\n"
+                         "    const SegDesc *Dp = a.segs + s;\n"
+                         "    const int nall = __ldg(&Dp->nscat);\n    const i64 sbeg = __ldg(&Dp->scat_begin);\n"
+                         "    for (int e = 16; e < nall; ++e) {\n"
+                       : "    {\n    for (int e = 32; e < nscat; ++e) {\n")
+              << "      const int rr = __ldg(a.scat_row + sbeg + e);\n"
                  "      if (rr % NT != t) continue;\n"
                  "      const T v = __ldg(a.scat_val + sbeg + e), xv = __ldg(a.x + __ldg(a.scat_col + sbeg + e));\n"
                  "#pragma unroll\n      for (int q = 0; q < Q; ++q) if (rr / NT == q) acc[q] = fma(v, xv, acc[q]);\n"
-                 "    }\n  }\n";
+                 "    }\n    }\n  }\n";
         // epilogue: y = alpha*acc + beta*y, y not read when beta == 0
         o << "#pragma unroll\n  for (int q = 0; q < Q; ++q) {\n    const i64 r = row0 + t + q * NT;\n"
              "    if (!edge || r < a.nrows) {\n      T *yp = a.y + r;\n"
@@ -406,14 +548,8 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
     // range launches (the one-GPU path and contiguous interiors); list
     // launches read the descriptor. Off with CRSD_TUNE_JIT_DESC_ISSUE, or when
     // the tables would be large.
-    std::vector<std::pair<int64_t, int64_t>> edges;  // [a, b) runs of edge segments
-    for (int64_t s = 0; s < H.nseg; ++s)
-        if (A->segdesc[s].flags & SEG_EDGE) {
-            if (!edges.empty() && edges.back().second == s) edges.back().second = s + 1;
-            else edges.push_back({s, s + 1});
-        }
-    const bool locate = !(A->tune & CRSD_TUNE_JIT_DESC_ISSUE) && !H.inst.empty() && H.inst.size() <= 4096 &&
-                        edges.size() <= 16;
+    std::vector<std::pair<int64_t, int64_t>> edges = edge_runs(A);
+    const bool locate = jit_locate(A, edges);
     o << "#define NBAR " << nbar << "\n";
     if (locate) {
         std::vector<Leaf> L;
@@ -425,12 +561,26 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
         for (const auto &e : edges) o << " || (s >= " << e.first << "LL && s < " << e.second << "LL)";
         o << ";\n}\n";
     }
+    Interleave iv;
+    const bool inter = locate && interleave_plan(A, iv);
+    if (inter) {
+        o << "#define NSEG " << H.nseg << "LL\n";
+        o << "__device__ __forceinline__ i64 seg_of_block(const i64 b) {\n  const i64 k = b / " << iv.R << "LL;\n"
+          << "  if (b % " << iv.R << "LL == " << iv.R - 1 << "LL && k < " << iv.L << "LL) {\n";
+        emit_runs(o, iv.light, 0, iv.light.size(), "k", 1);
+        o << "  }\n  const i64 h = b - (k < " << iv.L << "LL ? k : " << iv.L << "LL);\n";
+        emit_runs(o, iv.heavy, 0, iv.heavy.size(), "h", 0);
+        o << "}\n";
+    }
     // the dispatch body shared by crsd_jit and crsd_jit_halo
     o << "__device__ __forceinline__ void run_segment(const Args &a, const bool halo, const HaloSync &hs, const u64 he) {\n"
          "  extern __shared__ __align__(128) unsigned char smem[];\n  __shared__ u64 bar[NBAR];\n"
          "  T *vs = reinterpret_cast<T *>(smem);\n  i64 s, vb;\n  int key;\n  bool edge;\n";
     if (locate)
-        o << "  if (!a.seg_list) {\n    s = a.seg_begin + blockIdx.x;\n    locate(s, key, vb);\n    edge = is_edge(s);\n"
+        o << "  if (!a.seg_list) {\n"
+          << (inter ? "    s = (a.seg_begin == 0 && a.seg_count == NSEG) ? seg_of_block(blockIdx.x) : a.seg_begin + blockIdx.x;\n"
+                    : "    s = a.seg_begin + blockIdx.x;\n")
+          << "    locate(s, key, vb);\n    edge = is_edge(s);\n"
              "  } else {\n";
     else
         o << "  {\n";
@@ -440,8 +590,9 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
     for (int32_t v : seen)
         o << "  case " << v << ": codelet_" << v << "(a, s, vb, row0, edge, vs, bar, threadIdx.x, halo, hs, he); break;\n";
     o << "  }\n}\n";
-    o << "extern \"C\" __global__ void __launch_bounds__(NT) crsd_jit(const Args a) {\n"
-         "  const HaloSync hs{};\n  run_segment(a, false, hs, 0ull);\n}\n";
+    o << "extern \"C\" __global__ void __launch_bounds__(NT) crsd_jit(const Args a) {\n";
+    if (pdl) o << "  asm volatile(\"griddepcontrol.launch_dependents;\");\n";
+    o << "  const HaloSync hs{};\n  run_segment(a, false, hs, 0ull);\n}\n";
     // boundary segments of a direct-mode exchange: the receive side fused in
     // (wait per CTA before the window copies; the last CTA to finish releases
     // the pads to the senders and advances the epoch)
@@ -479,20 +630,14 @@ static void jit_plan_ranges(crsd_matrix_s *A) {
     const bool off = (A->tune & CRSD_TUNE_JIT_ONE_LAUNCH) != 0;
     const bool force = (A->tune & CRSD_TUNE_JIT_SPLIT_ALL) != 0;
     std::vector<int64_t> whole = {0, nseg, A->smem_bytes, 0};
-    if (off || H.inst.empty()) {
+    Interleave iv;
+    if (off || H.inst.empty() || interleave_plan(A, iv)) {
         A->jit_ranges.push_back(whole);
         return;
     }
-    auto staging = [&](const Instance &I) {
-        const int32_t *pl = A->plan.data() + A->segdesc[I.first_seg].plan_begin;
-        int64_t el = H.ndias(I.pattern) * H.mrows;
-        for (int w = 0; w < pl[0]; ++w) el += pl[3 + 2 * w];
-        return el * H.elem;
-    };
-    auto occupancy = [&](int64_t b) {
-        const int64_t per_cta = (b + 127) / 128 * 128 + 1024 + 256;  // + driver reserve + static smem (barriers)
-        return std::min<int64_t>(2048 / nt, (228 * 1024) / per_cta);
-    };
+    (void)nt;
+    auto staging = [&](const Instance &I) { return inst_staging(A, I); };
+    auto occupancy = [&](int64_t b) { return occupancy_of(A, b); };
     std::vector<std::vector<int64_t>> runs;
     int64_t run_occ = -1;
     for (const Instance &I : H.inst) {
@@ -607,6 +752,7 @@ static crsd_status_t jit_compile(crsd_matrix_s *A) {
 crsd_status_t jit_build(crsd_matrix_s *A) {
     DriverApi &dr = driver();
     if (!dr.ok) return fail(CRSD_ERR_UNSUPPORTED, "JIT variant: driver entry point " + dr.err);
+    jit_plan_ranges(A);  // before generating: decides whether the codelets are built for PDL
     crsd_status_t st = jit_compile(A);
     if (st) return st;
     CUmodule mod;
@@ -631,7 +777,6 @@ crsd_status_t jit_build(crsd_matrix_s *A) {
     A->jit_module = mod;
     A->jit_function = fn;
     A->jit_halo_function = fh;
-    jit_plan_ranges(A);
     return CRSD_OK;
 }
 
@@ -651,9 +796,41 @@ void jit_free(crsd_matrix_s *A) {
     A->jit_halo_function = nullptr;
 }
 
+// One launch of fn; pdl: with the programmatic-stream-serialization
+// attribute (the kernel may start while the previous kernel on the stream
+// drains; the codelets wait for it with griddepcontrol.wait).
+static CUresult launch_fn(CUfunction fn, unsigned grid, unsigned nt, unsigned smem, CUstream st, void **params,
+                          bool pdl) {
+    if (!pdl) return driver().launch(fn, grid, 1, 1, nt, 1, 1, smem, st, params, nullptr);
+    CUlaunchAttribute at[1];
+    std::memset(at, 0, sizeof(at));
+    at[0].id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
+    at[0].value.programmaticStreamSerializationAllowed = 1;
+    CUlaunchConfig cfg;
+    std::memset(&cfg, 0, sizeof(cfg));
+    cfg.gridDimX = grid;
+    cfg.gridDimY = cfg.gridDimZ = 1;
+    cfg.blockDimX = nt;
+    cfg.blockDimY = cfg.blockDimZ = 1;
+    cfg.sharedMemBytes = smem;
+    cfg.hStream = st;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return driver().launch_ex(&cfg, fn, params, nullptr);
+}
+
 template <typename T>
 int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
     if (s.seg_count <= 0) return 0;
+    // PDL only where the codelets were generated for it (jit_pdl: one
+    // launch per SpMV), never under stream capture (graph batches keep plain
+    // launches)
+    bool pdl = s.pdl && !s.halo && !s.seg_list && jit_pdl(A) && driver().launch_ex;
+    if (pdl) {
+        cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+        if (cudaStreamIsCapturing((cudaStream_t)stream, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone)
+            pdl = false;
+    }
     JitArgs<T> j;
     j.vals = s.vals;
     j.segs = s.segs;
@@ -669,6 +846,7 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
     j.scat_col = s.scat_col;
     j.scat_val = s.scat_val;
     j.scat_rec = s.scat_rec;
+    j.scat_slab = s.scat_slab;
     j.alpha = s.alpha;
     j.beta = s.beta;
     const unsigned nt = (unsigned)(A->H.mrows / jit_q(A));
@@ -749,8 +927,8 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
                 j.seg_begin = lo;
                 j.seg_count = hi - lo;
                 void *params[] = {&j};
-                if (driver().launch((CUfunction)A->jit_function, (unsigned)(hi - lo), 1, 1, nt, 1, 1, (unsigned)rg[2],
-                                    st, params, nullptr) != CUDA_SUCCESS) {
+                if (launch_fn((CUfunction)A->jit_function, (unsigned)(hi - lo), nt, (unsigned)rg[2], st, params,
+                              false) != CUDA_SUCCESS) {
                     join();
                     return -(int)cudaErrorLaunchFailure;
                 }
@@ -760,8 +938,8 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
         return join() ? n : -(int)cudaErrorLaunchFailure;
     }
     void *params[] = {&j};
-    const CUresult r = driver().launch((CUfunction)A->jit_function, (unsigned)s.seg_count, 1, 1, nt, 1, 1,
-                                       (unsigned)A->smem_bytes, (CUstream)stream, params, nullptr);
+    const CUresult r = launch_fn((CUfunction)A->jit_function, (unsigned)s.seg_count, nt, (unsigned)A->smem_bytes,
+                                 (CUstream)stream, params, pdl);
     return r == CUDA_SUCCESS ? 1 : -(int)cudaErrorLaunchFailure;
 }
 

@@ -6,6 +6,7 @@ array bytes, scatter lists), and must round-trip to the canonical COO through
 the independent oracle decoder.
 """
 import ctypes
+import os
 
 import numpy as np
 import pytest
@@ -270,6 +271,100 @@ def test_jit_codelets_compile_for_sm100a(case, dt, tmp_path):
     sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", str(cub)], capture_output=True, text=True).stdout
     if A.info()["max_ndias"] > 0:
         assert "UBLKCP" in sass and "SYNCS" in sass
+
+
+@pytest.mark.parametrize("case", ["c3s", "empty"])
+def test_jit_pdl_codelets(case):
+    """Codelets for programmatic dependent launch (the default for one-launch
+    handles; not with CRSD_TUNE_JIT_NO_PDL): the value copies are issued before
+    griddepcontrol.wait, every x window copy after it, and the kernel lets
+    its dependent launch start (griddepcontrol.launch_dependents); the cubin
+    holds the SASS for both (ACQBULK, PREEXIT)."""
+    import subprocess
+
+    from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_NO_PDL
+
+    a = gen.config3(n=20)
+    if case == "empty":
+        keep = (a.row < 1024) | (a.row >= 2048)
+        a = gen.COO(a.nrows, a.ncols, a.row[keep], a.col[keep], a.val[keep])
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, host_only=True, variant=4)
+    src = A.jit_source()
+    assert src.count("griddepcontrol.launch_dependents") == 1
+    for body in src.split("__device__ __forceinline__ void codelet_")[1:]:
+        body = body.split("  T acc[Q];")[0]
+        w = body.index("griddepcontrol.wait")
+        # value copies (a.vals) before the wait, window copies (a.x) of the
+        # non-halo path only after it
+        for line in body[:w].splitlines():
+            if "g2s(" in line and "a.x" in line:
+                assert "if (!edge) g2s" in line  # the halo kernel's windows (after halo_wait)
+        assert "a.vals" not in body[w:]
+    B = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, host_only=True, variant=4, tune=TUNE_JIT_NO_PDL)
+    assert "griddepcontrol" not in B.jit_source()
+    p = "/tmp/_crsd_pdl_%d.cubin" % os.getpid()
+    with open(p, "wb") as f:
+        f.write(A.jit_cubin())
+    sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", p], capture_output=True, text=True).stdout
+    os.unlink(p)
+    assert "ACQBULK" in sass and "PREEXIT" in sass
+
+
+def test_jit_scatter_slab_codegen():
+    """Matrices with scatter points: the codelets load a CTA's first 16
+    points from the per-segment slab (an address known without any load) and
+    read the segment descriptor only for the points beyond them;
+    CRSD_TUNE_JIT_NO_SLAB keeps the descriptor-first gather; matrices without
+    scatter points have no scatter code at all."""
+    from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_NO_SLAB
+
+    a = gen.config3(n=20)
+    src = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, host_only=True, variant=4).jit_source()
+    assert "a.scat_slab + s * 16" in src and "if (nscat > 16)" in src and "a.scat_rec[" not in src
+    src = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, host_only=True, variant=4,
+                              tune=TUNE_JIT_NO_SLAB).jit_source()
+    assert "a.scat_slab + s" not in src and "a.scat_rec[sbeg + lane]" in src
+    b = gen.config2(n=24)
+    src = CRSDMatrix.from_coo(b.nrows, b.ncols, b.row, b.col, b.val, host_only=True, variant=4).jit_source()
+    assert "g_mask" not in src and "scat_slab + s" not in src
+
+
+@pytest.mark.parametrize("n", [40, 64, 96])
+def test_jit_interleave_map_is_a_bijection(n):
+    """CRSD_TUNE_JIT_INTERLEAVE bakes a block -> segment map into the kernel
+    (light instances' segments spread among the heavy ones). Re-evaluated
+    here from the generated source's literals: every block maps to a distinct
+    segment, every segment is visited, light segments sit at every R-th block
+    and each class keeps its segment order."""
+    import re
+
+    from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_INTERLEAVE
+
+    a = gen.config3(n=n)
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, host_only=True, variant=4, tune=TUNE_JIT_INTERLEAVE)
+    src = A.jit_source()
+    nseg = A.info()["nseg"]
+    body = src[src.index("i64 seg_of_block(") :]
+    body = body[: body.index("\n}\n")]
+    R = int(re.search(r"const i64 k = b / (\d+)LL", body).group(1))
+    L = int(re.search(r"&& k < (\d+)LL\) \{", body).group(1))
+    light_part, heavy_part = body.split("const i64 h = ")
+    leaf = lambda part, v: [(int(m[1]), int(m[0])) for m in re.findall(r"return (\d+)LL \+ \(" + v + r" - (\d+)LL\);", part)]
+    light, heavy = leaf(light_part, "k"), leaf(heavy_part, "h")  # (first index, first segment), in index order
+
+    def run(runs, i):
+        f, s0 = [r for r in runs if r[0] <= i][-1]
+        return s0 + (i - f)
+
+    seg = []
+    for b in range(nseg):
+        k = b // R
+        seg.append(run(light, k) if (b % R == R - 1 and k < L) else run(heavy, b - min(k, L)))
+    assert sorted(seg) == list(range(nseg))
+    lights = [seg[b] for b in range(nseg) if b % R == R - 1 and b // R < L]
+    assert len(lights) == L and lights == sorted(lights)
+    heavies = [s for b, s in enumerate(seg) if not (b % R == R - 1 and b // R < L)]
+    assert heavies == sorted(heavies)
 
 
 def test_paper_ell_export_fig2_golden(fig2, fig2_expected):

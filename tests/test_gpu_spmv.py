@@ -134,6 +134,89 @@ def test_jit_occupancy_ranges(torch_cuda, dt, alpha, beta):
     y3 = _run(torch_cuda, C, x, alpha, beta, y0, a.nrows)
     assert C.last_launch_count() > 1
     assert np.array_equal(y1, y3)
+    # range handles keep their concurrent launches (no PDL chain)
+    assert A.info()["pdl"] == 0 and A.info()["jit_launches"] == A.last_launch_count()
+    assert B.info()["pdl"] == 1 and B.info()["jit_launches"] == 1
+
+
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+@pytest.mark.parametrize("n", [96, 192])
+def test_jit_interleave_one_launch(torch_cuda, dt, n):
+    """CRSD_TUNE_JIT_INTERLEAVE: one launch visits every segment once, the
+    light instances' segments spread among the heavy ones by a baked block ->
+    segment map (C3's idle blocks). y is NaN-filled first (beta = 0: a segment
+    the map skipped stays NaN); the result must match the oracle -- at full
+    size on sampled rows -- and the occupancy-class ranges bit for bit."""
+    from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_INTERLEAVE
+
+    torch = torch_cuda
+    a = cached("c3", gen.config3, n=n).astype(dt)
+    tdt = torch.float64 if dt == np.float64 else torch.float32
+    x = np.random.default_rng(5).uniform(-1, 1, a.ncols).astype(dt)
+    ys = []
+    for tune in (0, TUNE_JIT_INTERLEAVE):
+        A = _mat(a, variant=4, tune=tune)
+        y = torch.full((a.nrows,), float("nan"), dtype=tdt, device="cuda")
+        A.spmv(torch.from_numpy(x).cuda(), y, 1.0, 0.0)
+        torch.cuda.synchronize()
+        if tune:
+            assert A.last_launch_count() == 1 and A.info()["pdl"] == 1
+            assert "seg_of_block" in A.jit_source()
+        ys.append(y.cpu().numpy())
+        A.close()
+    assert not np.isnan(ys[1]).any()
+    assert np.array_equal(ys[0], ys[1])
+    rows = np.unique(np.concatenate([np.arange(0, a.nrows, 997), [a.nrows - 1]]))
+    o = np.lexsort((a.col, a.row))
+    ptr = np.searchsorted(a.row[o], np.arange(a.nrows + 1))
+    yref, scale = coo.rows_spmv(rows, ptr, a.col[o], a.val[o], x)
+    assert coo.parity_error(ys[1][rows], yref, scale) <= TOL[dt]
+
+
+@pytest.mark.parametrize("case", ["c3:f64", "c3:f32", "c2:f64", "c4:f32"])
+def test_pdl_dependent_chain(torch_cuda, case):
+    """Programmatic dependent launch (the default for one-launch handles;
+    CRSD_TUNE_JIT_NO_PDL turns it off) lets each SpMV start while the
+    previous kernel drains: its CTAs stream the matrix values first and wait
+    (griddepcontrol.wait) before touching x or y. A ping-pong chain
+    u_{k+1} = alpha A u_k + beta u_{k-1}, issued back to back with no host
+    sync, has both hazards PDL must respect -- step k+1 reads what step k
+    writes (RAW) and writes what step k reads (WAR). It must give the bits of
+    the plain launches, and its first step the oracle's. C4 (occupancy-class
+    ranges) stays on plain concurrent launches."""
+    from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_NO_PDL
+
+    torch = torch_cuda
+    cfg, dts = case.split(":")
+    dt = np.float64 if dts == "f64" else np.float32
+    a = {"c3": lambda: gen.config3(n=96), "c2": lambda: gen.config2(n=128), "c4": lambda: gen.config4(n=8_000_000)}[cfg]()
+    a = a.astype(dt)
+    tdt = torch.float64 if dt == np.float64 else torch.float32
+    rng = np.random.default_rng(11)
+    v0 = rng.uniform(-1, 1, a.nrows).astype(dt)
+    v1 = rng.uniform(-1, 1, a.nrows).astype(dt)
+    alpha, beta = 0.03, 0.5
+    yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, v1, alpha, beta, v0)
+    outs = []
+    for tune in (TUNE_JIT_NO_PDL, 0):
+        A = _mat(a, variant=4, mrows=512 if cfg == "c4" else 0, tune=tune)
+        inf = A.info()
+        assert inf["pdl"] == (1 if tune == 0 and inf["jit_launches"] == 1 else 0)
+        assert inf["jit_launches"] == 1 or cfg in ("c3", "c4")
+        # b = [u_{k-1}, u_k]; step k: b[k % 2] <- alpha A b[(k + 1) % 2] + beta b[k % 2]
+        b = [torch.from_numpy(v0).cuda(), torch.from_numpy(v1).cuda()]
+        A.spmv(b[1], b[0], alpha, beta)
+        torch.cuda.synchronize()
+        first = b[0].cpu().numpy().copy()
+        for k in range(1, 24):
+            A.spmv(b[(k + 1) % 2], b[k % 2], alpha, beta)
+        torch.cuda.synchronize()
+        outs.append((first, [u.cpu().numpy().copy() for u in b]))
+        A.close()
+    assert coo.parity_error(outs[0][0], yref, scale) <= TOL[dt]
+    assert np.array_equal(outs[0][0], outs[1][0])
+    for u, w in zip(outs[0][1], outs[1][1]):
+        assert np.array_equal(u, w)
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
@@ -612,10 +695,14 @@ def test_jit_staging_chunks_and_issue(torch_cuda, case, dt):
     """The JIT codelet's staging chunks (opts.jit_chunk: one mbarrier per x
     window by default, the whole segment on one barrier, or windows split into
     runs of k diagonals) and its copy issue (baked instance lookup by default,
-    CRSD_TUNE_JIT_DESC_ISSUE: after the descriptor load) change only when the
-    FMAs start, never their order: every setting matches the oracle and all
-    settings give the same bits."""
-    from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_DESC_ISSUE
+    CRSD_TUNE_JIT_DESC_ISSUE: after the descriptor load), the launch (PDL or
+    not) and where a CTA finds its scatter points (the per-segment slab of the
+    first 16 by default -- "dense_scatter" has segments with more, which take
+    the descriptor path for the rest -- or the descriptor alone,
+    CRSD_TUNE_JIT_NO_SLAB) change only when the FMAs start, never their
+    order: every setting matches the oracle and all settings give the same
+    bits."""
+    from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_DESC_ISSUE, TUNE_JIT_NO_PDL, TUNE_JIT_NO_SLAB
 
     if case == "c1":
         a = gen.config1()
@@ -637,7 +724,7 @@ def test_jit_staging_chunks_and_issue(torch_cuda, case, dt):
     yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, x, -0.75, 0.5, y0)
     first = None
     for chunk in (0, -1, 1, 5):
-        for tune in (0, TUNE_JIT_DESC_ISSUE):
+        for tune in (0, TUNE_JIT_DESC_ISSUE, TUNE_JIT_NO_PDL, TUNE_JIT_NO_SLAB, TUNE_JIT_NO_SLAB | TUNE_JIT_DESC_ISSUE):
             A = _mat(a, variant=4, jit_chunk=chunk, tune=tune)
             y = _run(torch_cuda, A, x, -0.75, 0.5, y0, a.nrows)
             assert coo.parity_error(y, yref, scale) <= TOL[dt], (chunk, tune)
