@@ -135,9 +135,6 @@ typedef struct {
                                               the receive fused into the boundary kernel (crsd_jit_halo) */
 #define CRSD_TUNE_JIT_NO_SLAB 0x100u       /* JIT: each CTA finds its scatter points through its segment descriptor
                                               instead of the per-segment slab of the first 16 */
-#define CRSD_TUNE_JIT_INTERLEAVE 0x200u    /* JIT, one GPU: one launch in which the light instances' segments are
-                                              spread evenly among the heavy ones, instead of occupancy-class range
-                                              launches */
 #define CRSD_TUNE_JIT_NO_PDL 0x80u         /* crsd_spmv, JIT: plain launches instead of programmatic dependent launch.
                                               By default a one-GPU handle whose matrix runs as ONE launch is
                                               launched with PDL: it may start while the previous kernel on the

@@ -287,14 +287,6 @@ static int64_t occupancy_of(const crsd_matrix_s *A, int64_t b) {
     return std::min<int64_t>(2048 / nt, (228 * 1024) / per_cta);
 }
 
-// Interleaved single launch (CRSD_TUNE_JIT_INTERLEAVE): instead of launching
-// the light instances (staging small enough for >= 2x the CTAs per SM of the
-// largest) as separate occupancy-class ranges, ONE launch visits them spread
-// evenly among the heavy segments: block b takes light segment b / R when
-// b % R == R - 1 (and light ones remain), else the next heavy segment in
-// order. A light CTA then shares its SM with heavy CTAs whose staging keeps
-// HBM busy, instead of a run of light CTAs that cannot (C3's idle block B3:
-// one diagonal per segment), and the handle stays one launch (PDL applies).
 // [a, b) runs of edge segments
 static std::vector<std::pair<int64_t, int64_t>> edge_runs(const crsd_matrix_s *A) {
     std::vector<std::pair<int64_t, int64_t>> edges;
@@ -309,45 +301,6 @@ static std::vector<std::pair<int64_t, int64_t>> edge_runs(const crsd_matrix_s *A
 static bool jit_locate(const crsd_matrix_s *A, const std::vector<std::pair<int64_t, int64_t>> &edges) {
     return !(A->tune & CRSD_TUNE_JIT_DESC_ISSUE) && !A->H.inst.empty() && A->H.inst.size() <= 4096 &&
            edges.size() <= 16;
-}
-
-struct Interleave {
-    int64_t R = 0, L = 0;
-    std::vector<std::vector<int64_t>> light, heavy;  // runs {first index, first segment, length}
-};
-static bool interleave_plan(const crsd_matrix_s *A, Interleave &iv) {
-    const HostCRSD &H = A->H;
-    if (!(A->tune & CRSD_TUNE_JIT_INTERLEAVE) || H.partitioned || !jit_locate(A, edge_runs(A))) return false;
-    const int64_t occ_max = occupancy_of(A, A->smem_bytes);
-    auto add = [](std::vector<std::vector<int64_t>> &runs, int64_t &count, const Instance &I) {
-        if (!runs.empty() && runs.back()[1] + runs.back()[2] == I.first_seg) runs.back()[2] += I.nseg;
-        else runs.push_back({count, I.first_seg, I.nseg});
-        count += I.nseg;
-    };
-    int64_t nl = 0, nh = 0;
-    for (const Instance &I : H.inst) {
-        if (occupancy_of(A, inst_staging(A, I)) >= 2 * occ_max) add(iv.light, nl, I);
-        else add(iv.heavy, nh, I);
-    }
-    if (nl == 0 || nh == 0 || iv.light.size() > 256 || iv.heavy.size() > 256) return false;
-    iv.L = nl;
-    iv.R = H.nseg / nl;
-    return iv.R >= 2;
-}
-
-static void emit_runs(std::ostringstream &o, const std::vector<std::vector<int64_t>> &L, size_t lo, size_t hi,
-                      const char *idx, int depth) {
-    const std::string ind(2 + 2 * depth, ' ');
-    if (hi - lo == 1) {
-        o << ind << "return " << L[lo][1] << "LL + (" << idx << " - " << L[lo][0] << "LL);\n";
-        return;
-    }
-    const size_t mid = (lo + hi) / 2;
-    o << ind << "if (" << idx << " < " << L[mid][0] << "LL) {\n";
-    emit_runs(o, L, lo, mid, idx, depth + 1);
-    o << ind << "} else {\n";
-    emit_runs(o, L, mid, hi, idx, depth + 1);
-    o << ind << "}\n";
 }
 
 // Generate the codelets of every distinct pattern of A (one CTA per segment,
@@ -561,26 +514,12 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
         for (const auto &e : edges) o << " || (s >= " << e.first << "LL && s < " << e.second << "LL)";
         o << ";\n}\n";
     }
-    Interleave iv;
-    const bool inter = locate && interleave_plan(A, iv);
-    if (inter) {
-        o << "#define NSEG " << H.nseg << "LL\n";
-        o << "__device__ __forceinline__ i64 seg_of_block(const i64 b) {\n  const i64 k = b / " << iv.R << "LL;\n"
-          << "  if (b % " << iv.R << "LL == " << iv.R - 1 << "LL && k < " << iv.L << "LL) {\n";
-        emit_runs(o, iv.light, 0, iv.light.size(), "k", 1);
-        o << "  }\n  const i64 h = b - (k < " << iv.L << "LL ? k : " << iv.L << "LL);\n";
-        emit_runs(o, iv.heavy, 0, iv.heavy.size(), "h", 0);
-        o << "}\n";
-    }
     // the dispatch body shared by crsd_jit and crsd_jit_halo
     o << "__device__ __forceinline__ void run_segment(const Args &a, const bool halo, const HaloSync &hs, const u64 he) {\n"
          "  extern __shared__ __align__(128) unsigned char smem[];\n  __shared__ u64 bar[NBAR];\n"
          "  T *vs = reinterpret_cast<T *>(smem);\n  i64 s, vb;\n  int key;\n  bool edge;\n";
     if (locate)
-        o << "  if (!a.seg_list) {\n"
-          << (inter ? "    s = (a.seg_begin == 0 && a.seg_count == NSEG) ? seg_of_block(blockIdx.x) : a.seg_begin + blockIdx.x;\n"
-                    : "    s = a.seg_begin + blockIdx.x;\n")
-          << "    locate(s, key, vb);\n    edge = is_edge(s);\n"
+        o << "  if (!a.seg_list) {\n    s = a.seg_begin + blockIdx.x;\n    locate(s, key, vb);\n    edge = is_edge(s);\n"
              "  } else {\n";
     else
         o << "  {\n";
@@ -626,16 +565,13 @@ static void jit_plan_ranges(crsd_matrix_s *A) {
     const HostCRSD &H = A->H;
     A->jit_ranges.clear();
     const int64_t nseg = H.nseg;
-    const int64_t nt = H.mrows / jit_q(A);
     const bool off = (A->tune & CRSD_TUNE_JIT_ONE_LAUNCH) != 0;
     const bool force = (A->tune & CRSD_TUNE_JIT_SPLIT_ALL) != 0;
     std::vector<int64_t> whole = {0, nseg, A->smem_bytes, 0};
-    Interleave iv;
-    if (off || H.inst.empty() || interleave_plan(A, iv)) {
+    if (off || H.inst.empty()) {
         A->jit_ranges.push_back(whole);
         return;
     }
-    (void)nt;
     auto staging = [&](const Instance &I) { return inst_staging(A, I); };
     auto occupancy = [&](int64_t b) { return occupancy_of(A, b); };
     std::vector<std::vector<int64_t>> runs;

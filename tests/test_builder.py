@@ -329,44 +329,6 @@ def test_jit_scatter_slab_codegen():
     assert "g_mask" not in src and "scat_slab + s" not in src
 
 
-@pytest.mark.parametrize("n", [40, 64, 96])
-def test_jit_interleave_map_is_a_bijection(n):
-    """CRSD_TUNE_JIT_INTERLEAVE bakes a block -> segment map into the kernel
-    (light instances' segments spread among the heavy ones). Re-evaluated
-    here from the generated source's literals: every block maps to a distinct
-    segment, every segment is visited, light segments sit at every R-th block
-    and each class keeps its segment order."""
-    import re
-
-    from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_INTERLEAVE
-
-    a = gen.config3(n=n)
-    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, host_only=True, variant=4, tune=TUNE_JIT_INTERLEAVE)
-    src = A.jit_source()
-    nseg = A.info()["nseg"]
-    body = src[src.index("i64 seg_of_block(") :]
-    body = body[: body.index("\n}\n")]
-    R = int(re.search(r"const i64 k = b / (\d+)LL", body).group(1))
-    L = int(re.search(r"&& k < (\d+)LL\) \{", body).group(1))
-    light_part, heavy_part = body.split("const i64 h = ")
-    leaf = lambda part, v: [(int(m[1]), int(m[0])) for m in re.findall(r"return (\d+)LL \+ \(" + v + r" - (\d+)LL\);", part)]
-    light, heavy = leaf(light_part, "k"), leaf(heavy_part, "h")  # (first index, first segment), in index order
-
-    def run(runs, i):
-        f, s0 = [r for r in runs if r[0] <= i][-1]
-        return s0 + (i - f)
-
-    seg = []
-    for b in range(nseg):
-        k = b // R
-        seg.append(run(light, k) if (b % R == R - 1 and k < L) else run(heavy, b - min(k, L)))
-    assert sorted(seg) == list(range(nseg))
-    lights = [seg[b] for b in range(nseg) if b % R == R - 1 and b // R < L]
-    assert len(lights) == L and lights == sorted(lights)
-    heavies = [s for b, s in enumerate(seg) if not (b % R == R - 1 and b // R < L)]
-    assert heavies == sorted(heavies)
-
-
 def test_paper_ell_export_fig2_golden(fig2, fig2_expected):
     """CRSD_PAPER_ELL: the product's scatter-row ELL arrays equal Fig. 4's
     (num_scatter_rows, scatter_rowno, num_scatter_width, scatter_colval,

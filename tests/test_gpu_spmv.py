@@ -139,40 +139,6 @@ def test_jit_occupancy_ranges(torch_cuda, dt, alpha, beta):
     assert B.info()["pdl"] == 1 and B.info()["jit_launches"] == 1
 
 
-@pytest.mark.parametrize("dt", [np.float64, np.float32])
-@pytest.mark.parametrize("n", [96, 192])
-def test_jit_interleave_one_launch(torch_cuda, dt, n):
-    """CRSD_TUNE_JIT_INTERLEAVE: one launch visits every segment once, the
-    light instances' segments spread among the heavy ones by a baked block ->
-    segment map (C3's idle blocks). y is NaN-filled first (beta = 0: a segment
-    the map skipped stays NaN); the result must match the oracle -- at full
-    size on sampled rows -- and the occupancy-class ranges bit for bit."""
-    from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_INTERLEAVE
-
-    torch = torch_cuda
-    a = cached("c3", gen.config3, n=n).astype(dt)
-    tdt = torch.float64 if dt == np.float64 else torch.float32
-    x = np.random.default_rng(5).uniform(-1, 1, a.ncols).astype(dt)
-    ys = []
-    for tune in (0, TUNE_JIT_INTERLEAVE):
-        A = _mat(a, variant=4, tune=tune)
-        y = torch.full((a.nrows,), float("nan"), dtype=tdt, device="cuda")
-        A.spmv(torch.from_numpy(x).cuda(), y, 1.0, 0.0)
-        torch.cuda.synchronize()
-        if tune:
-            assert A.last_launch_count() == 1 and A.info()["pdl"] == 1
-            assert "seg_of_block" in A.jit_source()
-        ys.append(y.cpu().numpy())
-        A.close()
-    assert not np.isnan(ys[1]).any()
-    assert np.array_equal(ys[0], ys[1])
-    rows = np.unique(np.concatenate([np.arange(0, a.nrows, 997), [a.nrows - 1]]))
-    o = np.lexsort((a.col, a.row))
-    ptr = np.searchsorted(a.row[o], np.arange(a.nrows + 1))
-    yref, scale = coo.rows_spmv(rows, ptr, a.col[o], a.val[o], x)
-    assert coo.parity_error(ys[1][rows], yref, scale) <= TOL[dt]
-
-
 @pytest.mark.parametrize("case", ["c3:f64", "c3:f32", "c2:f64", "c4:f32"])
 def test_pdl_dependent_chain(torch_cuda, case):
     """Programmatic dependent launch (the default for one-launch handles;
