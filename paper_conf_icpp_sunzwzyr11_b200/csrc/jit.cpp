@@ -713,6 +713,7 @@ crsd_status_t jit_build(crsd_matrix_s *A) {
     A->jit_module = mod;
     A->jit_function = fn;
     A->jit_halo_function = fh;
+
     return CRSD_OK;
 }
 
