@@ -139,6 +139,49 @@ def test_jit_occupancy_ranges(torch_cuda, dt, alpha, beta):
     assert B.info()["pdl"] == 1 and B.info()["jit_launches"] == 1
 
 
+@pytest.mark.parametrize("flag", ["NO_SLAB", "NO_PDL"])
+@pytest.mark.parametrize("case", ["c1:f64", "c3s:f64", "c3:f64", "c3:f32", "c2s:f64", "c4:f32", "rand:f64", "rand:f32", "dense:f64"])
+def test_jit_schedule_flags_full(torch_cuda, case, flag):
+    """The kept scheduling alternatives at full size (CRSD_TUNE_JIT_NO_SLAB:
+    scatter points through the segment descriptor; CRSD_TUNE_JIT_NO_PDL:
+    plain launches): every segment once (y NaN-filled, beta = 0; then
+    alpha/beta back to back), the same bits as the default codelets, and the
+    oracle on sampled rows."""
+    import paper_conf_icpp_sunzwzyr11_b200 as P
+
+    torch = torch_cuda
+    cfg, dts = case.split(":")
+    dt = np.float64 if dts == "f64" else np.float32
+    a = {"c1": lambda: gen.config1(), "c3s": lambda: gen.config3(n=96), "c3": lambda: cached("c3", gen.config3, n=192),
+         "c2s": lambda: gen.config2(n=128), "c4": lambda: gen.config4(n=8_000_000),
+         "rand": lambda: gen.random_diagonal(40000, 39000, 7, ndiag=12, max_off=900, p_break=0.02, max_break=400, n_scatter=2000),
+         "dense": lambda: gen.random_diagonal(8192, 8192, 5, ndiag=3, n_scatter=30000, max_off=64)}[cfg]().astype(dt)
+    tdt = torch.float64 if dt == np.float64 else torch.float32
+    rng = np.random.default_rng(13)
+    x = rng.uniform(-1, 1, a.ncols).astype(dt)
+    y0 = rng.uniform(-1, 1, a.nrows).astype(dt)
+    xd = torch.from_numpy(x).cuda()
+    outs = []
+    for tune in (0, getattr(P, "TUNE_JIT_" + flag)):
+        A = _mat(a, variant=4, mrows=512 if cfg == "c4" else 0, tune=tune)
+        y = torch.full((a.nrows,), float("nan"), dtype=tdt, device="cuda")
+        A.spmv(xd, y, 1.0, 0.0)
+        y2 = torch.from_numpy(y0).cuda()
+        for _ in range(3):  # back to back; the last one counts
+            y2.copy_(torch.from_numpy(y0).cuda())
+            A.spmv(xd, y2, -0.75, 0.5)
+        torch.cuda.synchronize()
+        outs.append((y.cpu().numpy(), y2.cpu().numpy()))
+        A.close()
+    assert not np.isnan(outs[1][0]).any()
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+    rows = np.unique(np.concatenate([np.arange(0, a.nrows, max(1, a.nrows // 20000)), [a.nrows - 1]]))
+    o = np.lexsort((a.col, a.row))
+    ptr = np.searchsorted(a.row[o], np.arange(a.nrows + 1))
+    yref, scale = coo.rows_spmv(rows, ptr, a.col[o], a.val[o], x, -0.75, 0.5, y0)
+    assert coo.parity_error(outs[1][1][rows], yref, scale) <= TOL[dt]
+
+
 @pytest.mark.parametrize("case", ["c3:f64", "c3:f32", "c2:f64", "c4:f32"])
 def test_pdl_dependent_chain(torch_cuda, case):
     """Programmatic dependent launch (the default for one-launch handles;
