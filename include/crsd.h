@@ -247,6 +247,11 @@ crsd_status_t crsd_destroy(crsd_matrix_t A);
  * Asynchronous; launch errors (CUDA) returned. UNSUPPORTED for host-only or
  * row-partitioned handles (use crsd_spmv_dist). x must be finite: a filled
  * zero computes 0*x (as DIA does).
+ * Stream order: JIT handles that run as one launch use programmatic dependent
+ * launch (CRSD_TUNE_JIT_NO_PDL), so the kernel may start while the previous
+ * kernel on `stream` drains, but it reads only the handle's own (immutable)
+ * matrix arrays until that kernel has completed; every x / y access is
+ * ordered after it, exactly as with a plain launch.
  */
 crsd_status_t crsd_spmv(crsd_matrix_t A, const void *alpha, const void *x, const void *beta, void *y,
                         void *stream);
