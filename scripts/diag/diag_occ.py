@@ -1,3 +1,23 @@
+"""Forced-occupancy diagnostic (
+profiles/r02/diag_forced_occupancy.jsonl). NOT a product path: it needs a
+diagnostic build of libcrsd.so in which launch_fn (csrc/jit.cpp) pads the
+dynamic shared memory so that at most CRSD_DIAG_OCC CTAs fit per SM:
+
+    if (const char *e = getenv("CRSD_DIAG_OCC")) {
+        const int occ = atoi(e);
+        if (occ > 0) {
+            const unsigned want = (unsigned)((228 * 1024) / occ - 1280 - 128) / 128 * 128;
+            if (want > smem) smem = want;
+            driver().set_attr(fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)smem);
+        }
+    }
+
+With the product build the variable has no effect. (The per-launch
+cuFuncSetAttribute of the diagnostic build costs a little on its own: compare
+forced values with each other, not with "0".)
+
+usage: python scripts/diag/diag_occ.py c3:f64:one c3:f64 c2:f64
+"""
 import json, os, sys
 import torch
 sys.path.insert(0, os.environ.get("GRAFT_REPO_ROOT", "/root/repo"))

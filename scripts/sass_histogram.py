@@ -64,7 +64,11 @@ def histogram(cubin: bytes):
 
 
 def main():
-    out = {"how": "crsd_jit_cubin (NVRTC, sm_100a) | cuobjdump -sass; static instruction counts of the whole module",
+    out = {"how": "crsd_jit_cubin (NVRTC, sm_100a) | cuobjdump -sass; static instruction counts of the whole module "
+                  "(crsd_jit, crsd_jit_halo). Host-only handles plan no occupancy-class ranges, so every one-GPU module "
+                  "here is generated in its one-launch form with programmatic dependent launch (PREEXIT = "
+                  "griddepcontrol.launch_dependents, ACQBULK = griddepcontrol.wait); the C5 rank block is "
+                  "row-partitioned (no PDL)",
            "kernels": []}
     for name, A in cases():
         inf = A.info()
@@ -75,7 +79,7 @@ def main():
             "mrows": inf["mrows"],
             "patterns": inf["npat"],
             "instances": inf["ninst"],
-            "families": {k: fam[k] for k in ("UBLKCP", "SYNCS", "LDS", "LDG", "DFMA", "FFMA", "STG", "BAR", "SHFL")},
+            "families": {k: fam[k] for k in ("UBLKCP", "SYNCS", "LDS", "LDG", "DFMA", "FFMA", "STG", "BAR", "SHFL", "PREEXIT", "ACQBULK")},
             "total_instructions": sum(ops.values()),
             "ldg_variants": {k: v for k, v in sorted(ops.items()) if k.startswith("LDG")},
             "syncs_variants": {k: v for k, v in sorted(ops.items()) if k.startswith("SYNCS")},
