@@ -819,7 +819,7 @@ def run_cg(args):
     kw = {"mrows": args.mrows} if args.mrows else {}
     if world > 1:
         kw["row_range"] = (rb, re)
-    A = CRSDMatrix.from_coo(N, N, a.row, a.col, a.val, device=local_rank, **kw)
+    A = CRSDMatrix.from_coo(N, N, a.row, a.col, a.val, device=local_rank, tune=args.tune, **kw)
     info = A.info()
     comm, transport = None, None
     if world > 1:
@@ -971,6 +971,7 @@ def main():
     ap.add_argument("--dtype", default=None, choices=["f64", "f32"], help="default: f64 (f32 for c4)")
     ap.add_argument("--mrows", type=int, default=0)
     ap.add_argument("--variant", default="auto", choices=list(VARIANTS))
+    ap.add_argument("--tune", type=lambda v: int(v, 0), default=0, help="--workload cg: opts.tune of the handle (CRSD_TUNE_*; A/B only)")
     ap.add_argument("--impl", default="crsd", choices=["crsd", "reference"])
     ap.add_argument("--workload", default="spmv", choices=["spmv", "cg"], help="cg: K steps of crsd_cg (N>1: row-partitioned, halo + allreduce)")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
