@@ -135,6 +135,10 @@ typedef struct {
                                               the receive fused into the boundary kernel (crsd_jit_halo) */
 #define CRSD_TUNE_JIT_NO_SLAB 0x100u       /* JIT: each CTA finds its scatter points through its segment descriptor
                                               instead of the per-segment slab of the first 16 */
+#define CRSD_TUNE_JIT_NO_REGSTAGE 0x200u   /* JIT, one GPU: no register staging. By default, when staging the last
+                                              diagonals of the heavy patterns in registers (one more CTA per SM)
+                                              lets the handle run as one launch instead of occupancy-class
+                                              ranges, those segments run in a second kernel; DESIGN.md "Kernels" */
 #define CRSD_TUNE_JIT_NO_PDL 0x80u         /* crsd_spmv, JIT: plain launches instead of programmatic dependent launch.
                                               By default a one-GPU handle whose matrix runs as ONE launch is
                                               launched with PDL: it may start while the previous kernel on the

@@ -25,4 +25,5 @@ from .crsd import (  # noqa: F401
     TUNE_HALO_UNFUSED,
     TUNE_JIT_NO_PDL,
     TUNE_JIT_NO_SLAB,
+    TUNE_JIT_NO_REGSTAGE,
 )

@@ -31,7 +31,7 @@ VARIANT_AUTO, VARIANT_LDG, VARIANT_TMA, VARIANT_PIPE, VARIANT_JIT = 0, 1, 2, 3, 
 # opts.tune (include/crsd.h CRSD_TUNE_*)
 TUNE_JIT_DESC_ISSUE, TUNE_JIT_ONE_LAUNCH, TUNE_JIT_SPLIT_ALL = 0x1, 0x2, 0x4
 TUNE_JIT_SEQUENTIAL, TUNE_DIST_BOUNDARY_SERIAL, TUNE_NO_JIT = 0x8, 0x10, 0x20
-TUNE_HALO_UNFUSED, TUNE_JIT_NO_PDL, TUNE_JIT_NO_SLAB = 0x40, 0x80, 0x100
+TUNE_HALO_UNFUSED, TUNE_JIT_NO_PDL, TUNE_JIT_NO_SLAB, TUNE_JIT_NO_REGSTAGE = 0x40, 0x80, 0x100, 0x200
 
 # every symbol include/crsd.h declares
 EXPORTED = [

@@ -23,6 +23,8 @@ struct crsd_matrix_s {
     void *jit_module = nullptr;
     void *jit_function = nullptr;
     void *jit_halo_function = nullptr;  // the same codelets with the fused halo receive (crsd_jit_halo)
+    void *jit_rs_function = nullptr;    // register-staged codelets (crsd_jit_rs)
+    int regstage = -1;                  // register staging in use (jit_decide; -1: not decided yet)
     std::vector<char> jit_cubin;    // the compiled codelets (crsd_jit_cubin)
     int32_t jit_chunk = 0;          // opts.jit_chunk: diagonals per staging chunk (0 = per x window, <0 = one)
     uint32_t tune = 0;              // opts.tune: CRSD_TUNE_* switches

@@ -274,7 +274,7 @@ static int jit_q(const crsd_matrix_s *A) {
 
 // Staging bytes (values + x windows) of one CTA of instance I, and the CTAs
 // per SM a launch with `b` bytes of dynamic shared memory per CTA allows.
-static int64_t inst_staging(const crsd_matrix_s *A, const Instance &I) {
+static int64_t staging_smem(const crsd_matrix_s *A, const Instance &I) {
     const HostCRSD &H = A->H;
     const int32_t *pl = A->plan.data() + A->segdesc[I.first_seg].plan_begin;
     int64_t el = H.ndias(I.pattern) * H.mrows;
@@ -285,6 +285,43 @@ static int64_t occupancy_of(const crsd_matrix_s *A, int64_t b) {
     const int64_t nt = A->H.mrows / jit_q(A);
     const int64_t per_cta = (b + 127) / 128 * 128 + 1024 + 256;  // + driver reserve + static smem (barriers)
     return std::min<int64_t>(2048 / nt, (228 * 1024) / per_cta);
+}
+// Register staging (one-GPU handles; jit_decide): the values of the last R
+// diagonals of instance I's pattern are loaded by their own threads into
+// registers (coalesced streaming loads issued at CTA start) instead of
+// staged in shared memory, R just large enough that one more CTA fits per SM
+// -- bytes in flight are what the kernel's rate follows and
+// shared memory caps them. Such segments run in a second kernel
+// (crsd_jit_rs) whose launch bounds give the registers for it.
+// Returns R (0: no register staging for this pattern) and the target CTAs
+// per SM.
+static int reg_diags(const crsd_matrix_s *A, const Instance &I, int64_t *target = nullptr) {
+    const HostCRSD &H = A->H;
+    if (A->regstage <= 0 || (A->tune & CRSD_TUNE_JIT_NO_REGSTAGE) || H.partitioned) return 0;
+    const int Q = jit_q(A), nt = H.mrows / Q, nd = (int)H.ndias(I.pattern);
+    const int64_t S = staging_smem(A, I), occ = occupancy_of(A, S), run = (int64_t)H.mrows * H.elem;
+    const int64_t tgt = occ + 1;
+    if (tgt > 2048 / nt) return 0;
+    const int64_t cap = ((228 * 1024) / tgt - 1024 - 256) / 128 * 128;
+    const int64_t R = (S - cap + run - 1) / run;
+    if (R <= 0 || R > nd) return 0;
+    // registers: ~32 for the codelet itself plus R * Q values (two per fp64)
+    const int64_t allowed = (65536 / (tgt * nt)) / 8 * 8;
+    if (32 + R * Q * (H.elem / 4) > allowed) return 0;
+    if (target) *target = tgt;
+    return (int)R;
+}
+static int64_t inst_staging(const crsd_matrix_s *A, const Instance &I) {
+    return staging_smem(A, I) - (int64_t)reg_diags(A, I) * A->H.mrows * A->H.elem;
+}
+// the register-staged kernel's CTAs per SM (0: no instance uses it)
+static int64_t rs_min_blocks(const crsd_matrix_s *A) {
+    int64_t mb = 0;
+    for (const Instance &I : A->H.inst) {
+        int64_t t = 0;
+        if (reg_diags(A, I, &t) > 0) mb = std::max(mb, t);
+    }
+    return mb;
 }
 
 // [a, b) runs of edge segments
@@ -348,7 +385,13 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
         // neighbours' one-sided puts -- thread 0 issues the value copies,
         // waits for the senders, then issues the window copies; the scatter
         // gathers move after the CTA barrier
-        o << "__device__ __forceinline__ void codelet_" << key
+        // pass 0: the codelet; pass 1 (register staging, reg_diags > 0): the
+        // same codelet with the values of the last R diagonals loaded into
+        // registers by their own threads instead of staged in shared memory
+        const int rdiag = reg_diags(A, I);
+        for (int pass = 0; pass < (rdiag > 0 ? 2 : 1); ++pass) {
+        const int R = pass ? rdiag : 0, ns = nd - R;  // ns diagonals staged in shared memory
+        o << "__device__ __forceinline__ void codelet_" << (pass ? "rs_" : "") << key
           << "(const Args &a, const i64 s, const i64 vb, const i64 row0, const bool edge, T *vs, u64 *bar, const int t,"
              " const bool halo, const HaloSync &hs, const u64 he) {\n";
         if (slab)
@@ -359,20 +402,21 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
                  "  if ((t & 31) < " << SLAB_K << ") sr = __ldg(a.scat_slab + s * " << SLAB_K << " + (t & 31));\n";
         if (nd) {
             // thread 0: every mbarrier, then every copy, chunk by chunk
-            o << "  T *xs = vs + " << (int64_t)nd * m << ";\n";
+            o << "  T *xs = vs + " << (int64_t)ns * m << ";\n";
             o << "  if (t == 0) {\n";
             for (size_t c = 0; c < ch.size(); ++c) o << "    bar_init(bar + " << c << ");\n";
             o << "    bar_fence_init();\n    const u64 pf = pol_first(), pn = pol_normal();\n";
             for (size_t c = 0; c < ch.size(); ++c) {
                 const Chunk &k = ch[c];
-                const int64_t vbytes = (int64_t)(k.d1 - k.d0) * m * es;
+                const int64_t vbytes = (int64_t)std::max(0, std::min(k.d1, ns) - k.d0) * m * es;
                 int64_t xbytes = 0;
                 if (k.win == -2) xbytes = wbase[nwin] * es;
                 else if (k.win >= 0) xbytes = (int64_t)pl[3 + 2 * k.win] * es;
                 o << "    bar_expect(bar + " << c << ", " << vbytes << "u" << (xbytes ? " + (edge ? 0u : " : "")
                   << (xbytes ? std::to_string(xbytes) + "u)" : "") << ");\n";
-                o << "    g2s(vs + " << (int64_t)k.d0 * m << ", a.vals + vb + " << (int64_t)k.d0 * m << ", " << vbytes
-                  << "u, bar + " << c << ", pf);\n";
+                if (vbytes)
+                    o << "    g2s(vs + " << (int64_t)k.d0 * m << ", a.vals + vb + " << (int64_t)k.d0 * m << ", " << vbytes
+                      << "u, bar + " << c << ", pf);\n";
                 if (xbytes && !pdl) {
                     o << "    if (!edge && !halo) {\n";
                     for (int w = 0; w < nwin; ++w) {
@@ -396,6 +440,11 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
             }
             o << "    }\n";
             o << "  }\n";
+            // register-staged values: coalesced streaming loads of the last R
+            // diagonals, issued before anything waits (the matrix never changes)
+            for (int d = ns; d < nd; ++d)
+                o << "  T rv" << d << "[Q];\n#pragma unroll\n  for (int q = 0; q < Q; ++q) rv" << d
+                  << "[q] = __ldcs(a.vals + vb + " << (int64_t)d * m << " + t + q * NT);\n";
             if (pdl) {
                 // every thread orders its x / y accesses after the previous
                 // kernel on the stream; then thread 0 issues the windows
@@ -457,15 +506,17 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
         for (size_t c = 0; c < ch.size(); ++c) {
             o << "    bar_wait(bar + " << c << ");\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n      const int r = t + q * NT;\n";
             for (int d = ch[c].d0; d < ch[c].d1; ++d)
-                o << "      acc[q] = fma(vs[" << (int64_t)d * m << " + r], xs[" << xoff[d] << " + r], acc[q]);\n";
+                o << "      acc[q] = fma(" << (d < ns ? "vs[" + std::to_string((int64_t)d * m) + " + r]" : "rv" + std::to_string(d) + "[q]")
+                  << ", xs[" << xoff[d] << " + r], acc[q]);\n";
             o << "    }\n";
         }
         o << "  } else {\n";
         for (size_t c = 0; c < ch.size(); ++c) {
             o << "    bar_wait(bar + " << c << ");\n#pragma unroll\n    for (int q = 0; q < Q; ++q) {\n      const i64 r = row0 + t + q * NT;\n";
             for (int d = ch[c].d0; d < ch[c].d1; ++d)
-                o << "      { const i64 i = r + (" << offs[d] << "); acc[q] = fma(vs[" << (int64_t)d * m
-                  << " + t + q * NT], (i >= a.x_lo && i < a.x_hi) ? __ldg(a.x + i) : T(0), acc[q]); }\n";
+                o << "      { const i64 i = r + (" << offs[d] << "); acc[q] = fma("
+                  << (d < ns ? "vs[" + std::to_string((int64_t)d * m) + " + t + q * NT]" : "rv" + std::to_string(d) + "[q]")
+                  << ", (i >= a.x_lo && i < a.x_hi) ? __ldg(a.x + i) : T(0), acc[q]); }\n";
             o << "    }\n";
         }
         o << "  }\n";
@@ -496,6 +547,7 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
              "    if (!edge || r < a.nrows) {\n      T *yp = a.y + r;\n"
              "      __stcs(yp, (a.beta != T(0)) ? fma(a.alpha, acc[q], a.beta * *yp) : a.alpha * acc[q]);\n    }\n"
              "  }\n}\n";
+        }  // pass
     }
     // Baked segment -> (pattern, value base) lookup and edge test, used for
     // range launches (the one-GPU path and contiguous interiors); list
@@ -532,6 +584,27 @@ static std::string generate(const crsd_matrix_s *A, int Q) {
     o << "extern \"C\" __global__ void __launch_bounds__(NT) crsd_jit(const Args a) {\n";
     if (pdl) o << "  asm volatile(\"griddepcontrol.launch_dependents;\");\n";
     o << "  const HaloSync hs{};\n  run_segment(a, false, hs, 0ull);\n}\n";
+    // register staging: the same dispatch into the register-staged codelets,
+    // launch bounds for its CTAs per SM (range launches, baked lookup)
+    const int64_t rsb = locate ? rs_min_blocks(A) : 0;
+    if (rsb > 0) {
+        o << "extern \"C\" __global__ void __launch_bounds__(NT, " << rsb << ") crsd_jit_rs(const Args a) {\n";
+        if (pdl) o << "  asm volatile(\"griddepcontrol.launch_dependents;\");\n";
+        o << "  extern __shared__ __align__(128) unsigned char smem[];\n  __shared__ u64 bar[NBAR];\n"
+             "  T *vs = reinterpret_cast<T *>(smem);\n  const HaloSync hs{};\n  i64 vb;\n  int key;\n"
+             "  const i64 s = a.seg_begin + blockIdx.x;\n  locate(s, key, vb);\n  const bool edge = is_edge(s);\n"
+             "  const i64 row0 = s * MROWS;\n  switch (key) {\n";
+        for (const Instance &I : H.inst) {
+            const int32_t key = A->segdesc[I.first_seg].plan_begin;
+            bool first = true;
+            for (const Instance &J : H.inst)
+                if (&J != &I && A->segdesc[J.first_seg].plan_begin == key && &J < &I) first = false;
+            if (!first) continue;
+            o << "  case " << key << ": codelet_" << (reg_diags(A, I) > 0 ? "rs_" : "") << key
+              << "(a, s, vb, row0, edge, vs, bar, threadIdx.x, false, hs, 0ull); break;\n";
+        }
+        o << "  }\n}\n";
+    }
     // boundary segments of a direct-mode exchange: the receive side fused in
     // (wait per CTA before the window copies; the last CTA to finish releases
     // the pads to the senders and advances the epoch)
@@ -561,13 +634,16 @@ static bool jit_concurrent(const crsd_matrix_s *A) { return !(A->tune & CRSD_TUN
 // staging size (see below for when it pays). CRSD_TUNE_JIT_ONE_LAUNCH
 // disables the split, CRSD_TUNE_JIT_SPLIT_ALL forces it at every class
 // change (tests, sanitizer runs).
-static void jit_plan_ranges(crsd_matrix_s *A) {
+static void jit_plan_ranges_impl(crsd_matrix_s *A) {
     const HostCRSD &H = A->H;
     A->jit_ranges.clear();
     const int64_t nseg = H.nseg;
     const bool off = (A->tune & CRSD_TUNE_JIT_ONE_LAUNCH) != 0;
     const bool force = (A->tune & CRSD_TUNE_JIT_SPLIT_ALL) != 0;
-    std::vector<int64_t> whole = {0, nseg, A->smem_bytes, 0};
+    int64_t smax = 0;
+    for (const Instance &I : H.inst) smax = std::max(smax, inst_staging(A, I));
+    if (H.inst.empty()) smax = A->smem_bytes;
+    std::vector<int64_t> whole = {0, nseg, smax, 0};
     if (off || H.inst.empty()) {
         A->jit_ranges.push_back(whole);
         return;
@@ -636,11 +712,11 @@ static void jit_plan_ranges(crsd_matrix_s *A) {
     // C3 (idle blocks B1 and B3 only, 16 % of the rows): ~32 MB vs ~130 MB
     // -> one launch (measured: a 5-launch split ran at 0.90 against 0.96,
     // sweep24b).
-    const int64_t occ_whole = occupancy(A->smem_bytes);
+    const int64_t occ_whole = occupancy(smax);
     double gain = 0.0;
     for (const std::vector<int64_t> &r : merged)
         gain += (double)r[1] * (double)r[2] * (1.0 - (double)occ_whole / (double)occupancy(r[2]));
-    const double wave = (double)A->sm_count * (double)occ_whole * (double)A->smem_bytes;
+    const double wave = (double)A->sm_count * (double)occ_whole * (double)smax;
     // Concurrent range launches have no boundary to drain; what a split still
     // costs (launches that do not fully overlap, fork/join) is taken as 3/4
     // of a wave in total -- a threshold fitted to sweep25, not derived: C3
@@ -655,6 +731,34 @@ static void jit_plan_ranges(crsd_matrix_s *A) {
     }
     merged.insert(merged.end(), aux.begin(), aux.end());
     A->jit_ranges = merged;
+}
+
+// ... and mark each range that holds a register-staged instance (element 4):
+// it launches crsd_jit_rs.
+static void jit_plan_ranges(crsd_matrix_s *A) {
+    jit_plan_ranges_impl(A);
+    for (std::vector<int64_t> &rg : A->jit_ranges) {
+        int64_t rs = 0;
+        for (const Instance &I : A->H.inst)
+            if (I.first_seg < rg[0] + rg[1] && rg[0] < I.first_seg + I.nseg && reg_diags(A, I) > 0) rs = 1;
+        rg.push_back(rs);
+    }
+}
+
+// Launch plan and register staging: register staging is kept where it turns
+// a handle that needs occupancy-class range launches into ONE launch (C3
+// f64: its heavy and light instances then all run at 4-5 CTAs per SM, and
+// the single launch gets PDL; 1.018 vs 1.002 for the 5 concurrent ranges,
+// profiles/r02/sweep12_regstage*.jsonl); where the split remains (C4) it
+// measured 1% slower and is not used.
+static void jit_decide(crsd_matrix_s *A) {
+    // the register-staged kernel dispatches through the baked lookup
+    A->regstage = (A->tune & CRSD_TUNE_JIT_NO_REGSTAGE) || A->H.partitioned || !jit_locate(A, edge_runs(A)) ? 0 : 1;
+    jit_plan_ranges(A);
+    if (A->regstage && (A->jit_ranges.size() > 1 || rs_min_blocks(A) == 0)) {
+        A->regstage = 0;
+        jit_plan_ranges(A);
+    }
 }
 
 // Generate and compile A's codelets for sm_100a (NVRTC only; no device needed).
@@ -688,7 +792,7 @@ static crsd_status_t jit_compile(crsd_matrix_s *A) {
 crsd_status_t jit_build(crsd_matrix_s *A) {
     DriverApi &dr = driver();
     if (!dr.ok) return fail(CRSD_ERR_UNSUPPORTED, "JIT variant: driver entry point " + dr.err);
-    jit_plan_ranges(A);  // before generating: decides whether the codelets are built for PDL
+    jit_decide(A);  // before generating: PDL and register staging depend on the launch plan
     crsd_status_t st = jit_compile(A);
     if (st) return st;
     CUmodule mod;
@@ -710,9 +814,18 @@ crsd_status_t jit_build(crsd_matrix_s *A) {
         dr.unload(mod);
         return fail(CRSD_ERR_CUDA, "crsd_jit_halo: cuModuleGetFunction / cuFuncSetAttribute failed");
     }
+    CUfunction frs = nullptr;
+    if (rs_min_blocks(A) > 0 &&
+        (dr.get_function(&frs, mod, "crsd_jit_rs") != CUDA_SUCCESS ||
+         (A->smem_bytes > 48 * 1024 &&
+          dr.set_attr(frs, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)A->smem_bytes) != CUDA_SUCCESS))) {
+        dr.unload(mod);
+        return fail(CRSD_ERR_CUDA, "crsd_jit_rs: cuModuleGetFunction / cuFuncSetAttribute failed");
+    }
     A->jit_module = mod;
     A->jit_function = fn;
     A->jit_halo_function = fh;
+    A->jit_rs_function = frs;
 
     return CRSD_OK;
 }
@@ -731,6 +844,7 @@ void jit_free(crsd_matrix_s *A) {
     A->jit_module = nullptr;
     A->jit_function = nullptr;
     A->jit_halo_function = nullptr;
+    A->jit_rs_function = nullptr;
 }
 
 // One launch of fn; pdl: with the programmatic-stream-serialization
@@ -864,8 +978,9 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
                 j.seg_begin = lo;
                 j.seg_count = hi - lo;
                 void *params[] = {&j};
-                if (launch_fn((CUfunction)A->jit_function, (unsigned)(hi - lo), nt, (unsigned)rg[2], st, params,
-                              false) != CUDA_SUCCESS) {
+                const bool rs = rg.size() > 4 && rg[4] && A->jit_rs_function;
+                if (launch_fn((CUfunction)(rs ? A->jit_rs_function : A->jit_function), (unsigned)(hi - lo), nt,
+                              (unsigned)rg[2], st, params, false) != CUDA_SUCCESS) {
                     join();
                     return -(int)cudaErrorLaunchFailure;
                 }
@@ -875,8 +990,12 @@ int jit_launch(const crsd_matrix_s *A, const SpmvArgs<T> &s, void *stream) {
         return join() ? n : -(int)cudaErrorLaunchFailure;
     }
     void *params[] = {&j};
-    const CUresult r = launch_fn((CUfunction)A->jit_function, (unsigned)s.seg_count, nt, (unsigned)A->smem_bytes,
-                                 (CUstream)stream, params, pdl);
+    // one range over a one-GPU handle: its own kernel and staging size
+    // (register staging); lists and row-partitioned handles: the plain kernel
+    const bool one = !s.seg_list && A->jit_ranges.size() == 1;
+    const bool rs = one && A->jit_ranges[0].size() > 4 && A->jit_ranges[0][4] && A->jit_rs_function;
+    const CUresult r = launch_fn((CUfunction)(rs ? A->jit_rs_function : A->jit_function), (unsigned)s.seg_count, nt,
+                                 (unsigned)(one ? A->jit_ranges[0][2] : A->smem_bytes), (CUstream)stream, params, pdl);
     return r == CUDA_SUCCESS ? 1 : -(int)cudaErrorLaunchFailure;
 }
 
@@ -889,6 +1008,7 @@ extern "C" crsd_status_t crsd_jit_source(crsd_matrix_t A, char *buf, int64_t cap
     if (!A || !len) return crsd::fail(CRSD_ERR_INVALID_ARG, "NULL argument");
     if (A->smem_bytes > 200 * 1024)
         return crsd::fail(CRSD_ERR_UNSUPPORTED, "JIT codelets need a segment's staging <= 200 KB");
+    if (A->jit_source.empty() && A->jit_ranges.empty()) crsd::jit_decide(A);  // host-only handles: plan as on a device
     const std::string src = A->jit_source.empty() ? crsd::jit_generate(A) : A->jit_source;
     *len = (int64_t)src.size();
     if (buf && cap > 0) {
@@ -902,6 +1022,7 @@ extern "C" crsd_status_t crsd_jit_source(crsd_matrix_t A, char *buf, int64_t cap
 extern "C" crsd_status_t crsd_jit_cubin(crsd_matrix_t A, void *buf, int64_t cap, int64_t *len) {
     if (!A || !len) return crsd::fail(CRSD_ERR_INVALID_ARG, "NULL argument");
     if (A->jit_cubin.empty()) {
+        if (A->jit_ranges.empty()) crsd::jit_decide(A);
         const crsd_status_t st = crsd::jit_compile(A);
         if (st) return st;
     }

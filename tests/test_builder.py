@@ -250,8 +250,14 @@ def test_jit_codelets_compile_for_sm100a(case, dt, tmp_path):
     npat = A.info()["npat"]
     # one codelet + one case per distinct pattern; the baked segment ->
     # pattern lookup has one leaf per instance (the paper's Table II rows)
-    assert src.count("__device__ __forceinline__ void codelet_") == npat
-    assert src.count("case ") == npat
+    import re
+
+    assert len(re.findall(r"__device__ __forceinline__ void codelet_\d+\(", src)) == npat
+    # the register-staged kernel (crsd_jit_rs, when it is used) dispatches
+    # every pattern again, some into their register-staged codelets
+    n_rs = src.count("crsd_jit_rs(")
+    assert src.count("case ") == npat * (1 + n_rs)
+    assert len(re.findall(r"void codelet_rs_\d+\(", src)) <= npat * n_rs
     assert src.count("{ key = ") == A.info()["ninst"]
     # two entry points: the plain kernel and the boundary kernel with the
     # fused halo receive (wait on the senders' flags, proxy fence, release)
@@ -290,7 +296,9 @@ def test_jit_pdl_codelets(case):
         a = gen.COO(a.nrows, a.ncols, a.row[keep], a.col[keep], a.val[keep])
     A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, host_only=True, variant=4)
     src = A.jit_source()
-    assert src.count("griddepcontrol.launch_dependents") == 1
+    # once per entry kernel that crsd_spmv launches (crsd_jit, and crsd_jit_rs
+    # when register staging is used)
+    assert src.count("griddepcontrol.launch_dependents") == 1 + src.count("crsd_jit_rs(")
     for body in src.split("__device__ __forceinline__ void codelet_")[1:]:
         body = body.split("  T acc[Q];")[0]
         w = body.index("griddepcontrol.wait")

@@ -139,7 +139,7 @@ def test_jit_occupancy_ranges(torch_cuda, dt, alpha, beta):
     assert B.info()["pdl"] == 1 and B.info()["jit_launches"] == 1
 
 
-@pytest.mark.parametrize("flag", ["NO_SLAB", "NO_PDL"])
+@pytest.mark.parametrize("flag", ["NO_SLAB", "NO_PDL", "NO_REGSTAGE"])
 @pytest.mark.parametrize("case", ["c1:f64", "c3s:f64", "c3:f64", "c3:f32", "c2s:f64", "c4:f32", "rand:f64", "rand:f32", "dense:f64"])
 def test_jit_schedule_flags_full(torch_cuda, case, flag):
     """The kept scheduling alternatives at full size (CRSD_TUNE_JIT_NO_SLAB:
@@ -711,7 +711,7 @@ def test_jit_staging_chunks_and_issue(torch_cuda, case, dt):
     CRSD_TUNE_JIT_NO_SLAB) change only when the FMAs start, never their
     order: every setting matches the oracle and all settings give the same
     bits."""
-    from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_DESC_ISSUE, TUNE_JIT_NO_PDL, TUNE_JIT_NO_SLAB
+    from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_DESC_ISSUE, TUNE_JIT_NO_PDL, TUNE_JIT_NO_SLAB, TUNE_JIT_NO_REGSTAGE
 
     if case == "c1":
         a = gen.config1()
@@ -733,7 +733,8 @@ def test_jit_staging_chunks_and_issue(torch_cuda, case, dt):
     yref, scale = coo.coo_spmv(a.nrows, a.ncols, a.row, a.col, a.val, x, -0.75, 0.5, y0)
     first = None
     for chunk in (0, -1, 1, 5):
-        for tune in (0, TUNE_JIT_DESC_ISSUE, TUNE_JIT_NO_PDL, TUNE_JIT_NO_SLAB, TUNE_JIT_NO_SLAB | TUNE_JIT_DESC_ISSUE):
+        for tune in (0, TUNE_JIT_DESC_ISSUE, TUNE_JIT_NO_PDL, TUNE_JIT_NO_SLAB, TUNE_JIT_NO_SLAB | TUNE_JIT_DESC_ISSUE,
+                     TUNE_JIT_NO_REGSTAGE):
             A = _mat(a, variant=4, jit_chunk=chunk, tune=tune)
             y = _run(torch_cuda, A, x, -0.75, 0.5, y0, a.nrows)
             assert coo.parity_error(y, yref, scale) <= TOL[dt], (chunk, tune)
