@@ -65,10 +65,10 @@ def histogram(cubin: bytes):
 
 def main():
     out = {"how": "crsd_jit_cubin (NVRTC, sm_100a) | cuobjdump -sass; static instruction counts of the whole module "
-                  "(crsd_jit, crsd_jit_halo). Host-only handles plan no occupancy-class ranges, so every one-GPU module "
-                  "here is generated in its one-launch form with programmatic dependent launch (PREEXIT = "
-                  "griddepcontrol.launch_dependents, ACQBULK = griddepcontrol.wait); the C5 rank block is "
-                  "row-partitioned (no PDL)",
+                  "(crsd_jit, crsd_jit_halo, and crsd_jit_rs where register staging is used: C3 f64). The launch plan "
+                  "is the one a device handle makes (148 SMs): one-launch handles carry programmatic dependent launch "
+                  "(PREEXIT = griddepcontrol.launch_dependents, ACQBULK = griddepcontrol.wait); C4 (occupancy-class "
+                  "ranges) and the row-partitioned C5 rank block do not",
            "kernels": []}
     for name, A in cases():
         inf = A.info()
