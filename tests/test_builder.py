@@ -337,6 +337,53 @@ def test_jit_scatter_slab_codegen():
     assert "g_mask" not in src and "scat_slab + s" not in src
 
 
+@pytest.mark.parametrize("dt", [np.float64, np.float32])
+def test_jit_register_staging_codegen(dt):
+    """Register staging (C3's 27-diagonal patterns): each register-staged
+    codelet loads the values of its last R diagonals with coalesced streaming
+    loads (rv<d>[q]), bulk-copies only the first nd - R value runs, and runs
+    the FMAs in the plain codelet's order with the same x operands; the
+    second kernel (crsd_jit_rs) dispatches to it. CRSD_TUNE_JIT_NO_REGSTAGE
+    removes both. fp32 C3 (6 CTAs/SM by shared memory, 8 by threads, no
+    registers to spare at 7) gets none."""
+    import re
+
+    from paper_conf_icpp_sunzwzyr11_b200 import TUNE_JIT_NO_REGSTAGE
+
+    a = gen.config3(n=48).astype(dt)
+    A = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, host_only=True, variant=4)
+    src = A.jit_source()
+    m, es = A.info()["mrows"], np.dtype(dt).itemsize
+    B = CRSDMatrix.from_coo(a.nrows, a.ncols, a.row, a.col, a.val, host_only=True, variant=4, tune=TUNE_JIT_NO_REGSTAGE)
+    assert "crsd_jit_rs(" not in B.jit_source() and "codelet_rs_" not in B.jit_source()
+    if dt == np.float32:
+        assert "crsd_jit_rs(" not in src
+        return
+    assert "crsd_jit_rs(" in src
+    keys = re.findall(r"void codelet_rs_(\d+)\(", src)
+    assert keys
+    for k in keys:
+        plain = src.split("void codelet_" + k + "(")[1].split("\n}\n")[0]
+        rs = src.split("void codelet_rs_" + k + "(")[1].split("\n}\n")[0]
+        nd = len(re.findall(r"acc\[q\] = fma\(", plain.split("} else {")[0]))
+        rv = sorted(set(int(d) for d in re.findall(r"T rv(\d+)\[Q\];", rs)))
+        R = len(rv)
+        assert R > 0 and rv == list(range(nd - R, nd))  # a suffix of the pattern
+        for d in rv:
+            assert "rv%d[q] = __ldcs(a.vals + vb + %d + t + q * NT)" % (d, d * m) in rs
+        copied = sum(int(b) for b in re.findall(r"g2s\(vs \+ \d+, a\.vals \+ vb \+ \d+, (\d+)u", rs))
+        assert copied == (nd - R) * m * es
+        # the same FMAs in the same order: x operands equal, values from
+        # shared memory for d < nd - R, from registers after
+        fp = re.findall(r"acc\[q\] = fma\((.*?), (xs\[\d+ \+ r\])", plain.split("} else {")[0])
+        fr = re.findall(r"acc\[q\] = fma\((.*?), (xs\[\d+ \+ r\])", rs.split("} else {")[0])
+        assert len(fp) == len(fr) == nd and [x for _, x in fp] == [x for _, x in fr]
+        for d, ((vp, _), (vr, _)) in enumerate(zip(fp, fr)):
+            assert vr == (vp if d < nd - R else "rv%d[q]" % d)
+        # x windows land after the staged values
+        assert "T *xs = vs + %d;" % ((nd - R) * m) in rs
+
+
 def test_paper_ell_export_fig2_golden(fig2, fig2_expected):
     """CRSD_PAPER_ELL: the product's scatter-row ELL arrays equal Fig. 4's
     (num_scatter_rows, scatter_rowno, num_scatter_width, scatter_colval,
