@@ -339,7 +339,7 @@ def sub_record(cfg, dtype, args, dev):
     ub = info["unique_bytes_beta0"]
     peak, _ = measured_peaks()
     achieved = ub / (ms * 1e-3) / 1e9
-    kname = KNAME[info["variant"]]
+    kname = KNAME[info["variant"]] + ("_rs" if info.get("regstage") else "")
     rec = {
         "workload": desc,
         "value": round(2.0 * info["nnz"] / (ms * 1e-3) / 1e9, 3),
@@ -646,7 +646,7 @@ def run_spmv(args):
         cpu = cpu_baseline(args.config, args.dtype)
     box_copy = copy_bandwidth(dev)
     box_read = read_bandwidth()
-    kname = KNAME[info["variant"]]
+    kname = KNAME[info["variant"]] + ("_rs" if info.get("regstage") else "")
     line = {
         "metric": METRIC,
         "value": round(gflops, 3),

@@ -184,6 +184,9 @@ typedef struct {
     int64_t unique_bytes_beta1;     /* ... with beta != 0 (y also read) */
     int32_t jit_launches;           /* JIT: kernel launches of one crsd_spmv (occupancy-class ranges), else 1 */
     int32_t pdl;                    /* 1: crsd_spmv launches with programmatic dependent launch (CRSD_TUNE_JIT_NO_PDL) */
+    int32_t regstage;               /* 1: register staging in use -- crsd_spmv launches the register-staged kernel
+                                       (crsd_jit_rs) for some segments (CRSD_TUNE_JIT_NO_REGSTAGE) */
+    int32_t reserved_;
 } crsd_info_t;
 
 /*

@@ -108,6 +108,7 @@ _INFO_FIELDS = [
     ("variant", ctypes.c_int32), ("smem_bytes", ctypes.c_int32),
     ("unique_bytes_beta0", ctypes.c_int64), ("unique_bytes_beta1", ctypes.c_int64),
     ("jit_launches", ctypes.c_int32), ("pdl", ctypes.c_int32),
+    ("regstage", ctypes.c_int32), ("reserved_", ctypes.c_int32),
 ]
 
 

@@ -691,6 +691,7 @@ crsd_status_t crsd_get_info(crsd_matrix_t A, crsd_info_t *I) {
     I->unique_bytes_beta1 = base + H.n_local * es;
     I->jit_launches = A->variant == VARIANT_JIT ? (int32_t)std::max<size_t>(1, A->jit_ranges.size()) : 1;
     I->pdl = (A->variant == VARIANT_JIT && !A->host_only && jit_pdl(A)) ? 1 : 0;
+    I->regstage = (A->variant == VARIANT_JIT && A->jit_rs_function) ? 1 : 0;
     return CRSD_OK;
 }
 

@@ -164,6 +164,11 @@ def test_jit_schedule_flags_full(torch_cuda, case, flag):
     outs = []
     for tune in (0, getattr(P, "TUNE_JIT_" + flag)):
         A = _mat(a, variant=4, mrows=512 if cfg == "c4" else 0, tune=tune)
+        if case == "c3:f64" and flag == "NO_REGSTAGE":
+            # the north-star matrix runs register-staged as one launch by
+            # default, as 5 occupancy-class ranges without
+            inf = A.info()
+            assert (inf["regstage"], inf["jit_launches"]) == ((1, 1) if tune == 0 else (0, 5))
         y = torch.full((a.nrows,), float("nan"), dtype=tdt, device="cuda")
         A.spmv(xd, y, 1.0, 0.0)
         y2 = torch.from_numpy(y0).cuda()
