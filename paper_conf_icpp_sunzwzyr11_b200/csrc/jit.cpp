@@ -24,7 +24,18 @@
 // -> pattern) is baked into the kernel as a comparison tree over
 // the instances' first segments, with each instance's value base as a
 // literal, so thread 0 issues the bulk copies without waiting for any memory
-// load; the segment descriptor (scatter list) is read while they fly.
+// load. A segment's first 16 scatter points come from a fixed-address slab
+// (SlabRec), loaded as the CTA's first instruction; only points beyond them
+// need the segment descriptor.
+//
+// Register staging (reg_diags / crsd_jit_rs): where it turns a handle that
+// needs occupancy-class range launches into one launch, the values of the
+// last diagonals of heavy patterns are loaded into registers instead of
+// shared memory, so one more CTA (and its bytes in flight) fits per SM.
+//
+// Programmatic dependent launch (jit_pdl): one-launch handles let the next
+// crsd_spmv's CTAs start during the previous kernel's tail; they stream the
+// (immutable) values first and wait (griddepcontrol.wait) before x and y.
 //
 // NVRTC (libnvrtc.so.12) and the CUDA driver API are resolved at runtime
 // (dlopen / cudaGetDriverEntryPoint), so libcrsd.so loads on machines
